@@ -1,0 +1,21 @@
+# libctaclust: sm_100a only (SASS, no PTX fallback); oracle: plain gcc.
+NVCC ?= nvcc
+PKG := paper_conf_asplos_lis0l0c17_b200
+SRC := $(PKG)/csrc
+LIB := $(PKG)/libctaclust.so
+NVFLAGS := -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo \
+           -Xcompiler -fPIC -Xcompiler -Wall -Xptxas -v --expt-relaxed-constexpr -I include
+HDRS := $(wildcard $(SRC)/*.cuh) include/ctaclust.h
+
+all: $(LIB) oracle/liboracle.so
+
+$(LIB): $(SRC)/ctaclust.cu $(HDRS)
+	$(NVCC) $(NVFLAGS) -shared -o $@ $(SRC)/ctaclust.cu 2> build_ptxas.log || (cat build_ptxas.log; exit 1)
+
+oracle/liboracle.so: oracle/oracle.c
+	gcc -O2 -fPIC -shared -std=c11 -o $@ $<
+
+clean:
+	rm -f $(LIB) oracle/liboracle.so build_ptxas.log
+
+.PHONY: all clean

@@ -1,0 +1,227 @@
+/*
+ * ctaclust.h -- C ABI of libctaclust, a B200 (sm_100a) implementation of
+ * locality-aware CTA clustering (Li, Song, Liu, Liu, Kumar, Corporaal,
+ * "Locality-Aware CTA Clustering for Modern GPUs", ASPLOS'17).
+ * Citations "P:<n>" are line numbers of the paper transcript;
+ * the section / equation / listing is named next to each.
+ *
+ * Conventions (all entry points):
+ *  - Every function returns cc_status (CC_OK == 0).  Nothing aborts, throws or
+ *    prints across the ABI; cc_last_error() gives a thread-local message for the
+ *    most recent failure on the calling thread.
+ *  - Pointers are plain host or device pointers as stated per argument; no
+ *    framework types.  The caller owns every buffer it passes; the library owns
+ *    only what a cc_plan holds (its device tables and default workspace).
+ *  - Launches are asynchronous on the caller's stream (a cudaStream_t passed as
+ *    void*; NULL = legacy default stream).  Errors detected at launch time are
+ *    returned; asynchronous kernel faults surface at the caller's next
+ *    synchronisation as usual for CUDA.
+ *  - Sizes are validated; logical grids whose CTA count overflows int32 give
+ *    CC_ERR_OVERFLOW.
+ */
+#ifndef CTACLUST_H
+#define CTACLUST_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    CC_OK = 0,
+    CC_ERR_INVALID_ARG = -1,     /* null/negative/misaligned argument, grid mismatch */
+    CC_ERR_OVERFLOW = -2,        /* gx*gy (or a derived size) exceeds int32 */
+    CC_ERR_NOT_PERMUTATION = -3, /* USER order is not a permutation of [0, gx*gy) */
+    CC_ERR_CUDA = -4,            /* a CUDA runtime call failed; see cc_last_cuda_error() */
+    CC_ERR_NCCL = -5,            /* reserved for the NCCL-backed entry points */
+    CC_ERR_UNSUPPORTED = -6,     /* valid request this build / device cannot serve */
+    CC_ERR_NO_DEVICE = -7        /* plan created host-only (device < 0) was asked to launch */
+} cc_status;
+
+/* ---------------------------------------------------------------------------
+ * Planner: Step 1 partitioning f and Step 2 inverting f^-1 (§4.2)
+ *
+ * The logical grid O of gx*gy CTAs is put in the order of a CTA indexing method
+ * (Fig. 7) and cut into M balanced contiguous clusters (Eq. 2-5,
+ * P:1869-1875): with q = |V|/M and r = |V|%M the first r clusters hold q+1 CTAs,
+ * the rest q (readings R1/R2 for the garbled Eq. 4/5).  v denotes a
+ * CTA's position in that order; slot (w, i) is position w of cluster i and
+ * v = f^-1(w, i) = i*(q+1) + w + min(r-i, 0)   (Eq. 7).
+ * Tables name CTAs by their row-major linear id lin = by*gx + bx.
+ * ------------------------------------------------------------------------- */
+typedef enum {
+    CC_ORDER_ROW = 0,  /* v = by*gx + bx : the paper's "Y-partitioning"   */
+    CC_ORDER_COL = 1,  /* v = bx*gy + by : the paper's "X-partitioning"   */
+    CC_ORDER_TILE = 2, /* tile_w x tile_h CTA tiles, row-major over tiles and inside
+                          each tile, edge tiles clipped (Fig. 7 tile panel; R6)    */
+    CC_ORDER_USER = 3  /* arbitrary order: user_order[v] = lin ("customized") */
+} cc_order;
+
+typedef struct {
+    int32_t gx, gy;             /* logical grid (gridDim.x, gridDim.y of O); >= 0    */
+    int32_t order;              /* cc_order                                         */
+    int32_t tile_w, tile_h;     /* TILE only, >= 1                                  */
+    int32_t num_clusters;       /* M; 0 => number of SMs of `device` ("size
+                                   of C equal to the number of SMs, 1-to-1")        */
+    const int32_t* user_order;  /* HOST, gx*gy entries, USER only; copied at create  */
+    int32_t device;             /* CUDA ordinal owning the device tables; -1 => a
+                                   host-only plan (tables/lookups, no launches)     */
+} cc_plan_desc;
+
+typedef struct cc_plan_s* cc_plan;   /* opaque; immutable after create except for
+                                        its self-resetting launch workspace        */
+
+/* Build the partition.  Errors: INVALID_ARG (null, negative grid, M < 1 when
+ * device < 0, bad tile dims, bad order), OVERFLOW, NOT_PERMUTATION, CUDA. */
+cc_status cc_plan_create(const cc_plan_desc* desc, cc_plan* out);
+/* Free the plan.  The caller must have synchronised every stream that used it. */
+cc_status cc_plan_destroy(cc_plan plan);
+/* |V|, M, q = |V|/M, r = |V|%M.  Any output pointer may be NULL. */
+cc_status cc_plan_info(cc_plan plan, int64_t* num_ctas, int32_t* num_clusters,
+                       int32_t* q, int32_t* r);
+/* Copy the partition to HOST arrays the caller allocated: perm[|V|] (cluster-
+ * major list of lin ids: perm[offsets[i] + w] = lin of slot (w,i)) and
+ * offsets[M+1].  Either pointer may be NULL. */
+cc_status cc_plan_table(cc_plan plan, int32_t* perm, int32_t* offsets);
+/* f(v) = (w, i)  (Eq. 2-5).  INVALID_ARG when v is outside [0, |V|). */
+cc_status cc_plan_lookup(cc_plan plan, int32_t v, int32_t* w, int32_t* i);
+/* f^-1(w, i) = v (Eq. 7).  INVALID_ARG when (w, i) is not a slot of the plan. */
+cc_status cc_plan_invert(cc_plan plan, int32_t w, int32_t i, int32_t* v);
+
+/* ---------------------------------------------------------------------------
+ * Device facts used for binding (§4.2.3 Step 3)
+ * ------------------------------------------------------------------------- */
+/* num_sms = cudaDevAttrMultiProcessorCount; smid_span = %nsmid (the range of the
+ * virtual %smid register); l2_bytes = L2 size.  Outputs may be NULL. */
+cc_status cc_device_info(int32_t device, int32_t* num_sms, int32_t* smid_span,
+                         int32_t* l2_bytes);
+/* The dense SM rank table the agent runtime binds clusters with: rank_of_smid
+ * (HOST, smid_span entries) maps a %smid value to a rank in [0, num_sms) or -1
+ * if that smid was never observed.  Built once per device by a probe kernel
+ * (reading R7: %smid is virtual and may be sparse, so cluster i binds to the
+ * SM of dense rank i rather than to smid i as Listing 5 l.14-15 does). */
+cc_status cc_sm_rank_table(int32_t device, int32_t* rank_of_smid, int32_t capacity,
+                           int32_t* smid_span);
+
+/* ---------------------------------------------------------------------------
+ * Launch: Step 3 binding + the task loop (§4.2.3-4.3, Listing 5)
+ * ------------------------------------------------------------------------- */
+typedef enum {
+    CC_BACKEND_DEFAULT = 0,        /* hardware CTA order: grid (gx, gy), body(blockIdx) --
+                                      the paper's baseline "BSL"              */
+    CC_BACKEND_AGENT = 1,          /* agent-based clustering (Listing 5; "CLU",
+                                      with throttling "CLU+TOT")                       */
+    CC_BACKEND_TBCLUSTER = 2,      /* Blackwell thread-block clusters: the hardware form
+                                      of clustering (conv2d only in this build)        */
+    CC_BACKEND_AGENT_IDENTITY = 3, /* persistence-only control: same agents, one global
+                                      queue in row-major order, no locality grouping   */
+    CC_BACKEND_REDIRECT = 4        /* redirection-based clustering "RD" (Listing 4,
+                                      Eq. 8 + Eq. 7; relies on RR dispatch)    */
+} cc_backend;
+
+typedef struct {
+    int32_t backend;        /* cc_backend                                               */
+    int32_t active_agents;  /* agents per SM that work (throttling, §4.3(I));
+                               0 => max_agents                                          */
+    int32_t max_agents;     /* agents launched per SM (MAX_AGENTS, Fig. 10); 0 => the
+                               occupancy limit of the kernel                            */
+    int32_t prefetch;       /* 1 => prefetch the next task's tile into L2 while the
+                               current one runs (§4.3(III), Listing 5 l.34-37)          */
+    int32_t steal;          /* 1 (default) => an agent whose cluster queue is empty
+                               takes work from other clusters, so every CTA runs exactly
+                               once whatever the hardware does with agent placement
+                               (reading R10); 0 => paper-faithful: CTAs of a cluster
+                               with no active agent are NOT run (census shows it)       */
+    int32_t cluster_size;   /* TBCLUSTER: CTAs per cluster along y (1..8)               */
+    uint32_t* d_census;     /* DEVICE, |V|, optional: census[lin] += 1 per execution;
+                               caller zeroes it                                        */
+    int32_t* d_exec_sm;     /* DEVICE, |V|, optional: %smid that executed lin          */
+    int32_t* d_map;         /* DEVICE, |V|, optional: d_map[v] = lin executed for the
+                               slot at order position v (agent/redirect/identity)      */
+} cc_launch_opts;
+
+/* Fill *opts with defaults: AGENT backend, max/active from occupancy, steal = 1,
+ * prefetch = 0, cluster_size = 2, no census/map. */
+cc_status cc_launch_opts_default(cc_launch_opts* opts);
+
+typedef enum {
+    CC_K_CENSUS = 0,   /* empty body: exercises binding/census only                */
+    CC_K_MATVEC = 1,   /* cc_matvec_args   (Listing 2; config 1)           */
+    CC_K_ATAX = 2,     /* cc_atax_args     (Table 2 ATX; config 2)                  */
+    CC_K_BICG = 3,     /* cc_bicg_args     (Table 2 BC)                             */
+    CC_K_MVT = 4,      /* cc_mvt_args      (Table 2 MVT)                            */
+    CC_K_JACOBI5 = 5,  /* cc_jacobi5_args  (config 3)                               */
+    CC_K_CONV2D = 6,   /* cc_conv2d_args   (config 4)                               */
+    CC_K_SPMV = 7      /* cc_spmv_args     (config 5)                               */
+} cc_kernel;
+
+/* CC_K_CENSUS: no data. */
+typedef struct { int32_t gx, gy; } cc_census_args;
+
+/* y += A x, A m x n row-major fp32 (DEVICE), lda % 4 == 0, lda >= n, A/x/y
+ * 16-byte aligned.  Logical CTA (bx, by) = 32 x 32 tile: rows 32*by.., columns
+ * 32*bx.. (Listing 2 layout: bx -> B[idx], by -> C[idy]); grid ceil(n/32) x
+ * ceil(m/32).  y is NOT zeroed (Listing 2 accumulates with atomicAdd). */
+typedef struct { const float* A; int64_t lda; int32_t m, n; const float* x; float* y; } cc_matvec_args;
+
+/* The ATAX/BICG/MVT family share one tile body: logical CTA (bx, by) is the
+ * 32 x 256 tile A[32*by .. +32, 256*bx .. +256]; grid ceil(n/256) x ceil(m/32).
+ * A m x n row-major fp32 DEVICE, lda % 4 == 0, lda >= n, 16-byte aligned. */
+/* ATAX: tmp = A x ; y = A^T tmp (two launches; tmp and y are zeroed by the call). */
+typedef struct { const float* A; int64_t lda; int32_t m, n; const float* x; float* tmp; float* y; } cc_atax_args;
+/* BICG: q = A p ; s = A^T r (one fused pass; q and s zeroed by the call). */
+typedef struct { const float* A; int64_t lda; int32_t m, n; const float* p; const float* r; float* q; float* s; } cc_bicg_args;
+/* MVT: x1 += A y1 ; x2 += A^T y2 (one fused pass, in place). */
+typedef struct { const float* A; int64_t lda; int32_t m, n; const float* y1; const float* y2; float* x1; float* x2; } cc_mvt_args;
+
+/* 5-point Jacobi sweeps (R14): b[i][j] = 0.2f*(c + w + e + n + s) on the interior,
+ * boundary rows/cols copied.  `iters` sweeps ping-pong a -> b -> a ...; on
+ * return *result_is_b (HOST, optional) says which buffer holds the last sweep.
+ * rows x cols fp32 DEVICE with leading dim ld (% 4 == 0).  Logical CTA = 32 x 32
+ * output tile; grid ceil(cols/32) x ceil(rows/32). */
+typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t iters; int32_t* result_is_b; } cc_jacobi5_args;
+
+/* 2D cross-correlation (R15) with a (2R+1)^2 filter w (HOST, copied into the
+ * launch parameters), R in {1, 3}; out = 0 outside [R, rows-R) x [R, cols-R).
+ * in/out rows x cols fp32 DEVICE, leading dim ld (% 4 == 0).  Logical CTA = 32x32
+ * output tile; grid ceil(cols/32) x ceil(rows/32). */
+typedef struct { const float* in; float* out; int64_t ld; int32_t rows, cols; int32_t R; const float* w; } cc_conv2d_args;
+
+/* CSR SpMV y = A x (R16).  DEVICE row_ptr[rows+1], col[nnz], val[nnz], x[cols],
+ * y[rows] (zeroed by the call), int32 indices, nnz < 2^31.  Logical CTA b owns
+ * the merge-path diagonals [4096 b, 4096 (b+1)) of the row-ends x nonzeros merge
+ * grid (so power-law rows are balanced); grid = ceil((rows+nnz)/4096) x 1.
+ * part (DEVICE, grid+1 entries) is the split table cc_spmv_partition fills once
+ * per matrix structure. */
+typedef struct { int32_t rows, cols; int64_t nnz; const int32_t* row_ptr; const int32_t* col;
+                 const float* val; const float* x; float* y; const int32_t* part; } cc_spmv_args;
+/* Fill args->part-sized DEVICE table `part` (gx+1 entries, gx from
+ * cc_kernel_grid) with the merge-path row coordinate of each logical CTA's
+ * first diagonal.  Asynchronous on `stream`. */
+cc_status cc_spmv_partition(const cc_spmv_args* args, int32_t* part, void* stream);
+
+/* Logical grid a kernel needs for `args` (so the caller can build the plan). */
+cc_status cc_kernel_grid(int32_t kernel, const void* args, int32_t* gx, int32_t* gy);
+/* Occupancy limit (agents per SM) of `kernel`'s agent body on `device`. */
+cc_status cc_max_agents(int32_t kernel, int32_t device, int32_t* max_agents);
+
+/* Run `kernel` over the plan's logical grid with the chosen backend, on
+ * `stream`.  The plan's grid must equal cc_kernel_grid(kernel, args).  The
+ * agent backends use the plan's workspace, which resets itself at the end of
+ * each launch, so launches sharing a plan must be stream-ordered.
+ * `launches` (HOST, optional) receives the number of kernels this call queued. */
+cc_status cc_launch(cc_plan plan, int32_t kernel, const void* args,
+                    const cc_launch_opts* opts, void* stream, int32_t* launches);
+
+/* Messages. */
+const char* cc_status_string(cc_status s);
+const char* cc_last_error(void);       /* thread-local detail of the last failure */
+int         cc_last_cuda_error(void);  /* cudaError_t behind the last CC_ERR_CUDA */
+const char* cc_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CTACLUST_H */

@@ -1,0 +1,607 @@
+// ctaclust.cu -- the C ABI of libctaclust (include/ctaclust.h): planner,
+// device binding facts, and the launch dispatcher over the kernel bodies.
+#include "../../include/ctaclust.h"
+
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "cc_index.cuh"
+#include "cc_runtime.cuh"
+#include "k_gemv.cuh"
+#include "k_spmv.cuh"
+#include "k_stencil.cuh"
+#include "k_tbcluster.cuh"
+
+using namespace cc;
+
+// ---------------------------------------------------------------------------
+// error plumbing: nothing crosses the ABI but a status and a thread-local text
+// ---------------------------------------------------------------------------
+static thread_local std::string g_err;
+static thread_local int g_cuda_err = 0;
+
+static cc_status fail(cc_status s, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+static cc_status fail(cc_status s, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return s;
+}
+static cc_status cuda_fail(cudaError_t e, const char* what) {
+    g_cuda_err = (int)e;
+    cudaGetLastError();   // clear sticky-free errors
+    return fail(CC_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+#define CC_CUDA(call)                                              \
+    do {                                                           \
+        cudaError_t e_ = (call);                                   \
+        if (e_ != cudaSuccess) return cuda_fail(e_, #call);        \
+    } while (0)
+
+// ---------------------------------------------------------------------------
+// per-device binding facts: SM count, %nsmid span and the dense rank table
+// ---------------------------------------------------------------------------
+__global__ void k_smid_probe(int32_t* out, int32_t* span, long long spin) {
+    if (threadIdx.x == 0) {
+        out[blockIdx.x] = (int32_t)smid();
+        if (blockIdx.x == 0) *span = (int32_t)nsmid();
+        long long t0 = clock64();
+        while (clock64() - t0 < spin) {}
+    }
+}
+
+struct DevFacts {
+    bool ready = false;
+    int num_sms = 0, smid_span = 0, l2 = 0;
+    std::vector<int32_t> rank_of_smid;   // host copy
+    int32_t* d_rank = nullptr;           // device copy (never freed: process lifetime)
+};
+static std::mutex g_dev_mu;
+static DevFacts g_dev[64];
+
+static cc_status dev_facts(int device, DevFacts** out) {
+    if (device < 0 || device >= 64) return fail(CC_ERR_INVALID_ARG, "device %d out of range", device);
+    std::lock_guard<std::mutex> lk(g_dev_mu);
+    DevFacts& f = g_dev[device];
+    if (f.ready) { *out = &f; return CC_OK; }
+    int prev = 0;
+    CC_CUDA(cudaGetDevice(&prev));
+    CC_CUDA(cudaSetDevice(device));
+    CC_CUDA(cudaDeviceGetAttribute(&f.num_sms, cudaDevAttrMultiProcessorCount, device));
+    CC_CUDA(cudaDeviceGetAttribute(&f.l2, cudaDevAttrL2CacheSize, device));
+    // probe: resident CTAs spinning on every SM record %smid (Listing 3 l.4)
+    std::vector<int32_t> seen;
+    int32_t span = 0;
+    for (int attempt = 0; attempt < 4; ++attempt) {
+        int nblk = f.num_sms * (attempt == 0 ? 8 : 16);
+        int32_t *d_out = nullptr, *d_span = nullptr;
+        CC_CUDA(cudaMalloc(&d_out, sizeof(int32_t) * nblk));
+        CC_CUDA(cudaMalloc(&d_span, sizeof(int32_t)));
+        k_smid_probe<<<nblk, 32>>>(d_out, d_span, 200000LL << attempt);
+        cudaError_t e = cudaDeviceSynchronize();
+        std::vector<int32_t> h(nblk);
+        if (e == cudaSuccess) e = cudaMemcpy(h.data(), d_out, sizeof(int32_t) * nblk, cudaMemcpyDeviceToHost);
+        if (e == cudaSuccess) e = cudaMemcpy(&span, d_span, sizeof(int32_t), cudaMemcpyDeviceToHost);
+        cudaFree(d_out);
+        cudaFree(d_span);
+        if (e != cudaSuccess) return cuda_fail(e, "smid probe");
+        seen.insert(seen.end(), h.begin(), h.end());
+        std::sort(seen.begin(), seen.end());
+        seen.erase(std::unique(seen.begin(), seen.end()), seen.end());
+        if ((int)seen.size() >= f.num_sms) break;
+    }
+    if (span <= 0) span = seen.empty() ? f.num_sms : seen.back() + 1;
+    span = std::max(span, seen.empty() ? 0 : seen.back() + 1);
+    f.smid_span = span;
+    f.rank_of_smid.assign(span, -1);
+    for (size_t k = 0; k < seen.size(); ++k) f.rank_of_smid[seen[k]] = (int32_t)k;
+    CC_CUDA(cudaMalloc(&f.d_rank, sizeof(int32_t) * span));
+    CC_CUDA(cudaMemcpy(f.d_rank, f.rank_of_smid.data(), sizeof(int32_t) * span, cudaMemcpyHostToDevice));
+    CC_CUDA(cudaSetDevice(prev));
+    f.ready = true;
+    *out = &f;
+    return CC_OK;
+}
+
+// ---------------------------------------------------------------------------
+// planner
+// ---------------------------------------------------------------------------
+struct cc_plan_s {
+    Grid g{};
+    int device = -1;
+    std::vector<int32_t> perm, offsets, user;
+    int32_t* d_user = nullptr;
+    int32_t* d_ws = nullptr;
+    DevFacts* facts = nullptr;
+};
+
+extern "C" cc_status cc_plan_create(const cc_plan_desc* d, cc_plan* out) {
+    if (!d || !out) return fail(CC_ERR_INVALID_ARG, "null argument");
+    *out = nullptr;
+    if (d->gx < 0 || d->gy < 0) return fail(CC_ERR_INVALID_ARG, "negative grid");
+    if (d->order < CC_ORDER_ROW || d->order > CC_ORDER_USER) return fail(CC_ERR_INVALID_ARG, "bad order %d", d->order);
+    if (d->order == CC_ORDER_TILE && (d->tile_w < 1 || d->tile_h < 1))
+        return fail(CC_ERR_INVALID_ARG, "tile dims must be >= 1");
+    int64_t V = (int64_t)d->gx * (int64_t)d->gy;
+    if (V > INT32_MAX) return fail(CC_ERR_OVERFLOW, "gx*gy = %lld exceeds int32", (long long)V);
+    if (d->order == CC_ORDER_USER && V > 0 && !d->user_order) return fail(CC_ERR_INVALID_ARG, "USER order needs user_order");
+    int M = d->num_clusters;
+    DevFacts* facts = nullptr;
+    if (d->device >= 0) {
+        cc_status s = dev_facts(d->device, &facts);
+        if (s != CC_OK) return s;
+        if (M == 0) M = facts->num_sms;
+    }
+    if (M < 1) return fail(CC_ERR_INVALID_ARG, "num_clusters must be >= 1 (or 0 with a device)");
+    cc_plan_s* p = new cc_plan_s();
+    p->device = d->device;
+    p->facts = facts;
+    Grid& g = p->g;
+    g.gx = d->gx; g.gy = d->gy; g.order = d->order;
+    g.tw = d->order == CC_ORDER_TILE ? d->tile_w : 1;
+    g.th = d->order == CC_ORDER_TILE ? d->tile_h : 1;
+    g.V = (int32_t)V; g.M = M; g.q = (int32_t)(V / M); g.r = (int32_t)(V % M);
+    if (d->order == CC_ORDER_USER) {
+        p->user.assign(d->user_order, d->user_order + V);
+        std::vector<uint8_t> hit(V, 0);
+        for (int64_t k = 0; k < V; ++k) {
+            int32_t l = p->user[k];
+            if (l < 0 || l >= V || hit[l]) { delete p; return fail(CC_ERR_NOT_PERMUTATION, "user_order[%lld] = %d", (long long)k, l); }
+            hit[l] = 1;
+        }
+    }
+    // Step 1 + 2: perm[v] = lin of the CTA at order position v.  Clusters are
+    // contiguous chunks of the order, so the cluster-major table is the order.
+    p->perm.resize(V);
+    for (int32_t v = 0; v < (int32_t)V; ++v) {
+        if (d->order == CC_ORDER_USER) { p->perm[v] = p->user[v]; continue; }
+        int32_t bx, by;
+        decode(g, v, &bx, &by);
+        p->perm[v] = by * g.gx + bx;
+    }
+    p->offsets.resize(M + 1);
+    for (int i = 0; i <= M; ++i) p->offsets[i] = i < M ? cluster_start(g, i) : g.V;
+    if (d->device >= 0) {
+        int prev = 0;
+        cudaError_t e = cudaGetDevice(&prev);
+        if (e == cudaSuccess) e = cudaSetDevice(d->device);
+        if (e == cudaSuccess) e = cudaMalloc(&p->d_ws, sizeof(int32_t) * ws_ints(M));
+        if (e == cudaSuccess) e = cudaMemset(p->d_ws, 0, sizeof(int32_t) * ws_ints(M));
+        if (e == cudaSuccess && d->order == CC_ORDER_USER && V > 0) {
+            e = cudaMalloc(&p->d_user, sizeof(int32_t) * V);
+            if (e == cudaSuccess) e = cudaMemcpy(p->d_user, p->user.data(), sizeof(int32_t) * V, cudaMemcpyHostToDevice);
+        }
+        if (e == cudaSuccess) e = cudaDeviceSynchronize();
+        cudaSetDevice(prev);
+        if (e != cudaSuccess) { cudaFree(p->d_ws); cudaFree(p->d_user); delete p; return cuda_fail(e, "plan device tables"); }
+    }
+    *out = p;
+    return CC_OK;
+}
+
+extern "C" cc_status cc_plan_destroy(cc_plan p) {
+    if (!p) return CC_OK;
+    if (p->d_ws) cudaFree(p->d_ws);
+    if (p->d_user) cudaFree(p->d_user);
+    delete p;
+    return CC_OK;
+}
+
+extern "C" cc_status cc_plan_info(cc_plan p, int64_t* V, int32_t* M, int32_t* q, int32_t* r) {
+    if (!p) return fail(CC_ERR_INVALID_ARG, "null plan");
+    if (V) *V = p->g.V;
+    if (M) *M = p->g.M;
+    if (q) *q = p->g.q;
+    if (r) *r = p->g.r;
+    return CC_OK;
+}
+
+extern "C" cc_status cc_plan_table(cc_plan p, int32_t* perm, int32_t* offsets) {
+    if (!p) return fail(CC_ERR_INVALID_ARG, "null plan");
+    if (perm && !p->perm.empty()) memcpy(perm, p->perm.data(), sizeof(int32_t) * p->perm.size());
+    if (offsets) memcpy(offsets, p->offsets.data(), sizeof(int32_t) * p->offsets.size());
+    return CC_OK;
+}
+
+extern "C" cc_status cc_plan_lookup(cc_plan p, int32_t v, int32_t* w, int32_t* i) {
+    if (!p || !w || !i) return fail(CC_ERR_INVALID_ARG, "null argument");
+    if (v < 0 || v >= p->g.V) return fail(CC_ERR_INVALID_ARG, "v = %d outside [0, %d)", v, p->g.V);
+    f_of(p->g, v, w, i);
+    return CC_OK;
+}
+
+extern "C" cc_status cc_plan_invert(cc_plan p, int32_t w, int32_t i, int32_t* v) {
+    if (!p || !v) return fail(CC_ERR_INVALID_ARG, "null argument");
+    if (i < 0 || i >= p->g.M || w < 0 || w >= cluster_size(p->g, i))
+        return fail(CC_ERR_INVALID_ARG, "(w, i) = (%d, %d) is not a slot", w, i);
+    *v = f_inv(p->g, w, i);
+    return CC_OK;
+}
+
+extern "C" cc_status cc_device_info(int32_t device, int32_t* num_sms, int32_t* smid_span, int32_t* l2) {
+    DevFacts* f = nullptr;
+    cc_status s = dev_facts(device, &f);
+    if (s != CC_OK) return s;
+    if (num_sms) *num_sms = f->num_sms;
+    if (smid_span) *smid_span = f->smid_span;
+    if (l2) *l2 = f->l2;
+    return CC_OK;
+}
+
+extern "C" cc_status cc_sm_rank_table(int32_t device, int32_t* rank, int32_t cap, int32_t* span) {
+    DevFacts* f = nullptr;
+    cc_status s = dev_facts(device, &f);
+    if (s != CC_OK) return s;
+    if (span) *span = f->smid_span;
+    if (rank) {
+        if (cap < f->smid_span) return fail(CC_ERR_INVALID_ARG, "capacity %d < smid span %d", cap, f->smid_span);
+        memcpy(rank, f->rank_of_smid.data(), sizeof(int32_t) * f->smid_span);
+    }
+    return CC_OK;
+}
+
+// ---------------------------------------------------------------------------
+// launch
+// ---------------------------------------------------------------------------
+extern "C" cc_status cc_launch_opts_default(cc_launch_opts* o) {
+    if (!o) return fail(CC_ERR_INVALID_ARG, "null opts");
+    memset(o, 0, sizeof *o);
+    o->backend = CC_BACKEND_AGENT;
+    o->steal = 1;
+    o->cluster_size = 2;
+    return CC_OK;
+}
+
+#define CC_TRY(x) do { cc_status s_ = (x); if (s_ != CC_OK) return s_; } while (0)
+
+static inline int32_t cdiv(int64_t a, int64_t b) { return (int32_t)((a + b - 1) / b); }
+static inline bool al16(const void* p) { return ((uintptr_t)p & 15) == 0; }
+
+extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32_t* gy) {
+    if (!a || !gx || !gy) return fail(CC_ERR_INVALID_ARG, "null argument");
+    switch (k) {
+    case CC_K_CENSUS: { auto* c = (const cc_census_args*)a; *gx = c->gx; *gy = c->gy; return CC_OK; }
+    case CC_K_MATVEC: { auto* c = (const cc_matvec_args*)a; *gx = cdiv(c->n, 32); *gy = cdiv(c->m, 32); return CC_OK; }
+    case CC_K_ATAX: { auto* c = (const cc_atax_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
+    case CC_K_BICG: { auto* c = (const cc_bicg_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
+    case CC_K_MVT: { auto* c = (const cc_mvt_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
+    case CC_K_JACOBI5: { auto* c = (const cc_jacobi5_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
+    case CC_K_CONV2D: { auto* c = (const cc_conv2d_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
+    case CC_K_SPMV: {
+        auto* c = (const cc_spmv_args*)a;
+        int64_t b = ((int64_t)c->rows + c->nnz + SPMV_IPC - 1) / SPMV_IPC;
+        if (b > INT32_MAX - 1) return fail(CC_ERR_OVERFLOW, "spmv grid");
+        *gx = (int32_t)b; *gy = 1; return CC_OK;
+    }
+    default: return fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
+    }
+}
+
+struct CensusParams { int32_t dummy; };
+struct CensusBody {
+    static constexpr int kThreads = 128;
+    using Params = CensusParams;
+    __device__ __forceinline__ explicit CensusBody(const CensusParams&) {}
+    __device__ __forceinline__ void run(int32_t, int32_t) {}
+    __device__ __forceinline__ void prefetch_l2(int32_t, int32_t) {}
+    __device__ __forceinline__ void finish() {}
+};
+
+using MatvecB = GemvBody<32, 32, true, false>;
+using RowB = GemvBody<32, 256, true, false>;
+using ColB = GemvBody<32, 256, false, true>;
+using BothB = GemvBody<32, 256, true, true>;
+
+template <class Body>
+static cc_status occupancy(int device, int* occ) {
+    static std::mutex mu;
+    static int cache[64] = {0};
+    std::lock_guard<std::mutex> lk(mu);
+    if (device < 0 || device >= 64) return fail(CC_ERR_INVALID_ARG, "device");
+    if (!cache[device]) {
+        int prev = 0, n = 0;
+        CC_CUDA(cudaGetDevice(&prev));
+        CC_CUDA(cudaSetDevice(device));
+        CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_agent<Body>, Body::kThreads, 0));
+        CC_CUDA(cudaSetDevice(prev));
+        cache[device] = n > 0 ? n : 1;
+    }
+    *occ = cache[device];
+    return CC_OK;
+}
+
+extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
+    if (!out) return fail(CC_ERR_INVALID_ARG, "null out");
+    int occ = 0;
+    cc_status s;
+    switch (k) {
+    case CC_K_CENSUS: s = occupancy<CensusBody>(device, &occ); break;
+    case CC_K_MATVEC: s = occupancy<MatvecB>(device, &occ); break;
+    case CC_K_ATAX: s = occupancy<RowB>(device, &occ); break;
+    case CC_K_BICG: case CC_K_MVT: s = occupancy<BothB>(device, &occ); break;
+    case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, &occ); break;
+    case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, &occ); break;
+    case CC_K_SPMV: s = occupancy<SpmvBody>(device, &occ); break;
+    default: return fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
+    }
+    if (s == CC_OK) *out = occ;
+    return s;
+}
+
+struct LaunchCtx {
+    cc_plan p;
+    const cc_launch_opts* o;
+    cudaStream_t st;
+    int32_t* nl;
+};
+
+template <class Body>
+static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& prm) {
+    const Grid& g = c.p->g;
+    if (g.V == 0) return CC_OK;
+    const cc_launch_opts& o = *c.o;
+    Sched s{};
+    s.g = g;
+    s.user = c.p->d_user;
+    s.rank_of_smid = c.p->facts->d_rank;
+    s.smid_span = c.p->facts->smid_span;
+    s.ws = c.p->d_ws;
+    s.steal = o.steal;
+    s.prefetch = o.prefetch;
+    s.census = o.d_census;
+    s.exec_sm = o.d_exec_sm;
+    s.map = o.d_map;
+    switch (o.backend) {
+    case CC_BACKEND_DEFAULT: {
+        if (g.gy > 65535) return fail(CC_ERR_UNSUPPORTED, "default backend: gy %d > 65535", g.gy);
+        s.map = nullptr;
+        k_default<Body><<<dim3(g.gx, g.gy), Body::kThreads, 0, c.st>>>(s, prm);
+        break;
+    }
+    case CC_BACKEND_REDIRECT:
+        k_redirect<Body><<<g.V, Body::kThreads, 0, c.st>>>(s, prm);
+        break;
+    case CC_BACKEND_AGENT:
+    case CC_BACKEND_AGENT_IDENTITY: {
+        int occ = 0;
+        cc_status st = occupancy<Body>(c.p->device, &occ);
+        if (st != CC_OK) return st;
+        int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
+        int act = o.active_agents > 0 ? std::min(o.active_agents, maxa) : maxa;
+        s.active_agents = act;
+        s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
+        int grid = c.p->facts->num_sms * maxa;
+        k_agent<Body><<<grid, Body::kThreads, 0, c.st>>>(s, prm);
+        break;
+    }
+    default:
+        return fail(CC_ERR_UNSUPPORTED, "backend %d not available for this kernel", o.backend);
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+    if (c.nl) ++*c.nl;
+    return CC_OK;
+}
+
+
+// ---- thread-block-cluster backend (conv2d) --------------------------------
+static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
+    static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaDriverEntryPointQueryResult q;
+        void* f = nullptr;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (PFN_cuTensorMapEncodeTiled_v12000)f;
+    });
+    return fn;
+}
+
+static cc_status make_tmap(CUtensorMap* m, const float* base, int32_t rows, int32_t cols, int64_t ld, int box_rows) {
+    auto enc = tmap_encoder();
+    if (!enc) return fail(CC_ERR_UNSUPPORTED, "cuTensorMapEncodeTiled unavailable");
+    cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+    cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
+    cuuint32_t box[2] = {(cuuint32_t)TBC_COLS, (cuuint32_t)box_rows};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)base, dims, strides, box, estr,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) return fail(CC_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+    return CC_OK;
+}
+
+template <int R>
+static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
+    const Grid& g = c.p->g;
+    if (g.V == 0) return CC_OK;
+    const int C = c.o->cluster_size;
+    if (C != 1 && C != 2 && C != 4 && C != 8) return fail(CC_ERR_INVALID_ARG, "cluster_size %d (1, 2, 4 or 8)", C);
+    const int gy_pad = (g.gy + C - 1) / C * C;
+    if (gy_pad > 65535) return fail(CC_ERR_UNSUPPORTED, "tbcluster: gy %d too large", g.gy);
+    CUtensorMap m_rows, m_halo;
+    CC_TRY(make_tmap(&m_rows, prm.in, prm.rows, prm.cols, prm.ld, 32));
+    CC_TRY(make_tmap(&m_halo, prm.in, prm.rows, prm.cols, prm.ld, TBC_HALO));
+    Sched s{};
+    s.g = g;
+    s.census = c.o->d_census;
+    s.exec_sm = c.o->d_exec_sm;
+    const size_t smem = tbc_smem_bytes(C);
+    CC_CUDA(cudaFuncSetAttribute(k_conv_tbc<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(g.gx, gy_pad);
+    cfg.blockDim = dim3(256);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = c.st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 1;
+    at[0].val.clusterDim.y = C;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    CC_CUDA(cudaLaunchKernelEx(&cfg, k_conv_tbc<R>, m_rows, m_halo, s, prm, (int32_t)C));
+    if (c.nl) ++*c.nl;
+    return CC_OK;
+}
+
+static cc_status check_mat(const float* A, int64_t lda, int32_t m, int32_t n) {
+    if (m < 0 || n < 0) return fail(CC_ERR_INVALID_ARG, "negative size");
+    if ((int64_t)m * n > 0 && !A) return fail(CC_ERR_INVALID_ARG, "null matrix");
+    if (lda < n || lda % 4) return fail(CC_ERR_INVALID_ARG, "lda %lld must be >= n and a multiple of 4", (long long)lda);
+    if (!al16(A)) return fail(CC_ERR_INVALID_ARG, "matrix not 16-byte aligned");
+    return CC_OK;
+}
+static cc_status check_vec(const void* v, int64_t len, const char* name) {
+    if (len > 0 && !v) return fail(CC_ERR_INVALID_ARG, "null %s", name);
+    if (!al16(v)) return fail(CC_ERR_INVALID_ARG, "%s not 16-byte aligned", name);
+    return CC_OK;
+}
+
+extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_launch_opts* opts,
+                               void* stream, int32_t* launches) {
+    if (!p || !a) return fail(CC_ERR_INVALID_ARG, "null plan or args");
+    if (launches) *launches = 0;
+    if (p->device < 0) return fail(CC_ERR_NO_DEVICE, "plan was created host-only");
+    cc_launch_opts dflt;
+    cc_launch_opts_default(&dflt);
+    const cc_launch_opts* o = opts ? opts : &dflt;
+    int32_t gx = 0, gy = 0;
+    CC_TRY(cc_kernel_grid(k, a, &gx, &gy));
+    if (gx != p->g.gx || gy != p->g.gy)
+        return fail(CC_ERR_INVALID_ARG, "plan grid %dx%d != kernel grid %dx%d", p->g.gx, p->g.gy, gx, gy);
+    if (o->backend == CC_BACKEND_TBCLUSTER && k != CC_K_CONV2D)
+        return fail(CC_ERR_UNSUPPORTED, "TBCLUSTER backend is implemented for conv2d only");
+    int prev = 0;
+    CC_CUDA(cudaGetDevice(&prev));
+    if (prev != p->device) CC_CUDA(cudaSetDevice(p->device));
+    cudaStream_t st = (cudaStream_t)stream;
+    LaunchCtx c{p, o, st, launches};
+    cc_status s = CC_OK;
+    switch (k) {
+    case CC_K_CENSUS: s = launch_body<CensusBody>(c, CensusParams{0}); break;
+    case CC_K_MATVEC: {
+        auto* x = (const cc_matvec_args*)a;
+        CC_TRY(check_mat(x->A, x->lda, x->m, x->n));
+        CC_TRY(check_vec(x->x, x->n, "x")); CC_TRY(check_vec(x->y, x->m, "y"));
+        s = launch_body<MatvecB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->x, nullptr, x->y, nullptr});
+        break;
+    }
+    case CC_K_ATAX: {
+        auto* x = (const cc_atax_args*)a;
+        CC_TRY(check_mat(x->A, x->lda, x->m, x->n));
+        CC_TRY(check_vec(x->x, x->n, "x")); CC_TRY(check_vec(x->tmp, x->m, "tmp")); CC_TRY(check_vec(x->y, x->n, "y"));
+        if (x->m) CC_CUDA(cudaMemsetAsync(x->tmp, 0, sizeof(float) * x->m, st));
+        if (x->n) CC_CUDA(cudaMemsetAsync(x->y, 0, sizeof(float) * x->n, st));
+        s = launch_body<RowB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->x, nullptr, x->tmp, nullptr});
+        if (s == CC_OK) s = launch_body<ColB>(c, GemvParams{x->A, x->lda, x->m, x->n, nullptr, x->tmp, nullptr, x->y});
+        break;
+    }
+    case CC_K_BICG: {
+        auto* x = (const cc_bicg_args*)a;
+        CC_TRY(check_mat(x->A, x->lda, x->m, x->n));
+        CC_TRY(check_vec(x->p, x->n, "p")); CC_TRY(check_vec(x->r, x->m, "r"));
+        CC_TRY(check_vec(x->q, x->m, "q")); CC_TRY(check_vec(x->s, x->n, "s"));
+        if (x->m) CC_CUDA(cudaMemsetAsync(x->q, 0, sizeof(float) * x->m, st));
+        if (x->n) CC_CUDA(cudaMemsetAsync(x->s, 0, sizeof(float) * x->n, st));
+        s = launch_body<BothB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->p, x->r, x->q, x->s});
+        break;
+    }
+    case CC_K_MVT: {
+        auto* x = (const cc_mvt_args*)a;
+        CC_TRY(check_mat(x->A, x->lda, x->m, x->n));
+        CC_TRY(check_vec(x->y1, x->n, "y1")); CC_TRY(check_vec(x->y2, x->m, "y2"));
+        CC_TRY(check_vec(x->x1, x->m, "x1")); CC_TRY(check_vec(x->x2, x->n, "x2"));
+        s = launch_body<BothB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->y1, x->y2, x->x1, x->x2});
+        break;
+    }
+    case CC_K_JACOBI5: {
+        auto* x = (const cc_jacobi5_args*)a;
+        CC_TRY(check_mat(x->a, x->ld, x->rows, x->cols));
+        CC_TRY(check_mat(x->b, x->ld, x->rows, x->cols));
+        if (x->iters < 0) return fail(CC_ERR_INVALID_ARG, "iters < 0");
+        float* src = x->a;
+        float* dst = x->b;
+        for (int it = 0; it < x->iters && s == CC_OK; ++it) {
+            s = launch_body<Jacobi5Body>(c, JacobiParams{src, dst, x->ld, x->rows, x->cols});
+            std::swap(src, dst);
+        }
+        if (x->result_is_b) *x->result_is_b = (x->iters & 1) ? 1 : 0;
+        break;
+    }
+    case CC_K_CONV2D: {
+        auto* x = (const cc_conv2d_args*)a;
+        CC_TRY(check_mat(x->in, x->ld, x->rows, x->cols));
+        CC_TRY(check_mat(x->out, x->ld, x->rows, x->cols));
+        if (!x->w) return fail(CC_ERR_INVALID_ARG, "null filter");
+        if (x->R == 1) {
+            ConvParams<1> cp{x->in, x->out, x->ld, x->rows, x->cols, {}};
+            memcpy(cp.w, x->w, sizeof cp.w);
+            s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<1>(c, cp)
+                                                   : launch_body<Conv2dBody<1>>(c, cp);
+        } else if (x->R == 3) {
+            ConvParams<3> cp{x->in, x->out, x->ld, x->rows, x->cols, {}};
+            memcpy(cp.w, x->w, sizeof cp.w);
+            s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<3>(c, cp)
+                                                   : launch_body<Conv2dBody<3>>(c, cp);
+        } else {
+            return fail(CC_ERR_UNSUPPORTED, "conv2d radius %d (1 or 3 supported)", x->R);
+        }
+        break;
+    }
+    case CC_K_SPMV: {
+        auto* x = (const cc_spmv_args*)a;
+        if (x->rows < 0 || x->cols < 0 || x->nnz < 0 || x->nnz > INT32_MAX) return fail(CC_ERR_INVALID_ARG, "spmv sizes");
+        if (!x->row_ptr || !x->part || !x->y || (x->nnz && (!x->col || !x->val || !x->x)))
+            return fail(CC_ERR_INVALID_ARG, "spmv null pointer");
+        if (x->rows) CC_CUDA(cudaMemsetAsync(x->y, 0, sizeof(float) * x->rows, st));
+        s = launch_body<SpmvBody>(c, SpmvParams{x->rows, x->nnz, x->row_ptr, x->col, x->val, x->x, x->y, x->part});
+        break;
+    }
+    default:
+        s = fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
+    }
+    if (prev != p->device) cudaSetDevice(prev);
+    return s;
+}
+
+extern "C" cc_status cc_spmv_partition(const cc_spmv_args* x, int32_t* part, void* stream) {
+    if (!x || !part || !x->row_ptr) return fail(CC_ERR_INVALID_ARG, "null argument");
+    int32_t gx = 0, gy = 0;
+    CC_TRY(cc_kernel_grid(CC_K_SPMV, x, &gx, &gy));
+    int n = gx + 1;
+    k_spmv_partition<<<(n + 255) / 256, 256, 0, (cudaStream_t)stream>>>(x->row_ptr, x->rows, x->nnz, gx, part);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "spmv partition");
+    return CC_OK;
+}
+
+extern "C" const char* cc_status_string(cc_status s) {
+    switch (s) {
+    case CC_OK: return "ok";
+    case CC_ERR_INVALID_ARG: return "invalid argument";
+    case CC_ERR_OVERFLOW: return "size overflow";
+    case CC_ERR_NOT_PERMUTATION: return "user order is not a permutation";
+    case CC_ERR_CUDA: return "CUDA error";
+    case CC_ERR_NCCL: return "NCCL error";
+    case CC_ERR_UNSUPPORTED: return "unsupported";
+    case CC_ERR_NO_DEVICE: return "plan has no device";
+    }
+    return "unknown status";
+}
+extern "C" const char* cc_last_error(void) { return g_err.c_str(); }
+extern "C" int cc_last_cuda_error(void) { return g_cuda_err; }
+extern "C" const char* cc_version(void) { return "libctaclust 0.1 (sm_100a)"; }

@@ -1,0 +1,159 @@
+// k_spmv.cuh -- CSR SpMV tile body (data-related locality class).
+//
+// y[i] = sum_{k in [rp[i], rp[i+1])} val[k] * x[col[k]]
+//
+// Logical CTA b owns the merge-path diagonal range [b*IPC, (b+1)*IPC) of the
+// (row ends) x (nonzeros) merge grid, so every logical CTA gets the same number
+// of rows + nonzeros however skewed the power-law degree distribution is.  Its
+// start coordinate comes from a precomputed table (cc_spmv_partition).  Inside
+// the CTA each thread merges IPT items; partial rows are stitched with a
+// CTA-wide segmented scan, so at most two atomics per logical CTA touch y
+// (the rows it shares with its neighbours); every other row is a plain store.
+// The x gathers go through L1 (the data-dependent inter-CTA reuse the paper
+// calls hard to exploit); val/col stream past it.
+#pragma once
+#include "cc_mem.cuh"
+
+namespace cc {
+
+struct SpmvParams {
+    int32_t rows; int64_t nnz;
+    const int32_t* row_ptr; const int32_t* col; const float* val; const float* x; float* y;
+    const int32_t* part;   // part[b] = row coordinate of diagonal b*IPC
+};
+
+constexpr int SPMV_IPT = 16;
+constexpr int SPMV_THREADS = 256;
+constexpr int SPMV_IPC = SPMV_IPT * SPMV_THREADS;   // merge items per logical CTA
+
+// Merge-path search (row ends a[0..a_len) vs natural numbers b[k] = k):
+// number of row ends consumed at diagonal d.
+__device__ __forceinline__ int64_t merge_search_global(const int32_t* row_end, int64_t a_len,
+                                                       int64_t b_len, int64_t d) {
+    int64_t lo = d - b_len > 0 ? d - b_len : 0;
+    int64_t hi = d < a_len ? d : a_len;
+    while (lo < hi) {
+        int64_t pv = (lo + hi) >> 1;
+        if ((int64_t)row_end[pv] <= d - pv - 1) lo = pv + 1;
+        else hi = pv;
+    }
+    return lo;
+}
+
+__global__ void k_spmv_partition(const int32_t* row_ptr, int32_t rows, int64_t nnz,
+                                 int32_t nblocks, int32_t* part) {
+    int32_t b = blockIdx.x * blockDim.x + threadIdx.x;
+    if (b > nblocks) return;
+    int64_t total = (int64_t)rows + nnz;
+    int64_t d = (int64_t)b * SPMV_IPC;
+    if (d > total) d = total;
+    part[b] = (int32_t)merge_search_global(row_ptr + 1, rows, nnz, d);
+}
+
+struct SpmvBody {
+    static constexpr int kThreads = SPMV_THREADS;
+    using Params = SpmvParams;
+    SpmvParams p;
+    __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}
+
+    __device__ __forceinline__ void run(int32_t bx, int32_t /*by*/) {
+        __shared__ int32_t s_rowend[SPMV_IPC + 1];
+        __shared__ float s_prod[SPMV_IPT][SPMV_THREADS];
+        __shared__ float s_wv[SPMV_THREADS / 32];
+        __shared__ int32_t s_wf[SPMV_THREADS / 32];
+        const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+        const int64_t total = (int64_t)p.rows + p.nnz;
+        const int64_t d0 = (int64_t)bx * SPMV_IPC;
+        const int64_t d1 = d0 + SPMV_IPC < total ? d0 + SPMV_IPC : total;
+        const int32_t x0 = p.part[bx], x1 = p.part[bx + 1];
+        const int64_t y0 = d0 - x0, y1 = d1 - x1;
+        const int32_t xl = x1 < p.rows ? x1 : p.rows - 1;      // last row to stage
+        for (int32_t i = t; i <= xl - x0; i += kThreads) s_rowend[i] = p.row_ptr[x0 + i + 1];
+        __syncthreads();
+        // this thread's start on the merge path, relative to the CTA rectangle
+        const int32_t span = (int32_t)(d1 - d0);
+        const int32_t dt = t * SPMV_IPT < span ? t * SPMV_IPT : span;
+        int32_t lo = dt - (int32_t)(y1 - y0); if (lo < 0) lo = 0;
+        int32_t hi = dt < (x1 - x0) ? dt : (x1 - x0);
+        while (lo < hi) {
+            int32_t pv = (lo + hi) >> 1;
+            if ((int64_t)s_rowend[pv] <= y0 + dt - pv - 1) lo = pv + 1;
+            else hi = pv;
+        }
+        const int32_t tx = x0 + lo;
+        const int64_t ty = y0 + dt - lo;
+        // products for up to IPT nonzeros from ty (independent loads: MLP)
+#pragma unroll
+        for (int k = 0; k < SPMV_IPT; ++k) {
+            int64_t idx = ty + k;
+            float pr = 0.f;
+            if (idx < y1) {
+                int32_t c = __ldcs(p.col + idx);
+                float v = __ldcs(p.val + idx);
+                pr = v * ld_cached(p.x + c);
+            }
+            s_prod[k][t] = pr;
+        }
+        // merge walk (s_prod column t is private to this thread: no barrier)
+        const int32_t items = span - dt < SPMV_IPT ? span - dt : SPMV_IPT;
+        float sum = 0.f, first_val = 0.f;
+        int32_t first_row = -1;
+        bool has_end = false;
+        int32_t cx = tx;
+        int64_t cy = ty;
+        for (int it = 0; it < items; ++it) {
+            if (cx < p.rows && cy < (int64_t)s_rowend[cx - x0]) {
+                sum += s_prod[cy - ty][t];
+                ++cy;
+            } else {
+                if (!has_end) { first_row = cx; first_val = sum; has_end = true; }
+                else p.y[cx] = sum;                 // row began and ended in this thread
+                sum = 0.f;
+                ++cx;
+            }
+        }
+        // segmented inclusive scan of (has_end, carry): T[t] = carry + (has_end ? 0 : T[t-1])
+        bool f = has_end;
+        float v = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            float vu = __shfl_up_sync(0xffffffffu, v, o);
+            int fu = __shfl_up_sync(0xffffffffu, (int)f, o);
+            if (lane >= o) { if (!f) v += vu; f = f || fu; }
+        }
+        if (lane == 31) { s_wv[warp] = v; s_wf[warp] = f; }
+        __syncthreads();
+        float pv = 0.f;                      // prefix of earlier warps
+        for (int w = 0; w < warp; ++w) pv = s_wf[w] ? s_wv[w] : pv + s_wv[w];
+        const float T = f ? v : pv + v;      // outgoing carry of this thread
+        float incoming = __shfl_up_sync(0xffffffffu, T, 1);
+        if (lane == 0) incoming = pv;
+        if (t == 0) incoming = 0.f;
+        if (has_end) {
+            float val = incoming + first_val;
+            const bool started_before = (first_row == x0) && (y0 > row_start(x0));
+            if (started_before) atomicAdd(p.y + first_row, val);
+            else p.y[first_row] = val;
+        }
+        if (t == kThreads - 1 && x1 < p.rows && T != 0.f) atomicAdd(p.y + x1, T);
+        __syncthreads();                     // s_wv / s_rowend reuse by the next task
+    }
+    __device__ __forceinline__ int64_t row_start(int32_t r) const {
+        return r == 0 ? 0 : (int64_t)p.row_ptr[r];
+    }
+    __device__ __forceinline__ void prefetch_l2(int32_t bx, int32_t) {
+        const int32_t x0 = p.part[bx];
+        const int64_t y0 = (int64_t)bx * SPMV_IPC - x0;
+        int64_t n = p.nnz - y0; if (n > SPMV_IPC) n = SPMV_IPC;
+        if (n <= 0) return;
+        const int32_t* c = p.col + y0;
+        const float* v = p.val + y0;
+        uintptr_t a = (uintptr_t)c & ~(uintptr_t)15, e = ((uintptr_t)(c + n) + 15) & ~(uintptr_t)15;
+        prefetch_l2_bulk((const void*)a, (uint32_t)(e - a));
+        a = (uintptr_t)v & ~(uintptr_t)15; e = ((uintptr_t)(v + n) + 15) & ~(uintptr_t)15;
+        prefetch_l2_bulk((const void*)a, (uint32_t)(e - a));
+    }
+    __device__ __forceinline__ void finish() {}
+};
+
+}  // namespace cc

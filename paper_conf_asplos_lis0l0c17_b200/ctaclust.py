@@ -1,0 +1,277 @@
+"""Thin ctypes binding over ``libctaclust.so`` (include/ctaclust.h).
+
+Argument marshalling only: every step of the hot path runs in the library's
+sm_100a kernels.  Names follow the C ABI (``cc_plan_create`` -> :class:`Plan`,
+``cc_launch`` -> :func:`launch` and the per-kernel helpers).  Device buffers are
+passed as torch CUDA tensors (PyTorch is used for memory and streams only).
+A missing library raises :class:`CtaclustError`; there is no fallback.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libctaclust.so")
+
+# ---- enums (ctaclust.h) ----------------------------------------------------
+ORDER_ROW, ORDER_COL, ORDER_TILE, ORDER_USER = 0, 1, 2, 3
+ORDERS = {"row": ORDER_ROW, "col": ORDER_COL, "tile": ORDER_TILE, "user": ORDER_USER}
+BACKEND_DEFAULT, BACKEND_AGENT, BACKEND_TBCLUSTER, BACKEND_AGENT_IDENTITY, BACKEND_REDIRECT = 0, 1, 2, 3, 4
+BACKENDS = {"default": 0, "agent": 1, "tbcluster": 2, "identity": 3, "redirect": 4}
+K_CENSUS, K_MATVEC, K_ATAX, K_BICG, K_MVT, K_JACOBI5, K_CONV2D, K_SPMV = range(8)
+KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7}
+STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_ERR_NOT_PERMUTATION",
+          -4: "CC_ERR_CUDA", -5: "CC_ERR_NCCL", -6: "CC_ERR_UNSUPPORTED", -7: "CC_ERR_NO_DEVICE"}
+
+# every symbol include/ctaclust.h declares (checked by tests/test_abi.py)
+EXPORTS = ["cc_plan_create", "cc_plan_destroy", "cc_plan_info", "cc_plan_table", "cc_plan_lookup",
+           "cc_plan_invert", "cc_device_info", "cc_sm_rank_table", "cc_launch_opts_default",
+           "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_status_string",
+           "cc_last_error", "cc_last_cuda_error", "cc_version"]
+
+
+class CtaclustError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+# ---- structs ----------------------------------------------------------------
+_i32, _i64, _vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_void_p
+
+
+class PlanDesc(ctypes.Structure):
+    _fields_ = [("gx", _i32), ("gy", _i32), ("order", _i32), ("tile_w", _i32), ("tile_h", _i32),
+                ("num_clusters", _i32), ("user_order", _vp), ("device", _i32)]
+
+
+class LaunchOpts(ctypes.Structure):
+    _fields_ = [("backend", _i32), ("active_agents", _i32), ("max_agents", _i32), ("prefetch", _i32),
+                ("steal", _i32), ("cluster_size", _i32), ("d_census", _vp), ("d_exec_sm", _vp),
+                ("d_map", _vp)]
+
+
+class CensusArgs(ctypes.Structure):
+    _fields_ = [("gx", _i32), ("gy", _i32)]
+
+
+class MatvecArgs(ctypes.Structure):
+    _fields_ = [("A", _vp), ("lda", _i64), ("m", _i32), ("n", _i32), ("x", _vp), ("y", _vp)]
+
+
+class AtaxArgs(ctypes.Structure):
+    _fields_ = [("A", _vp), ("lda", _i64), ("m", _i32), ("n", _i32), ("x", _vp), ("tmp", _vp), ("y", _vp)]
+
+
+class BicgArgs(ctypes.Structure):
+    _fields_ = [("A", _vp), ("lda", _i64), ("m", _i32), ("n", _i32), ("p", _vp), ("r", _vp), ("q", _vp), ("s", _vp)]
+
+
+class MvtArgs(ctypes.Structure):
+    _fields_ = [("A", _vp), ("lda", _i64), ("m", _i32), ("n", _i32), ("y1", _vp), ("y2", _vp), ("x1", _vp), ("x2", _vp)]
+
+
+class Jacobi5Args(ctypes.Structure):
+    _fields_ = [("a", _vp), ("b", _vp), ("ld", _i64), ("rows", _i32), ("cols", _i32), ("iters", _i32),
+                ("result_is_b", _vp)]
+
+
+class Conv2dArgs(ctypes.Structure):
+    _fields_ = [("inp", _vp), ("out", _vp), ("ld", _i64), ("rows", _i32), ("cols", _i32), ("R", _i32), ("w", _vp)]
+
+
+class SpmvArgs(ctypes.Structure):
+    _fields_ = [("rows", _i32), ("cols", _i32), ("nnz", _i64), ("row_ptr", _vp), ("col", _vp), ("val", _vp),
+                ("x", _vp), ("y", _vp), ("part", _vp)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libctaclust.so (raises if it was not built: no fallback path)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise CtaclustError(-6, f"{LIB_PATH} not built (run `make` or __graft_entry__.build())")
+        L = ctypes.CDLL(LIB_PATH)
+        for name in EXPORTS:
+            getattr(L, name)   # fail loudly on a missing export
+        L.cc_status_string.restype = ctypes.c_char_p
+        L.cc_last_error.restype = ctypes.c_char_p
+        L.cc_version.restype = ctypes.c_char_p
+        _lib = L
+    return _lib
+
+
+def _check(status: int):
+    if status != 0:
+        raise CtaclustError(status, lib().cc_last_error().decode())
+
+
+def version() -> str:
+    return lib().cc_version().decode()
+
+
+# ---- device facts -----------------------------------------------------------
+def device_info(device: int = 0) -> dict:
+    n, span, l2 = _i32(), _i32(), _i32()
+    _check(lib().cc_device_info(_i32(device), ctypes.byref(n), ctypes.byref(span), ctypes.byref(l2)))
+    return {"num_sms": n.value, "smid_span": span.value, "l2_bytes": l2.value}
+
+
+def sm_rank_table(device: int = 0) -> np.ndarray:
+    span = _i32()
+    _check(lib().cc_sm_rank_table(_i32(device), None, _i32(0), ctypes.byref(span)))
+    out = np.zeros(span.value, dtype=np.int32)
+    _check(lib().cc_sm_rank_table(_i32(device), out.ctypes.data_as(_vp), _i32(span.value), ctypes.byref(span)))
+    return out
+
+
+def max_agents(kernel, device: int = 0) -> int:
+    k = KERNELS[kernel] if isinstance(kernel, str) else kernel
+    out = _i32()
+    _check(lib().cc_max_agents(_i32(k), _i32(device), ctypes.byref(out)))
+    return out.value
+
+
+# ---- planner ------------------------------------------------------------------
+class Plan:
+    """A cluster partition of a gx x gy logical grid (cc_plan)."""
+
+    def __init__(self, gx: int, gy: int, order="row", num_clusters: int = 0, tile=(1, 1),
+                 user_order=None, device: int | None = 0):
+        o = ORDERS[order] if isinstance(order, str) else int(order)
+        self._user = None
+        if user_order is not None:
+            self._user = np.ascontiguousarray(user_order, dtype=np.int32)
+        d = PlanDesc(gx, gy, o, int(tile[0]), int(tile[1]), num_clusters,
+                     self._user.ctypes.data if self._user is not None else None,
+                     -1 if device is None else device)
+        h = _vp()
+        _check(lib().cc_plan_create(ctypes.byref(d), ctypes.byref(h)))
+        self.handle = h
+        self.gx, self.gy, self.order, self.device = gx, gy, o, device
+        V, M, q, r = _i64(), _i32(), _i32(), _i32()
+        _check(lib().cc_plan_info(h, ctypes.byref(V), ctypes.byref(M), ctypes.byref(q), ctypes.byref(r)))
+        self.V, self.M, self.q, self.r = V.value, M.value, q.value, r.value
+
+    def table(self):
+        perm = np.zeros(self.V, dtype=np.int32)
+        off = np.zeros(self.M + 1, dtype=np.int32)
+        _check(lib().cc_plan_table(self.handle, perm.ctypes.data_as(_vp), off.ctypes.data_as(_vp)))
+        return perm, off
+
+    def lookup(self, v: int):
+        w, i = _i32(), _i32()
+        _check(lib().cc_plan_lookup(self.handle, _i32(v), ctypes.byref(w), ctypes.byref(i)))
+        return w.value, i.value
+
+    def invert(self, w: int, i: int) -> int:
+        v = _i32()
+        _check(lib().cc_plan_invert(self.handle, _i32(w), _i32(i), ctypes.byref(v)))
+        return v.value
+
+    def close(self):
+        if getattr(self, "handle", None):
+            lib().cc_plan_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+# ---- launch --------------------------------------------------------------------
+def _ptr(t):
+    return None if t is None else t.data_ptr()
+
+
+def _stream(stream):
+    import torch
+    s = torch.cuda.current_stream() if stream is None else stream
+    return s.cuda_stream
+
+
+def make_opts(backend="agent", active_agents=0, max_agents=0, prefetch=0, steal=1, cluster_size=2,
+              census=None, exec_sm=None, map=None) -> LaunchOpts:
+    b = BACKENDS[backend] if isinstance(backend, str) else int(backend)
+    return LaunchOpts(b, active_agents, max_agents, int(prefetch), int(steal), cluster_size,
+                      _ptr(census), _ptr(exec_sm), _ptr(map))
+
+
+def kernel_grid(kernel, args) -> tuple[int, int]:
+    k = KERNELS[kernel] if isinstance(kernel, str) else kernel
+    gx, gy = _i32(), _i32()
+    _check(lib().cc_kernel_grid(_i32(k), ctypes.byref(args), ctypes.byref(gx), ctypes.byref(gy)))
+    return gx.value, gy.value
+
+
+def launch(plan: Plan, kernel, args, opts: LaunchOpts | None = None, stream=None) -> int:
+    """cc_launch; returns the number of kernels queued."""
+    k = KERNELS[kernel] if isinstance(kernel, str) else kernel
+    n = _i32()
+    _check(lib().cc_launch(plan.handle, _i32(k), ctypes.byref(args),
+                           ctypes.byref(opts) if opts is not None else None,
+                           _vp(_stream(stream)), ctypes.byref(n)))
+    return n.value
+
+
+def _lda(A):
+    assert A.dim() == 2 and A.stride(1) == 1, "row-major 2D tensor expected"
+    return A.stride(0)
+
+
+def matvec_args(A, x, y, m=None, n=None) -> MatvecArgs:
+    m = A.shape[0] if m is None else m
+    n = A.shape[1] if n is None else n
+    return MatvecArgs(A.data_ptr(), _lda(A), m, n, x.data_ptr(), y.data_ptr())
+
+
+def atax_args(A, x, tmp, y, m=None, n=None) -> AtaxArgs:
+    m = A.shape[0] if m is None else m
+    n = A.shape[1] if n is None else n
+    return AtaxArgs(A.data_ptr(), _lda(A), m, n, x.data_ptr(), tmp.data_ptr(), y.data_ptr())
+
+
+def bicg_args(A, p, r, q, s, m=None, n=None) -> BicgArgs:
+    m = A.shape[0] if m is None else m
+    n = A.shape[1] if n is None else n
+    return BicgArgs(A.data_ptr(), _lda(A), m, n, p.data_ptr(), r.data_ptr(), q.data_ptr(), s.data_ptr())
+
+
+def mvt_args(A, y1, y2, x1, x2, m=None, n=None) -> MvtArgs:
+    m = A.shape[0] if m is None else m
+    n = A.shape[1] if n is None else n
+    return MvtArgs(A.data_ptr(), _lda(A), m, n, y1.data_ptr(), y2.data_ptr(), x1.data_ptr(), x2.data_ptr())
+
+
+def jacobi5_args(a, b, iters, rows=None, cols=None) -> tuple[Jacobi5Args, ctypes.c_int32]:
+    flag = _i32(0)
+    rows = a.shape[0] if rows is None else rows
+    cols = a.shape[1] if cols is None else cols
+    args = Jacobi5Args(a.data_ptr(), b.data_ptr(), _lda(a), rows, cols, iters, ctypes.addressof(flag))
+    return args, flag
+
+
+def conv2d_args(inp, out, w, rows=None, cols=None) -> tuple[Conv2dArgs, np.ndarray]:
+    w = np.ascontiguousarray(np.asarray(w, dtype=np.float32))
+    K = w.shape[0]
+    rows = inp.shape[0] if rows is None else rows
+    cols = inp.shape[1] if cols is None else cols
+    return Conv2dArgs(inp.data_ptr(), out.data_ptr(), _lda(inp), rows, cols, K // 2, w.ctypes.data), w
+
+
+def spmv_args(row_ptr, col, val, x, y, part=None) -> SpmvArgs:
+    rows = row_ptr.numel() - 1
+    return SpmvArgs(rows, x.numel(), col.numel(), row_ptr.data_ptr(), col.data_ptr(), val.data_ptr(),
+                    x.data_ptr(), y.data_ptr(), _ptr(part))
+
+
+def spmv_partition(args: SpmvArgs, part, stream=None):
+    _check(lib().cc_spmv_partition(ctypes.byref(args), _vp(part.data_ptr()), _vp(_stream(stream))))

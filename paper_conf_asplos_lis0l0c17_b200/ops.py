@@ -1,0 +1,122 @@
+"""Tensor-level entry points over the C ABI (what tests, bench and users call).
+
+Each function allocates outputs with torch on the inputs' device, builds (and
+caches) the cluster plan for the kernel's logical grid, and issues one
+``cc_launch``.  No arithmetic of the method happens here.
+"""
+from __future__ import annotations
+
+import torch
+
+from . import ctaclust as cc
+
+# default partition per kernel (Table 2 / §4.2.1): the ATAX family is X-P
+# (column-major indexing, "X-P" for ATX/MVT/BC in Table 2);
+# stencils use tile-wise indexing (Fig. 7); matvec row-clustering per config 1.
+DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": ("col", (1, 1)),
+                 "bicg": ("col", (1, 1)), "mvt": ("col", (1, 1)), "jacobi5": ("tile", (8, 8)),
+                 "conv2d": ("tile", (8, 8)), "spmv": ("row", (1, 1))}
+
+_plans: dict = {}
+
+
+def plan_for(kernel: str, args, order=None, tile=None, num_clusters: int = 0, device: int = 0,
+             user_order=None) -> cc.Plan:
+    gx, gy = cc.kernel_grid(kernel, args)
+    o, t = DEFAULT_ORDER[kernel]
+    order = o if order is None else order
+    tile = t if tile is None else tile
+    if user_order is not None:
+        return cc.Plan(gx, gy, "user", num_clusters, user_order=user_order, device=device)
+    key = (gx, gy, order, tuple(tile) if order == "tile" else (1, 1), num_clusters, device)
+    p = _plans.get(key)
+    if p is None:
+        p = cc.Plan(gx, gy, order, num_clusters, tile=tile, device=device)
+        _plans[key] = p
+    return p
+
+
+def _dev(t: torch.Tensor) -> int:
+    if not t.is_cuda:
+        raise cc.CtaclustError(-1, "libctaclust operates on CUDA tensors only")
+    return t.device.index or 0
+
+
+def _launch(kernel, args, backend, order, tile, num_clusters, device, stream, **kw):
+    p = plan_for(kernel, args, order, tile, num_clusters, device)
+    return cc.launch(p, kernel, args, cc.make_opts(backend, **kw), stream)
+
+
+def matvec(A, x, y=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+    """y (+)= A x  (Listing 2).  y is accumulated into when given, else zero-initialised."""
+    y = torch.zeros(A.shape[0], dtype=torch.float32, device=A.device) if y is None else y
+    _launch("matvec", cc.matvec_args(A, x, y), backend, order, tile, num_clusters, _dev(A), stream, **kw)
+    return y
+
+
+def atax(A, x, backend="agent", order=None, tile=None, num_clusters=0, stream=None, out=None, **kw):
+    tmp, y = out if out is not None else (torch.empty(A.shape[0], device=A.device), torch.empty(A.shape[1], device=A.device))
+    _launch("atax", cc.atax_args(A, x, tmp, y), backend, order, tile, num_clusters, _dev(A), stream, **kw)
+    return tmp, y
+
+
+def bicg(A, p, r, backend="agent", order=None, tile=None, num_clusters=0, stream=None, out=None, **kw):
+    q, s = out if out is not None else (torch.empty(A.shape[0], device=A.device), torch.empty(A.shape[1], device=A.device))
+    _launch("bicg", cc.bicg_args(A, p, r, q, s), backend, order, tile, num_clusters, _dev(A), stream, **kw)
+    return q, s
+
+
+def mvt(A, y1, y2, x1, x2, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+    """In place: x1 += A y1 ; x2 += A^T y2."""
+    _launch("mvt", cc.mvt_args(A, y1, y2, x1, x2), backend, order, tile, num_clusters, _dev(A), stream, **kw)
+    return x1, x2
+
+
+def jacobi5(a, b, iters, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+    """`iters` sweeps ping-ponging a <-> b; returns the buffer holding the result."""
+    args, flag = cc.jacobi5_args(a, b, iters)
+    _launch("jacobi5", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
+    return b if flag.value else a
+
+
+def conv2d(inp, w, out=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+    out = torch.empty_like(inp) if out is None else out
+    args, _w = cc.conv2d_args(inp, out, w)
+    _launch("conv2d", args, backend, order, tile, num_clusters, _dev(inp), stream, **kw)
+    return out
+
+
+class SpmvMatrix:
+    """A CSR matrix resident on the device plus its merge-path split table."""
+
+    def __init__(self, row_ptr, col, val, n_cols=None, stream=None):
+        self.row_ptr, self.col, self.val = row_ptr, col, val
+        self.rows = row_ptr.numel() - 1
+        self.cols = self.rows if n_cols is None else n_cols
+        x = torch.empty(0, device=row_ptr.device)
+        probe = cc.SpmvArgs(self.rows, self.cols, col.numel(), row_ptr.data_ptr(), col.data_ptr(),
+                            val.data_ptr(), x.data_ptr(), x.data_ptr(), None)
+        gx, _ = cc.kernel_grid("spmv", probe)
+        self.part = torch.empty(gx + 1, dtype=torch.int32, device=row_ptr.device)
+        cc.spmv_partition(probe, self.part, stream)
+
+
+def spmv(Amat: SpmvMatrix, x, y=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+    y = torch.empty(Amat.rows, dtype=torch.float32, device=x.device) if y is None else y
+    args = cc.SpmvArgs(Amat.rows, Amat.cols, Amat.col.numel(), Amat.row_ptr.data_ptr(), Amat.col.data_ptr(),
+                       Amat.val.data_ptr(), x.data_ptr(), y.data_ptr(), Amat.part.data_ptr())
+    _launch("spmv", args, backend, order, tile, num_clusters, _dev(x), stream, **kw)
+    return y
+
+
+def census(gx, gy, backend="agent", order="row", tile=(1, 1), num_clusters=0, device=0, stream=None,
+           user_order=None, with_map=True, **kw):
+    """Run the empty body over a gx x gy grid; returns (census, exec_sm, map, plan)."""
+    args = cc.CensusArgs(gx, gy)
+    p = plan_for("census", args, order, tile, num_clusters, device, user_order)
+    dv = torch.device("cuda", device)
+    cen = torch.zeros(gx * gy, dtype=torch.int32, device=dv)
+    sm = torch.full((gx * gy,), -1, dtype=torch.int32, device=dv)
+    mp = torch.full((gx * gy,), -1, dtype=torch.int32, device=dv) if with_map else None
+    cc.launch(p, "census", args, cc.make_opts(backend, census=cen, exec_sm=sm, map=mp, **kw), stream)
+    return cen, sm, mp, p

@@ -1,0 +1,61 @@
+"""Row sharding of the ATAX/BICG/MVT family over G GPUs.
+
+Rank g owns rows [row_lo(g), row_hi(g)) of A and the matching slices of the
+row-indexed vectors; column-indexed inputs are replicated.  The row products
+(A x, A p, A y1) are then purely local; the transposed products (A^T tmp,
+A^T r, A^T y2) are sums over all row blocks, so each rank produces a partial
+n-vector and one all-reduce (NCCL over NVLink; gloo in the CPU tests) forms
+the total -- the only data-path exchange.  ATAX needs no exchange between its
+passes: pass 2 consumes exactly the tmp rows pass 1 produced locally.
+Row-indexed outputs are gathered at the end (all-gather).
+
+`compute` callables do the per-rank arithmetic (the CUDA kernels in bench and
+users' code; the oracle in the CPU tests); this module only moves vectors.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+
+def row_range(n_rows: int, world: int, rank: int) -> tuple[int, int]:
+    """Balanced contiguous row blocks: the first n_rows % world ranks get one more."""
+    q, r = divmod(n_rows, world)
+    lo = rank * q + min(rank, r)
+    return lo, lo + q + (1 if rank < r else 0)
+
+
+def _allreduce(t: torch.Tensor, world: int):
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return t
+
+
+def _allgather_rows(local: torch.Tensor, n_rows: int, world: int) -> torch.Tensor:
+    if world == 1:
+        return local
+    sizes = [row_range(n_rows, world, g) for g in range(world)]
+    cap = max(hi - lo for lo, hi in sizes)
+    buf = torch.zeros(cap, dtype=local.dtype, device=local.device)
+    buf[: local.numel()] = local
+    out = [torch.empty_like(buf) for _ in range(world)]
+    dist.all_gather(out, buf)
+    return torch.cat([out[g][: hi - lo] for g, (lo, hi) in enumerate(sizes)])
+
+
+def sharded_step(compute, n_rows: int, world: int, rank: int, gather: bool = True) -> dict:
+    """One ATAX + BICG + MVT step on this rank's row block.
+
+    ``compute(lo, hi)`` runs the local kernels and returns a dict with the
+    row-part outputs ``tmp``, ``q``, ``x1`` (length hi-lo) and the partial
+    column-part outputs ``y``, ``s``, ``x2d`` (length n; x2d is the A^T y2
+    contribution only).  Returns the combined results (x2 = x2_init + sum x2d
+    is left to the caller, which owns x2_init)."""
+    lo, hi = row_range(n_rows, world, rank)
+    part = compute(lo, hi)
+    for key in ("y", "s", "x2d"):
+        _allreduce(part[key], world)
+    if gather:
+        for key in ("tmp", "q", "x1"):
+            part[key] = _allgather_rows(part[key], n_rows, world)
+    return part

@@ -22,26 +22,28 @@ _M32 = 0xFFFFFFFF
 
 
 def _mix_np(x):
-    # lowbias32 finaliser on uint64-held 32-bit words
-    x = x ^ (x >> np.uint64(16))
-    x = (x * np.uint64(0x7FEB352D)) & np.uint64(_M32)
-    x = x ^ (x >> np.uint64(15))
-    x = (x * np.uint64(0x846CA68B)) & np.uint64(_M32)
-    x = x ^ (x >> np.uint64(16))
+    # lowbias32 finaliser on uint32 words (numpy uint32 arithmetic wraps mod 2^32)
+    x = x ^ (x >> np.uint32(16))
+    x = x * np.uint32(0x7FEB352D)
+    x = x ^ (x >> np.uint32(15))
+    x = x * np.uint32(0x846CA68B)
+    x = x ^ (x >> np.uint32(16))
     return x
 
 
 def _seed_word(seed: int, stream: int) -> int:
-    s = np.uint64(((seed * 0x9E3779B9) + 0x632BE5AB + stream * 0x2545F491) & _M32)
-    return int(_mix_np(np.array([s], dtype=np.uint64))[0])
+    s = np.uint32(((seed * 0x9E3779B9) + 0x632BE5AB + stream * 0x2545F491) & _M32)
+    return int(_mix_np(np.array([s], dtype=np.uint32))[0])
 
 
-def hash_u32_np(seed: int, idx: np.ndarray, stream: int = 0) -> np.ndarray:
-    """32-bit hash of (seed, stream, idx) for int64 idx >= 0, as uint64 words."""
+def hash_u32_np(seed: int, idx, stream: int = 0) -> np.ndarray:
+    """32-bit hash of (seed, stream, idx) for int64 idx >= 0, as uint32 words."""
     idx = np.asarray(idx, dtype=np.uint64)
-    s = np.uint64(_seed_word(seed, stream))
-    h = _mix_np((idx & np.uint64(_M32)) ^ s)
-    h = _mix_np(h ^ ((idx >> np.uint64(32)) & np.uint64(_M32)) ^ np.uint64(0x85EBCA6B))
+    s = np.uint32(_seed_word(seed, stream))
+    lo = (idx & np.uint64(_M32)).astype(np.uint32)
+    hi = (idx >> np.uint64(32)).astype(np.uint32)
+    h = _mix_np(lo ^ s)
+    h = _mix_np(h ^ hi ^ np.uint32(0x85EBCA6B))
     return h
 
 
@@ -67,9 +69,13 @@ def uniform(seed: int, count: int, start: int = 0, *, backend: str = "numpy",
             device=None, stream: int = 0, chunk: int = 1 << 26):
     """``count`` U[0,1) fp32 values for logical indices start..start+count-1."""
     if backend == "numpy":
-        idx = np.arange(start, start + count, dtype=np.uint64)
-        h = hash_u32_np(seed, idx, stream)
-        return ((h >> np.uint64(8)).astype(np.float64) * (2.0 ** -24)).astype(np.float32)
+        out = np.empty(count, dtype=np.float32)
+        for c0 in range(0, count, chunk):
+            c1 = min(count, c0 + chunk)
+            idx = np.arange(start + c0, start + c1, dtype=np.uint64)
+            h = hash_u32_np(seed, idx, stream)
+            out[c0:c1] = (h >> np.uint32(8)).astype(np.float32) * np.float32(2.0 ** -24)
+        return out
     import torch
     out = torch.empty(count, dtype=torch.float32, device=device)
     for c0 in range(0, count, chunk):
@@ -87,7 +93,7 @@ def small_int(seed: int, count: int, start: int = 0, *, lo: int = -8, hi: int = 
     if backend == "numpy":
         idx = np.arange(start, start + count, dtype=np.uint64)
         h = hash_u32_np(seed, idx, stream)
-        return ((h % np.uint64(span)).astype(np.int64) + lo).astype(np.float32)
+        return ((h % np.uint32(span)).astype(np.int64) + lo).astype(np.float32)
     import torch
     idx = torch.arange(start, start + count, dtype=torch.int64, device=device)
     h = hash_u32_torch(seed, idx, stream)
@@ -126,8 +132,10 @@ def matrix(seed: int, rows: int, cols: int, *, ld: int | None = None, kind: str 
 RMAT_ABCD = (0.57, 0.19, 0.19, 0.05)
 
 
-def rmat_csr(seed: int, scale: int, edge_factor: int, *, chunk: int = 1 << 22):
-    """CSR of an R-MAT graph with 2**scale rows (numpy; deterministic)."""
+def rmat_csr(seed: int, scale: int, edge_factor: int, *, chunk: int = 1 << 22,
+             backend: str = "numpy", device=None):
+    """CSR of an R-MAT graph with 2**scale rows; numpy and torch give identical
+    graphs (same hash draws and integer thresholds)."""
     n = 1 << scale
     nedges = edge_factor * n
     a, b, c, _ = RMAT_ABCD
@@ -135,29 +143,54 @@ def rmat_csr(seed: int, scale: int, edge_factor: int, *, chunk: int = 1 << 22):
     t_a = int(a * (1 << 24))
     t_ab = int((a + b) * (1 << 24))
     t_abc = int((a + b + c) * (1 << 24))
-    keys = np.empty(nedges, dtype=np.int64)
+    if backend == "numpy":
+        keys = np.empty(nedges, dtype=np.int64)
+        for e0 in range(0, nedges, chunk):
+            e1 = min(nedges, e0 + chunk)
+            e = np.arange(e0, e1, dtype=np.uint64)
+            row = np.zeros(e1 - e0, dtype=np.int64)
+            col = np.zeros(e1 - e0, dtype=np.int64)
+            for lvl in range(scale):
+                u = (hash_u32_np(seed, e * np.uint64(scale) + np.uint64(lvl), stream=7) >> np.uint32(8)).astype(np.int64)
+                down = (u >= t_ab)                                  # quadrant c or d -> row bit
+                right = ((u >= t_a) & (u < t_ab)) | (u >= t_abc)    # quadrant b or d -> col bit
+                bit = np.int64(1) << np.int64(scale - 1 - lvl)
+                row |= np.where(down, bit, 0)
+                col |= np.where(right, bit, 0)
+            keys[e0:e1] = row * n + col
+        keys = np.unique(keys)                                      # sorts and drops duplicates
+        rows_of = (keys // n).astype(np.int64)
+        cols = (keys % n).astype(np.int32)
+        counts = np.bincount(rows_of, minlength=n)
+        row_ptr = np.zeros(n + 1, dtype=np.int64)
+        np.cumsum(counts, out=row_ptr[1:])
+        if row_ptr[-1] >= 2 ** 31:
+            raise ValueError("nnz exceeds int32 row_ptr")
+        return row_ptr.astype(np.int32), cols
+    import torch
+    chunk = max(chunk, 1 << 24)
+    parts = []
     for e0 in range(0, nedges, chunk):
         e1 = min(nedges, e0 + chunk)
-        e = np.arange(e0, e1, dtype=np.uint64)
-        row = np.zeros(e1 - e0, dtype=np.int64)
-        col = np.zeros(e1 - e0, dtype=np.int64)
+        e = torch.arange(e0, e1, dtype=torch.int64, device=device)
+        row = torch.zeros(e1 - e0, dtype=torch.int64, device=device)
+        col = torch.zeros_like(row)
         for lvl in range(scale):
-            u = (hash_u32_np(seed, e * np.uint64(scale) + np.uint64(lvl), stream=7) >> np.uint64(8)).astype(np.int64)
-            down = (u >= t_ab)                      # quadrant c or d -> row bit
-            right = ((u >= t_a) & (u < t_ab)) | (u >= t_abc)   # quadrant b or d -> col bit
-            bit = np.int64(1) << np.int64(scale - 1 - lvl)
-            row |= np.where(down, bit, 0)
-            col |= np.where(right, bit, 0)
-        keys[e0:e1] = row * n + col
-    keys = np.unique(keys)                          # sorts and drops duplicates
-    rows_of = (keys // n).astype(np.int64)
-    cols = (keys % n).astype(np.int32)
-    counts = np.bincount(rows_of, minlength=n)
-    row_ptr = np.zeros(n + 1, dtype=np.int64)
-    np.cumsum(counts, out=row_ptr[1:])
-    if row_ptr[-1] >= 2 ** 31:
+            u = hash_u32_torch(seed, e * scale + lvl, stream=7) >> 8
+            bit = 1 << (scale - 1 - lvl)
+            row |= (u >= t_ab).to(torch.int64) * bit
+            col |= (((u >= t_a) & (u < t_ab)) | (u >= t_abc)).to(torch.int64) * bit
+        parts.append(torch.unique(row * n + col))
+    keys = torch.unique(torch.cat(parts))
+    del parts
+    rows_of = keys // n
+    cols = (keys % n).to(torch.int32)
+    counts = torch.bincount(rows_of, minlength=n)
+    row_ptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    torch.cumsum(counts, 0, out=row_ptr[1:])
+    if int(row_ptr[-1]) >= 2 ** 31:
         raise ValueError("nnz exceeds int32 row_ptr")
-    return row_ptr.astype(np.int32), cols
+    return row_ptr.to(torch.int32), cols
 
 
 def random_permutation(seed: int, n: int) -> np.ndarray:

@@ -1,0 +1,158 @@
+"""CPU-only checks of the C ABI: the library loads without a GPU, exports every
+symbol include/ctaclust.h declares, its struct layouts match the binding, and
+its host-only planner equals the independent oracle partition bit for bit."""
+import ctypes
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+from oracle import plan as OP
+from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "ctaclust.h")
+
+
+def header_functions():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(cc_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_header_declares_what_binding_lists():
+    assert header_functions() == sorted(cc.EXPORTS)
+
+
+def test_library_exports_every_declared_symbol():
+    out = subprocess.check_output(["nm", "-D", "--defined-only", cc.LIB_PATH], text=True)
+    syms = {ln.split()[-1] for ln in out.splitlines() if ln.strip()}
+    missing = [f for f in header_functions() if f not in syms]
+    assert not missing, missing
+    L = cc.lib()
+    assert cc.version().startswith("libctaclust")
+    assert L.cc_status_string(-3) == b"user order is not a permutation"
+
+
+LAYOUT_C = r"""
+#include <stdio.h>
+#include <stddef.h>
+#include "ctaclust.h"
+#define S(T) printf(#T " %zu\n", sizeof(T));
+#define O(T, f) printf(#T "." #f " %zu\n", offsetof(T, f));
+int main(void) {
+  S(cc_plan_desc) O(cc_plan_desc, user_order) O(cc_plan_desc, device)
+  S(cc_launch_opts) O(cc_launch_opts, d_census) O(cc_launch_opts, d_map)
+  S(cc_matvec_args) O(cc_matvec_args, y) S(cc_atax_args) O(cc_atax_args, y)
+  S(cc_bicg_args) O(cc_bicg_args, s) S(cc_mvt_args) O(cc_mvt_args, x2)
+  S(cc_jacobi5_args) O(cc_jacobi5_args, result_is_b) S(cc_conv2d_args) O(cc_conv2d_args, w)
+  S(cc_spmv_args) O(cc_spmv_args, part) O(cc_spmv_args, nnz)
+  return 0;
+}
+"""
+
+
+def test_struct_layouts_match_binding(tmp_path):
+    src = tmp_path / "layout.c"
+    src.write_text(LAYOUT_C)
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), "-o", str(exe), str(src)])
+    got = dict(ln.rsplit(" ", 1) for ln in subprocess.check_output([str(exe)], text=True).splitlines())
+    py = {"cc_plan_desc": cc.PlanDesc, "cc_launch_opts": cc.LaunchOpts, "cc_matvec_args": cc.MatvecArgs,
+          "cc_atax_args": cc.AtaxArgs, "cc_bicg_args": cc.BicgArgs, "cc_mvt_args": cc.MvtArgs,
+          "cc_jacobi5_args": cc.Jacobi5Args, "cc_conv2d_args": cc.Conv2dArgs, "cc_spmv_args": cc.SpmvArgs}
+    for key, val in got.items():
+        if "." in key:
+            t, f = key.split(".")
+            f = {"w": "w"}.get(f, f)
+            assert getattr(py[t], f).offset == int(val), key
+        else:
+            assert ctypes.sizeof(py[key]) == int(val), key
+
+
+# ---- host-only planner vs the oracle ----------------------------------------
+@pytest.mark.parametrize("order", ["row", "col", "tile"])
+def test_planner_matches_oracle_tiny_grids(order):
+    o = cc.ORDERS[order]
+    for gx in range(1, 9):
+        for gy in range(1, 9):
+            for M in (1, 2, 3, 7, gx * gy, gx * gy + 3):
+                p = cc.Plan(gx, gy, order, num_clusters=M, tile=(3, 2), device=None)
+                perm, off = p.table()
+                ref = OP.plan(gx, gy, o, M, 3, 2)
+                assert np.array_equal(perm, ref["perm"]) and np.array_equal(off, ref["offsets"])
+                assert (p.q, p.r) == (ref["q"], ref["r"])
+                V = gx * gy
+                for v in range(V):
+                    w, i = p.lookup(v)
+                    assert (w, i) == OP.f(V, M, v)
+                    assert p.invert(w, i) == v
+
+
+@pytest.mark.parametrize("gx,gy,order,tile,M", [
+    (32, 32, "row", (1, 1), 148),        # config 1 matvec grid
+    (64, 512, "col", (1, 1), 148),       # config 2 ATAX-family grid (n = 16384, 32x256 tiles)
+    (512, 512, "tile", (8, 8), 148),     # config 3 Jacobi grid
+    (256, 256, "tile", (4, 4), 148),     # config 4 conv grid
+    (300, 7, "tile", (8, 3), 37),        # ragged tiles
+])
+def test_planner_matches_oracle_config_grids(gx, gy, order, tile, M):
+    p = cc.Plan(gx, gy, order, num_clusters=M, tile=tile, device=None)
+    perm, off = p.table()
+    ref = OP.plan(gx, gy, cc.ORDERS[order], M, *tile)
+    assert np.array_equal(perm, ref["perm"]) and np.array_equal(off, ref["offsets"])
+
+
+def test_planner_user_order_and_errors():
+    rng = np.random.default_rng(0)
+    u = rng.permutation(35).astype(np.int32)
+    p = cc.Plan(7, 5, "user", num_clusters=4, user_order=u, device=None)
+    perm, off = p.table()
+    ref = OP.plan(7, 5, OP.USER, 4, user_order=u)
+    assert np.array_equal(perm, ref["perm"]) and np.array_equal(off, ref["offsets"])
+    bad = u.copy()
+    bad[3] = bad[4]
+    with pytest.raises(cc.CtaclustError) as e:
+        cc.Plan(7, 5, "user", num_clusters=4, user_order=bad, device=None)
+    assert e.value.status == -3
+    with pytest.raises(cc.CtaclustError) as e:
+        cc.Plan(70000, 70000, "row", num_clusters=4, device=None)
+    assert e.value.status == -2
+    with pytest.raises(cc.CtaclustError) as e:
+        cc.Plan(-1, 4, "row", num_clusters=4, device=None)
+    assert e.value.status == -1
+    with pytest.raises(cc.CtaclustError) as e:
+        cc.Plan(4, 4, "tile", num_clusters=4, tile=(0, 2), device=None)
+    assert e.value.status == -1
+    with pytest.raises(cc.CtaclustError) as e:
+        cc.Plan(4, 4, "row", num_clusters=0, device=None)        # M = 0 needs a device
+    assert e.value.status == -1
+    p = cc.Plan(4, 4, "row", num_clusters=3, device=None)
+    with pytest.raises(cc.CtaclustError):
+        p.lookup(16)
+    with pytest.raises(cc.CtaclustError):
+        p.invert(5, 2)                                           # cluster 2 has 5 slots: w <= 4
+    with pytest.raises(cc.CtaclustError) as e:                   # host-only plan cannot launch
+        cc._check(cc.lib().cc_launch(p.handle, 0, ctypes.byref(cc.CensusArgs(4, 4)), None, None, None))
+    assert e.value.status == -7
+
+
+def test_empty_grid_and_more_clusters_than_ctas():
+    p = cc.Plan(0, 5, "row", num_clusters=4, device=None)
+    perm, off = p.table()
+    assert p.V == 0 and list(off) == [0, 0, 0, 0, 0]
+    p = cc.Plan(2, 2, "col", num_clusters=9, device=None)      # reading R8: surplus clusters empty
+    perm, off = p.table()
+    assert list(off) == [0, 1, 2, 3, 4, 4, 4, 4, 4, 4]
+
+
+def test_kernel_grid():
+    assert cc.kernel_grid("matvec", cc.MatvecArgs(None, 1024, 1024, 1024, None, None)) == (32, 32)
+    assert cc.kernel_grid("bicg", cc.BicgArgs(None, 16384, 16384, 16384)) == (64, 512)
+    assert cc.kernel_grid("atax", cc.AtaxArgs(None, 1004, 1001, 1001)) == (4, 32)
+    assert cc.kernel_grid("jacobi5", cc.Jacobi5Args(None, None, 16384, 16384, 16384, 1)) == (512, 512)
+    assert cc.kernel_grid("conv2d", cc.Conv2dArgs(None, None, 8192, 8192, 8192, 3)) == (256, 256)
+    a = cc.SpmvArgs(1 << 24, 1 << 24, 1 << 28)
+    assert cc.kernel_grid("spmv", a) == (((1 << 24) + (1 << 28) + 4095) // 4096, 1)

@@ -1,0 +1,112 @@
+"""GPU: binding + agent runtime exactly-once coverage and bit-exact maps.
+
+For every backend, order, throttle level and (fake) topology the execution
+census must be exactly 1 for every logical CTA, and the slot -> CTA map the
+device decoded must equal the oracle's partition table bit for bit."""
+import numpy as np
+import pytest
+import torch
+
+from oracle import plan as OP
+from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc, ops
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def nsm():
+    return cc.device_info(0)["num_sms"]
+
+
+def test_device_facts_and_rank_table(nsm):
+    info = cc.device_info(0)
+    assert info["num_sms"] == torch.cuda.get_device_properties(0).multi_processor_count
+    ranks = cc.sm_rank_table(0)
+    seen = ranks[ranks >= 0]
+    assert sorted(seen.tolist()) == list(range(len(seen)))      # dense
+    assert len(seen) == nsm                                      # the probe saw every SM
+
+
+GRIDS = [(1, 1), (37, 23), (32, 32), (64, 512), (3 * 148 + 5, 1)]
+
+
+@pytest.mark.parametrize("gx,gy", GRIDS)
+@pytest.mark.parametrize("order,tile", [("row", (1, 1)), ("col", (1, 1)), ("tile", (8, 8)), ("tile", (3, 5))])
+def test_agent_census_and_map(gx, gy, order, tile, nsm):
+    cen, sm, mp, p = ops.census(gx, gy, "agent", order, tile)
+    torch.cuda.synchronize()
+    assert torch.all(cen == 1), "exactly-once violated"
+    ref = OP.plan(gx, gy, cc.ORDERS[order], nsm, *tile)
+    assert np.array_equal(mp.cpu().numpy(), ref["perm"])
+    assert torch.all(sm >= 0)
+
+
+@pytest.mark.parametrize("backend", ["default", "identity", "redirect"])
+@pytest.mark.parametrize("gx,gy", GRIDS)
+def test_other_backends_census(backend, gx, gy, nsm):
+    cen, sm, mp, p = ops.census(gx, gy, backend, "row")
+    torch.cuda.synchronize()
+    assert torch.all(cen == 1)
+    if backend == "identity":
+        assert np.array_equal(mp.cpu().numpy(), np.arange(gx * gy))
+    if backend == "redirect":   # Listing 4: slot v ran CTA perm[v]
+        ref = OP.plan(gx, gy, OP.ROW, nsm)
+        assert np.array_equal(mp.cpu().numpy(), ref["perm"])
+        red = np.array([OP.rd_redirect(gx * gy, nsm, u) for u in range(gx * gy)])
+        assert sorted(red.tolist()) == list(range(gx * gy))
+
+
+@pytest.mark.parametrize("active", [1, 2, 0])
+@pytest.mark.parametrize("M", [7, 148, 300, 5000])
+def test_throttling_and_fake_topologies(active, M):
+    """Fewer/more clusters than SMs, throttled agents: coverage still exactly once
+    (clusters with no home agent are stolen)."""
+    gx, gy = 128, 64
+    cen, sm, mp, p = ops.census(gx, gy, "agent", "tile", (4, 4), num_clusters=M, active_agents=active)
+    torch.cuda.synchronize()
+    assert torch.all(cen == 1)
+    ref = OP.plan(gx, gy, OP.TILE, M, 4, 4)
+    assert np.array_equal(mp.cpu().numpy(), ref["perm"])
+
+
+def test_forced_starvation_single_agent():
+    cen, *_ = ops.census(512, 16, "agent", "row", max_agents=1, active_agents=1)
+    torch.cuda.synchronize()
+    assert torch.all(cen == 1)
+
+
+def test_home_fraction_without_stealing(nsm):
+    """steal = 0 is the paper's scheme (static binding): with every SM holding
+    agents the census is still complete, and every CTA runs on its home SM."""
+    gx, gy = 64, 64
+    cen, sm, mp, p = ops.census(gx, gy, "agent", "row", steal=0)
+    torch.cuda.synchronize()
+    c = cen.cpu().numpy()
+    assert c.max() <= 1
+    if c.min() == 1:
+        ranks = cc.sm_rank_table(0)
+        perm, off = p.table()
+        home = np.empty(gx * gy, dtype=np.int64)
+        for i in range(p.M):
+            home[perm[off[i]:off[i + 1]]] = i
+        ran = ranks[sm.cpu().numpy()]
+        assert np.all(ran == home)
+
+
+def test_repeated_launches_reset_workspace():
+    args = cc.CensusArgs(200, 100)
+    p = ops.plan_for("census", args, "col")
+    cen = torch.zeros(20000, dtype=torch.int32, device="cuda")
+    for _ in range(25):
+        cc.launch(p, "census", args, cc.make_opts("agent", census=cen, active_agents=3))
+    torch.cuda.synchronize()
+    assert torch.all(cen == 25)
+
+
+def test_user_order():
+    rng = np.random.default_rng(3)
+    u = rng.permutation(50 * 30).astype(np.int32)
+    cen, sm, mp, p = ops.census(50, 30, "agent", user_order=u)
+    torch.cuda.synchronize()
+    assert torch.all(cen == 1)
+    assert np.array_equal(mp.cpu().numpy(), u)
