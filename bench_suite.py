@@ -1,0 +1,217 @@
+#!/usr/bin/env python
+"""bench_suite.py -- every BASELINE config, clustered vs default CTA order.
+
+For each reuse kernel this times the default hardware order ("BSL"),
+the agent runtime with the config's clustering ("CLU"), throttled agents
+("CLU+TOT"), the prefetch variant, the persistence-only control (identity
+order) and redirection ("RD"), and reports ms, algorithmic GB/s (fraction of
+the measured HBM copy peak) and speedup over default.  L2-sector reductions
+come from the ncu captures (scripts/ncu_suite.sh -> profiles/).
+
+    python bench_suite.py out.json [--only matvec,atax,jacobi,conv,spmv] [--quick]
+"""
+from __future__ import annotations
+
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+
+def _peak():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
+    except Exception:
+        return 6650.0
+
+
+def time_ms(fn, reps, warm=3, inner=1):
+    import torch
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    out = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        for _ in range(inner):
+            fn()
+        b.record()
+        b.synchronize()
+        out.append(a.elapsed_time(b) / inner)
+    out.sort()
+    return out[len(out) // 2]
+
+
+def _row(name, ms, nbytes, base_ms, extra=None):
+    gbs = nbytes / (ms * 1e-3) / 1e9
+    d = {"variant": name, "ms": round(ms, 5), "GBps": round(gbs, 1), "frac_hbm": round(gbs / _peak(), 4),
+         "speedup_vs_default": round(base_ms / ms, 4) if base_ms else 1.0}
+    if extra:
+        d.update(extra)
+    return d
+
+
+def suite_matvec(quick):
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    n = 1024
+    A = synth.matrix(1, n, n, backend="torch", device="cuda")
+    x = synth.uniform(2, n, backend="torch", device="cuda")
+    y = torch.zeros(n, device="cuda")
+    nbytes = 4 * n * n + 8 * n
+    variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
+                ("agent-col", dict(backend="agent", order="col")),
+                ("agent-row-tot1", dict(backend="agent", order="row", active_agents=1)),
+                ("agent-row-tot2", dict(backend="agent", order="row", active_agents=2)),
+                ("identity", dict(backend="identity")), ("redirect-row", dict(backend="redirect", order="row"))]
+    rows, base = [], None
+    for name, kw in variants:
+        ms = time_ms(lambda: ops.matvec(A, x, y, **kw), 20 if quick else 50, inner=50)
+        base = ms if base is None else base
+        rows.append(_row(name, ms, nbytes, base))
+    return {"config": "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident", "bytes": nbytes, "rows": rows}
+
+
+def suite_atax(quick):
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    n = 16384
+    A = synth.matrix(3, n, n, backend="torch", device="cuda")
+    v = lambda s: synth.uniform(s, n, backend="torch", device="cuda")
+    x, p, r, y1, y2, x1, x2 = v(10), v(11), v(12), v(15), v(16), v(13), v(14)
+    tmp, y, q, s = (torch.empty(n, device="cuda") for _ in range(4))
+    Ab = 4 * n * n
+    kernels = {
+        "atax": (lambda kw: ops.atax(A, x, out=(tmp, y), **kw), 2 * Ab + 16 * n),
+        "bicg": (lambda kw: ops.bicg(A, p, r, out=(q, s), **kw), Ab + 16 * n),
+        "mvt": (lambda kw: ops.mvt(A, y1, y2, x1, x2, **kw), Ab + 24 * n),
+    }
+    variants = [("default", dict(backend="default")), ("agent-col", dict(backend="agent", order="col")),
+                ("agent-row", dict(backend="agent", order="row")),
+                ("agent-col-tot1", dict(backend="agent", order="col", active_agents=1)),
+                ("agent-col-tot2", dict(backend="agent", order="col", active_agents=2)),
+                ("agent-col-prefetch", dict(backend="agent", order="col", prefetch=1)),
+                ("identity", dict(backend="identity")), ("redirect-col", dict(backend="redirect", order="col"))]
+    out = {}
+    for kname, (fn, nbytes) in kernels.items():
+        rows, base = [], None
+        for name, kw in variants:
+            ms = time_ms(lambda: fn(kw), 5 if quick else 15)
+            base = ms if base is None else base
+            rows.append(_row(name, ms, nbytes, base))
+        out[kname] = {"bytes": nbytes, "rows": rows}
+    return {"config": "PolyBench ATAX/BICG/MVT fp32 n=16384, 32x256 tiles (64x512 grid)", "kernels": out}
+
+
+def suite_jacobi(quick):
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    N, T = 16384, (20 if quick else 100)
+    a = synth.matrix(4, N, N, backend="torch", device="cuda")
+    b = torch.empty_like(a)
+    nbytes = 8 * N * N * T
+    variants = [("default", dict(backend="default")), ("agent-tile8x8", dict(backend="agent", order="tile", tile=(8, 8))),
+                ("agent-tile4x4", dict(backend="agent", order="tile", tile=(4, 4))),
+                ("agent-tile16x16", dict(backend="agent", order="tile", tile=(16, 16))),
+                ("agent-col", dict(backend="agent", order="col")), ("agent-row", dict(backend="agent", order="row")),
+                ("agent-tile8x8-tot4", dict(backend="agent", order="tile", tile=(8, 8), active_agents=4)),
+                ("identity", dict(backend="identity"))]
+    rows, base = [], None
+    for name, kw in variants:
+        ms = time_ms(lambda: ops.jacobi5(a, b, T, **kw), 3, warm=1)
+        base = ms if base is None else base
+        rows.append(_row(name, ms, nbytes, base, {"ms_per_sweep": round(ms / T, 5)}))
+    return {"config": f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)", "bytes": nbytes, "rows": rows}
+
+
+def suite_conv(quick):
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    N = 8192
+    img = synth.matrix(5, N, N, backend="torch", device="cuda")
+    out = torch.empty_like(img)
+    res = {}
+    for R in (1, 3):
+        w = synth.uniform(6, (2 * R + 1) ** 2).reshape(2 * R + 1, 2 * R + 1)
+        w = w / w.sum()
+        nbytes = 8 * N * N
+        flops = 2 * (2 * R + 1) ** 2 * (N - 2 * R) ** 2
+        variants = [("default", dict(backend="default")),
+                    ("agent-tile8x8", dict(backend="agent", order="tile", tile=(8, 8))),
+                    ("agent-col", dict(backend="agent", order="col")),
+                    ("tbcluster-2", dict(backend="tbcluster", cluster_size=2)),
+                    ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
+                    ("tbcluster-8", dict(backend="tbcluster", cluster_size=8)),
+                    ("identity", dict(backend="identity"))]
+        rows, base = [], None
+        for name, kw in variants:
+            ms = time_ms(lambda: ops.conv2d(img, w, out=out, **kw), 5 if quick else 20)
+            base = ms if base is None else base
+            rows.append(_row(name, ms, nbytes, base, {"TFLOPs": round(flops / (ms * 1e-3) / 1e12, 2)}))
+        res[f"{2 * R + 1}x{2 * R + 1}"] = {"bytes": nbytes, "flops": flops, "rows": rows}
+    return {"config": f"2D conv fp32 {N}x{N}, 32x32 tiles (256x256 grid)", "filters": res}
+
+
+def suite_spmv(quick):
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    scale = 20 if quick else 24
+    t0 = time.time()
+    rp, col = synth.rmat_csr(7, scale, 16, backend="torch", device="cuda")
+    gen_s = time.time() - t0
+    rows_n = rp.numel() - 1
+    nnz = col.numel()
+    val = synth.uniform(8, nnz, backend="torch", device="cuda")
+    x = synth.uniform(9, rows_n, backend="torch", device="cuda")
+    Am = ops.SpmvMatrix(rp, col, val)
+    y = torch.empty(rows_n, device="cuda")
+    nbytes = 8 * nnz + 4 * (rows_n + 1) + 8 * rows_n
+    variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
+                ("agent-row-tot1", dict(backend="agent", order="row", active_agents=1)),
+                ("agent-row-tot2", dict(backend="agent", order="row", active_agents=2)),
+                ("agent-row-tot4", dict(backend="agent", order="row", active_agents=4)),
+                ("agent-row-prefetch", dict(backend="agent", order="row", prefetch=1)),
+                ("identity", dict(backend="identity"))]
+    rows, base = [], None
+    for name, kw in variants:
+        ms = time_ms(lambda: ops.spmv(Am, x, y, **kw), 5 if quick else 20)
+        base = ms if base is None else base
+        rows.append(_row(name, ms, nbytes, base))
+    return {"config": f"CSR SpMV fp32 R-MAT scale {scale} ef 16: {rows_n} rows, {nnz} nnz (gen {gen_s:.1f}s)",
+            "bytes": nbytes, "rows": rows}
+
+
+SUITES = {"matvec": suite_matvec, "atax": suite_atax, "jacobi": suite_jacobi, "conv": suite_conv, "spmv": suite_spmv}
+
+
+def run(path, only=None, quick=False):
+    import torch
+    res = {"device": torch.cuda.get_device_name(0), "hbm_peak_GBps": _peak()}
+    for k, fn in SUITES.items():
+        if only and k not in only:
+            continue
+        t0 = time.time()
+        try:
+            res[k] = fn(quick)
+        except Exception as e:  # keep the other configs
+            res[k] = {"error": repr(e)}
+        res[k]["wall_s"] = round(time.time() - t0, 1)
+        torch.cuda.empty_cache()
+        json.dump(res, open(path, "w"), indent=1)
+    return res
+
+
+if __name__ == "__main__":
+    import argparse
+    ap = argparse.ArgumentParser()
+    ap.add_argument("out")
+    ap.add_argument("--only", default=None)
+    ap.add_argument("--quick", action="store_true")
+    a = ap.parse_args()
+    run(a.out, a.only.split(",") if a.only else None, a.quick)
+    print(open(a.out).read())
