@@ -187,7 +187,7 @@ def main():
     torch.cuda.synchronize()
 
     def run_step(backend, order, ev=None, count=None):
-        kw = dict(backend=backend, order=order, active_agents=a.active_agents, prefetch=a.prefetch)
+        kw = dict(backend=backend, active_agents=a.active_agents, prefetch=a.prefetch)
         nl = 0
         if ev is not None: ev[0].record(stream)
         pl = ops.plan_for("atax", cc.atax_args(A, x, tmp, y), order)
