@@ -1,0 +1,84 @@
+#!/usr/bin/env python
+"""Launch one kernel variant a few times for ncu (each launch is tagged with an
+NVTX-free marker: the variant runs `--reps` launches after `--warm` warm-ups).
+
+    python scripts/ncu_target.py --kernel bicg --backend agent --order col [--reps 2]
+Kernels: matvec atax bicg mvt jacobi conv3 conv7 spmv.  Sizes are the BASELINE
+configs (jacobi: one sweep of 16384^2).
+"""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--kernel", required=True)
+    ap.add_argument("--backend", default="agent")
+    ap.add_argument("--order", default=None)
+    ap.add_argument("--tile", default=None)
+    ap.add_argument("--active", type=int, default=0)
+    ap.add_argument("--prefetch", type=int, default=0)
+    ap.add_argument("--cluster", type=int, default=2)
+    ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--warm", type=int, default=1)
+    ap.add_argument("--scale", type=int, default=24)
+    a = ap.parse_args()
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    kw = dict(backend=a.backend, active_agents=a.active, prefetch=a.prefetch)
+    if a.order:
+        kw["order"] = a.order
+    if a.tile:
+        kw["tile"] = tuple(int(t) for t in a.tile.split("x"))
+    if a.backend == "tbcluster":
+        kw["cluster_size"] = a.cluster
+    dev = "cuda"
+    k = a.kernel
+    if k == "matvec":
+        n = 1024
+        A = synth.matrix(1, n, n, backend="torch", device=dev)
+        x = synth.uniform(2, n, backend="torch", device=dev)
+        y = torch.zeros(n, device=dev)
+        fn = lambda: ops.matvec(A, x, y, **kw)
+    elif k in ("atax", "bicg", "mvt"):
+        n = 16384
+        A = synth.matrix(3, n, n, backend="torch", device=dev)
+        v = lambda s: synth.uniform(s, n, backend="torch", device=dev)
+        x, p, r, y1, y2, x1, x2 = v(10), v(11), v(12), v(15), v(16), v(13), v(14)
+        bufs = (torch.empty(n, device=dev), torch.empty(n, device=dev))
+        fn = {"atax": lambda: ops.atax(A, x, out=bufs, **kw),
+              "bicg": lambda: ops.bicg(A, p, r, out=bufs, **kw),
+              "mvt": lambda: ops.mvt(A, y1, y2, x1, x2, **kw)}[k]
+    elif k == "jacobi":
+        N = 16384
+        a_ = synth.matrix(4, N, N, backend="torch", device=dev)
+        b_ = torch.empty_like(a_)
+        fn = lambda: ops.jacobi5(a_, b_, 1, **kw)
+    elif k in ("conv3", "conv7"):
+        N, R = 8192, (1 if k == "conv3" else 3)
+        img = synth.matrix(5, N, N, backend="torch", device=dev)
+        out = torch.empty_like(img)
+        w = synth.uniform(6, (2 * R + 1) ** 2).reshape(2 * R + 1, 2 * R + 1)
+        w = w / w.sum()
+        fn = lambda: ops.conv2d(img, w, out=out, **kw)
+    elif k == "spmv":
+        rp, col = synth.rmat_csr(7, a.scale, 16, backend="torch", device=dev)
+        val = synth.uniform(8, col.numel(), backend="torch", device=dev)
+        x = synth.uniform(9, rp.numel() - 1, backend="torch", device=dev)
+        Am = ops.SpmvMatrix(rp, col, val)
+        y = torch.empty(rp.numel() - 1, device=dev)
+        fn = lambda: ops.spmv(Am, x, y, **kw)
+    else:
+        raise SystemExit(f"unknown kernel {k}")
+    torch.cuda.synchronize()
+    for _ in range(a.warm + a.reps):
+        fn()
+    torch.cuda.synchronize()
+
+
+if __name__ == "__main__":
+    main()
