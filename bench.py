@@ -42,7 +42,8 @@ def parse():
     ap.add_argument("--backend", default="agent")
     ap.add_argument("--order", default="col")
     ap.add_argument("--active-agents", type=int, default=0)
-    ap.add_argument("--prefetch", type=int, default=0)
+    ap.add_argument("--stages", type=int, default=0)
+    ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--suite", default=None, help="also run every BASELINE config, write JSON here")
@@ -187,7 +188,7 @@ def main():
     torch.cuda.synchronize()
 
     def run_step(backend, order, ev=None, count=None):
-        kw = dict(backend=backend, active_agents=a.active_agents, prefetch=a.prefetch)
+        kw = dict(backend=backend, active_agents=a.active_agents, stages=a.stages, batch=a.batch)
         nl = 0
         if ev is not None: ev[0].record(stream)
         pl = ops.plan_for("atax", cc.atax_args(A, x, tmp, y), order)
@@ -300,7 +301,7 @@ def main():
                 "data": "synthetic (counter-hash U[0,1), generated on device)",
                 "config": {"workload": f"ATAX+BICG+MVT fp32 n={n} (BASELINE config 2)",
                            "backend": a.backend, "order": a.order, "active_agents": a.active_agents or "max",
-                           "prefetch": a.prefetch, "tile": "32x256", "parallelism": f"row-shard x{world}",
+                           "stages": a.stages or "default", "batch": a.batch or "default", "tile": "32x256", "parallelism": f"row-shard x{world}",
                            "l2": "inputs (1 GiB) larger than L2 (126 MB); no flush"},
                 "speedup_vs_default": round(ms_def / ms_clu, 4),
                 "ms_per_step_default": round(ms_def, 4),

@@ -3,7 +3,7 @@
 
 For each reuse kernel this times the default hardware order ("BSL"),
 the agent runtime with the config's clustering ("CLU"), throttled agents
-("CLU+TOT"), the prefetch variant, the persistence-only control (identity
+("CLU+TOT"), the staging-depth variants, the persistence-only control (identity
 order) and redirection ("RD"), and reports ms, algorithmic GB/s (fraction of
 the measured HBM copy peak) and speedup over default.  L2-sector reductions
 come from the ncu captures (scripts/ncu_suite.sh -> profiles/).
@@ -94,7 +94,8 @@ def suite_atax(quick):
                 ("agent-row", dict(backend="agent", order="row")),
                 ("agent-col-tot1", dict(backend="agent", order="col", active_agents=1)),
                 ("agent-col-tot2", dict(backend="agent", order="col", active_agents=2)),
-                ("agent-col-prefetch", dict(backend="agent", order="col", prefetch=1)),
+                ("agent-col-s2", dict(backend="agent", order="col", stages=2)),
+                ("agent-col-s6", dict(backend="agent", order="col", stages=6)),
                 ("identity", dict(backend="identity")), ("redirect-col", dict(backend="redirect", order="col"))]
     out = {}
     for kname, (fn, nbytes) in kernels.items():
@@ -175,7 +176,7 @@ def suite_spmv(quick):
                 ("agent-row-tot1", dict(backend="agent", order="row", active_agents=1)),
                 ("agent-row-tot2", dict(backend="agent", order="row", active_agents=2)),
                 ("agent-row-tot4", dict(backend="agent", order="row", active_agents=4)),
-                ("agent-row-prefetch", dict(backend="agent", order="row", prefetch=1)),
+                ("agent-row-s4b8", dict(backend="agent", order="row", stages=4, batch=8)),
                 ("identity", dict(backend="identity"))]
     rows, base = [], None
     for name, kw in variants:

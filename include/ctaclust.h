@@ -127,8 +127,11 @@ typedef struct {
                                0 => max_agents                                          */
     int32_t max_agents;     /* agents launched per SM (MAX_AGENTS, Fig. 10); 0 => the
                                occupancy limit of the kernel                            */
-    int32_t prefetch;       /* 1 => prefetch the next task's tile into L2 while the
-                               current one runs (§4.3(III), Listing 5 l.34-37)          */
+    int32_t stages;         /* agent backends: depth of the per-agent shared-memory ring
+                               the scheduler warp stages upcoming tasks into -- the
+                               B200 form of "prefetch the next CTA" (§4.3(III),
+                               Listing 5 l.34-37); 0 => the kernel's default, 1..8   */
+    int32_t batch;          /* logical CTAs claimed per queue atomic; 0 => default   */
     int32_t steal;          /* 1 (default) => an agent whose cluster queue is empty
                                takes work from other clusters, so every CTA runs exactly
                                once whatever the hardware does with agent placement
@@ -143,7 +146,7 @@ typedef struct {
 } cc_launch_opts;
 
 /* Fill *opts with defaults: AGENT backend, max/active from occupancy, steal = 1,
- * prefetch = 0, cluster_size = 2, no census/map. */
+ * stages/batch per kernel, cluster_size = 2, no census/map. */
 cc_status cc_launch_opts_default(cc_launch_opts* opts);
 
 typedef enum {

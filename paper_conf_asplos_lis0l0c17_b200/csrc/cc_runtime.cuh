@@ -1,20 +1,32 @@
 // cc_runtime.cuh -- the agent runtime (binding + task loop) for sm_100a.
 //
 // PAPER.md §4.2.3 Step 3 "Binding", §4.2.4(2) agent-based
-// clustering (Fig. 8(D), Listing 5) and §4.3(I) CTA throttling
-// (P:2183).  B200-first differences from Listing 5:
+// clustering (Fig. 8(D), Listing 5), §4.3(I) CTA throttling
+// and §4.3(III) prefetching.
+//
+// An agent is a persistent, warp-specialised CTA:
+//   warp 0        scheduler/producer: binds the agent to its SM's cluster,
+//                 pops logical-CTA slots ahead of use and stages each task's
+//                 input tile into a ring of `stages` shared-memory buffers
+//                 (bulk async copies / cp.async, completion on an mbarrier);
+//   warps 1..8    consumers: run the original kernel body on each staged
+//                 task in order, then release the buffer (empty mbarrier).
+// The ring is the B200 form of Listing 5's "prefetch the next CTA" -- the
+// next tasks' data is in flight while the current one computes -- and it makes
+// the bytes in flight independent of how many agents are active, so
+// throttling (active_agents) no longer starves the memory system.
+//
+// B200-first differences from Listing 5:
 //   * cluster i binds to the SM of dense rank i from a probe-built table, not to
 //     raw %smid (virtual, possibly sparse; reading R7);
-//   * agents pop slots from a per-cluster queue with relaxed atomics instead of
-//     a static stride v += ACTIVE_AGENTS, and steal from other clusters when
-//     their own is empty, so coverage is exactly-once even if the hardware
-//     places fewer agents on an SM than expected (reading R10);
-//   * the pop for the next task is issued before the current body runs and only
-//     consumed after it, hiding the L2 atomic round trip;
-//   * no gpu-scope fence or acquire anywhere in the loop: on sm_100a those emit
-//     CCTL.IVALL, which would wipe the very L1 contents clustering tries to keep;
-//   * the workspace resets itself: the last agent to leave zeroes the counters,
-//     so a launch is one kernel (no memset node).
+//   * slots are popped in batches from a per-cluster queue with relaxed atomics
+//     (the next batch's atomic is issued as soon as the current batch starts),
+//     instead of a static stride v += ACTIVE_AGENTS; an agent whose queue is
+//     empty steals, scanning all queues warp-parallel, so every logical CTA runs
+//     exactly once whatever the hardware does with agent placement (R9/R10);
+//   * no gpu-scope fence or acquire anywhere: on sm_100a those emit CCTL.IVALL,
+//     which would wipe the very L1 contents clustering tries to keep;
+//   * the workspace resets itself (last agent out), so a launch is one kernel.
 #pragma once
 #include <stdint.h>
 #include <cuda_runtime.h>
@@ -23,6 +35,8 @@
 namespace cc {
 
 enum : int32_t { MODE_AGENT = 0, MODE_IDENTITY = 1 };
+constexpr int MAX_STAGES = 8;
+constexpr int PRODUCER_THREADS = 32;
 
 // Everything a task loop needs, passed by value as a kernel parameter.
 struct Sched {
@@ -34,7 +48,9 @@ struct Sched {
     int32_t mode;                 // MODE_AGENT / MODE_IDENTITY
     int32_t active_agents;
     int32_t steal;
-    int32_t prefetch;
+    int32_t stages;               // ring depth (agent backends; 1 for one-shot CTAs)
+    int32_t batch;                // slots claimed per queue atomic
+    uint32_t stage_bytes;         // bytes per ring buffer (128-byte multiple)
     uint32_t* census;             // optional outputs (see ctaclust.h)
     int32_t* exec_sm;
     int32_t* map;
@@ -46,6 +62,9 @@ __device__ __forceinline__ int32_t* ws_gq(const Sched& s) { return s.ws + 2 * s.
 __device__ __forceinline__ int32_t* ws_done(const Sched& s) { return s.ws + 2 * s.g.M + 2; }
 inline size_t ws_ints(int32_t M) { return (size_t)(2 * M + 3); }
 
+// ---------------------------------------------------------------------------
+// PTX helpers
+// ---------------------------------------------------------------------------
 __device__ __forceinline__ uint32_t smid() {
     uint32_t r;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(r));
@@ -56,7 +75,6 @@ __device__ __forceinline__ uint32_t nsmid() {
     asm volatile("mov.u32 %0, %%nsmid;" : "=r"(r));
     return r;
 }
-// relaxed gpu-scope load (no fence, no L1 invalidation)
 __device__ __forceinline__ int32_t ld_relaxed(const int32_t* p) {
     int32_t v;
     asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -66,6 +84,58 @@ __device__ __forceinline__ int32_t atom_add_relaxed(int32_t* p, int32_t v) {
     int32_t old;
     asm volatile("atom.relaxed.gpu.global.add.s32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
     return old;
+}
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra WAIT_%=;\n}" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+// 1D bulk async copy global -> shared, completion counted on `bar` (UBLKCP).
+// dst, src 16-byte aligned, bytes a multiple of 16.
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+// 16-byte cp.async that also allocates the line in L1 (.ca): the staged data
+// doubles as L1-resident data for neighbouring tasks on the same SM.
+// src_bytes < 16 zero-fills the rest (0 => pure zero fill, no read).
+__device__ __forceinline__ void cp_async_ca16(void* dst, const void* src, uint32_t src_bytes) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(src_bytes) : "memory");
+}
+// this thread's prior cp.async ops complete -> one (pre-counted) arrival on bar
+__device__ __forceinline__ void cp_async_arrive(uint64_t* bar) {
+    asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
+// named barrier among the consumer warps only (the producer warp never joins)
+template <int N>
+__device__ __forceinline__ void consumer_sync() {
+    asm volatile("bar.sync 1, %0;" :: "n"(N) : "memory");
+}
+
+// Stage protocol for Body::produce (warp 0, all lanes): the full barrier has
+// an arrival count of 1.  Lanes may first issue cp.async + cp_async_arrive
+// (each pre-counts itself), then call stage_commit(), which makes lane 0's
+// single arrival carrying the byte count of the bulk copies issued after it.
+__device__ __forceinline__ void stage_commit(uint64_t* full, int lane, uint32_t bulk_bytes) {
+    __syncwarp();
+    if (lane == 0) mbar_arrive_tx(full, bulk_bytes);
+    __syncwarp();
 }
 
 __device__ __forceinline__ void lin_to_bxby(const Sched& s, int32_t v, int32_t* lin, int32_t* bx, int32_t* by) {
@@ -80,156 +150,237 @@ __device__ __forceinline__ void lin_to_bxby(const Sched& s, int32_t v, int32_t* 
     }
 }
 
-// Queue cursor of one agent (thread 0 only).
-struct Cursor {
-    int32_t q;        // cluster queue being drained, -1 = finished
-    int32_t home;     // first queue scanned
-    int32_t scanned;  // queues visited so far
-};
-
-// Next order position for this agent or -1.  Own cluster first, then (steal)
-// the other clusters round-robin from home.
-__device__ __forceinline__ int32_t next_position(const Sched& s, Cursor& c) {
-    if (s.mode == MODE_IDENTITY) {
-        if (c.q < 0) return -1;
-        int32_t v = atom_add_relaxed(ws_gq(s), 1);
-        if (v < s.g.V) return v;
-        c.q = -1;
-        return -1;
-    }
-    int32_t* head = ws_head(s);
-    while (c.q >= 0) {
-        int32_t size = cluster_size(s.g, c.q);
-        if (ld_relaxed(head + c.q) < size) {
-            int32_t w = atom_add_relaxed(head + c.q, 1);
-            if (w < size) return cluster_start(s.g, c.q) + w;
-        }
-        if (!s.steal || ++c.scanned >= s.g.M) { c.q = -1; break; }
-        c.q = c.home + c.scanned;
-        if (c.q >= s.g.M) c.q -= s.g.M;
-    }
-    return -1;
-}
-
 __device__ __forceinline__ void record(const Sched& s, int32_t v, int32_t lin) {
     if (s.census) atomicAdd(s.census + lin, 1u);
     if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();
     if (s.map) s.map[v] = lin;
 }
 
-// Body concept (all methods called by every thread, with CTA-uniform args):
-//   run(bx, by)            one logical CTA of the original kernel
-//   prefetch_l2(bx, by)    thread 0 only: warm L2 with the next task's tile
-//   finish()               agent is retiring: flush carried state
+// ---------------------------------------------------------------------------
+// Scheduler (producer warp).  Lane 0 owns the queue state; the whole warp
+// helps with the steal scan.
+// ---------------------------------------------------------------------------
+struct Prod {
+    int32_t q;        // queue being drained (-1: none left)
+    int32_t home;     // first queue, and where the steal scan starts
+    int32_t bq, bw, be;   // current batch: slots [bw, be) of queue bq
+    int32_t sq, sw;   // speculative claim in flight: raw fetch-add result on queue sq
+    int32_t spec;
+};
+
+__device__ __forceinline__ int32_t q_size(const Sched& s, int32_t q) {
+    return s.mode == MODE_IDENTITY ? s.g.V : cluster_size(s.g, q);
+}
+__device__ __forceinline__ int32_t q_start(const Sched& s, int32_t q) {
+    return s.mode == MODE_IDENTITY ? 0 : cluster_start(s.g, q);
+}
+__device__ __forceinline__ int32_t* q_head(const Sched& s, int32_t q) {
+    return s.mode == MODE_IDENTITY ? ws_gq(s) : ws_head(s) + q;
+}
+
+// lane 0 only.  Returns an order position, or -1 with *scan = 1 when the queue
+// being drained is empty and a steal scan should follow, or -1 with *scan = 0
+// when this agent is done.
+__device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* scan) {
+    *scan = 0;
+    if (P.bw < P.be) return q_start(s, P.bq) + P.bw++;
+    for (;;) {
+        int32_t sq, w;
+        if (P.spec) { sq = P.sq; w = P.sw; P.spec = 0; }
+        else if (P.q >= 0) { sq = P.q; w = atom_add_relaxed(q_head(s, sq), s.batch); }
+        else return -1;
+        const int32_t size = q_size(s, sq);
+        if (w < size) {
+            P.bq = sq; P.bw = w + 1; P.be = w + s.batch < size ? w + s.batch : size;
+            if (w + s.batch < size) {                  // claim the next batch early
+                P.sq = sq; P.sw = atom_add_relaxed(q_head(s, sq), s.batch); P.spec = 1;
+            }
+            return q_start(s, sq) + w;
+        }
+        if (sq == P.q) {
+            if (!s.steal || s.mode == MODE_IDENTITY) { P.q = -1; return -1; }
+            *scan = 1;
+            return -1;
+        }
+    }
+}
+
+// warp-parallel scan for a queue with unclaimed slots, nearest first from home.
+__device__ __forceinline__ int32_t steal_scan(const Sched& s, int32_t home, int lane) {
+    const int32_t M = s.g.M;
+    for (int32_t base = 0; base < M; base += 32) {
+        int32_t k = base + lane;
+        bool avail = false;
+        int32_t q = -1;
+        if (k < M) {
+            q = home + 1 + k;
+            q -= (q >= M) ? M : 0;
+            q -= (q >= M) ? M : 0;
+            avail = ld_relaxed(ws_head(s) + q) < cluster_size(s.g, q);
+        }
+        uint32_t m = __ballot_sync(0xffffffffu, avail);
+        if (m) return __shfl_sync(0xffffffffu, q, __ffs(m) - 1);
+    }
+    return -1;
+}
+
+__device__ __forceinline__ int32_t producer_next(const Sched& s, Prod& P, int lane) {
+    int32_t v = -1, scan = 0;
+    if (lane == 0) v = lane0_next(s, P, &scan);
+    scan = __shfl_sync(0xffffffffu, scan, 0);
+    while (scan) {
+        int32_t q = steal_scan(s, __shfl_sync(0xffffffffu, P.home, 0), lane);
+        if (lane == 0) {
+            if (q < 0) { P.q = -1; v = -1; scan = 0; }
+            else { P.q = q; P.spec = 0; v = lane0_next(s, P, &scan); }
+        }
+        scan = __shfl_sync(0xffffffffu, scan, 0);
+    }
+    return __shfl_sync(0xffffffffu, v, 0);
+}
+
+// ---------------------------------------------------------------------------
+// Body concept (see k_gemv.cuh / k_stencil.cuh / k_spmv.cuh):
+//   kConsumers, kStageBytes, kDefaultStages, kDefaultBatch
+//   produce(bx, by, stage, full, lane)  warp 0, all lanes: stage the task's
+//                                       input and commit (stage_commit)
+//   consume(bx, by, stage, ctid)        consumer threads ctid in [0, kConsumers)
+//   finish(ctid)                        consumers, agent retiring: flush state
+// ---------------------------------------------------------------------------
+struct RingShared {
+    uint64_t full[MAX_STAGES];
+    uint64_t empty[MAX_STAGES];
+    int32_t slot[MAX_STAGES];
+};
+
+__device__ __forceinline__ uint8_t* ring_base(uint8_t* dyn) {
+    const uint32_t a = smem_u32(dyn);
+    return dyn + (((a + 127u) & ~127u) - a);
+}
+
 template <class Body>
 __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
-    __shared__ int32_t s_agent;
-    __shared__ int32_t s_next[2];
-    Cursor cur_c;
+    extern __shared__ uint8_t dyn_smem[];
+    __shared__ RingShared R;
+    __shared__ int32_t s_active;
+    uint8_t* ring = ring_base(dyn_smem);
+    const int S = s.stages;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    constexpr int kConsumerWarps = Body::kConsumers / 32;
     if (threadIdx.x == 0) {
-        // binding: dense SM rank from %smid, agent id by arrival
-        uint32_t sm = smid();
-        int32_t rank = (int32_t)sm < s.smid_span ? s.rank_of_smid[sm] : -1;
-        int32_t arank = rank;                             // rank used for the agent id
-        if (rank >= s.g.M) rank = -1;                     // fewer clusters than SMs
-        int32_t a = atom_add_relaxed(ws_agent_ctr(s) + (arank < 0 || arank >= s.g.M ? s.g.M : arank), 1);
-        // agents with no cluster of their own only steal, from a spread-out start
-        cur_c.home = rank >= 0 ? rank : (int32_t)(blockIdx.x % (uint32_t)(s.g.M > 0 ? s.g.M : 1));
-        cur_c.scanned = 0;
-        cur_c.q = (s.g.V > 0 && s.g.M > 0) ? cur_c.home : -1;
-        // throttling (Listing 5 l.20): agents past active_agents retire at once
-        const bool active = (a < s.active_agents) && (rank >= 0 || s.steal || s.mode == MODE_IDENTITY);
-        if (!active) cur_c.q = -1;
-        s_agent = active ? 1 : 0;
-        s_next[0] = active ? next_position(s, cur_c) : -1;
+        for (int i = 0; i < S; ++i) { mbar_init(&R.full[i], 1); mbar_init(&R.empty[i], kConsumerWarps); }
+        fence_mbar_init();
     }
     __syncthreads();
-    int32_t v = s_next[0];
-    int32_t t = 0;
-    while (v >= 0) {
-        int32_t lin, bx, by;
-        lin_to_bxby(s, v, &lin, &bx, &by);
-        int32_t nxt = -1;
-        int32_t spec_q = -1, spec_w = 0;
-        if (threadIdx.x == 0) {
-            if (s.prefetch) {
-                nxt = next_position(s, cur_c);
-                if (nxt >= 0) {
-                    int32_t nl, nbx, nby;
-                    lin_to_bxby(s, nxt, &nl, &nbx, &nby);
-                    body.prefetch_l2(nbx, nby);
-                }
-            } else if (s.mode == MODE_AGENT && cur_c.q >= 0) {
-                // speculative pop: issue the atomic now, look at it after the body
-                spec_q = cur_c.q;
-                spec_w = atom_add_relaxed(ws_head(s) + spec_q, 1);
+    if (warp == 0) {
+        // ---- binding: dense SM rank from %smid, agent id by arrival
+        Prod P{};
+        int32_t active = 0;
+        if (lane == 0) {
+            uint32_t sm = smid();
+            int32_t rank = (int32_t)sm < s.smid_span ? s.rank_of_smid[sm] : -1;
+            int32_t slot = (rank < 0 || rank >= s.g.M) ? s.g.M : rank;
+            int32_t a = atom_add_relaxed(ws_agent_ctr(s) + slot, 1);
+            if (rank >= s.g.M) rank = -1;                       // fewer clusters than SMs
+            P.home = rank >= 0 ? rank : (int32_t)(blockIdx.x % (uint32_t)(s.g.M > 0 ? s.g.M : 1));
+            P.q = (s.g.V > 0 && s.g.M > 0) ? P.home : -1;
+            // throttling (Listing 5 l.20): agents past active_agents retire at once
+            active = (a < s.active_agents) && (rank >= 0 || s.steal || s.mode == MODE_IDENTITY);
+            if (!active) P.q = -1;
+            if (s.mode == MODE_IDENTITY && active) P.q = 0;
+            s_active = active;
+        }
+        // ---- producer ring
+        for (int32_t t = 0;; ++t) {
+            const int st = t % S;
+            if (t >= S) mbar_wait(&R.empty[st], ((t / S) - 1) & 1);
+            const int32_t v = producer_next(s, P, lane);
+            if (lane == 0) R.slot[st] = v;
+            if (v < 0) {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&R.full[st]);        // end marker
+                break;
+            }
+            int32_t lin, bx, by;
+            lin_to_bxby(s, v, &lin, &bx, &by);
+            body.produce(bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
+        }
+        // ---- the last agent out resets the workspace for the next launch.  Every
+        // other agent's producer has consumed the results of all its atomics
+        // (including any speculative claim) before arriving here.
+        if (lane == 0) {
+            const int32_t total = (int32_t)(gridDim.x * gridDim.y * gridDim.z);
+            if (atom_add_relaxed(ws_done(s), 1) == total - 1) {
+                const int32_t n = 2 * s.g.M + 2;
+                for (int32_t k = 0; k < n; ++k) s.ws[k] = 0;
+                *ws_done(s) = 0;
             }
         }
-        body.run(bx, by);
-        if (threadIdx.x == 0) {
-            record(s, v, lin);
-            if (!s.prefetch) {
-                if (spec_q >= 0 && spec_w < cluster_size(s.g, spec_q)) nxt = cluster_start(s.g, spec_q) + spec_w;
-                else {
-                    if (spec_q >= 0 && cur_c.q == spec_q) {   // own queue ran dry: move on
-                        if (!s.steal || ++cur_c.scanned >= s.g.M) cur_c.q = -1;
-                        else { cur_c.q = cur_c.home + cur_c.scanned; if (cur_c.q >= s.g.M) cur_c.q -= s.g.M; }
-                    }
-                    nxt = next_position(s, cur_c);
-                }
-            }
-            s_next[(t + 1) & 1] = nxt;
+    } else {
+        const int ctid = threadIdx.x - PRODUCER_THREADS;
+        for (int32_t t = 0;; ++t) {
+            const int st = t % S;
+            mbar_wait(&R.full[st], (t / S) & 1);
+            const int32_t v = R.slot[st];
+            if (v < 0) break;
+            int32_t lin, bx, by;
+            lin_to_bxby(s, v, &lin, &bx, &by);
+            body.consume(bx, by, ring + (size_t)st * s.stage_bytes, ctid);
+            if (ctid == 0) record(s, v, lin);
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&R.empty[st]);
         }
-        __syncthreads();
-        v = s_next[(t + 1) & 1];
-        ++t;
+        if (s_active) body.finish(ctid);
     }
-    if (s_agent) body.finish();
-    // the last agent out resets the workspace for the next launch.  Every other
-    // agent has consumed the results of all its atomics before arriving here,
-    // so no counter can still be in use.
-    if (threadIdx.x == 0) {
-        int32_t total = (int32_t)(gridDim.x * gridDim.y * gridDim.z);
-        if (atom_add_relaxed(ws_done(s), 1) == total - 1) {
-            int32_t n = 2 * s.g.M + 2;
-            for (int32_t k = 0; k < n; ++k) s.ws[k] = 0;
-            *ws_done(s) = 0;
+}
+
+// One-shot CTA (default hardware order, or redirection): the same producer /
+// consumer split with a single stage and a single task.
+template <class Body>
+__device__ __forceinline__ void one_shot(const Sched& s, Body& body, int32_t v, int32_t lin, int32_t bx, int32_t by) {
+    extern __shared__ uint8_t dyn_smem[];
+    __shared__ uint64_t full;
+    uint8_t* ring = ring_base(dyn_smem);
+    if (threadIdx.x == 0) { mbar_init(&full, 1); fence_mbar_init(); }
+    __syncthreads();
+    if (threadIdx.x < PRODUCER_THREADS) {
+        body.produce(bx, by, ring, &full, threadIdx.x);
+    } else {
+        const int ctid = threadIdx.x - PRODUCER_THREADS;
+        mbar_wait(&full, 0);
+        body.consume(bx, by, ring, ctid);
+        if (ctid == 0) {
+            if (s.census) atomicAdd(s.census + lin, 1u);
+            if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();
+            if (s.map && v >= 0) s.map[v] = lin;
         }
+        body.finish(ctid);
     }
 }
 
 // ---- kernels: one per (body, backend) ------------------------------------
 template <class Body>
-__global__ void __launch_bounds__(Body::kThreads) k_agent(Sched s, typename Body::Params p) {
+__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_agent(Sched s, typename Body::Params p) {
     Body body(p);
     agent_loop(s, body);
 }
 
 template <class Body>
-__global__ void __launch_bounds__(Body::kThreads) k_default(Sched s, typename Body::Params p) {
+__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_default(Sched s, typename Body::Params p) {
     Body body(p);
-    int32_t bx = blockIdx.x, by = blockIdx.y;
-    body.run(bx, by);
-    if (threadIdx.x == 0) {
-        int32_t lin = by * s.g.gx + bx;
-        if (s.census) atomicAdd(s.census + lin, 1u);
-        if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();
-    }
-    body.finish();
+    const int32_t bx = blockIdx.x, by = blockIdx.y;
+    one_shot(s, body, -1, by * s.g.gx + bx, bx, by);
 }
 
 // Redirection-based clustering (Listing 4, Fig. 9): same number of CTAs as O;
 // CTA u runs v = rd_redirect(u).
 template <class Body>
-__global__ void __launch_bounds__(Body::kThreads) k_redirect(Sched s, typename Body::Params p) {
+__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_redirect(Sched s, typename Body::Params p) {
     Body body(p);
-    int32_t u = blockIdx.x;
-    int32_t v = rd_redirect(s.g, u);
+    const int32_t v = rd_redirect(s.g, (int32_t)blockIdx.x);
     int32_t lin, bx, by;
     lin_to_bxby(s, v, &lin, &bx, &by);
-    body.run(bx, by);
-    if (threadIdx.x == 0) record(s, v, lin);
-    body.finish();
+    one_shot(s, body, v, lin, bx, by);
 }
 
 }  // namespace cc

@@ -261,6 +261,8 @@ extern "C" cc_status cc_launch_opts_default(cc_launch_opts* o) {
     o->backend = CC_BACKEND_AGENT;
     o->steal = 1;
     o->cluster_size = 2;
+    o->stages = 0;
+    o->batch = 0;
     return CC_OK;
 }
 
@@ -290,13 +292,16 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
 }
 
 struct CensusParams { int32_t dummy; };
-struct CensusBody {
-    static constexpr int kThreads = 128;
+struct CensusBody {   // empty body: binding, queues and census only
+    static constexpr int kConsumers = 32;
+    static constexpr int kStageBytes = 128;
+    static constexpr int kDefaultStages = 2;
+    static constexpr int kDefaultBatch = 1;
     using Params = CensusParams;
     __device__ __forceinline__ explicit CensusBody(const CensusParams&) {}
-    __device__ __forceinline__ void run(int32_t, int32_t) {}
-    __device__ __forceinline__ void prefetch_l2(int32_t, int32_t) {}
-    __device__ __forceinline__ void finish() {}
+    __device__ __forceinline__ void produce(int32_t, int32_t, uint8_t*, uint64_t* full, int lane) { stage_commit(full, lane, 0); }
+    __device__ __forceinline__ void consume(int32_t, int32_t, const uint8_t*, int) {}
+    __device__ __forceinline__ void finish(int) {}
 };
 
 using MatvecB = GemvBody<32, 32, true, false>;
@@ -305,20 +310,45 @@ using ColB = GemvBody<32, 256, false, true>;
 using BothB = GemvBody<32, 256, true, true>;
 
 template <class Body>
-static cc_status occupancy(int device, int* occ) {
+static size_t dyn_smem(int stages) { return (size_t)stages * Body::kStageBytes + 128; }
+
+// Opt every instantiation of a body into large dynamic shared memory once.
+template <class Body>
+static cc_status prepare_body(int device) {
     static std::mutex mu;
-    static int cache[64] = {0};
+    static bool done[64] = {false};
     std::lock_guard<std::mutex> lk(mu);
     if (device < 0 || device >= 64) return fail(CC_ERR_INVALID_ARG, "device");
-    if (!cache[device]) {
+    if (!done[device]) {
+        const int mx = (int)dyn_smem<Body>(MAX_STAGES);
+        const int one = (int)dyn_smem<Body>(1);
+        CC_CUDA(cudaFuncSetAttribute(k_agent<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, std::min(mx, 227 * 1024)));
+        CC_CUDA(cudaFuncSetAttribute(k_default<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, one));
+        CC_CUDA(cudaFuncSetAttribute(k_redirect<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, one));
+        done[device] = true;
+    }
+    return CC_OK;
+}
+
+// agents per SM the hardware can keep resident for `stages` ring buffers
+template <class Body>
+static cc_status occupancy(int device, int stages, int* occ) {
+    CC_TRY(prepare_body<Body>(device));
+    static std::mutex mu;
+    static int cache[64][MAX_STAGES + 1] = {};
+    std::lock_guard<std::mutex> lk(mu);
+    if (stages < 1 || stages > MAX_STAGES) return fail(CC_ERR_INVALID_ARG, "stages %d outside [1, %d]", stages, MAX_STAGES);
+    if (!cache[device][stages]) {
         int prev = 0, n = 0;
         CC_CUDA(cudaGetDevice(&prev));
         CC_CUDA(cudaSetDevice(device));
-        CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_agent<Body>, Body::kThreads, 0));
+        CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_agent<Body>, Body::kConsumers + PRODUCER_THREADS,
+                                                              dyn_smem<Body>(stages)));
         CC_CUDA(cudaSetDevice(prev));
-        cache[device] = n > 0 ? n : 1;
+        cache[device][stages] = n > 0 ? n : -1;
     }
-    *occ = cache[device];
+    *occ = cache[device][stages];
+    if (*occ < 0) return fail(CC_ERR_UNSUPPORTED, "%d stages of %d bytes do not fit one SM", stages, Body::kStageBytes);
     return CC_OK;
 }
 
@@ -327,13 +357,13 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     int occ = 0;
     cc_status s;
     switch (k) {
-    case CC_K_CENSUS: s = occupancy<CensusBody>(device, &occ); break;
-    case CC_K_MATVEC: s = occupancy<MatvecB>(device, &occ); break;
-    case CC_K_ATAX: s = occupancy<RowB>(device, &occ); break;
-    case CC_K_BICG: case CC_K_MVT: s = occupancy<BothB>(device, &occ); break;
-    case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, &occ); break;
-    case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, &occ); break;
-    case CC_K_SPMV: s = occupancy<SpmvBody>(device, &occ); break;
+    case CC_K_CENSUS: s = occupancy<CensusBody>(device, CensusBody::kDefaultStages, &occ); break;
+    case CC_K_MATVEC: s = occupancy<MatvecB>(device, MatvecB::kDefaultStages, &occ); break;
+    case CC_K_ATAX: s = occupancy<RowB>(device, RowB::kDefaultStages, &occ); break;
+    case CC_K_BICG: case CC_K_MVT: s = occupancy<BothB>(device, BothB::kDefaultStages, &occ); break;
+    case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, Jacobi5Body::kDefaultStages, &occ); break;
+    case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, Conv2dBody<3>::kDefaultStages, &occ); break;
+    case CC_K_SPMV: s = occupancy<SpmvBody>(device, SpmvBody::kDefaultStages, &occ); break;
     default: return fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
     }
     if (s == CC_OK) *out = occ;
@@ -352,6 +382,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     const Grid& g = c.p->g;
     if (g.V == 0) return CC_OK;
     const cc_launch_opts& o = *c.o;
+    CC_TRY(prepare_body<Body>(c.p->device));
     Sched s{};
     s.g = g;
     s.user = c.p->d_user;
@@ -359,31 +390,35 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     s.smid_span = c.p->facts->smid_span;
     s.ws = c.p->d_ws;
     s.steal = o.steal;
-    s.prefetch = o.prefetch;
+    s.batch = o.batch > 0 ? o.batch : Body::kDefaultBatch;
+    s.stage_bytes = Body::kStageBytes;
     s.census = o.d_census;
     s.exec_sm = o.d_exec_sm;
     s.map = o.d_map;
+    const int threads = Body::kConsumers + PRODUCER_THREADS;
     switch (o.backend) {
     case CC_BACKEND_DEFAULT: {
         if (g.gy > 65535) return fail(CC_ERR_UNSUPPORTED, "default backend: gy %d > 65535", g.gy);
         s.map = nullptr;
-        k_default<Body><<<dim3(g.gx, g.gy), Body::kThreads, 0, c.st>>>(s, prm);
+        s.stages = 1;
+        k_default<Body><<<dim3(g.gx, g.gy), threads, dyn_smem<Body>(1), c.st>>>(s, prm);
         break;
     }
     case CC_BACKEND_REDIRECT:
-        k_redirect<Body><<<g.V, Body::kThreads, 0, c.st>>>(s, prm);
+        s.stages = 1;
+        k_redirect<Body><<<g.V, threads, dyn_smem<Body>(1), c.st>>>(s, prm);
         break;
     case CC_BACKEND_AGENT:
     case CC_BACKEND_AGENT_IDENTITY: {
+        const int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
         int occ = 0;
-        cc_status st = occupancy<Body>(c.p->device, &occ);
-        if (st != CC_OK) return st;
-        int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
-        int act = o.active_agents > 0 ? std::min(o.active_agents, maxa) : maxa;
-        s.active_agents = act;
+        CC_TRY(occupancy<Body>(c.p->device, S, &occ));
+        const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
+        s.active_agents = o.active_agents > 0 ? std::min(o.active_agents, maxa) : maxa;
         s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
-        int grid = c.p->facts->num_sms * maxa;
-        k_agent<Body><<<grid, Body::kThreads, 0, c.st>>>(s, prm);
+        s.stages = S;
+        const int grid = c.p->facts->num_sms * maxa;
+        k_agent<Body><<<grid, threads, dyn_smem<Body>(S), c.st>>>(s, prm);
         break;
     }
     default:
@@ -394,7 +429,6 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     if (c.nl) ++*c.nl;
     return CC_OK;
 }
-
 
 // ---- thread-block-cluster backend (conv2d) --------------------------------
 static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {

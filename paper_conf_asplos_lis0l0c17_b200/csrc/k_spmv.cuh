@@ -13,6 +13,7 @@
 // calls hard to exploit); val/col stream past it.
 #pragma once
 #include "cc_mem.cuh"
+#include "cc_runtime.cuh"
 
 namespace cc {
 
@@ -51,25 +52,32 @@ __global__ void k_spmv_partition(const int32_t* row_ptr, int32_t rows, int64_t n
 }
 
 struct SpmvBody {
-    static constexpr int kThreads = SPMV_THREADS;
+    static constexpr int kConsumers = SPMV_THREADS;
+    static constexpr int kStageBytes = 128;       // nothing staged: reads go straight to L1/L2
+    static constexpr int kDefaultStages = 2;
+    static constexpr int kDefaultBatch = 2;
     using Params = SpmvParams;
     SpmvParams p;
     __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}
 
-    __device__ __forceinline__ void run(int32_t bx, int32_t /*by*/) {
+    __device__ __forceinline__ void produce(int32_t, int32_t, uint8_t*, uint64_t* full, int lane) {
+        stage_commit(full, lane, 0);
+    }
+
+    __device__ __forceinline__ void consume(int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
         __shared__ int32_t s_rowend[SPMV_IPC + 1];
         __shared__ float s_prod[SPMV_IPT][SPMV_THREADS];
         __shared__ float s_wv[SPMV_THREADS / 32];
         __shared__ int32_t s_wf[SPMV_THREADS / 32];
-        const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+        const int t = ctid, lane = t & 31, warp = t >> 5;
         const int64_t total = (int64_t)p.rows + p.nnz;
         const int64_t d0 = (int64_t)bx * SPMV_IPC;
         const int64_t d1 = d0 + SPMV_IPC < total ? d0 + SPMV_IPC : total;
         const int32_t x0 = p.part[bx], x1 = p.part[bx + 1];
         const int64_t y0 = d0 - x0, y1 = d1 - x1;
         const int32_t xl = x1 < p.rows ? x1 : p.rows - 1;      // last row to stage
-        for (int32_t i = t; i <= xl - x0; i += kThreads) s_rowend[i] = p.row_ptr[x0 + i + 1];
-        __syncthreads();
+        for (int32_t i = t; i <= xl - x0; i += kConsumers) s_rowend[i] = p.row_ptr[x0 + i + 1];
+        consumer_sync<kConsumers>();
         // this thread's start on the merge path, relative to the CTA rectangle
         const int32_t span = (int32_t)(d1 - d0);
         const int32_t dt = t * SPMV_IPT < span ? t * SPMV_IPT : span;
@@ -122,7 +130,7 @@ struct SpmvBody {
             if (lane >= o) { if (!f) v += vu; f = f || fu; }
         }
         if (lane == 31) { s_wv[warp] = v; s_wf[warp] = f; }
-        __syncthreads();
+        consumer_sync<kConsumers>();
         float pv = 0.f;                      // prefix of earlier warps
         for (int w = 0; w < warp; ++w) pv = s_wf[w] ? s_wv[w] : pv + s_wv[w];
         const float T = f ? v : pv + v;      // outgoing carry of this thread
@@ -135,25 +143,13 @@ struct SpmvBody {
             if (started_before) atomicAdd(p.y + first_row, val);
             else p.y[first_row] = val;
         }
-        if (t == kThreads - 1 && x1 < p.rows && T != 0.f) atomicAdd(p.y + x1, T);
-        __syncthreads();                     // s_wv / s_rowend reuse by the next task
+        if (t == kConsumers - 1 && x1 < p.rows && T != 0.f) atomicAdd(p.y + x1, T);
+        consumer_sync<kConsumers>();                     // s_wv / s_rowend reuse by the next task
     }
     __device__ __forceinline__ int64_t row_start(int32_t r) const {
         return r == 0 ? 0 : (int64_t)p.row_ptr[r];
     }
-    __device__ __forceinline__ void prefetch_l2(int32_t bx, int32_t) {
-        const int32_t x0 = p.part[bx];
-        const int64_t y0 = (int64_t)bx * SPMV_IPC - x0;
-        int64_t n = p.nnz - y0; if (n > SPMV_IPC) n = SPMV_IPC;
-        if (n <= 0) return;
-        const int32_t* c = p.col + y0;
-        const float* v = p.val + y0;
-        uintptr_t a = (uintptr_t)c & ~(uintptr_t)15, e = ((uintptr_t)(c + n) + 15) & ~(uintptr_t)15;
-        prefetch_l2_bulk((const void*)a, (uint32_t)(e - a));
-        a = (uintptr_t)v & ~(uintptr_t)15; e = ((uintptr_t)(v + n) + 15) & ~(uintptr_t)15;
-        prefetch_l2_bulk((const void*)a, (uint32_t)(e - a));
-    }
-    __device__ __forceinline__ void finish() {}
+    __device__ __forceinline__ void finish(int) {}
 };
 
 }  // namespace cc

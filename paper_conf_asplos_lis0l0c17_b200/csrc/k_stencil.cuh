@@ -1,17 +1,46 @@
 // k_stencil.cuh -- 5-point Jacobi and 2D cross-correlation tile bodies.
 //
 // Logical CTA (bx, by) computes the 32 x 32 output tile at rows 32*by..,
-// columns 32*bx.. .  The inter-CTA reuse is the halo: rows above/below and
-// the columns left/right of a tile are the border data of its four neighbours
-// (the cache-line/algorithm-related classes).  Halo and centre loads
-// allocate in L1, so when clustering runs neighbouring tiles on the same SM
-// close together (TILE order, Fig. 7) the halo comes from L1 instead of L2.
-// 256 threads: thread (r = tid/8, c4 = tid%8) owns the float4 at row r,
-// columns 4*c4 .. 4*c4+3 of the tile.
+// columns 32*bx.. .  The inter-CTA reuse is the halo: the H rows above/below
+// and the columns left/right of a tile are the border data of its neighbours
+// (the cache-line/algorithm-related classes).
+//
+// The producer warp stages the tile plus halo -- rows y0-H .. y0+31+H, columns
+// x0-4 .. x0+35 (10 aligned 16-byte chunks per row) -- into shared memory with
+// cp.async.ca, which also allocates every line in L1.  A neighbouring tile
+// staged soon after on the same SM therefore finds its halo (and the shared
+// 16-byte edge chunks) in L1 instead of L2: clustering neighbouring tiles onto
+// one SM (TILE order, Fig. 7) turns that halo traffic into L1 hits.  Chunks
+// outside the image are zero-filled without a read.
+// Consumers: 256 threads; thread (r = ctid/8, c4 = ctid%8) owns the float4 at
+// row r, columns 4*c4 .. 4*c4+3 of the tile.
 #pragma once
 #include "cc_mem.cuh"
+#include "cc_runtime.cuh"
 
 namespace cc {
+
+constexpr int ST_COLS = 40;                 // staged floats per row (x0-4 .. x0+35)
+
+template <int H>
+struct HaloTile {
+    static constexpr int kRows = 32 + 2 * H;
+    static constexpr int kBytes = ((kRows * ST_COLS * 4) + 127) & ~127;
+    // warp-collective: stage rows y0-H.., columns x0-4.. of `src`.
+    __device__ __forceinline__ static void stage(const float* src, int64_t ld, int32_t rows, int32_t cols,
+                                                 int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane) {
+        const int32_t cols4 = (cols + 3) & ~3;   // last 16-byte chunk stays inside ld
+        for (int idx = lane; idx < kRows * 10; idx += 32) {
+            const int rr = idx / 10, cc = idx - rr * 10;
+            const int32_t gy = y0 - H + rr, gx = x0 - 4 + 4 * cc;
+            const bool ok = gy >= 0 && gy < rows && gx >= 0 && gx < cols4;
+            const float* g = ok ? src + (int64_t)gy * ld + gx : src;
+            cp_async_ca16(dst + (rr * ST_COLS + 4 * cc) * 4, g, ok ? 16u : 0u);
+        }
+        cp_async_arrive(full);
+        stage_commit(full, lane, 0);
+    }
+};
 
 // ---------------------------------------------------------------------------
 // Jacobi 5-point sweep (reading R14, PolyBench jacobi-2d form):
@@ -23,35 +52,28 @@ namespace cc {
 struct JacobiParams { const float* a; float* b; int64_t ld; int32_t rows, cols; };
 
 struct Jacobi5Body {
-    static constexpr int kThreads = 256;
+    static constexpr int kConsumers = 256;
+    static constexpr int kStageBytes = HaloTile<1>::kBytes;
+    static constexpr int kDefaultStages = 3;
+    static constexpr int kDefaultBatch = 4;
     using Params = JacobiParams;
     JacobiParams p;
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
 
-    __device__ __forceinline__ void run(int32_t bx, int32_t by) {
-        __shared__ float4 tile[34][8];
-        const int r = threadIdx.x >> 3, c4 = threadIdx.x & 7;
-        const int x0 = bx * 32, y0 = by * 32;
-        const int gy = y0 + r, gx = x0 + 4 * c4;
-        const bool in_row = gy < p.rows, in_col = gx < p.cols;
-        const float* a = p.a;
-        float4 c = (in_row && in_col) ? ld_cached4(a + (int64_t)gy * p.ld + gx) : f4_zero();
-        float4 up_h = f4_zero(), dn_h = f4_zero();
-        if (r == 0 && y0 > 0 && in_col) up_h = ld_cached4(a + (int64_t)(y0 - 1) * p.ld + gx);
-        if (r == 31 && y0 + 32 < p.rows && in_col) dn_h = ld_cached4(a + (int64_t)(y0 + 32) * p.ld + gx);
-        float left = 0.f, right = 0.f;
-        if (c4 == 0 && x0 > 0 && in_row) left = ld_cached(a + (int64_t)gy * p.ld + x0 - 1);
-        if (c4 == 7 && x0 + 32 < p.cols && in_row) right = ld_cached(a + (int64_t)gy * p.ld + x0 + 32);
-        tile[r + 1][c4] = c;
-        if (r == 0) tile[0][c4] = up_h;
-        if (r == 31) tile[33][c4] = dn_h;
-        __syncthreads();
-        const float4 up = tile[r][c4], dn = tile[r + 2][c4];
-        float lw = __shfl_up_sync(0xffffffffu, c.w, 1, 8);
-        float re = __shfl_down_sync(0xffffffffu, c.x, 1, 8);
-        if (c4 == 0) lw = left;
-        if (c4 == 7) re = right;
-        if (!(in_row && in_col)) return;   // after the barrier and the shuffles
+    __device__ __forceinline__ void produce(int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane);
+    }
+
+    __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        const int r = ctid >> 3, c4 = ctid & 7;
+        const int gy = by * 32 + r, gx = bx * 32 + 4 * c4;
+        if (gy >= p.rows || gx >= p.cols) return;
+        const float* t = reinterpret_cast<const float*>(stage);
+        const float* mid = t + (r + 1) * ST_COLS + 4 + 4 * c4;
+        const float4 c = *reinterpret_cast<const float4*>(mid);
+        const float4 up = *reinterpret_cast<const float4*>(mid - ST_COLS);
+        const float4 dn = *reinterpret_cast<const float4*>(mid + ST_COLS);
+        const float lw = mid[-1], re = mid[4];
         float4 o;
         o.x = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.x, lw), c.y), up.x), dn.x));
         o.y = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.y, c.x), c.z), up.y), dn.y));
@@ -71,94 +93,70 @@ struct Jacobi5Body {
             if (gx + 2 < p.cols) dst[2] = o.z;
         }
     }
-    __device__ __forceinline__ void prefetch_l2(int32_t bx, int32_t by) {
-        const int x0 = bx * 32;
-        if (x0 >= p.cols) return;
-        int cols = p.cols - x0 < 32 ? p.cols - x0 : 32;
-        uint32_t bytes = (uint32_t)((cols * 4 + 15) & ~15);
-        for (int k = -1; k <= 32; ++k) {
-            int row = by * 32 + k;
-            if (row < 0) continue;
-            if (row >= p.rows) break;
-            prefetch_l2_bulk(p.a + (int64_t)row * p.ld + x0, bytes);
-        }
-    }
-    __device__ __forceinline__ void finish() {}
+    __device__ __forceinline__ void finish(int) {}
 };
 
 // ---------------------------------------------------------------------------
 // 2D cross-correlation with a (2R+1)^2 filter (reading R15):
 //   out[i][j] = sum_{a,b} w[a+R][b+R] * in[i+a][j+b]   interior, else 0.
-// The input tile plus an R halo is staged in shared memory with aligned
-// float4 loads covering columns x0-4 .. x0+35.
+// The filter lives in the kernel parameter bank (constant-bank operands).
 // ---------------------------------------------------------------------------
 template <int R>
 struct ConvParams { const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
 
 template <int R>
+__device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const float* rows_base,
+                                                  int32_t bx, int32_t by, int ctid) {
+    // rows_base points at the staged row holding input row y0 - R, column x0 - 4
+    constexpr int K = 2 * R + 1;
+    const int r = ctid >> 3, c4 = ctid & 7;
+    const int gy = by * 32 + r, gx = bx * 32 + 4 * c4;
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+    for (int dy = 0; dy < K; ++dy) {
+        const float4* row = reinterpret_cast<const float4*>(rows_base + (r + dy) * ST_COLS + 4 * c4);
+        float4 q0 = row[0], q1 = row[1], q2 = row[2];
+        const float win[12] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w, q2.x, q2.y, q2.z, q2.w};
+#pragma unroll
+        for (int dx = 0; dx < K; ++dx) {
+            const float wt = p.w[dy * K + dx];
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[e] = fmaf(wt, win[4 + e + dx - R], acc[e]);
+        }
+    }
+    if (gy >= p.rows || gx >= p.cols) return;
+    const bool row_in = gy >= R && gy < p.rows - R;
+    float4 o;
+    o.x = (row_in && gx + 0 >= R && gx + 0 < p.cols - R) ? acc[0] : 0.f;
+    o.y = (row_in && gx + 1 >= R && gx + 1 < p.cols - R) ? acc[1] : 0.f;
+    o.z = (row_in && gx + 2 >= R && gx + 2 < p.cols - R) ? acc[2] : 0.f;
+    o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[3] : 0.f;
+    float* dst = p.out + (int64_t)gy * p.ld + gx;
+    if (gx + 4 <= p.cols) *reinterpret_cast<float4*>(dst) = o;
+    else {
+        dst[0] = o.x;
+        if (gx + 1 < p.cols) dst[1] = o.y;
+        if (gx + 2 < p.cols) dst[2] = o.z;
+    }
+}
+
+template <int R>
 struct Conv2dBody {
-    static constexpr int kThreads = 256;
-    static constexpr int K = 2 * R + 1;
-    static constexpr int SR = 32 + 2 * R;   // staged rows
+    static constexpr int kConsumers = 256;
+    static constexpr int kStageBytes = HaloTile<R>::kBytes;
+    static constexpr int kDefaultStages = 3;
+    static constexpr int kDefaultBatch = 4;
     using Params = ConvParams<R>;
-    ConvParams<R> p;   // filter lives in the parameter bank (constant operands)
+    ConvParams<R> p;
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
 
-    __device__ __forceinline__ void run(int32_t bx, int32_t by) {
-        __shared__ float4 s_in[SR][10];
-        const int x0 = bx * 32, y0 = by * 32;
-        for (int idx = threadIdx.x; idx < SR * 10; idx += kThreads) {
-            const int rr = idx / 10, cc = idx - rr * 10;
-            const int gy = y0 - R + rr, gx = x0 - 4 + 4 * cc;
-            float4 v = f4_zero();
-            if (gy >= 0 && gy < p.rows && gx >= 0 && gx < p.cols) v = ld_cached4(p.in + (int64_t)gy * p.ld + gx);
-            s_in[rr][cc] = v;
-        }
-        __syncthreads();
-        const int r = threadIdx.x >> 3, c4 = threadIdx.x & 7;
-        const int gy = y0 + r, gx = x0 + 4 * c4;
-        float acc[4] = {0.f, 0.f, 0.f, 0.f};
-#pragma unroll
-        for (int dy = 0; dy < K; ++dy) {
-            const float4* row = &s_in[r + dy][c4];
-            float4 q0 = row[0], q1 = row[1], q2 = row[2];
-            const float win[12] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w, q2.x, q2.y, q2.z, q2.w};
-#pragma unroll
-            for (int dx = 0; dx < K; ++dx) {
-                const float wt = p.w[dy * K + dx];
-#pragma unroll
-                for (int e = 0; e < 4; ++e) acc[e] = fmaf(wt, win[4 + e + dx - R], acc[e]);
-            }
-        }
-        if (gy >= p.rows || gx >= p.cols) return;
-        const bool row_in = gy >= R && gy < p.rows - R;
-        float4 o;
-        o.x = (row_in && gx + 0 >= R && gx + 0 < p.cols - R) ? acc[0] : 0.f;
-        o.y = (row_in && gx + 1 >= R && gx + 1 < p.cols - R) ? acc[1] : 0.f;
-        o.z = (row_in && gx + 2 >= R && gx + 2 < p.cols - R) ? acc[2] : 0.f;
-        o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[3] : 0.f;
-        float* dst = p.out + (int64_t)gy * p.ld + gx;
-        if (gx + 4 <= p.cols) *reinterpret_cast<float4*>(dst) = o;
-        else {
-            dst[0] = o.x;
-            if (gx + 1 < p.cols) dst[1] = o.y;
-            if (gx + 2 < p.cols) dst[2] = o.z;
-        }
+    __device__ __forceinline__ void produce(int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane);
     }
-    __device__ __forceinline__ void prefetch_l2(int32_t bx, int32_t by) {
-        const int x0 = bx * 32 - 4;
-        int c0 = x0 < 0 ? 0 : x0;
-        int c1 = bx * 32 + 36; if (c1 > p.cols) c1 = p.cols;
-        if (c1 <= c0) return;
-        uint32_t bytes = (uint32_t)(((c1 - c0) * 4 + 15) & ~15);
-        for (int k = -R; k < 32 + R; ++k) {
-            int row = by * 32 + k;
-            if (row < 0) continue;
-            if (row >= p.rows) break;
-            prefetch_l2_bulk(p.in + (int64_t)row * p.ld + c0, bytes);
-        }
+    __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        conv_tile_compute<R>(p, reinterpret_cast<const float*>(stage), bx, by, ctid);
     }
-    __device__ __forceinline__ void finish() {}
+    __device__ __forceinline__ void finish(int) {}
 };
 
 }  // namespace cc

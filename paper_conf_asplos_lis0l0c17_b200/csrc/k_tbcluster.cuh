@@ -25,9 +25,6 @@ constexpr int TBC_COLS = 40;            // staged columns per row (x0-4 .. x0+35
 constexpr int TBC_ROW_BYTES = TBC_COLS * 4;
 constexpr int TBC_HALO = 8;             // halo box height (keeps boxes 128-B aligned)
 
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-    return (uint32_t)__cvta_generic_to_shared(p);
-}
 __device__ __forceinline__ uint32_t cluster_ctarank() {
     uint32_t r;
     asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
@@ -35,22 +32,6 @@ __device__ __forceinline__ uint32_t cluster_ctarank() {
 }
 __device__ __forceinline__ void cluster_sync_all() {
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void fence_mbar_init() {
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n}" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
 }
 // 2D TMA load of box (x, y) multicast to every CTA in `mask` (same smem offset
 // and same mbarrier offset in each destination CTA).
@@ -71,7 +52,6 @@ template <int R>
 __global__ void __launch_bounds__(256) k_conv_tbc(const __grid_constant__ CUtensorMap map_rows,
                                                   const __grid_constant__ CUtensorMap map_halo,
                                                   Sched s, ConvParams<R> p, int32_t C) {
-    constexpr int K = 2 * R + 1;
     extern __shared__ __align__(128) uint8_t smem_raw[];
     uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw);
     const uint32_t sbase = smem_u32(smem_raw);
@@ -88,44 +68,15 @@ __global__ void __launch_bounds__(256) k_conv_tbc(const __grid_constant__ CUtens
     }
     cluster_sync_all();                         // every barrier initialised before any multicast lands
     if (threadIdx.x == 0) {
-        mbar_expect_tx(bar, total);
+        mbar_arrive_tx(bar, total);
         tma_load_2d_mc(&map_rows, region + (TBC_HALO + 32 * rank) * TBC_COLS, bar, x0 - 4, r0 + 32 * rank, mask);
         if (rank == 0) tma_load_2d_mc(&map_halo, region, bar, x0 - 4, r0 - TBC_HALO, mask);
         if (rank == C - 1)
             tma_load_2d_mc(&map_halo, region + (TBC_HALO + 32 * C) * TBC_COLS, bar, x0 - 4, r0 + 32 * C, mask);
     }
     mbar_wait(bar, 0);
-    const int r = threadIdx.x >> 3, c4 = threadIdx.x & 7;
-    const int gy = by * 32 + r, gx = x0 + 4 * c4;
-    float acc[4] = {0.f, 0.f, 0.f, 0.f};
-    const float* base = region + (TBC_HALO + 32 * rank + r - R) * TBC_COLS + 4 * c4;
-#pragma unroll
-    for (int dy = 0; dy < K; ++dy) {
-        const float4* row = reinterpret_cast<const float4*>(base + dy * TBC_COLS);
-        float4 q0 = row[0], q1 = row[1], q2 = row[2];
-        const float win[12] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w, q2.x, q2.y, q2.z, q2.w};
-#pragma unroll
-        for (int dx = 0; dx < K; ++dx) {
-            const float wt = p.w[dy * K + dx];
-#pragma unroll
-            for (int e = 0; e < 4; ++e) acc[e] = fmaf(wt, win[4 + e + dx - R], acc[e]);
-        }
-    }
-    if (by < s.g.gy && gy < p.rows && gx < p.cols) {
-        const bool row_in = gy >= R && gy < p.rows - R;
-        float4 o;
-        o.x = (row_in && gx + 0 >= R && gx + 0 < p.cols - R) ? acc[0] : 0.f;
-        o.y = (row_in && gx + 1 >= R && gx + 1 < p.cols - R) ? acc[1] : 0.f;
-        o.z = (row_in && gx + 2 >= R && gx + 2 < p.cols - R) ? acc[2] : 0.f;
-        o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[3] : 0.f;
-        float* dst = p.out + (int64_t)gy * p.ld + gx;
-        if (gx + 4 <= p.cols) *reinterpret_cast<float4*>(dst) = o;
-        else {
-            dst[0] = o.x;
-            if (gx + 1 < p.cols) dst[1] = o.y;
-            if (gx + 2 < p.cols) dst[2] = o.z;
-        }
-    }
+    if (by < s.g.gy)
+        conv_tile_compute<R>(p, region + (TBC_HALO + 32 * rank - R) * TBC_COLS, bx, by, threadIdx.x);
     if (threadIdx.x == 0 && by < s.g.gy) {
         int32_t lin = by * s.g.gx + bx;
         if (s.census) atomicAdd(s.census + lin, 1u);

@@ -22,7 +22,8 @@ VARIANTS = [
     dict(backend="agent", order="col"),
     dict(backend="agent", order="tile", tile=(4, 4)),
     dict(backend="agent", order="col", active_agents=1),
-    dict(backend="agent", order="col", prefetch=1),
+    dict(backend="agent", order="col", stages=1),
+    dict(backend="agent", order="col", stages=6, batch=3),
     dict(backend="identity"),
     dict(backend="redirect", order="row"),
 ]
@@ -127,7 +128,7 @@ def test_bicg_full_size_config2():
 # ---------------------------------------------------------------- Jacobi
 JVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(8, 8)),
              dict(backend="agent", order="row"), dict(backend="agent", order="col", active_agents=2),
-             dict(backend="agent", order="tile", tile=(2, 2), prefetch=1), dict(backend="identity"),
+             dict(backend="agent", order="tile", tile=(2, 2), stages=8, batch=7), dict(backend="identity"),
              dict(backend="redirect", order="tile", tile=(4, 4))]
 
 
@@ -167,7 +168,7 @@ def test_jacobi_full_size_sampled():
 
 # ---------------------------------------------------------------- conv2d
 CVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(8, 8)),
-             dict(backend="agent", order="col", prefetch=1), dict(backend="identity"),
+             dict(backend="agent", order="col", stages=1, batch=1), dict(backend="identity"),
              dict(backend="tbcluster", cluster_size=1), dict(backend="tbcluster", cluster_size=2),
              dict(backend="tbcluster", cluster_size=4), dict(backend="tbcluster", cluster_size=8),
              dict(backend="redirect", order="row")]
@@ -228,7 +229,7 @@ def _csr_dev(rp, col, val):
 
 
 SVARIANTS = [dict(backend="default"), dict(backend="agent", order="row"), dict(backend="agent", active_agents=1),
-             dict(backend="agent", prefetch=1), dict(backend="identity"), dict(backend="redirect")]
+             dict(backend="agent", stages=4, batch=5), dict(backend="identity"), dict(backend="redirect")]
 
 
 def _edge_matrices():
