@@ -120,6 +120,11 @@ def suite_jacobi(quick):
                 ("agent-tile16x16", dict(backend="agent", order="tile", tile=(16, 16))),
                 ("agent-col", dict(backend="agent", order="col")), ("agent-row", dict(backend="agent", order="row")),
                 ("agent-tile8x8-tot4", dict(backend="agent", order="tile", tile=(8, 8), active_agents=4)),
+                ("agent-tile8x8-bps", dict(backend="agent", order="tile", tile=(8, 8), bypass=1)),
+                ("agent-row-bps", dict(backend="agent", order="row", bypass=1)),
+                ("agent-tile8x8-s2", dict(backend="agent", order="tile", tile=(8, 8), stages=2)),
+                ("agent-tile8x8-s5", dict(backend="agent", order="tile", tile=(8, 8), stages=5)),
+                ("default-bps", dict(backend="default", bypass=1)),
                 ("identity", dict(backend="identity"))]
     rows, base = [], None
     for name, kw in variants:
@@ -145,6 +150,9 @@ def suite_conv(quick):
         variants = [("default", dict(backend="default")),
                     ("agent-tile8x8", dict(backend="agent", order="tile", tile=(8, 8))),
                     ("agent-col", dict(backend="agent", order="col")),
+                    ("agent-tile8x8-bps", dict(backend="agent", order="tile", tile=(8, 8), bypass=1)),
+                    ("agent-col-bps", dict(backend="agent", order="col", bypass=1)),
+                    ("default-bps", dict(backend="default", bypass=1)),
                     ("tbcluster-2", dict(backend="tbcluster", cluster_size=2)),
                     ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
                     ("tbcluster-8", dict(backend="tbcluster", cluster_size=8)),

@@ -132,6 +132,9 @@ typedef struct {
                                B200 form of "prefetch the next CTA" (§4.3(III),
                                Listing 5 l.34-37); 0 => the kernel's default, 1..8   */
     int32_t batch;          /* logical CTAs claimed per queue atomic; 0 => default   */
+    int32_t bypass;         /* cache bypassing "BPS" (§4.3(II)): 1 => the
+                               staged tile loads skip L1 (cp.async.cg); 0 => they
+                               allocate in L1 so neighbouring tasks can hit them     */
     int32_t steal;          /* 1 (default) => an agent whose cluster queue is empty
                                takes work from other clusters, so every CTA runs exactly
                                once whatever the hardware does with agent placement

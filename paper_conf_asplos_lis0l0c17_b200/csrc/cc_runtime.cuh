@@ -51,6 +51,7 @@ struct Sched {
     int32_t stages;               // ring depth (agent backends; 1 for one-shot CTAs)
     int32_t batch;                // slots claimed per queue atomic
     uint32_t stage_bytes;         // bytes per ring buffer (128-byte multiple)
+    int32_t bypass;               // staged loads skip L1 (BPS, §4.3(II))
     uint32_t* census;             // optional outputs (see ctaclust.h)
     int32_t* exec_sm;
     int32_t* map;
@@ -116,6 +117,11 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // src_bytes < 16 zero-fills the rest (0 => pure zero fill, no read).
 __device__ __forceinline__ void cp_async_ca16(void* dst, const void* src, uint32_t src_bytes) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 16, %2;"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(src_bytes) : "memory");
+}
+// the bypassing variant (.cg: cached in L2 only)
+__device__ __forceinline__ void cp_async_cg16(void* dst, const void* src, uint32_t src_bytes) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;"
                  :: "r"(smem_u32(dst)), "l"(src), "r"(src_bytes) : "memory");
 }
 // this thread's prior cp.async ops complete -> one (pre-counted) arrival on bar
@@ -242,7 +248,7 @@ __device__ __forceinline__ int32_t producer_next(const Sched& s, Prod& P, int la
 // ---------------------------------------------------------------------------
 // Body concept (see k_gemv.cuh / k_stencil.cuh / k_spmv.cuh):
 //   kConsumers, kStageBytes, kDefaultStages, kDefaultBatch
-//   produce(bx, by, stage, full, lane)  warp 0, all lanes: stage the task's
+//   produce(s, bx, by, stage, full, lane)  warp 0, all lanes: stage the task's
 //                                       input and commit (stage_commit)
 //   consume(bx, by, stage, ctid)        consumer threads ctid in [0, kConsumers)
 //   finish(ctid)                        consumers, agent retiring: flush state
@@ -303,7 +309,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             }
             int32_t lin, bx, by;
             lin_to_bxby(s, v, &lin, &bx, &by);
-            body.produce(bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
+            body.produce(s, bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
         }
         // ---- the last agent out resets the workspace for the next launch.  Every
         // other agent's producer has consumed the results of all its atomics
@@ -344,7 +350,7 @@ __device__ __forceinline__ void one_shot(const Sched& s, Body& body, int32_t v, 
     if (threadIdx.x == 0) { mbar_init(&full, 1); fence_mbar_init(); }
     __syncthreads();
     if (threadIdx.x < PRODUCER_THREADS) {
-        body.produce(bx, by, ring, &full, threadIdx.x);
+        body.produce(s, bx, by, ring, &full, threadIdx.x);
     } else {
         const int ctid = threadIdx.x - PRODUCER_THREADS;
         mbar_wait(&full, 0);

@@ -299,7 +299,7 @@ struct CensusBody {   // empty body: binding, queues and census only
     static constexpr int kDefaultBatch = 1;
     using Params = CensusParams;
     __device__ __forceinline__ explicit CensusBody(const CensusParams&) {}
-    __device__ __forceinline__ void produce(int32_t, int32_t, uint8_t*, uint64_t* full, int lane) { stage_commit(full, lane, 0); }
+    __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) { stage_commit(full, lane, 0); }
     __device__ __forceinline__ void consume(int32_t, int32_t, const uint8_t*, int) {}
     __device__ __forceinline__ void finish(int) {}
 };
@@ -320,9 +320,13 @@ static cc_status prepare_body(int device) {
     std::lock_guard<std::mutex> lk(mu);
     if (device < 0 || device >= 64) return fail(CC_ERR_INVALID_ARG, "device");
     if (!done[device]) {
-        const int mx = (int)dyn_smem<Body>(MAX_STAGES);
+        int optin = 0;
+        CC_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
+        cudaFuncAttributes fa{};
+        CC_CUDA(cudaFuncGetAttributes(&fa, k_agent<Body>));
+        const int mx = (int)std::min(dyn_smem<Body>(MAX_STAGES), (size_t)(optin - (int)fa.sharedSizeBytes));
         const int one = (int)dyn_smem<Body>(1);
-        CC_CUDA(cudaFuncSetAttribute(k_agent<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, std::min(mx, 227 * 1024)));
+        CC_CUDA(cudaFuncSetAttribute(k_agent<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
         CC_CUDA(cudaFuncSetAttribute(k_default<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, one));
         CC_CUDA(cudaFuncSetAttribute(k_redirect<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, one));
         done[device] = true;
@@ -391,6 +395,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     s.ws = c.p->d_ws;
     s.steal = o.steal;
     s.batch = o.batch > 0 ? o.batch : Body::kDefaultBatch;
+    s.bypass = o.bypass;
     s.stage_bytes = Body::kStageBytes;
     s.census = o.d_census;
     s.exec_sm = o.d_exec_sm;

@@ -61,7 +61,7 @@ struct GemvBody {
     }
 
     // ---- producer: one bulk copy per tile row (rows past m are not copied)
-    __device__ __forceinline__ void produce(int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+    __device__ __forceinline__ void produce(const Sched&, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
         const int col0 = bx * TC;
         const int cols = p.n - col0 < TC ? p.n - col0 : TC;
         const uint32_t bytes = (uint32_t)((cols * 4 + 15) & ~15);    // within lda (lda % 4 == 0)

@@ -60,7 +60,7 @@ struct SpmvBody {
     SpmvParams p;
     __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}
 
-    __device__ __forceinline__ void produce(int32_t, int32_t, uint8_t*, uint64_t* full, int lane) {
+    __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) {
         stage_commit(full, lane, 0);
     }
 

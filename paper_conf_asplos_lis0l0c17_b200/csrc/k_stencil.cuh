@@ -28,14 +28,22 @@ struct HaloTile {
     static constexpr int kBytes = ((kRows * ST_COLS * 4) + 127) & ~127;
     // warp-collective: stage rows y0-H.., columns x0-4.. of `src`.
     __device__ __forceinline__ static void stage(const float* src, int64_t ld, int32_t rows, int32_t cols,
-                                                 int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane) {
+                                                 int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
+                                                 int32_t bypass) {
         const int32_t cols4 = (cols + 3) & ~3;   // last 16-byte chunk stays inside ld
-        for (int idx = lane; idx < kRows * 10; idx += 32) {
-            const int rr = idx / 10, cc = idx - rr * 10;
-            const int32_t gy = y0 - H + rr, gx = x0 - 4 + 4 * cc;
-            const bool ok = gy >= 0 && gy < rows && gx >= 0 && gx < cols4;
-            const float* g = ok ? src + (int64_t)gy * ld + gx : src;
-            cp_async_ca16(dst + (rr * ST_COLS + 4 * cc) * 4, g, ok ? 16u : 0u);
+        // lanes 0..29 cover three staged rows (10 chunks each) per step
+        const int r0 = lane / 10, cc = lane - r0 * 10;
+        const int32_t gx = x0 - 4 + 4 * cc;
+        const bool col_ok = lane < 30 && gx >= 0 && gx < cols4;
+        if (lane < 30) {
+            for (int rr = r0; rr < kRows; rr += 3) {
+                const int32_t gy = y0 - H + rr;
+                const bool ok = col_ok && gy >= 0 && gy < rows;
+                const float* g = ok ? src + (int64_t)gy * ld + gx : src;
+                uint8_t* d = dst + (rr * ST_COLS + 4 * cc) * 4;
+                if (bypass) cp_async_cg16(d, g, ok ? 16u : 0u);
+                else cp_async_ca16(d, g, ok ? 16u : 0u);
+            }
         }
         cp_async_arrive(full);
         stage_commit(full, lane, 0);
@@ -60,8 +68,8 @@ struct Jacobi5Body {
     JacobiParams p;
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
 
-    __device__ __forceinline__ void produce(int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane);
+    __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass);
     }
 
     __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
@@ -150,8 +158,8 @@ struct Conv2dBody {
     ConvParams<R> p;
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
 
-    __device__ __forceinline__ void produce(int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane);
+    __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass);
     }
     __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         conv_tile_compute<R>(p, reinterpret_cast<const float*>(stage), bx, by, ctid);

@@ -50,7 +50,8 @@ class PlanDesc(ctypes.Structure):
 
 class LaunchOpts(ctypes.Structure):
     _fields_ = [("backend", _i32), ("active_agents", _i32), ("max_agents", _i32), ("stages", _i32),
-                ("batch", _i32), ("steal", _i32), ("cluster_size", _i32), ("d_census", _vp), ("d_exec_sm", _vp),
+                ("batch", _i32), ("bypass", _i32), ("steal", _i32), ("cluster_size", _i32), ("d_census", _vp),
+                ("d_exec_sm", _vp),
                 ("d_map", _vp)]
 
 
@@ -198,10 +199,10 @@ def _stream(stream):
     return s.cuda_stream
 
 
-def make_opts(backend="agent", active_agents=0, max_agents=0, stages=0, batch=0, steal=1, cluster_size=2,
-              census=None, exec_sm=None, map=None) -> LaunchOpts:
+def make_opts(backend="agent", active_agents=0, max_agents=0, stages=0, batch=0, bypass=0, steal=1,
+              cluster_size=2, census=None, exec_sm=None, map=None) -> LaunchOpts:
     b = BACKENDS[backend] if isinstance(backend, str) else int(backend)
-    return LaunchOpts(b, active_agents, max_agents, int(stages), int(batch), int(steal), cluster_size,
+    return LaunchOpts(b, active_agents, max_agents, int(stages), int(batch), int(bypass), int(steal), cluster_size,
                       _ptr(census), _ptr(exec_sm), _ptr(map))
 
 
