@@ -366,7 +366,8 @@ __device__ __forceinline__ void one_shot(const Sched& s, Body& body, int32_t v, 
 
 // ---- kernels: one per (body, backend) ------------------------------------
 template <class Body>
-__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_agent(Sched s, typename Body::Params p) {
+__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS, Body::kMinAgents)
+k_agent(Sched s, typename Body::Params p) {
     Body body(p);
     agent_loop(s, body);
 }

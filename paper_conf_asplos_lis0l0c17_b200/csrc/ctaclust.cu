@@ -297,6 +297,7 @@ struct CensusBody {   // empty body: binding, queues and census only
     static constexpr int kStageBytes = 128;
     static constexpr int kDefaultStages = 2;
     static constexpr int kDefaultBatch = 1;
+    static constexpr int kMinAgents = 8;
     using Params = CensusParams;
     __device__ __forceinline__ explicit CensusBody(const CensusParams&) {}
     __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) { stage_commit(full, lane, 0); }

@@ -19,8 +19,12 @@
 //     (vector) RED only when the row (column) changes -- temporal inter-CTA
 //     reuse kept on chip.  Under the default backend every CTA is a fresh task,
 //     so it flushes every time: same code, no clustering.
-// Consumers: 256 threads; CT = TC/4 threads cover one tile row with float4,
-// RG = 256/CT row groups, each thread owns RPT = TR/RG rows.
+//
+// Consumer mapping (256 threads = 8 warps): a tile row is covered by LPR =
+// min(32, TC/4) lanes, each holding FPL = TC/(4 LPR) float4 columns; a warp
+// covers RPW = 32/LPR rows per pass and runs NP = TR/(8 RPW) passes.  Row sums
+// reduce inside a warp (shuffles only); column sums only need the other warps
+// at a column flush, which clustering makes rare.
 #pragma once
 #include "cc_mem.cuh"
 #include "cc_runtime.cuh"
@@ -39,26 +43,31 @@ template <int TR, int TC, bool DO_ROW, bool DO_COL>
 struct GemvBody {
     static constexpr int kConsumers = 256;
     static constexpr int kStageBytes = TR * TC * 4;
-    static constexpr int kDefaultStages = TC >= 256 ? 4 : 3;
+    static constexpr int kDefaultStages = 2;
     static constexpr int kDefaultBatch = TC >= 256 ? 2 : 1;
-    static constexpr int CT = TC / 4;
-    static constexpr int RG = kConsumers / CT;
-    static constexpr int RPT = TR / RG;
-    static_assert(TC % 4 == 0 && kConsumers % CT == 0 && TR % RG == 0 && TR <= 32, "tile/thread shape");
-    static_assert(CT <= 32 || CT % 32 == 0, "row group must be whole warps or a warp slice");
-    static constexpr int WPR = CT > 32 ? CT / 32 : 1;   // warps per row group
+    static constexpr int kMinAgents = 3;
+    static constexpr int CW = TC / 4;                    // float4 columns per row
+    static constexpr int LPR = CW < 32 ? CW : 32;        // lanes per row
+    static constexpr int FPL = CW / LPR;                 // float4 per lane per row
+    static constexpr int RPW = 32 / LPR;                 // rows per warp pass
+    static constexpr int NP = TR / (8 * RPW);            // passes
+    static_assert(TC % 4 == 0 && CW % LPR == 0 && 32 % LPR == 0 && TR % (8 * RPW) == 0 && NP >= 1, "tile shape");
     using Params = GemvParams;
 
     GemvParams p;
     int32_t cur_ti, cur_tj;
-    float racc[RPT];
-    float4 cacc;
+    float racc[NP];
+    float4 cacc[FPL];
 
     __device__ __forceinline__ explicit GemvBody(const GemvParams& prm) : p(prm), cur_ti(-1), cur_tj(-1) {
 #pragma unroll
-        for (int k = 0; k < RPT; ++k) racc[k] = 0.f;
-        cacc = f4_zero();
+        for (int k = 0; k < NP; ++k) racc[k] = 0.f;
+#pragma unroll
+        for (int f = 0; f < FPL; ++f) cacc[f] = f4_zero();
     }
+    // tile-local row of (warp, pass, sub-row) and float4 column of (lane, f)
+    __device__ __forceinline__ static int trow(int warp, int k, int sub) { return (k * RPW + sub) * 8 + warp; }
+    __device__ __forceinline__ static int tcol4(int cl, int f) { return f * LPR + cl; }
 
     // ---- producer: one bulk copy per tile row (rows past m are not copied)
     __device__ __forceinline__ void produce(const Sched&, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
@@ -68,121 +77,96 @@ struct GemvBody {
         const int row0 = by * TR;
         const int nrows = p.m - row0 < TR ? p.m - row0 : TR;
         stage_commit(full, lane, bytes * (uint32_t)nrows);
-        if (lane < nrows)
-            bulk_g2s(stage + lane * (TC * 4), p.A + (int64_t)(row0 + lane) * p.lda + col0, bytes, full);
+        for (int r = lane; r < nrows; r += 32)
+            bulk_g2s(stage + r * (TC * 4), p.A + (int64_t)(row0 + r) * p.lda + col0, bytes, full);
     }
 
-    // ---- ROW flush: sum racc over the CT threads of a row group, one RED per row
+    // ---- ROW flush: warp-level sum over the LPR lanes of each row, one RED per row
     __device__ __forceinline__ void flush_row(int ctid) {
-        __shared__ float s_part[DO_ROW && WPR > 1 ? WPR : 1][DO_ROW && WPR > 1 ? TR : 1];
-        const int cg = ctid % CT, rg = ctid / CT, lane = ctid & 31;
-        constexpr int W = CT < 32 ? CT : 32;
+        const int warp = ctid >> 5, lane = ctid & 31, sub = lane / LPR, cl = lane % LPR;
 #pragma unroll
-        for (int k = 0; k < RPT; ++k) {
+        for (int k = 0; k < NP; ++k) {
             float v = racc[k];
 #pragma unroll
-            for (int o = W / 2; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o, W);
-            racc[k] = v;
+            for (int o = LPR / 2; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o, LPR);
+            const int row = cur_ti * TR + trow(warp, k, sub);
+            if (cl == 0 && row < p.m) red_add(p.out_r + row, v);
+            racc[k] = 0.f;
         }
-        const int row0 = cur_ti * TR;
-        if constexpr (WPR == 1) {
-            if (cg == 0) {
-#pragma unroll
-                for (int k = 0; k < RPT; ++k) {
-                    int row = row0 + rg + k * RG;
-                    if (row < p.m) red_add(p.out_r + row, racc[k]);
-                }
-            }
-        } else {
-            if (lane == 0) {
-#pragma unroll
-                for (int k = 0; k < RPT; ++k) s_part[cg / 32][rg + k * RG] = racc[k];
-            }
-            consumer_sync<kConsumers>();
-            if (ctid < TR) {
-                float v = 0.f;
-#pragma unroll
-                for (int w = 0; w < WPR; ++w) v += s_part[w][ctid];
-                int row = row0 + ctid;
-                if (row < p.m) red_add(p.out_r + row, v);
-            }
-            consumer_sync<kConsumers>();
-        }
-#pragma unroll
-        for (int k = 0; k < RPT; ++k) racc[k] = 0.f;
     }
 
-    // ---- COL flush: sum cacc over the RG row groups, one vector RED per 4 columns
+    // ---- COL flush: sum cacc over the 8 * RPW row slots, one vector RED per 4 columns
     __device__ __forceinline__ void flush_col(int ctid) {
-        const int cg = ctid % CT, rg = ctid / CT;
-        const int col = cur_tj * TC + cg * 4;
-        float4 v = cacc;
-        if constexpr (RG > 1) {
-            __shared__ float4 s_col[DO_COL ? RG : 1][DO_COL ? CT : 1];
-            s_col[rg][cg] = cacc;
-            consumer_sync<kConsumers>();
-            if (ctid < CT) {
-                v = s_col[0][ctid];
+        __shared__ float4 s_col[DO_COL ? 8 * RPW : 1][DO_COL ? CW : 1];
+        const int warp = ctid >> 5, lane = ctid & 31, sub = lane / LPR, cl = lane % LPR;
 #pragma unroll
-                for (int g = 1; g < RG; ++g) {
-                    float4 u = s_col[g][ctid];
-                    v.x += u.x; v.y += u.y; v.z += u.z; v.w += u.w;
+        for (int f = 0; f < FPL; ++f) s_col[warp * RPW + sub][tcol4(cl, f)] = cacc[f];
+        consumer_sync<kConsumers>();
+        for (int c4 = ctid; c4 < CW; c4 += kConsumers) {
+            float4 v = s_col[0][c4];
+#pragma unroll
+            for (int g = 1; g < 8 * RPW; ++g) {
+                const float4 u = s_col[g][c4];
+                v.x += u.x; v.y += u.y; v.z += u.z; v.w += u.w;
+            }
+            const int col = cur_tj * TC + c4 * 4;
+            if (col < p.n) {
+                if (col + 4 <= p.n) red_add4(p.out_c + col, v);
+                else {
+                    red_add(p.out_c + col, v.x);
+                    if (col + 1 < p.n) red_add(p.out_c + col + 1, v.y);
+                    if (col + 2 < p.n) red_add(p.out_c + col + 2, v.z);
                 }
             }
-            consumer_sync<kConsumers>();
         }
-        if (ctid < CT && col < p.n) {
-            if (col + 4 <= p.n) red_add4(p.out_c + col, v);
-            else {
-                red_add(p.out_c + col, v.x);
-                if (col + 1 < p.n) red_add(p.out_c + col + 1, v.y);
-                if (col + 2 < p.n) red_add(p.out_c + col + 2, v.z);
-            }
-        }
-        cacc = f4_zero();
+        consumer_sync<kConsumers>();
+#pragma unroll
+        for (int f = 0; f < FPL; ++f) cacc[f] = f4_zero();
     }
 
     // ---- consumers: one logical CTA from the staged tile
     __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         if (DO_ROW && by != cur_ti) { if (cur_ti >= 0) flush_row(ctid); cur_ti = by; }
         if (DO_COL && bx != cur_tj) { if (cur_tj >= 0) flush_col(ctid); cur_tj = bx; }
-        const int cg = ctid % CT, rg = ctid / CT;
-        const int col = bx * TC + cg * 4;
-        const int rowb = by * TR + rg;
-        if (col >= p.n) return;
-        float4 xv = f4_zero();
-        if (DO_ROW) {
-            if (col + 4 <= p.n) xv = ld_cached4(p.vc + col);
-            else {
-                xv.x = ld_cached(p.vc + col);
-                if (col + 1 < p.n) xv.y = ld_cached(p.vc + col + 1);
-                if (col + 2 < p.n) xv.z = ld_cached(p.vc + col + 2);
-            }
-        }
-        float rv[RPT];
-        if (DO_COL) {
+        const int warp = ctid >> 5, lane = ctid & 31, sub = lane / LPR, cl = lane % LPR;
+        const int col0 = bx * TC, row0 = by * TR;
+        float4 xv[FPL];
+        bool cok[FPL];
 #pragma unroll
-            for (int k = 0; k < RPT; ++k) {
-                int row = rowb + k * RG;
-                rv[k] = row < p.m ? ld_cached(p.vr + row) : 0.f;
+        for (int f = 0; f < FPL; ++f) {
+            const int col = col0 + tcol4(cl, f) * 4;
+            cok[f] = col < p.n;
+            xv[f] = f4_zero();
+            if (DO_ROW && cok[f]) {
+                if (col + 4 <= p.n) xv[f] = ld_cached4(p.vc + col);
+                else {
+                    xv[f].x = ld_cached(p.vc + col);
+                    if (col + 1 < p.n) xv[f].y = ld_cached(p.vc + col + 1);
+                    if (col + 2 < p.n) xv[f].z = ld_cached(p.vc + col + 2);
+                }
             }
         }
         const float4* tile = reinterpret_cast<const float4*>(stage);
-        const bool ragged = col + 4 > p.n;
 #pragma unroll
-        for (int k = 0; k < RPT; ++k) {
-            const int r = rg + k * RG;
-            if (rowb + k * RG >= p.m) break;
-            float4 a = tile[r * CT + cg];
-            if (ragged) {                                // lanes past n hold padding
-                if (col + 1 >= p.n) a.y = 0.f;
-                if (col + 2 >= p.n) a.z = 0.f;
-                a.w = 0.f;
-            }
-            if (DO_ROW) racc[k] += a.x * xv.x + a.y * xv.y + a.z * xv.z + a.w * xv.w;
-            if (DO_COL) {
-                cacc.x += a.x * rv[k]; cacc.y += a.y * rv[k];
-                cacc.z += a.z * rv[k]; cacc.w += a.w * rv[k];
+        for (int k = 0; k < NP; ++k) {
+            const int r = trow(warp, k, sub);
+            if (row0 + r >= p.m) continue;                 // never staged
+            const float rv = DO_COL ? ld_cached(p.vr + row0 + r) : 0.f;
+#pragma unroll
+            for (int f = 0; f < FPL; ++f) {
+                if (!cok[f]) continue;
+                float4 a = tile[r * CW + tcol4(cl, f)];
+                const int col = col0 + tcol4(cl, f) * 4;
+                if (col + 4 > p.n) {                         // lanes past n hold padding
+                    if (col + 1 >= p.n) a.y = 0.f;
+                    if (col + 2 >= p.n) a.z = 0.f;
+                    a.w = 0.f;
+                }
+                if (DO_ROW) racc[k] += a.x * xv[f].x + a.y * xv[f].y + a.z * xv[f].z + a.w * xv[f].w;
+                if (DO_COL) {
+                    cacc[f].x += a.x * rv; cacc[f].y += a.y * rv;
+                    cacc[f].z += a.z * rv; cacc[f].w += a.w * rv;
+                }
             }
         }
     }

@@ -56,6 +56,7 @@ struct SpmvBody {
     static constexpr int kStageBytes = 128;       // nothing staged: reads go straight to L1/L2
     static constexpr int kDefaultStages = 2;
     static constexpr int kDefaultBatch = 2;
+    static constexpr int kMinAgents = 5;
     using Params = SpmvParams;
     SpmvParams p;
     __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}

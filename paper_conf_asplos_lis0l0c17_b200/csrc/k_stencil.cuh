@@ -31,6 +31,24 @@ struct HaloTile {
                                                  int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
                                                  int32_t bypass) {
         const int32_t cols4 = (cols + 3) & ~3;   // last 16-byte chunk stays inside ld
+        if (bypass) {
+            // BPS: one bulk copy per staged row, L2 -> shared memory, no L1
+            // allocation.  Rows/columns outside the image are not copied (their
+            // staged values only ever feed border outputs, which are not computed
+            // from them).
+            const int32_t xs = x0 - 4 < 0 ? 0 : x0 - 4;
+            const int32_t xe = x0 + 36 < cols4 ? x0 + 36 : cols4;
+            const uint32_t bytes = xe > xs ? (uint32_t)(xe - xs) * 4u : 0u;
+            const int32_t ys = y0 - H < 0 ? 0 : y0 - H;
+            const int32_t ye = y0 + 32 + H < rows ? y0 + 32 + H : rows;
+            const int32_t nr = ye > ys ? ye - ys : 0;
+            stage_commit(full, lane, bytes * (uint32_t)nr);
+            if (bytes)
+                for (int r = lane; r < nr; r += 32)
+                    bulk_g2s(dst + ((ys + r - (y0 - H)) * ST_COLS + (xs - (x0 - 4))) * 4,
+                             src + (int64_t)(ys + r) * ld + xs, bytes, full);
+            return;
+        }
         // lanes 0..29 cover three staged rows (10 chunks each) per step
         const int r0 = lane / 10, cc = lane - r0 * 10;
         const int32_t gx = x0 - 4 + 4 * cc;
@@ -64,6 +82,7 @@ struct Jacobi5Body {
     static constexpr int kStageBytes = HaloTile<1>::kBytes;
     static constexpr int kDefaultStages = 3;
     static constexpr int kDefaultBatch = 4;
+    static constexpr int kMinAgents = 6;
     using Params = JacobiParams;
     JacobiParams p;
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
@@ -154,6 +173,7 @@ struct Conv2dBody {
     static constexpr int kStageBytes = HaloTile<R>::kBytes;
     static constexpr int kDefaultStages = 3;
     static constexpr int kDefaultBatch = 4;
+    static constexpr int kMinAgents = 6;
     using Params = ConvParams<R>;
     ConvParams<R> p;
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
