@@ -1,6 +1,7 @@
 // cc_mem.cuh -- memory-access helpers (sm_100a PTX).
 #pragma once
 #include <stdint.h>
+#include <cuda.h>            // CUtensorMap
 #include <cuda_runtime.h>
 
 namespace cc {

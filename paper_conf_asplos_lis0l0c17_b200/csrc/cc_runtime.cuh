@@ -128,6 +128,12 @@ __device__ __forceinline__ void cp_async_cg16(void* dst, const void* src, uint32
 __device__ __forceinline__ void cp_async_arrive(uint64_t* bar) {
     asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" :: "r"(smem_u32(bar)) : "memory");
 }
+// 2D TMA tile load (UTMALDG) of the box at (x, y) -- out-of-range elements are
+// zero-filled -- completion counted on `bar` (the box's full byte count).
+__device__ __forceinline__ void tma_load_2d(void* dst, const void* tmap, int32_t x, int32_t y, uint64_t* bar) {
+    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                 :: "r"(smem_u32(dst)), "l"(tmap), "r"(x), "r"(y), "r"(smem_u32(bar)) : "memory");
+}
 // named barrier among the consumer warps only (the producer warp never joins)
 template <int N>
 __device__ __forceinline__ void consumer_sync() {
@@ -297,9 +303,10 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             s_active = active;
         }
         // ---- producer ring
+        int st = 0;
+        uint32_t ph = 0;                                       // empty-barrier parity
         for (int32_t t = 0;; ++t) {
-            const int st = t % S;
-            if (t >= S) mbar_wait(&R.empty[st], ((t / S) - 1) & 1);
+            if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
             const int32_t v = producer_next(s, P, lane);
             if (lane == 0) R.slot[st] = v;
             if (v < 0) {
@@ -310,6 +317,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             int32_t lin, bx, by;
             lin_to_bxby(s, v, &lin, &bx, &by);
             body.produce(s, bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
+            if (++st == S) { st = 0; ph ^= 1u; }
         }
         // ---- the last agent out resets the workspace for the next launch.  Every
         // other agent's producer has consumed the results of all its atomics
@@ -324,9 +332,10 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         }
     } else {
         const int ctid = threadIdx.x - PRODUCER_THREADS;
-        for (int32_t t = 0;; ++t) {
-            const int st = t % S;
-            mbar_wait(&R.full[st], (t / S) & 1);
+        int st = 0;
+        uint32_t ph = 0;                                       // full-barrier parity
+        for (;;) {
+            mbar_wait(&R.full[st], ph);
             const int32_t v = R.slot[st];
             if (v < 0) break;
             int32_t lin, bx, by;
@@ -335,6 +344,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             if (ctid == 0) record(s, v, lin);
             __syncwarp();
             if (lane == 0) mbar_arrive(&R.empty[st]);
+            if (++st == S) { st = 0; ph ^= 1u; }
         }
         if (s_active) body.finish(ctid);
     }
@@ -367,13 +377,14 @@ __device__ __forceinline__ void one_shot(const Sched& s, Body& body, int32_t v, 
 // ---- kernels: one per (body, backend) ------------------------------------
 template <class Body>
 __global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS, Body::kMinAgents)
-k_agent(Sched s, typename Body::Params p) {
+k_agent(const __grid_constant__ Sched s, const __grid_constant__ typename Body::Params p) {
     Body body(p);
     agent_loop(s, body);
 }
 
 template <class Body>
-__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_default(Sched s, typename Body::Params p) {
+__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_default(const __grid_constant__ Sched s,
+                                                                             const __grid_constant__ typename Body::Params p) {
     Body body(p);
     const int32_t bx = blockIdx.x, by = blockIdx.y;
     one_shot(s, body, -1, by * s.g.gx + bx, bx, by);
@@ -382,7 +393,8 @@ __global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_default
 // Redirection-based clustering (Listing 4, Fig. 9): same number of CTAs as O;
 // CTA u runs v = rd_redirect(u).
 template <class Body>
-__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_redirect(Sched s, typename Body::Params p) {
+__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS) k_redirect(const __grid_constant__ Sched s,
+                                                                              const __grid_constant__ typename Body::Params p) {
     Body body(p);
     const int32_t v = rd_redirect(s.g, (int32_t)blockIdx.x);
     int32_t lin, bx, by;

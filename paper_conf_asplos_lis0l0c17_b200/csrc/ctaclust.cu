@@ -266,7 +266,7 @@ extern "C" cc_status cc_launch_opts_default(cc_launch_opts* o) {
     return CC_OK;
 }
 
-#define CC_TRY(x) do { cc_status s_ = (x); if (s_ != CC_OK) return s_; } while (0)
+#define CC_TRY(...) do { cc_status s_ = (__VA_ARGS__); if (s_ != CC_OK) return s_; } while (0)
 
 static inline int32_t cdiv(int64_t a, int64_t b) { return (int32_t)((a + b - 1) / b); }
 static inline bool al16(const void* p) { return ((uintptr_t)p & 15) == 0; }
@@ -450,12 +450,13 @@ static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
     return fn;
 }
 
-static cc_status make_tmap(CUtensorMap* m, const float* base, int32_t rows, int32_t cols, int64_t ld, int box_rows) {
+static cc_status make_tmap(CUtensorMap* m, const float* base, int32_t rows, int32_t cols, int64_t ld, int box_cols,
+                           int box_rows) {
     auto enc = tmap_encoder();
     if (!enc) return fail(CC_ERR_UNSUPPORTED, "cuTensorMapEncodeTiled unavailable");
     cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
     cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
-    cuuint32_t box[2] = {(cuuint32_t)TBC_COLS, (cuuint32_t)box_rows};
+    cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
     cuuint32_t estr[2] = {1, 1};
     CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)base, dims, strides, box, estr,
                      CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -473,8 +474,8 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     const int gy_pad = (g.gy + C - 1) / C * C;
     if (gy_pad > 65535) return fail(CC_ERR_UNSUPPORTED, "tbcluster: gy %d too large", g.gy);
     CUtensorMap m_rows, m_halo;
-    CC_TRY(make_tmap(&m_rows, prm.in, prm.rows, prm.cols, prm.ld, 32));
-    CC_TRY(make_tmap(&m_halo, prm.in, prm.rows, prm.cols, prm.ld, TBC_HALO));
+    CC_TRY(make_tmap(&m_rows, prm.in, prm.rows, prm.cols, prm.ld, TBC_COLS, 32));
+    CC_TRY(make_tmap(&m_halo, prm.in, prm.rows, prm.cols, prm.ld, TBC_COLS, TBC_HALO));
     Sched s{};
     s.g = g;
     s.census = c.o->d_census;
@@ -495,6 +496,15 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     cfg.numAttrs = 1;
     CC_CUDA(cudaLaunchKernelEx(&cfg, k_conv_tbc<R>, m_rows, m_halo, s, prm, (int32_t)C));
     if (c.nl) ++*c.nl;
+    return CC_OK;
+}
+
+template <int TR, int TC>
+static cc_status gemv_params(GemvParams* P, const float* A, int64_t lda, int32_t m, int32_t n, const float* vc,
+                             const float* vr, float* out_r, float* out_c) {
+    memset(P, 0, sizeof *P);
+    P->A = A; P->lda = lda; P->m = m; P->n = n; P->vc = vc; P->vr = vr; P->out_r = out_r; P->out_c = out_c;
+    if (m > 0 && n > 0) CC_TRY(make_tmap(&P->tmap, A, m, n, lda, TC, TR));
     return CC_OK;
 }
 
@@ -537,7 +547,9 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         auto* x = (const cc_matvec_args*)a;
         CC_TRY(check_mat(x->A, x->lda, x->m, x->n));
         CC_TRY(check_vec(x->x, x->n, "x")); CC_TRY(check_vec(x->y, x->m, "y"));
-        s = launch_body<MatvecB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->x, nullptr, x->y, nullptr});
+        GemvParams gp;
+        CC_TRY(gemv_params<32, 32>(&gp, x->A, x->lda, x->m, x->n, x->x, nullptr, x->y, nullptr));
+        s = launch_body<MatvecB>(c, gp);
         break;
     }
     case CC_K_ATAX: {
@@ -546,8 +558,11 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         CC_TRY(check_vec(x->x, x->n, "x")); CC_TRY(check_vec(x->tmp, x->m, "tmp")); CC_TRY(check_vec(x->y, x->n, "y"));
         if (x->m) CC_CUDA(cudaMemsetAsync(x->tmp, 0, sizeof(float) * x->m, st));
         if (x->n) CC_CUDA(cudaMemsetAsync(x->y, 0, sizeof(float) * x->n, st));
-        s = launch_body<RowB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->x, nullptr, x->tmp, nullptr});
-        if (s == CC_OK) s = launch_body<ColB>(c, GemvParams{x->A, x->lda, x->m, x->n, nullptr, x->tmp, nullptr, x->y});
+        GemvParams g1, g2;
+        CC_TRY(gemv_params<32, 256>(&g1, x->A, x->lda, x->m, x->n, x->x, nullptr, x->tmp, nullptr));
+        CC_TRY(gemv_params<32, 256>(&g2, x->A, x->lda, x->m, x->n, nullptr, x->tmp, nullptr, x->y));
+        s = launch_body<RowB>(c, g1);
+        if (s == CC_OK) s = launch_body<ColB>(c, g2);
         break;
     }
     case CC_K_BICG: {
@@ -557,7 +572,9 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         CC_TRY(check_vec(x->q, x->m, "q")); CC_TRY(check_vec(x->s, x->n, "s"));
         if (x->m) CC_CUDA(cudaMemsetAsync(x->q, 0, sizeof(float) * x->m, st));
         if (x->n) CC_CUDA(cudaMemsetAsync(x->s, 0, sizeof(float) * x->n, st));
-        s = launch_body<BothB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->p, x->r, x->q, x->s});
+        GemvParams gp;
+        CC_TRY(gemv_params<32, 256>(&gp, x->A, x->lda, x->m, x->n, x->p, x->r, x->q, x->s));
+        s = launch_body<BothB>(c, gp);
         break;
     }
     case CC_K_MVT: {
@@ -565,7 +582,9 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         CC_TRY(check_mat(x->A, x->lda, x->m, x->n));
         CC_TRY(check_vec(x->y1, x->n, "y1")); CC_TRY(check_vec(x->y2, x->m, "y2"));
         CC_TRY(check_vec(x->x1, x->m, "x1")); CC_TRY(check_vec(x->x2, x->n, "x2"));
-        s = launch_body<BothB>(c, GemvParams{x->A, x->lda, x->m, x->n, x->y1, x->y2, x->x1, x->x2});
+        GemvParams gp;
+        CC_TRY(gemv_params<32, 256>(&gp, x->A, x->lda, x->m, x->n, x->y1, x->y2, x->x1, x->x2));
+        s = launch_body<BothB>(c, gp);
         break;
     }
     case CC_K_JACOBI5: {
@@ -576,7 +595,11 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         float* src = x->a;
         float* dst = x->b;
         for (int it = 0; it < x->iters && s == CC_OK; ++it) {
-            s = launch_body<Jacobi5Body>(c, JacobiParams{src, dst, x->ld, x->rows, x->cols});
+            JacobiParams jp;
+            memset(&jp, 0, sizeof jp);
+            jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
+            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
+            s = launch_body<Jacobi5Body>(c, jp);
             std::swap(src, dst);
         }
         if (x->result_is_b) *x->result_is_b = (x->iters & 1) ? 1 : 0;
@@ -588,13 +611,19 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         CC_TRY(check_mat(x->out, x->ld, x->rows, x->cols));
         if (!x->w) return fail(CC_ERR_INVALID_ARG, "null filter");
         if (x->R == 1) {
-            ConvParams<1> cp{x->in, x->out, x->ld, x->rows, x->cols, {}};
+            ConvParams<1> cp;
+            memset(&cp, 0, sizeof cp);
+            cp.in = x->in; cp.out = x->out; cp.ld = x->ld; cp.rows = x->rows; cp.cols = x->cols;
             memcpy(cp.w, x->w, sizeof cp.w);
+            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 34));
             s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<1>(c, cp)
                                                    : launch_body<Conv2dBody<1>>(c, cp);
         } else if (x->R == 3) {
-            ConvParams<3> cp{x->in, x->out, x->ld, x->rows, x->cols, {}};
+            ConvParams<3> cp;
+            memset(&cp, 0, sizeof cp);
+            cp.in = x->in; cp.out = x->out; cp.ld = x->ld; cp.rows = x->rows; cp.cols = x->cols;
             memcpy(cp.w, x->w, sizeof cp.w);
+            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 38));
             s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<3>(c, cp)
                                                    : launch_body<Conv2dBody<3>>(c, cp);
         } else {

@@ -8,9 +8,9 @@
 // This is the cache-line-related class of Table 2 (ATX/MVT/BC).
 //
 // Data movement:
-//   * the A tile (streamed, no reuse) is staged by the producer warp with one
-//     bulk async copy per tile row straight into shared memory (UBLKCP; it
-//     never touches L1, the B200 form of the paper's bypass §4.3(II));
+//   * the A tile (streamed, no reuse) is staged by the producer warp with ONE
+//     2D TMA load straight into shared memory (UTMALDG; it never touches L1,
+//     the B200 form of the paper's bypass §4.3(II); ragged edges zero-filled);
 //   * the vc / vr slices -- the inter-CTA shared data -- are read by the
 //     consumers with L1-allocating loads, so tasks of one SM that share bx (vc)
 //     or by (vr) hit L1;
@@ -32,6 +32,7 @@
 namespace cc {
 
 struct GemvParams {
+    CUtensorMap tmap;  // A as an n x m fp32 tensor, box TC x TR (filled by the launcher)
     const float* A; int64_t lda; int32_t m, n;
     const float* vc;   // ROW-product input, n entries
     const float* vr;   // COL-product input, m entries
@@ -54,7 +55,7 @@ struct GemvBody {
     static_assert(TC % 4 == 0 && CW % LPR == 0 && 32 % LPR == 0 && TR % (8 * RPW) == 0 && NP >= 1, "tile shape");
     using Params = GemvParams;
 
-    GemvParams p;
+    const GemvParams& p;   // the __grid_constant__ kernel parameter (TMA needs its address)
     int32_t cur_ti, cur_tj;
     float racc[NP];
     float4 cacc[FPL];
@@ -69,16 +70,10 @@ struct GemvBody {
     __device__ __forceinline__ static int trow(int warp, int k, int sub) { return (k * RPW + sub) * 8 + warp; }
     __device__ __forceinline__ static int tcol4(int cl, int f) { return f * LPR + cl; }
 
-    // ---- producer: one bulk copy per tile row (rows past m are not copied)
+    // ---- producer: one 2D TMA load of the whole tile (OOB rows/cols zero-filled)
     __device__ __forceinline__ void produce(const Sched&, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        const int col0 = bx * TC;
-        const int cols = p.n - col0 < TC ? p.n - col0 : TC;
-        const uint32_t bytes = (uint32_t)((cols * 4 + 15) & ~15);    // within lda (lda % 4 == 0)
-        const int row0 = by * TR;
-        const int nrows = p.m - row0 < TR ? p.m - row0 : TR;
-        stage_commit(full, lane, bytes * (uint32_t)nrows);
-        for (int r = lane; r < nrows; r += 32)
-            bulk_g2s(stage + r * (TC * 4), p.A + (int64_t)(row0 + r) * p.lda + col0, bytes, full);
+        stage_commit(full, lane, (uint32_t)kStageBytes);
+        if (lane == 0) tma_load_2d(stage, &p.tmap, bx * TC, by * TR, full);
     }
 
     // ---- ROW flush: warp-level sum over the LPR lanes of each row, one RED per row

@@ -58,7 +58,7 @@ struct SpmvBody {
     static constexpr int kDefaultBatch = 2;
     static constexpr int kMinAgents = 5;
     using Params = SpmvParams;
-    SpmvParams p;
+    const SpmvParams& p;
     __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) {

@@ -6,8 +6,9 @@
 // (the cache-line/algorithm-related classes).
 //
 // The producer warp stages the tile plus halo -- rows y0-H .. y0+31+H, columns
-// x0-4 .. x0+35 (10 aligned 16-byte chunks per row) -- into shared memory with
-// cp.async.ca, which also allocates every line in L1.  A neighbouring tile
+// x0-4 .. x0+35 (10 aligned 16-byte chunks per row) -- into shared memory,
+// either with one 2D TMA load (bypass = 1: L2 -> smem, L1 untouched) or with
+// cp.async.ca chunks (bypass = 0), which also allocate every line in L1.  A neighbouring tile
 // staged soon after on the same SM therefore finds its halo (and the shared
 // 16-byte edge chunks) in L1 instead of L2: clustering neighbouring tiles onto
 // one SM (TILE order, Fig. 7) turns that halo traffic into L1 hits.  Chunks
@@ -29,24 +30,13 @@ struct HaloTile {
     // warp-collective: stage rows y0-H.., columns x0-4.. of `src`.
     __device__ __forceinline__ static void stage(const float* src, int64_t ld, int32_t rows, int32_t cols,
                                                  int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
-                                                 int32_t bypass) {
+                                                 int32_t bypass, const CUtensorMap* tmap) {
         const int32_t cols4 = (cols + 3) & ~3;   // last 16-byte chunk stays inside ld
         if (bypass) {
-            // BPS: one bulk copy per staged row, L2 -> shared memory, no L1
-            // allocation.  Rows/columns outside the image are not copied (their
-            // staged values only ever feed border outputs, which are not computed
-            // from them).
-            const int32_t xs = x0 - 4 < 0 ? 0 : x0 - 4;
-            const int32_t xe = x0 + 36 < cols4 ? x0 + 36 : cols4;
-            const uint32_t bytes = xe > xs ? (uint32_t)(xe - xs) * 4u : 0u;
-            const int32_t ys = y0 - H < 0 ? 0 : y0 - H;
-            const int32_t ye = y0 + 32 + H < rows ? y0 + 32 + H : rows;
-            const int32_t nr = ye > ys ? ye - ys : 0;
-            stage_commit(full, lane, bytes * (uint32_t)nr);
-            if (bytes)
-                for (int r = lane; r < nr; r += 32)
-                    bulk_g2s(dst + ((ys + r - (y0 - H)) * ST_COLS + (xs - (x0 - 4))) * 4,
-                             src + (int64_t)(ys + r) * ld + xs, bytes, full);
+            // BPS: one 2D TMA load of the (32+2H) x 40 box, L2 -> shared memory,
+            // no L1 allocation; the image border is zero-filled by the TMA unit.
+            stage_commit(full, lane, (uint32_t)(kRows * ST_COLS * 4));
+            if (lane == 0) tma_load_2d(dst, tmap, x0 - 4, y0 - H, full);
             return;
         }
         // lanes 0..29 cover three staged rows (10 chunks each) per step
@@ -75,7 +65,7 @@ struct HaloTile {
 // fp32, summed in that fixed order with no contraction, so the sweep is
 // bit-reproducible against oracle_jacobi5_f32.
 // ---------------------------------------------------------------------------
-struct JacobiParams { const float* a; float* b; int64_t ld; int32_t rows, cols; };
+struct JacobiParams { CUtensorMap tmap; const float* a; float* b; int64_t ld; int32_t rows, cols; };
 
 struct Jacobi5Body {
     static constexpr int kConsumers = 256;
@@ -84,11 +74,11 @@ struct Jacobi5Body {
     static constexpr int kDefaultBatch = 4;
     static constexpr int kMinAgents = 6;
     using Params = JacobiParams;
-    JacobiParams p;
+    const JacobiParams& p;   // __grid_constant__ kernel parameter
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass);
+        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass, &p.tmap);
     }
 
     __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
@@ -129,7 +119,7 @@ struct Jacobi5Body {
 // The filter lives in the kernel parameter bank (constant-bank operands).
 // ---------------------------------------------------------------------------
 template <int R>
-struct ConvParams { const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
+struct ConvParams { CUtensorMap tmap; const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
 
 template <int R>
 __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const float* rows_base,
@@ -175,11 +165,11 @@ struct Conv2dBody {
     static constexpr int kDefaultBatch = 4;
     static constexpr int kMinAgents = 6;
     using Params = ConvParams<R>;
-    ConvParams<R> p;
+    const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass);
+        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass, &p.tmap);
     }
     __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         conv_tile_compute<R>(p, reinterpret_cast<const float*>(stage), bx, by, ctid);
