@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--active-agents", type=int, default=0)
     ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--batch", type=int, default=0)
+    ap.add_argument("--staging", default="default", choices=["default", "tma", "direct"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--suite", default=None, help="also run every BASELINE config, write JSON here")
@@ -187,8 +188,9 @@ def main():
     x1, x2 = x1_0.clone(), x2_0.clone() if rank == 0 else torch.zeros(n, device=dev)
     torch.cuda.synchronize()
 
-    def run_step(backend, order, ev=None, count=None):
-        kw = dict(backend=backend, active_agents=a.active_agents, stages=a.stages, batch=a.batch)
+    def run_step(backend, order, ev=None, count=None, staging=None):
+        kw = dict(backend=backend, active_agents=a.active_agents, stages=a.stages, batch=a.batch,
+                  staging=a.staging if staging is None else staging)
         nl = 0
         if ev is not None: ev[0].record(stream)
         pl = ops.plan_for("atax", cc.atax_args(A, x, tmp, y), order)
@@ -204,9 +206,9 @@ def main():
         if count is not None:
             count[0] += nl
 
-    def timed(backend, order, steps, per_kernel=False):
+    def timed(backend, order, steps, per_kernel=False, staging=None):
         for _ in range(max(3, a.warmup)):
-            run_step(backend, order)
+            run_step(backend, order, staging=staging)
         evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(steps)] if per_kernel else None
         t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         if world > 1:
@@ -215,7 +217,7 @@ def main():
         count = [0]
         t0.record(stream)
         for k in range(steps):
-            run_step(backend, order, evs[k] if evs else None, count)
+            run_step(backend, order, evs[k] if evs else None, count, staging)
         t1.record(stream)
         torch.cuda.synchronize()
         ms = t0.elapsed_time(t1)
@@ -234,7 +236,12 @@ def main():
     clocks = Clocks(local)
     ms_clu, per_clu, launches = timed(a.backend, a.order, a.steps, per_kernel=True)
     clk = clocks.stop()
-    ms_def, per_def, _ = timed("default", "row", a.steps, per_kernel=True)
+    # default hardware CTA order: the same TMA-staged body, and the plain
+    # direct-load kernel; the faster one is the comparator
+    ms_def_tma, per_def_tma, _ = timed("default", "row", a.steps, per_kernel=True, staging="tma")
+    ms_def_dir, per_def_dir, _ = timed("default", "row", a.steps, per_kernel=True, staging="direct")
+    ms_def, per_def, def_kind = ((ms_def_tma, per_def_tma, "tma-staged") if ms_def_tma <= ms_def_dir
+                                 else (ms_def_dir, per_def_dir, "direct-load"))
     ms_id, _, _ = timed("identity", "row", max(20, a.steps // 5))
     bytes_all = step_bytes(n, n)              # whole job: every rank's rows together
     value = bytes_all["total"] / (ms_clu * 1e-3) / 1e9
@@ -301,10 +308,12 @@ def main():
                 "data": "synthetic (counter-hash U[0,1), generated on device)",
                 "config": {"workload": f"ATAX+BICG+MVT fp32 n={n} (BASELINE config 2)",
                            "backend": a.backend, "order": a.order, "active_agents": a.active_agents or "max",
-                           "stages": a.stages or "default", "batch": a.batch or "default", "tile": "32x256", "parallelism": f"row-shard x{world}",
+                           "stages": a.stages or "default", "batch": a.batch or "default", "staging": a.staging,
+                           "tile": "32x256", "parallelism": f"row-shard x{world}",
                            "l2": "inputs (1 GiB) larger than L2 (126 MB); no flush"},
                 "speedup_vs_default": round(ms_def / ms_clu, 4),
-                "ms_per_step_default": round(ms_def, 4),
+                "ms_per_step_default": round(ms_def, 4), "default_kind": def_kind,
+                "ms_per_step_default_tma": round(ms_def_tma, 4), "ms_per_step_default_direct": round(ms_def_dir, 4),
                 "ms_per_step_identity": round(ms_id, 4),
                 "per_kernel_ms": {k: round(v, 4) for k, v in per_clu.items()},
                 "per_kernel_ms_default": {k: round(v, 4) for k, v in per_def.items()},

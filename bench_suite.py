@@ -1,12 +1,15 @@
 #!/usr/bin/env python
 """bench_suite.py -- every BASELINE config, clustered vs default CTA order.
 
-For each reuse kernel this times the default hardware order ("BSL"),
-the agent runtime with the config's clustering ("CLU"), throttled agents
-("CLU+TOT"), the staging-depth variants, the persistence-only control (identity
-order) and redirection ("RD"), and reports ms, algorithmic GB/s (fraction of
-the measured HBM copy peak) and speedup over default.  L2-sector reductions
-come from the ncu captures (scripts/ncu_suite.sh -> profiles/).
+For each reuse kernel this times the default hardware order ("BSL") --
+both with the library's TMA-staged body and with the plain direct-load body,
+the faster of the two being the comparator -- against the agent runtime with
+the config's clustering ("CLU"), throttled agents ("CLU+TOT"), staging
+variants (TMA = L1-bypassing "BPS", L1-allocating cp.async, direct loads), ring
+depth, the persistence-only control (identity order) and redirection ("RD").
+Reports ms, algorithmic GB/s (fraction of the measured HBM copy peak) and the
+speedup over the best default.  L2-sector reductions come from the ncu
+captures (scripts/ncu_suite.sh -> profiles/).
 
     python bench_suite.py out.json [--only matvec,atax,jacobi,conv,spmv] [--quick]
 """
@@ -46,13 +49,43 @@ def time_ms(fn, reps, warm=3, inner=1):
     return out[len(out) // 2]
 
 
-def _row(name, ms, nbytes, base_ms, extra=None):
-    gbs = nbytes / (ms * 1e-3) / 1e9
-    d = {"variant": name, "ms": round(ms, 5), "GBps": round(gbs, 1), "frac_hbm": round(gbs / _peak(), 4),
-         "speedup_vs_default": round(base_ms / ms, 4) if base_ms else 1.0}
-    if extra:
-        d.update(extra)
-    return d
+def measure(variants, fn, reps, nbytes, extra=None, warm=3, inner=1):
+    rows = []
+    for name, kw in variants:
+        ms = time_ms(lambda: fn(kw), reps, warm=warm, inner=inner)
+        gbs = nbytes / (ms * 1e-3) / 1e9
+        d = {"variant": name, "ms": round(ms, 5), "GBps": round(gbs, 1), "frac_hbm": round(gbs / _peak(), 4)}
+        if extra:
+            d.update(extra(ms))
+        rows.append(d)
+    best_def = min(r["ms"] for r in rows if r["variant"].startswith("default"))
+    for r in rows:
+        r["speedup_vs_best_default"] = round(best_def / r["ms"], 4)
+    return {"bytes": nbytes, "best_default_ms": best_def, "rows": rows}
+
+
+def variants_for(order, tile=(1, 1), stencil=False):
+    o = dict(order=order, tile=tile) if order == "tile" else dict(order=order)
+    tag = f"{order}{tile[0]}x{tile[1]}" if order == "tile" else order
+    v = [("default", dict(backend="default")),
+         ("default-direct", dict(backend="default", staging="direct")),
+         (f"agent-{tag}", dict(backend="agent", **o)),
+         (f"agent-{tag}-direct", dict(backend="agent", staging="direct", **o)),
+         (f"agent-{tag}-tot1", dict(backend="agent", active_agents=1, **o)),
+         (f"agent-{tag}-tot2", dict(backend="agent", active_agents=2, **o)),
+         (f"agent-{tag}-s2", dict(backend="agent", stages=2, **o)),
+         ("identity", dict(backend="identity")),
+         ("identity-direct", dict(backend="identity", staging="direct")),
+         (f"redirect-{tag}", dict(backend="redirect", **o))]
+    if stencil:
+        v += [("default-l1", dict(backend="default", staging="l1")),
+              (f"agent-{tag}-l1", dict(backend="agent", staging="l1", **o)),
+              ("agent-row", dict(backend="agent", order="row")),
+              ("agent-col", dict(backend="agent", order="col")),
+              ("agent-tile4x4", dict(backend="agent", order="tile", tile=(4, 4))),
+              ("agent-row-l1", dict(backend="agent", order="row", staging="l1")),
+              (f"agent-{tag}-s6", dict(backend="agent", stages=6, **o))]
+    return v
 
 
 def suite_matvec(quick):
@@ -62,18 +95,10 @@ def suite_matvec(quick):
     A = synth.matrix(1, n, n, backend="torch", device="cuda")
     x = synth.uniform(2, n, backend="torch", device="cuda")
     y = torch.zeros(n, device="cuda")
-    nbytes = 4 * n * n + 8 * n
-    variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
-                ("agent-col", dict(backend="agent", order="col")),
-                ("agent-row-tot1", dict(backend="agent", order="row", active_agents=1)),
-                ("agent-row-tot2", dict(backend="agent", order="row", active_agents=2)),
-                ("identity", dict(backend="identity")), ("redirect-row", dict(backend="redirect", order="row"))]
-    rows, base = [], None
-    for name, kw in variants:
-        ms = time_ms(lambda: ops.matvec(A, x, y, **kw), 20 if quick else 50, inner=50)
-        base = ms if base is None else base
-        rows.append(_row(name, ms, nbytes, base))
-    return {"config": "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident", "bytes": nbytes, "rows": rows}
+    v = variants_for("row") + [("agent-col", dict(backend="agent", order="col"))]
+    r = measure(v, lambda kw: ops.matvec(A, x, y, **kw), 20 if quick else 50, 4 * n * n + 8 * n, inner=50)
+    r["config"] = "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident"
+    return r
 
 
 def suite_atax(quick):
@@ -90,21 +115,9 @@ def suite_atax(quick):
         "bicg": (lambda kw: ops.bicg(A, p, r, out=(q, s), **kw), Ab + 16 * n),
         "mvt": (lambda kw: ops.mvt(A, y1, y2, x1, x2, **kw), Ab + 24 * n),
     }
-    variants = [("default", dict(backend="default")), ("agent-col", dict(backend="agent", order="col")),
-                ("agent-row", dict(backend="agent", order="row")),
-                ("agent-col-tot1", dict(backend="agent", order="col", active_agents=1)),
-                ("agent-col-tot2", dict(backend="agent", order="col", active_agents=2)),
-                ("agent-col-s2", dict(backend="agent", order="col", stages=2)),
-                ("agent-col-s6", dict(backend="agent", order="col", stages=6)),
-                ("identity", dict(backend="identity")), ("redirect-col", dict(backend="redirect", order="col"))]
-    out = {}
-    for kname, (fn, nbytes) in kernels.items():
-        rows, base = [], None
-        for name, kw in variants:
-            ms = time_ms(lambda: fn(kw), 5 if quick else 15)
-            base = ms if base is None else base
-            rows.append(_row(name, ms, nbytes, base))
-        out[kname] = {"bytes": nbytes, "rows": rows}
+    variants = variants_for("col") + [("agent-row", dict(backend="agent", order="row")),
+                                      ("agent-col-s3", dict(backend="agent", order="col", stages=3))]
+    out = {k: measure(variants, fn, 5 if quick else 15, nb) for k, (fn, nb) in kernels.items()}
     return {"config": "PolyBench ATAX/BICG/MVT fp32 n=16384, 32x256 tiles (64x512 grid)", "kernels": out}
 
 
@@ -114,28 +127,13 @@ def suite_jacobi(quick):
     N, T = 16384, (20 if quick else 100)
     a = synth.matrix(4, N, N, backend="torch", device="cuda")
     b = torch.empty_like(a)
-    nbytes = 8 * N * N * T
-    variants = [("default", dict(backend="default")), ("agent-tile8x8", dict(backend="agent", order="tile", tile=(8, 8))),
-                ("agent-tile4x4", dict(backend="agent", order="tile", tile=(4, 4))),
-                ("agent-tile16x16", dict(backend="agent", order="tile", tile=(16, 16))),
-                ("agent-col", dict(backend="agent", order="col")), ("agent-row", dict(backend="agent", order="row")),
-                ("agent-tile8x8-tot4", dict(backend="agent", order="tile", tile=(8, 8), active_agents=4)),
-                ("agent-tile8x8-bps", dict(backend="agent", order="tile", tile=(8, 8), bypass=1)),
-                ("agent-row-bps", dict(backend="agent", order="row", bypass=1)),
-                ("agent-tile8x8-s2", dict(backend="agent", order="tile", tile=(8, 8), stages=2)),
-                ("agent-tile8x8-s5", dict(backend="agent", order="tile", tile=(8, 8), stages=5)),
-                ("default-bps", dict(backend="default", bypass=1)),
-                ("identity", dict(backend="identity"))]
-    rows, base = [], None
-    for name, kw in variants:
-        ms = time_ms(lambda: ops.jacobi5(a, b, T, **kw), 3, warm=1)
-        base = ms if base is None else base
-        rows.append(_row(name, ms, nbytes, base, {"ms_per_sweep": round(ms / T, 5)}))
-    return {"config": f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)", "bytes": nbytes, "rows": rows}
+    r = measure(variants_for("tile", (8, 8), stencil=True), lambda kw: ops.jacobi5(a, b, T, **kw), 3, 8 * N * N * T,
+                extra=lambda ms: {"ms_per_sweep": round(ms / T, 5)}, warm=1)
+    r["config"] = f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)"
+    return r
 
 
 def suite_conv(quick):
-    import numpy as np
     import torch
     from paper_conf_asplos_lis0l0c17_b200 import ops, synth
     N = 8192
@@ -145,24 +143,15 @@ def suite_conv(quick):
     for R in (1, 3):
         w = synth.uniform(6, (2 * R + 1) ** 2).reshape(2 * R + 1, 2 * R + 1)
         w = w / w.sum()
-        nbytes = 8 * N * N
         flops = 2 * (2 * R + 1) ** 2 * (N - 2 * R) ** 2
-        variants = [("default", dict(backend="default")),
-                    ("agent-tile8x8", dict(backend="agent", order="tile", tile=(8, 8))),
-                    ("agent-col", dict(backend="agent", order="col")),
-                    ("agent-tile8x8-bps", dict(backend="agent", order="tile", tile=(8, 8), bypass=1)),
-                    ("agent-col-bps", dict(backend="agent", order="col", bypass=1)),
-                    ("default-bps", dict(backend="default", bypass=1)),
-                    ("tbcluster-2", dict(backend="tbcluster", cluster_size=2)),
-                    ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
-                    ("tbcluster-8", dict(backend="tbcluster", cluster_size=8)),
-                    ("identity", dict(backend="identity"))]
-        rows, base = [], None
-        for name, kw in variants:
-            ms = time_ms(lambda: ops.conv2d(img, w, out=out, **kw), 5 if quick else 20)
-            base = ms if base is None else base
-            rows.append(_row(name, ms, nbytes, base, {"TFLOPs": round(flops / (ms * 1e-3) / 1e12, 2)}))
-        res[f"{2 * R + 1}x{2 * R + 1}"] = {"bytes": nbytes, "flops": flops, "rows": rows}
+        v = variants_for("tile", (8, 8), stencil=True) + [
+            ("tbcluster-2", dict(backend="tbcluster", cluster_size=2)),
+            ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
+            ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))]
+        res[f"{2 * R + 1}x{2 * R + 1}"] = measure(
+            v, lambda kw: ops.conv2d(img, w, out=out, **kw), 5 if quick else 20, 8 * N * N,
+            extra=lambda ms: {"TFLOPs": round(flops / (ms * 1e-3) / 1e12, 2)})
+        res[f"{2 * R + 1}x{2 * R + 1}"]["flops"] = flops
     return {"config": f"2D conv fp32 {N}x{N}, 32x32 tiles (256x256 grid)", "filters": res}
 
 
@@ -179,20 +168,16 @@ def suite_spmv(quick):
     x = synth.uniform(9, rows_n, backend="torch", device="cuda")
     Am = ops.SpmvMatrix(rp, col, val)
     y = torch.empty(rows_n, device="cuda")
-    nbytes = 8 * nnz + 4 * (rows_n + 1) + 8 * rows_n
     variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
                 ("agent-row-tot1", dict(backend="agent", order="row", active_agents=1)),
                 ("agent-row-tot2", dict(backend="agent", order="row", active_agents=2)),
                 ("agent-row-tot4", dict(backend="agent", order="row", active_agents=4)),
-                ("agent-row-s4b8", dict(backend="agent", order="row", stages=4, batch=8)),
-                ("identity", dict(backend="identity"))]
-    rows, base = [], None
-    for name, kw in variants:
-        ms = time_ms(lambda: ops.spmv(Am, x, y, **kw), 5 if quick else 20)
-        base = ms if base is None else base
-        rows.append(_row(name, ms, nbytes, base))
-    return {"config": f"CSR SpMV fp32 R-MAT scale {scale} ef 16: {rows_n} rows, {nnz} nnz (gen {gen_s:.1f}s)",
-            "bytes": nbytes, "rows": rows}
+                ("agent-row-b8", dict(backend="agent", order="row", batch=8)),
+                ("identity", dict(backend="identity")), ("redirect-row", dict(backend="redirect", order="row"))]
+    r = measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 5 if quick else 20,
+                8 * nnz + 4 * (rows_n + 1) + 8 * rows_n)
+    r["config"] = f"CSR SpMV fp32 R-MAT scale {scale} ef 16: {rows_n} rows, {nnz} nnz (gen {gen_s:.1f}s)"
+    return r
 
 
 SUITES = {"matvec": suite_matvec, "atax": suite_atax, "jacobi": suite_jacobi, "conv": suite_conv, "spmv": suite_spmv}
@@ -215,6 +200,20 @@ def run(path, only=None, quick=False):
     return res
 
 
+def table(path):
+    d = json.load(open(path))
+    lines = []
+    for k, v in d.items():
+        if not isinstance(v, dict):
+            continue
+        groups = {k: v} if "rows" in v else {f"{k}/{kk}": vv for sub in ("kernels", "filters") for kk, vv in v.get(sub, {}).items()}
+        for g, vv in groups.items():
+            lines.append(f"== {g}  {v.get('config', '')}")
+            for r in vv.get("rows", []):
+                lines.append(f"   {r['variant']:26s} {r['ms']:10.4f} ms {r['GBps']:8.1f} GB/s  frac {r['frac_hbm']:.3f}  x{r['speedup_vs_best_default']:.3f}")
+    return "\n".join(lines)
+
+
 if __name__ == "__main__":
     import argparse
     ap = argparse.ArgumentParser()
@@ -223,4 +222,4 @@ if __name__ == "__main__":
     ap.add_argument("--quick", action="store_true")
     a = ap.parse_args()
     run(a.out, a.only.split(",") if a.only else None, a.quick)
-    print(open(a.out).read())
+    print(table(a.out))

@@ -121,6 +121,8 @@ typedef enum {
                                       Eq. 8 + Eq. 7; relies on RR dispatch)    */
 } cc_backend;
 
+typedef enum { CC_STAGING_DEFAULT = 0, CC_STAGING_TMA = 1, CC_STAGING_L1 = 2, CC_STAGING_DIRECT = 3 } cc_staging;
+
 typedef struct {
     int32_t backend;        /* cc_backend                                               */
     int32_t active_agents;  /* agents per SM that work (throttling, §4.3(I));
@@ -132,9 +134,15 @@ typedef struct {
                                B200 form of "prefetch the next CTA" (§4.3(III),
                                Listing 5 l.34-37); 0 => the kernel's default, 1..8   */
     int32_t batch;          /* logical CTAs claimed per queue atomic; 0 => default   */
-    int32_t bypass;         /* cache bypassing "BPS" (§4.3(II)): 1 => the
-                               staged tile loads skip L1 (cp.async.cg); 0 => they
-                               allocate in L1 so neighbouring tasks can hit them     */
+    int32_t staging;        /* how a task's input tile reaches the body (cc_staging):
+                               0 default (= TMA), 1 TMA: one 2D tensor load per tile,
+                               L2 -> smem, L1 bypassed (the B200 form of "BPS",
+                               §4.3(II)); 2 cp.async.ca: 16-byte copies
+                               that also allocate in L1, so neighbouring tasks on the
+                               same SM hit the shared halo (the paper's L1 reuse;
+                               stencils only); 3 direct: no producer staging, the
+                               consumers load through L1 themselves (the plain
+                               kernel form).  SpMV always loads directly.            */
     int32_t steal;          /* 1 (default) => an agent whose cluster queue is empty
                                takes work from other clusters, so every CTA runs exactly
                                once whatever the hardware does with agent placement

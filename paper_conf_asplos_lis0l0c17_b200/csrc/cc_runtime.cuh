@@ -51,7 +51,7 @@ struct Sched {
     int32_t stages;               // ring depth (agent backends; 1 for one-shot CTAs)
     int32_t batch;                // slots claimed per queue atomic
     uint32_t stage_bytes;         // bytes per ring buffer (128-byte multiple)
-    int32_t bypass;               // staged loads skip L1 (BPS, §4.3(II))
+    int32_t staging;              // cc_staging: 1 TMA, 2 L1-allocating cp.async, 3 direct
     uint32_t* census;             // optional outputs (see ctaclust.h)
     int32_t* exec_sm;
     int32_t* map;
@@ -340,7 +340,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             if (v < 0) break;
             int32_t lin, bx, by;
             lin_to_bxby(s, v, &lin, &bx, &by);
-            body.consume(bx, by, ring + (size_t)st * s.stage_bytes, ctid);
+            body.consume(s, bx, by, ring + (size_t)st * s.stage_bytes, ctid);
             if (ctid == 0) record(s, v, lin);
             __syncwarp();
             if (lane == 0) mbar_arrive(&R.empty[st]);
@@ -364,7 +364,7 @@ __device__ __forceinline__ void one_shot(const Sched& s, Body& body, int32_t v, 
     } else {
         const int ctid = threadIdx.x - PRODUCER_THREADS;
         mbar_wait(&full, 0);
-        body.consume(bx, by, ring, ctid);
+        body.consume(s, bx, by, ring, ctid);
         if (ctid == 0) {
             if (s.census) atomicAdd(s.census + lin, 1u);
             if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();

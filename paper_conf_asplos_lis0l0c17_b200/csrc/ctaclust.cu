@@ -301,7 +301,7 @@ struct CensusBody {   // empty body: binding, queues and census only
     using Params = CensusParams;
     __device__ __forceinline__ explicit CensusBody(const CensusParams&) {}
     __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) { stage_commit(full, lane, 0); }
-    __device__ __forceinline__ void consume(int32_t, int32_t, const uint8_t*, int) {}
+    __device__ __forceinline__ void consume(const Sched&, int32_t, int32_t, const uint8_t*, int) {}
     __device__ __forceinline__ void finish(int) {}
 };
 
@@ -396,7 +396,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     s.ws = c.p->d_ws;
     s.steal = o.steal;
     s.batch = o.batch > 0 ? o.batch : Body::kDefaultBatch;
-    s.bypass = o.bypass;
+    s.staging = o.staging == CC_STAGING_DEFAULT ? CC_STAGING_TMA : o.staging;
     s.stage_bytes = Body::kStageBytes;
     s.census = o.d_census;
     s.exec_sm = o.d_exec_sm;

@@ -71,7 +71,8 @@ struct GemvBody {
     __device__ __forceinline__ static int tcol4(int cl, int f) { return f * LPR + cl; }
 
     // ---- producer: one 2D TMA load of the whole tile (OOB rows/cols zero-filled)
-    __device__ __forceinline__ void produce(const Sched&, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+    __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+        if (s.staging == 3) { stage_commit(full, lane, 0); return; }   // direct: consumers load A
         stage_commit(full, lane, (uint32_t)kStageBytes);
         if (lane == 0) tma_load_2d(stage, &p.tmap, bx * TC, by * TR, full);
     }
@@ -120,19 +121,38 @@ struct GemvBody {
     }
 
     // ---- consumers: one logical CTA from the staged tile
-    __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+    __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         if (DO_ROW && by != cur_ti) { if (cur_ti >= 0) flush_row(ctid); cur_ti = by; }
         if (DO_COL && bx != cur_tj) { if (cur_tj >= 0) flush_col(ctid); cur_tj = bx; }
         const int warp = ctid >> 5, lane = ctid & 31, sub = lane / LPR, cl = lane % LPR;
         const int col0 = bx * TC, row0 = by * TR;
+        const bool direct = s.staging == 3;
+        if (col0 + TC <= p.n && row0 + TR <= p.m) {
+            // interior tile: no bounds anywhere in the hot loop
+            float4 xv[FPL];
+#pragma unroll
+            for (int f = 0; f < FPL; ++f) xv[f] = DO_ROW ? ld_cached4(p.vc + col0 + tcol4(cl, f) * 4) : f4_zero();
+#pragma unroll
+            for (int k = 0; k < NP; ++k) {
+                const int r = trow(warp, k, sub);
+                const float rv = DO_COL ? ld_cached(p.vr + row0 + r) : 0.f;
+#pragma unroll
+                for (int f = 0; f < FPL; ++f) {
+                    const float4 a = direct ? ld_stream4(p.A + (int64_t)(row0 + r) * p.lda + col0 + tcol4(cl, f) * 4)
+                                            : reinterpret_cast<const float4*>(stage)[r * CW + tcol4(cl, f)];
+                    accumulate(k, f, a, xv[f], rv);
+                }
+            }
+            return;
+        }
+        // ragged edge tile.  Staged tiles are zero-filled past m / n by the TMA
+        // unit; only the vector reads (and direct loads) need bounds.
         float4 xv[FPL];
-        bool cok[FPL];
 #pragma unroll
         for (int f = 0; f < FPL; ++f) {
             const int col = col0 + tcol4(cl, f) * 4;
-            cok[f] = col < p.n;
             xv[f] = f4_zero();
-            if (DO_ROW && cok[f]) {
+            if (DO_ROW && col < p.n) {
                 if (col + 4 <= p.n) xv[f] = ld_cached4(p.vc + col);
                 else {
                     xv[f].x = ld_cached(p.vc + col);
@@ -141,28 +161,34 @@ struct GemvBody {
                 }
             }
         }
-        const float4* tile = reinterpret_cast<const float4*>(stage);
 #pragma unroll
         for (int k = 0; k < NP; ++k) {
             const int r = trow(warp, k, sub);
-            if (row0 + r >= p.m) continue;                 // never staged
+            if (row0 + r >= p.m) continue;
             const float rv = DO_COL ? ld_cached(p.vr + row0 + r) : 0.f;
 #pragma unroll
             for (int f = 0; f < FPL; ++f) {
-                if (!cok[f]) continue;
-                float4 a = tile[r * CW + tcol4(cl, f)];
                 const int col = col0 + tcol4(cl, f) * 4;
-                if (col + 4 > p.n) {                         // lanes past n hold padding
-                    if (col + 1 >= p.n) a.y = 0.f;
+                if (col >= p.n) continue;
+                float4 a;
+                if (direct) {
+                    a = ld_stream4(p.A + (int64_t)(row0 + r) * p.lda + col);   // inside lda (lda % 4 == 0)
+                    if (col + 1 >= p.n) a.y = 0.f;                              // padding past n
                     if (col + 2 >= p.n) a.z = 0.f;
-                    a.w = 0.f;
+                    if (col + 3 >= p.n) a.w = 0.f;
+                } else {
+                    a = reinterpret_cast<const float4*>(stage)[r * CW + tcol4(cl, f)];
                 }
-                if (DO_ROW) racc[k] += a.x * xv[f].x + a.y * xv[f].y + a.z * xv[f].z + a.w * xv[f].w;
-                if (DO_COL) {
-                    cacc[f].x += a.x * rv; cacc[f].y += a.y * rv;
-                    cacc[f].z += a.z * rv; cacc[f].w += a.w * rv;
-                }
+                accumulate(k, f, a, xv[f], rv);
             }
+        }
+    }
+
+    __device__ __forceinline__ void accumulate(int k, int f, const float4& a, const float4& xv, float rv) {
+        if (DO_ROW) racc[k] += a.x * xv.x + a.y * xv.y + a.z * xv.z + a.w * xv.w;
+        if (DO_COL) {
+            cacc[f].x += a.x * rv; cacc[f].y += a.y * rv;
+            cacc[f].z += a.z * rv; cacc[f].w += a.w * rv;
         }
     }
 

@@ -65,7 +65,7 @@ struct SpmvBody {
         stage_commit(full, lane, 0);
     }
 
-    __device__ __forceinline__ void consume(int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
+    __device__ __forceinline__ void consume(const Sched&, int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
         __shared__ int32_t s_rowend[SPMV_IPC + 1];
         __shared__ float s_prod[SPMV_IPT][SPMV_THREADS];
         __shared__ float s_wv[SPMV_THREADS / 32];

@@ -5,14 +5,16 @@
 // and the columns left/right of a tile are the border data of its neighbours
 // (the cache-line/algorithm-related classes).
 //
-// The producer warp stages the tile plus halo -- rows y0-H .. y0+31+H, columns
-// x0-4 .. x0+35 (10 aligned 16-byte chunks per row) -- into shared memory,
-// either with one 2D TMA load (bypass = 1: L2 -> smem, L1 untouched) or with
-// cp.async.ca chunks (bypass = 0), which also allocate every line in L1.  A neighbouring tile
-// staged soon after on the same SM therefore finds its halo (and the shared
-// 16-byte edge chunks) in L1 instead of L2: clustering neighbouring tiles onto
-// one SM (TILE order, Fig. 7) turns that halo traffic into L1 hits.  Chunks
-// outside the image are zero-filled without a read.
+// How the tile plus halo (rows y0-H .. y0+31+H, columns x0-4 .. x0+35, i.e.
+// 10 aligned 16-byte chunks per row) reaches the consumers (Sched::staging):
+//   TMA    one 2D tensor load per tile, L2 -> shared memory, L1 untouched;
+//          the image border is zero-filled by the TMA unit (default);
+//   L1     cp.async.ca 16-byte chunks: every line also allocates in L1, so a
+//          neighbouring tile staged soon after on the same SM finds its halo
+//          in L1 -- the paper's inter-CTA L1 reuse, which clustering
+//          neighbouring tiles onto one SM (TILE order, Fig. 7) is meant to
+//          exploit;
+//   direct no staging: consumers load through L1 themselves (plain kernel).
 // Consumers: 256 threads; thread (r = ctid/8, c4 = ctid%8) owns the float4 at
 // row r, columns 4*c4 .. 4*c4+3 of the tile.
 #pragma once
@@ -21,24 +23,24 @@
 
 namespace cc {
 
+enum : int32_t { STAGE_TMA = 1, STAGE_L1 = 2, STAGE_DIRECT = 3 };
 constexpr int ST_COLS = 40;                 // staged floats per row (x0-4 .. x0+35)
 
 template <int H>
 struct HaloTile {
     static constexpr int kRows = 32 + 2 * H;
     static constexpr int kBytes = ((kRows * ST_COLS * 4) + 127) & ~127;
-    // warp-collective: stage rows y0-H.., columns x0-4.. of `src`.
+    // warp-collective: stage rows y0-H.., columns x0-4.. of `src` (TMA or L1 mode).
     __device__ __forceinline__ static void stage(const float* src, int64_t ld, int32_t rows, int32_t cols,
                                                  int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
-                                                 int32_t bypass, const CUtensorMap* tmap) {
-        const int32_t cols4 = (cols + 3) & ~3;   // last 16-byte chunk stays inside ld
-        if (bypass) {
-            // BPS: one 2D TMA load of the (32+2H) x 40 box, L2 -> shared memory,
-            // no L1 allocation; the image border is zero-filled by the TMA unit.
+                                                 int32_t mode, const CUtensorMap* tmap) {
+        if (mode == STAGE_DIRECT) { stage_commit(full, lane, 0); return; }
+        if (mode == STAGE_TMA) {
             stage_commit(full, lane, (uint32_t)(kRows * ST_COLS * 4));
             if (lane == 0) tma_load_2d(dst, tmap, x0 - 4, y0 - H, full);
             return;
         }
+        const int32_t cols4 = (cols + 3) & ~3;   // last 16-byte chunk stays inside ld
         // lanes 0..29 cover three staged rows (10 chunks each) per step
         const int r0 = lane / 10, cc = lane - r0 * 10;
         const int32_t gx = x0 - 4 + 4 * cc;
@@ -48,9 +50,7 @@ struct HaloTile {
                 const int32_t gy = y0 - H + rr;
                 const bool ok = col_ok && gy >= 0 && gy < rows;
                 const float* g = ok ? src + (int64_t)gy * ld + gx : src;
-                uint8_t* d = dst + (rr * ST_COLS + 4 * cc) * 4;
-                if (bypass) cp_async_cg16(d, g, ok ? 16u : 0u);
-                else cp_async_ca16(d, g, ok ? 16u : 0u);
+                cp_async_ca16(dst + (rr * ST_COLS + 4 * cc) * 4, g, ok ? 16u : 0u);
             }
         }
         cp_async_arrive(full);
@@ -58,19 +58,44 @@ struct HaloTile {
     }
 };
 
+__device__ __forceinline__ void store4_masked(float* dst, float4 o, int gx, int cols) {
+    if (gx + 4 <= cols) *reinterpret_cast<float4*>(dst) = o;
+    else {
+        dst[0] = o.x;
+        if (gx + 1 < cols) dst[1] = o.y;
+        if (gx + 2 < cols) dst[2] = o.z;
+    }
+}
+
 // ---------------------------------------------------------------------------
 // Jacobi 5-point sweep (reading R14, PolyBench jacobi-2d form):
 //   b[i][j] = 0.2f * ((((c + w) + e) + n) + s)     on the interior,
 //   b[i][j] = a[i][j]                               on the boundary.
 // fp32, summed in that fixed order with no contraction, so the sweep is
-// bit-reproducible against oracle_jacobi5_f32.
+// bit-reproducible against oracle_jacobi5_f32 in every staging mode.
 // ---------------------------------------------------------------------------
 struct JacobiParams { CUtensorMap tmap; const float* a; float* b; int64_t ld; int32_t rows, cols; };
+
+__device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, float lw, float re,
+                                               int gy, int gx, int rows, int cols) {
+    float4 o;
+    o.x = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.x, lw), c.y), up.x), dn.x));
+    o.y = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.y, c.x), c.z), up.y), dn.y));
+    o.z = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.z, c.y), c.w), up.z), dn.z));
+    o.w = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.w, c.z), re), up.w), dn.w));
+    const bool row_bd = (gy == 0) || (gy == rows - 1);
+    const int cl = cols - 1;
+    if (row_bd || gx == 0 || gx == cl) o.x = c.x;
+    if (row_bd || gx + 1 == cl) o.y = c.y;
+    if (row_bd || gx + 2 == cl) o.z = c.z;
+    if (row_bd || gx + 3 == cl) o.w = c.w;
+    return o;
+}
 
 struct Jacobi5Body {
     static constexpr int kConsumers = 256;
     static constexpr int kStageBytes = HaloTile<1>::kBytes;
-    static constexpr int kDefaultStages = 3;
+    static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
     static constexpr int kMinAgents = 6;
     using Params = JacobiParams;
@@ -78,37 +103,36 @@ struct Jacobi5Body {
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass, &p.tmap);
+        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap);
     }
 
-    __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+    __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         const int r = ctid >> 3, c4 = ctid & 7;
         const int gy = by * 32 + r, gx = bx * 32 + 4 * c4;
-        if (gy >= p.rows || gx >= p.cols) return;
-        const float* t = reinterpret_cast<const float*>(stage);
-        const float* mid = t + (r + 1) * ST_COLS + 4 + 4 * c4;
-        const float4 c = *reinterpret_cast<const float4*>(mid);
-        const float4 up = *reinterpret_cast<const float4*>(mid - ST_COLS);
-        const float4 dn = *reinterpret_cast<const float4*>(mid + ST_COLS);
-        const float lw = mid[-1], re = mid[4];
-        float4 o;
-        o.x = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.x, lw), c.y), up.x), dn.x));
-        o.y = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.y, c.x), c.z), up.y), dn.y));
-        o.z = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.z, c.y), c.w), up.z), dn.z));
-        o.w = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.w, c.z), re), up.w), dn.w));
-        const bool row_bd = (gy == 0) || (gy == p.rows - 1);
-        const int cl = p.cols - 1;
-        if (row_bd || gx == 0 || gx == cl) o.x = c.x;
-        if (row_bd || gx + 1 == cl) o.y = c.y;
-        if (row_bd || gx + 2 == cl) o.z = c.z;
-        if (row_bd || gx + 3 == cl) o.w = c.w;
-        float* dst = p.b + (int64_t)gy * p.ld + gx;
-        if (gx + 4 <= p.cols) *reinterpret_cast<float4*>(dst) = o;
-        else {
-            dst[0] = o.x;
-            if (gx + 1 < p.cols) dst[1] = o.y;
-            if (gx + 2 < p.cols) dst[2] = o.z;
+        const bool in = gy < p.rows && gx < p.cols;
+        float4 c, up, dn;
+        float lw, re;
+        if (s.staging == STAGE_DIRECT) {
+            // plain-kernel form: every load goes through L1 (rows r-1 / r+1 of
+            // the tile are other threads' centre rows -> L1 hits)
+            const float* a = p.a + (int64_t)gy * p.ld + gx;
+            c = in ? ld_cached4(a) : f4_zero();
+            up = (in && gy > 0) ? ld_cached4(a - p.ld) : f4_zero();
+            dn = (in && gy + 1 < p.rows) ? ld_cached4(a + p.ld) : f4_zero();
+            lw = __shfl_up_sync(0xffffffffu, c.w, 1, 8);
+            re = __shfl_down_sync(0xffffffffu, c.x, 1, 8);
+            if (c4 == 0) lw = (in && gx > 0) ? ld_cached(a - 1) : 0.f;
+            if (c4 == 7) re = (in && gx + 4 < p.cols) ? ld_cached(a + 4) : 0.f;
+        } else {
+            const float* mid = reinterpret_cast<const float*>(stage) + (r + 1) * ST_COLS + 4 + 4 * c4;
+            c = *reinterpret_cast<const float4*>(mid);
+            up = *reinterpret_cast<const float4*>(mid - ST_COLS);
+            dn = *reinterpret_cast<const float4*>(mid + ST_COLS);
+            lw = mid[-1];
+            re = mid[4];
         }
+        if (!in) return;
+        store4_masked(p.b + (int64_t)gy * p.ld + gx, jacobi_point4(c, up, dn, lw, re, gy, gx, p.rows, p.cols), gx, p.cols);
     }
     __device__ __forceinline__ void finish(int) {}
 };
@@ -148,20 +172,14 @@ __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const 
     o.y = (row_in && gx + 1 >= R && gx + 1 < p.cols - R) ? acc[1] : 0.f;
     o.z = (row_in && gx + 2 >= R && gx + 2 < p.cols - R) ? acc[2] : 0.f;
     o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[3] : 0.f;
-    float* dst = p.out + (int64_t)gy * p.ld + gx;
-    if (gx + 4 <= p.cols) *reinterpret_cast<float4*>(dst) = o;
-    else {
-        dst[0] = o.x;
-        if (gx + 1 < p.cols) dst[1] = o.y;
-        if (gx + 2 < p.cols) dst[2] = o.z;
-    }
+    store4_masked(p.out + (int64_t)gy * p.ld + gx, o, gx, p.cols);
 }
 
 template <int R>
 struct Conv2dBody {
     static constexpr int kConsumers = 256;
     static constexpr int kStageBytes = HaloTile<R>::kBytes;
-    static constexpr int kDefaultStages = 3;
+    static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
     static constexpr int kMinAgents = 6;
     using Params = ConvParams<R>;
@@ -169,9 +187,25 @@ struct Conv2dBody {
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.bypass, &p.tmap);
+        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap);
     }
-    __device__ __forceinline__ void consume(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+    __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        if (s.staging == STAGE_DIRECT) {
+            // plain-kernel form: the consumers stage the tile themselves through L1
+            __shared__ float4 s_in[HaloTile<R>::kRows][ST_COLS / 4];
+            const int x0 = bx * 32, y0 = by * 32;
+            for (int idx = ctid; idx < HaloTile<R>::kRows * 10; idx += kConsumers) {
+                const int rr = idx / 10, cc = idx - rr * 10;
+                const int gy = y0 - R + rr, gx = x0 - 4 + 4 * cc;
+                float4 v = f4_zero();
+                if (gy >= 0 && gy < p.rows && gx >= 0 && gx < p.cols) v = ld_cached4(p.in + (int64_t)gy * p.ld + gx);
+                s_in[rr][cc] = v;
+            }
+            consumer_sync<kConsumers>();
+            conv_tile_compute<R>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid);
+            consumer_sync<kConsumers>();                 // s_in is rewritten by the next task
+            return;
+        }
         conv_tile_compute<R>(p, reinterpret_cast<const float*>(stage), bx, by, ctid);
     }
     __device__ __forceinline__ void finish(int) {}

@@ -22,6 +22,7 @@ ORDERS = {"row": ORDER_ROW, "col": ORDER_COL, "tile": ORDER_TILE, "user": ORDER_
 BACKEND_DEFAULT, BACKEND_AGENT, BACKEND_TBCLUSTER, BACKEND_AGENT_IDENTITY, BACKEND_REDIRECT = 0, 1, 2, 3, 4
 BACKENDS = {"default": 0, "agent": 1, "tbcluster": 2, "identity": 3, "redirect": 4}
 K_CENSUS, K_MATVEC, K_ATAX, K_BICG, K_MVT, K_JACOBI5, K_CONV2D, K_SPMV = range(8)
+STAGINGS = {"default": 0, "tma": 1, "l1": 2, "direct": 3}
 KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7}
 STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_ERR_NOT_PERMUTATION",
           -4: "CC_ERR_CUDA", -5: "CC_ERR_NCCL", -6: "CC_ERR_UNSUPPORTED", -7: "CC_ERR_NO_DEVICE"}
@@ -50,7 +51,7 @@ class PlanDesc(ctypes.Structure):
 
 class LaunchOpts(ctypes.Structure):
     _fields_ = [("backend", _i32), ("active_agents", _i32), ("max_agents", _i32), ("stages", _i32),
-                ("batch", _i32), ("bypass", _i32), ("steal", _i32), ("cluster_size", _i32), ("d_census", _vp),
+                ("batch", _i32), ("staging", _i32), ("steal", _i32), ("cluster_size", _i32), ("d_census", _vp),
                 ("d_exec_sm", _vp),
                 ("d_map", _vp)]
 
@@ -199,10 +200,10 @@ def _stream(stream):
     return s.cuda_stream
 
 
-def make_opts(backend="agent", active_agents=0, max_agents=0, stages=0, batch=0, bypass=0, steal=1,
+def make_opts(backend="agent", active_agents=0, max_agents=0, stages=0, batch=0, staging=0, steal=1,
               cluster_size=2, census=None, exec_sm=None, map=None) -> LaunchOpts:
     b = BACKENDS[backend] if isinstance(backend, str) else int(backend)
-    return LaunchOpts(b, active_agents, max_agents, int(stages), int(batch), int(bypass), int(steal), cluster_size,
+    return LaunchOpts(b, active_agents, max_agents, int(stages), int(batch), STAGINGS.get(staging, staging) if isinstance(staging, str) else int(staging), int(steal), cluster_size,
                       _ptr(census), _ptr(exec_sm), _ptr(map))
 
 

@@ -23,6 +23,7 @@ def main():
     ap.add_argument("--active", type=int, default=0)
     ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--batch", type=int, default=0)
+    ap.add_argument("--staging", default="default")
     ap.add_argument("--cluster", type=int, default=2)
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--warm", type=int, default=1)
@@ -30,7 +31,7 @@ def main():
     a = ap.parse_args()
     import torch
     from paper_conf_asplos_lis0l0c17_b200 import ops, synth
-    kw = dict(backend=a.backend, active_agents=a.active, stages=a.stages, batch=a.batch)
+    kw = dict(backend=a.backend, active_agents=a.active, stages=a.stages, batch=a.batch, staging=a.staging)
     if a.order:
         kw["order"] = a.order
     if a.tile:

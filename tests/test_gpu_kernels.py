@@ -26,6 +26,9 @@ VARIANTS = [
     dict(backend="agent", order="col", stages=6, batch=3),
     dict(backend="identity"),
     dict(backend="redirect", order="row"),
+    dict(backend="default", staging="direct"),
+    dict(backend="agent", order="col", staging="direct"),
+    dict(backend="agent", order="row", staging="tma", stages=3, batch=2),
 ]
 
 
@@ -129,7 +132,10 @@ def test_bicg_full_size_config2():
 JVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(8, 8)),
              dict(backend="agent", order="row"), dict(backend="agent", order="col", active_agents=2),
              dict(backend="agent", order="tile", tile=(2, 2), stages=8, batch=7), dict(backend="identity"),
-             dict(backend="redirect", order="tile", tile=(4, 4))]
+             dict(backend="redirect", order="tile", tile=(4, 4)),
+             dict(backend="default", staging="l1"), dict(backend="default", staging="direct"),
+             dict(backend="agent", order="tile", tile=(8, 8), staging="l1"),
+             dict(backend="agent", order="row", staging="direct")]
 
 
 @pytest.mark.parametrize("v", JVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
@@ -171,7 +177,10 @@ CVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(
              dict(backend="agent", order="col", stages=1, batch=1), dict(backend="identity"),
              dict(backend="tbcluster", cluster_size=1), dict(backend="tbcluster", cluster_size=2),
              dict(backend="tbcluster", cluster_size=4), dict(backend="tbcluster", cluster_size=8),
-             dict(backend="redirect", order="row")]
+             dict(backend="redirect", order="row"),
+             dict(backend="default", staging="l1"), dict(backend="default", staging="direct"),
+             dict(backend="agent", order="tile", tile=(8, 8), staging="l1"),
+             dict(backend="agent", order="col", staging="direct")]
 
 
 @pytest.mark.parametrize("v", CVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
