@@ -49,10 +49,26 @@ def time_ms(fn, reps, warm=3, inner=1):
     return out[len(out) // 2]
 
 
-def measure(variants, fn, reps, nbytes, extra=None, warm=3, inner=1):
+def graph_ms(fn, reps, inner):
+    """Time `inner` launches captured in one CUDA graph (removes the Python /
+    host launch overhead that dominates microsecond kernels)."""
+    import torch
+    for _ in range(3):
+        fn()
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for _ in range(inner):
+            fn()
+    g.replay()
+    torch.cuda.synchronize()
+    return time_ms(g.replay, reps, warm=1) / inner
+
+
+def measure(variants, fn, reps, nbytes, extra=None, warm=3, inner=1, graph=False):
     rows = []
     for name, kw in variants:
-        ms = time_ms(lambda: fn(kw), reps, warm=warm, inner=inner)
+        ms = graph_ms(lambda: fn(kw), reps, inner) if graph else time_ms(lambda: fn(kw), reps, warm=warm, inner=inner)
         gbs = nbytes / (ms * 1e-3) / 1e9
         d = {"variant": name, "ms": round(ms, 5), "GBps": round(gbs, 1), "frac_hbm": round(gbs / _peak(), 4)}
         if extra:
@@ -96,8 +112,8 @@ def suite_matvec(quick):
     x = synth.uniform(2, n, backend="torch", device="cuda")
     y = torch.zeros(n, device="cuda")
     v = variants_for("row") + [("agent-col", dict(backend="agent", order="col"))]
-    r = measure(v, lambda kw: ops.matvec(A, x, y, **kw), 20 if quick else 50, 4 * n * n + 8 * n, inner=50)
-    r["config"] = "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident"
+    r = measure(v, lambda kw: ops.matvec(A, x, y, **kw), 20 if quick else 50, 4 * n * n + 8 * n, inner=50, graph=True)
+    r["config"] = "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident; 50 launches per CUDA graph"
     return r
 
 

@@ -11,10 +11,51 @@ namespace cc {
 // L1::no_allocate is the cheap bypass -> LDG.E.NA).  Used for operands with no
 // inter-CTA reuse so they do not evict the reused slices.
 __device__ __forceinline__ float4 ld_stream4(const float* p) {
+    // not volatile: a pure read of data no one writes during the kernel, so the
+    // compiler may hoist and batch these loads
+    float4 v;
+    asm("ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0,%1,%2,%3}, [%4];"
+        : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+    return v;
+}
+// Same load as a volatile asm: volatile asm statements keep their program order,
+// so a run of these issued back to back stays batched (all in flight at once)
+// instead of being sunk next to their consumers by the scheduler.
+__device__ __forceinline__ float4 ld_stream4_batched(const float* p) {
     float4 v;
     asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0,%1,%2,%3}, [%4];"
                  : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
     return v;
+}
+// Four streaming 16-byte loads issued by one asm statement: they leave the SM
+// back to back whatever the scheduler does with their consumers.
+__device__ __forceinline__ void ld_stream4_x4(float4& a, float4& b, float4& c, float4& d,
+                                              const float* pa, const float* pb, const float* pc, const float* pd) {
+    asm volatile(
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0,%1,%2,%3}, [%16];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%4,%5,%6,%7}, [%17];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%8,%9,%10,%11}, [%18];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%12,%13,%14,%15}, [%19];"
+        : "=f"(a.x), "=f"(a.y), "=f"(a.z), "=f"(a.w), "=f"(b.x), "=f"(b.y), "=f"(b.z), "=f"(b.w),
+          "=f"(c.x), "=f"(c.y), "=f"(c.z), "=f"(c.w), "=f"(d.x), "=f"(d.y), "=f"(d.z), "=f"(d.w)
+        : "l"(pa), "l"(pb), "l"(pc), "l"(pd));
+}
+// Eight of them in one statement (the 32 x 256 gemv tile: 4 rows x 2 float4 per lane).
+__device__ __forceinline__ void ld_stream4_x8(float4* v, const float* const* p) {
+    asm volatile(
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0,%1,%2,%3}, [%32];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%4,%5,%6,%7}, [%33];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%8,%9,%10,%11}, [%34];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%12,%13,%14,%15}, [%35];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%16,%17,%18,%19}, [%36];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%20,%21,%22,%23}, [%37];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%24,%25,%26,%27}, [%38];\n\t"
+        "ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%28,%29,%30,%31}, [%39];"
+        : "=f"(v[0].x), "=f"(v[0].y), "=f"(v[0].z), "=f"(v[0].w), "=f"(v[1].x), "=f"(v[1].y), "=f"(v[1].z), "=f"(v[1].w),
+          "=f"(v[2].x), "=f"(v[2].y), "=f"(v[2].z), "=f"(v[2].w), "=f"(v[3].x), "=f"(v[3].y), "=f"(v[3].z), "=f"(v[3].w),
+          "=f"(v[4].x), "=f"(v[4].y), "=f"(v[4].z), "=f"(v[4].w), "=f"(v[5].x), "=f"(v[5].y), "=f"(v[5].z), "=f"(v[5].w),
+          "=f"(v[6].x), "=f"(v[6].y), "=f"(v[6].z), "=f"(v[6].w), "=f"(v[7].x), "=f"(v[7].y), "=f"(v[7].z), "=f"(v[7].w)
+        : "l"(p[0]), "l"(p[1]), "l"(p[2]), "l"(p[3]), "l"(p[4]), "l"(p[5]), "l"(p[6]), "l"(p[7]));
 }
 // Default-cached load (allocates in L1): operands that other CTAs of the same
 // cluster re-read (vector slices, halos).

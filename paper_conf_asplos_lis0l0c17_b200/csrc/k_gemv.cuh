@@ -130,19 +130,55 @@ struct GemvBody {
         if (col0 + TC <= p.n && row0 + TR <= p.m) {
             // interior tile: no bounds anywhere in the hot loop
             float4 xv[FPL];
+            float rv[NP];
 #pragma unroll
             for (int f = 0; f < FPL; ++f) xv[f] = DO_ROW ? ld_cached4(p.vc + col0 + tcol4(cl, f) * 4) : f4_zero();
 #pragma unroll
-            for (int k = 0; k < NP; ++k) {
-                const int r = trow(warp, k, sub);
-                const float rv = DO_COL ? ld_cached(p.vr + row0 + r) : 0.f;
+            for (int k = 0; k < NP; ++k) rv[k] = DO_COL ? ld_cached(p.vr + row0 + trow(warp, k, sub)) : 0.f;
+            if (direct) {
+                // plain-kernel form: issue every A load of the tile first (NP*FPL
+                // independent 16-byte loads in flight per thread), then reduce
+                float4 av[NP][FPL];
+                const float* base = p.A + (int64_t)row0 * p.lda + col0;
+                if constexpr (NP * FPL == 8) {
+                    float4 v8[8];
+                    const float* ptr[8];
 #pragma unroll
-                for (int f = 0; f < FPL; ++f) {
-                    const float4 a = direct ? ld_stream4(p.A + (int64_t)(row0 + r) * p.lda + col0 + tcol4(cl, f) * 4)
-                                            : reinterpret_cast<const float4*>(stage)[r * CW + tcol4(cl, f)];
-                    accumulate(k, f, a, xv[f], rv);
+                    for (int q = 0; q < 8; ++q)
+                        ptr[q] = base + (int64_t)trow(warp, q / FPL, sub) * p.lda + tcol4(cl, q % FPL) * 4;
+                    ld_stream4_x8(v8, ptr);
+#pragma unroll
+                    for (int q = 0; q < 8; ++q) av[q / FPL][q % FPL] = v8[q];
+                } else if constexpr ((NP * FPL) % 4 == 0) {
+#pragma unroll
+                    for (int q = 0; q < NP * FPL; q += 4) {
+                        const int k0 = q / FPL, f0 = q % FPL, k1 = (q + 1) / FPL, f1 = (q + 1) % FPL;
+                        const int k2 = (q + 2) / FPL, f2 = (q + 2) % FPL, k3 = (q + 3) / FPL, f3 = (q + 3) % FPL;
+                        ld_stream4_x4(av[k0][f0], av[k1][f1], av[k2][f2], av[k3][f3],
+                                      base + (int64_t)trow(warp, k0, sub) * p.lda + tcol4(cl, f0) * 4,
+                                      base + (int64_t)trow(warp, k1, sub) * p.lda + tcol4(cl, f1) * 4,
+                                      base + (int64_t)trow(warp, k2, sub) * p.lda + tcol4(cl, f2) * 4,
+                                      base + (int64_t)trow(warp, k3, sub) * p.lda + tcol4(cl, f3) * 4);
+                    }
+                } else {
+#pragma unroll
+                    for (int k = 0; k < NP; ++k)
+#pragma unroll
+                        for (int f = 0; f < FPL; ++f)
+                            av[k][f] = ld_stream4_batched(base + (int64_t)trow(warp, k, sub) * p.lda + tcol4(cl, f) * 4);
                 }
+#pragma unroll
+                for (int k = 0; k < NP; ++k)
+#pragma unroll
+                    for (int f = 0; f < FPL; ++f) accumulate(k, f, av[k][f], xv[f], rv[k]);
+                return;
             }
+#pragma unroll
+            for (int k = 0; k < NP; ++k)
+#pragma unroll
+                for (int f = 0; f < FPL; ++f)
+                    accumulate(k, f, reinterpret_cast<const float4*>(stage)[trow(warp, k, sub) * CW + tcol4(cl, f)],
+                               xv[f], rv[k]);
             return;
         }
         // ragged edge tile.  Staged tiles are zero-filled past m / n by the TMA

@@ -67,7 +67,9 @@ struct SpmvBody {
 
     __device__ __forceinline__ void consume(const Sched&, int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
         __shared__ int32_t s_rowend[SPMV_IPC + 1];
-        __shared__ float s_prod[SPMV_IPT][SPMV_THREADS];
+        // products of the CTA's nonzeros, index j stored at j + j/16 (the pad
+        // keeps each thread's 16-long private run conflict-free)
+        __shared__ float s_prod[SPMV_IPC + SPMV_IPC / SPMV_IPT];
         __shared__ float s_wv[SPMV_THREADS / 32];
         __shared__ int32_t s_wf[SPMV_THREADS / 32];
         const int t = ctid, lane = t & 31, warp = t >> 5;
@@ -78,6 +80,18 @@ struct SpmvBody {
         const int64_t y0 = d0 - x0, y1 = d1 - x1;
         const int32_t xl = x1 < p.rows ? x1 : p.rows - 1;      // last row to stage
         for (int32_t i = t; i <= xl - x0; i += kConsumers) s_rowend[i] = p.row_ptr[x0 + i + 1];
+        // all products of the CTA, coalesced: val/col stream past L1, the x
+        // gathers go through it (16 independent loads per thread in flight)
+        const int32_t nz = (int32_t)(y1 - y0);
+#pragma unroll
+        for (int k = 0; k < SPMV_IPT; ++k) {
+            const int32_t j = t + k * kConsumers;
+            if (j < nz) {
+                const int32_t c = __ldcs(p.col + y0 + j);
+                const float v = __ldcs(p.val + y0 + j);
+                s_prod[j + (j >> 4)] = v * ld_cached(p.x + c);
+            }
+        }
         consumer_sync<kConsumers>();
         // this thread's start on the merge path, relative to the CTA rectangle
         const int32_t span = (int32_t)(d1 - d0);
@@ -91,19 +105,7 @@ struct SpmvBody {
         }
         const int32_t tx = x0 + lo;
         const int64_t ty = y0 + dt - lo;
-        // products for up to IPT nonzeros from ty (independent loads: MLP)
-#pragma unroll
-        for (int k = 0; k < SPMV_IPT; ++k) {
-            int64_t idx = ty + k;
-            float pr = 0.f;
-            if (idx < y1) {
-                int32_t c = __ldcs(p.col + idx);
-                float v = __ldcs(p.val + idx);
-                pr = v * ld_cached(p.x + c);
-            }
-            s_prod[k][t] = pr;
-        }
-        // merge walk (s_prod column t is private to this thread: no barrier)
+        // merge walk over this thread's IPT items
         const int32_t items = span - dt < SPMV_IPT ? span - dt : SPMV_IPT;
         float sum = 0.f, first_val = 0.f;
         int32_t first_row = -1;
@@ -112,7 +114,8 @@ struct SpmvBody {
         int64_t cy = ty;
         for (int it = 0; it < items; ++it) {
             if (cx < p.rows && cy < (int64_t)s_rowend[cx - x0]) {
-                sum += s_prod[cy - ty][t];
+                const int32_t j = (int32_t)(cy - y0);
+                sum += s_prod[j + (j >> 4)];
                 ++cy;
             } else {
                 if (!has_end) { first_row = cx; first_val = sum; has_end = true; }
