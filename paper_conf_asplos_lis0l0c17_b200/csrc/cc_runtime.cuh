@@ -44,7 +44,7 @@ struct Sched {
     const int32_t* user;          // USER order table: v -> lin (device)
     const int32_t* rank_of_smid;  // %smid -> dense SM rank or -1 (device)
     int32_t smid_span;
-    int32_t* ws;                  // workspace: agent_ctr[M+1] | head[M] | gq | done
+    int32_t* ws;                  // workspace: agent_ctr[M+1] | head[M] | gq | done | claimed
     int32_t mode;                 // MODE_AGENT / MODE_IDENTITY
     int32_t active_agents;
     int32_t steal;
@@ -61,7 +61,8 @@ __device__ __forceinline__ int32_t* ws_agent_ctr(const Sched& s) { return s.ws; 
 __device__ __forceinline__ int32_t* ws_head(const Sched& s) { return s.ws + s.g.M + 1; }
 __device__ __forceinline__ int32_t* ws_gq(const Sched& s) { return s.ws + 2 * s.g.M + 1; }
 __device__ __forceinline__ int32_t* ws_done(const Sched& s) { return s.ws + 2 * s.g.M + 2; }
-inline size_t ws_ints(int32_t M) { return (size_t)(2 * M + 3); }
+__device__ __forceinline__ int32_t* ws_claimed(const Sched& s) { return s.ws + 2 * s.g.M + 3; }
+inline size_t ws_ints(int32_t M) { return (size_t)(2 * M + 4); }
 
 // ---------------------------------------------------------------------------
 // PTX helpers
@@ -204,6 +205,7 @@ __device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* 
         const int32_t size = q_size(s, sq);
         if (w < size) {
             P.bq = sq; P.bw = w + 1; P.be = w + s.batch < size ? w + s.batch : size;
+            atomicAdd(ws_claimed(s), P.be - w);       // RED: lets finished agents skip the scan
             if (w + s.batch < size) {                  // claim the next batch early
                 P.sq = sq; P.sw = atom_add_relaxed(q_head(s, sq), s.batch); P.spec = 1;
             }
@@ -211,6 +213,7 @@ __device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* 
         }
         if (sq == P.q) {
             if (!s.steal || s.mode == MODE_IDENTITY) { P.q = -1; return -1; }
+            if (ld_relaxed(ws_claimed(s)) >= s.g.V) { P.q = -1; return -1; }   // nothing left anywhere
             *scan = 1;
             return -1;
         }
@@ -322,13 +325,17 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         // ---- the last agent out resets the workspace for the next launch.  Every
         // other agent's producer has consumed the results of all its atomics
         // (including any speculative claim) before arriving here.
+        int32_t last = 0;
         if (lane == 0) {
             const int32_t total = (int32_t)(gridDim.x * gridDim.y * gridDim.z);
-            if (atom_add_relaxed(ws_done(s), 1) == total - 1) {
-                const int32_t n = 2 * s.g.M + 2;
-                for (int32_t k = 0; k < n; ++k) s.ws[k] = 0;
-                *ws_done(s) = 0;
-            }
+            // order this agent's fire-and-forget `claimed` REDs before its arrival
+            // (the L1 flush this fence costs is irrelevant: the scheduler is done)
+            __threadfence();
+            last = atom_add_relaxed(ws_done(s), 1) == total - 1;
+        }
+        if (__shfl_sync(0xffffffffu, last, 0)) {
+            const int32_t n = 2 * s.g.M + 4;
+            for (int32_t k = lane; k < n; k += 32) s.ws[k] = 0;
         }
     } else {
         const int ctid = threadIdx.x - PRODUCER_THREADS;

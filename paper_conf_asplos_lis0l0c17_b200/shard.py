@@ -59,3 +59,64 @@ def sharded_step(compute, n_rows: int, world: int, rank: int, gather: bool = Tru
         for key in ("tmp", "q", "x1"):
             part[key] = _allgather_rows(part[key], n_rows, world)
     return part
+
+
+# --------------------------------------------------------------------------
+# Slab sharding of the stencils (Jacobi, conv2d): rank g owns image rows
+# [lo, hi) and keeps H halo rows on each side that are not global boundary.
+# One halo exchange per Jacobi sweep (point-to-point with the two neighbours:
+# NCCL send/recv over NVLink on GPUs, gloo in the CPU tests); conv2d needs one
+# exchange before its single pass.  The per-slab sweep treats the slab's first
+# and last rows as fixed boundary -- exactly what a halo row is during a sweep.
+# --------------------------------------------------------------------------
+def slab_range(rows: int, world: int, rank: int, halo: int = 1) -> tuple[int, int, int, int]:
+    """(lo, hi, llo, lhi): owned rows [lo, hi) and local rows [llo, lhi)."""
+    lo, hi = row_range(rows, world, rank)
+    return lo, hi, max(lo - halo, 0), min(hi + halo, rows)
+
+
+def exchange_halos(buf: torch.Tensor, rows: int, world: int, rank: int, halo: int = 1):
+    """Refresh the halo rows of the local slab `buf` (local rows [llo, lhi)) with
+    the neighbours' owned boundary rows."""
+    if world == 1:
+        return
+    lo, hi, llo, lhi = slab_range(rows, world, rank, halo)
+    reqs = []
+    if rank > 0:         # my first owned rows -> rank-1 ; its last owned rows -> my top halo
+        reqs.append(dist.isend(buf[lo - llo: lo - llo + halo].contiguous(), rank - 1))
+        top = torch.empty_like(buf[0:halo])
+        reqs.append(dist.irecv(top, rank - 1))
+    if rank < world - 1:  # my last owned rows -> rank+1 ; its first owned rows -> my bottom halo
+        reqs.append(dist.isend(buf[hi - halo - llo: hi - llo].contiguous(), rank + 1))
+        bot = torch.empty_like(buf[0:halo])
+        reqs.append(dist.irecv(bot, rank + 1))
+    for r in reqs:
+        r.wait()
+    if rank > 0:
+        buf[0:halo] = top
+    if rank < world - 1:
+        buf[lhi - llo - halo: lhi - llo] = bot
+
+
+def jacobi_slab(sweep, a: torch.Tensor, b: torch.Tensor, iters: int, rows: int, world: int, rank: int):
+    """`iters` sweeps of the sharded Jacobi.  `sweep(src, dst)` runs one sweep on
+    the local slab (global boundary and halo rows copied through).  Returns the
+    local buffer holding the result."""
+    src, dst = a, b
+    for _ in range(iters):
+        sweep(src, dst)
+        exchange_halos(dst, rows, world, rank, 1)
+        src, dst = dst, src
+    return src
+
+
+def gather_rows(local_owned: torch.Tensor, rows: int, world: int, rank: int) -> torch.Tensor:
+    """All-gather the owned row blocks of a 2D slab decomposition (final gather)."""
+    if world == 1:
+        return local_owned
+    cap = max(hi - lo for lo, hi in (row_range(rows, world, g) for g in range(world)))
+    buf = torch.zeros((cap,) + tuple(local_owned.shape[1:]), dtype=local_owned.dtype, device=local_owned.device)
+    buf[: local_owned.shape[0]] = local_owned
+    out = [torch.empty_like(buf) for _ in range(world)]
+    dist.all_gather(out, buf)
+    return torch.cat([out[g][: row_range(rows, world, g)[1] - row_range(rows, world, g)[0]] for g in range(world)])

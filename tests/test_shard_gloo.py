@@ -79,3 +79,52 @@ def test_sharded_step_equals_unsharded(world):
     assert np.array_equal(got["tmp"], tmp) and np.array_equal(got["y"], y)
     assert np.array_equal(got["q"], qq) and np.array_equal(got["s"], s)
     assert np.array_equal(got["x1"], o1) and np.array_equal(got["x2d"], o2)
+
+
+def _jacobi_worker(rank, world, port, R, C, T, q):
+    import oracle as O
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    u0 = synth.matrix(4, R, C)
+    lo, hi, llo, lhi = shard.slab_range(R, world, rank, 1)
+    a = torch.from_numpy(u0[llo:lhi].copy())
+    b = torch.zeros_like(a)
+
+    def sweep(src, dst):       # one fp32 sweep of the slab (its first/last rows fixed)
+        dst.copy_(torch.from_numpy(O.jacobi5_f32(src.numpy(), 1)))
+
+    out = shard.jacobi_slab(sweep, a, b, T, R, world, rank)
+    full = shard.gather_rows(out[lo - llo: hi - llo], R, world, rank)
+    if rank == 0:
+        q.put(full.numpy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_jacobi_slab_halo_exchange_is_exact(world):
+    """Slab-sharded Jacobi with one halo exchange per sweep equals the unsharded
+    fp32 sweep bit for bit (same evaluation order, R14)."""
+    import oracle as O
+    R, C, T = 23, 17, 9
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_jacobi_worker, args=(g, world, port, R, C, T, q)) for g in range(world)]
+    for pr in procs:
+        pr.start()
+    got = q.get(timeout=120)
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    assert np.array_equal(got, O.jacobi5_f32(synth.matrix(4, R, C), T))
+
+
+def test_slab_range():
+    for rows in (5, 16384, 17):
+        for world in (1, 2, 8):
+            for halo in (1, 3):
+                for g in range(world):
+                    lo, hi, llo, lhi = shard.slab_range(rows, world, g, halo)
+                    assert 0 <= llo <= lo <= hi <= lhi <= rows
+                    assert lo - llo == (halo if g > 0 and lo >= halo else lo - llo)
