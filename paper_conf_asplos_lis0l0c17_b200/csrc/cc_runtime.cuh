@@ -47,6 +47,7 @@ struct Sched {
     int32_t* ws;                  // workspace: agent_ctr[M+1] | head[M] | gq | done | claimed
     int32_t mode;                 // MODE_AGENT / MODE_IDENTITY
     int32_t active_agents;
+    int32_t throttle;             // active_agents < agents launched per SM
     int32_t steal;
     int32_t stages;               // ring depth (agent backends; 1 for one-shot CTAs)
     int32_t batch;                // slots claimed per queue atomic
@@ -179,6 +180,7 @@ struct Prod {
     int32_t bq, bw, be;   // current batch: slots [bw, be) of queue bq
     int32_t sq, sw;   // speculative claim in flight: raw fetch-add result on queue sq
     int32_t spec;
+    int32_t mine;     // slots claimed since the last flush to the global `claimed` count
 };
 
 __device__ __forceinline__ int32_t q_size(const Sched& s, int32_t q) {
@@ -205,7 +207,7 @@ __device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* 
         const int32_t size = q_size(s, sq);
         if (w < size) {
             P.bq = sq; P.bw = w + 1; P.be = w + s.batch < size ? w + s.batch : size;
-            atomicAdd(ws_claimed(s), P.be - w);       // RED: lets finished agents skip the scan
+            P.mine += P.be - w;
             if (w + s.batch < size) {                  // claim the next batch early
                 P.sq = sq; P.sw = atom_add_relaxed(q_head(s, sq), s.batch); P.spec = 1;
             }
@@ -213,7 +215,13 @@ __device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* 
         }
         if (sq == P.q) {
             if (!s.steal || s.mode == MODE_IDENTITY) { P.q = -1; return -1; }
-            if (ld_relaxed(ws_claimed(s)) >= s.g.V) { P.q = -1; return -1; }   // nothing left anywhere
+            // publish this agent's claims; if every slot of the launch is claimed
+            // there is nothing left to steal (the returned value is consumed, so the
+            // add is performed before this agent can reach its exit)
+            const int32_t all = P.mine ? atom_add_relaxed(ws_claimed(s), P.mine) + P.mine
+                                       : ld_relaxed(ws_claimed(s));
+            P.mine = 0;
+            if (all >= s.g.V) { P.q = -1; return -1; }
             *scan = 1;
             return -1;
         }
@@ -295,7 +303,8 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             uint32_t sm = smid();
             int32_t rank = (int32_t)sm < s.smid_span ? s.rank_of_smid[sm] : -1;
             int32_t slot = (rank < 0 || rank >= s.g.M) ? s.g.M : rank;
-            int32_t a = atom_add_relaxed(ws_agent_ctr(s) + slot, 1);
+            // agent id by arrival order (Listing 5 l.17-18) -- only needed to throttle
+            int32_t a = s.throttle ? atom_add_relaxed(ws_agent_ctr(s) + slot, 1) : 0;
             if (rank >= s.g.M) rank = -1;                       // fewer clusters than SMs
             P.home = rank >= 0 ? rank : (int32_t)(blockIdx.x % (uint32_t)(s.g.M > 0 ? s.g.M : 1));
             P.q = (s.g.V > 0 && s.g.M > 0) ? P.home : -1;
@@ -328,9 +337,6 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         int32_t last = 0;
         if (lane == 0) {
             const int32_t total = (int32_t)(gridDim.x * gridDim.y * gridDim.z);
-            // order this agent's fire-and-forget `claimed` REDs before its arrival
-            // (the L1 flush this fence costs is irrelevant: the scheduler is done)
-            __threadfence();
             last = atom_add_relaxed(ws_done(s), 1) == total - 1;
         }
         if (__shfl_sync(0xffffffffu, last, 0)) {

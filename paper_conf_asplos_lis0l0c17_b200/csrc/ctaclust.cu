@@ -421,6 +421,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         CC_TRY(occupancy<Body>(c.p->device, S, &occ));
         const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
         s.active_agents = o.active_agents > 0 ? std::min(o.active_agents, maxa) : maxa;
+        s.throttle = s.active_agents < maxa;
         s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
         s.stages = S;
         const int grid = c.p->facts->num_sms * maxa;

@@ -1,6 +1,6 @@
 # L2-sector / L1-hit / DRAM evidence for default vs clustered CTA order, every config.
 # Run under gpurun from the repo root:  bash scripts/ncu_suite.sh [tag]
-TAG=${1:-r01}
+TAG=${1:-r02}
 OUT=gpurun_out/ncu_$TAG
 mkdir -p $OUT
 M=lts__t_sectors.sum,lts__t_sectors_srcunit_tex.sum,lts__t_sectors_srcunit_tex_op_read.sum,lts__t_sectors_srcunit_tex_op_write.sum,lts__t_sectors_srcunit_tex_op_red.sum,lts__t_sectors_srcunit_tex_op_atom.sum,lts__t_sector_hit_rate.pct,l1tex__t_sector_hit_rate.pct,l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__warps_active.avg.pct_of_peak_sustained_active,gpu__time_duration.sum
@@ -12,26 +12,35 @@ run() {  # name, per-call launches, args...
   echo "$name rc=$?"
 }
 run matvec_default 1 --kernel matvec --backend default
-run matvec_agent_row 1 --kernel matvec --backend agent --order row
-run matvec_agent_col 1 --kernel matvec --backend agent --order col
+run matvec_default-direct 1 --kernel matvec --backend default --staging direct
+run matvec_agent-row 1 --kernel matvec --backend agent --order row
+run matvec_agent-col 1 --kernel matvec --backend agent --order col
+run matvec_agent-row-direct 1 --kernel matvec --backend agent --order row --staging direct
 run matvec_identity 1 --kernel matvec --backend identity
 for k in atax bicg mvt; do
   per=1; [ $k = atax ] && per=2
   run ${k}_default $per --kernel $k --backend default
-  run ${k}_agent_col $per --kernel $k --backend agent --order col
-  run ${k}_agent_row $per --kernel $k --backend agent --order row
+  run ${k}_default-direct $per --kernel $k --backend default --staging direct
+  run ${k}_agent-col $per --kernel $k --backend agent --order col
+  run ${k}_agent-row $per --kernel $k --backend agent --order row
+  run ${k}_agent-col-direct $per --kernel $k --backend agent --order col --staging direct
   run ${k}_identity $per --kernel $k --backend identity
 done
-run jacobi_default 1 --kernel jacobi --backend default
-run jacobi_agent_tile8 1 --kernel jacobi --backend agent --order tile --tile 8x8
-run jacobi_agent_col 1 --kernel jacobi --backend agent --order col
-run jacobi_identity 1 --kernel jacobi --backend identity
-for k in conv3 conv7; do
+for k in jacobi conv3 conv7; do
   run ${k}_default 1 --kernel $k --backend default
-  run ${k}_agent_tile8 1 --kernel $k --backend agent --order tile --tile 8x8
-  run ${k}_tbc4 1 --kernel $k --backend tbcluster --cluster 4
+  run ${k}_default-l1 1 --kernel $k --backend default --staging l1
+  run ${k}_default-direct 1 --kernel $k --backend default --staging direct
+  run ${k}_agent-row 1 --kernel $k --backend agent --order row
+  run ${k}_agent-tile8 1 --kernel $k --backend agent --order tile --tile 8x8
+  run ${k}_agent-tile8-l1 1 --kernel $k --backend agent --order tile --tile 8x8 --staging l1
+  run ${k}_agent-tile8-direct 1 --kernel $k --backend agent --order tile --tile 8x8 --staging direct
+  run ${k}_agent-row-l1 1 --kernel $k --backend agent --order row --staging l1
   run ${k}_identity 1 --kernel $k --backend identity
 done
+for k in conv3 conv7; do
+  run ${k}_tbc2 1 --kernel $k --backend tbcluster --cluster 2
+  run ${k}_tbc8 1 --kernel $k --backend tbcluster --cluster 8
+done
 run spmv_default 1 --kernel spmv --backend default
-run spmv_agent_row 1 --kernel spmv --backend agent --order row
+run spmv_agent-row 1 --kernel spmv --backend agent --order row
 run spmv_identity 1 --kernel spmv --backend identity
