@@ -252,11 +252,23 @@ def main():
     dom = max(per_clu, key=per_clu.get)
     b_local = step_bytes(m, n)
     achieved = b_local[dom] / (per_clu[dom] * 1e-3) / 1e9
-    traffic = None
-    prof = os.path.join(ROOT, "profiles", "ncu_r01_summary.json")
-    if os.path.exists(prof):
+    # DRAM bytes per launch of that kernel from the newest committed ncu capture
+    # (profiles/ncu_<round>_summary.json, scripts/ncu_suite.sh); the L2-sector
+    # reduction vs default order comes from the same capture.
+    traffic, l2red, prof_name = None, None, None
+    import glob
+    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "ncu_r*_summary.json")))
+    if profs:
         try:
-            traffic = json.load(open(prof)).get("dram_bytes_per_launch", {}).get(f"{dom}_{a.backend}_{a.order}")
+            pj = json.load(open(profs[-1]))
+            prof_name = os.path.relpath(profs[-1], ROOT)
+            key = f"{dom}_{a.backend}-{a.order}" + ("" if a.staging in ("default", "tma") else f"-{a.staging}")
+            traffic = pj.get("dram_bytes_per_launch", {}).get(key)
+            if traffic is not None and dom == "atax":
+                traffic = traffic / 2                       # two launches per ATAX call
+            l2red = {f"{r['kernel']}:{r['variant']}": round(r["l2_sm_sector_reduction_vs_default"], 4)
+                     for r in pj.get("rows", []) if r.get("l2_sm_sector_reduction_vs_default") is not None
+                     and r["kernel"] in ("atax", "bicg", "mvt")}
         except Exception:
             traffic = None
 
@@ -321,7 +333,8 @@ def main():
                              "peak": peak, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if pk else "fallback 6.65 TB/s",
                              "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic},
                 "clocks": clk, "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": launches,
-                "l2_sector_reduction": "see profiles/ncu_r01_summary.json"}
+                "l2_sector_reduction": {"source": prof_name, "vs_default_order": l2red,
+                                        "metric": "1 - lts__t_sectors_srcunit_tex(variant) / (default order)"}}
         print(json.dumps(line), flush=True)
     if a.suite and rank == 0 and world == 1:
         import bench_suite

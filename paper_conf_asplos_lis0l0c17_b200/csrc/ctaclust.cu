@@ -311,7 +311,10 @@ using ColB = GemvBody<32, 256, false, true>;
 using BothB = GemvBody<32, 256, true, true>;
 
 template <class Body>
-static size_t dyn_smem(int stages) { return (size_t)stages * Body::kStageBytes + 128; }
+static size_t dyn_smem(int stages, bool direct = false) {
+    // direct loads stage nothing: keep the ring minimal so L1 keeps the space
+    return (size_t)stages * (direct ? 128 : Body::kStageBytes) + 128;
+}
 
 // Opt every instantiation of a body into large dynamic shared memory once.
 template <class Body>
@@ -337,22 +340,22 @@ static cc_status prepare_body(int device) {
 
 // agents per SM the hardware can keep resident for `stages` ring buffers
 template <class Body>
-static cc_status occupancy(int device, int stages, int* occ) {
+static cc_status occupancy(int device, int stages, int* occ, bool direct = false) {
     CC_TRY(prepare_body<Body>(device));
     static std::mutex mu;
-    static int cache[64][MAX_STAGES + 1] = {};
+    static int cache[64][MAX_STAGES + 1][2] = {};
     std::lock_guard<std::mutex> lk(mu);
     if (stages < 1 || stages > MAX_STAGES) return fail(CC_ERR_INVALID_ARG, "stages %d outside [1, %d]", stages, MAX_STAGES);
-    if (!cache[device][stages]) {
+    if (!cache[device][stages][direct]) {
         int prev = 0, n = 0;
         CC_CUDA(cudaGetDevice(&prev));
         CC_CUDA(cudaSetDevice(device));
         CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_agent<Body>, Body::kConsumers + PRODUCER_THREADS,
-                                                              dyn_smem<Body>(stages)));
+                                                              dyn_smem<Body>(stages, direct)));
         CC_CUDA(cudaSetDevice(prev));
-        cache[device][stages] = n > 0 ? n : -1;
+        cache[device][stages][direct] = n > 0 ? n : -1;
     }
-    *occ = cache[device][stages];
+    *occ = cache[device][stages][direct];
     if (*occ < 0) return fail(CC_ERR_UNSUPPORTED, "%d stages of %d bytes do not fit one SM", stages, Body::kStageBytes);
     return CC_OK;
 }
@@ -397,7 +400,8 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     s.steal = o.steal;
     s.batch = o.batch > 0 ? o.batch : Body::kDefaultBatch;
     s.staging = o.staging == CC_STAGING_DEFAULT ? CC_STAGING_TMA : o.staging;
-    s.stage_bytes = Body::kStageBytes;
+    const bool direct = s.staging == CC_STAGING_DIRECT;
+    s.stage_bytes = direct ? 128u : (uint32_t)Body::kStageBytes;
     s.census = o.d_census;
     s.exec_sm = o.d_exec_sm;
     s.map = o.d_map;
@@ -407,25 +411,25 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         if (g.gy > 65535) return fail(CC_ERR_UNSUPPORTED, "default backend: gy %d > 65535", g.gy);
         s.map = nullptr;
         s.stages = 1;
-        k_default<Body><<<dim3(g.gx, g.gy), threads, dyn_smem<Body>(1), c.st>>>(s, prm);
+        k_default<Body><<<dim3(g.gx, g.gy), threads, dyn_smem<Body>(1, direct), c.st>>>(s, prm);
         break;
     }
     case CC_BACKEND_REDIRECT:
         s.stages = 1;
-        k_redirect<Body><<<g.V, threads, dyn_smem<Body>(1), c.st>>>(s, prm);
+        k_redirect<Body><<<g.V, threads, dyn_smem<Body>(1, direct), c.st>>>(s, prm);
         break;
     case CC_BACKEND_AGENT:
     case CC_BACKEND_AGENT_IDENTITY: {
         const int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
         int occ = 0;
-        CC_TRY(occupancy<Body>(c.p->device, S, &occ));
+        CC_TRY(occupancy<Body>(c.p->device, S, &occ, direct));
         const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
         s.active_agents = o.active_agents > 0 ? std::min(o.active_agents, maxa) : maxa;
         s.throttle = s.active_agents < maxa;
         s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
         s.stages = S;
         const int grid = c.p->facts->num_sms * maxa;
-        k_agent<Body><<<grid, threads, dyn_smem<Body>(S), c.st>>>(s, prm);
+        k_agent<Body><<<grid, threads, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
         break;
     }
     default:
