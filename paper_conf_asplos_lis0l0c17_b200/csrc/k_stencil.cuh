@@ -145,43 +145,64 @@ struct Jacobi5Body {
 template <int R>
 struct ConvParams { CUtensorMap tmap; const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
 
-template <int R>
+// Thread ctid computes RB vertically adjacent rows x 4 columns of the tile
+// (256/RB threads per tile).  Each staged input row is read once (3 LDS.128)
+// and feeds every output row it is a tap of: RB = 2 cuts the shared-memory
+// reads per output by 33 % (3x3) / 43 % (7x7) -- the conv is otherwise
+// shared-memory-bandwidth bound.  The summation order per output is the
+// filter's row-major tap order, as in the oracle.
+template <int R, int RB = 1>
 __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const float* rows_base,
                                                   int32_t bx, int32_t by, int ctid) {
     // rows_base points at the staged row holding input row y0 - R, column x0 - 4
     constexpr int K = 2 * R + 1;
-    const int r = ctid >> 3, c4 = ctid & 7;
-    const int gy = by * 32 + r, gx = bx * 32 + 4 * c4;
-    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+    const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
+    const int gx = bx * 32 + 4 * c4;
+    float acc[RB][4];
 #pragma unroll
-    for (int dy = 0; dy < K; ++dy) {
-        const float4* row = reinterpret_cast<const float4*>(rows_base + (r + dy) * ST_COLS + 4 * c4);
+    for (int j = 0; j < RB; ++j)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
+#pragma unroll
+    for (int ir = 0; ir < K + RB - 1; ++ir) {           // staged rows r0 .. r0+K+RB-2
+        const float4* row = reinterpret_cast<const float4*>(rows_base + (r0 + ir) * ST_COLS + 4 * c4);
         float4 q0 = row[0], q1 = row[1], q2 = row[2];
         const float win[12] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w, q2.x, q2.y, q2.z, q2.w};
 #pragma unroll
-        for (int dx = 0; dx < K; ++dx) {
-            const float wt = p.w[dy * K + dx];
+        for (int j = 0; j < RB; ++j) {
+            const int dy = ir - j;                        // tap row of output row r0+j
+            if (dy < 0 || dy >= K) continue;
 #pragma unroll
-            for (int e = 0; e < 4; ++e) acc[e] = fmaf(wt, win[4 + e + dx - R], acc[e]);
+            for (int dx = 0; dx < K; ++dx) {
+                const float wt = p.w[dy * K + dx];
+#pragma unroll
+                for (int e = 0; e < 4; ++e) acc[j][e] = fmaf(wt, win[4 + e + dx - R], acc[j][e]);
+            }
         }
     }
-    if (gy >= p.rows || gx >= p.cols) return;
-    const bool row_in = gy >= R && gy < p.rows - R;
-    float4 o;
-    o.x = (row_in && gx + 0 >= R && gx + 0 < p.cols - R) ? acc[0] : 0.f;
-    o.y = (row_in && gx + 1 >= R && gx + 1 < p.cols - R) ? acc[1] : 0.f;
-    o.z = (row_in && gx + 2 >= R && gx + 2 < p.cols - R) ? acc[2] : 0.f;
-    o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[3] : 0.f;
-    store4_masked(p.out + (int64_t)gy * p.ld + gx, o, gx, p.cols);
+    if (gx >= p.cols) return;
+#pragma unroll
+    for (int j = 0; j < RB; ++j) {
+        const int gy = by * 32 + r0 + j;
+        if (gy >= p.rows) break;
+        const bool row_in = gy >= R && gy < p.rows - R;
+        float4 o;
+        o.x = (row_in && gx + 0 >= R && gx + 0 < p.cols - R) ? acc[j][0] : 0.f;
+        o.y = (row_in && gx + 1 >= R && gx + 1 < p.cols - R) ? acc[j][1] : 0.f;
+        o.z = (row_in && gx + 2 >= R && gx + 2 < p.cols - R) ? acc[j][2] : 0.f;
+        o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[j][3] : 0.f;
+        store4_masked(p.out + (int64_t)gy * p.ld + gx, o, gx, p.cols);
+    }
 }
 
 template <int R>
 struct Conv2dBody {
-    static constexpr int kConsumers = 256;
+    static constexpr int RB = 2;                  // output rows per consumer thread
+    static constexpr int kConsumers = 256 / RB;
     static constexpr int kStageBytes = HaloTile<R>::kBytes;
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
-    static constexpr int kMinAgents = 6;
+    static constexpr int kMinAgents = 8;
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
@@ -202,11 +223,11 @@ struct Conv2dBody {
                 s_in[rr][cc] = v;
             }
             consumer_sync<kConsumers>();
-            conv_tile_compute<R>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid);
+            conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid);
             consumer_sync<kConsumers>();                 // s_in is rewritten by the next task
             return;
         }
-        conv_tile_compute<R>(p, reinterpret_cast<const float*>(stage), bx, by, ctid);
+        conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid);
     }
     __device__ __forceinline__ void finish(int) {}
 };
