@@ -137,9 +137,11 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const void* tmap, int32_t
                  :: "r"(smem_u32(dst)), "l"(tmap), "r"(x), "r"(y), "r"(smem_u32(bar)) : "memory");
 }
 // named barrier among the consumer warps only (the producer warp never joins)
+// (barrier 1 + g for consumer group g of N threads; groups never share one)
 template <int N>
 __device__ __forceinline__ void consumer_sync() {
-    asm volatile("bar.sync 1, %0;" :: "n"(N) : "memory");
+    const int id = 1 + (int)(threadIdx.x - 32) / N;
+    asm volatile("bar.sync %0, %1;" :: "r"(id), "n"(N) : "memory");
 }
 
 // Stage protocol for Body::produce (warp 0, all lanes): the full barrier has
@@ -314,22 +316,29 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             if (s.mode == MODE_IDENTITY && active) P.q = 0;
             s_active = active;
         }
-        // ---- producer ring
+        // ---- producer ring (task t -> slot t % S, consumed by group t % G)
         int st = 0;
         uint32_t ph = 0;                                       // empty-barrier parity
-        for (int32_t t = 0;; ++t) {
+        int32_t t = 0;
+        for (;; ++t) {
             if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
             const int32_t v = producer_next(s, P, lane);
             if (lane == 0) R.slot[st] = v;
-            if (v < 0) {
-                __syncwarp();
-                if (lane == 0) mbar_arrive(&R.full[st]);        // end marker
-                break;
-            }
+            if (v < 0) break;
             int32_t lin, bx, by;
             lin_to_bxby(s, v, &lin, &bx, &by);
             body.produce(s, bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
             if (++st == S) { st = 0; ph ^= 1u; }
+        }
+        // one end marker per consumer group: slots t .. t+G-1
+        for (int k = 0; k < Body::kGroups; ++k) {
+            if (k > 0) {
+                if (++st == S) { st = 0; ph ^= 1u; }
+                if (t + k >= S) mbar_wait(&R.empty[st], ph ^ 1u);
+                if (lane == 0) R.slot[st] = -1;
+            }
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&R.full[st]);
         }
         // ---- the last agent out resets the workspace for the next launch.  Every
         // other agent's producer has consumed the results of all its atomics
@@ -344,9 +353,10 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             for (int32_t k = lane; k < n; k += 32) s.ws[k] = 0;
         }
     } else {
-        const int ctid = threadIdx.x - PRODUCER_THREADS;
-        int st = 0;
-        uint32_t ph = 0;                                       // full-barrier parity
+        const int grp = (threadIdx.x - PRODUCER_THREADS) / Body::kConsumers;
+        const int ctid = (threadIdx.x - PRODUCER_THREADS) % Body::kConsumers;
+        int st = grp;                                          // group g takes tasks g, g+G, ...
+        uint32_t ph = 0;                                       // full-barrier parity (G <= S)
         for (;;) {
             mbar_wait(&R.full[st], ph);
             const int32_t v = R.slot[st];
@@ -357,7 +367,8 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             if (ctid == 0) record(s, v, lin);
             __syncwarp();
             if (lane == 0) mbar_arrive(&R.empty[st]);
-            if (++st == S) { st = 0; ph ^= 1u; }
+            st += Body::kGroups;
+            if (st >= S) { st -= S; ph ^= 1u; }
         }
         if (s_active) body.finish(ctid);
     }
@@ -389,7 +400,7 @@ __device__ __forceinline__ void one_shot(const Sched& s, Body& body, int32_t v, 
 
 // ---- kernels: one per (body, backend) ------------------------------------
 template <class Body>
-__global__ void __launch_bounds__(Body::kConsumers + PRODUCER_THREADS, Body::kMinAgents)
+__global__ void __launch_bounds__(Body::kGroups * Body::kConsumers + PRODUCER_THREADS, Body::kMinAgents)
 k_agent(const __grid_constant__ Sched s, const __grid_constant__ typename Body::Params p) {
     Body body(p);
     agent_loop(s, body);

@@ -298,6 +298,7 @@ struct CensusBody {   // empty body: binding, queues and census only
     static constexpr int kDefaultStages = 2;
     static constexpr int kDefaultBatch = 1;
     static constexpr int kMinAgents = 8;
+    static constexpr int kGroups = 1;
     using Params = CensusParams;
     __device__ __forceinline__ explicit CensusBody(const CensusParams&) {}
     __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) { stage_commit(full, lane, 0); }
@@ -350,7 +351,7 @@ static cc_status occupancy(int device, int stages, int* occ, bool direct = false
         int prev = 0, n = 0;
         CC_CUDA(cudaGetDevice(&prev));
         CC_CUDA(cudaSetDevice(device));
-        CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_agent<Body>, Body::kConsumers + PRODUCER_THREADS,
+        CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_agent<Body>, Body::kGroups * Body::kConsumers + PRODUCER_THREADS,
                                                               dyn_smem<Body>(stages, direct)));
         CC_CUDA(cudaSetDevice(prev));
         cache[device][stages][direct] = n > 0 ? n : -1;
@@ -420,7 +421,8 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         break;
     case CC_BACKEND_AGENT:
     case CC_BACKEND_AGENT_IDENTITY: {
-        const int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
+        int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
+        if (S < Body::kGroups) S = Body::kGroups;             // every consumer group needs a slot
         int occ = 0;
         CC_TRY(occupancy<Body>(c.p->device, S, &occ, direct));
         const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
@@ -429,7 +431,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
         s.stages = S;
         const int grid = c.p->facts->num_sms * maxa;
-        k_agent<Body><<<grid, threads, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
+        k_agent<Body><<<grid, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
         break;
     }
     default:

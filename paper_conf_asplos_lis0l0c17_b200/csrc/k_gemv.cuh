@@ -47,6 +47,7 @@ struct GemvBody {
     static constexpr int kDefaultStages = 2;
     static constexpr int kDefaultBatch = TC >= 256 ? 2 : 1;
     static constexpr int kMinAgents = 3;
+    static constexpr int kGroups = 1;
     static constexpr int CW = TC / 4;                    // float4 columns per row
     static constexpr int LPR = CW < 32 ? CW : 32;        // lanes per row
     static constexpr int FPL = CW / LPR;                 // float4 per lane per row

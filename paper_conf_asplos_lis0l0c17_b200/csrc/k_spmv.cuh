@@ -57,6 +57,7 @@ struct SpmvBody {
     static constexpr int kDefaultStages = 2;
     static constexpr int kDefaultBatch = 2;
     static constexpr int kMinAgents = 5;
+    static constexpr int kGroups = 1;
     using Params = SpmvParams;
     const SpmvParams& p;
     __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}

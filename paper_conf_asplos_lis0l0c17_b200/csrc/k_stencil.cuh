@@ -98,6 +98,7 @@ struct Jacobi5Body {
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
     static constexpr int kMinAgents = 6;
+    static constexpr int kGroups = 1;
     using Params = JacobiParams;
     const JacobiParams& p;   // __grid_constant__ kernel parameter
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
@@ -202,7 +203,8 @@ struct Conv2dBody {
     static constexpr int kStageBytes = HaloTile<R>::kBytes;
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
-    static constexpr int kMinAgents = 8;
+    static constexpr int kMinAgents = 5;
+    static constexpr int kGroups = 2;              // two 4-warp groups consume alternate tiles
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
