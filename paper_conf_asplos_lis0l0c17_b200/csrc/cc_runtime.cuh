@@ -140,8 +140,13 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const void* tmap, int32_t
 // (barrier 1 + g for consumer group g of N threads; groups never share one)
 template <int N>
 __device__ __forceinline__ void consumer_sync() {
-    const int id = 1 + (int)(threadIdx.x - 32) / N;
-    asm volatile("bar.sync %0, %1;" :: "r"(id), "n"(N) : "memory");
+    // literal ids, so ptxas reserves only the barriers actually used
+    switch ((int)(threadIdx.x - 32) / N) {
+    case 0: asm volatile("bar.sync 1, %0;" :: "n"(N) : "memory"); break;
+    case 1: asm volatile("bar.sync 2, %0;" :: "n"(N) : "memory"); break;
+    case 2: asm volatile("bar.sync 3, %0;" :: "n"(N) : "memory"); break;
+    default: asm volatile("bar.sync 4, %0;" :: "n"(N) : "memory"); break;
+    }
 }
 
 // Stage protocol for Body::produce (warp 0, all lanes): the full barrier has
