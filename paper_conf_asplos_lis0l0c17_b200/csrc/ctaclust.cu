@@ -478,8 +478,6 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     if (g.V == 0) return CC_OK;
     const int C = c.o->cluster_size;
     if (C != 1 && C != 2 && C != 4 && C != 8) return fail(CC_ERR_INVALID_ARG, "cluster_size %d (1, 2, 4 or 8)", C);
-    const int gy_pad = (g.gy + C - 1) / C * C;
-    if (gy_pad > 65535) return fail(CC_ERR_UNSUPPORTED, "tbcluster: gy %d too large", g.gy);
     CUtensorMap m_rows, m_halo;
     CC_TRY(make_tmap(&m_rows, prm.in, prm.rows, prm.cols, prm.ld, TBC_COLS, 32));
     CC_TRY(make_tmap(&m_halo, prm.in, prm.rows, prm.cols, prm.ld, TBC_COLS, TBC_HALO));
@@ -489,18 +487,26 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     s.exec_sm = c.o->d_exec_sm;
     const size_t smem = tbc_smem_bytes(C);
     CC_CUDA(cudaFuncSetAttribute(k_conv_tbc<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CC_CUDA(cudaFuncSetAttribute(k_conv_tbc<R>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(g.gx, gy_pad);
-    cfg.blockDim = dim3(256);
+    cfg.blockDim = dim3(TBC_THREADS);
     cfg.dynamicSmemBytes = smem;
     cfg.stream = c.st;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeClusterDimension;
-    at[0].val.clusterDim.x = 1;
-    at[0].val.clusterDim.y = C;
+    at[0].val.clusterDim.x = C;
+    at[0].val.clusterDim.y = 1;
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
+    // persistent: as many clusters as can be co-resident (not more than units)
+    const long units = (long)g.gx * ((g.gy + C - 1) / C);
+    cfg.gridDim = dim3(C);
+    int nc = 0;
+    CC_CUDA(cudaOccupancyMaxActiveClusters(&nc, k_conv_tbc<R>, &cfg));
+    if (nc < 1) return fail(CC_ERR_UNSUPPORTED, "tbcluster: no cluster of %d fits", C);
+    if (nc > units) nc = (int)units;
+    cfg.gridDim = dim3(nc * C);
     CC_CUDA(cudaLaunchKernelEx(&cfg, k_conv_tbc<R>, m_rows, m_halo, s, prm, (int32_t)C));
     if (c.nl) ++*c.nl;
     return CC_OK;
