@@ -101,12 +101,15 @@ __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
 __device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
+// The suspend-time hint lets a waiting warp sleep in hardware until the phase
+// completes (or the hint expires) instead of re-issuing try_wait: spinning
+// consumer warps otherwise eat the issue slots the working warps need.
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile(
         "{\n\t.reg .pred p;\n"
         "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n}" :: "r"(smem_u32(bar)), "r"(parity) : "memory");
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+        "@!p bra WAIT_%=;\n}" :: "r"(smem_u32(bar)), "r"(parity), "r"(1000000u) : "memory");
 }
 // 1D bulk async copy global -> shared, completion counted on `bar` (UBLKCP).
 // dst, src 16-byte aligned, bytes a multiple of 16.
