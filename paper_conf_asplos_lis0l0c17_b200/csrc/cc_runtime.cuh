@@ -283,7 +283,7 @@ __device__ __forceinline__ int32_t producer_next(const Sched& s, Prod& P, int la
 struct RingShared {
     uint64_t full[MAX_STAGES];
     uint64_t empty[MAX_STAGES];
-    int32_t slot[MAX_STAGES];
+    int4 slot[MAX_STAGES];       // (v, lin, bx, by) decoded once by the scheduler warp
 };
 
 __device__ __forceinline__ uint8_t* ring_base(uint8_t* dyn) {
@@ -331,10 +331,13 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         for (;; ++t) {
             if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
             const int32_t v = producer_next(s, P, lane);
-            if (lane == 0) R.slot[st] = v;
-            if (v < 0) break;
+            if (v < 0) {
+                if (lane == 0) R.slot[st] = make_int4(-1, 0, 0, 0);
+                break;
+            }
             int32_t lin, bx, by;
             lin_to_bxby(s, v, &lin, &bx, &by);
+            if (lane == 0) R.slot[st] = make_int4(v, lin, bx, by);
             body.produce(s, bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
             if (++st == S) { st = 0; ph ^= 1u; }
         }
@@ -343,7 +346,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             if (k > 0) {
                 if (++st == S) { st = 0; ph ^= 1u; }
                 if (t + k >= S) mbar_wait(&R.empty[st], ph ^ 1u);
-                if (lane == 0) R.slot[st] = -1;
+                if (lane == 0) R.slot[st] = make_int4(-1, 0, 0, 0);
             }
             __syncwarp();
             if (lane == 0) mbar_arrive(&R.full[st]);
@@ -367,12 +370,10 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         uint32_t ph = 0;                                       // full-barrier parity (G <= S)
         for (;;) {
             mbar_wait(&R.full[st], ph);
-            const int32_t v = R.slot[st];
-            if (v < 0) break;
-            int32_t lin, bx, by;
-            lin_to_bxby(s, v, &lin, &bx, &by);
-            body.consume(s, bx, by, ring + (size_t)st * s.stage_bytes, ctid);
-            if (ctid == 0) record(s, v, lin);
+            const int4 sl = R.slot[st];
+            if (sl.x < 0) break;
+            body.consume(s, sl.z, sl.w, ring + (size_t)st * s.stage_bytes, ctid);
+            if (ctid == 0) record(s, sl.x, sl.y);
             __syncwarp();
             if (lane == 0) mbar_arrive(&R.empty[st]);
             st += Body::kGroups;
