@@ -239,20 +239,30 @@ __device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* 
 }
 
 // warp-parallel scan for a queue with unclaimed slots, nearest first from home.
+// Each lane issues all its head loads (8 rounds of 32 queues) before any ballot,
+// so a scan over up to 256 clusters costs one L2 round trip, not one per round.
 __device__ __forceinline__ int32_t steal_scan(const Sched& s, int32_t home, int lane) {
     const int32_t M = s.g.M;
-    for (int32_t base = 0; base < M; base += 32) {
-        int32_t k = base + lane;
-        bool avail = false;
-        int32_t q = -1;
-        if (k < M) {
-            q = home + 1 + k;
-            q -= (q >= M) ? M : 0;
-            q -= (q >= M) ? M : 0;
-            avail = ld_relaxed(ws_head(s) + q) < cluster_size(s.g, q);
+    for (int32_t base = 0; base < M; base += 256) {
+        int32_t h[8], q[8];
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            const int32_t k = base + r * 32 + lane;
+            q[r] = -1;
+            h[r] = 0;
+            if (k < M) {
+                int32_t qq = home + 1 + k;
+                qq %= M;
+                q[r] = qq;
+                h[r] = ld_relaxed(ws_head(s) + qq);
+            }
         }
-        uint32_t m = __ballot_sync(0xffffffffu, avail);
-        if (m) return __shfl_sync(0xffffffffu, q, __ffs(m) - 1);
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            const bool avail = q[r] >= 0 && h[r] < cluster_size(s.g, q[r]);
+            const uint32_t m = __ballot_sync(0xffffffffu, avail);
+            if (m) return __shfl_sync(0xffffffffu, q[r], __ffs(m) - 1);
+        }
     }
     return -1;
 }
