@@ -9,8 +9,8 @@ HDRS := $(wildcard $(SRC)/*.cuh) include/ctaclust.h
 
 all: $(LIB) oracle/liboracle.so
 
-$(LIB): $(SRC)/ctaclust.cu $(HDRS)
-	$(NVCC) $(NVFLAGS) -shared -o $@ $(SRC)/ctaclust.cu 2> build_ptxas.log || (cat build_ptxas.log; exit 1)
+$(LIB): $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu $(HDRS)
+	$(NVCC) $(NVFLAGS) -shared -o $@ $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu -ldl 2> build_ptxas.log || (cat build_ptxas.log; exit 1)
 
 oracle/liboracle.so: oracle/oracle.c
 	gcc -O2 -fPIC -shared -std=c11 -o $@ $<

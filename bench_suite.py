@@ -111,7 +111,9 @@ def suite_matvec(quick):
     A = synth.matrix(1, n, n, backend="torch", device="cuda")
     x = synth.uniform(2, n, backend="torch", device="cuda")
     y = torch.zeros(n, device="cuda")
-    v = variants_for("row") + [("agent-col", dict(backend="agent", order="col"))]
+    v = variants_for("row") + [("agent-col", dict(backend="agent", order="col")),
+                               ("agent-row-m1s4b4", dict(backend="agent", order="row", max_agents=1, stages=4, batch=4)),
+                               ("agent-row-m2s3b2", dict(backend="agent", order="row", max_agents=2, stages=3, batch=2))]
     r = measure(v, lambda kw: ops.matvec(A, x, y, **kw), 20 if quick else 50, 4 * n * n + 8 * n, inner=50, graph=True)
     r["config"] = "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident; 50 launches per CUDA graph"
     return r

@@ -229,6 +229,32 @@ cc_status cc_max_agents(int32_t kernel, int32_t device, int32_t* max_agents);
 cc_status cc_launch(cc_plan plan, int32_t kernel, const void* args,
                     const cc_launch_opts* opts, void* stream, int32_t* launches);
 
+/* ---------------------------------------------------------------------------
+ * Multi-GPU exchange steps (S§8(e)): one process per GPU, NCCL over NVLink /
+ * NVSwitch.  NCCL is resolved at run time (the copy the process already maps,
+ * e.g. PyTorch's, or the file named by CC_NCCL_LIBRARY); without it these
+ * return CC_ERR_UNSUPPORTED.  All are asynchronous on `stream`.
+ * ------------------------------------------------------------------------- */
+typedef struct cc_comm_s* cc_comm;
+/* Rank 0 creates the 128-byte NCCL unique id (HOST out) and shares it with the
+ * other ranks out of band (e.g. a torch.distributed broadcast). */
+cc_status cc_comm_unique_id(void* id128);
+/* Collective over all ranks: communicator of `nranks`, this process is `rank`
+ * on CUDA `device`.  Errors: INVALID_ARG, UNSUPPORTED (no NCCL), NCCL. */
+cc_status cc_comm_init(const void* id128, int32_t nranks, int32_t rank, int32_t device, cc_comm* comm);
+cc_status cc_comm_destroy(cc_comm comm);
+/* Slab halo exchange for the sharded stencils: `slab` (DEVICE, rows x cols fp32,
+ * leading dim ld) holds this rank's owned rows plus `halo` rows above (unless
+ * rank 0) and below (unless the last rank); the halo rows are overwritten with
+ * the neighbours' owned boundary rows (one grouped send/recv per neighbour). */
+cc_status cc_halo_exchange(cc_comm comm, float* slab, int64_t ld, int32_t rows, int32_t cols, int32_t halo,
+                           void* stream);
+/* In-place sum over ranks of `count` fp32 (DEVICE): the transposed products of
+ * the row-sharded ATAX family. */
+cc_status cc_allreduce_sum(cc_comm comm, float* buf, size_t count, void* stream);
+/* Gather `count_per_rank` fp32 from every rank, rank-major into recv (DEVICE). */
+cc_status cc_allgather(cc_comm comm, const float* send, float* recv, size_t count_per_rank, void* stream);
+
 /* Messages. */
 const char* cc_status_string(cc_status s);
 const char* cc_last_error(void);       /* thread-local detail of the last failure */

@@ -39,6 +39,9 @@ static cc_status fail(cc_status s, const char* fmt, ...) {
     g_err = buf;
     return s;
 }
+extern "C" __attribute__((visibility("hidden"))) cc_status cc_internal_fail(cc_status s, const char* msg) {
+    return fail(s, "%s", msg);
+}
 static cc_status cuda_fail(cudaError_t e, const char* what) {
     g_cuda_err = (int)e;
     cudaGetLastError();   // clear sticky-free errors

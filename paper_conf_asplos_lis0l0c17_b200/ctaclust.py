@@ -30,8 +30,9 @@ STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_E
 # every symbol include/ctaclust.h declares (checked by tests/test_abi.py)
 EXPORTS = ["cc_plan_create", "cc_plan_destroy", "cc_plan_info", "cc_plan_table", "cc_plan_lookup",
            "cc_plan_invert", "cc_device_info", "cc_sm_rank_table", "cc_launch_opts_default",
-           "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_status_string",
-           "cc_last_error", "cc_last_cuda_error", "cc_version"]
+           "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_comm_unique_id",
+           "cc_comm_init", "cc_comm_destroy", "cc_halo_exchange", "cc_allreduce_sum", "cc_allgather",
+           "cc_status_string", "cc_last_error", "cc_last_cuda_error", "cc_version"]
 
 
 class CtaclustError(RuntimeError):
@@ -277,3 +278,45 @@ def spmv_args(row_ptr, col, val, x, y, part=None) -> SpmvArgs:
 
 def spmv_partition(args: SpmvArgs, part, stream=None):
     _check(lib().cc_spmv_partition(ctypes.byref(args), _vp(part.data_ptr()), _vp(_stream(stream))))
+
+
+# ---- multi-GPU exchange steps (NCCL, one process per GPU) ---------------------
+class Comm:
+    """cc_comm: an NCCL communicator owned by the library.  Rank 0 creates the
+    unique id (`Comm.unique_id()`), shares it out of band (torch.distributed
+    broadcast), then every rank constructs `Comm(uid, nranks, rank, device)`."""
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = ctypes.create_string_buffer(128)
+        _check(lib().cc_comm_unique_id(buf))
+        return buf.raw
+
+    def __init__(self, uid: bytes, nranks: int, rank: int, device: int = 0):
+        h = _vp()
+        idb = ctypes.create_string_buffer(bytes(uid), 128)
+        _check(lib().cc_comm_init(idb, _i32(nranks), _i32(rank), _i32(device), ctypes.byref(h)))
+        self.handle, self.nranks, self.rank = h, nranks, rank
+
+    def halo_exchange(self, slab, halo: int, stream=None):
+        """Refresh the halo rows of a local slab (rows x cols, row-major torch tensor)."""
+        _check(lib().cc_halo_exchange(self.handle, _vp(slab.data_ptr()), _i64(slab.stride(0)), _i32(slab.shape[0]),
+                                      _i32(slab.shape[1]), _i32(halo), _vp(_stream(stream))))
+
+    def allreduce_sum(self, t, stream=None):
+        _check(lib().cc_allreduce_sum(self.handle, _vp(t.data_ptr()), ctypes.c_size_t(t.numel()), _vp(_stream(stream))))
+
+    def allgather(self, send, recv, stream=None):
+        _check(lib().cc_allgather(self.handle, _vp(send.data_ptr()), _vp(recv.data_ptr()),
+                                  ctypes.c_size_t(send.numel()), _vp(_stream(stream))))
+
+    def close(self):
+        if getattr(self, "handle", None):
+            lib().cc_comm_destroy(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
