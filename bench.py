@@ -170,6 +170,13 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    comm = None
+    if world > 1:
+        # the library's own NCCL communicator (cc_comm_*); torch.distributed only
+        # carries the unique id
+        box = [cc.Comm.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(box, src=0)
+        comm = cc.Comm(box[0], world, rank, local)
     dev = torch.device("cuda", local)
     n = a.n
     lo, hi = shard.row_range(n, world, rank)
@@ -201,8 +208,8 @@ def main():
         nl += cc.launch(pl, "mvt", cc.mvt_args(A, y1, y2, x1, x2), cc.make_opts(**kw), stream)
         if ev is not None: ev[3].record(stream)
         if world > 1:
-            for t_ in (y, s, x2):
-                dist.all_reduce(t_)
+            for t_ in (y, s, x2):                    # transposed products: one sum over ranks
+                comm.allreduce_sum(t_, stream)
         if count is not None:
             count[0] += nl
 
