@@ -93,12 +93,13 @@ __device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, 
 }
 
 struct Jacobi5Body {
-    static constexpr int kConsumers = 256;
+    static constexpr int RB = 2;                  // output rows per consumer thread
+    static constexpr int kConsumers = 256 / RB;
     static constexpr int kStageBytes = HaloTile<1>::kBytes;
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
-    static constexpr int kMinAgents = 6;
-    static constexpr int kGroups = 1;
+    static constexpr int kMinAgents = 4;
+    static constexpr int kGroups = 2;              // two 4-warp groups consume alternate tiles
     using Params = JacobiParams;
     const JacobiParams& p;   // __grid_constant__ kernel parameter
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
@@ -107,33 +108,51 @@ struct Jacobi5Body {
         HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap);
     }
 
+    // thread (rows r0 .. r0+RB-1, columns 4*c4 .. 4*c4+3): the RB+2 input rows
+    // it touches are read once each
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
-        const int r = ctid >> 3, c4 = ctid & 7;
-        const int gy = by * 32 + r, gx = bx * 32 + 4 * c4;
-        const bool in = gy < p.rows && gx < p.cols;
-        float4 c, up, dn;
-        float lw, re;
+        const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
+        const int gx = bx * 32 + 4 * c4;
+        const int gy0 = by * 32 + r0;
+        const bool in_col = gx < p.cols;
+        float4 row[RB + 2];                        // input rows gy0-1 .. gy0+RB
+        float lw[RB], re[RB];
         if (s.staging == STAGE_DIRECT) {
-            // plain-kernel form: every load goes through L1 (rows r-1 / r+1 of
-            // the tile are other threads' centre rows -> L1 hits)
-            const float* a = p.a + (int64_t)gy * p.ld + gx;
-            c = in ? ld_cached4(a) : f4_zero();
-            up = (in && gy > 0) ? ld_cached4(a - p.ld) : f4_zero();
-            dn = (in && gy + 1 < p.rows) ? ld_cached4(a + p.ld) : f4_zero();
-            lw = __shfl_up_sync(0xffffffffu, c.w, 1, 8);
-            re = __shfl_down_sync(0xffffffffu, c.x, 1, 8);
-            if (c4 == 0) lw = (in && gx > 0) ? ld_cached(a - 1) : 0.f;
-            if (c4 == 7) re = (in && gx + 4 < p.cols) ? ld_cached(a + 4) : 0.f;
+            // plain-kernel form: every load goes through L1 (neighbouring rows are
+            // other threads' rows -> L1 hits)
+            const float* a = p.a + (int64_t)gy0 * p.ld + gx;
+#pragma unroll
+            for (int k = 0; k < RB + 2; ++k) {
+                const int gy = gy0 - 1 + k;
+                row[k] = (in_col && gy >= 0 && gy < p.rows) ? ld_cached4(a + (int64_t)(k - 1) * p.ld) : f4_zero();
+            }
+#pragma unroll
+            for (int j = 0; j < RB; ++j) {
+                const int gy = gy0 + j;
+                lw[j] = __shfl_up_sync(0xffffffffu, row[j + 1].w, 1, 8);
+                re[j] = __shfl_down_sync(0xffffffffu, row[j + 1].x, 1, 8);
+                const bool in = in_col && gy < p.rows;
+                if (c4 == 0) lw[j] = (in && gx > 0) ? ld_cached(a + (int64_t)j * p.ld - 1) : 0.f;
+                if (c4 == 7) re[j] = (in && gx + 4 < p.cols) ? ld_cached(a + (int64_t)j * p.ld + 4) : 0.f;
+            }
         } else {
-            const float* mid = reinterpret_cast<const float*>(stage) + (r + 1) * ST_COLS + 4 + 4 * c4;
-            c = *reinterpret_cast<const float4*>(mid);
-            up = *reinterpret_cast<const float4*>(mid - ST_COLS);
-            dn = *reinterpret_cast<const float4*>(mid + ST_COLS);
-            lw = mid[-1];
-            re = mid[4];
+            const float* t = reinterpret_cast<const float*>(stage) + r0 * ST_COLS + 4 + 4 * c4;   // staged row r0 = gy0-1
+#pragma unroll
+            for (int k = 0; k < RB + 2; ++k) row[k] = *reinterpret_cast<const float4*>(t + k * ST_COLS);
+#pragma unroll
+            for (int j = 0; j < RB; ++j) {
+                lw[j] = t[(j + 1) * ST_COLS - 1];
+                re[j] = t[(j + 1) * ST_COLS + 4];
+            }
         }
-        if (!in) return;
-        store4_masked(p.b + (int64_t)gy * p.ld + gx, jacobi_point4(c, up, dn, lw, re, gy, gx, p.rows, p.cols), gx, p.cols);
+        if (!in_col) return;
+#pragma unroll
+        for (int j = 0; j < RB; ++j) {
+            const int gy = gy0 + j;
+            if (gy >= p.rows) break;
+            store4_masked(p.b + (int64_t)gy * p.ld + gx,
+                          jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx, p.cols);
+        }
     }
     __device__ __forceinline__ void finish(int) {}
 };
