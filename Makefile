@@ -4,7 +4,7 @@ PKG := paper_conf_asplos_lis0l0c17_b200
 SRC := $(PKG)/csrc
 LIB := $(PKG)/libctaclust.so
 NVFLAGS := -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo \
-           -Xcompiler -fPIC -Xcompiler -Wall -Xptxas -v --expt-relaxed-constexpr -I include
+           -Xcompiler -fPIC -Xcompiler -Wall -Xptxas -v --expt-relaxed-constexpr -I include $(CC_DEFS)
 HDRS := $(wildcard $(SRC)/*.cuh) include/ctaclust.h
 
 all: $(LIB) oracle/liboracle.so

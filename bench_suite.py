@@ -65,7 +65,11 @@ def graph_ms(fn, reps, inner):
     return time_ms(g.replay, reps, warm=1) / inner
 
 
-def measure(variants, fn, reps, nbytes, extra=None, warm=3, inner=1, graph=False):
+def measure(variants, fn, reps, nbytes, extra=None, warm=3, inner=1, graph=False, context=None):
+    """`context`: {name: callable} vendor-library timings of the same
+    computation (cuBLAS / cuDNN / cuSPARSE via torch), reported as lib-* rows
+    for absolute context; they are not part of the default/clustered
+    comparison."""
     rows = []
     for name, kw in variants:
         ms = graph_ms(lambda: fn(kw), reps, inner) if graph else time_ms(lambda: fn(kw), reps, warm=warm, inner=inner)
@@ -74,8 +78,18 @@ def measure(variants, fn, reps, nbytes, extra=None, warm=3, inner=1, graph=False
         if extra:
             d.update(extra(ms))
         rows.append(d)
+    for name, cfn in (context or {}).items():
+        try:
+            ms = graph_ms(cfn, reps, inner) if graph else time_ms(cfn, reps, warm=warm, inner=inner)
+            gbs = nbytes / (ms * 1e-3) / 1e9
+            rows.append({"variant": "lib-" + name, "ms": round(ms, 5), "GBps": round(gbs, 1),
+                         "frac_hbm": round(gbs / _peak(), 4)})
+        except Exception as e:  # context only
+            rows.append({"variant": "lib-" + name, "error": repr(e)[:200]})
     best_def = min(r["ms"] for r in rows if r["variant"].startswith("default"))
     for r in rows:
+        if "ms" not in r:
+            continue
         r["speedup_vs_best_default"] = round(best_def / r["ms"], 4)
     return {"bytes": nbytes, "best_default_ms": best_def, "rows": rows}
 
@@ -114,7 +128,8 @@ def suite_matvec(quick):
     v = variants_for("row") + [("agent-col", dict(backend="agent", order="col")),
                                ("agent-row-m1s4b4", dict(backend="agent", order="row", max_agents=1, stages=4, batch=4)),
                                ("agent-row-m2s3b2", dict(backend="agent", order="row", max_agents=2, stages=3, batch=2))]
-    r = measure(v, lambda kw: ops.matvec(A, x, y, **kw), 20 if quick else 50, 4 * n * n + 8 * n, inner=50, graph=True)
+    r = measure(v, lambda kw: ops.matvec(A, x, y, **kw), 20 if quick else 50, 4 * n * n + 8 * n, inner=50, graph=True,
+                context={"cublas-mv": lambda: torch.mv(A, x, out=y)})
     r["config"] = "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident; 50 launches per CUDA graph"
     return r
 
@@ -135,7 +150,10 @@ def suite_atax(quick):
     }
     variants = variants_for("col") + [("agent-row", dict(backend="agent", order="row")),
                                       ("agent-col-s3", dict(backend="agent", order="col", stages=3))]
-    out = {k: measure(variants, fn, 5 if quick else 15, nb) for k, (fn, nb) in kernels.items()}
+    ctx = {"atax": {"cublas-2xmv": lambda: torch.mv(A.t(), torch.mv(A, x, out=tmp), out=y)},
+           "bicg": {"cublas-2xmv": lambda: (torch.mv(A, p, out=q), torch.mv(A.t(), r, out=s))},
+           "mvt": {"cublas-2xmv": lambda: (x1.add_(torch.mv(A, y1)), x2.add_(torch.mv(A.t(), y2)))}}
+    out = {k: measure(variants, fn, 5 if quick else 15, nb, context=ctx[k]) for k, (fn, nb) in kernels.items()}
     return {"config": "PolyBench ATAX/BICG/MVT fp32 n=16384, 32x256 tiles (64x512 grid)", "kernels": out}
 
 
@@ -166,9 +184,12 @@ def suite_conv(quick):
             ("tbcluster-2", dict(backend="tbcluster", cluster_size=2)),
             ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
             ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))]
+        wt = torch.from_numpy(w).cuda().view(1, 1, 2 * R + 1, 2 * R + 1)
+        img4 = img.view(1, 1, N, N)
         res[f"{2 * R + 1}x{2 * R + 1}"] = measure(
             v, lambda kw: ops.conv2d(img, w, out=out, **kw), 5 if quick else 20, 8 * N * N,
-            extra=lambda ms: {"TFLOPs": round(flops / (ms * 1e-3) / 1e12, 2)})
+            extra=lambda ms: {"TFLOPs": round(flops / (ms * 1e-3) / 1e12, 2)},
+            context={"cudnn-conv2d": lambda: torch.nn.functional.conv2d(img4, wt)})
         res[f"{2 * R + 1}x{2 * R + 1}"]["flops"] = flops
     return {"config": f"2D conv fp32 {N}x{N}, 32x32 tiles (256x256 grid)", "filters": res}
 
@@ -191,9 +212,14 @@ def suite_spmv(quick):
                 ("agent-row-tot2", dict(backend="agent", order="row", active_agents=2)),
                 ("agent-row-tot4", dict(backend="agent", order="row", active_agents=4)),
                 ("agent-row-b8", dict(backend="agent", order="row", batch=8)),
-                ("identity", dict(backend="identity")), ("redirect-row", dict(backend="redirect", order="row"))]
+                ("agent-row-s1", dict(backend="agent", order="row", stages=1)),
+                ("agent-row-s4", dict(backend="agent", order="row", stages=4)),
+                ("identity", dict(backend="identity")), ("identity-s1", dict(backend="identity", stages=1)),
+                ("redirect-row", dict(backend="redirect", order="row"))]
+    Acsr = torch.sparse_csr_tensor(rp, col, val, (rows_n, rows_n))
     r = measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 5 if quick else 20,
-                8 * nnz + 4 * (rows_n + 1) + 8 * rows_n)
+                8 * nnz + 4 * (rows_n + 1) + 8 * rows_n,
+                context={"cusparse-spmv": lambda: torch.mv(Acsr, x)})
     r["config"] = f"CSR SpMV fp32 R-MAT scale {scale} ef 16: {rows_n} rows, {nnz} nnz (gen {gen_s:.1f}s)"
     return r
 
@@ -228,7 +254,11 @@ def table(path):
         for g, vv in groups.items():
             lines.append(f"== {g}  {v.get('config', '')}")
             for r in vv.get("rows", []):
-                lines.append(f"   {r['variant']:26s} {r['ms']:10.4f} ms {r['GBps']:8.1f} GB/s  frac {r['frac_hbm']:.3f}  x{r['speedup_vs_best_default']:.3f}")
+                if "ms" not in r:
+                    lines.append(f"   {r['variant']:26s} {r.get('error', '')}")
+                    continue
+                sp = r.get("speedup_vs_best_default")
+                lines.append(f"   {r['variant']:26s} {r['ms']:10.4f} ms {r['GBps']:8.1f} GB/s  frac {r['frac_hbm']:.3f}  x{sp:.3f}")
     return "\n".join(lines)
 
 

@@ -64,6 +64,18 @@ __device__ __forceinline__ float4 ld_cached4(const float* p) {
 }
 __device__ __forceinline__ float ld_cached(const float* p) { return *p; }
 
+// Scalar streaming loads (read once; do not displace reused lines from L1).
+__device__ __forceinline__ float ld_stream_f32(const float* p) {
+    float v;
+    asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ int32_t ld_stream_i32(const int32_t* p) {
+    int32_t v;
+    asm("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+
 // Bulk L2 prefetch of `bytes` (multiple of 16, 16-byte aligned) at p
 // (cp.async.bulk.prefetch.L2 -> UBLKPF.L2), the B200 form of PREFETCH_L1
 // (Listing 5 l.34-37).

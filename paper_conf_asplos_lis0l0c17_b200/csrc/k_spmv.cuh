@@ -11,6 +11,12 @@
 // (the rows it shares with its neighbours); every other row is a plain store.
 // The x gathers go through L1 (the data-dependent inter-CTA reuse the paper
 // calls hard to exploit); val/col stream past it.
+//
+// Shared memory is kept small on purpose: on sm_100a L1 and shared memory are
+// one 256 KB array per SM, and every KB of smem a resident CTA holds is a KB
+// of L1 the R-MAT hub columns of x cannot use.  Row ends are staged only when
+// the CTA's row range fits SPMV_ROWCAP (the common case: ~IPC/17 rows at 16
+// nnz/row); a CTA over a run of (near-)empty rows reads them from global.
 #pragma once
 #include "cc_mem.cuh"
 #include "cc_runtime.cuh"
@@ -23,9 +29,19 @@ struct SpmvParams {
     const int32_t* part;   // part[b] = row coordinate of diagonal b*IPC
 };
 
-constexpr int SPMV_IPT = 16;
+#ifndef CC_SPMV_IPT
+#define CC_SPMV_IPT 16
+#endif
+constexpr int SPMV_IPT = CC_SPMV_IPT;
 constexpr int SPMV_THREADS = 256;
 constexpr int SPMV_IPC = SPMV_IPT * SPMV_THREADS;   // merge items per logical CTA
+constexpr int SPMV_ROWCAP = 512;                    // staged row ends per CTA
+#ifndef CC_SPMV_PREFETCH
+#define CC_SPMV_PREFETCH 1
+#endif
+#ifndef CC_SPMV_MIN_AGENTS
+#define CC_SPMV_MIN_AGENTS 5
+#endif
 
 // Merge-path search (row ends a[0..a_len) vs natural numbers b[k] = k):
 // number of row ends consumed at diagonal d.
@@ -56,20 +72,39 @@ struct SpmvBody {
     static constexpr int kStageBytes = 128;       // nothing staged: reads go straight to L1/L2
     static constexpr int kDefaultStages = 2;
     static constexpr int kDefaultBatch = 2;
-    static constexpr int kMinAgents = 5;
+    static constexpr int kMinAgents = CC_SPMV_MIN_AGENTS;
     static constexpr int kGroups = 1;
     using Params = SpmvParams;
     const SpmvParams& p;
     __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}
 
-    __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) {
+    // Nothing is staged in smem (it would cost L1, see above).  Instead the
+    // producer warp -- in an agent, one or more tasks ahead of the consumers --
+    // prefetches the task's col / val runs (and its row_ptr range) from DRAM
+    // into L2, so the consumers' streaming loads and the x gathers that depend
+    // on them pay one L2 round trip rather than DRAM + L2: the paper's CTA
+    // prefetching (section 4.3(III), Listing 5 l.34-37), which the persistent
+    // agent's ordered task stream makes possible.
+    __device__ __forceinline__ void produce(const Sched&, int32_t bx, int32_t, uint8_t*, uint64_t* full, int lane) {
+        if (CC_SPMV_PREFETCH && lane < 3) {
+            const int64_t total = (int64_t)p.rows + p.nnz;
+            const int64_t d0 = (int64_t)bx * SPMV_IPC;
+            const int64_t d1 = d0 + SPMV_IPC < total ? d0 + SPMV_IPC : total;
+            const int32_t x0 = p.part[bx], x1 = p.part[bx + 1];
+            const int64_t lo = lane == 2 ? x0 : d0 - x0, hi = lane == 2 ? (int64_t)x1 + 2 : d1 - x1;
+            const char* base = lane == 0 ? (const char*)p.col : lane == 1 ? (const char*)p.val
+                                                                          : (const char*)p.row_ptr;
+            const uintptr_t a0 = ((uintptr_t)(base + 4 * lo)) & ~(uintptr_t)15;
+            const uintptr_t a1 = ((uintptr_t)(base + 4 * hi) + 15) & ~(uintptr_t)15;
+            if (hi > lo) prefetch_l2_bulk((const void*)a0, (uint32_t)(a1 - a0));
+        }
         stage_commit(full, lane, 0);
     }
 
     __device__ __forceinline__ void consume(const Sched&, int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
-        __shared__ int32_t s_rowend[SPMV_IPC + 1];
-        // products of the CTA's nonzeros, index j stored at j + j/16 (the pad
-        // keeps each thread's 16-long private run conflict-free)
+        __shared__ int32_t s_rowend[SPMV_ROWCAP];
+        // products of the CTA's nonzeros, index j stored at j + j/IPT (the pad
+        // keeps each thread's IPT-long private run conflict-free)
         __shared__ float s_prod[SPMV_IPC + SPMV_IPC / SPMV_IPT];
         __shared__ float s_wv[SPMV_THREADS / 32];
         __shared__ int32_t s_wf[SPMV_THREADS / 32];
@@ -80,7 +115,9 @@ struct SpmvBody {
         const int32_t x0 = p.part[bx], x1 = p.part[bx + 1];
         const int64_t y0 = d0 - x0, y1 = d1 - x1;
         const int32_t xl = x1 < p.rows ? x1 : p.rows - 1;      // last row to stage
-        for (int32_t i = t; i <= xl - x0; i += kConsumers) s_rowend[i] = p.row_ptr[x0 + i + 1];
+        const bool staged = xl - x0 < SPMV_ROWCAP;
+        if (staged)
+            for (int32_t i = t; i <= xl - x0; i += kConsumers) s_rowend[i] = p.row_ptr[x0 + i + 1];
         // all products of the CTA, coalesced: val/col stream past L1, the x
         // gathers go through it (16 independent loads per thread in flight)
         const int32_t nz = (int32_t)(y1 - y0);
@@ -88,43 +125,50 @@ struct SpmvBody {
         for (int k = 0; k < SPMV_IPT; ++k) {
             const int32_t j = t + k * kConsumers;
             if (j < nz) {
-                const int32_t c = __ldcs(p.col + y0 + j);
-                const float v = __ldcs(p.val + y0 + j);
-                s_prod[j + (j >> 4)] = v * ld_cached(p.x + c);
+                const int32_t c = ld_stream_i32(p.col + y0 + j);
+                const float v = ld_stream_f32(p.val + y0 + j);
+                s_prod[j + j / SPMV_IPT] = v * ld_cached(p.x + c);
             }
         }
         consumer_sync<kConsumers>();
         // this thread's start on the merge path, relative to the CTA rectangle
         const int32_t span = (int32_t)(d1 - d0);
         const int32_t dt = t * SPMV_IPT < span ? t * SPMV_IPT : span;
-        int32_t lo = dt - (int32_t)(y1 - y0); if (lo < 0) lo = 0;
-        int32_t hi = dt < (x1 - x0) ? dt : (x1 - x0);
-        while (lo < hi) {
-            int32_t pv = (lo + hi) >> 1;
-            if ((int64_t)s_rowend[pv] <= y0 + dt - pv - 1) lo = pv + 1;
-            else hi = pv;
-        }
-        const int32_t tx = x0 + lo;
-        const int64_t ty = y0 + dt - lo;
-        // merge walk over this thread's IPT items
         const int32_t items = span - dt < SPMV_IPT ? span - dt : SPMV_IPT;
         float sum = 0.f, first_val = 0.f;
         int32_t first_row = -1;
         bool has_end = false;
-        int32_t cx = tx;
-        int64_t cy = ty;
-        for (int it = 0; it < items; ++it) {
-            if (cx < p.rows && cy < (int64_t)s_rowend[cx - x0]) {
-                const int32_t j = (int32_t)(cy - y0);
-                sum += s_prod[j + (j >> 4)];
-                ++cy;
-            } else {
-                if (!has_end) { first_row = cx; first_val = sum; has_end = true; }
-                else p.y[cx] = sum;                 // row began and ended in this thread
-                sum = 0.f;
-                ++cx;
+        // search + merge walk over this thread's IPT items; instantiated once
+        // with the smem row ends (LDS) and once with the global ones
+        auto walk = [&](const int32_t* rowend) {
+            int32_t lo = dt - (int32_t)(y1 - y0); if (lo < 0) lo = 0;
+            int32_t hi = dt < (x1 - x0) ? dt : (x1 - x0);
+            while (lo < hi) {
+                int32_t pv = (lo + hi) >> 1;
+                if ((int64_t)rowend[pv] <= y0 + dt - pv - 1) lo = pv + 1;
+                else hi = pv;
             }
-        }
+            int32_t cx = x0 + lo;
+            int32_t cj = (int32_t)(dt - lo);                 // nonzero index relative to y0
+            int32_t re = cx < p.rows ? (int32_t)(rowend[cx - x0] - y0) : INT32_MIN;
+#pragma unroll
+            for (int it = 0; it < SPMV_IPT; ++it) {
+                if (it < items) {
+                    if (cj < re) {
+                        sum += s_prod[cj + cj / SPMV_IPT];
+                        ++cj;
+                    } else {
+                        if (!has_end) { first_row = cx; first_val = sum; has_end = true; }
+                        else p.y[cx] = sum;                 // row began and ended in this thread
+                        sum = 0.f;
+                        ++cx;
+                        re = cx < p.rows ? (int32_t)(rowend[cx - x0] - y0) : INT32_MIN;
+                    }
+                }
+            }
+        };
+        if (staged) walk(s_rowend);
+        else walk(p.row_ptr + x0 + 1);
         // segmented inclusive scan of (has_end, carry): T[t] = carry + (has_end ? 0 : T[t-1])
         bool f = has_end;
         float v = sum;

@@ -73,7 +73,11 @@ def main():
         x = synth.uniform(9, rp.numel() - 1, backend="torch", device=dev)
         Am = ops.SpmvMatrix(rp, col, val)
         y = torch.empty(rp.numel() - 1, device=dev)
-        fn = lambda: ops.spmv(Am, x, y, **kw)
+        if a.backend == "cusparse":          # vendor library, for context only
+            Acsr = torch.sparse_csr_tensor(rp, col, val, (rp.numel() - 1, rp.numel() - 1))
+            fn = lambda: torch.mv(Acsr, x)
+        else:
+            fn = lambda: ops.spmv(Am, x, y, **kw)
     else:
         raise SystemExit(f"unknown kernel {k}")
     torch.cuda.synchronize()
