@@ -256,6 +256,17 @@ def _edge_matrices():
     yield "all-empty", rp2, np.zeros(0, np.int64), 300
     rp3, col3 = synth.rmat_csr(7, 12, 16)
     yield "rmat12", rp3.astype(np.int64), col3, 1 << 12
+    # mostly-empty rows: every logical CTA spans > SPMV_ROWCAP rows, so the
+    # merge walk reads its row ends from global memory (k_spmv.cuh)
+    n4 = 100003
+    deg4 = np.zeros(n4, np.int64)
+    deg4[::37] = 2
+    rp4 = np.zeros(n4 + 1, np.int64); np.cumsum(deg4, out=rp4[1:])
+    k4 = int(deg4.sum()) // 2
+    c0 = (synth.uniform(12, k4) * (n4 - 1)).astype(np.int64)
+    c1 = (c0 + 1 + (synth.uniform(13, k4) * (n4 - 2)).astype(np.int64)) % n4   # != c0
+    col4 = np.sort(np.stack([c0, c1], 1), axis=1).reshape(-1)
+    yield "mostly-empty", rp4, col4, n4
 
 
 @pytest.mark.parametrize("v", SVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
