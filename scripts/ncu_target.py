@@ -28,6 +28,8 @@ def main():
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--warm", type=int, default=1)
     ap.add_argument("--scale", type=int, default=24)
+    ap.add_argument("--small", action="store_true",
+                    help="reduced problem (categorizer probe, P:2275): n/4 matrices, scale-18 SpMV")
     a = ap.parse_args()
     import torch
     from paper_conf_asplos_lis0l0c17_b200 import ops, synth
@@ -47,7 +49,7 @@ def main():
         y = torch.zeros(n, device=dev)
         fn = lambda: ops.matvec(A, x, y, **kw)
     elif k in ("atax", "bicg", "mvt"):
-        n = 16384
+        n = 4096 if a.small else 16384
         A = synth.matrix(3, n, n, backend="torch", device=dev)
         v = lambda s: synth.uniform(s, n, backend="torch", device=dev)
         x, p, r, y1, y2, x1, x2 = v(10), v(11), v(12), v(15), v(16), v(13), v(14)
@@ -56,19 +58,19 @@ def main():
               "bicg": lambda: ops.bicg(A, p, r, out=bufs, **kw),
               "mvt": lambda: ops.mvt(A, y1, y2, x1, x2, **kw)}[k]
     elif k == "jacobi":
-        N = 16384
+        N = 4096 if a.small else 16384
         a_ = synth.matrix(4, N, N, backend="torch", device=dev)
         b_ = torch.empty_like(a_)
         fn = lambda: ops.jacobi5(a_, b_, 1, **kw)
     elif k in ("conv3", "conv7"):
-        N, R = 8192, (1 if k == "conv3" else 3)
+        N, R = (2048 if a.small else 8192), (1 if k == "conv3" else 3)
         img = synth.matrix(5, N, N, backend="torch", device=dev)
         out = torch.empty_like(img)
         w = synth.uniform(6, (2 * R + 1) ** 2).reshape(2 * R + 1, 2 * R + 1)
         w = w / w.sum()
         fn = lambda: ops.conv2d(img, w, out=out, **kw)
     elif k == "spmv":
-        rp, col = synth.rmat_csr(7, a.scale, 16, backend="torch", device=dev)
+        rp, col = synth.rmat_csr(7, 18 if a.small else a.scale, 16, backend="torch", device=dev)
         val = synth.uniform(8, col.numel(), backend="torch", device=dev)
         x = synth.uniform(9, rp.numel() - 1, backend="torch", device=dev)
         Am = ops.SpmvMatrix(rp, col, val)
