@@ -216,6 +216,19 @@ typedef struct { int32_t rows, cols; int64_t nnz; const int32_t* row_ptr; const 
  * first diagonal.  Asynchronous on `stream`. */
 cc_status cc_spmv_partition(const cc_spmv_args* args, int32_t* part, void* stream);
 
+/* Listing 3 microbenchmark (section 3.1): `ctas` one-warp CTAs
+ * in hardware order; thread 0 of CTA b times one L1-allocating load
+ * (plain ld.global -> LDG.E) of input[32 * smid] -- the address depends only on the SM,
+ * so only CTAs on the same SM can share the line -- optionally after spinning
+ * `stagger_cycles * b` cycles (the STAGGERED variant, l.7-9).  All pointers
+ * DEVICE, caller-owned: input >= 32 * smid_span floats (cc_device_info);
+ * outputs smid[ctas] (%smid of CTA b), ticks[ctas] (%clock64 cycles of the
+ * load), sink[ctas] (loaded value + 1; keeps the load alive).  Asynchronous on
+ * `stream`.  ctas < 0, stagger_cycles < 0 or a NULL pointer with ctas > 0:
+ * CC_ERR_INVALID_ARG; ctas == 0 is a no-op. */
+cc_status cc_l1_reuse_probe(int32_t ctas, int32_t stagger_cycles, const float* input, int32_t* smid,
+                            uint32_t* ticks, float* sink, void* stream);
+
 /* Logical grid a kernel needs for `args` (so the caller can build the plan). */
 cc_status cc_kernel_grid(int32_t kernel, const void* args, int32_t* gx, int32_t* gy);
 /* Occupancy limit (agents per SM) of `kernel`'s agent body on `device`. */

@@ -18,6 +18,7 @@
 #include "cc_runtime.cuh"
 #include "k_gemv.cuh"
 #include "k_spmv.cuh"
+#include "k_microbench.cuh"
 #include "k_stencil.cuh"
 #include "k_tbcluster.cuh"
 
@@ -661,6 +662,17 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
     }
     if (prev != p->device) cudaSetDevice(prev);
     return s;
+}
+
+extern "C" cc_status cc_l1_reuse_probe(int32_t ctas, int32_t stagger_cycles, const float* input, int32_t* smid,
+                                     uint32_t* ticks, float* sink, void* stream) {
+    if (ctas < 0 || stagger_cycles < 0) return fail(CC_ERR_INVALID_ARG, "ctas %d / stagger %d", ctas, stagger_cycles);
+    if (ctas == 0) return CC_OK;
+    if (!input || !smid || !ticks || !sink) return fail(CC_ERR_INVALID_ARG, "l1 reuse probe: null pointer");
+    k_l1_reuse_probe<<<ctas, 32, 0, (cudaStream_t)stream>>>(input, smid, ticks, sink, stagger_cycles);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "l1 reuse probe");
+    return CC_OK;
 }
 
 extern "C" cc_status cc_spmv_partition(const cc_spmv_args* x, int32_t* part, void* stream) {

@@ -30,7 +30,7 @@ STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_E
 # every symbol include/ctaclust.h declares (checked by tests/test_abi.py)
 EXPORTS = ["cc_plan_create", "cc_plan_destroy", "cc_plan_info", "cc_plan_table", "cc_plan_lookup",
            "cc_plan_invert", "cc_device_info", "cc_sm_rank_table", "cc_launch_opts_default",
-           "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_comm_unique_id",
+           "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_l1_reuse_probe", "cc_comm_unique_id",
            "cc_comm_init", "cc_comm_destroy", "cc_halo_exchange", "cc_allreduce_sum", "cc_allgather",
            "cc_status_string", "cc_last_error", "cc_last_cuda_error", "cc_version"]
 
@@ -274,6 +274,12 @@ def spmv_args(row_ptr, col, val, x, y, part=None) -> SpmvArgs:
     rows = row_ptr.numel() - 1
     return SpmvArgs(rows, x.numel(), col.numel(), row_ptr.data_ptr(), col.data_ptr(), val.data_ptr(),
                     x.data_ptr(), y.data_ptr(), _ptr(part))
+
+
+def l1_reuse_probe(ctas: int, stagger_cycles: int, inp, smid, ticks, sink, stream=None):
+    """cc_l1_reuse_probe: Listing 3 microbenchmark (device tensors, caller-owned)."""
+    _check(lib().cc_l1_reuse_probe(_i32(ctas), _i32(stagger_cycles), _vp(inp.data_ptr()), _vp(smid.data_ptr()),
+                                   _vp(ticks.data_ptr()), _vp(sink.data_ptr()), _vp(_stream(stream))))
 
 
 def spmv_partition(args: SpmvArgs, part, stream=None):

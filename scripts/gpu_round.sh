@@ -6,3 +6,4 @@ bash scripts/gpu_check.sh
 bash scripts/ncu_suite.sh $TAG > gpurun_out/ncu_suite_$TAG.log 2>&1; echo "ncu_suite done"
 bash scripts/ncu_bench.sh $TAG > gpurun_out/ncu_bench_$TAG.log 2>&1; echo "ncu_bench done"; cat gpurun_out/ncu_bench_$TAG.log
 timeout -k 10 1800 python scripts/categorize_run.py gpurun_out/categorize.json > gpurun_out/categorize.log 2>&1; echo "cat=$?"; tail -9 gpurun_out/categorize.log
+timeout -k 10 300 python scripts/listing3.py gpurun_out/listing3.json > gpurun_out/listing3.log 2>&1; echo "listing3=$?"
