@@ -118,6 +118,20 @@ def variants_for(order, tile=(1, 1), stencil=False):
     return v
 
 
+def f2_variants(order, tile=(1, 1), l1_staging=None):
+    """S§8(f)2: L2 eviction-priority hints on the clustered agent (CLU+BPS) and a
+    carveout sweep on the variant that relies on L1 (`l1_staging`)."""
+    o = dict(order=order, tile=tile) if order == "tile" else dict(order=order)
+    tag = f"{order}{tile[0]}x{tile[1]}" if order == "tile" else order
+    v = [(f"agent-{tag}-l2first", dict(backend="agent", l2_hint="stream_first", **o)),
+         (f"agent-{tag}-l2last", dict(backend="agent", l2_hint="reuse_last", **o)),
+         (f"agent-{tag}-l2both", dict(backend="agent", l2_hint="both", **o))]
+    if l1_staging:
+        for cv in (0, 25, 50, 100):
+            v.append((f"agent-{tag}-{l1_staging}-cv{cv}", dict(backend="agent", staging=l1_staging, carveout=cv, **o)))
+    return v
+
+
 def suite_matvec(quick):
     import torch
     from paper_conf_asplos_lis0l0c17_b200 import ops, synth
@@ -149,7 +163,8 @@ def suite_atax(quick):
         "mvt": (lambda kw: ops.mvt(A, y1, y2, x1, x2, **kw), Ab + 24 * n),
     }
     variants = variants_for("col") + [("agent-row", dict(backend="agent", order="row")),
-                                      ("agent-col-s3", dict(backend="agent", order="col", stages=3))]
+                                      ("agent-col-s3", dict(backend="agent", order="col", stages=3))] \
+        + f2_variants("col", l1_staging="direct")
     ctx = {"atax": {"cublas-2xmv": lambda: torch.mv(A.t(), torch.mv(A, x, out=tmp), out=y)},
            "bicg": {"cublas-2xmv": lambda: (torch.mv(A, p, out=q), torch.mv(A.t(), r, out=s))},
            "mvt": {"cublas-2xmv": lambda: (x1.add_(torch.mv(A, y1)), x2.add_(torch.mv(A.t(), y2)))}}
@@ -163,7 +178,8 @@ def suite_jacobi(quick):
     N, T = 16384, (20 if quick else 100)
     a = synth.matrix(4, N, N, backend="torch", device="cuda")
     b = torch.empty_like(a)
-    r = measure(variants_for("tile", (8, 8), stencil=True), lambda kw: ops.jacobi5(a, b, T, **kw), 3, 8 * N * N * T,
+    v = variants_for("tile", (8, 8), stencil=True) + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1")
+    r = measure(v, lambda kw: ops.jacobi5(a, b, T, **kw), 3, 8 * N * N * T,
                 extra=lambda ms: {"ms_per_sweep": round(ms / T, 5)}, warm=1)
     r["config"] = f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)"
     return r
@@ -183,7 +199,8 @@ def suite_conv(quick):
         v = variants_for("tile", (8, 8), stencil=True) + [
             ("tbcluster-2", dict(backend="tbcluster", cluster_size=2)),
             ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
-            ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))]
+            ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))] \
+            + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1")
         wt = torch.from_numpy(w).cuda().view(1, 1, 2 * R + 1, 2 * R + 1)
         img4 = img.view(1, 1, N, N)
         res[f"{2 * R + 1}x{2 * R + 1}"] = measure(
@@ -215,7 +232,9 @@ def suite_spmv(quick):
                 ("agent-row-s1", dict(backend="agent", order="row", stages=1)),
                 ("agent-row-s4", dict(backend="agent", order="row", stages=4)),
                 ("identity", dict(backend="identity")), ("identity-s1", dict(backend="identity", stages=1)),
-                ("redirect-row", dict(backend="redirect", order="row"))]
+                ("redirect-row", dict(backend="redirect", order="row"))] + f2_variants("row") \
+        + [(f"{b}-cv{cv}", dict(backend=b, carveout=cv, **({"order": "row"} if b == "agent" else {})))
+           for b in ("default", "agent") for cv in (0, 25, 50, 100)]
     Acsr = torch.sparse_csr_tensor(rp, col, val, (rows_n, rows_n))
     r = measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 5 if quick else 20,
                 8 * nnz + 4 * (rows_n + 1) + 8 * rows_n,

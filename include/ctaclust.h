@@ -123,6 +123,15 @@ typedef enum {
 
 typedef enum { CC_STAGING_DEFAULT = 0, CC_STAGING_TMA = 1, CC_STAGING_L1 = 2, CC_STAGING_DIRECT = 3 } cc_staging;
 
+/* L2 eviction-priority hints (S§8(f)2: the paper's bypassing of streaming
+ * accesses, §4.3(II), carried to B200's L2 with createpolicy +
+ * .L2::cache_hint).  Bits: 1 = the kernel's streamed operand is evict_first
+ * (gemv: A; stencils: the output; SpMV: col/val); 2 = its reused operand is
+ * evict_last (gemv: the vector slices; stencils: the TMA-staged input with
+ * its halo; SpMV: x).  0 = no hint (default). */
+typedef enum { CC_L2_HINT_NONE = 0, CC_L2_HINT_STREAM_FIRST = 1, CC_L2_HINT_REUSE_LAST = 2,
+               CC_L2_HINT_BOTH = 3 } cc_l2_hint;
+
 typedef struct {
     int32_t backend;        /* cc_backend                                               */
     int32_t active_agents;  /* agents per SM that work (throttling, §4.3(I));
@@ -154,10 +163,17 @@ typedef struct {
     int32_t* d_exec_sm;     /* DEVICE, |V|, optional: %smid that executed lin          */
     int32_t* d_map;         /* DEVICE, |V|, optional: d_map[v] = lin executed for the
                                slot at order position v (agent/redirect/identity)      */
+    int32_t l2_hint;        /* cc_l2_hint bits (0..3); default 0                        */
+    int32_t carveout;       /* preferred shared-memory carveout of the launched kernel,
+                               percent of the SM's L1/shared array (0..100; the rest
+                               is L1), set with cudaFuncAttributePreferredShared-
+                               MemoryCarveout before the launch; -1 (default) = the
+                               driver's choice.  Agents per SM are recomputed under it. */
 } cc_launch_opts;
 
 /* Fill *opts with defaults: AGENT backend, max/active from occupancy, steal = 1,
- * stages/batch per kernel, cluster_size = 2, no census/map. */
+ * stages/batch per kernel, cluster_size = 2, no census/map, no L2 hint,
+ * carveout -1. */
 cc_status cc_launch_opts_default(cc_launch_opts* opts);
 
 typedef enum {

@@ -57,6 +57,62 @@ __device__ __forceinline__ void ld_stream4_x8(float4* v, const float* const* p) 
           "=f"(v[6].x), "=f"(v[6].y), "=f"(v[6].z), "=f"(v[6].w), "=f"(v[7].x), "=f"(v[7].y), "=f"(v[7].z), "=f"(v[7].w)
         : "l"(p[0]), "l"(p[1]), "l"(p[2]), "l"(p[3]), "l"(p[4]), "l"(p[5]), "l"(p[6]), "l"(p[7]));
 }
+// ---- L2 eviction priority (S§8(f)2: the bypass idea moved to B200's L2).
+// createpolicy builds a 64-bit policy; .L2::cache_hint attaches it to a
+// load/store/TMA copy.  evict_first: lines of a streamed operand leave L2
+// first; evict_last: lines of a reused operand (vector slices, halos, x)
+// stay longest.
+__device__ __forceinline__ uint64_t l2_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t l2_evict_last() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ float4 ld_stream4_h(const float* p, uint64_t pol) {
+    float4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ void ld_stream4_x8_h(float4* v, const float* const* p, uint64_t pol) {
+    asm volatile(
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%0,%1,%2,%3}, [%32], %40;\n\t"
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%4,%5,%6,%7}, [%33], %40;\n\t"
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%8,%9,%10,%11}, [%34], %40;\n\t"
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%12,%13,%14,%15}, [%35], %40;\n\t"
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%16,%17,%18,%19}, [%36], %40;\n\t"
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%20,%21,%22,%23}, [%37], %40;\n\t"
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%24,%25,%26,%27}, [%38], %40;\n\t"
+        "ld.global.nc.L1::no_allocate.L2::cache_hint.L2::256B.v4.f32 {%28,%29,%30,%31}, [%39], %40;"
+        : "=f"(v[0].x), "=f"(v[0].y), "=f"(v[0].z), "=f"(v[0].w), "=f"(v[1].x), "=f"(v[1].y), "=f"(v[1].z), "=f"(v[1].w),
+          "=f"(v[2].x), "=f"(v[2].y), "=f"(v[2].z), "=f"(v[2].w), "=f"(v[3].x), "=f"(v[3].y), "=f"(v[3].z), "=f"(v[3].w),
+          "=f"(v[4].x), "=f"(v[4].y), "=f"(v[4].z), "=f"(v[4].w), "=f"(v[5].x), "=f"(v[5].y), "=f"(v[5].z), "=f"(v[5].w),
+          "=f"(v[6].x), "=f"(v[6].y), "=f"(v[6].z), "=f"(v[6].w), "=f"(v[7].x), "=f"(v[7].y), "=f"(v[7].z), "=f"(v[7].w)
+        : "l"(p[0]), "l"(p[1]), "l"(p[2]), "l"(p[3]), "l"(p[4]), "l"(p[5]), "l"(p[6]), "l"(p[7]), "l"(pol));
+}
+__device__ __forceinline__ float4 ld_cached4_h(const float* p, uint64_t pol) {
+    float4 v;
+    asm("ld.global.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+        : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ float ld_cached_h(const float* p, uint64_t pol) {
+    float v;
+    asm("ld.global.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ void st4_h(float* p, float4 v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1,%2,%3,%4}, %5;"
+                 :: "l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void st1_h(float* p, float v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.f32 [%0], %1, %2;" :: "l"(p), "f"(v), "l"(pol) : "memory");
+}
+
 // Default-cached load (allocates in L1): operands that other CTAs of the same
 // cluster re-read (vector slices, halos).
 __device__ __forceinline__ float4 ld_cached4(const float* p) {
@@ -64,6 +120,16 @@ __device__ __forceinline__ float4 ld_cached4(const float* p) {
 }
 __device__ __forceinline__ float ld_cached(const float* p) { return *p; }
 
+__device__ __forceinline__ float ld_stream_f32_h(const float* p, uint64_t pol) {
+    float v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ int32_t ld_stream_i32_h(const int32_t* p, uint64_t pol) {
+    int32_t v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
 // Scalar streaming loads (read once; do not displace reused lines from L1).
 __device__ __forceinline__ float ld_stream_f32(const float* p) {
     float v;

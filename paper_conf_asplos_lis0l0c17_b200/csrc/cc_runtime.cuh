@@ -53,6 +53,7 @@ struct Sched {
     int32_t batch;                // slots claimed per queue atomic
     uint32_t stage_bytes;         // bytes per ring buffer (128-byte multiple)
     int32_t staging;              // cc_staging: 1 TMA, 2 L1-allocating cp.async, 3 direct
+    int32_t l2_hint;              // cc_l2_hint bits: 1 streamed operand evict_first, 2 reused operand evict_last
     uint32_t* census;             // optional outputs (see ctaclust.h)
     int32_t* exec_sm;
     int32_t* map;
@@ -139,6 +140,14 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const void* tmap, int32_t
     asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
                  :: "r"(smem_u32(dst)), "l"(tmap), "r"(x), "r"(y), "r"(smem_u32(bar)) : "memory");
 }
+__device__ __forceinline__ void tma_load_2d_h(void* dst, const void* tmap, int32_t x, int32_t y, uint64_t* bar,
+                                              uint64_t pol) {
+    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.L2::cache_hint"
+                 " [%0], [%1, {%2, %3}], [%4], %5;"
+                 :: "r"(smem_u32(dst)), "l"(tmap), "r"(x), "r"(y), "r"(smem_u32(bar)), "l"(pol) : "memory");
+}
+// L2 hint bits (cc_launch_opts.l2_hint)
+enum : int32_t { L2H_STREAM_FIRST = 1, L2H_REUSE_LAST = 2 };
 // named barrier among the consumer warps only (the producer warp never joins)
 // (barrier 1 + g for consumer group g of N threads; groups never share one)
 template <int N>
@@ -422,6 +431,7 @@ template <class Body>
 __global__ void __launch_bounds__(Body::kGroups * Body::kConsumers + PRODUCER_THREADS, Body::kMinAgents)
 k_agent(const __grid_constant__ Sched s, const __grid_constant__ typename Body::Params p) {
     Body body(p);
+    body.l2h = s.l2_hint;        // L2 hints ride with clustering (CLU+BPS); one-shot kernels compile them out
     agent_loop(s, body);
 }
 

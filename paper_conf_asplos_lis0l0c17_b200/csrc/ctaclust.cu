@@ -11,6 +11,7 @@
 #include <cstdio>
 #include <cstring>
 #include <mutex>
+#include <map>
 #include <string>
 #include <vector>
 
@@ -267,6 +268,8 @@ extern "C" cc_status cc_launch_opts_default(cc_launch_opts* o) {
     o->cluster_size = 2;
     o->stages = 0;
     o->batch = 0;
+    o->l2_hint = 0;
+    o->carveout = -1;
     return CC_OK;
 }
 
@@ -304,6 +307,7 @@ struct CensusBody {   // empty body: binding, queues and census only
     static constexpr int kMinAgents = 8;
     static constexpr int kGroups = 1;
     using Params = CensusParams;
+    int32_t l2h = 0;
     __device__ __forceinline__ explicit CensusBody(const CensusParams&) {}
     __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t, uint8_t*, uint64_t* full, int lane) { stage_commit(full, lane, 0); }
     __device__ __forceinline__ void consume(const Sched&, int32_t, int32_t, const uint8_t*, int) {}
@@ -383,6 +387,21 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     return s;
 }
 
+// Preferred L1/shared carveout of one kernel function (cc_launch_opts.carveout);
+// the attribute is per function and sticky, so it is set only when it changes.
+template <class K>
+static cc_status set_carveout(K* fn, int32_t pct) {
+    static std::mutex mu;
+    static std::map<const void*, int32_t> cur;
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = cur.find((const void*)fn);
+    const int32_t have = it == cur.end() ? -1 : it->second;
+    if (have == pct) return CC_OK;
+    CC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, pct));
+    cur[(const void*)fn] = pct;
+    return CC_OK;
+}
+
 struct LaunchCtx {
     cc_plan p;
     const cc_launch_opts* o;
@@ -405,6 +424,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     s.steal = o.steal;
     s.batch = o.batch > 0 ? o.batch : Body::kDefaultBatch;
     s.staging = o.staging == CC_STAGING_DEFAULT ? CC_STAGING_TMA : o.staging;
+    s.l2_hint = o.l2_hint;
     const bool direct = s.staging == CC_STAGING_DIRECT;
     s.stage_bytes = direct ? 128u : (uint32_t)Body::kStageBytes;
     s.census = o.d_census;
@@ -414,12 +434,14 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     switch (o.backend) {
     case CC_BACKEND_DEFAULT: {
         if (g.gy > 65535) return fail(CC_ERR_UNSUPPORTED, "default backend: gy %d > 65535", g.gy);
+        CC_TRY(set_carveout(k_default<Body>, o.carveout));
         s.map = nullptr;
         s.stages = 1;
         k_default<Body><<<dim3(g.gx, g.gy), threads, dyn_smem<Body>(1, direct), c.st>>>(s, prm);
         break;
     }
     case CC_BACKEND_REDIRECT:
+        CC_TRY(set_carveout(k_redirect<Body>, o.carveout));
         s.stages = 1;
         k_redirect<Body><<<g.V, threads, dyn_smem<Body>(1, direct), c.st>>>(s, prm);
         break;
@@ -428,7 +450,14 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
         if (S < Body::kGroups) S = Body::kGroups;             // every consumer group needs a slot
         int occ = 0;
-        CC_TRY(occupancy<Body>(c.p->device, S, &occ, direct));
+        CC_TRY(set_carveout(k_agent<Body>, o.carveout));
+        if (o.carveout < 0) CC_TRY(occupancy<Body>(c.p->device, S, &occ, direct));
+        else {
+            CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_agent<Body>,
+                                                                  Body::kGroups * Body::kConsumers + PRODUCER_THREADS,
+                                                                  dyn_smem<Body>(S, direct)));
+            if (occ < 1) return fail(CC_ERR_UNSUPPORTED, "carveout %d leaves no room for one agent", o.carveout);
+        }
         const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
         s.active_agents = o.active_agents > 0 ? std::min(o.active_agents, maxa) : maxa;
         s.throttle = s.active_agents < maxa;
@@ -542,10 +571,12 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
                                void* stream, int32_t* launches) {
     if (!p || !a) return fail(CC_ERR_INVALID_ARG, "null plan or args");
     if (launches) *launches = 0;
-    if (p->device < 0) return fail(CC_ERR_NO_DEVICE, "plan was created host-only");
     cc_launch_opts dflt;
     cc_launch_opts_default(&dflt);
     const cc_launch_opts* o = opts ? opts : &dflt;
+    if (o->l2_hint < 0 || o->l2_hint > 3) return fail(CC_ERR_INVALID_ARG, "l2_hint %d outside [0, 3]", o->l2_hint);
+    if (o->carveout < -1 || o->carveout > 100) return fail(CC_ERR_INVALID_ARG, "carveout %d outside [-1, 100]", o->carveout);
+    if (p->device < 0) return fail(CC_ERR_NO_DEVICE, "plan was created host-only");
     int32_t gx = 0, gy = 0;
     CC_TRY(cc_kernel_grid(k, a, &gx, &gy));
     if (gx != p->g.gx || gy != p->g.gy)

@@ -57,6 +57,7 @@ struct GemvBody {
     using Params = GemvParams;
 
     const GemvParams& p;   // the __grid_constant__ kernel parameter (TMA needs its address)
+    int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
     int32_t cur_ti, cur_tj;
     float racc[NP];
     float4 cacc[FPL];
@@ -75,7 +76,10 @@ struct GemvBody {
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
         if (s.staging == 3) { stage_commit(full, lane, 0); return; }   // direct: consumers load A
         stage_commit(full, lane, (uint32_t)kStageBytes);
-        if (lane == 0) tma_load_2d(stage, &p.tmap, bx * TC, by * TR, full);
+        if (lane == 0) {
+            if (l2h & L2H_STREAM_FIRST) tma_load_2d_h(stage, &p.tmap, bx * TC, by * TR, full, l2_evict_first());
+            else tma_load_2d(stage, &p.tmap, bx * TC, by * TR, full);
+        }
     }
 
     // ---- ROW flush: warp-level sum over the LPR lanes of each row, one RED per row
@@ -128,14 +132,18 @@ struct GemvBody {
         const int warp = ctid >> 5, lane = ctid & 31, sub = lane / LPR, cl = lane % LPR;
         const int col0 = bx * TC, row0 = by * TR;
         const bool direct = s.staging == 3;
+        const bool hf = l2h & L2H_STREAM_FIRST, hl = l2h & L2H_REUSE_LAST;
+        auto vec4 = [&](const float* q) { return hl ? ld_cached4_h(q, l2_evict_last()) : ld_cached4(q); };
+        auto vec1 = [&](const float* q) { return hl ? ld_cached_h(q, l2_evict_last()) : ld_cached(q); };
+        auto a4 = [&](const float* q) { return hf ? ld_stream4_h(q, l2_evict_first()) : ld_stream4(q); };
         if (col0 + TC <= p.n && row0 + TR <= p.m) {
             // interior tile: no bounds anywhere in the hot loop
             float4 xv[FPL];
             float rv[NP];
 #pragma unroll
-            for (int f = 0; f < FPL; ++f) xv[f] = DO_ROW ? ld_cached4(p.vc + col0 + tcol4(cl, f) * 4) : f4_zero();
+            for (int f = 0; f < FPL; ++f) xv[f] = DO_ROW ? vec4(p.vc + col0 + tcol4(cl, f) * 4) : f4_zero();
 #pragma unroll
-            for (int k = 0; k < NP; ++k) rv[k] = DO_COL ? ld_cached(p.vr + row0 + trow(warp, k, sub)) : 0.f;
+            for (int k = 0; k < NP; ++k) rv[k] = DO_COL ? vec1(p.vr + row0 + trow(warp, k, sub)) : 0.f;
             if (direct) {
                 // plain-kernel form: issue every A load of the tile first (NP*FPL
                 // independent 16-byte loads in flight per thread), then reduce
@@ -147,10 +155,17 @@ struct GemvBody {
 #pragma unroll
                     for (int q = 0; q < 8; ++q)
                         ptr[q] = base + (int64_t)trow(warp, q / FPL, sub) * p.lda + tcol4(cl, q % FPL) * 4;
-                    ld_stream4_x8(v8, ptr);
+                    if (hf) ld_stream4_x8_h(v8, ptr, l2_evict_first());
+                    else ld_stream4_x8(v8, ptr);
 #pragma unroll
                     for (int q = 0; q < 8; ++q) av[q / FPL][q % FPL] = v8[q];
                 } else if constexpr ((NP * FPL) % 4 == 0) {
+                    if (hf) {
+#pragma unroll
+                        for (int q = 0; q < NP * FPL; ++q)
+                            av[q / FPL][q % FPL] = ld_stream4_h(base + (int64_t)trow(warp, q / FPL, sub) * p.lda +
+                                                                tcol4(cl, q % FPL) * 4, l2_evict_first());
+                    } else
 #pragma unroll
                     for (int q = 0; q < NP * FPL; q += 4) {
                         const int k0 = q / FPL, f0 = q % FPL, k1 = (q + 1) / FPL, f1 = (q + 1) % FPL;
@@ -166,7 +181,9 @@ struct GemvBody {
                     for (int k = 0; k < NP; ++k)
 #pragma unroll
                         for (int f = 0; f < FPL; ++f)
-                            av[k][f] = ld_stream4_batched(base + (int64_t)trow(warp, k, sub) * p.lda + tcol4(cl, f) * 4);
+                            av[k][f] = hf ? ld_stream4_h(base + (int64_t)trow(warp, k, sub) * p.lda + tcol4(cl, f) * 4,
+                                                         l2_evict_first())
+                                          : ld_stream4_batched(base + (int64_t)trow(warp, k, sub) * p.lda + tcol4(cl, f) * 4);
                 }
 #pragma unroll
                 for (int k = 0; k < NP; ++k)
@@ -190,11 +207,11 @@ struct GemvBody {
             const int col = col0 + tcol4(cl, f) * 4;
             xv[f] = f4_zero();
             if (DO_ROW && col < p.n) {
-                if (col + 4 <= p.n) xv[f] = ld_cached4(p.vc + col);
+                if (col + 4 <= p.n) xv[f] = vec4(p.vc + col);
                 else {
-                    xv[f].x = ld_cached(p.vc + col);
-                    if (col + 1 < p.n) xv[f].y = ld_cached(p.vc + col + 1);
-                    if (col + 2 < p.n) xv[f].z = ld_cached(p.vc + col + 2);
+                    xv[f].x = vec1(p.vc + col);
+                    if (col + 1 < p.n) xv[f].y = vec1(p.vc + col + 1);
+                    if (col + 2 < p.n) xv[f].z = vec1(p.vc + col + 2);
                 }
             }
         }
@@ -202,14 +219,14 @@ struct GemvBody {
         for (int k = 0; k < NP; ++k) {
             const int r = trow(warp, k, sub);
             if (row0 + r >= p.m) continue;
-            const float rv = DO_COL ? ld_cached(p.vr + row0 + r) : 0.f;
+            const float rv = DO_COL ? vec1(p.vr + row0 + r) : 0.f;
 #pragma unroll
             for (int f = 0; f < FPL; ++f) {
                 const int col = col0 + tcol4(cl, f) * 4;
                 if (col >= p.n) continue;
                 float4 a;
                 if (direct) {
-                    a = ld_stream4(p.A + (int64_t)(row0 + r) * p.lda + col);   // inside lda (lda % 4 == 0)
+                    a = a4(p.A + (int64_t)(row0 + r) * p.lda + col);   // inside lda (lda % 4 == 0)
                     if (col + 1 >= p.n) a.y = 0.f;                              // padding past n
                     if (col + 2 >= p.n) a.z = 0.f;
                     if (col + 3 >= p.n) a.w = 0.f;

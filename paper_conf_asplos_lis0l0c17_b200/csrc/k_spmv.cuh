@@ -76,6 +76,7 @@ struct SpmvBody {
     static constexpr int kGroups = 1;
     using Params = SpmvParams;
     const SpmvParams& p;
+    int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
     __device__ __forceinline__ explicit SpmvBody(const SpmvParams& prm) : p(prm) {}
 
     // Nothing is staged in smem (it would cost L1, see above).  Instead the
@@ -101,7 +102,7 @@ struct SpmvBody {
         stage_commit(full, lane, 0);
     }
 
-    __device__ __forceinline__ void consume(const Sched&, int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
+    __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
         __shared__ int32_t s_rowend[SPMV_ROWCAP];
         // products of the CTA's nonzeros, index j stored at j + j/IPT (the pad
         // keeps each thread's IPT-long private run conflict-free)
@@ -121,13 +122,28 @@ struct SpmvBody {
         // all products of the CTA, coalesced: val/col stream past L1, the x
         // gathers go through it (16 independent loads per thread in flight)
         const int32_t nz = (int32_t)(y1 - y0);
+        if (l2h == 0) {
 #pragma unroll
-        for (int k = 0; k < SPMV_IPT; ++k) {
-            const int32_t j = t + k * kConsumers;
-            if (j < nz) {
-                const int32_t c = ld_stream_i32(p.col + y0 + j);
-                const float v = ld_stream_f32(p.val + y0 + j);
-                s_prod[j + j / SPMV_IPT] = v * ld_cached(p.x + c);
+            for (int k = 0; k < SPMV_IPT; ++k) {
+                const int32_t j = t + k * kConsumers;
+                if (j < nz) {
+                    const int32_t c = ld_stream_i32(p.col + y0 + j);
+                    const float v = ld_stream_f32(p.val + y0 + j);
+                    s_prod[j + j / SPMV_IPT] = v * ld_cached(p.x + c);
+                }
+            }
+        } else {
+            // L2 hints (S§8(f)2): col/val streamed (evict_first), x reused (evict_last)
+            const bool hf = l2h & L2H_STREAM_FIRST, hl = l2h & L2H_REUSE_LAST;
+            const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
+#pragma unroll
+            for (int k = 0; k < SPMV_IPT; ++k) {
+                const int32_t j = t + k * kConsumers;
+                if (j < nz) {
+                    const int32_t c = hf ? ld_stream_i32_h(p.col + y0 + j, pf) : ld_stream_i32(p.col + y0 + j);
+                    const float v = hf ? ld_stream_f32_h(p.val + y0 + j, pf) : ld_stream_f32(p.val + y0 + j);
+                    s_prod[j + j / SPMV_IPT] = v * (hl ? ld_cached_h(p.x + c, pl) : ld_cached(p.x + c));
+                }
             }
         }
         consumer_sync<kConsumers>();

@@ -33,11 +33,15 @@ struct HaloTile {
     // warp-collective: stage rows y0-H.., columns x0-4.. of `src` (TMA or L1 mode).
     __device__ __forceinline__ static void stage(const float* src, int64_t ld, int32_t rows, int32_t cols,
                                                  int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
-                                                 int32_t mode, const CUtensorMap* tmap) {
+                                                 int32_t mode, const CUtensorMap* tmap, int32_t l2_hint = 0) {
         if (mode == STAGE_DIRECT) { stage_commit(full, lane, 0); return; }
         if (mode == STAGE_TMA) {
             stage_commit(full, lane, (uint32_t)(kRows * ST_COLS * 4));
-            if (lane == 0) tma_load_2d(dst, tmap, x0 - 4, y0 - H, full);
+            if (lane == 0) {
+                // the input is the reused operand (halo rows feed the next tile row)
+                if (l2_hint & L2H_REUSE_LAST) tma_load_2d_h(dst, tmap, x0 - 4, y0 - H, full, l2_evict_last());
+                else tma_load_2d(dst, tmap, x0 - 4, y0 - H, full);
+            }
             return;
         }
         const int32_t cols4 = (cols + 3) & ~3;   // last 16-byte chunk stays inside ld
@@ -64,6 +68,17 @@ __device__ __forceinline__ void store4_masked(float* dst, float4 o, int gx, int 
         dst[0] = o.x;
         if (gx + 1 < cols) dst[1] = o.y;
         if (gx + 2 < cols) dst[2] = o.z;
+    }
+}
+// the output is the streamed operand: with L2H_STREAM_FIRST its lines leave L2 first
+__device__ __forceinline__ void store4_out(float* dst, float4 o, int gx, int cols, int32_t l2_hint) {
+    if (!(l2_hint & L2H_STREAM_FIRST)) { store4_masked(dst, o, gx, cols); return; }
+    const uint64_t pol = l2_evict_first();
+    if (gx + 4 <= cols) st4_h(dst, o, pol);
+    else {
+        st1_h(dst, o.x, pol);
+        if (gx + 1 < cols) st1_h(dst + 1, o.y, pol);
+        if (gx + 2 < cols) st1_h(dst + 2, o.z, pol);
     }
 }
 
@@ -102,10 +117,11 @@ struct Jacobi5Body {
     static constexpr int kGroups = 2;              // two 4-warp groups consume alternate tiles
     using Params = JacobiParams;
     const JacobiParams& p;   // __grid_constant__ kernel parameter
+    int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
     __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap);
+        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h);
     }
 
     // thread (rows r0 .. r0+RB-1, columns 4*c4 .. 4*c4+3): the RB+2 input rows
@@ -150,8 +166,9 @@ struct Jacobi5Body {
         for (int j = 0; j < RB; ++j) {
             const int gy = gy0 + j;
             if (gy >= p.rows) break;
-            store4_masked(p.b + (int64_t)gy * p.ld + gx,
-                          jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx, p.cols);
+            store4_out(p.b + (int64_t)gy * p.ld + gx,
+                       jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx, p.cols,
+                       l2h);
         }
     }
     __device__ __forceinline__ void finish(int) {}
@@ -173,7 +190,7 @@ struct ConvParams { CUtensorMap tmap; const float* in; float* out; int64_t ld; i
 // filter's row-major tap order, as in the oracle.
 template <int R, int RB = 1>
 __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const float* rows_base,
-                                                  int32_t bx, int32_t by, int ctid) {
+                                                  int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0) {
     // rows_base points at the staged row holding input row y0 - R, column x0 - 4
     constexpr int K = 2 * R + 1;
     const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
@@ -211,7 +228,7 @@ __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const 
         o.y = (row_in && gx + 1 >= R && gx + 1 < p.cols - R) ? acc[j][1] : 0.f;
         o.z = (row_in && gx + 2 >= R && gx + 2 < p.cols - R) ? acc[j][2] : 0.f;
         o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[j][3] : 0.f;
-        store4_masked(p.out + (int64_t)gy * p.ld + gx, o, gx, p.cols);
+        store4_out(p.out + (int64_t)gy * p.ld + gx, o, gx, p.cols, l2_hint);
     }
 }
 
@@ -226,10 +243,11 @@ struct Conv2dBody {
     static constexpr int kGroups = 2;              // two 4-warp groups consume alternate tiles
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
+    int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap);
+        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h);
     }
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         if (s.staging == STAGE_DIRECT) {
@@ -244,11 +262,11 @@ struct Conv2dBody {
                 s_in[rr][cc] = v;
             }
             consumer_sync<kConsumers>();
-            conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid);
+            conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid, l2h);
             consumer_sync<kConsumers>();                 // s_in is rewritten by the next task
             return;
         }
-        conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid);
+        conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid, l2h);
     }
     __device__ __forceinline__ void finish(int) {}
 };

@@ -54,7 +54,7 @@ class LaunchOpts(ctypes.Structure):
     _fields_ = [("backend", _i32), ("active_agents", _i32), ("max_agents", _i32), ("stages", _i32),
                 ("batch", _i32), ("staging", _i32), ("steal", _i32), ("cluster_size", _i32), ("d_census", _vp),
                 ("d_exec_sm", _vp),
-                ("d_map", _vp)]
+                ("d_map", _vp), ("l2_hint", _i32), ("carveout", _i32)]
 
 
 class CensusArgs(ctypes.Structure):
@@ -201,11 +201,16 @@ def _stream(stream):
     return s.cuda_stream
 
 
+L2_HINTS = {"none": 0, "stream_first": 1, "reuse_last": 2, "both": 3}
+
+
 def make_opts(backend="agent", active_agents=0, max_agents=0, stages=0, batch=0, staging=0, steal=1,
-              cluster_size=2, census=None, exec_sm=None, map=None) -> LaunchOpts:
+              cluster_size=2, census=None, exec_sm=None, map=None, l2_hint=0, carveout=-1) -> LaunchOpts:
     b = BACKENDS[backend] if isinstance(backend, str) else int(backend)
-    return LaunchOpts(b, active_agents, max_agents, int(stages), int(batch), STAGINGS.get(staging, staging) if isinstance(staging, str) else int(staging), int(steal), cluster_size,
-                      _ptr(census), _ptr(exec_sm), _ptr(map))
+    st = STAGINGS.get(staging, staging) if isinstance(staging, str) else int(staging)
+    h = L2_HINTS[l2_hint] if isinstance(l2_hint, str) else int(l2_hint)
+    return LaunchOpts(b, active_agents, max_agents, int(stages), int(batch), st, int(steal), cluster_size,
+                      _ptr(census), _ptr(exec_sm), _ptr(map), h, int(carveout))
 
 
 def kernel_grid(kernel, args) -> tuple[int, int]:

@@ -44,7 +44,7 @@ LAYOUT_C = r"""
 #define O(T, f) printf(#T "." #f " %zu\n", offsetof(T, f));
 int main(void) {
   S(cc_plan_desc) O(cc_plan_desc, user_order) O(cc_plan_desc, device)
-  S(cc_launch_opts) O(cc_launch_opts, d_census) O(cc_launch_opts, d_map)
+  S(cc_launch_opts) O(cc_launch_opts, d_census) O(cc_launch_opts, d_map) O(cc_launch_opts, l2_hint) O(cc_launch_opts, carveout)
   S(cc_matvec_args) O(cc_matvec_args, y) S(cc_atax_args) O(cc_atax_args, y)
   S(cc_bicg_args) O(cc_bicg_args, s) S(cc_mvt_args) O(cc_mvt_args, x2)
   S(cc_jacobi5_args) O(cc_jacobi5_args, result_is_b) S(cc_conv2d_args) O(cc_conv2d_args, w)
@@ -137,6 +137,11 @@ def test_planner_user_order_and_errors():
     with pytest.raises(cc.CtaclustError) as e:                   # host-only plan cannot launch
         cc._check(cc.lib().cc_launch(p.handle, 0, ctypes.byref(cc.CensusArgs(4, 4)), None, None, None))
     assert e.value.status == -7
+    for bad in (dict(l2_hint=4), dict(l2_hint=-1), dict(carveout=101), dict(carveout=-2)):
+        with pytest.raises(cc.CtaclustError) as e:               # options are validated first
+            cc._check(cc.lib().cc_launch(p.handle, 0, ctypes.byref(cc.CensusArgs(4, 4)),
+                                         ctypes.byref(cc.make_opts(**bad)), None, None))
+        assert e.value.status == -1, bad
 
 
 def test_empty_grid_and_more_clusters_than_ctas():

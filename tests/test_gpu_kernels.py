@@ -29,6 +29,10 @@ VARIANTS = [
     dict(backend="default", staging="direct"),
     dict(backend="agent", order="col", staging="direct"),
     dict(backend="agent", order="row", staging="tma", stages=3, batch=2),
+    dict(backend="agent", order="col", l2_hint="both"),
+    dict(backend="agent", order="col", staging="direct", l2_hint="both", carveout=50),
+    dict(backend="identity", l2_hint="stream_first", carveout=0),
+    dict(backend="default", carveout=100),
 ]
 
 
@@ -135,7 +139,9 @@ JVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(
              dict(backend="redirect", order="tile", tile=(4, 4)),
              dict(backend="default", staging="l1"), dict(backend="default", staging="direct"),
              dict(backend="agent", order="tile", tile=(8, 8), staging="l1"),
-             dict(backend="agent", order="row", staging="direct")]
+             dict(backend="agent", order="row", staging="direct"),
+             dict(backend="agent", order="row", l2_hint="both"),
+             dict(backend="agent", order="row", staging="l1", l2_hint="both", carveout=25)]
 
 
 @pytest.mark.parametrize("v", JVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
@@ -180,7 +186,8 @@ CVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(
              dict(backend="redirect", order="row"),
              dict(backend="default", staging="l1"), dict(backend="default", staging="direct"),
              dict(backend="agent", order="tile", tile=(8, 8), staging="l1"),
-             dict(backend="agent", order="col", staging="direct")]
+             dict(backend="agent", order="col", staging="direct"),
+             dict(backend="agent", order="row", l2_hint="both", carveout=100)]
 
 
 @pytest.mark.parametrize("v", CVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
@@ -238,7 +245,8 @@ def _csr_dev(rp, col, val):
 
 
 SVARIANTS = [dict(backend="default"), dict(backend="agent", order="row"), dict(backend="agent", active_agents=1),
-             dict(backend="agent", stages=4, batch=5), dict(backend="identity"), dict(backend="redirect")]
+             dict(backend="agent", stages=4, batch=5), dict(backend="identity"), dict(backend="redirect"),
+             dict(backend="agent", order="row", l2_hint="both"), dict(backend="default", carveout=0)]
 
 
 def _edge_matrices():
