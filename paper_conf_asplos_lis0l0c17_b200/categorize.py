@@ -223,6 +223,9 @@ def candidates(v: Verdict, max_agents: int, has_staging: bool = True) -> list[tu
         # partition signal is often within noise (R22)
         alt = "col" if part == "row" else "row"
         out.append((f"CLU-{alt}", dict(backend="agent", order=alt)))
+        # persistence + prefetch in the hardware order (no clustering): on B200
+        # a single global wavefront can beat per-SM bands on DRAM page locality
+        out.append(("PFH-identity", dict(backend="identity")))
         if has_staging and "BPS" in v.optimizations:
             # BPS: streaming operand bypasses L1 (TMA / no_allocate) vs through it
             out.append((f"CLU-{part}+L1", dict(backend="agent", order=part, staging="l1")))
@@ -232,6 +235,7 @@ def candidates(v: Verdict, max_agents: int, has_staging: bool = True) -> list[tu
         # next tasks' operands; ring depth = prefetch distance
         for s in (1, 2, 4):
             out.append((f"PFH-row-s{s}", dict(backend="agent", order="row", stages=s)))
+        out.append(("PFH-identity", dict(backend="identity")))
         for a in range(1, max_agents + 1):
             out.append((f"PFH-row+TOT{a}", dict(backend="agent", order="row", active_agents=a)))
     return out

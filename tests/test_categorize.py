@@ -72,13 +72,14 @@ def test_candidates_cover_tot_sweep_and_bps():
     assert names[0] == "default"
     assert [n for n in names if "TOT" in n] == [f"CLU-col+TOT{a}" for a in range(1, 5)]
     assert ("CLU-row", dict(backend="agent", order="row")) in C.candidates(v, 4)
+    assert ("PFH-identity", dict(backend="identity")) in C.candidates(v, 4)
     assert "CLU-col+L1" in names and "CLU-col+direct" in names
-    assert all(kw.get("order", "col") == "col" for n, kw in C.candidates(v, 4) if n != "CLU-row")
+    assert all(kw.get("order", "col") == "col" for n, kw in C.candidates(v, 4) if n not in ("CLU-row", "PFH-identity"))
     assert not any("L1" in n for n, _ in C.candidates(v, 4, has_staging=False))
     nv = C.Verdict("data", None, False, ["PFH", "TOT"])
     names = [n for n, _ in C.candidates(nv, 3)]
-    assert names[:4] == ["default", "PFH-row-s1", "PFH-row-s2", "PFH-row-s4"]
-    assert names[4:] == [f"PFH-row+TOT{a}" for a in range(1, 4)]
+    assert names[:5] == ["default", "PFH-row-s1", "PFH-row-s2", "PFH-row-s4", "PFH-identity"]
+    assert names[5:] == [f"PFH-row+TOT{a}" for a in range(1, 4)]
 
 
 def test_tune_picks_fastest_with_fake_timer():
