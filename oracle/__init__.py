@@ -157,3 +157,12 @@ def spmv_csr(row_ptr, col, val, x):
     y, py = _out(rows)
     _load().oracle_spmv_csr(_I(rows), prp, pc, pv, px, py)
     return y
+
+
+def hist64(data):
+    """64-bin histogram of uint8 data (bin = byte >> 2); uint64 counts."""
+    data = np.ascontiguousarray(data, dtype=np.uint8)
+    out = np.zeros(64, dtype=np.uint64)
+    _load().oracle_hist64(ctypes.c_int64(data.size), data.ctypes.data_as(ctypes.c_void_p),
+                          out.ctypes.data_as(ctypes.c_void_p))
+    return out

@@ -186,3 +186,15 @@ void oracle_spmv_csr(int64_t rows, const int32_t* row_ptr, const int32_t* col,
         y_out[i] = acc;
     }
 }
+
+/* ------------------------------------------------------------------------
+ * S§8(f)3  64-bin histogram (HST): PAPER.md Table 2 ("histogram
+ * 64-bin histogramming", category Data; the data-related class of P:1761,
+ * source [40] = the CUDA SDK).  Reading R24: the SDK's histogram64 bins each
+ * input byte by its top six bits, so
+ *     counts[k] = #{ i < n : data[i] >> 2 == k },   k = 0..63.
+ */
+void oracle_hist64(int64_t n, const uint8_t* data, uint64_t* counts) {
+    for (int k = 0; k < 64; ++k) counts[k] = 0;
+    for (int64_t i = 0; i < n; ++i) counts[data[i] >> 2] += 1;
+}

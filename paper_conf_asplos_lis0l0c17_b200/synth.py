@@ -13,6 +13,8 @@ Recipes:
 * ``small_int`` integers in {-8..8} as fp32 -- the integer-exact mode (R18);
 * ``rmat_edges`` R-MAT (a,b,c,d) = (0.57,0.19,0.19,0.05) power-law graphs for
   the CSR SpMV workload (R16).
+* ``bytes_u8`` input bytes for the 64-bin histogram (S§8(f)3, R24): uniform
+  bytes, or ``skewed`` (75 % of bytes in bin 0: the contended case).
 """
 from __future__ import annotations
 
@@ -83,6 +85,38 @@ def uniform(seed: int, count: int, start: int = 0, *, backend: str = "numpy",
         idx = torch.arange(start + c0, start + c1, dtype=torch.int64, device=device)
         h = hash_u32_torch(seed, idx, stream)
         out[c0:c1] = (h >> 8).to(torch.float32) * (2.0 ** -24)
+    return out
+
+
+def bytes_u8(seed: int, count: int, start: int = 0, *, kind: str = "uniform", backend: str = "numpy",
+             device=None, chunk: int = 1 << 26):
+    """``count`` uint8 values: ``uniform`` = top byte of the hash; ``skewed`` =
+    with probability 3/4 (second hash stream) a value in 0..3, else uniform."""
+    if kind not in ("uniform", "skewed"):
+        raise ValueError(kind)
+    if backend == "numpy":
+        out = np.empty(count, dtype=np.uint8)
+        for c0 in range(0, count, chunk):
+            c1 = min(count, c0 + chunk)
+            idx = np.arange(start + c0, start + c1, dtype=np.uint64)
+            h = hash_u32_np(seed, idx)
+            b = (h >> np.uint32(24)).astype(np.uint8)
+            if kind == "skewed":
+                hot = (hash_u32_np(seed, idx, 1) >> np.uint32(24)) < np.uint32(192)
+                b = np.where(hot, (h >> np.uint32(30)).astype(np.uint8), b)
+            out[c0:c1] = b
+        return out
+    import torch
+    out = torch.empty(count, dtype=torch.uint8, device=device)
+    for c0 in range(0, count, chunk):
+        c1 = min(count, c0 + chunk)
+        idx = torch.arange(start + c0, start + c1, dtype=torch.int64, device=device)
+        h = hash_u32_torch(seed, idx)
+        b = h >> 24
+        if kind == "skewed":
+            hot = (hash_u32_torch(seed, idx, 1) >> 24) < 192
+            b = torch.where(hot, h >> 30, b)
+        out[c0:c1] = b.to(torch.uint8)
     return out
 
 

@@ -172,3 +172,39 @@ def test_synth_numpy_torch_identical():
     big = synth.uniform(1, 10, (1 << 33) + 5)               # high index word matters
     assert not np.array_equal(big, synth.uniform(1, 10, 5))
     assert torch.is_tensor(synth.uniform(1, 4, backend="torch"))
+
+
+# ---- S8(f)3 64-bin histogram (Table 2; reading R24: bin = byte >> 2) ----
+def test_hist64_closed_forms():
+    # every byte value r times: each bin holds its 4 byte values -> 4r
+    r = 37
+    counts = O.hist64(np.tile(np.arange(256, dtype=np.uint8), r))
+    assert counts.dtype == np.uint64 and counts.shape == (64,)
+    assert np.all(counts == 4 * r)
+    # a constant input lands in one bin: byte c -> bin floor(c / 4)
+    for c in (0, 3, 4, 130, 255):
+        counts = O.hist64(np.full(1001, c, dtype=np.uint8))
+        assert counts[c // 4] == 1001 and counts.sum() == 1001
+    assert np.all(O.hist64(np.zeros(0, dtype=np.uint8)) == 0)
+
+
+def test_hist64_threshold_counts_and_total():
+    # prefix sums of the histogram count the bytes below each bin edge 4k
+    for kind in ("uniform", "skewed"):
+        data = synth.bytes_u8(21, 100003, kind=kind)
+        counts = O.hist64(data)
+        assert int(counts.sum()) == data.size
+        cum = np.concatenate([[0], np.cumsum(counts)])
+        for k in range(65):
+            assert cum[k] == np.count_nonzero(data < 4 * k)
+
+
+def test_bytes_generator_backends_agree_and_skew():
+    import torch
+    a = synth.bytes_u8(5, 70001, kind="skewed")
+    b = synth.bytes_u8(5, 70001, kind="skewed", backend="torch").numpy()
+    assert np.array_equal(a, b)
+    frac0 = np.count_nonzero(a < 4) / a.size            # 3/4 hot + 1/4 * 4/256 uniform
+    assert abs(frac0 - (0.75 + 0.25 * 4 / 256)) < 0.01
+    u = synth.bytes_u8(6, 1 << 16)
+    assert abs(np.count_nonzero(u < 128) / u.size - 0.5) < 0.01
