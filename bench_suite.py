@@ -243,7 +243,31 @@ def suite_spmv(quick):
     return r
 
 
-SUITES = {"matvec": suite_matvec, "atax": suite_atax, "jacobi": suite_jacobi, "conv": suite_conv, "spmv": suite_spmv}
+def suite_hist(quick):
+    """S8(f)3: the paper's HST (64-bin histogram, data-related) -- CTA
+    prefetching with the agent's ordered stream (PFH) vs default order."""
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    n = 1 << (28 if quick else 30)
+    counts = torch.empty(64, dtype=torch.int32, device="cuda")
+    res = {}
+    for kind in ("uniform", "skewed"):
+        data = synth.bytes_u8(31, n, kind=kind, backend="torch", device="cuda")
+        v = [("default", dict(backend="default")), ("default-direct", dict(backend="default", staging="direct")),
+             ("agent-row", dict(backend="agent", order="row")),
+             ("agent-row-s1", dict(backend="agent", order="row", stages=1)),
+             ("agent-row-s2", dict(backend="agent", order="row", stages=2)),
+             ("agent-row-s4", dict(backend="agent", order="row", stages=4)),
+             ("agent-row-direct", dict(backend="agent", order="row", staging="direct")),
+             ("agent-row-tot1", dict(backend="agent", order="row", active_agents=1)),
+             ("agent-col", dict(backend="agent", order="col")),
+             ("identity", dict(backend="identity")), ("redirect-row", dict(backend="redirect", order="row"))]
+        res[kind] = measure(v, lambda kw: ops.hist64(data, counts, **kw), 5 if quick else 20, n + 256)
+        del data
+    return {"config": f"64-bin histogram (HST, R24) of {n} bytes, 32 KiB per logical CTA", "inputs": res}
+
+
+SUITES = {"matvec": suite_matvec, "atax": suite_atax, "jacobi": suite_jacobi, "conv": suite_conv, "spmv": suite_spmv, "hist": suite_hist}
 
 
 def run(path, only=None, quick=False):
@@ -269,7 +293,7 @@ def table(path):
     for k, v in d.items():
         if not isinstance(v, dict):
             continue
-        groups = {k: v} if "rows" in v else {f"{k}/{kk}": vv for sub in ("kernels", "filters") for kk, vv in v.get(sub, {}).items()}
+        groups = {k: v} if "rows" in v else {f"{k}/{kk}": vv for sub in ("kernels", "filters", "inputs") for kk, vv in v.get(sub, {}).items()}
         for g, vv in groups.items():
             lines.append(f"== {g}  {v.get('config', '')}")
             for r in vv.get("rows", []):

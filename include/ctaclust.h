@@ -184,7 +184,8 @@ typedef enum {
     CC_K_MVT = 4,      /* cc_mvt_args      (Table 2 MVT)                            */
     CC_K_JACOBI5 = 5,  /* cc_jacobi5_args  (config 3)                               */
     CC_K_CONV2D = 6,   /* cc_conv2d_args   (config 4)                               */
-    CC_K_SPMV = 7      /* cc_spmv_args     (config 5)                               */
+    CC_K_SPMV = 7,     /* cc_spmv_args     (config 5)                               */
+    CC_K_HIST64 = 8    /* cc_hist64_args   (S§8(f)3, the paper's HST)               */
 } cc_kernel;
 
 /* CC_K_CENSUS: no data. */
@@ -227,6 +228,16 @@ typedef struct { const float* in; float* out; int64_t ld; int32_t rows, cols; in
  * per matrix structure. */
 typedef struct { int32_t rows, cols; int64_t nnz; const int32_t* row_ptr; const int32_t* col;
                  const float* val; const float* x; float* y; const int32_t* part; } cc_spmv_args;
+/* CC_K_HIST64 -- 64-bin histogram, the paper's HST (Table 2; data-
+ * related); reading R24 (CUDA SDK histogram64):
+ *     counts[k] = #{ i < n : data[i] >> 2 == k },  k = 0..63.
+ * data: DEVICE, n bytes, 16-byte aligned; counts: DEVICE uint32[64], zeroed by
+ * the call (cudaMemsetAsync on `stream`) then accumulated; 0 <= n < 2^32.
+ * Logical CTA b counts the 32 KiB chunk [32768 b, 32768 (b+1)); grid =
+ * ceil(n / 32768) x 1.  Persistent agents keep per-warp shared sub-histograms
+ * across their chunks and flush once; one-shot CTAs flush per chunk. */
+typedef struct { const uint8_t* data; int64_t n; uint32_t* counts; } cc_hist64_args;
+
 /* Fill args->part-sized DEVICE table `part` (gx+1 entries, gx from
  * cc_kernel_grid) with the merge-path row coordinate of each logical CTA's
  * first diagonal.  Asynchronous on `stream`. */

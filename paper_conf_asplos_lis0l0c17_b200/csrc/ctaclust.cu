@@ -20,6 +20,7 @@
 #include "k_gemv.cuh"
 #include "k_spmv.cuh"
 #include "k_microbench.cuh"
+#include "k_hist.cuh"
 #include "k_stencil.cuh"
 #include "k_tbcluster.cuh"
 
@@ -294,6 +295,11 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
         if (b > INT32_MAX - 1) return fail(CC_ERR_OVERFLOW, "spmv grid");
         *gx = (int32_t)b; *gy = 1; return CC_OK;
     }
+    case CC_K_HIST64: {
+        auto* c = (const cc_hist64_args*)a;
+        if (c->n < 0 || c->n > (int64_t)UINT32_MAX) return fail(CC_ERR_INVALID_ARG, "hist64: n %lld outside [0, 2^32)", (long long)c->n);
+        *gx = cdiv(c->n, HIST_CHUNK); *gy = 1; return CC_OK;
+    }
     default: return fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
     }
 }
@@ -381,6 +387,7 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, Jacobi5Body::kDefaultStages, &occ); break;
     case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, Conv2dBody<3>::kDefaultStages, &occ); break;
     case CC_K_SPMV: s = occupancy<SpmvBody>(device, SpmvBody::kDefaultStages, &occ); break;
+    case CC_K_HIST64: s = occupancy<HistBody>(device, HistBody::kDefaultStages, &occ); break;
     default: return fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
     }
     if (s == CC_OK) *out = occ;
@@ -686,6 +693,14 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             return fail(CC_ERR_INVALID_ARG, "spmv null pointer");
         if (x->rows) CC_CUDA(cudaMemsetAsync(x->y, 0, sizeof(float) * x->rows, st));
         s = launch_body<SpmvBody>(c, SpmvParams{x->rows, x->nnz, x->row_ptr, x->col, x->val, x->x, x->y, x->part});
+        break;
+    }
+    case CC_K_HIST64: {
+        auto* x = (const cc_hist64_args*)a;
+        if (!x->counts || (x->n > 0 && !x->data)) return fail(CC_ERR_INVALID_ARG, "hist64 null pointer");
+        if (x->n > 0 && !al16(x->data)) return fail(CC_ERR_INVALID_ARG, "hist64: data must be 16-byte aligned");
+        CC_CUDA(cudaMemsetAsync(x->counts, 0, 64 * sizeof(uint32_t), st));
+        s = launch_body<HistBody>(c, HistParams{x->data, x->n, x->counts});
         break;
     }
     default:

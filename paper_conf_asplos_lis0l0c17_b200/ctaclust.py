@@ -23,7 +23,8 @@ BACKEND_DEFAULT, BACKEND_AGENT, BACKEND_TBCLUSTER, BACKEND_AGENT_IDENTITY, BACKE
 BACKENDS = {"default": 0, "agent": 1, "tbcluster": 2, "identity": 3, "redirect": 4}
 K_CENSUS, K_MATVEC, K_ATAX, K_BICG, K_MVT, K_JACOBI5, K_CONV2D, K_SPMV = range(8)
 STAGINGS = {"default": 0, "tma": 1, "l1": 2, "direct": 3}
-KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7}
+KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7,
+           "hist64": 8}
 STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_ERR_NOT_PERMUTATION",
           -4: "CC_ERR_CUDA", -5: "CC_ERR_NCCL", -6: "CC_ERR_UNSUPPORTED", -7: "CC_ERR_NO_DEVICE"}
 
@@ -273,6 +274,14 @@ def conv2d_args(inp, out, w, rows=None, cols=None) -> tuple[Conv2dArgs, np.ndarr
     rows = inp.shape[0] if rows is None else rows
     cols = inp.shape[1] if cols is None else cols
     return Conv2dArgs(inp.data_ptr(), out.data_ptr(), _lda(inp), rows, cols, K // 2, w.ctypes.data), w
+
+
+class Hist64Args(ctypes.Structure):
+    _fields_ = [("data", _vp), ("n", _i64), ("counts", _vp)]
+
+
+def hist64_args(data, counts) -> Hist64Args:
+    return Hist64Args(_ptr(data), int(data.numel()), _ptr(counts))
 
 
 def spmv_args(row_ptr, col, val, x, y, part=None) -> SpmvArgs:

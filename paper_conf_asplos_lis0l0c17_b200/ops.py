@@ -17,7 +17,7 @@ from . import ctaclust as cc
 # fastest with TMA staging, so it is the default here.
 DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": ("col", (1, 1)),
                  "bicg": ("col", (1, 1)), "mvt": ("col", (1, 1)), "jacobi5": ("row", (1, 1)),
-                 "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1))}
+                 "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1))}
 
 _plans: dict = {}
 
@@ -109,6 +109,16 @@ def spmv(Amat: SpmvMatrix, x, y=None, backend="agent", order=None, tile=None, nu
                        Amat.val.data_ptr(), x.data_ptr(), y.data_ptr(), Amat.part.data_ptr())
     _launch("spmv", args, backend, order, tile, num_clusters, _dev(x), stream, **kw)
     return y
+
+
+def hist64(data, counts=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+    """64-bin histogram of a uint8 device tensor (bin = byte >> 2, reading R24);
+    returns uint32[64] counts (zeroed by the call)."""
+    if data.dtype != torch.uint8 or not data.is_contiguous():
+        raise cc.CtaclustError(-1, "hist64 expects a contiguous uint8 tensor")
+    counts = torch.empty(64, dtype=torch.int32, device=data.device) if counts is None else counts
+    _launch("hist64", cc.hist64_args(data, counts), backend, order, tile, num_clusters, _dev(data), stream, **kw)
+    return counts
 
 
 def census(gx, gy, backend="agent", order="row", tile=(1, 1), num_clusters=0, device=0, stream=None,

@@ -19,7 +19,8 @@ sys.path.insert(0, ROOT)
 KERNELS = {  # name: (ncu_target kernel, launches per call, has L1/TMA staging, writes shifted reads)
     "matvec": ("matvec", 1, False, False), "atax": ("atax", 2, False, False), "bicg": ("bicg", 1, False, False),
     "mvt": ("mvt", 1, False, False), "jacobi5": ("jacobi", 1, True, False), "conv3x3": ("conv3", 1, True, False),
-    "conv7x7": ("conv7", 1, True, False), "spmv": ("spmv", 1, False, False)}
+    "conv7x7": ("conv7", 1, True, False), "spmv": ("spmv", 1, False, False),
+    "hist64": ("hist", 1, False, False)}
 
 
 def ncu_probe(out_dir, name, kern, per, args):
@@ -72,6 +73,10 @@ def full_size_runner(name):
         Am = ops.SpmvMatrix(rp, col, val)
         y = torch.empty(rp.numel() - 1, device="cuda")
         return (lambda **kw: ops.spmv(Am, x, y, **kw)), 1
+    if name == "hist64":
+        data = synth.bytes_u8(31, 1 << 30, backend="torch", device="cuda")
+        counts = torch.empty(64, dtype=torch.int32, device="cuda")
+        return (lambda **kw: ops.hist64(data, counts, **kw)), 1
     raise KeyError(name)
 
 

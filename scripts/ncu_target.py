@@ -80,6 +80,11 @@ def main():
             fn = lambda: torch.mv(Acsr, x)
         else:
             fn = lambda: ops.spmv(Am, x, y, **kw)
+    elif k in ("hist", "hist_skewed"):
+        n = 1 << (28 if a.small else 30)
+        data = synth.bytes_u8(31, n, kind="skewed" if k == "hist_skewed" else "uniform", backend="torch", device=dev)
+        counts = torch.empty(64, dtype=torch.int32, device=dev)
+        fn = lambda: ops.hist64(data, counts, **kw)
     else:
         raise SystemExit(f"unknown kernel {k}")
     torch.cuda.synchronize()

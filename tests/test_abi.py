@@ -49,6 +49,7 @@ int main(void) {
   S(cc_bicg_args) O(cc_bicg_args, s) S(cc_mvt_args) O(cc_mvt_args, x2)
   S(cc_jacobi5_args) O(cc_jacobi5_args, result_is_b) S(cc_conv2d_args) O(cc_conv2d_args, w)
   S(cc_spmv_args) O(cc_spmv_args, part) O(cc_spmv_args, nnz)
+  S(cc_hist64_args) O(cc_hist64_args, n) O(cc_hist64_args, counts)
   return 0;
 }
 """
@@ -62,7 +63,8 @@ def test_struct_layouts_match_binding(tmp_path):
     got = dict(ln.rsplit(" ", 1) for ln in subprocess.check_output([str(exe)], text=True).splitlines())
     py = {"cc_plan_desc": cc.PlanDesc, "cc_launch_opts": cc.LaunchOpts, "cc_matvec_args": cc.MatvecArgs,
           "cc_atax_args": cc.AtaxArgs, "cc_bicg_args": cc.BicgArgs, "cc_mvt_args": cc.MvtArgs,
-          "cc_jacobi5_args": cc.Jacobi5Args, "cc_conv2d_args": cc.Conv2dArgs, "cc_spmv_args": cc.SpmvArgs}
+          "cc_jacobi5_args": cc.Jacobi5Args, "cc_conv2d_args": cc.Conv2dArgs, "cc_spmv_args": cc.SpmvArgs,
+          "cc_hist64_args": cc.Hist64Args}
     for key, val in got.items():
         if "." in key:
             t, f = key.split(".")
@@ -161,3 +163,8 @@ def test_kernel_grid():
     assert cc.kernel_grid("conv2d", cc.Conv2dArgs(None, None, 8192, 8192, 8192, 3)) == (256, 256)
     a = cc.SpmvArgs(1 << 24, 1 << 24, 1 << 28)
     assert cc.kernel_grid("spmv", a) == (((1 << 24) + (1 << 28) + 4095) // 4096, 1)
+    assert cc.kernel_grid("hist64", cc.Hist64Args(None, 1 << 30, None)) == (32768, 1)
+    assert cc.kernel_grid("hist64", cc.Hist64Args(None, 32769, None)) == (2, 1)
+    assert cc.kernel_grid("hist64", cc.Hist64Args(None, 0, None)) == (0, 1)
+    with pytest.raises(cc.CtaclustError):
+        cc.kernel_grid("hist64", cc.Hist64Args(None, 1 << 32, None))

@@ -297,3 +297,35 @@ def test_spmv(v):
         torch.cuda.synchronize()
         assert np.array_equal(y.cpu().numpy().astype(np.float64),
                               O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), vi, xi)), name
+
+
+# ---- S8(f)3: 64-bin histogram (HST, reading R24) -- integer counts, bit-exact ----
+HVARIANTS = [dict(backend="default"), dict(backend="agent", order="row"), dict(backend="agent", order="col"),
+             dict(backend="identity"), dict(backend="redirect", order="row"),
+             dict(backend="default", staging="direct"), dict(backend="agent", order="row", staging="direct"),
+             dict(backend="agent", order="row", staging="l1"), dict(backend="agent", order="row", active_agents=1),
+             dict(backend="agent", order="row", stages=4, batch=3), dict(backend="agent", order="row", stages=1),
+             dict(backend="agent", order="row", l2_hint="both")]
+
+
+@pytest.mark.parametrize("v", HVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
+def test_hist64(v):
+    for n in (0, 1, 15, 16, 17, 32768, 32769, 100003, 5 * 32768 + 7):
+        for kind in ("uniform", "skewed"):
+            data = synth.bytes_u8(30 + n % 7, n, kind=kind)
+            got = ops.hist64(torch.from_numpy(data).cuda(), **v)
+            torch.cuda.synchronize()
+            ref = O.hist64(data)
+            assert np.array_equal(got.cpu().numpy().view(np.uint32).astype(np.uint64), ref), (n, kind)
+
+
+def test_hist64_full_size_and_errors():
+    n = 1 << 30
+    data = synth.bytes_u8(31, n, backend="torch", device="cuda")
+    ref = O.hist64(data.cpu().numpy())
+    for v in (dict(backend="default"), dict(backend="agent", order="row")):
+        got = ops.hist64(data, **v)
+        torch.cuda.synchronize()
+        assert np.array_equal(got.cpu().numpy().view(np.uint32).astype(np.uint64), ref), v
+    with pytest.raises(Exception):
+        ops.hist64(data[1:1025])                  # not 16-byte aligned
