@@ -44,3 +44,6 @@ done
 run spmv_default 1 --kernel spmv --backend default
 run spmv_agent-row 1 --kernel spmv --backend agent --order row
 run spmv_identity 1 --kernel spmv --backend identity
+run hist_default 1 --kernel hist --backend default
+run hist_agent-row 1 --kernel hist --backend agent --order row
+run hist_identity 1 --kernel hist --backend identity
