@@ -234,13 +234,16 @@ __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const 
 
 template <int R>
 struct Conv2dBody {
-    static constexpr int RB = 2;                  // output rows per consumer thread
+    // output rows per consumer thread: the 7x7 filter is FP32-issue bound, so
+    // each thread takes 4 rows (784 FFMA per task against a fixed per-task
+    // overhead of ~150 instructions per warp); the 3x3 is HBM bound
+    static constexpr int RB = R >= 3 ? 4 : 2;
     static constexpr int kConsumers = 256 / RB;
     static constexpr int kStageBytes = HaloTile<R>::kBytes;
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
-    static constexpr int kMinAgents = 5;
-    static constexpr int kGroups = 2;              // two 4-warp groups consume alternate tiles
+    static constexpr int kMinAgents = R >= 3 ? 4 : 5;
+    static constexpr int kGroups = 256 / kConsumers;   // 2 or 4 groups consume alternate tiles
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
@@ -252,7 +255,9 @@ struct Conv2dBody {
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         if (s.staging == STAGE_DIRECT) {
             // plain-kernel form: the consumers stage the tile themselves through L1
-            __shared__ float4 s_in[HaloTile<R>::kRows][ST_COLS / 4];
+            // (one buffer per consumer group: groups work on different tiles)
+            __shared__ float4 s_in_g[kGroups][HaloTile<R>::kRows][ST_COLS / 4];
+            auto& s_in = s_in_g[(threadIdx.x - PRODUCER_THREADS) / kConsumers];
             const int x0 = bx * 32, y0 = by * 32;
             for (int idx = ctid; idx < HaloTile<R>::kRows * 10; idx += kConsumers) {
                 const int rr = idx / 10, cc = idx - rr * 10;
