@@ -185,7 +185,8 @@ typedef enum {
     CC_K_JACOBI5 = 5,  /* cc_jacobi5_args  (config 3)                               */
     CC_K_CONV2D = 6,   /* cc_conv2d_args   (config 4)                               */
     CC_K_SPMV = 7,     /* cc_spmv_args     (config 5)                               */
-    CC_K_HIST64 = 8    /* cc_hist64_args   (S§8(f)3, the paper's HST)               */
+    CC_K_HIST64 = 8,   /* cc_hist64_args   (S§8(f)3, the paper's HST)               */
+    CC_K_JACOBI5_HALO = 9 /* cc_jacobi5_halo_args (S§8(f)4: sharded sweep, fused peer halo) */
 } cc_kernel;
 
 /* CC_K_CENSUS: no data. */
@@ -213,6 +214,62 @@ typedef struct { const float* A; int64_t lda; int32_t m, n; const float* y1; con
  * rows x cols fp32 DEVICE with leading dim ld (% 4 == 0).  Logical CTA = 32 x 32
  * output tile; grid ceil(cols/32) x ceil(rows/32). */
 typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t iters; int32_t* result_is_b; } cc_jacobi5_args;
+
+/* CC_K_JACOBI5_HALO -- S§8(f)4: one rank's slab of the slab-sharded Jacobi
+ * (S§8(e), config 3) with the per-sweep halo exchange fused into the sweep
+ * kernel over peer memory, replacing cc_halo_exchange's NCCL send/recv.
+ * The slab a/b (DEVICE, rows x cols, ld) holds this rank's owned rows plus one
+ * halo row above (row 0, when up_a != NULL) and below (row rows-1, when
+ * dn_a != NULL); the arithmetic is CC_K_JACOBI5's (halo and global boundary
+ * rows are fixed during a sweep).  In sweep s the tile computing the first
+ * (last) owned row also stores it into the upper (lower) neighbour's halo row
+ * of its destination buffer and raises the neighbour's flag for that tile
+ * column to s; a tile reading a halo row first waits until the neighbour's
+ * flags for columns bx-1..bx+1 reach s-1 (this covers RAW on the halo and
+ * WAR on the neighbour's copy).  Halo rows of this rank's b are written only
+ * by the neighbours.
+ *   a, b            this call's first source / destination (ping-pong as in
+ *                   CC_K_JACOBI5; *result_is_b as there)
+ *   iters, sweep0   runs absolute sweeps sweep0+1 .. sweep0+iters; flags
+ *                   count absolute sweeps since they were zeroed
+ *   up_a, up_b      the upper neighbour's a and b in the same roles, mapped
+ *                   into this process (same device, cc_peer_access, or
+ *                   cc_ipc_open); NULL = no upper neighbour.  up_rows: its
+ *                   slab rows (its bottom halo is row up_rows-1)
+ *   dn_a, dn_b      the lower neighbour's (its top halo is its row 0)
+ *   flags           DEVICE uint32[2*gx] (gx = ceil(cols/32)): [0,gx) deposits
+ *                   from up, [gx,2gx) from down; zeroed by the caller (on every
+ *                   rank, before any rank's sweep 1) with sweep0 = 0
+ *   up_flags, dn_flags  the neighbours' `flags`, mapped like up_a/dn_a
+ *   status          DEVICE int32, optional: set to 1 if a wait exceeded 4 s (a
+ *                   neighbour not running); results are then invalid
+ * Every rank uses the same cols and ld.  Staging must be TMA (default): halo
+ * rows are read after a system-scope acquire, never through L1.  Launches of
+ * neighbouring ranks may run concurrently (one GPU each) or be interleaved
+ * sweep by sweep on one stream (virtual slabs on one GPU); a rank's sweep s
+ * must not be queued behind a neighbour's sweep s+1 on one stream.
+ * Errors: INVALID_ARG (sizes, a neighbour pointer without its flags, owned
+ * rows < 1), UNSUPPORTED (staging other than TMA, TBCLUSTER backend). */
+typedef struct {
+    float* a; float* b; int64_t ld; int32_t rows, cols; int32_t iters; int32_t sweep0; int32_t* result_is_b;
+    float* up_a; float* up_b; int32_t up_rows;
+    float* dn_a; float* dn_b;
+    uint32_t* flags; uint32_t* up_flags; uint32_t* dn_flags;
+    int32_t* status;
+} cc_jacobi5_halo_args;
+
+/* Peer memory for CC_K_JACOBI5_HALO (S§8(f)4).  cc_peer_access enables P2P
+ * loads/stores from `device` to `peer` (NVLink on a B200 box); a no-op when
+ * device == peer or access is already enabled.  cc_ipc_handle exports the
+ * DEVICE allocation holding dptr (cudaIpcGetMemHandle; 64-byte HOST handle
+ * out) and dptr's byte offset in it (*offset, HOST); cc_ipc_open maps another
+ * process's handle into this one on `device` (*dptr out = the allocation's
+ * base: add the exporter's offset; close with cc_ipc_close).  Errors:
+ * INVALID_ARG, UNSUPPORTED (no P2P path), CUDA. */
+cc_status cc_peer_access(int32_t device, int32_t peer);
+cc_status cc_ipc_handle(const void* dptr, void* handle64, uint64_t* offset);
+cc_status cc_ipc_open(const void* handle64, int32_t device, void** dptr);
+cc_status cc_ipc_close(void* dptr);
 
 /* 2D cross-correlation (R15) with a (2R+1)^2 filter w (HOST, copied into the
  * launch parameters), R in {1, 3}; out = 0 outside [R, rows-R) x [R, cols-R).

@@ -288,6 +288,7 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
     case CC_K_BICG: { auto* c = (const cc_bicg_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
     case CC_K_MVT: { auto* c = (const cc_mvt_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
     case CC_K_JACOBI5: { auto* c = (const cc_jacobi5_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
+    case CC_K_JACOBI5_HALO: { auto* c = (const cc_jacobi5_halo_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
     case CC_K_CONV2D: { auto* c = (const cc_conv2d_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
     case CC_K_SPMV: {
         auto* c = (const cc_spmv_args*)a;
@@ -385,6 +386,7 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     case CC_K_ATAX: s = occupancy<RowB>(device, RowB::kDefaultStages, &occ); break;
     case CC_K_BICG: case CC_K_MVT: s = occupancy<BothB>(device, BothB::kDefaultStages, &occ); break;
     case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, Jacobi5Body::kDefaultStages, &occ); break;
+    case CC_K_JACOBI5_HALO: s = occupancy<Jacobi5HaloBody>(device, Jacobi5HaloBody::kDefaultStages, &occ); break;
     case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, Conv2dBody<3>::kDefaultStages, &occ); break;
     case CC_K_SPMV: s = occupancy<SpmvBody>(device, SpmvBody::kDefaultStages, &occ); break;
     case CC_K_HIST64: s = occupancy<HistBody>(device, HistBody::kDefaultStages, &occ); break;
@@ -660,6 +662,44 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         if (x->result_is_b) *x->result_is_b = (x->iters & 1) ? 1 : 0;
         break;
     }
+    case CC_K_JACOBI5_HALO: {
+        auto* x = (const cc_jacobi5_halo_args*)a;
+        CC_TRY(check_mat(x->a, x->ld, x->rows, x->cols));
+        CC_TRY(check_mat(x->b, x->ld, x->rows, x->cols));
+        if (x->iters < 0 || x->sweep0 < 0) return fail(CC_ERR_INVALID_ARG, "iters / sweep0 < 0");
+        const bool up = x->up_a || x->up_b, dn = x->dn_a || x->dn_b;
+        if (up && (!x->up_a || !x->up_b || !x->up_flags || x->up_rows < 2))
+            return fail(CC_ERR_INVALID_ARG, "upper neighbour needs up_a, up_b, up_flags and up_rows >= 2");
+        if (dn && (!x->dn_a || !x->dn_b || !x->dn_flags))
+            return fail(CC_ERR_INVALID_ARG, "lower neighbour needs dn_a, dn_b and dn_flags");
+        if ((up || dn) && !x->flags) return fail(CC_ERR_INVALID_ARG, "null flags");
+        if (x->rows - (up ? 1 : 0) - (dn ? 1 : 0) < 1) return fail(CC_ERR_INVALID_ARG, "slab has no owned row");
+        const int32_t st_mode = o->staging == CC_STAGING_DEFAULT ? CC_STAGING_TMA : o->staging;
+        if (st_mode != CC_STAGING_TMA) return fail(CC_ERR_UNSUPPORTED, "fused halo needs TMA staging");
+        float* src = x->a;
+        float* dst = x->b;
+        float* usrc = x->up_a; float* udst = x->up_b;
+        float* dsrc = x->dn_a; float* ddst = x->dn_b;
+        for (int it = 0; it < x->iters && s == CC_OK; ++it) {
+            JacobiParams jp;
+            memset(&jp, 0, sizeof jp);
+            jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
+            if (up || dn) {
+                jp.h.up_dst = up ? udst : nullptr;
+                jp.h.dn_dst = dn ? ddst : nullptr;
+                jp.h.up_row = x->up_rows - 1;
+                jp.h.gx = p->g.gx;
+                jp.h.flags = x->flags; jp.h.up_flags = x->up_flags; jp.h.dn_flags = x->dn_flags;
+                jp.h.status = x->status;
+                jp.h.sweep = (uint32_t)(x->sweep0 + it + 1);
+            }
+            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
+            s = (up || dn) ? launch_body<Jacobi5HaloBody>(c, jp) : launch_body<Jacobi5Body>(c, jp);
+            std::swap(src, dst); std::swap(usrc, udst); std::swap(dsrc, ddst);
+        }
+        if (x->result_is_b) *x->result_is_b = (x->iters & 1) ? 1 : 0;
+        break;
+    }
     case CC_K_CONV2D: {
         auto* x = (const cc_conv2d_args*)a;
         CC_TRY(check_mat(x->in, x->ld, x->rows, x->cols));
@@ -718,6 +758,66 @@ extern "C" cc_status cc_l1_reuse_probe(int32_t ctas, int32_t stagger_cycles, con
     k_l1_reuse_probe<<<ctas, 32, 0, (cudaStream_t)stream>>>(input, smid, ticks, sink, stagger_cycles);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "l1 reuse probe");
+    return CC_OK;
+}
+
+// ---- peer memory for the fused halo (S§8(f)4) -------------------------------
+extern "C" cc_status cc_peer_access(int32_t device, int32_t peer) {
+    if (device < 0 || peer < 0) return fail(CC_ERR_INVALID_ARG, "device %d / peer %d", device, peer);
+    if (device == peer) return CC_OK;
+    int ok = 0;
+    CC_CUDA(cudaDeviceCanAccessPeer(&ok, device, peer));
+    if (!ok) return fail(CC_ERR_UNSUPPORTED, "device %d cannot access peer %d", device, peer);
+    int prev = 0;
+    CC_CUDA(cudaGetDevice(&prev));
+    CC_CUDA(cudaSetDevice(device));
+    cudaError_t e = cudaDeviceEnablePeerAccess(peer, 0);
+    cudaSetDevice(prev);
+    if (e == cudaErrorPeerAccessAlreadyEnabled) { cudaGetLastError(); return CC_OK; }
+    if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceEnablePeerAccess");
+    return CC_OK;
+}
+// IPC maps whole allocations: the handle names the allocation holding dptr
+// (a caching allocator hands out sub-blocks), *offset is dptr's byte offset in it.
+extern "C" cc_status cc_ipc_handle(const void* dptr, void* handle64, uint64_t* offset) {
+    if (!dptr || !handle64 || !offset) return fail(CC_ERR_INVALID_ARG, "null pointer");
+    static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+    using RangeFn = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+    static RangeFn range = nullptr;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        cudaDriverEntryPointQueryResult q;
+        void* f = nullptr;
+        if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            range = (RangeFn)f;
+    });
+    if (!range) return fail(CC_ERR_UNSUPPORTED, "cuMemGetAddressRange unavailable");
+    CUdeviceptr base = 0;
+    size_t size = 0;
+    CUresult r = range(&base, &size, (CUdeviceptr)dptr);
+    if (r != CUDA_SUCCESS) return fail(CC_ERR_CUDA, "cuMemGetAddressRange failed (%d)", (int)r);
+    cudaIpcMemHandle_t h;
+    CC_CUDA(cudaIpcGetMemHandle(&h, (void*)base));
+    memcpy(handle64, &h, 64);
+    *offset = (uint64_t)((CUdeviceptr)dptr - base);
+    return CC_OK;
+}
+extern "C" cc_status cc_ipc_open(const void* handle64, int32_t device, void** dptr) {
+    if (!handle64 || !dptr || device < 0) return fail(CC_ERR_INVALID_ARG, "null pointer / device");
+    cudaIpcMemHandle_t h;
+    memcpy(&h, handle64, 64);
+    int prev = 0;
+    CC_CUDA(cudaGetDevice(&prev));
+    CC_CUDA(cudaSetDevice(device));
+    cudaError_t e = cudaIpcOpenMemHandle(dptr, h, cudaIpcMemLazyEnablePeerAccess);
+    cudaSetDevice(prev);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaIpcOpenMemHandle");
+    return CC_OK;
+}
+extern "C" cc_status cc_ipc_close(void* dptr) {
+    if (!dptr) return fail(CC_ERR_INVALID_ARG, "null pointer");
+    CC_CUDA(cudaIpcCloseMemHandle(dptr));
     return CC_OK;
 }
 

@@ -89,7 +89,70 @@ __device__ __forceinline__ void store4_out(float* dst, float4 o, int gx, int col
 // fp32, summed in that fixed order with no contraction, so the sweep is
 // bit-reproducible against oracle_jacobi5_f32 in every staging mode.
 // ---------------------------------------------------------------------------
-struct JacobiParams { CUtensorMap tmap; const float* a; float* b; int64_t ld; int32_t rows, cols; };
+// Fused peer-memory halo exchange of the slab-sharded sweep (S§8(f)4,
+// CC_K_JACOBI5_HALO): the tile that computes a slab's first (last) owned row
+// also stores it into the upper (lower) neighbour's halo row -- through
+// NVLink peer mappings on a multi-GPU box, or plain device pointers for
+// virtual slabs on one GPU -- and then raises that neighbour's per-tile-column
+// flag to the absolute sweep number.  A tile that reads a halo row (and so
+// also writes the neighbour's halo of the next buffer) first waits, in the
+// producer before its TMA, until the neighbour's tiles bx-1..bx+1 have
+// deposited sweep s-1: that one condition covers both the data it reads (RAW)
+// and the neighbour having finished reading the halo row it is about to
+// overwrite (WAR: the neighbour's depositing tile is its halo-reading tile).
+// All pointers null = the unsharded sweep.
+struct JacobiHalo {
+    float* up_dst;            // upper neighbour's destination buffer of this sweep (null: none)
+    float* dn_dst;            // lower neighbour's destination buffer (its top halo is row 0)
+    int32_t up_row;           // the upper neighbour's bottom halo row (its rows - 1)
+    int32_t gx;               // tile columns (same on every rank: equal cols)
+    uint32_t* flags;          // mine [2 gx]: [0, gx) deposits from up, [gx, 2 gx) from down
+    uint32_t* up_flags;       // upper neighbour's flags (I write its "from down" half)
+    uint32_t* dn_flags;       // lower neighbour's flags (I write its "from up" half)
+    int32_t* status;          // optional: 1 = a wait timed out (results invalid)
+    uint32_t sweep;           // absolute sweep number of this launch (1-based)
+};
+struct JacobiParams { CUtensorMap tmap; const float* a; float* b; int64_t ld; int32_t rows, cols; JacobiHalo h; };
+
+__device__ __forceinline__ uint64_t globaltimer() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+// wait until flags[bx-1 .. bx+1] >= need (acquire, system scope), bounded: a
+// call that waits longer than 4 s in total flags *status and gives up (as does
+// every later wait once *status is set), so a broken peer cannot hang the GPU;
+// then order the generic-proxy peer writes before this thread's TMA
+// (async-proxy) reads of the halo row.
+__device__ __forceinline__ void halo_wait(const uint32_t* flags, int32_t bx, int32_t gx, uint32_t need,
+                                          int32_t* status) {
+    const int32_t k0 = bx > 0 ? bx - 1 : 0, k1 = bx + 1 < gx ? bx + 1 : gx - 1;
+    uint64_t t0 = 0;
+    for (int32_t k = k0; k <= k1; ++k) {
+        while (ld_acquire_sys(flags + k) < need) {
+            if (t0 == 0) {
+                if (status && *(volatile int32_t*)status) break;      // an earlier wait already gave up
+                t0 = globaltimer();
+            }
+            __nanosleep(256);
+            if (globaltimer() - t0 > 4000000000ull) {
+                if (status) atomicExch(status, 1);
+                break;
+            }
+        }
+    }
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+// make this CTA's peer stores (ordered before us by the group barrier) visible
+// system-wide, then publish the sweep number in the neighbour's flag
+__device__ __forceinline__ void halo_signal(uint32_t* flag, uint32_t sweep) {
+    asm volatile("fence.acq_rel.sys;\n\tst.relaxed.sys.global.u32 [%0], %1;" :: "l"(flag), "r"(sweep) : "memory");
+}
 
 __device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, float lw, float re,
                                                int gy, int gx, int rows, int cols) {
@@ -107,7 +170,10 @@ __device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, 
     return o;
 }
 
-struct Jacobi5Body {
+// HALO = true is the fused peer-halo form (CC_K_JACOBI5_HALO); the plain
+// sweep is a separate instantiation, so it carries none of its code.
+template <bool HALO>
+struct Jacobi5BodyT {
     static constexpr int RB = 2;                  // output rows per consumer thread
     static constexpr int kConsumers = 256 / RB;
     static constexpr int kStageBytes = HaloTile<1>::kBytes;
@@ -118,9 +184,17 @@ struct Jacobi5Body {
     using Params = JacobiParams;
     const JacobiParams& p;   // __grid_constant__ kernel parameter
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
-    __device__ __forceinline__ explicit Jacobi5Body(const JacobiParams& prm) : p(prm) {}
+    __device__ __forceinline__ explicit Jacobi5BodyT(const JacobiParams& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+        if (HALO && p.h.flags) {                  // fused halo: wait for the neighbours' deposits of sweep s-1
+            if (lane == 0) {
+                if (p.h.up_dst && by == 0) halo_wait(p.h.flags, bx, p.h.gx, p.h.sweep - 1, p.h.status);
+                if (p.h.dn_dst && by * 32 + 32 >= p.rows - 1)
+                    halo_wait(p.h.flags + p.h.gx, bx, p.h.gx, p.h.sweep - 1, p.h.status);
+            }
+            __syncwarp();
+        }
         HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h);
     }
 
@@ -161,18 +235,43 @@ struct Jacobi5Body {
                 re[j] = t[(j + 1) * ST_COLS + 4];
             }
         }
-        if (!in_col) return;
+        if (!HALO || !p.h.flags) {
+            if (!in_col) return;
+#pragma unroll
+            for (int j = 0; j < RB; ++j) {
+                const int gy = gy0 + j;
+                if (gy >= p.rows) break;
+                store4_out(p.b + (int64_t)gy * p.ld + gx,
+                           jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx,
+                           p.cols, l2h);
+            }
+            return;
+        }
+        // fused halo: halo rows are the neighbours' to write; the first / last
+        // owned rows also go to the neighbours' halo rows
+        const bool up = p.h.up_dst != nullptr, dn = p.h.dn_dst != nullptr;
 #pragma unroll
         for (int j = 0; j < RB; ++j) {
             const int gy = gy0 + j;
-            if (gy >= p.rows) break;
-            store4_out(p.b + (int64_t)gy * p.ld + gx,
-                       jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx, p.cols,
-                       l2h);
+            if (!in_col || gy >= p.rows || (up && gy == 0) || (dn && gy == p.rows - 1)) continue;
+            const float4 o = jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols);
+            store4_masked(p.b + (int64_t)gy * p.ld + gx, o, gx, p.cols);
+            if (up && gy == 1) store4_masked(p.h.up_dst + (int64_t)p.h.up_row * p.ld + gx, o, gx, p.cols);
+            if (dn && gy == p.rows - 2) store4_masked(p.h.dn_dst + gx, o, gx, p.cols);
+        }
+        const bool to_up = up && by == 0, to_dn = dn && by == (p.rows - 2) / 32;   // uniform per tile
+        if (to_up || to_dn) {
+            consumer_sync<kConsumers>();             // every peer store of the tile precedes the signal
+            if (ctid == 0) {
+                if (to_up) halo_signal(p.h.up_flags + p.h.gx + bx, p.h.sweep);
+                if (to_dn) halo_signal(p.h.dn_flags + bx, p.h.sweep);
+            }
         }
     }
     __device__ __forceinline__ void finish(int) {}
 };
+using Jacobi5Body = Jacobi5BodyT<false>;
+using Jacobi5HaloBody = Jacobi5BodyT<true>;
 
 // ---------------------------------------------------------------------------
 // 2D cross-correlation with a (2R+1)^2 filter (reading R15):

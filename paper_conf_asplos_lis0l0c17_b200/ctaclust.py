@@ -24,7 +24,7 @@ BACKENDS = {"default": 0, "agent": 1, "tbcluster": 2, "identity": 3, "redirect":
 K_CENSUS, K_MATVEC, K_ATAX, K_BICG, K_MVT, K_JACOBI5, K_CONV2D, K_SPMV = range(8)
 STAGINGS = {"default": 0, "tma": 1, "l1": 2, "direct": 3}
 KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7,
-           "hist64": 8}
+           "hist64": 8, "jacobi5_halo": 9}
 STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_ERR_NOT_PERMUTATION",
           -4: "CC_ERR_CUDA", -5: "CC_ERR_NCCL", -6: "CC_ERR_UNSUPPORTED", -7: "CC_ERR_NO_DEVICE"}
 
@@ -33,7 +33,7 @@ EXPORTS = ["cc_plan_create", "cc_plan_destroy", "cc_plan_info", "cc_plan_table",
            "cc_plan_invert", "cc_device_info", "cc_sm_rank_table", "cc_launch_opts_default",
            "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_l1_reuse_probe", "cc_comm_unique_id",
            "cc_comm_init", "cc_comm_destroy", "cc_halo_exchange", "cc_allreduce_sum", "cc_allgather",
-           "cc_status_string", "cc_last_error", "cc_last_cuda_error", "cc_version"]
+           "cc_peer_access", "cc_ipc_handle", "cc_ipc_open", "cc_ipc_close", "cc_status_string", "cc_last_error", "cc_last_cuda_error", "cc_version"]
 
 
 class CtaclustError(RuntimeError):
@@ -81,6 +81,12 @@ class MvtArgs(ctypes.Structure):
 class Jacobi5Args(ctypes.Structure):
     _fields_ = [("a", _vp), ("b", _vp), ("ld", _i64), ("rows", _i32), ("cols", _i32), ("iters", _i32),
                 ("result_is_b", _vp)]
+
+
+class Jacobi5HaloArgs(ctypes.Structure):
+    _fields_ = [("a", _vp), ("b", _vp), ("ld", _i64), ("rows", _i32), ("cols", _i32), ("iters", _i32),
+                ("sweep0", _i32), ("result_is_b", _vp), ("up_a", _vp), ("up_b", _vp), ("up_rows", _i32),
+                ("dn_a", _vp), ("dn_b", _vp), ("flags", _vp), ("up_flags", _vp), ("dn_flags", _vp), ("status", _vp)]
 
 
 class Conv2dArgs(ctypes.Structure):
@@ -266,6 +272,44 @@ def jacobi5_args(a, b, iters, rows=None, cols=None) -> tuple[Jacobi5Args, ctypes
     cols = a.shape[1] if cols is None else cols
     args = Jacobi5Args(a.data_ptr(), b.data_ptr(), _lda(a), rows, cols, iters, ctypes.addressof(flag))
     return args, flag
+
+
+def jacobi5_halo_args(a, b, iters, sweep0=0, up=None, dn=None, flags=None, status=None):
+    """Args of one slab's fused-halo sweeps (CC_K_JACOBI5_HALO).  `up` / `dn` are
+    (a_ptr, b_ptr, flags_ptr, rows) of the neighbours' slabs as addresses valid
+    in this process (same-device tensors' data_ptr(), or cc_ipc_open results),
+    or None.  Returns (args, result_is_b flag)."""
+    flag = _i32(0)
+    u = up or (None, None, None, 0)
+    d = dn or (None, None, None, 0)
+    args = Jacobi5HaloArgs(a.data_ptr(), b.data_ptr(), _lda(a), a.shape[0], a.shape[1], iters, sweep0,
+                           ctypes.addressof(flag), u[0], u[1], u[3], d[0], d[1], _ptr(flags), u[2], d[2],
+                           _ptr(status))
+    return args, flag
+
+
+def peer_access(device: int, peer: int):
+    _check(lib().cc_peer_access(_i32(device), _i32(peer)))
+
+
+def ipc_handle(t) -> tuple[bytes, int]:
+    """cc_ipc_handle: (64-byte handle of the allocation holding device tensor t,
+    t's byte offset in that allocation)."""
+    buf = ctypes.create_string_buffer(64)
+    off = ctypes.c_uint64(0)
+    _check(lib().cc_ipc_handle(_vp(t.data_ptr()), buf, ctypes.byref(off)))
+    return buf.raw, off.value
+
+
+def ipc_open(handle: bytes, device: int = 0) -> int:
+    out = _vp()
+    hb = ctypes.create_string_buffer(bytes(handle), 64)
+    _check(lib().cc_ipc_open(hb, _i32(device), ctypes.byref(out)))
+    return out.value
+
+
+def ipc_close(ptr: int):
+    _check(lib().cc_ipc_close(_vp(ptr)))
 
 
 def conv2d_args(inp, out, w, rows=None, cols=None) -> tuple[Conv2dArgs, np.ndarray]:

@@ -17,7 +17,8 @@ from . import ctaclust as cc
 # fastest with TMA staging, so it is the default here.
 DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": ("col", (1, 1)),
                  "bicg": ("col", (1, 1)), "mvt": ("col", (1, 1)), "jacobi5": ("row", (1, 1)),
-                 "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1))}
+                 "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1)),
+                 "jacobi5_halo": ("row", (1, 1))}
 
 _plans: dict = {}
 
@@ -78,6 +79,17 @@ def jacobi5(a, b, iters, backend="agent", order=None, tile=None, num_clusters=0,
     """`iters` sweeps ping-ponging a <-> b; returns the buffer holding the result."""
     args, flag = cc.jacobi5_args(a, b, iters)
     _launch("jacobi5", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
+    return b if flag.value else a
+
+
+def jacobi5_halo(a, b, iters, sweep0=0, up=None, dn=None, flags=None, status=None, backend="agent", order=None,
+                 tile=None, num_clusters=0, stream=None, **kw):
+    """One slab's sweeps sweep0+1 .. sweep0+iters with the halo exchange fused
+    into the sweep kernel (CC_K_JACOBI5_HALO, S§8(f)4).  `up` / `dn`: the
+    neighbours' (a_ptr, b_ptr, flags_ptr, rows) as addresses valid here, or
+    None.  Returns the buffer holding this slab's result."""
+    args, flag = cc.jacobi5_halo_args(a, b, iters, sweep0, up, dn, flags, status)
+    _launch("jacobi5_halo", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
     return b if flag.value else a
 
 

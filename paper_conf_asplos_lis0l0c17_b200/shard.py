@@ -120,3 +120,71 @@ def gather_rows(local_owned: torch.Tensor, rows: int, world: int, rank: int) -> 
     out = [torch.empty_like(buf) for _ in range(world)]
     dist.all_gather(out, buf)
     return torch.cat([out[g][: row_range(rows, world, g)[1] - row_range(rows, world, g)[0]] for g in range(world)])
+
+
+# --------------------------------------------------------------------------
+# Fused peer-memory halo (S§8(f)4, CC_K_JACOBI5_HALO): instead of a separate
+# exchange per sweep, each rank's sweep kernel stores its boundary rows
+# straight into the neighbours' halo rows (NVLink peer mappings opened with
+# CUDA IPC) and raises per-tile-column flags the neighbour's next sweep waits
+# on.  The host only wires the neighbours once; no collective runs per sweep.
+# --------------------------------------------------------------------------
+def neighbours(world: int, rank: int) -> tuple[int | None, int | None]:
+    """(upper, lower) neighbour ranks of a slab decomposition, None at the ends."""
+    return (rank - 1 if rank > 0 else None), (rank + 1 if rank < world - 1 else None)
+
+
+class PeerHaloSlab:
+    """This rank's slab buffers a/b (owned rows plus halo rows, as slab_range)
+    and the mapped addresses of its neighbours' buffers and flags.
+
+    Collective over the process group at construction (one all_gather_object
+    of IPC handles) and at `close`; `sweeps` runs with no host exchange."""
+
+    def __init__(self, a: torch.Tensor, b: torch.Tensor, world: int, rank: int):
+        from . import ctaclust as cc
+        self.cc, self.a, self.b, self.world, self.rank = cc, a, b, world, rank
+        self.device = a.device.index or 0
+        gx = (a.shape[1] + 31) // 32
+        self.flags = torch.zeros(2 * gx, dtype=torch.int32, device=a.device)
+        self.status = torch.zeros(1, dtype=torch.int32, device=a.device)
+        mine = {"rows": a.shape[0], "pid": __import__("os").getpid(), "dev": self.device,
+                "h": [cc.ipc_handle(t) for t in (a, b, self.flags)] if world > 1 else None,
+                "p": [t.data_ptr() for t in (a, b, self.flags)]}
+        allv = [None] * world
+        if world > 1:
+            dist.all_gather_object(allv, mine)
+        else:
+            allv = [mine]
+        self._opened = []
+        self.up = self.dn = None
+        up, dn = neighbours(world, rank)
+        for which, g in (("up", up), ("dn", dn)):
+            if g is None:
+                continue
+            other = allv[g]
+            if other["pid"] == mine["pid"]:            # same process: addresses are valid as they are
+                ptrs = other["p"]
+            else:                                      # one mapping per exported allocation
+                ptrs, bases = [], {}
+                for h, off in other["h"]:
+                    if h not in bases:
+                        bases[h] = cc.ipc_open(h, self.device)
+                        self._opened.append(bases[h])
+                    ptrs.append(bases[h] + off)
+            setattr(self, which, (ptrs[0], ptrs[1], ptrs[2], other["rows"]))
+        torch.cuda.synchronize(self.device)
+        if world > 1:
+            dist.barrier()                             # every rank's flags are zero before any sweep
+
+    def sweeps(self, iters: int, sweep0: int = 0, **kw) -> torch.Tensor:
+        from . import ops
+        return ops.jacobi5_halo(self.a, self.b, iters, sweep0, self.up, self.dn, self.flags, self.status, **kw)
+
+    def close(self):
+        torch.cuda.synchronize(self.device)
+        if self.world > 1:
+            dist.barrier()                             # no neighbour still stores into our buffers
+        for base in self._opened:
+            self.cc.ipc_close(base)
+        self._opened = []

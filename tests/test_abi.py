@@ -50,6 +50,8 @@ int main(void) {
   S(cc_jacobi5_args) O(cc_jacobi5_args, result_is_b) S(cc_conv2d_args) O(cc_conv2d_args, w)
   S(cc_spmv_args) O(cc_spmv_args, part) O(cc_spmv_args, nnz)
   S(cc_hist64_args) O(cc_hist64_args, n) O(cc_hist64_args, counts)
+  S(cc_jacobi5_halo_args) O(cc_jacobi5_halo_args, sweep0) O(cc_jacobi5_halo_args, up_rows)
+  O(cc_jacobi5_halo_args, dn_a) O(cc_jacobi5_halo_args, flags) O(cc_jacobi5_halo_args, status)
   return 0;
 }
 """
@@ -64,7 +66,7 @@ def test_struct_layouts_match_binding(tmp_path):
     py = {"cc_plan_desc": cc.PlanDesc, "cc_launch_opts": cc.LaunchOpts, "cc_matvec_args": cc.MatvecArgs,
           "cc_atax_args": cc.AtaxArgs, "cc_bicg_args": cc.BicgArgs, "cc_mvt_args": cc.MvtArgs,
           "cc_jacobi5_args": cc.Jacobi5Args, "cc_conv2d_args": cc.Conv2dArgs, "cc_spmv_args": cc.SpmvArgs,
-          "cc_hist64_args": cc.Hist64Args}
+          "cc_hist64_args": cc.Hist64Args, "cc_jacobi5_halo_args": cc.Jacobi5HaloArgs}
     for key, val in got.items():
         if "." in key:
             t, f = key.split(".")
