@@ -132,6 +132,18 @@ def f2_variants(order, tile=(1, 1), l1_staging=None):
     return v
 
 
+def static_variants(kernel, order, tile=(1, 1), ks=None):
+    """CC_BACKEND_AGENT_STATIC rows: M = SMs x k clusters, CTA i runs cluster i
+    (binding by construction: no %smid, queue atomics or stealing)."""
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    nsm = cc.device_info(0)["num_sms"]
+    amax = cc.max_agents(kernel)
+    o = dict(order=order, tile=tile) if order == "tile" else dict(order=order)
+    tag = f"{order}{tile[0]}x{tile[1]}" if order == "tile" else order
+    ks = sorted(set(ks or (1, 2, amax)))
+    return [(f"static-{tag}-m{k}", dict(backend="static", num_clusters=nsm * k, **o)) for k in ks if k <= 4 * amax]
+
+
 def suite_matvec(quick):
     import torch
     from paper_conf_asplos_lis0l0c17_b200 import ops, synth
@@ -141,7 +153,10 @@ def suite_matvec(quick):
     y = torch.zeros(n, device="cuda")
     v = variants_for("row") + [("agent-col", dict(backend="agent", order="col")),
                                ("agent-row-m1s4b4", dict(backend="agent", order="row", max_agents=1, stages=4, batch=4)),
-                               ("agent-row-m2s3b2", dict(backend="agent", order="row", max_agents=2, stages=3, batch=2))]
+                               ("agent-row-m2s3b2", dict(backend="agent", order="row", max_agents=2, stages=3, batch=2))] \
+        + static_variants("matvec", "row", ks=(1, 2, 3, 4, 7)) \
+        + [("static-row-m1-s6", dict(backend="static", order="row", num_clusters=148, stages=6)),
+           ("static-row-m2-s4", dict(backend="static", order="row", num_clusters=296, stages=4))]
     r = measure(v, lambda kw: ops.matvec(A, x, y, **kw), 20 if quick else 50, 4 * n * n + 8 * n, inner=50, graph=True,
                 context={"cublas-mv": lambda: torch.mv(A, x, out=y)})
     r["config"] = "tiled fp32 matvec n=1024, 32x32 tiles (32x32 grid), L2-resident; 50 launches per CUDA graph"
@@ -164,7 +179,7 @@ def suite_atax(quick):
     }
     variants = variants_for("col") + [("agent-row", dict(backend="agent", order="row")),
                                       ("agent-col-s3", dict(backend="agent", order="col", stages=3))] \
-        + f2_variants("col", l1_staging="direct")
+        + f2_variants("col", l1_staging="direct") + static_variants("bicg", "col") + static_variants("bicg", "row", ks=(3,))
     ctx = {"atax": {"cublas-2xmv": lambda: torch.mv(A.t(), torch.mv(A, x, out=tmp), out=y)},
            "bicg": {"cublas-2xmv": lambda: (torch.mv(A, p, out=q), torch.mv(A.t(), r, out=s))},
            "mvt": {"cublas-2xmv": lambda: (x1.add_(torch.mv(A, y1)), x2.add_(torch.mv(A.t(), y2)))}}
@@ -178,7 +193,8 @@ def suite_jacobi(quick):
     N, T = 16384, (20 if quick else 100)
     a = synth.matrix(4, N, N, backend="torch", device="cuda")
     b = torch.empty_like(a)
-    v = variants_for("tile", (8, 8), stencil=True) + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1")
+    v = variants_for("tile", (8, 8), stencil=True) + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
+        + static_variants("jacobi5", "row") + static_variants("jacobi5", "tile", (8, 8), ks=(4,))
     r = measure(v, lambda kw: ops.jacobi5(a, b, T, **kw), 3, 8 * N * N * T,
                 extra=lambda ms: {"ms_per_sweep": round(ms / T, 5)}, warm=1)
     r["config"] = f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)"
@@ -200,7 +216,8 @@ def suite_conv(quick):
             ("tbcluster-2", dict(backend="tbcluster", cluster_size=2)),
             ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
             ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))] \
-            + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1")
+            + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
+            + static_variants("conv2d", "row") + static_variants("conv2d", "tile", (8, 8), ks=(4,))
         wt = torch.from_numpy(w).cuda().view(1, 1, 2 * R + 1, 2 * R + 1)
         img4 = img.view(1, 1, N, N)
         res[f"{2 * R + 1}x{2 * R + 1}"] = measure(
@@ -234,7 +251,7 @@ def suite_spmv(quick):
                 ("identity", dict(backend="identity")), ("identity-s1", dict(backend="identity", stages=1)),
                 ("redirect-row", dict(backend="redirect", order="row"))] + f2_variants("row") \
         + [(f"{b}-cv{cv}", dict(backend=b, carveout=cv, **({"order": "row"} if b == "agent" else {})))
-           for b in ("default", "agent") for cv in (0, 25, 50, 100)]
+           for b in ("default", "agent") for cv in (0, 25, 50, 100)] + static_variants("spmv", "row")
     Acsr = torch.sparse_csr_tensor(rp, col, val, (rows_n, rows_n))
     r = measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 5 if quick else 20,
                 8 * nnz + 4 * (rows_n + 1) + 8 * rows_n,
@@ -261,13 +278,86 @@ def suite_hist(quick):
              ("agent-row-direct", dict(backend="agent", order="row", staging="direct")),
              ("agent-row-tot1", dict(backend="agent", order="row", active_agents=1)),
              ("agent-col", dict(backend="agent", order="col")),
-             ("identity", dict(backend="identity")), ("redirect-row", dict(backend="redirect", order="row"))]
+             ("identity", dict(backend="identity")), ("redirect-row", dict(backend="redirect", order="row"))] \
+            + static_variants("hist64", "row")
         res[kind] = measure(v, lambda kw: ops.hist64(data, counts, **kw), 5 if quick else 20, n + 256)
         del data
     return {"config": f"64-bin histogram (HST, R24) of {n} bytes, 32 KiB per logical CTA", "inputs": res}
 
 
-SUITES = {"matvec": suite_matvec, "atax": suite_atax, "jacobi": suite_jacobi, "conv": suite_conv, "spmv": suite_spmv, "hist": suite_hist}
+def suite_slabs(quick):
+    """Config 3's slab sharding (S§8(e)) on one GPU: G = 8 virtual slabs of the
+    16384^2 Jacobi, 100 sweeps, each slab's sweep a separate launch, the slabs'
+    sweeps interleaved on one stream (captured in one CUDA graph).  Halo
+    exchange either fused into the sweep kernel (S§8(f)4, CC_K_JACOBI5_HALO:
+    tagged peer stores into the neighbours' LL buffers) or done as separate device-to-device row copies after
+    every sweep (the single-GPU stand-in for NCCL send/recv).  The unsharded
+    sweep is the reference; the difference is the cost of sharding + exchange."""
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc, ops, shard, synth
+    N, T, G = 16384, (20 if quick else 100), 8
+    u = synth.matrix(4, N, N, backend="torch", device="cuda")
+    slabs = []
+    for g in range(G):
+        lo, hi, llo, lhi = shard.slab_range(N, G, g, 1)
+        a = u[llo:lhi].clone()
+        slabs.append(dict(a=a, b=torch.empty_like(a), lo=lo, hi=hi, llo=llo, lhi=lhi,
+                          ll=torch.zeros(cc.ll_words(N), dtype=torch.int64, device="cuda")))
+    full_b = torch.empty_like(u)
+
+    def fused(kw):
+        for x in slabs:
+            x["ll"].zero_()
+        nb = lambda h: slabs[h]["ll"].data_ptr() if 0 <= h < G else None
+        for s in range(T):
+            for g, x in enumerate(slabs):
+                src, dst = (x["a"], x["b"]) if s % 2 == 0 else (x["b"], x["a"])
+                ops.jacobi5_halo(src, dst, 1, s, x["ll"], nb(g - 1), nb(g + 1), None, **kw)
+
+    def copies(kw):
+        for s in range(T):
+            outs = []
+            for x in slabs:
+                src, dst = (x["a"], x["b"]) if s % 2 == 0 else (x["b"], x["a"])
+                ops.jacobi5(src, dst, 1, **kw)
+                outs.append(dst)
+            for g in range(G - 1):                 # halo rows <- neighbours' owned boundary rows
+                outs[g][-1].copy_(outs[g + 1][1])
+                outs[g + 1][0].copy_(outs[g][-2])
+
+    def nohalo(kw):                                # the sharded sweeps with no exchange at all (timing only)
+        for s in range(T):
+            for x in slabs:
+                src, dst = (x["a"], x["b"]) if s % 2 == 0 else (x["b"], x["a"])
+                ops.jacobi5(src, dst, 1, **kw)
+
+    rows = []
+    nbytes = 8 * N * N * T
+    peak = _peak()
+    for name, fn, kw in [("unsharded-agent-row", lambda kw: ops.jacobi5(u, full_b, T, **kw), dict(backend="agent", order="row")),
+                         ("unsharded-identity", lambda kw: ops.jacobi5(u, full_b, T, **kw), dict(backend="identity")),
+                         ("unsharded-default", lambda kw: ops.jacobi5(u, full_b, T, **kw), dict(backend="default")),
+                         ("slabs8-fused-agent-row", fused, dict(backend="agent", order="row")),
+                         ("slabs8-fused-identity", fused, dict(backend="identity")),
+                         ("slabs8-fused-default", fused, dict(backend="default")),
+                         ("slabs8-copies-agent-row", copies, dict(backend="agent", order="row")),
+                         ("slabs8-copies-identity", copies, dict(backend="identity")),
+                         ("slabs8-copies-default", copies, dict(backend="default")),
+                         ("slabs8-noexchange-agent-row", nohalo, dict(backend="agent", order="row")),
+                         ("slabs8-noexchange-identity", nohalo, dict(backend="identity"))]:
+        ms = graph_ms(lambda: fn(kw), 3, 1)
+        gbs = nbytes / (ms * 1e-3) / 1e9
+        rows.append({"variant": name, "ms": round(ms, 4), "ms_per_sweep": round(ms / T, 5), "GBps": round(gbs, 1),
+                     "frac_hbm": round(gbs / peak, 4)})
+    best = min(r["ms"] for r in rows if r["variant"].startswith("unsharded"))
+    for r in rows:
+        r["speedup_vs_best_default"] = round(best / r["ms"], 4)       # here: vs the best unsharded run
+    return {"config": f"Jacobi {N}^2 x {T} sweeps as {G} virtual slabs on one GPU (fused peer halo vs "
+                      f"separate row copies; vs unsharded)", "bytes": nbytes, "rows": rows}
+
+
+SUITES = {"matvec": suite_matvec, "atax": suite_atax, "jacobi": suite_jacobi, "conv": suite_conv, "spmv": suite_spmv, "hist": suite_hist,
+          "slabs": suite_slabs}
 
 
 def run(path, only=None, quick=False):

@@ -117,8 +117,15 @@ typedef enum {
                                       of clustering (conv2d only in this build)        */
     CC_BACKEND_AGENT_IDENTITY = 3, /* persistence-only control: same agents, one global
                                       queue in row-major order, no locality grouping   */
-    CC_BACKEND_REDIRECT = 4        /* redirection-based clustering "RD" (Listing 4,
+    CC_BACKEND_REDIRECT = 4,       /* redirection-based clustering "RD" (Listing 4,
                                       Eq. 8 + Eq. 7; relies on RR dispatch)    */
+    CC_BACKEND_AGENT_STATIC = 5    /* static binding: grid = the plan's M CTAs, CTA i runs
+                                      cluster i's tasks in Eq. 7 order through the same
+                                      staging ring.  A cluster's tasks share an SM by
+                                      construction (one CTA), with no %smid probe, queue
+                                      atomics, stealing or workspace; active_agents and
+                                      steal are ignored.  Pick M (num_clusters) as a
+                                      multiple of the SM count x resident CTAs.      */
 } cc_backend;
 
 typedef enum { CC_STAGING_DEFAULT = 0, CC_STAGING_TMA = 1, CC_STAGING_L1 = 2, CC_STAGING_DIRECT = 3 } cc_staging;
@@ -219,42 +226,37 @@ typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t ite
  * (S§8(e), config 3) with the per-sweep halo exchange fused into the sweep
  * kernel over peer memory, replacing cc_halo_exchange's NCCL send/recv.
  * The slab a/b (DEVICE, rows x cols, ld) holds this rank's owned rows plus one
- * halo row above (row 0, when up_a != NULL) and below (row rows-1, when
- * dn_a != NULL); the arithmetic is CC_K_JACOBI5's (halo and global boundary
- * rows are fixed during a sweep).  In sweep s the tile computing the first
- * (last) owned row also stores it into the upper (lower) neighbour's halo row
- * of its destination buffer and raises the neighbour's flag for that tile
- * column to s; a tile reading a halo row first waits until the neighbour's
- * flags for columns bx-1..bx+1 reach s-1 (this covers RAW on the halo and
- * WAR on the neighbour's copy).  Halo rows of this rank's b are written only
- * by the neighbours.
+ * halo row above (row 0, when up_ll != NULL) and below (row rows-1, when
+ * dn_ll != NULL); the arithmetic is CC_K_JACOBI5's (halo and global boundary
+ * rows are fixed during a sweep).  Halo values cross as 64-bit words {fp32
+ * bits, absolute sweep number} ("LL" form, no fences): in sweep s the threads
+ * computing the first (last) owned row also store it, tagged s, into the
+ * upper (lower) neighbour's LL buffer of parity s & 1; in sweep s > 1 the
+ * tiles needing a halo row read this rank's LL buffer of parity (s-1) & 1 (a
+ * bulk copy riding with the tile's TMA) and re-poll any word not yet carrying
+ * tag s-1.  Sweep 1 uses the halo rows already in a.  The body visits the
+ * boundary tile rows first (a fixed bijection on tile rows).
  *   a, b            this call's first source / destination (ping-pong as in
  *                   CC_K_JACOBI5; *result_is_b as there)
- *   iters, sweep0   runs absolute sweeps sweep0+1 .. sweep0+iters; flags
- *                   count absolute sweeps since they were zeroed
- *   up_a, up_b      the upper neighbour's a and b in the same roles, mapped
- *                   into this process (same device, cc_peer_access, or
- *                   cc_ipc_open); NULL = no upper neighbour.  up_rows: its
- *                   slab rows (its bottom halo is row up_rows-1)
- *   dn_a, dn_b      the lower neighbour's (its top halo is its row 0)
- *   flags           DEVICE uint32[2*gx] (gx = ceil(cols/32)): [0,gx) deposits
- *                   from up, [gx,2gx) from down; zeroed by the caller (on every
- *                   rank, before any rank's sweep 1) with sweep0 = 0
- *   up_flags, dn_flags  the neighbours' `flags`, mapped like up_a/dn_a
- *   status          DEVICE int32, optional: set to 1 if a wait exceeded 4 s (a
- *                   neighbour not running); results are then invalid
- * Every rank uses the same cols and ld.  Staging must be TMA (default): halo
- * rows are read after a system-scope acquire, never through L1.  Launches of
+ *   iters, sweep0   runs absolute sweeps sweep0+1 .. sweep0+iters
+ *   ll              DEVICE uint64[4 * ldl], ldl = cols rounded up to 32, 16-byte
+ *                   aligned: [parity 0/1][side 0 = from up / 1 = from down][ldl];
+ *                   zeroed by the caller (on every rank, before any rank's
+ *                   sweep 1) when sweep0 = 0
+ *   up_ll, dn_ll    the neighbours' `ll`, mapped into this process (same
+ *                   device, cc_peer_access, or cc_ipc_open); NULL = no such
+ *                   neighbour (that slab edge is the global boundary)
+ *   status          DEVICE int32, optional: set to 1 if a poll exceeded 4 s in
+ *                   total (a neighbour not running); results are then invalid
+ * Every rank uses the same cols.  Halo rows of b are not written.  Launches of
  * neighbouring ranks may run concurrently (one GPU each) or be interleaved
  * sweep by sweep on one stream (virtual slabs on one GPU); a rank's sweep s
  * must not be queued behind a neighbour's sweep s+1 on one stream.
- * Errors: INVALID_ARG (sizes, a neighbour pointer without its flags, owned
- * rows < 1), UNSUPPORTED (staging other than TMA, TBCLUSTER backend). */
+ * Errors: INVALID_ARG (sizes, a neighbour without `ll`, misaligned ll, owned
+ * rows < 1), UNSUPPORTED (TBCLUSTER backend). */
 typedef struct {
     float* a; float* b; int64_t ld; int32_t rows, cols; int32_t iters; int32_t sweep0; int32_t* result_is_b;
-    float* up_a; float* up_b; int32_t up_rows;
-    float* dn_a; float* dn_b;
-    uint32_t* flags; uint32_t* up_flags; uint32_t* dn_flags;
+    uint64_t* ll; uint64_t* up_ll; uint64_t* dn_ll;
     int32_t* status;
 } cc_jacobi5_halo_args;
 

@@ -34,7 +34,7 @@
 
 namespace cc {
 
-enum : int32_t { MODE_AGENT = 0, MODE_IDENTITY = 1 };
+enum : int32_t { MODE_AGENT = 0, MODE_IDENTITY = 1, MODE_STATIC = 2 };
 constexpr int MAX_STAGES = 8;
 constexpr int PRODUCER_THREADS = 32;
 
@@ -45,7 +45,7 @@ struct Sched {
     const int32_t* rank_of_smid;  // %smid -> dense SM rank or -1 (device)
     int32_t smid_span;
     int32_t* ws;                  // workspace: agent_ctr[M+1] | head[M] | gq | done | claimed
-    int32_t mode;                 // MODE_AGENT / MODE_IDENTITY
+    int32_t mode;                 // MODE_AGENT / MODE_IDENTITY / MODE_STATIC
     int32_t active_agents;
     int32_t throttle;             // active_agents < agents launched per SM
     int32_t steal;
@@ -98,6 +98,9 @@ __device__ __forceinline__ void fence_mbar_init() {
 }
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.expect_tx.relaxed.cta.shared::cta.b64 [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
 __device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
     asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" :: "r"(smem_u32(bar)), "r"(bytes) : "memory");
@@ -276,7 +279,13 @@ __device__ __forceinline__ int32_t steal_scan(const Sched& s, int32_t home, int 
     return -1;
 }
 
+template <bool kStatic>
 __device__ __forceinline__ int32_t producer_next(const Sched& s, Prod& P, int lane) {
+    if constexpr (kStatic) {                               // CTA i owns cluster i: a local cursor
+        int32_t v = -1;
+        if (lane == 0 && P.q >= 0 && P.bw < cluster_size(s.g, P.q)) v = cluster_start(s.g, P.q) + P.bw++;
+        return __shfl_sync(0xffffffffu, v, 0);
+    }
     int32_t v = -1, scan = 0;
     if (lane == 0) v = lane0_next(s, P, &scan);
     scan = __shfl_sync(0xffffffffu, scan, 0);
@@ -310,7 +319,7 @@ __device__ __forceinline__ uint8_t* ring_base(uint8_t* dyn) {
     return dyn + (((a + 127u) & ~127u) - a);
 }
 
-template <class Body>
+template <class Body, bool kStatic = false>
 __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
     extern __shared__ uint8_t dyn_smem[];
     __shared__ RingShared R;
@@ -328,7 +337,13 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         // ---- binding: dense SM rank from %smid, agent id by arrival
         Prod P{};
         int32_t active = 0;
-        if (lane == 0) {
+        if constexpr (kStatic) {                               // binding by construction
+            if (lane == 0) {
+                P.q = (int32_t)blockIdx.x < s.g.M ? (int32_t)blockIdx.x : -1;
+                P.bw = 0;
+                s_active = active = 1;
+            }
+        } else if (lane == 0) {
             uint32_t sm = smid();
             int32_t rank = (int32_t)sm < s.smid_span ? s.rank_of_smid[sm] : -1;
             int32_t slot = (rank < 0 || rank >= s.g.M) ? s.g.M : rank;
@@ -349,7 +364,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         int32_t t = 0;
         for (;; ++t) {
             if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
-            const int32_t v = producer_next(s, P, lane);
+            const int32_t v = producer_next<kStatic>(s, P, lane);
             if (v < 0) {
                 if (lane == 0) R.slot[st] = make_int4(-1, 0, 0, 0);
                 break;
@@ -374,7 +389,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         // other agent's producer has consumed the results of all its atomics
         // (including any speculative claim) before arriving here.
         int32_t last = 0;
-        if (lane == 0) {
+        if (lane == 0 && !kStatic) {                           // the static backend has no workspace
             const int32_t total = (int32_t)(gridDim.x * gridDim.y * gridDim.z);
             last = atom_add_relaxed(ws_done(s), 1) == total - 1;
         }
@@ -433,6 +448,15 @@ k_agent(const __grid_constant__ Sched s, const __grid_constant__ typename Body::
     Body body(p);
     body.l2h = s.l2_hint;        // L2 hints ride with clustering (CLU+BPS); one-shot kernels compile them out
     agent_loop(s, body);
+}
+
+// static binding (CC_BACKEND_AGENT_STATIC): grid = M, CTA i runs cluster i
+template <class Body>
+__global__ void __launch_bounds__(Body::kGroups * Body::kConsumers + PRODUCER_THREADS, Body::kMinAgents)
+k_static(const __grid_constant__ Sched s, const __grid_constant__ typename Body::Params p) {
+    Body body(p);
+    body.l2h = s.l2_hint;
+    agent_loop<Body, true>(s, body);
 }
 
 template <class Body>

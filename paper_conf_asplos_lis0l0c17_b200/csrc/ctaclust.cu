@@ -347,6 +347,7 @@ static cc_status prepare_body(int device) {
         const int mx = (int)std::min(dyn_smem<Body>(MAX_STAGES), (size_t)(optin - (int)fa.sharedSizeBytes));
         const int one = (int)dyn_smem<Body>(1);
         CC_CUDA(cudaFuncSetAttribute(k_agent<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
+        CC_CUDA(cudaFuncSetAttribute(k_static<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
         CC_CUDA(cudaFuncSetAttribute(k_default<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, one));
         CC_CUDA(cudaFuncSetAttribute(k_redirect<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, one));
         done[device] = true;
@@ -474,6 +475,18 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         s.stages = S;
         const int grid = c.p->facts->num_sms * maxa;
         k_agent<Body><<<grid, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
+        break;
+    }
+    case CC_BACKEND_AGENT_STATIC: {
+        int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
+        if (S < Body::kGroups) S = Body::kGroups;
+        CC_TRY(set_carveout(k_static<Body>, o.carveout));
+        s.active_agents = 1;
+        s.throttle = 0;
+        s.steal = 0;
+        s.mode = MODE_STATIC;
+        s.stages = S;
+        k_static<Body><<<g.M, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
         break;
     }
     default:
@@ -667,35 +680,25 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         CC_TRY(check_mat(x->a, x->ld, x->rows, x->cols));
         CC_TRY(check_mat(x->b, x->ld, x->rows, x->cols));
         if (x->iters < 0 || x->sweep0 < 0) return fail(CC_ERR_INVALID_ARG, "iters / sweep0 < 0");
-        const bool up = x->up_a || x->up_b, dn = x->dn_a || x->dn_b;
-        if (up && (!x->up_a || !x->up_b || !x->up_flags || x->up_rows < 2))
-            return fail(CC_ERR_INVALID_ARG, "upper neighbour needs up_a, up_b, up_flags and up_rows >= 2");
-        if (dn && (!x->dn_a || !x->dn_b || !x->dn_flags))
-            return fail(CC_ERR_INVALID_ARG, "lower neighbour needs dn_a, dn_b and dn_flags");
-        if ((up || dn) && !x->flags) return fail(CC_ERR_INVALID_ARG, "null flags");
+        const bool up = x->up_ll != nullptr, dn = x->dn_ll != nullptr;
+        if ((up || dn) && !x->ll) return fail(CC_ERR_INVALID_ARG, "neighbours given but no own ll buffer");
+        if (!al16(x->ll) || !al16(x->up_ll) || !al16(x->dn_ll)) return fail(CC_ERR_INVALID_ARG, "ll buffers must be 16-byte aligned");
         if (x->rows - (up ? 1 : 0) - (dn ? 1 : 0) < 1) return fail(CC_ERR_INVALID_ARG, "slab has no owned row");
-        const int32_t st_mode = o->staging == CC_STAGING_DEFAULT ? CC_STAGING_TMA : o->staging;
-        if (st_mode != CC_STAGING_TMA) return fail(CC_ERR_UNSUPPORTED, "fused halo needs TMA staging");
         float* src = x->a;
         float* dst = x->b;
-        float* usrc = x->up_a; float* udst = x->up_b;
-        float* dsrc = x->dn_a; float* ddst = x->dn_b;
         for (int it = 0; it < x->iters && s == CC_OK; ++it) {
             JacobiParams jp;
             memset(&jp, 0, sizeof jp);
             jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
             if (up || dn) {
-                jp.h.up_dst = up ? udst : nullptr;
-                jp.h.dn_dst = dn ? ddst : nullptr;
-                jp.h.up_row = x->up_rows - 1;
-                jp.h.gx = p->g.gx;
-                jp.h.flags = x->flags; jp.h.up_flags = x->up_flags; jp.h.dn_flags = x->dn_flags;
-                jp.h.status = x->status;
+                jp.h.ll = x->ll; jp.h.up_ll = x->up_ll; jp.h.dn_ll = x->dn_ll;
+                jp.h.ldl = (x->cols + 31) & ~31;
                 jp.h.sweep = (uint32_t)(x->sweep0 + it + 1);
+                jp.h.status = x->status;
             }
             if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
             s = (up || dn) ? launch_body<Jacobi5HaloBody>(c, jp) : launch_body<Jacobi5Body>(c, jp);
-            std::swap(src, dst); std::swap(usrc, udst); std::swap(dsrc, ddst);
+            std::swap(src, dst);
         }
         if (x->result_is_b) *x->result_is_b = (x->iters & 1) ? 1 : 0;
         break;

@@ -90,27 +90,35 @@ __device__ __forceinline__ void store4_out(float* dst, float4 o, int gx, int col
 // bit-reproducible against oracle_jacobi5_f32 in every staging mode.
 // ---------------------------------------------------------------------------
 // Fused peer-memory halo exchange of the slab-sharded sweep (S§8(f)4,
-// CC_K_JACOBI5_HALO): the tile that computes a slab's first (last) owned row
-// also stores it into the upper (lower) neighbour's halo row -- through
-// NVLink peer mappings on a multi-GPU box, or plain device pointers for
-// virtual slabs on one GPU -- and then raises that neighbour's per-tile-column
-// flag to the absolute sweep number.  A tile that reads a halo row (and so
-// also writes the neighbour's halo of the next buffer) first waits, in the
-// producer before its TMA, until the neighbour's tiles bx-1..bx+1 have
-// deposited sweep s-1: that one condition covers both the data it reads (RAW)
-// and the neighbour having finished reading the halo row it is about to
-// overwrite (WAR: the neighbour's depositing tile is its halo-reading tile).
-// All pointers null = the unsharded sweep.
+// CC_K_JACOBI5_HALO), in the flag-in-data ("low latency", LL) form: every halo
+// value crosses as one 64-bit word {fp32 bits, absolute sweep number}.  The
+// thread that computes a slab's first (last) owned row of sweep s also stores
+// it, tagged s, into the upper (lower) neighbour's LL buffer of parity s & 1
+// -- NVLink peer stores on a multi-GPU box, plain stores for virtual slabs on
+// one GPU.  The thread that needs a halo row in sweep s (> 1) polls its own LL
+// buffer of parity (s-1) & 1 until every word it needs carries tag s-1.  An
+// 8-byte word is written and read in one piece, so the tag vouches for its
+// value: no fence on either side (a system-scope fence per tile drains the
+// SM's whole store queue and cost more than the exchange saved).  WAR: the
+// writer of sweep s+2 first read tag s+1 at the same columns, which the
+// neighbour's thread deposited only after (by data dependence) reading the
+// sweep-s words being overwritten.  Sweep 1 reads the caller's initial halo
+// rows from the slab.  All LL pointers null = the unsharded sweep.
+// Only the tile rows next to a halo differ from the plain sweep.  Their
+// producer adds one 256-byte bulk copy of the tile's 32 LL words per halo row
+// to the stage (same mbarrier as the tile's TMA), so the LL read rides with
+// the tile copy instead of stalling anyone; the consumers check the tags in
+// shared memory and only re-poll global memory (strong loads) for words
+// whose tag is stale.  A word is 8-byte aligned inside a 32-byte sector, so
+// no copy can split a value from its tag.  (A consumer-side poll cost ~5 us
+// per launch, a producer-side one ~4 us: measured.)
 struct JacobiHalo {
-    float* up_dst;            // upper neighbour's destination buffer of this sweep (null: none)
-    float* dn_dst;            // lower neighbour's destination buffer (its top halo is row 0)
-    int32_t up_row;           // the upper neighbour's bottom halo row (its rows - 1)
-    int32_t gx;               // tile columns (same on every rank: equal cols)
-    uint32_t* flags;          // mine [2 gx]: [0, gx) deposits from up, [gx, 2 gx) from down
-    uint32_t* up_flags;       // upper neighbour's flags (I write its "from down" half)
-    uint32_t* dn_flags;       // lower neighbour's flags (I write its "from up" half)
-    int32_t* status;          // optional: 1 = a wait timed out (results invalid)
+    uint64_t* ll;             // mine: [2 parity][2 side][ldl]; side 0 = from up, 1 = from down
+    uint64_t* up_ll;          // upper neighbour's LL (I deposit my first owned row into its side 1); null: none
+    uint64_t* dn_ll;          // lower neighbour's LL (my last owned row into its side 0); null: none
+    int32_t ldl;              // LL row length: cols rounded up to 32 (whole tiles)
     uint32_t sweep;           // absolute sweep number of this launch (1-based)
+    int32_t* status;          // optional: 1 = a poll timed out (results invalid)
 };
 struct JacobiParams { CUtensorMap tmap; const float* a; float* b; int64_t ld; int32_t rows, cols; JacobiHalo h; };
 
@@ -119,39 +127,72 @@ __device__ __forceinline__ uint64_t globaltimer() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
-__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t* p) {
-    uint32_t v;
-    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
+// Diagnostic builds only (make CC_DEFS=...; never the shipped library):
+// CC_LL_GPU_SCOPE uses .gpu instead of .sys for the LL words (valid only for
+// virtual slabs on one GPU); CC_LL_NOSTORE drops the deposits (wrong
+// results; to time their share).
+#ifdef CC_LL_GPU_SCOPE
+#define CC_LL_SCOPE "gpu"
+#else
+#define CC_LL_SCOPE "sys"
+#endif
+__device__ __forceinline__ uint64_t ll_word(float v, uint32_t tag) {
+    return ((uint64_t)tag << 32) | (uint64_t)__float_as_uint(v);
 }
-// wait until flags[bx-1 .. bx+1] >= need (acquire, system scope), bounded: a
-// call that waits longer than 4 s in total flags *status and gives up (as does
-// every later wait once *status is set), so a broken peer cannot hang the GPU;
-// then order the generic-proxy peer writes before this thread's TMA
-// (async-proxy) reads of the halo row.
-__device__ __forceinline__ void halo_wait(const uint32_t* flags, int32_t bx, int32_t gx, uint32_t need,
-                                          int32_t* status) {
-    const int32_t k0 = bx > 0 ? bx - 1 : 0, k1 = bx + 1 < gx ? bx + 1 : gx - 1;
-    uint64_t t0 = 0;
-    for (int32_t k = k0; k <= k1; ++k) {
-        while (ld_acquire_sys(flags + k) < need) {
-            if (t0 == 0) {
-                if (status && *(volatile int32_t*)status) break;      // an earlier wait already gave up
-                t0 = globaltimer();
-            }
-            __nanosleep(256);
-            if (globaltimer() - t0 > 4000000000ull) {
-                if (status) atomicExch(status, 1);
-                break;
-            }
-        }
+// deposit 4 consecutive values (16-byte aligned group of 4 words; the first
+// `valid` are inside the image) tagged `tag`
+__device__ __forceinline__ void ll_store4(uint64_t* dst, float4 o, uint32_t tag, int valid) {
+    if (valid >= 4) {
+        asm volatile("st.relaxed." CC_LL_SCOPE ".global.v2.u64 [%0], {%1, %2};\n\t"
+                     "st.relaxed." CC_LL_SCOPE ".global.v2.u64 [%0+16], {%3, %4};"
+                     :: "l"(dst), "l"(ll_word(o.x, tag)), "l"(ll_word(o.y, tag)), "l"(ll_word(o.z, tag)),
+                        "l"(ll_word(o.w, tag)) : "memory");
+        return;
     }
-    asm volatile("fence.proxy.async.global;" ::: "memory");
+    const float v[3] = {o.x, o.y, o.z};
+    for (int e = 0; e < valid; ++e)
+        asm volatile("st.relaxed." CC_LL_SCOPE ".global.u64 [%0], %1;" :: "l"(dst + e), "l"(ll_word(v[e], tag)) : "memory");
 }
-// make this CTA's peer stores (ordered before us by the group barrier) visible
-// system-wide, then publish the sweep number in the neighbour's flag
-__device__ __forceinline__ void halo_signal(uint32_t* flag, uint32_t sweep) {
-    asm volatile("fence.acq_rel.sys;\n\tst.relaxed.sys.global.u32 [%0], %1;" :: "l"(flag), "r"(sweep) : "memory");
+// poll 4 words until the first `valid` carry `tag`; bounded: after 4 s in
+// total (or once *status is set by an earlier timeout) give up and set *status
+__device__ __forceinline__ float4 ll_load4(const uint64_t* src, uint32_t tag, int valid, int32_t* status) {
+    uint64_t w[4];
+    uint64_t t0 = 0;
+    for (;;) {
+        asm volatile("ld.relaxed." CC_LL_SCOPE ".global.v2.u64 {%0, %1}, [%4];\n\t"
+                     "ld.relaxed." CC_LL_SCOPE ".global.v2.u64 {%2, %3}, [%4+16];"
+                     : "=l"(w[0]), "=l"(w[1]), "=l"(w[2]), "=l"(w[3]) : "l"(src) : "memory");
+        bool ok = true;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) ok &= e >= valid || (uint32_t)(w[e] >> 32) == tag;
+        if (ok) break;
+        if (t0 == 0) {
+            if (status && *(volatile int32_t*)status) break;      // an earlier poll already gave up
+            t0 = globaltimer();
+        } else if (globaltimer() - t0 > 4000000000ull) {
+            if (status) atomicExch(status, 1);
+            break;
+        }
+        __nanosleep(128);
+    }
+    return make_float4(__uint_as_float((uint32_t)w[0]), __uint_as_float((uint32_t)w[1]),
+                       __uint_as_float((uint32_t)w[2]), __uint_as_float((uint32_t)w[3]));
+}
+// the 4 words from the stage copy if all carry `tag`, else poll global memory
+__device__ __forceinline__ float4 ll_take4(const uint64_t* staged, const uint64_t* src, uint32_t tag, int valid,
+                                           int32_t* status) {
+    if (staged) {
+        const ulonglong2 a = *reinterpret_cast<const ulonglong2*>(staged);
+        const ulonglong2 b = *reinterpret_cast<const ulonglong2*>(staged + 2);
+        const uint64_t w[4] = {a.x, a.y, b.x, b.y};
+        bool ok = true;
+#pragma unroll
+        for (int e = 0; e < 4; ++e) ok &= e >= valid || (uint32_t)(w[e] >> 32) == tag;
+        if (ok)
+            return make_float4(__uint_as_float((uint32_t)w[0]), __uint_as_float((uint32_t)w[1]),
+                               __uint_as_float((uint32_t)w[2]), __uint_as_float((uint32_t)w[3]));
+    }
+    return ll_load4(src, tag, valid, status);
 }
 
 __device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, float lw, float re,
@@ -176,7 +217,8 @@ template <bool HALO>
 struct Jacobi5BodyT {
     static constexpr int RB = 2;                  // output rows per consumer thread
     static constexpr int kConsumers = 256 / RB;
-    static constexpr int kStageBytes = HaloTile<1>::kBytes;
+    static constexpr int kTileBytes = HaloTile<1>::kBytes;
+    static constexpr int kStageBytes = kTileBytes + (HALO ? 2 * 32 * 8 : 0);   // + the two LL halo rows (words)
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
     static constexpr int kMinAgents = 4;
@@ -186,14 +228,37 @@ struct Jacobi5BodyT {
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
     __device__ __forceinline__ explicit Jacobi5BodyT(const JacobiParams& prm) : p(prm) {}
 
+    // fused halo: which halo rows this tile row needs / which owned rows it deposits
+    __device__ __forceinline__ bool need_top(int32_t by) const { return HALO && p.h.up_ll && by == 0; }
+    __device__ __forceinline__ bool need_bot(int32_t by) const { return HALO && p.h.dn_ll && by == (p.rows - 2) / 32; }
+    // Boundary tile rows first: the body visits tile row L = (rows-2)/32 (the
+    // lower deposit) right after row 0, then the rest in order -- a fixed
+    // bijection on tile rows applied to whatever order the plan gives, so
+    // coverage is untouched.  The deposits then land at the start of every
+    // sweep, and the next sweep's polls (also at its start) find them: no LL
+    // round trip sits in a launch's tail (the classic boundary-first overlap).
+    __device__ __forceinline__ int32_t phys_row(int32_t by) const {
+        if (!HALO || !p.h.dn_ll) return by;
+        const int32_t L = (p.rows - 2) / 32, first = p.h.up_ll ? 1 : 0;
+        if (by < first || by > L) return by;
+        return by == first ? L : by - 1;
+    }
+
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        if (HALO && p.h.flags) {                  // fused halo: wait for the neighbours' deposits of sweep s-1
+        by = phys_row(by);
+        if (HALO && p.h.sweep > 1 && s.staging == STAGE_TMA && (need_top(by) || need_bot(by))) {
+            // the tile's TMA plus one bulk copy of its 32 LL words per halo row
+            const bool top = need_top(by), bot = need_bot(by);
+            const int32_t par = (int32_t)((p.h.sweep - 1) & 1u) * 2 * p.h.ldl;
+            const uint32_t ll_bytes = (top ? 256u : 0u) + (bot ? 256u : 0u);
+            stage_commit(full, lane, (uint32_t)(HaloTile<1>::kRows * ST_COLS * 4) + ll_bytes);
             if (lane == 0) {
-                if (p.h.up_dst && by == 0) halo_wait(p.h.flags, bx, p.h.gx, p.h.sweep - 1, p.h.status);
-                if (p.h.dn_dst && by * 32 + 32 >= p.rows - 1)
-                    halo_wait(p.h.flags + p.h.gx, bx, p.h.gx, p.h.sweep - 1, p.h.status);
+                tma_load_2d(stage, &p.tmap, bx * 32 - 4, by * 32 - 1, full);
+                uint8_t* extra = stage + kTileBytes;
+                if (top) bulk_g2s(extra, p.h.ll + par + bx * 32, 256u, full);
+                if (bot) bulk_g2s(extra + 256, p.h.ll + par + p.h.ldl + bx * 32, 256u, full);
             }
-            __syncwarp();
+            return;
         }
         HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h);
     }
@@ -201,6 +266,7 @@ struct Jacobi5BodyT {
     // thread (rows r0 .. r0+RB-1, columns 4*c4 .. 4*c4+3): the RB+2 input rows
     // it touches are read once each
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        by = phys_row(by);
         const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
         const int gx = bx * 32 + 4 * c4;
         const int gy0 = by * 32 + r0;
@@ -235,37 +301,47 @@ struct Jacobi5BodyT {
                 re[j] = t[(j + 1) * ST_COLS + 4];
             }
         }
-        if (!HALO || !p.h.flags) {
-            if (!in_col) return;
+        if (!in_col) return;
+        const bool top = need_top(by), bot = need_bot(by);
+        if (HALO && (top || bot)) {
+            // halo rows of sweep s-1: the LL values (sweep 1: the caller's rows, as staged)
+            const uint32_t sw = p.h.sweep;
+            const int valid = p.cols - gx < 4 ? p.cols - gx : 4;
+            const int32_t par = (int32_t)((sw - 1) & 1u) * 2 * p.h.ldl;
+            const uint64_t* extra = reinterpret_cast<const uint64_t*>(stage + kTileBytes);
+            if (sw > 1) {
+#pragma unroll
+                for (int k = 0; k < RB + 2; ++k) {
+                    const int gy = gy0 - 1 + k;
+                    if (top && gy == 0)
+                        row[k] = ll_take4(s.staging == STAGE_TMA ? extra + 4 * c4 : nullptr, p.h.ll + par + gx, sw - 1,
+                                          valid, p.h.status);
+                    if (bot && gy == p.rows - 1)
+                        row[k] = ll_take4(s.staging == STAGE_TMA ? extra + 32 + 4 * c4 : nullptr,
+                                          p.h.ll + par + p.h.ldl + gx, sw - 1, valid, p.h.status);
+                }
+            }
+            const int32_t opar = (int32_t)(sw & 1u) * 2 * p.h.ldl;        // parity this sweep deposits into
 #pragma unroll
             for (int j = 0; j < RB; ++j) {
                 const int gy = gy0 + j;
                 if (gy >= p.rows) break;
-                store4_out(p.b + (int64_t)gy * p.ld + gx,
-                           jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx,
-                           p.cols, l2h);
+                const float4 o = jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols);
+                store4_masked(p.b + (int64_t)gy * p.ld + gx, o, gx, p.cols);
+#ifndef CC_LL_NOSTORE
+                if (top && gy == 1) ll_store4(p.h.up_ll + opar + p.h.ldl + gx, o, sw, valid);
+                if (bot && gy == p.rows - 2) ll_store4(p.h.dn_ll + opar + gx, o, sw, valid);
+#endif
             }
             return;
         }
-        // fused halo: halo rows are the neighbours' to write; the first / last
-        // owned rows also go to the neighbours' halo rows
-        const bool up = p.h.up_dst != nullptr, dn = p.h.dn_dst != nullptr;
 #pragma unroll
         for (int j = 0; j < RB; ++j) {
             const int gy = gy0 + j;
-            if (!in_col || gy >= p.rows || (up && gy == 0) || (dn && gy == p.rows - 1)) continue;
-            const float4 o = jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols);
-            store4_masked(p.b + (int64_t)gy * p.ld + gx, o, gx, p.cols);
-            if (up && gy == 1) store4_masked(p.h.up_dst + (int64_t)p.h.up_row * p.ld + gx, o, gx, p.cols);
-            if (dn && gy == p.rows - 2) store4_masked(p.h.dn_dst + gx, o, gx, p.cols);
-        }
-        const bool to_up = up && by == 0, to_dn = dn && by == (p.rows - 2) / 32;   // uniform per tile
-        if (to_up || to_dn) {
-            consumer_sync<kConsumers>();             // every peer store of the tile precedes the signal
-            if (ctid == 0) {
-                if (to_up) halo_signal(p.h.up_flags + p.h.gx + bx, p.h.sweep);
-                if (to_dn) halo_signal(p.h.dn_flags + bx, p.h.sweep);
-            }
+            if (gy >= p.rows) break;
+            store4_out(p.b + (int64_t)gy * p.ld + gx,
+                       jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx,
+                       p.cols, l2h);
         }
     }
     __device__ __forceinline__ void finish(int) {}

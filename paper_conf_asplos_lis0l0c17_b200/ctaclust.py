@@ -14,13 +14,15 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libctaclust.so")
+# CTACLUST_LIB: an alternative build of the same library (diagnostic builds
+# with CC_DEFS, scripts/); still the CUDA library, never a fallback
+LIB_PATH = os.environ.get("CTACLUST_LIB") or os.path.join(_HERE, "libctaclust.so")
 
 # ---- enums (ctaclust.h) ----------------------------------------------------
 ORDER_ROW, ORDER_COL, ORDER_TILE, ORDER_USER = 0, 1, 2, 3
 ORDERS = {"row": ORDER_ROW, "col": ORDER_COL, "tile": ORDER_TILE, "user": ORDER_USER}
-BACKEND_DEFAULT, BACKEND_AGENT, BACKEND_TBCLUSTER, BACKEND_AGENT_IDENTITY, BACKEND_REDIRECT = 0, 1, 2, 3, 4
-BACKENDS = {"default": 0, "agent": 1, "tbcluster": 2, "identity": 3, "redirect": 4}
+BACKEND_DEFAULT, BACKEND_AGENT, BACKEND_TBCLUSTER, BACKEND_AGENT_IDENTITY, BACKEND_REDIRECT, BACKEND_AGENT_STATIC = 0, 1, 2, 3, 4, 5
+BACKENDS = {"default": 0, "agent": 1, "tbcluster": 2, "identity": 3, "redirect": 4, "static": 5}
 K_CENSUS, K_MATVEC, K_ATAX, K_BICG, K_MVT, K_JACOBI5, K_CONV2D, K_SPMV = range(8)
 STAGINGS = {"default": 0, "tma": 1, "l1": 2, "direct": 3}
 KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7,
@@ -85,8 +87,7 @@ class Jacobi5Args(ctypes.Structure):
 
 class Jacobi5HaloArgs(ctypes.Structure):
     _fields_ = [("a", _vp), ("b", _vp), ("ld", _i64), ("rows", _i32), ("cols", _i32), ("iters", _i32),
-                ("sweep0", _i32), ("result_is_b", _vp), ("up_a", _vp), ("up_b", _vp), ("up_rows", _i32),
-                ("dn_a", _vp), ("dn_b", _vp), ("flags", _vp), ("up_flags", _vp), ("dn_flags", _vp), ("status", _vp)]
+                ("sweep0", _i32), ("result_is_b", _vp), ("ll", _vp), ("up_ll", _vp), ("dn_ll", _vp), ("status", _vp)]
 
 
 class Conv2dArgs(ctypes.Structure):
@@ -274,18 +275,21 @@ def jacobi5_args(a, b, iters, rows=None, cols=None) -> tuple[Jacobi5Args, ctypes
     return args, flag
 
 
-def jacobi5_halo_args(a, b, iters, sweep0=0, up=None, dn=None, flags=None, status=None):
-    """Args of one slab's fused-halo sweeps (CC_K_JACOBI5_HALO).  `up` / `dn` are
-    (a_ptr, b_ptr, flags_ptr, rows) of the neighbours' slabs as addresses valid
-    in this process (same-device tensors' data_ptr(), or cc_ipc_open results),
-    or None.  Returns (args, result_is_b flag)."""
+def jacobi5_halo_args(a, b, iters, sweep0=0, ll=None, up_ll=None, dn_ll=None, status=None):
+    """Args of one slab's fused-halo sweeps (CC_K_JACOBI5_HALO).  `ll`: this
+    slab's LL buffer (int64 tensor of 4 * ldl words); `up_ll` / `dn_ll`: the
+    neighbours' LL buffers as addresses valid in this process (same-device
+    tensors' data_ptr(), or cc_ipc_open results), or None.  Returns (args,
+    result_is_b flag)."""
     flag = _i32(0)
-    u = up or (None, None, None, 0)
-    d = dn or (None, None, None, 0)
     args = Jacobi5HaloArgs(a.data_ptr(), b.data_ptr(), _lda(a), a.shape[0], a.shape[1], iters, sweep0,
-                           ctypes.addressof(flag), u[0], u[1], u[3], d[0], d[1], _ptr(flags), u[2], d[2],
-                           _ptr(status))
+                           ctypes.addressof(flag), _ptr(ll), up_ll, dn_ll, _ptr(status))
     return args, flag
+
+
+def ll_words(cols: int) -> int:
+    """Words of a slab's LL buffer: 2 parities x 2 sides x cols rounded up to 32."""
+    return 4 * ((cols + 31) & ~31)
 
 
 def peer_access(device: int, peer: int):

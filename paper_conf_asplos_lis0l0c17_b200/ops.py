@@ -82,13 +82,14 @@ def jacobi5(a, b, iters, backend="agent", order=None, tile=None, num_clusters=0,
     return b if flag.value else a
 
 
-def jacobi5_halo(a, b, iters, sweep0=0, up=None, dn=None, flags=None, status=None, backend="agent", order=None,
+def jacobi5_halo(a, b, iters, sweep0=0, ll=None, up_ll=None, dn_ll=None, status=None, backend="agent", order=None,
                  tile=None, num_clusters=0, stream=None, **kw):
     """One slab's sweeps sweep0+1 .. sweep0+iters with the halo exchange fused
-    into the sweep kernel (CC_K_JACOBI5_HALO, S§8(f)4).  `up` / `dn`: the
-    neighbours' (a_ptr, b_ptr, flags_ptr, rows) as addresses valid here, or
-    None.  Returns the buffer holding this slab's result."""
-    args, flag = cc.jacobi5_halo_args(a, b, iters, sweep0, up, dn, flags, status)
+    into the sweep kernel (CC_K_JACOBI5_HALO, S§8(f)4).  `ll`: this slab's LL
+    buffer (int64, cc.ll_words(cols) words); `up_ll` / `dn_ll`: the neighbours'
+    LL buffers as addresses valid here, or None.  Returns the buffer holding
+    this slab's result."""
+    args, flag = cc.jacobi5_halo_args(a, b, iters, sweep0, ll, up_ll, dn_ll, status)
     _launch("jacobi5_halo", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
     return b if flag.value else a
 

@@ -110,6 +110,44 @@ def jacobi_slab(sweep, a: torch.Tensor, b: torch.Tensor, iters: int, rows: int, 
     return src
 
 
+def conv_slab(conv, slab: torch.Tensor, rows: int, world: int, rank: int, R: int) -> torch.Tensor:
+    """Slab-sharded 2D convolution (S§8(e)): one exchange of the R halo rows on
+    each side, then `conv(slab)` on the local slab (its edges act as image
+    borders: every owned row is at least R rows from an edge that is not the
+    global border, so the owned outputs equal the unsharded ones).  Returns the
+    owned rows of the output."""
+    exchange_halos(slab, rows, world, rank, R)
+    lo, hi, llo, _ = slab_range(rows, world, rank, R)
+    return conv(slab)[lo - llo: hi - llo]
+
+
+def spmv_row_range(row_ptr, world: int, rank: int) -> tuple[int, int]:
+    """nnz-balanced contiguous rows for CSR SpMV (S§8(e)): rank g owns rows
+    [lo, hi) with lo the first row whose start is >= g * (rows + nnz) / world on
+    the merged rows+nnz axis (the merge-path measure the kernel balances, so
+    power-law hubs and empty rows both count)."""
+    import numpy as np
+    rp = np.asarray(row_ptr.cpu() if hasattr(row_ptr, "cpu") else row_ptr, dtype=np.int64)
+    rows = rp.size - 1
+    cost = rp[:rows] + np.arange(rows)             # merged coordinate of each row's start
+    total = rows + int(rp[-1])
+
+    def cut(g):
+        if g <= 0:
+            return 0
+        if g >= world:
+            return rows
+        return int(np.searchsorted(cost, (g * total) // world, side="left"))
+    return cut(rank), cut(rank + 1)
+
+
+def spmv_local(row_ptr, col, val, lo: int, hi: int):
+    """The CSR block of rows [lo, hi): (row_ptr rebased to 0, col, val) views."""
+    base = int(row_ptr[lo])
+    end = int(row_ptr[hi])
+    return row_ptr[lo: hi + 1] - base, col[base:end], val[base:end]
+
+
 def gather_rows(local_owned: torch.Tensor, rows: int, world: int, rank: int) -> torch.Tensor:
     """All-gather the owned row blocks of a 2D slab decomposition (final gather)."""
     if world == 1:
@@ -124,10 +162,10 @@ def gather_rows(local_owned: torch.Tensor, rows: int, world: int, rank: int) -> 
 
 # --------------------------------------------------------------------------
 # Fused peer-memory halo (S§8(f)4, CC_K_JACOBI5_HALO): instead of a separate
-# exchange per sweep, each rank's sweep kernel stores its boundary rows
-# straight into the neighbours' halo rows (NVLink peer mappings opened with
-# CUDA IPC) and raises per-tile-column flags the neighbour's next sweep waits
-# on.  The host only wires the neighbours once; no collective runs per sweep.
+# exchange per sweep, each rank's sweep kernel stores its boundary rows, each
+# value tagged with the sweep number, straight into the neighbours' LL buffers
+# (NVLink peer mappings opened with CUDA IPC); the neighbour's next sweep polls
+# the tags.  The host only wires the neighbours once; no collective per sweep.
 # --------------------------------------------------------------------------
 def neighbours(world: int, rank: int) -> tuple[int | None, int | None]:
     """(upper, lower) neighbour ranks of a slab decomposition, None at the ends."""
@@ -135,8 +173,8 @@ def neighbours(world: int, rank: int) -> tuple[int | None, int | None]:
 
 
 class PeerHaloSlab:
-    """This rank's slab buffers a/b (owned rows plus halo rows, as slab_range)
-    and the mapped addresses of its neighbours' buffers and flags.
+    """This rank's slab buffers a/b (owned rows plus halo rows, as slab_range),
+    its LL buffer, and the mapped addresses of its neighbours' LL buffers.
 
     Collective over the process group at construction (one all_gather_object
     of IPC handles) and at `close`; `sweeps` runs with no host exchange."""
@@ -145,46 +183,41 @@ class PeerHaloSlab:
         from . import ctaclust as cc
         self.cc, self.a, self.b, self.world, self.rank = cc, a, b, world, rank
         self.device = a.device.index or 0
-        gx = (a.shape[1] + 31) // 32
-        self.flags = torch.zeros(2 * gx, dtype=torch.int32, device=a.device)
+        self.ll = torch.zeros(cc.ll_words(a.shape[1]), dtype=torch.int64, device=a.device)
         self.status = torch.zeros(1, dtype=torch.int32, device=a.device)
-        mine = {"rows": a.shape[0], "pid": __import__("os").getpid(), "dev": self.device,
-                "h": [cc.ipc_handle(t) for t in (a, b, self.flags)] if world > 1 else None,
-                "p": [t.data_ptr() for t in (a, b, self.flags)]}
-        allv = [None] * world
+        mine = {"pid": __import__("os").getpid(), "ll": self.ll.data_ptr(),
+                "h": cc.ipc_handle(self.ll) if world > 1 else None}
+        allv = [mine]
         if world > 1:
+            allv = [None] * world
             dist.all_gather_object(allv, mine)
-        else:
-            allv = [mine]
         self._opened = []
-        self.up = self.dn = None
+        self.up_ll = self.dn_ll = None
         up, dn = neighbours(world, rank)
-        for which, g in (("up", up), ("dn", dn)):
+        for which, g in (("up_ll", up), ("dn_ll", dn)):
             if g is None:
                 continue
             other = allv[g]
-            if other["pid"] == mine["pid"]:            # same process: addresses are valid as they are
-                ptrs = other["p"]
-            else:                                      # one mapping per exported allocation
-                ptrs, bases = [], {}
-                for h, off in other["h"]:
-                    if h not in bases:
-                        bases[h] = cc.ipc_open(h, self.device)
-                        self._opened.append(bases[h])
-                    ptrs.append(bases[h] + off)
-            setattr(self, which, (ptrs[0], ptrs[1], ptrs[2], other["rows"]))
+            if other["pid"] == mine["pid"]:            # same process: the address is valid as it is
+                ptr = other["ll"]
+            else:
+                h, off = other["h"]
+                base = cc.ipc_open(h, self.device)
+                self._opened.append(base)
+                ptr = base + off
+            setattr(self, which, ptr)
         torch.cuda.synchronize(self.device)
         if world > 1:
-            dist.barrier()                             # every rank's flags are zero before any sweep
+            dist.barrier()                             # every rank's LL buffer is zero before any sweep
 
     def sweeps(self, iters: int, sweep0: int = 0, **kw) -> torch.Tensor:
         from . import ops
-        return ops.jacobi5_halo(self.a, self.b, iters, sweep0, self.up, self.dn, self.flags, self.status, **kw)
+        return ops.jacobi5_halo(self.a, self.b, iters, sweep0, self.ll, self.up_ll, self.dn_ll, self.status, **kw)
 
     def close(self):
         torch.cuda.synchronize(self.device)
         if self.world > 1:
-            dist.barrier()                             # no neighbour still stores into our buffers
+            dist.barrier()                             # no neighbour still stores into our buffer
         for base in self._opened:
             self.cc.ipc_close(base)
         self._opened = []

@@ -50,8 +50,8 @@ int main(void) {
   S(cc_jacobi5_args) O(cc_jacobi5_args, result_is_b) S(cc_conv2d_args) O(cc_conv2d_args, w)
   S(cc_spmv_args) O(cc_spmv_args, part) O(cc_spmv_args, nnz)
   S(cc_hist64_args) O(cc_hist64_args, n) O(cc_hist64_args, counts)
-  S(cc_jacobi5_halo_args) O(cc_jacobi5_halo_args, sweep0) O(cc_jacobi5_halo_args, up_rows)
-  O(cc_jacobi5_halo_args, dn_a) O(cc_jacobi5_halo_args, flags) O(cc_jacobi5_halo_args, status)
+  S(cc_jacobi5_halo_args) O(cc_jacobi5_halo_args, sweep0) O(cc_jacobi5_halo_args, ll)
+  O(cc_jacobi5_halo_args, dn_ll) O(cc_jacobi5_halo_args, status)
   return 0;
 }
 """

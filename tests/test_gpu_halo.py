@@ -2,7 +2,7 @@
 
 The slab-sharded Jacobi (S§8(e)) with the per-sweep halo exchange done inside
 the sweep kernel -- boundary rows stored straight into the neighbours' halo
-rows, per-tile-column flags for the dependency -- must equal the unsharded
+rows' LL buffers as {value, sweep} words, no fences -- must equal the unsharded
 fp32 oracle bit for bit (S§8(c) "Multi-GPU" pin: the G-shard result equals the
 1-GPU result; virtual-slab mode on one GPU).  Virtual slabs: G slabs on one
 GPU, their sweeps interleaved on one stream.  The two-process case maps the
@@ -35,21 +35,17 @@ def virtual_slabs(u0, world, iters, **kw):
         a = torch.zeros(lhi - llo, ld, device="cuda")[:, :cols]
         a.copy_(torch.from_numpy(np.ascontiguousarray(u0[llo:lhi])))
         b = torch.zeros(lhi - llo, ld, device="cuda")[:, :cols]
-        flags = torch.zeros(2 * ((cols + 31) // 32), dtype=torch.int32, device="cuda")
+        ll = torch.zeros(cc.ll_words(cols), dtype=torch.int64, device="cuda")
         status = torch.zeros(1, dtype=torch.int32, device="cuda")
-        slabs.append(dict(a=a, b=b, flags=flags, status=status, lo=lo, hi=hi, llo=llo))
+        slabs.append(dict(a=a, b=b, ll=ll, status=status, lo=lo, hi=hi, llo=llo))
 
-    def peer(g, s):          # neighbour g's buffers in the roles of sweep s+1
-        if g < 0 or g >= world:
-            return None
-        x = slabs[g]
-        src, dst = (x["a"], x["b"]) if s % 2 == 0 else (x["b"], x["a"])
-        return (src.data_ptr(), dst.data_ptr(), x["flags"].data_ptr(), x["a"].shape[0])
+    def nb(g):
+        return slabs[g]["ll"].data_ptr() if 0 <= g < world else None
 
     for s in range(iters):                    # sweep s+1 of every slab, in slab order
         for g, x in enumerate(slabs):
             src, dst = (x["a"], x["b"]) if s % 2 == 0 else (x["b"], x["a"])
-            ops.jacobi5_halo(src, dst, 1, s, peer(g - 1, s), peer(g + 1, s), x["flags"], x["status"], **kw)
+            ops.jacobi5_halo(src, dst, 1, s, x["ll"], nb(g - 1), nb(g + 1), x["status"], **kw)
     torch.cuda.synchronize()
     res = []
     for x in slabs:
@@ -60,7 +56,8 @@ def virtual_slabs(u0, world, iters, **kw):
 
 HVARIANTS = [dict(backend="agent", order="row"), dict(backend="default"), dict(backend="identity"),
              dict(backend="agent", order="tile", tile=(2, 2), stages=2, batch=1),
-             dict(backend="redirect", order="col")]
+             dict(backend="redirect", order="col"), dict(backend="agent", order="row", staging="direct"),
+             dict(backend="default", staging="l1")]
 
 
 @pytest.mark.parametrize("v", HVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
@@ -97,17 +94,15 @@ def test_virtual_slabs_full_width_sampled():
 
 
 def test_missing_neighbour_deposit_times_out_not_hangs():
-    """Sweep 2 of slab 0 launched without slab 1's sweep 1: the bounded wait
+    """Sweep 2 of slab 0 launched without slab 1's sweep 1: the bounded poll
     gives up after ~4 s and reports it in `status` instead of hanging."""
     u0 = synth.matrix(4, 64, 64)
     a = torch.from_numpy(u0[:33].copy()).cuda()
     b = torch.zeros_like(a)
-    pa, pb = torch.zeros(33, 64, device="cuda"), torch.zeros(33, 64, device="cuda")
-    pflags = torch.zeros(4, dtype=torch.int32, device="cuda")
-    flags = torch.zeros(4, dtype=torch.int32, device="cuda")
+    ll = torch.zeros(cc.ll_words(64), dtype=torch.int64, device="cuda")
+    pll = torch.zeros_like(ll)
     status = torch.zeros(1, dtype=torch.int32, device="cuda")
-    ops.jacobi5_halo(b, a, 1, 1, None, (pb.data_ptr(), pa.data_ptr(), pflags.data_ptr(), 33), flags, status,
-                     backend="default")
+    ops.jacobi5_halo(b, a, 1, 1, ll, None, pll.data_ptr(), status, backend="default")
     torch.cuda.synchronize()
     assert status.item() == 1
 
@@ -115,16 +110,15 @@ def test_missing_neighbour_deposit_times_out_not_hangs():
 def test_argument_errors():
     a = torch.zeros(40, 64, device="cuda")
     b = torch.zeros_like(a)
-    flags = torch.zeros(4, dtype=torch.int32, device="cuda")
-    nb = (a.data_ptr(), b.data_ptr(), flags.data_ptr(), 40)
-    with pytest.raises(cc.CtaclustError) as e:          # neighbour without my flags
-        ops.jacobi5_halo(a, b, 1, 0, nb, None, None)
+    ll = torch.zeros(cc.ll_words(64), dtype=torch.int64, device="cuda")
+    with pytest.raises(cc.CtaclustError) as e:          # a neighbour but no own LL buffer
+        ops.jacobi5_halo(a, b, 1, 0, None, ll.data_ptr(), None)
     assert e.value.status == -1
-    with pytest.raises(cc.CtaclustError) as e:          # halo rows must be read through TMA, not L1
-        ops.jacobi5_halo(a, b, 1, 0, nb, None, flags, staging="direct")
-    assert e.value.status == -6
-    with pytest.raises(cc.CtaclustError) as e:          # up neighbour's flags missing
-        ops.jacobi5_halo(a, b, 1, 0, (a.data_ptr(), b.data_ptr(), None, 40), None, flags)
+    with pytest.raises(cc.CtaclustError) as e:          # misaligned neighbour LL
+        ops.jacobi5_halo(a, b, 1, 0, ll, ll.data_ptr() + 8, None)
+    assert e.value.status == -1
+    with pytest.raises(cc.CtaclustError) as e:          # a 2-row slab with both halos owns nothing
+        ops.jacobi5_halo(a[:2], b[:2], 1, 0, ll, ll.data_ptr(), ll.data_ptr())
     assert e.value.status == -1
     # no neighbours: the plain sweep, equal to CC_K_JACOBI5
     u0 = synth.matrix(4, 40, 64)
@@ -159,8 +153,8 @@ WORKER = textwrap.dedent("""
 
 
 def test_two_processes_ipc_one_gpu(tmp_path):
-    """Two ranks in two processes on the same GPU: neighbours' buffers and flags
-    are mapped with CUDA IPC (cc_ipc_handle / cc_ipc_open), as across GPUs.
+    """Two ranks in two processes on the same GPU: the neighbour's LL buffer is
+    mapped with CUDA IPC (cc_ipc_handle / cc_ipc_open), as across GPUs.
     Without MPS the two contexts time-slice, so each sweep's wait may span a
     slice; the kernel's bounded wait keeps a failure from hanging."""
     script = tmp_path / "w.py"

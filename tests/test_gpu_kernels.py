@@ -33,6 +33,9 @@ VARIANTS = [
     dict(backend="agent", order="col", staging="direct", l2_hint="both", carveout=50),
     dict(backend="identity", l2_hint="stream_first", carveout=0),
     dict(backend="default", carveout=100),
+    dict(backend="static", order="col"),
+    dict(backend="static", order="row", num_clusters=592, stages=3),
+    dict(backend="static", order="tile", tile=(2, 2), num_clusters=5, staging="direct"),
 ]
 
 
@@ -141,7 +144,8 @@ JVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(
              dict(backend="agent", order="tile", tile=(8, 8), staging="l1"),
              dict(backend="agent", order="row", staging="direct"),
              dict(backend="agent", order="row", l2_hint="both"),
-             dict(backend="agent", order="row", staging="l1", l2_hint="both", carveout=25)]
+             dict(backend="agent", order="row", staging="l1", l2_hint="both", carveout=25),
+             dict(backend="static", order="row", num_clusters=592), dict(backend="static", order="tile", tile=(2, 2))]
 
 
 @pytest.mark.parametrize("v", JVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
@@ -187,7 +191,8 @@ CVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(
              dict(backend="default", staging="l1"), dict(backend="default", staging="direct"),
              dict(backend="agent", order="tile", tile=(8, 8), staging="l1"),
              dict(backend="agent", order="col", staging="direct"),
-             dict(backend="agent", order="row", l2_hint="both", carveout=100)]
+             dict(backend="agent", order="row", l2_hint="both", carveout=100),
+             dict(backend="static", order="row", num_clusters=740), dict(backend="static", order="col", staging="direct")]
 
 
 @pytest.mark.parametrize("v", CVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
@@ -246,7 +251,8 @@ def _csr_dev(rp, col, val):
 
 SVARIANTS = [dict(backend="default"), dict(backend="agent", order="row"), dict(backend="agent", active_agents=1),
              dict(backend="agent", stages=4, batch=5), dict(backend="identity"), dict(backend="redirect"),
-             dict(backend="agent", order="row", l2_hint="both"), dict(backend="default", carveout=0)]
+             dict(backend="agent", order="row", l2_hint="both"), dict(backend="default", carveout=0),
+             dict(backend="static", order="row", num_clusters=740), dict(backend="static", order="row", num_clusters=3)]
 
 
 def _edge_matrices():
@@ -305,7 +311,8 @@ HVARIANTS = [dict(backend="default"), dict(backend="agent", order="row"), dict(b
              dict(backend="default", staging="direct"), dict(backend="agent", order="row", staging="direct"),
              dict(backend="agent", order="row", staging="l1"), dict(backend="agent", order="row", active_agents=1),
              dict(backend="agent", order="row", stages=4, batch=3), dict(backend="agent", order="row", stages=1),
-             dict(backend="agent", order="row", l2_hint="both")]
+             dict(backend="agent", order="row", l2_hint="both"), dict(backend="static", order="row", num_clusters=888),
+             dict(backend="static", order="row", num_clusters=2, staging="direct")]
 
 
 @pytest.mark.parametrize("v", HVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))

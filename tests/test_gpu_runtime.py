@@ -41,6 +41,25 @@ def test_agent_census_and_map(gx, gy, order, tile, nsm):
     assert torch.all(sm >= 0)
 
 
+@pytest.mark.parametrize("gx,gy", GRIDS)
+@pytest.mark.parametrize("order,tile,M", [("row", (1, 1), 0), ("col", (1, 1), 296), ("tile", (8, 8), 1000),
+                                          ("row", (1, 1), 7), ("tile", (3, 5), 100000)])
+def test_static_binding_census_map_and_one_sm_per_cluster(gx, gy, order, tile, M, nsm):
+    """CC_BACKEND_AGENT_STATIC: CTA i runs cluster i.  Exactly once, the map is
+    the oracle's partition, and -- binding by construction -- every task of a
+    cluster ran on one SM (home coherence 1, exactly)."""
+    cen, sm, mp, p = ops.census(gx, gy, "static", order, tile, num_clusters=M)
+    torch.cuda.synchronize()
+    assert torch.all(cen == 1)
+    MM = M if M else nsm
+    ref = OP.plan(gx, gy, cc.ORDERS[order], MM, *tile)
+    assert np.array_equal(mp.cpu().numpy(), ref["perm"])
+    smv, perm, off = sm.cpu().numpy(), ref["perm"], ref["offsets"]
+    for i in range(min(MM, gx * gy)):
+        members = perm[off[i]:off[i + 1]]
+        assert len(set(smv[members].tolist())) <= 1, i
+
+
 @pytest.mark.parametrize("backend", ["default", "identity", "redirect"])
 @pytest.mark.parametrize("gx,gy", GRIDS)
 def test_other_backends_census(backend, gx, gy, nsm):
