@@ -144,6 +144,19 @@ def static_variants(kernel, order, tile=(1, 1), ks=None):
     return [(f"static-{tag}-m{k}", dict(backend="static", num_clusters=nsm * k, **o)) for k in ks if k <= 4 * amax]
 
 
+def band_variants(gy):
+    """Stencil orders that keep a global front (like the identity control) while
+    clustering: TILE blocks one or a few tile columns wide and the grid tall, one
+    block per cluster, so each SM walks its column band top to bottom (vertical
+    halos reused within ~1-4 tasks) while all SMs sweep the same rows together
+    (whole DRAM rows per step)."""
+    return [("agent-band4-m128", dict(backend="agent", order="tile", tile=(4, gy), num_clusters=128)),
+            ("static-band1-m512", dict(backend="static", order="tile", tile=(1, gy), num_clusters=512)),
+            ("static-band2-m256", dict(backend="static", order="tile", tile=(2, gy), num_clusters=256)),
+            ("agent-tile16x16", dict(backend="agent", order="tile", tile=(16, 16))),
+            ("agent-tile32x8", dict(backend="agent", order="tile", tile=(32, 8)))]
+
+
 def suite_matvec(quick):
     import torch
     from paper_conf_asplos_lis0l0c17_b200 import ops, synth
@@ -194,7 +207,7 @@ def suite_jacobi(quick):
     a = synth.matrix(4, N, N, backend="torch", device="cuda")
     b = torch.empty_like(a)
     v = variants_for("tile", (8, 8), stencil=True) + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
-        + static_variants("jacobi5", "row") + static_variants("jacobi5", "tile", (8, 8), ks=(4,))
+        + static_variants("jacobi5", "row") + static_variants("jacobi5", "tile", (8, 8), ks=(4,)) + band_variants(N // 32)
     r = measure(v, lambda kw: ops.jacobi5(a, b, T, **kw), 3, 8 * N * N * T,
                 extra=lambda ms: {"ms_per_sweep": round(ms / T, 5)}, warm=1)
     r["config"] = f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)"
@@ -217,7 +230,7 @@ def suite_conv(quick):
             ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
             ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))] \
             + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
-            + static_variants("conv2d", "row") + static_variants("conv2d", "tile", (8, 8), ks=(4,))
+            + static_variants("conv2d", "row") + static_variants("conv2d", "tile", (8, 8), ks=(4,)) + band_variants(N // 32)
         wt = torch.from_numpy(w).cuda().view(1, 1, 2 * R + 1, 2 * R + 1)
         img4 = img.view(1, 1, N, N)
         res[f"{2 * R + 1}x{2 * R + 1}"] = measure(

@@ -4,7 +4,7 @@ TAG=${1:-r02}
 OUT=gpurun_out/ncu_$TAG
 mkdir -p $OUT
 M=lts__t_sectors.sum,lts__t_sectors_srcunit_tex.sum,lts__t_sectors_srcunit_tex_op_read.sum,lts__t_sectors_srcunit_tex_op_write.sum,lts__t_sectors_srcunit_tex_op_red.sum,lts__t_sectors_srcunit_tex_op_atom.sum,lts__t_sector_hit_rate.pct,l1tex__t_sector_hit_rate.pct,l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum,dram__bytes_read.sum,dram__bytes_write.sum,sm__warps_active.avg.pct_of_peak_sustained_active,gpu__time_duration.sum
-K='regex:k_(agent|default|redirect|conv_tbc)'
+K='regex:k_(agent|static|default|redirect|conv_tbc)'
 run() {  # name, per-call launches, args...
   name=$1; per=$2; shift 2
   timeout -k 5 300 ncu --metrics $M --clock-control none -k "$K" -s $per -c $per --csv \
@@ -17,6 +17,8 @@ run matvec_agent-row 1 --kernel matvec --backend agent --order row
 run matvec_agent-col 1 --kernel matvec --backend agent --order col
 run matvec_agent-row-direct 1 --kernel matvec --backend agent --order row --staging direct
 run matvec_identity 1 --kernel matvec --backend identity
+run matvec_static-row-m2 1 --kernel matvec --backend static --order row --clusters 296
+run matvec_static-row-m3 1 --kernel matvec --backend static --order row --clusters 444
 for k in atax bicg mvt; do
   per=1; [ $k = atax ] && per=2
   run ${k}_default $per --kernel $k --backend default
@@ -25,6 +27,7 @@ for k in atax bicg mvt; do
   run ${k}_agent-row $per --kernel $k --backend agent --order row
   run ${k}_agent-col-direct $per --kernel $k --backend agent --order col --staging direct
   run ${k}_identity $per --kernel $k --backend identity
+  run ${k}_static-col-m3 $per --kernel $k --backend static --order col --clusters 444
 done
 for k in jacobi conv3 conv7; do
   run ${k}_default 1 --kernel $k --backend default
@@ -36,6 +39,7 @@ for k in jacobi conv3 conv7; do
   run ${k}_agent-tile8-direct 1 --kernel $k --backend agent --order tile --tile 8x8 --staging direct
   run ${k}_agent-row-l1 1 --kernel $k --backend agent --order row --staging l1
   run ${k}_identity 1 --kernel $k --backend identity
+  run ${k}_static-row-m4 1 --kernel $k --backend static --order row --clusters 592
 done
 for k in conv3 conv7; do
   run ${k}_tbc2 1 --kernel $k --backend tbcluster --cluster 2

@@ -25,6 +25,7 @@ def main():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--staging", default="default")
     ap.add_argument("--cluster", type=int, default=2)
+    ap.add_argument("--clusters", type=int, default=0, help="num_clusters M of the plan (static backend)")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--warm", type=int, default=1)
     ap.add_argument("--scale", type=int, default=24)
@@ -40,6 +41,8 @@ def main():
         kw["tile"] = tuple(int(t) for t in a.tile.split("x"))
     if a.backend == "tbcluster":
         kw["cluster_size"] = a.cluster
+    if a.clusters:
+        kw["num_clusters"] = a.clusters
     dev = "cuda"
     k = a.kernel
     if k == "matvec":
