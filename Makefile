@@ -1,5 +1,6 @@
 # libctaclust: sm_100a only (SASS, no PTX fallback); oracle: plain gcc.
 NVCC ?= nvcc
+PTXLOG ?= build_ptxas.log
 PKG := paper_conf_asplos_lis0l0c17_b200
 SRC := $(PKG)/csrc
 LIB := $(PKG)/libctaclust.so
@@ -10,7 +11,7 @@ HDRS := $(wildcard $(SRC)/*.cuh) include/ctaclust.h
 all: $(LIB) oracle/liboracle.so
 
 $(LIB): $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu $(HDRS)
-	$(NVCC) $(NVFLAGS) -shared -o $@ $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu -ldl 2> build_ptxas.log || (cat build_ptxas.log; exit 1)
+	$(NVCC) $(NVFLAGS) -shared -o $@ $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu -ldl 2> $(PTXLOG) || (cat $(PTXLOG); exit 1)
 
 oracle/liboracle.so: oracle/oracle.c
 	gcc -O2 -fPIC -shared -std=c11 -o $@ $<

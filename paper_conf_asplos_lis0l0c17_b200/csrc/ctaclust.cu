@@ -329,7 +329,8 @@ using BothB = GemvBody<32, 256, true, true>;
 template <class Body>
 static size_t dyn_smem(int stages, bool direct = false) {
     // direct loads stage nothing: keep the ring minimal so L1 keeps the space
-    return (size_t)stages * (direct ? 128 : Body::kStageBytes) + 128;
+    // (bodies whose direct path needs a per-task buffer size it themselves)
+    return (size_t)stages * (direct ? direct_stage_bytes<Body>() : Body::kStageBytes) + 128;
 }
 
 // Opt every instantiation of a body into large dynamic shared memory once.
@@ -436,7 +437,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     s.staging = o.staging == CC_STAGING_DEFAULT ? CC_STAGING_TMA : o.staging;
     s.l2_hint = o.l2_hint;
     const bool direct = s.staging == CC_STAGING_DIRECT;
-    s.stage_bytes = direct ? 128u : (uint32_t)Body::kStageBytes;
+    s.stage_bytes = direct ? (uint32_t)direct_stage_bytes<Body>() : (uint32_t)Body::kStageBytes;
     s.census = o.d_census;
     s.exec_sm = o.d_exec_sm;
     s.map = o.d_map;

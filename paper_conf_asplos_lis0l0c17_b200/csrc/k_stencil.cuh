@@ -415,10 +415,18 @@ struct Conv2dBody {
     static constexpr int RB = R >= 3 ? 4 : 2;
     static constexpr int kConsumers = 256 / RB;
     static constexpr int kStageBytes = HaloTile<R>::kBytes;
-    static constexpr int kDefaultStages = 4;
+    static constexpr int kDirectStageBytes = kStageBytes;  // the direct path stages into its own slot
+    // Two consumer groups per agent (alternate tiles).  One scheduler warp per
+    // two groups: with four 2-warp groups per agent (7x7) the single producer,
+    // which gets only its fair share of issue slots, could not keep them fed
+    // (measured 0.91x -> 0.99x of default order with two groups).
+#ifndef CC_CONV_GROUPS                                  // diagnostic builds: consumer groups per agent
+#define CC_CONV_GROUPS 2
+#endif
+    static constexpr int kGroups = CC_CONV_GROUPS;
+    static constexpr int kDefaultStages = 2 * kGroups; // two slots per group: the next tile lands while one computes
     static constexpr int kDefaultBatch = 4;
-    static constexpr int kMinAgents = R >= 3 ? 4 : 5;
-    static constexpr int kGroups = 256 / kConsumers;   // 2 or 4 groups consume alternate tiles
+    static constexpr int kMinAgents = (R >= 3 ? 12 : 10) / kGroups;
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
@@ -429,10 +437,9 @@ struct Conv2dBody {
     }
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         if (s.staging == STAGE_DIRECT) {
-            // plain-kernel form: the consumers stage the tile themselves through L1
-            // (one buffer per consumer group: groups work on different tiles)
-            __shared__ float4 s_in_g[kGroups][HaloTile<R>::kRows][ST_COLS / 4];
-            auto& s_in = s_in_g[(threadIdx.x - PRODUCER_THREADS) / kConsumers];
+            // plain-kernel form: the consumers stage the tile themselves through L1,
+            // into this task's ring slot (the group owns it until it releases it)
+            auto& s_in = *reinterpret_cast<float4 (*)[HaloTile<R>::kRows][ST_COLS / 4]>(const_cast<uint8_t*>(stage));
             const int x0 = bx * 32, y0 = by * 32;
             for (int idx = ctid; idx < HaloTile<R>::kRows * 10; idx += kConsumers) {
                 const int rr = idx / 10, cc = idx - rr * 10;
@@ -442,8 +449,9 @@ struct Conv2dBody {
                 s_in[rr][cc] = v;
             }
             consumer_sync<kConsumers>();
+            // (no trailing barrier: the slot is reused only after every warp of the
+            // group has released it)
             conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid, l2h);
-            consumer_sync<kConsumers>();                 // s_in is rewritten by the next task
             return;
         }
         conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid, l2h);
