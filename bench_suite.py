@@ -146,11 +146,16 @@ def static_variants(kernel, order, tile=(1, 1), ks=None):
 
 def band_variants(gy):
     """Stencil orders that keep a global front (like the identity control) while
-    clustering: TILE blocks one or a few tile columns wide and the grid tall, one
-    block per cluster, so each SM walks its column band top to bottom (vertical
-    halos reused within ~1-4 tasks) while all SMs sweep the same rows together
-    (whole DRAM rows per step)."""
-    return [("agent-band4-m128", dict(backend="agent", order="tile", tile=(4, gy), num_clusters=128)),
+    clustering.  rowfront: the static backend with one cluster per tile row (M =
+    gy): every row is a CTA walking left to right, all rows at once, so a tile's
+    vertical neighbours are processed at the same moment by the CTAs of the
+    rows above and below (halo re-reads hit L2).  band: TILE blocks one or a
+    few tile columns wide and the grid tall, each SM walking its band top to
+    bottom."""
+    return [("static-rowfront-M" + str(gy), dict(backend="static", order="row", num_clusters=gy)),
+            ("static-rowfront-M" + str(2 * gy), dict(backend="static", order="row", num_clusters=2 * gy)),
+            ("static-rowfront-M" + str(gy // 2), dict(backend="static", order="row", num_clusters=gy // 2)),
+            ("agent-band4-m128", dict(backend="agent", order="tile", tile=(4, gy), num_clusters=128)),
             ("static-band1-m512", dict(backend="static", order="tile", tile=(1, gy), num_clusters=512)),
             ("static-band2-m256", dict(backend="static", order="tile", tile=(2, gy), num_clusters=256)),
             ("agent-tile16x16", dict(backend="agent", order="tile", tile=(16, 16))),

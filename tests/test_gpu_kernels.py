@@ -135,6 +135,38 @@ def test_bicg_full_size_config2():
     assert relerr(q.cpu().numpy(), rq) <= TOL and relerr(s.cpu().numpy(), rs) <= TOL
 
 
+def test_atax_mvt_full_size_config2():
+    """BASELINE config 2 at full size n = 16384 for the other two kernels of the
+    bench step (ATAX two passes, MVT fused), in the bench's launch config
+    (agent backend, column clustering) and the static binding: every output."""
+    n = 16384
+    A = synth.matrix(3, n, n)
+    Ad = dev(A)
+    x, y1, y2 = synth.uniform(10, n), synth.uniform(15, n), synth.uniform(16, n)
+    x1, x2 = synth.uniform(13, n), synth.uniform(14, n)
+    rtmp, ry = O.atax(A, x)
+    r1, r2 = O.mvt(A, x1, x2, y1, y2)
+    for v in (dict(backend="agent", order="col"), dict(backend="static", order="col", num_clusters=444)):
+        tmp, y = ops.atax(Ad, dev(x), **v)
+        X1, X2 = dev(x1), dev(x2)
+        ops.mvt(Ad, dev(y1), dev(y2), X1, X2, **v)
+        torch.cuda.synchronize()
+        assert relerr(tmp.cpu().numpy(), rtmp) <= TOL and relerr(y.cpu().numpy(), ry) <= TOL, v
+        assert relerr(X1.cpu().numpy(), r1) <= TOL and relerr(X2.cpu().numpy(), r2) <= TOL, v
+
+
+def test_matvec_config1_static_binding():
+    """Config 1 (n = 1024, 32 x 32 tiles) in the configuration that measures
+    fastest (static binding, M = 3 x SMs, row clustering) and the agent."""
+    A, x = mat(1, 1024, 1024), synth.uniform(2, 1024)
+    ref = O.matvec(A, x)
+    for v in (dict(backend="static", order="row", num_clusters=444), dict(backend="static", order="row", num_clusters=296),
+              dict(backend="agent", order="row")):
+        y = ops.matvec(dev(A), dev(x), **v)
+        torch.cuda.synchronize()
+        assert relerr(y.cpu().numpy(), ref) <= TOL, v
+
+
 # ---------------------------------------------------------------- Jacobi
 JVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(8, 8)),
              dict(backend="agent", order="row"), dict(backend="agent", order="col", active_agents=2),
@@ -238,7 +270,7 @@ def test_conv2d_full_size_sampled():
                 i0, i1, j0, j1 = max(0, i - R), min(N, i + R + 1), max(0, j - R), min(N, j + R + 1)
                 win = np.stack([synth.uniform(5, j1 - j0, r * N + j0) for r in range(i0, i1)])
                 if R <= i < N - R and R <= j < N - R:
-                    ref = float(np.sum(w.astype(np.float64) * win.astype(np.float64)))
+                    ref = float(O.conv2d(win, w)[R, R])      # the oracle on the (2R+1)^2 window
                     assert abs(o[i, j].item() - ref) <= TOL * abs(ref), (R, i, j, v)
                 else:
                     assert o[i, j].item() == 0.0
@@ -303,6 +335,35 @@ def test_spmv(v):
         torch.cuda.synchronize()
         assert np.array_equal(y.cpu().numpy().astype(np.float64),
                               O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), vi, xi)), name
+
+
+def test_spmv_full_size_sampled():
+    """Config 5 at full size (R-MAT scale 24, edge factor 16, ~263 M nnz) in the
+    bench suite's launch configs: 3000 sampled rows plus the 20 heaviest rows
+    (the power-law hubs, spanning many logical CTAs) checked against the oracle
+    run on exactly those rows."""
+    rp, col = synth.rmat_csr(7, 24, 16, backend="torch", device="cuda")
+    nnz, n = col.numel(), rp.numel() - 1
+    val = synth.uniform(8, nnz, backend="torch", device="cuda")
+    x = synth.uniform(9, n, backend="torch", device="cuda")
+    Am = ops.SpmvMatrix(rp, col, val)
+    rph = rp.cpu().numpy().astype(np.int64)
+    deg = np.diff(rph)
+    rng = np.random.default_rng(5)
+    rows = np.unique(np.concatenate([rng.integers(0, n, 3000), np.argsort(deg)[-20:], [0, n - 1]]))
+    sub_rp = np.zeros(rows.size + 1, np.int64)
+    np.cumsum(deg[rows], out=sub_rp[1:])
+    idx = torch.from_numpy(np.concatenate([np.arange(rph[r], rph[r + 1]) for r in rows])).cuda()
+    sub_col = col[idx].cpu().numpy()
+    sub_val = val[idx].cpu().numpy()
+    ref = O.spmv_csr(sub_rp.astype(np.int32), sub_col.astype(np.int32), sub_val, x.cpu().numpy())
+    for v in (dict(backend="default"), dict(backend="agent", order="row"), dict(backend="identity")):
+        y = ops.spmv(Am, x, **v)
+        torch.cuda.synchronize()
+        got = y[torch.from_numpy(rows).cuda()].cpu().numpy()
+        nz = ref != 0
+        assert np.all(got[~nz] == 0), v
+        assert relerr(got[nz], ref[nz]) <= TOL, v
 
 
 # ---- S8(f)3: 64-bin histogram (HST, reading R24) -- integer counts, bit-exact ----
