@@ -119,6 +119,24 @@ __device__ __forceinline__ float4 ld_cached4(const float* p) {
     return *reinterpret_cast<const float4*>(p);
 }
 __device__ __forceinline__ float ld_cached(const float* p) { return *p; }
+// Issue-ordered forms for gathers: volatile asm keeps program order, so a run
+// of them leaves the SM back to back (all in flight) before any result is
+// used -- the compiler otherwise interleaves each gather with its consumer.
+__device__ __forceinline__ float ld_cached_issue(const float* p) {
+    float v;
+    asm volatile("ld.global.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ int32_t ld_stream_i32_issue(const int32_t* p) {
+    int32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ float ld_stream_f32_issue(const float* p) {
+    float v;
+    asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}
 
 __device__ __forceinline__ float ld_stream_f32_h(const float* p, uint64_t pol) {
     float v;

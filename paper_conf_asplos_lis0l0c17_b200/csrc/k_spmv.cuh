@@ -36,6 +36,10 @@ constexpr int SPMV_IPT = CC_SPMV_IPT;
 constexpr int SPMV_THREADS = 256;
 constexpr int SPMV_IPC = SPMV_IPT * SPMV_THREADS;   // merge items per logical CTA
 constexpr int SPMV_ROWCAP = 512;                    // staged row ends per CTA
+#ifndef CC_SPMV_GB
+#define CC_SPMV_GB 4
+#endif
+constexpr int SPMV_GB = CC_SPMV_GB;                 // gathers in flight per thread (batch)
 #ifndef CC_SPMV_PREFETCH
 #define CC_SPMV_PREFETCH 1
 #endif
@@ -122,17 +126,30 @@ struct SpmvBody {
         // all products of the CTA, coalesced: val/col stream past L1, the x
         // gathers go through it (16 independent loads per thread in flight)
         const int32_t nz = (int32_t)(y1 - y0);
-        if (l2h == 0) {
+        if (l2h == 0 && nz > 0) {
+            // two phases per batch of SPMV_GB items: all col/val loads in flight,
+            // then all x gathers in flight, then the products -- the gathers'
+            // latency is paid once per batch, not once per item
 #pragma unroll
-            for (int k = 0; k < SPMV_IPT; ++k) {
-                const int32_t j = t + k * kConsumers;
-                if (j < nz) {
-                    const int32_t c = ld_stream_i32(p.col + y0 + j);
-                    const float v = ld_stream_f32(p.val + y0 + j);
-                    s_prod[j + j / SPMV_IPT] = v * ld_cached(p.x + c);
+            for (int k0 = 0; k0 < SPMV_IPT; k0 += SPMV_GB) {
+                int32_t c[SPMV_GB];
+                float v[SPMV_GB], xv[SPMV_GB];
+#pragma unroll
+                for (int k = 0; k < SPMV_GB; ++k) {
+                    const int32_t j = t + (k0 + k) * kConsumers;
+                    const bool ok = j < nz;           // past the end: re-read item 0 (nz > 0)
+                    c[k] = ld_stream_i32_issue(p.col + y0 + (ok ? j : 0));
+                    v[k] = ld_stream_f32_issue(p.val + y0 + (ok ? j : 0));
+                }
+#pragma unroll
+                for (int k = 0; k < SPMV_GB; ++k) xv[k] = ld_cached_issue(p.x + c[k]);
+#pragma unroll
+                for (int k = 0; k < SPMV_GB; ++k) {
+                    const int32_t j = t + (k0 + k) * kConsumers;
+                    if (j < nz) s_prod[j + j / SPMV_IPT] = v[k] * xv[k];
                 }
             }
-        } else {
+        } else if (l2h != 0) {
             // L2 hints (S§8(f)2): col/val streamed (evict_first), x reused (evict_last)
             const bool hf = l2h & L2H_STREAM_FIRST, hl = l2h & L2H_REUSE_LAST;
             const uint64_t pf = l2_evict_first(), pl = l2_evict_last();
