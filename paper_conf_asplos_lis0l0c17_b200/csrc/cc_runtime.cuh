@@ -332,10 +332,20 @@ template <class B> struct DirectStageBytes<B, decltype((void)B::kDirectStageByte
 };
 template <class B> constexpr int direct_stage_bytes() { return DirectStageBytes<B>::value; }
 
+// Merged staging (kMerge = 2): a body may take two logical CTAs per ring slot
+// when the scheduler pops them back to back and they are horizontal
+// neighbours (same by, bx and bx+1) -- consecutive positions of a ROW or TILE
+// cluster.  Their tiles share halo columns, so one wider copy stages both:
+// the clustered order is what makes the pair co-located, and the shared
+// halo is then reused from shared memory instead of being copied twice.
+template <class B, class = void> struct MergeOf { static constexpr int value = 1; };
+template <class B> struct MergeOf<B, decltype((void)B::kMerge)> { static constexpr int value = B::kMerge; };
+
 struct RingShared {
     uint64_t full[MAX_STAGES];
     uint64_t empty[MAX_STAGES];
     int4 slot[MAX_STAGES];       // (v, lin, bx, by) decoded once by the scheduler warp
+    int4 slot2[MAX_STAGES];      // merged slots: (v, lin) of the second CTA, and n
 };
 
 __device__ __forceinline__ uint8_t* ring_base(uint8_t* dyn) {
@@ -386,9 +396,11 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         int st = 0;
         uint32_t ph = 0;                                       // empty-barrier parity
         int32_t t = 0;
+        int32_t pending = -1;                                  // popped but not yet staged (merge miss)
         for (;; ++t) {
             if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
-            const int32_t v = producer_next<kStatic>(s, P, lane);
+            const int32_t v = pending >= 0 ? pending : producer_next<kStatic>(s, P, lane);
+            pending = -1;
             if (v < 0) {
                 if (lane == 0) R.slot[st] = make_int4(-1, 0, 0, 0);
                 break;
@@ -396,7 +408,26 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             int32_t lin, bx, by;
             lin_to_bxby(s, v, &lin, &bx, &by);
             if (lane == 0) R.slot[st] = make_int4(v, lin, bx, by);
-            body.produce(s, bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
+            if constexpr (MergeOf<Body>::value > 1) {
+                int n = 1;
+                if (body.can_merge(s)) {
+                    const int32_t v2 = producer_next<kStatic>(s, P, lane);
+                    if (v2 >= 0) {
+                        int32_t lin2, bx2, by2;
+                        lin_to_bxby(s, v2, &lin2, &bx2, &by2);
+                        if (by2 == by && bx2 == bx + 1) {
+                            n = 2;
+                            if (lane == 0) R.slot2[st] = make_int4(v2, lin2, 2, 0);
+                        } else {
+                            pending = v2;                      // next slot starts with it
+                        }
+                    }
+                }
+                if (n == 1 && lane == 0) R.slot2[st] = make_int4(-1, 0, 1, 0);
+                body.produce_n(s, bx, by, n, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
+            } else {
+                body.produce(s, bx, by, ring + (size_t)st * s.stage_bytes, &R.full[st], lane);
+            }
             if (++st == S) { st = 0; ph ^= 1u; }
         }
         // one end marker per consumer group: slots t .. t+G-1
@@ -430,8 +461,17 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
             mbar_wait(&R.full[st], ph);
             const int4 sl = R.slot[st];
             if (sl.x < 0) break;
-            body.consume(s, sl.z, sl.w, ring + (size_t)st * s.stage_bytes, ctid);
-            if (ctid == 0) record(s, sl.x, sl.y);
+            if constexpr (MergeOf<Body>::value > 1) {
+                const int4 s2 = R.slot2[st];
+                body.consume_n(s, sl.z, sl.w, s2.z, ring + (size_t)st * s.stage_bytes, ctid);
+                if (ctid == 0) {
+                    record(s, sl.x, sl.y);
+                    if (s2.z > 1) record(s, s2.x, s2.y);
+                }
+            } else {
+                body.consume(s, sl.z, sl.w, ring + (size_t)st * s.stage_bytes, ctid);
+                if (ctid == 0) record(s, sl.x, sl.y);
+            }
             __syncwarp();
             if (lane == 0) mbar_arrive(&R.empty[st]);
             st += Body::kGroups;

@@ -669,7 +669,10 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             JacobiParams jp;
             memset(&jp, 0, sizeof jp);
             jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
-            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
+            if (x->rows > 0 && x->cols > 0) {
+                CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
+                CC_TRY(make_tmap(&jp.tmap2, src, x->rows, x->cols, x->ld, ST_COLS2, 34));
+            }
             s = launch_body<Jacobi5Body>(c, jp);
             std::swap(src, dst);
         }
@@ -714,7 +717,10 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             memset(&cp, 0, sizeof cp);
             cp.in = x->in; cp.out = x->out; cp.ld = x->ld; cp.rows = x->rows; cp.cols = x->cols;
             memcpy(cp.w, x->w, sizeof cp.w);
-            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 34));
+            if (x->rows > 0 && x->cols > 0) {
+                CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 34));
+                CC_TRY(make_tmap(&cp.tmap2, x->in, x->rows, x->cols, x->ld, ST_COLS2, 34));
+            }
             s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<1>(c, cp)
                                                    : launch_body<Conv2dBody<1>>(c, cp);
         } else if (x->R == 3) {
@@ -722,7 +728,10 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             memset(&cp, 0, sizeof cp);
             cp.in = x->in; cp.out = x->out; cp.ld = x->ld; cp.rows = x->rows; cp.cols = x->cols;
             memcpy(cp.w, x->w, sizeof cp.w);
-            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 38));
+            if (x->rows > 0 && x->cols > 0) {
+                CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 38));
+                CC_TRY(make_tmap(&cp.tmap2, x->in, x->rows, x->cols, x->ld, ST_COLS2, 38));
+            }
             s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<3>(c, cp)
                                                    : launch_body<Conv2dBody<3>>(c, cp);
         } else {

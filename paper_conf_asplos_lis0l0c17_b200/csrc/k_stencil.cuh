@@ -25,11 +25,22 @@ namespace cc {
 
 enum : int32_t { STAGE_TMA = 1, STAGE_L1 = 2, STAGE_DIRECT = 3 };
 constexpr int ST_COLS = 40;                 // staged floats per row (x0-4 .. x0+35)
+constexpr int ST_COLS2 = 72;                // merged slot: two neighbouring tiles (x0-4 .. x0+67)
 
 template <int H>
 struct HaloTile {
     static constexpr int kRows = 32 + 2 * H;
     static constexpr int kBytes = ((kRows * ST_COLS * 4) + 127) & ~127;
+    static constexpr int kBytes2 = ((kRows * ST_COLS2 * 4) + 127) & ~127;   // two tiles, one box
+    // warp-collective: stage the merged box of tiles (bx, by), (bx+1, by) by TMA
+    __device__ __forceinline__ static void stage2(int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
+                                                  const CUtensorMap* tmap2, int32_t l2_hint) {
+        stage_commit(full, lane, (uint32_t)(kRows * ST_COLS2 * 4));
+        if (lane == 0) {
+            if (l2_hint & L2H_REUSE_LAST) tma_load_2d_h(dst, tmap2, x0 - 4, y0 - H, full, l2_evict_last());
+            else tma_load_2d(dst, tmap2, x0 - 4, y0 - H, full);
+        }
+    }
     // warp-collective: stage rows y0-H.., columns x0-4.. of `src` (TMA or L1 mode).
     __device__ __forceinline__ static void stage(const float* src, int64_t ld, int32_t rows, int32_t cols,
                                                  int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
@@ -120,7 +131,7 @@ struct JacobiHalo {
     uint32_t sweep;           // absolute sweep number of this launch (1-based)
     int32_t* status;          // optional: 1 = a poll timed out (results invalid)
 };
-struct JacobiParams { CUtensorMap tmap; const float* a; float* b; int64_t ld; int32_t rows, cols; JacobiHalo h; };
+struct JacobiParams { CUtensorMap tmap; CUtensorMap tmap2; const float* a; float* b; int64_t ld; int32_t rows, cols; JacobiHalo h; };
 
 __device__ __forceinline__ uint64_t globaltimer() {
     uint64_t t;
@@ -217,7 +228,8 @@ template <bool HALO>
 struct Jacobi5BodyT {
     static constexpr int RB = 2;                  // output rows per consumer thread
     static constexpr int kConsumers = 256 / RB;
-    static constexpr int kTileBytes = HaloTile<1>::kBytes;
+    static constexpr int kMerge = HALO ? 1 : 2;    // two neighbouring tiles per slot (cc_runtime.cuh: MergeOf)
+    static constexpr int kTileBytes = HALO ? HaloTile<1>::kBytes : HaloTile<1>::kBytes2;
     static constexpr int kStageBytes = kTileBytes + (HALO ? 2 * 32 * 8 : 0);   // + the two LL halo rows (words)
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
@@ -263,9 +275,31 @@ struct Jacobi5BodyT {
         HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h);
     }
 
-    // thread (rows r0 .. r0+RB-1, columns 4*c4 .. 4*c4+3): the RB+2 input rows
-    // it touches are read once each
+    // merged slots (plain sweep, TMA staging): tiles (bx, by), (bx+1, by) in one box
+    __device__ __forceinline__ bool can_merge(const Sched& s) const { return s.staging == STAGE_TMA; }
+    __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
+                                              uint64_t* full, int lane) {
+        if (n == 2) HaloTile<1>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h);
+        else produce(s, bx, by, stage, full, lane);
+    }
+    __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
+                                              int ctid) {
+        if (n == 2) {
+            consume_at(s, bx, by, stage, ctid, ST_COLS2, 0);
+            consume_at(s, bx + 1, by, stage, ctid, ST_COLS2, 32);
+        } else {
+            consume_at(s, bx, by, stage, ctid, ST_COLS, 0);
+        }
+    }
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        consume_at(s, bx, by, stage, ctid, ST_COLS, 0);
+    }
+
+    // thread (rows r0 .. r0+RB-1, columns 4*c4 .. 4*c4+3): the RB+2 input rows
+    // it touches are read once each.  The staged box has `pitch` floats per row
+    // and this tile's columns start `coff` floats in.
+    __device__ __forceinline__ void consume_at(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid,
+                                               int pitch, int coff) {
         by = phys_row(by);
         const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
         const int gx = bx * 32 + 4 * c4;
@@ -292,13 +326,13 @@ struct Jacobi5BodyT {
                 if (c4 == 7) re[j] = (in && gx + 4 < p.cols) ? ld_cached(a + (int64_t)j * p.ld + 4) : 0.f;
             }
         } else {
-            const float* t = reinterpret_cast<const float*>(stage) + r0 * ST_COLS + 4 + 4 * c4;   // staged row r0 = gy0-1
+            const float* t = reinterpret_cast<const float*>(stage) + r0 * pitch + coff + 4 + 4 * c4;   // staged row r0 = gy0-1
 #pragma unroll
-            for (int k = 0; k < RB + 2; ++k) row[k] = *reinterpret_cast<const float4*>(t + k * ST_COLS);
+            for (int k = 0; k < RB + 2; ++k) row[k] = *reinterpret_cast<const float4*>(t + k * pitch);
 #pragma unroll
             for (int j = 0; j < RB; ++j) {
-                lw[j] = t[(j + 1) * ST_COLS - 1];
-                re[j] = t[(j + 1) * ST_COLS + 4];
+                lw[j] = t[(j + 1) * pitch - 1];
+                re[j] = t[(j + 1) * pitch + 4];
             }
         }
         if (!in_col) return;
@@ -355,7 +389,7 @@ using Jacobi5HaloBody = Jacobi5BodyT<true>;
 // The filter lives in the kernel parameter bank (constant-bank operands).
 // ---------------------------------------------------------------------------
 template <int R>
-struct ConvParams { CUtensorMap tmap; const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
+struct ConvParams { CUtensorMap tmap; CUtensorMap tmap2; const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
 
 // Thread ctid computes RB vertically adjacent rows x 4 columns of the tile
 // (256/RB threads per tile).  Each staged input row is read once (3 LDS.128)
@@ -365,7 +399,8 @@ struct ConvParams { CUtensorMap tmap; const float* in; float* out; int64_t ld; i
 // filter's row-major tap order, as in the oracle.
 template <int R, int RB = 1>
 __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const float* rows_base,
-                                                  int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0) {
+                                                  int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0,
+                                                  int pitch = ST_COLS) {
     // rows_base points at the staged row holding input row y0 - R, column x0 - 4
     constexpr int K = 2 * R + 1;
     const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
@@ -377,7 +412,7 @@ __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const 
         for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
 #pragma unroll
     for (int ir = 0; ir < K + RB - 1; ++ir) {           // staged rows r0 .. r0+K+RB-2
-        const float4* row = reinterpret_cast<const float4*>(rows_base + (r0 + ir) * ST_COLS + 4 * c4);
+        const float4* row = reinterpret_cast<const float4*>(rows_base + (r0 + ir) * pitch + 4 * c4);
         float4 q0 = row[0], q1 = row[1], q2 = row[2];
         const float win[12] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w, q2.x, q2.y, q2.z, q2.w};
 #pragma unroll
@@ -414,8 +449,12 @@ struct Conv2dBody {
     // overhead of ~150 instructions per warp); the 3x3 is HBM bound
     static constexpr int RB = R >= 3 ? 4 : 2;
     static constexpr int kConsumers = 256 / RB;
-    static constexpr int kStageBytes = HaloTile<R>::kBytes;
-    static constexpr int kDirectStageBytes = kStageBytes;  // the direct path stages into its own slot
+    // two neighbouring tiles per slot for the HBM-bound 3x3 (cc_runtime.cuh:
+    // MergeOf); the FP32-bound 7x7 gains nothing from the shared halo and
+    // measured 1-2 % slower merged
+    static constexpr int kMerge = R >= 3 ? 1 : 2;
+    static constexpr int kStageBytes = kMerge > 1 ? HaloTile<R>::kBytes2 : HaloTile<R>::kBytes;
+    static constexpr int kDirectStageBytes = HaloTile<R>::kBytes;  // the direct path stages into its own slot
     // Two consumer groups per agent (alternate tiles).  One scheduler warp per
     // two groups: with four 2-warp groups per agent (7x7) the single producer,
     // which gets only its fair share of issue slots, could not keep them fed
@@ -426,7 +465,10 @@ struct Conv2dBody {
     static constexpr int kGroups = CC_CONV_GROUPS;
     static constexpr int kDefaultStages = 2 * kGroups; // two slots per group: the next tile lands while one computes
     static constexpr int kDefaultBatch = 4;
-    static constexpr int kMinAgents = (R >= 3 ? 12 : 10) / kGroups;
+#ifndef CC_CONV3_MIN_AGENTS                             // 3x3 agents per SM: 4 (56 registers, no
+#define CC_CONV3_MIN_AGENTS 4                           // spill) measured 5 % faster than 5 (40 + spills)
+#endif
+    static constexpr int kMinAgents = R >= 3 ? 12 / kGroups : CC_CONV3_MIN_AGENTS;
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
@@ -455,6 +497,25 @@ struct Conv2dBody {
             return;
         }
         conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid, l2h);
+    }
+    // merged slots (TMA staging): tiles (bx, by), (bx+1, by) from one box
+    __device__ __forceinline__ bool can_merge(const Sched& s) const { return s.staging == STAGE_TMA; }
+    __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
+                                              uint64_t* full, int lane) {
+        if (n == 2) HaloTile<R>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h);
+        else produce(s, bx, by, stage, full, lane);
+    }
+    __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
+                                              int ctid) {
+        if (n == 2) {
+            // one instance of the tile code, run twice (two unrolled copies would
+            // not fit the register budget of the resident agents)
+            const float* b = reinterpret_cast<const float*>(stage);
+#pragma unroll 1
+            for (int k = 0; k < 2; ++k) conv_tile_compute<R, RB>(p, b + 32 * k, bx + k, by, ctid, l2h, ST_COLS2);
+        } else {
+            consume(s, bx, by, stage, ctid);
+        }
     }
     __device__ __forceinline__ void finish(int) {}
 };
