@@ -545,7 +545,7 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     CC_CUDA(cudaFuncSetAttribute(k_conv_tbc<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     CC_CUDA(cudaFuncSetAttribute(k_conv_tbc<R>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     cudaLaunchConfig_t cfg = {};
-    cfg.blockDim = dim3(TBC_THREADS);
+    cfg.blockDim = dim3(tbc_threads<R>());
     cfg.dynamicSmemBytes = smem;
     cfg.stream = c.st;
     cudaLaunchAttribute at[1];

@@ -33,8 +33,10 @@ constexpr int TBC_ROW_BYTES = TBC_COLS * 4;
 constexpr int TBC_HALO = 8;             // halo box height (keeps every TMA box 128-B aligned)
 constexpr int TBC_ROWS = 2 * TBC_HALO + 32;
 constexpr int TBC_BUF_BYTES = TBC_ROWS * TBC_ROW_BYTES;
-constexpr int TBC_THREADS = 128;        // 4 warps, 2 output rows x 4 columns per thread
-constexpr int TBC_RB = 2;
+// output rows per thread: 2 for the HBM-bound 3x3 (4 warps per CTA), 4 for the
+// FP32-bound 7x7 (2 warps: each staged row feeds more outputs, as in the agents)
+template <int R> constexpr int tbc_rb() { return R >= 3 ? 4 : 2; }
+template <int R> constexpr int tbc_threads() { return 256 / tbc_rb<R>(); }
 // smem per buffer: [0, 8) top halo box | [8, 40) centre | [40, 48) bottom halo box
 inline size_t tbc_smem_bytes(int) { return 256 + 2 * (size_t)TBC_BUF_BYTES; }
 
@@ -78,10 +80,10 @@ __device__ __forceinline__ void mbar_arrive_remote(uint64_t* bar, uint32_t rank)
 }
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) { mbar_wait(bar, parity); }
 
-// Persistent grid of NC clusters x C CTAs (1D, cluster dims (C,1,1)), 128 threads,
-// dynamic smem tbc_smem_bytes(C).
+// Persistent grid of NC clusters x C CTAs (1D, cluster dims (C,1,1)),
+// tbc_threads<R>() threads, dynamic smem tbc_smem_bytes(C).
 template <int R>
-__global__ void __launch_bounds__(TBC_THREADS) k_conv_tbc(const __grid_constant__ CUtensorMap map_rows,
+__global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_constant__ CUtensorMap map_rows,
                                                           const __grid_constant__ CUtensorMap map_halo,
                                                           const __grid_constant__ Sched s,
                                                           const __grid_constant__ ConvParams<R> p, int32_t C) {
@@ -137,7 +139,7 @@ __global__ void __launch_bounds__(TBC_THREADS) k_conv_tbc(const __grid_constant_
                 if (rank < C - 1) mbar_arrive_remote(&ready[b], rank + 1);
             }
             mbar_wait_cluster(&ready[b], par);           // theirs landed too
-            for (int idx = threadIdx.x; idx < 2 * R * 10; idx += TBC_THREADS) {
+            for (int idx = threadIdx.x; idx < 2 * R * 10; idx += tbc_threads<R>()) {
                 const int side = idx / (R * 10), rem = idx - side * R * 10;
                 const int rr = rem / 10, cc = rem - rr * 10;
                 if (side == 0 && rank > 0) {             // rows 8-R.. <- rank-1's centre rows 32-R..
@@ -157,7 +159,7 @@ __global__ void __launch_bounds__(TBC_THREADS) k_conv_tbc(const __grid_constant_
         }
         const int bx = u % gx, by = (u / gx) * C + rank;
         if (by < gy) {
-            conv_tile_compute<R, TBC_RB>(p, buf + (TBC_HALO - R) * TBC_COLS, bx, by, threadIdx.x);
+            conv_tile_compute<R, tbc_rb<R>()>(p, buf + (TBC_HALO - R) * TBC_COLS, bx, by, threadIdx.x);
             if (threadIdx.x == 0) {
                 const int32_t lin = by * gx + bx;
                 if (s.census) atomicAdd(s.census + lin, 1u);
