@@ -1,7 +1,7 @@
 # Full evidence pass for one round tag (1 GPU): correctness, bench line, suite,
 # ncu L2-sector suite, bench launch list + full captures, categorizer.
 #   bash scripts/gpu_round.sh r05
-TAG=${1:-r05}
+TAG=${1:-r07}
 bash scripts/gpu_check.sh
 bash scripts/ncu_suite.sh $TAG > gpurun_out/ncu_suite_$TAG.log 2>&1; echo "ncu_suite done"
 bash scripts/ncu_bench.sh $TAG > gpurun_out/ncu_bench_$TAG.log 2>&1; echo "ncu_bench done"; cat gpurun_out/ncu_bench_$TAG.log
