@@ -65,12 +65,19 @@ def graph_ms(fn, reps, inner):
     return time_ms(g.replay, reps, warm=1) / inner
 
 
+VARIANT_FILTER = None   # --variants REGEX: keep matching rows (plus the default-order rows)
+
+
 def measure(variants, fn, reps, nbytes, extra=None, warm=3, inner=1, graph=False, context=None):
     """`context`: {name: callable} vendor-library timings of the same
     computation (cuBLAS / cuDNN / cuSPARSE via torch), reported as lib-* rows
     for absolute context; they are not part of the default/clustered
     comparison."""
     rows = []
+    if VARIANT_FILTER:
+        import re
+        variants = [(n, kw) for n, kw in variants if n.startswith("default") or re.search(VARIANT_FILTER, n)]
+        context = None
     for name, kw in variants:
         ms = graph_ms(lambda: fn(kw), reps, inner) if graph else time_ms(lambda: fn(kw), reps, warm=warm, inner=inner)
         gbs = nbytes / (ms * 1e-3) / 1e9
@@ -162,6 +169,33 @@ def band_variants(gy):
             ("agent-tile32x8", dict(backend="agent", order="tile", tile=(32, 8)))]
 
 
+def interleaved_order(gx, gy, M, c):
+    """USER order for a time-aligned row clustering: the row-major sequence is
+    cut into chunks of c horizontally adjacent tiles and chunk k goes to
+    cluster k mod M, so every cluster holds co-located pairs (merged staging)
+    while all clusters sweep the image top to bottom together (the vertical
+    halo is re-read from L2 while it is still there)."""
+    import numpy as np
+    V = gx * gy
+    K = (V + c - 1) // c
+    seq = []
+    for i in range(M):
+        for k in range(i, K, M):
+            seq.extend(range(k * c, min(V, (k + 1) * c)))
+    out = np.asarray(seq, dtype=np.int32)
+    assert out.size == V
+    return out
+
+
+def ilv_variants(gx, gy, cs=(2, 4, 8), static_ks=(2, 4)):
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    nsm = cc.device_info(0)["num_sms"]
+    v = [(f"agent-ilv-c{c}", dict(backend="agent", user_order=interleaved_order(gx, gy, nsm, c))) for c in cs]
+    v += [(f"static-ilv-c2-m{k}", dict(backend="static", num_clusters=nsm * k,
+                                        user_order=interleaved_order(gx, gy, nsm * k, 2))) for k in static_ks]
+    return v
+
+
 def suite_matvec(quick):
     import torch
     from paper_conf_asplos_lis0l0c17_b200 import ops, synth
@@ -212,7 +246,8 @@ def suite_jacobi(quick):
     a = synth.matrix(4, N, N, backend="torch", device="cuda")
     b = torch.empty_like(a)
     v = variants_for("tile", (8, 8), stencil=True) + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
-        + static_variants("jacobi5", "row") + static_variants("jacobi5", "tile", (8, 8), ks=(4,)) + band_variants(N // 32)
+        + static_variants("jacobi5", "row") + static_variants("jacobi5", "tile", (8, 8), ks=(4,)) + band_variants(N // 32) \
+        + ilv_variants(N // 32, N // 32)
     r = measure(v, lambda kw: ops.jacobi5(a, b, T, **kw), 3, 8 * N * N * T,
                 extra=lambda ms: {"ms_per_sweep": round(ms / T, 5)}, warm=1)
     r["config"] = f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)"
@@ -235,7 +270,8 @@ def suite_conv(quick):
             ("tbcluster-4", dict(backend="tbcluster", cluster_size=4)),
             ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))] \
             + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
-            + static_variants("conv2d", "row") + static_variants("conv2d", "tile", (8, 8), ks=(4,)) + band_variants(N // 32)
+            + static_variants("conv2d", "row") + static_variants("conv2d", "tile", (8, 8), ks=(4,)) + band_variants(N // 32) \
+            + ilv_variants(N // 32, N // 32)
         wt = torch.from_numpy(w).cuda().view(1, 1, 2 * R + 1, 2 * R + 1)
         img4 = img.view(1, 1, N, N)
         res[f"{2 * R + 1}x{2 * R + 1}"] = measure(
@@ -419,6 +455,8 @@ if __name__ == "__main__":
     ap.add_argument("out")
     ap.add_argument("--only", default=None)
     ap.add_argument("--quick", action="store_true")
+    ap.add_argument("--variants", default=None, help="regex: time only matching variants (and default order)")
     a = ap.parse_args()
+    VARIANT_FILTER = a.variants
     run(a.out, a.only.split(",") if a.only else None, a.quick)
     print(table(a.out))

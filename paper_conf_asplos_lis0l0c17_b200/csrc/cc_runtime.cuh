@@ -201,6 +201,31 @@ __device__ __forceinline__ void lin_to_bxby(const Sched& s, int32_t v, int32_t* 
     }
 }
 
+// Producer-warp form (v warp-uniform, all 32 lanes present).  A USER order
+// table lookup is a dependent L2 round trip per task on the scheduler's
+// critical path (measured 2.3x slower conv 3x3 than the computed orders);
+// the warp instead loads a window of 32 consecutive positions with one
+// coalesced load into shared memory (win[0] = base, win[1..32] = entries;
+// nothing held in registers across the task loop) and serves the cluster's
+// consecutive pops from it.
+__device__ __forceinline__ void lin_to_bxby_warp(const Sched& s, int32_t* win, int32_t v, int lane, int32_t* lin,
+                                                 int32_t* bx, int32_t* by) {
+    if (s.mode != MODE_IDENTITY && s.g.order == ORDER_USER) {
+        const int32_t base = *(volatile int32_t*)win;
+        if (v < base || v >= base + 32) {
+            const int32_t u = v + lane < s.g.V ? s.user[v + lane] : 0;
+            __syncwarp();
+            win[1 + lane] = u;
+            if (lane == 0) win[0] = v;
+            __syncwarp();
+        }
+        const int32_t l = ((volatile int32_t*)win)[1 + v - *(volatile int32_t*)win];
+        *by = l / s.g.gx; *bx = l - *by * s.g.gx; *lin = l;
+    } else {
+        lin_to_bxby(s, v, lin, bx, by);
+    }
+}
+
 __device__ __forceinline__ void record(const Sched& s, int32_t v, int32_t lin) {
     if (s.census) atomicAdd(s.census + lin, 1u);
     if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();
@@ -397,6 +422,9 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         uint32_t ph = 0;                                       // empty-barrier parity
         int32_t t = 0;
         int32_t pending = -1;                                  // popped but not yet staged (merge miss)
+        __shared__ int32_t s_uwin[33];                         // USER-order window (lin_to_bxby_warp)
+        if (lane == 0) s_uwin[0] = -64;
+        __syncwarp();
         for (;; ++t) {
             if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
             const int32_t v = pending >= 0 ? pending : producer_next<kStatic>(s, P, lane);
@@ -406,7 +434,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
                 break;
             }
             int32_t lin, bx, by;
-            lin_to_bxby(s, v, &lin, &bx, &by);
+            lin_to_bxby_warp(s, s_uwin, v, lane, &lin, &bx, &by);
             if (lane == 0) R.slot[st] = make_int4(v, lin, bx, by);
             if constexpr (MergeOf<Body>::value > 1) {
                 int n = 1;
@@ -414,7 +442,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
                     const int32_t v2 = producer_next<kStatic>(s, P, lane);
                     if (v2 >= 0) {
                         int32_t lin2, bx2, by2;
-                        lin_to_bxby(s, v2, &lin2, &bx2, &by2);
+                        lin_to_bxby_warp(s, s_uwin, v2, lane, &lin2, &bx2, &by2);
                         if (by2 == by && bx2 == bx + 1) {
                             n = 2;
                             if (lane == 0) R.slot2[st] = make_int4(v2, lin2, 2, 0);

@@ -30,7 +30,14 @@ def plan_for(kernel: str, args, order=None, tile=None, num_clusters: int = 0, de
     order = o if order is None else order
     tile = t if tile is None else tile
     if user_order is not None:
-        return cc.Plan(gx, gy, "user", num_clusters, user_order=user_order, device=device)
+        # cached per table object (hashing a large table on every launch costs
+        # more host time than the kernel); the plan copies the table when it is
+        # created, so pass a new array to change the order
+        key = (gx, gy, "user", id(user_order), num_clusters, device)
+        hit = _plans.get(key)
+        if hit is None or hit[0] is not user_order:
+            hit = _plans[key] = (user_order, cc.Plan(gx, gy, "user", num_clusters, user_order=user_order, device=device))
+        return hit[1]
     key = (gx, gy, order, tuple(tile) if order == "tile" else (1, 1), num_clusters, device)
     p = _plans.get(key)
     if p is None:
@@ -45,8 +52,8 @@ def _dev(t: torch.Tensor) -> int:
     return t.device.index or 0
 
 
-def _launch(kernel, args, backend, order, tile, num_clusters, device, stream, **kw):
-    p = plan_for(kernel, args, order, tile, num_clusters, device)
+def _launch(kernel, args, backend, order, tile, num_clusters, device, stream, user_order=None, **kw):
+    p = plan_for(kernel, args, order, tile, num_clusters, device, user_order)
     return cc.launch(p, kernel, args, cc.make_opts(backend, **kw), stream)
 
 

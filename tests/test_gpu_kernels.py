@@ -276,6 +276,52 @@ def test_conv2d_full_size_sampled():
                     assert o[i, j].item() == 0.0
 
 
+def _user_orders(gx, gy):
+    """USER-order plans (reading of the paper's user-defined partition): a
+    random permutation and the time-aligned interleaved row order."""
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    M = cc.device_info(0)["num_sms"]
+    V, c = gx * gy, 2
+    K = (V + c - 1) // c
+    ilv = np.concatenate([np.arange(k * c, min(V, (k + 1) * c)) for i in range(M) for k in range(i, K, M)])
+    rnd = np.random.default_rng(gx * 131 + gy).permutation(V)
+    return [("ilv", ilv.astype(np.int32)), ("rand", rnd.astype(np.int32))]
+
+
+@pytest.mark.parametrize("backend", ["agent", "static"])
+@pytest.mark.parametrize("rows,cols,ld", [(300, 257, 260), (100, 70, 72)])
+def test_stencils_user_order(backend, rows, cols, ld):
+    """Jacobi (bit-exact vs the fp32 oracle) and conv 3x3 / 7x7 under USER orders."""
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    u0 = mat(4, rows, cols)
+    a = padded(u0, ld).as_strided((rows, cols), (ld, 1))
+    b = torch.zeros((rows, ld), device="cuda").as_strided((rows, cols), (ld, 1))
+    args, _ = cc.jacobi5_args(a, b, 1)
+    gx, gy = cc.kernel_grid("jacobi5", args)
+    ref_j = O.jacobi5_f32(u0, 5)
+    for name, uo in _user_orders(gx, gy):
+        a.copy_(torch.from_numpy(u0).cuda())
+        out = ops.jacobi5(a, b, 5, backend=backend, user_order=uo, num_clusters=0 if backend == "agent" else 296)
+        torch.cuda.synchronize()
+        assert np.array_equal(out.cpu().numpy(), ref_j), name
+    img = mat(5, rows, cols)
+    a.copy_(torch.from_numpy(img).cuda())
+    for R in (1, 3):
+        w = synth.uniform(6, (2 * R + 1) ** 2).reshape(2 * R + 1, 2 * R + 1)
+        w = w / w.sum()
+        ref = O.conv2d(img, w)
+        args, _w = cc.conv2d_args(a, b, w)
+        gx, gy = cc.kernel_grid("conv2d", args)
+        for name, uo in _user_orders(gx, gy):
+            b.fill_(7.0)
+            ops.conv2d(a, w, out=b, backend=backend, user_order=uo, num_clusters=0 if backend == "agent" else 296)
+            torch.cuda.synchronize()
+            got = b.cpu().numpy()
+            assert np.all(got[ref == 0] == 0), (R, name)
+            nz = ref != 0
+            assert relerr(got[nz], ref[nz]) <= TOL, (R, name)
+
+
 # ---------------------------------------------------------------- SpMV
 def _csr_dev(rp, col, val):
     return ops.SpmvMatrix(dev(rp.astype(np.int32)), dev(col.astype(np.int32)), dev(val.astype(np.float32)))
