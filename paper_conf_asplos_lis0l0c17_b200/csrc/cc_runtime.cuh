@@ -285,12 +285,25 @@ __device__ __forceinline__ int32_t* q_head(const Sched& s, int32_t q) {
     return s.mode == MODE_IDENTITY ? ws_gq(s) : ws_head(s) + q;
 }
 
+// Position of slot w of queue q.  Build option CC_ALT_DIR: odd clusters are
+// drained back to front, so neighbouring clusters reach their common boundary
+// at the same time (both at the start or both at the end of the launch) and
+// the halo rows they share are re-read from L2 instead of DRAM.  Execution
+// order inside a cluster is not part of the partition (reading R9).
+#ifndef CC_ALT_DIR
+#define CC_ALT_DIR 0
+#endif
+__device__ __forceinline__ int32_t q_pos(const Sched& s, int32_t q, int32_t w) {
+    if (CC_ALT_DIR && s.mode != MODE_IDENTITY && (q & 1)) return q_start(s, q) + q_size(s, q) - 1 - w;
+    return q_start(s, q) + w;
+}
+
 // lane 0 only.  Returns an order position, or -1 with *scan = 1 when the queue
 // being drained is empty and a steal scan should follow, or -1 with *scan = 0
 // when this agent is done.
 __device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* scan) {
     *scan = 0;
-    if (P.bw < P.be) return q_start(s, P.bq) + P.bw++;
+    if (P.bw < P.be) return q_pos(s, P.bq, P.bw++);
     for (;;) {
         int32_t sq, w;
         if (P.spec) { sq = P.sq; w = P.sw; P.spec = 0; }
@@ -303,7 +316,7 @@ __device__ __forceinline__ int32_t lane0_next(const Sched& s, Prod& P, int32_t* 
             if (w + s.batch < size) {                  // claim the next batch early
                 P.sq = sq; P.sw = atom_add_relaxed(q_head(s, sq), s.batch); P.spec = 1;
             }
-            return q_start(s, sq) + w;
+            return q_pos(s, sq, w);
         }
         if (sq == P.q) {
             if (!s.steal || s.mode == MODE_IDENTITY) { P.q = -1; return -1; }
@@ -353,7 +366,7 @@ template <bool kStatic>
 __device__ __forceinline__ int32_t producer_next(const Sched& s, Prod& P, int lane) {
     if constexpr (kStatic) {                               // CTA i owns cluster i: a local cursor
         int32_t v = -1;
-        if (lane == 0 && P.q >= 0 && P.bw < cluster_size(s.g, P.q)) v = cluster_start(s.g, P.q) + P.bw++;
+        if (lane == 0 && P.q >= 0 && P.bw < cluster_size(s.g, P.q)) v = q_pos(s, P.q, P.bw++);
         return __shfl_sync(0xffffffffu, v, 0);
     }
     int32_t v = -1, scan = 0;
@@ -476,6 +489,13 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
                         if (by2 == by && bx2 == bx + 1) {
                             n = 2;
                             if (lane == 0) R.slot2[st] = make_int4(v2, lin2, 2, 0);
+                        } else if (by2 == by && bx2 == bx - 1) {       // popped right to left
+                            n = 2;
+                            if (lane == 0) {
+                                R.slot[st] = make_int4(v2, lin2, bx2, by2);
+                                R.slot2[st] = make_int4(v, lin, 2, 0);
+                            }
+                            bx = bx2;
                         } else {
                             pending = v2;                      // next slot starts with it
                         }
