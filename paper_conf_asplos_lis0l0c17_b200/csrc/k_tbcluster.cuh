@@ -30,7 +30,13 @@ namespace cc {
 
 constexpr int TBC_COLS = ST_COLS;       // staged columns per row (x0-4 .. x0+35)
 constexpr int TBC_ROW_BYTES = TBC_COLS * 4;
-constexpr int TBC_HALO = 8;             // halo box height (keeps every TMA box 128-B aligned)
+#ifndef CC_TBC_HALO
+#define CC_TBC_HALO 8
+#endif
+// halo box height: a multiple of 4 rows (4 x 160 B = 5 x 128 B) keeps every
+// TMA destination 128-B aligned; >= R
+constexpr int TBC_HALO = CC_TBC_HALO;
+static_assert(TBC_HALO % 4 == 0 && TBC_HALO >= 3, "halo box");
 constexpr int TBC_ROWS = 2 * TBC_HALO + 32;
 constexpr int TBC_BUF_BYTES = TBC_ROWS * TBC_ROW_BYTES;
 // output rows per thread: 2 for the HBM-bound 3x3 (4 warps per CTA), 4 for the
