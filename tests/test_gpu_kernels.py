@@ -443,3 +443,59 @@ def test_hist64_full_size_and_errors():
         assert np.array_equal(got.cpu().numpy().view(np.uint32).astype(np.uint64), ref), v
     with pytest.raises(Exception):
         ops.hist64(data[1:1025])                  # not 16-byte aligned
+
+
+# ---------------------------------------------------------------- degenerate sizes
+DEG_BACKENDS = [dict(backend="default"), dict(backend="agent", order="row"), dict(backend="agent", order="col"),
+                dict(backend="static", order="row"), dict(backend="identity")]
+
+
+@pytest.mark.parametrize("v", DEG_BACKENDS, ids=lambda v: "-".join(str(x) for x in v.values()))
+@pytest.mark.parametrize("m,n", [(0, 5), (5, 0), (1, 1), (1, 4), (3, 1), (0, 0)])
+def test_gemv_family_degenerate(v, m, n):
+    """Empty and one-element operands: y = A x over an empty dimension is the
+    zero vector (an empty sum), never uninitialised memory."""
+    ld = max(4, (n + 3) // 4 * 4)
+    A = mat(3, m, n)
+    Ad = padded(A, ld).as_strided((m, n), (ld, 1)) if m > 0 else torch.zeros((0, ld), device="cuda")[:, :n]
+    x, p, r = synth.uniform(10, n), synth.uniform(11, n), synth.uniform(12, m)
+    yz = ops.matvec(Ad, dev(x), **v)                              # zero-initialised y
+    q, s = ops.bicg(Ad, dev(p), dev(r), **v)
+    tmp, yy = ops.atax(Ad, dev(x), **v)
+    torch.cuda.synchronize()
+    np.testing.assert_allclose(yz.cpu().numpy(), O.matvec(A, x), rtol=TOL, atol=0)
+    rq, rs = O.bicg(A, p, r)
+    np.testing.assert_allclose(q.cpu().numpy(), rq, rtol=TOL, atol=0)
+    np.testing.assert_allclose(s.cpu().numpy(), rs, rtol=TOL, atol=0)
+    rt, ry = O.atax(A, x)
+    np.testing.assert_allclose(tmp.cpu().numpy(), rt, rtol=TOL, atol=0)
+    np.testing.assert_allclose(yy.cpu().numpy(), ry, rtol=TOL, atol=0)
+
+
+@pytest.mark.parametrize("v", DEG_BACKENDS + [dict(backend="tbcluster", cluster_size=2)],
+                         ids=lambda v: "-".join(str(x) for x in v.values()))
+@pytest.mark.parametrize("rows,cols", [(1, 1), (2, 2), (3, 3), (5, 5), (1, 40), (40, 1)])
+def test_stencils_degenerate(v, rows, cols):
+    """Grids with no interior (Jacobi keeps the boundary; conv outputs are all
+    border zeros when the image is smaller than the filter) and one-cell-wide
+    interiors."""
+    ld = max(4, (cols + 3) // 4 * 4)
+    img = mat(5, rows, cols)
+    a = padded(img, ld).as_strided((rows, cols), (ld, 1))
+    for R in (1, 3):
+        w = synth.uniform(6, (2 * R + 1) ** 2).reshape(2 * R + 1, 2 * R + 1)
+        o = torch.full((rows, ld), 7.0, device="cuda").as_strided((rows, cols), (ld, 1))
+        ops.conv2d(a, w, out=o, **v)
+        torch.cuda.synchronize()
+        ref = O.conv2d(img, w)
+        got = o.cpu().numpy()
+        assert np.all(got[ref == 0] == 0), (R, v)
+        nz = ref != 0
+        assert relerr(got[nz], ref[nz]) <= TOL, (R, v)
+    if v["backend"] == "tbcluster":
+        return
+    b = torch.full((rows, ld), 7.0, device="cuda").as_strided((rows, cols), (ld, 1))
+    a2 = padded(img, ld).as_strided((rows, cols), (ld, 1))
+    out = ops.jacobi5(a2, b, 3, **v)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), O.jacobi5_f32(img, 3)), v
