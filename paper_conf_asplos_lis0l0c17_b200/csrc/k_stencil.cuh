@@ -468,7 +468,10 @@ struct Conv2dBody {
 #ifndef CC_CONV3_MIN_AGENTS                             // 3x3 agents per SM: 4 (56 registers, no
 #define CC_CONV3_MIN_AGENTS 4                           // spill) measured 5 % faster than 5 (40 + spills)
 #endif
-    static constexpr int kMinAgents = R >= 3 ? 12 / kGroups : CC_CONV3_MIN_AGENTS;
+#ifndef CC_CONV7_MIN_AGENTS                             // 7x7 agents per SM (56 registers at 6)
+#define CC_CONV7_MIN_AGENTS (12 / CC_CONV_GROUPS)
+#endif
+    static constexpr int kMinAgents = R >= 3 ? CC_CONV7_MIN_AGENTS : CC_CONV3_MIN_AGENTS;
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
