@@ -144,6 +144,15 @@ def f2_variants(order, tile=(1, 1), l1_staging=None):
     return v
 
 
+def halo_hint_variants():
+    """Stencils: CC_L2_HINT_HALO_LAST (the rows the next tile row re-reads as its
+    top halo evict_last, the rest evict_first), alone and with the output
+    stores evict_first."""
+    return [("agent-row-l2halo", dict(backend="agent", order="row", l2_hint="halo_last")),
+            ("agent-row-l2halo-sf", dict(backend="agent", order="row", l2_hint="halo_last_stream_first")),
+            ("agent-tile8x8-l2halo", dict(backend="agent", order="tile", tile=(8, 8), l2_hint="halo_last"))]
+
+
 def static_variants(kernel, order, tile=(1, 1), ks=None):
     """CC_BACKEND_AGENT_STATIC rows: M = SMs x k clusters, CTA i runs cluster i
     (binding by construction: no %smid, queue atomics or stealing)."""
@@ -252,7 +261,7 @@ def suite_jacobi(quick):
     b = torch.empty_like(a)
     v = variants_for("tile", (8, 8), stencil=True) + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
         + static_variants("jacobi5", "row") + static_variants("jacobi5", "tile", (8, 8), ks=(4,)) + band_variants(N // 32) \
-        + ilv_variants(N // 32, N // 32)
+        + ilv_variants(N // 32, N // 32) + halo_hint_variants()
     r = measure(v, lambda kw: ops.jacobi5(a, b, T, **kw), 3, 8 * N * N * T,
                 extra=lambda ms: {"ms_per_sweep": round(ms / T, 5)}, warm=1)
     r["config"] = f"2D 5-point Jacobi fp32 {N}x{N}, {T} sweeps, 32x32 tiles (512x512 grid)"
@@ -276,7 +285,7 @@ def suite_conv(quick):
             ("tbcluster-8", dict(backend="tbcluster", cluster_size=8))] \
             + f2_variants("row") + f2_variants("tile", (8, 8), l1_staging="l1") \
             + static_variants("conv2d", "row") + static_variants("conv2d", "tile", (8, 8), ks=(4,)) + band_variants(N // 32) \
-            + ilv_variants(N // 32, N // 32)
+            + ilv_variants(N // 32, N // 32) + halo_hint_variants()
         wt = torch.from_numpy(w).cuda().view(1, 1, 2 * R + 1, 2 * R + 1)
         img4 = img.view(1, 1, N, N)
         res[f"{2 * R + 1}x{2 * R + 1}"] = measure(

@@ -135,9 +135,13 @@ typedef enum { CC_STAGING_DEFAULT = 0, CC_STAGING_TMA = 1, CC_STAGING_L1 = 2, CC
  * .L2::cache_hint).  Bits: 1 = the kernel's streamed operand is evict_first
  * (gemv: A; stencils: the output; SpMV: col/val); 2 = its reused operand is
  * evict_last (gemv: the vector slices; stencils: the TMA-staged input with
- * its halo; SpMV: x).  0 = no hint (default). */
+ * its halo; SpMV: x); 4 = stencils (Jacobi, conv) only: stage each tile as two
+ * TMA boxes, the rows the next tile row re-reads as its top halo evict_last
+ * and the rest of the input evict_first (takes precedence over bit 2 there;
+ * ignored by the other kernels).  0 = no hint (default).  One-shot backends
+ * (default, redirect) ignore every bit. */
 typedef enum { CC_L2_HINT_NONE = 0, CC_L2_HINT_STREAM_FIRST = 1, CC_L2_HINT_REUSE_LAST = 2,
-               CC_L2_HINT_BOTH = 3 } cc_l2_hint;
+               CC_L2_HINT_BOTH = 3, CC_L2_HINT_HALO_LAST = 4 } cc_l2_hint;
 
 typedef struct {
     int32_t backend;        /* cc_backend                                               */
@@ -170,7 +174,7 @@ typedef struct {
     int32_t* d_exec_sm;     /* DEVICE, |V|, optional: %smid that executed lin          */
     int32_t* d_map;         /* DEVICE, |V|, optional: d_map[v] = lin executed for the
                                slot at order position v (agent/redirect/identity)      */
-    int32_t l2_hint;        /* cc_l2_hint bits (0..3); default 0                        */
+    int32_t l2_hint;        /* cc_l2_hint bits (0..7); default 0                        */
     int32_t carveout;       /* preferred shared-memory carveout of the launched kernel,
                                percent of the SM's L1/shared array (0..100; the rest
                                is L1), set with cudaFuncAttributePreferredShared-

@@ -195,7 +195,7 @@ __device__ __forceinline__ void tma_load_2d_h(void* dst, const void* tmap, int32
                  :: "r"(smem_u32(dst)), "l"(tmap), "r"(x), "r"(y), "r"(smem_u32(bar)), "l"(pol) : "memory");
 }
 // L2 hint bits (cc_launch_opts.l2_hint)
-enum : int32_t { L2H_STREAM_FIRST = 1, L2H_REUSE_LAST = 2 };
+enum : int32_t { L2H_STREAM_FIRST = 1, L2H_REUSE_LAST = 2, L2H_HALO_LAST = 4 };
 // named barrier among the consumer warps only (the producer warp never joins)
 // (barrier 1 + g for consumer group g of N threads; groups never share one)
 template <int N>

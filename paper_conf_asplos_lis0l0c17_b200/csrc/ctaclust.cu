@@ -528,6 +528,15 @@ static cc_status make_tmap(CUtensorMap* m, const float* base, int32_t rows, int3
     return CC_OK;
 }
 
+// the four boxes of CC_L2_HINT_HALO_LAST split staging (k_stencil.cuh SplitMaps)
+static cc_status make_split(SplitMaps* m, const float* base, int32_t rows, int32_t cols, int64_t ld, int H) {
+    CC_TRY(make_tmap(&m->t, base, rows, cols, ld, ST_COLS, 32));
+    CC_TRY(make_tmap(&m->b, base, rows, cols, ld, ST_COLS, 2 * H));
+    CC_TRY(make_tmap(&m->t2, base, rows, cols, ld, ST_COLS2, 32));
+    CC_TRY(make_tmap(&m->b2, base, rows, cols, ld, ST_COLS2, 2 * H));
+    return CC_OK;
+}
+
 template <int R>
 static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     const Grid& g = c.p->g;
@@ -597,7 +606,7 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
     cc_launch_opts dflt;
     cc_launch_opts_default(&dflt);
     const cc_launch_opts* o = opts ? opts : &dflt;
-    if (o->l2_hint < 0 || o->l2_hint > 3) return fail(CC_ERR_INVALID_ARG, "l2_hint %d outside [0, 3]", o->l2_hint);
+    if (o->l2_hint < 0 || o->l2_hint > 7) return fail(CC_ERR_INVALID_ARG, "l2_hint %d outside [0, 7]", o->l2_hint);
     if (o->carveout < -1 || o->carveout > 100) return fail(CC_ERR_INVALID_ARG, "carveout %d outside [-1, 100]", o->carveout);
     if (p->device < 0) return fail(CC_ERR_NO_DEVICE, "plan was created host-only");
     int32_t gx = 0, gy = 0;
@@ -672,6 +681,7 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             if (x->rows > 0 && x->cols > 0) {
                 CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
                 CC_TRY(make_tmap(&jp.tmap2, src, x->rows, x->cols, x->ld, ST_COLS2, 34));
+                if (o->l2_hint & L2H_HALO_LAST) CC_TRY(make_split(&jp.split, src, x->rows, x->cols, x->ld, 1));
             }
             s = launch_body<Jacobi5Body>(c, jp);
             std::swap(src, dst);
@@ -700,7 +710,10 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
                 jp.h.sweep = (uint32_t)(x->sweep0 + it + 1);
                 jp.h.status = x->status;
             }
-            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
+            if (x->rows > 0 && x->cols > 0) {
+                CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
+                if (o->l2_hint & L2H_HALO_LAST) CC_TRY(make_split(&jp.split, src, x->rows, x->cols, x->ld, 1));
+            }
             s = (up || dn) ? launch_body<Jacobi5HaloBody>(c, jp) : launch_body<Jacobi5Body>(c, jp);
             std::swap(src, dst);
         }
@@ -720,6 +733,7 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             if (x->rows > 0 && x->cols > 0) {
                 CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 34));
                 CC_TRY(make_tmap(&cp.tmap2, x->in, x->rows, x->cols, x->ld, ST_COLS2, 34));
+                if (o->l2_hint & L2H_HALO_LAST) CC_TRY(make_split(&cp.split, x->in, x->rows, x->cols, x->ld, 1));
             }
             s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<1>(c, cp)
                                                    : launch_body<Conv2dBody<1>>(c, cp);
@@ -731,6 +745,7 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             if (x->rows > 0 && x->cols > 0) {
                 CC_TRY(make_tmap(&cp.tmap, x->in, x->rows, x->cols, x->ld, ST_COLS, 38));
                 CC_TRY(make_tmap(&cp.tmap2, x->in, x->rows, x->cols, x->ld, ST_COLS2, 38));
+                if (o->l2_hint & L2H_HALO_LAST) CC_TRY(make_split(&cp.split, x->in, x->rows, x->cols, x->ld, 3));
             }
             s = o->backend == CC_BACKEND_TBCLUSTER ? launch_tbc<3>(c, cp)
                                                    : launch_body<Conv2dBody<3>>(c, cp);

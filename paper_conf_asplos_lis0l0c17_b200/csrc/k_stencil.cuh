@@ -27,6 +27,15 @@ enum : int32_t { STAGE_TMA = 1, STAGE_L1 = 2, STAGE_DIRECT = 3 };
 constexpr int ST_COLS = 40;                 // staged floats per row (x0-4 .. x0+35)
 constexpr int ST_COLS2 = 72;                // merged slot: two neighbouring tiles (x0-4 .. x0+67)
 
+// Split staging for CC_L2_HINT_HALO_LAST: the tile's box as two TMA loads --
+// the first 32 rows (evict_first: nothing reads them again after this tile
+// and the tile below it) and the last 2H rows (evict_last: the next tile row
+// re-reads them as its top halo, about one tile row of the cluster later,
+// after the ROW cluster's other traffic has turned L2 over).  t / b: 40-column
+// boxes, t2 / b2: the merged 72-column boxes.  Filled by the host only when
+// the hint is requested.
+struct SplitMaps { CUtensorMap t, b, t2, b2; };
+
 template <int H>
 struct HaloTile {
     static constexpr int kRows = 32 + 2 * H;
@@ -34,24 +43,38 @@ struct HaloTile {
     static constexpr int kBytes2 = ((kRows * ST_COLS2 * 4) + 127) & ~127;   // two tiles, one box
     // warp-collective: stage the merged box of tiles (bx, by), (bx+1, by) by TMA
     __device__ __forceinline__ static void stage2(int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
-                                                  const CUtensorMap* tmap2, int32_t l2_hint) {
+                                                  const CUtensorMap* tmap2, int32_t l2_hint,
+                                                  const SplitMaps* split = nullptr) {
         stage_commit(full, lane, (uint32_t)(kRows * ST_COLS2 * 4));
         if (lane == 0) {
-            if (l2_hint & L2H_REUSE_LAST) tma_load_2d_h(dst, tmap2, x0 - 4, y0 - H, full, l2_evict_last());
-            else tma_load_2d(dst, tmap2, x0 - 4, y0 - H, full);
+            if ((l2_hint & L2H_HALO_LAST) && split) {
+                tma_load_2d(dst, &split->t2, x0 - 4, y0 - H, full);
+                tma_load_2d_h(dst + 32 * ST_COLS2 * 4, &split->b2, x0 - 4, y0 + 32 - H, full, l2_evict_last());
+            } else if (l2_hint & L2H_REUSE_LAST) {
+                tma_load_2d_h(dst, tmap2, x0 - 4, y0 - H, full, l2_evict_last());
+            } else {
+                tma_load_2d(dst, tmap2, x0 - 4, y0 - H, full);
+            }
         }
     }
     // warp-collective: stage rows y0-H.., columns x0-4.. of `src` (TMA or L1 mode).
     __device__ __forceinline__ static void stage(const float* src, int64_t ld, int32_t rows, int32_t cols,
                                                  int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
-                                                 int32_t mode, const CUtensorMap* tmap, int32_t l2_hint = 0) {
+                                                 int32_t mode, const CUtensorMap* tmap, int32_t l2_hint = 0,
+                                                 const SplitMaps* split = nullptr) {
         if (mode == STAGE_DIRECT) { stage_commit(full, lane, 0); return; }
         if (mode == STAGE_TMA) {
             stage_commit(full, lane, (uint32_t)(kRows * ST_COLS * 4));
             if (lane == 0) {
                 // the input is the reused operand (halo rows feed the next tile row)
-                if (l2_hint & L2H_REUSE_LAST) tma_load_2d_h(dst, tmap, x0 - 4, y0 - H, full, l2_evict_last());
-                else tma_load_2d(dst, tmap, x0 - 4, y0 - H, full);
+                if ((l2_hint & L2H_HALO_LAST) && split) {
+                    tma_load_2d(dst, &split->t, x0 - 4, y0 - H, full);
+                    tma_load_2d_h(dst + 32 * ST_COLS * 4, &split->b, x0 - 4, y0 + 32 - H, full, l2_evict_last());
+                } else if (l2_hint & L2H_REUSE_LAST) {
+                    tma_load_2d_h(dst, tmap, x0 - 4, y0 - H, full, l2_evict_last());
+                } else {
+                    tma_load_2d(dst, tmap, x0 - 4, y0 - H, full);
+                }
             }
             return;
         }
@@ -131,7 +154,7 @@ struct JacobiHalo {
     uint32_t sweep;           // absolute sweep number of this launch (1-based)
     int32_t* status;          // optional: 1 = a poll timed out (results invalid)
 };
-struct JacobiParams { CUtensorMap tmap; CUtensorMap tmap2; const float* a; float* b; int64_t ld; int32_t rows, cols; JacobiHalo h; };
+struct JacobiParams { CUtensorMap tmap; CUtensorMap tmap2; SplitMaps split; const float* a; float* b; int64_t ld; int32_t rows, cols; JacobiHalo h; };
 
 __device__ __forceinline__ uint64_t globaltimer() {
     uint64_t t;
@@ -272,14 +295,15 @@ struct Jacobi5BodyT {
             }
             return;
         }
-        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h);
+        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h,
+                           &p.split);
     }
 
     // merged slots (plain sweep, TMA staging): tiles (bx, by), (bx+1, by) in one box
     __device__ __forceinline__ bool can_merge(const Sched& s) const { return s.staging == STAGE_TMA; }
     __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
                                               uint64_t* full, int lane) {
-        if (n == 2) HaloTile<1>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h);
+        if (n == 2) HaloTile<1>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
         else produce(s, bx, by, stage, full, lane);
     }
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
@@ -389,7 +413,7 @@ using Jacobi5HaloBody = Jacobi5BodyT<true>;
 // The filter lives in the kernel parameter bank (constant-bank operands).
 // ---------------------------------------------------------------------------
 template <int R>
-struct ConvParams { CUtensorMap tmap; CUtensorMap tmap2; const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
+struct ConvParams { CUtensorMap tmap; CUtensorMap tmap2; SplitMaps split; const float* in; float* out; int64_t ld; int32_t rows, cols; float w[(2 * R + 1) * (2 * R + 1)]; };
 
 // Thread ctid computes RB vertically adjacent rows x 4 columns of the tile
 // (256/RB threads per tile).  Each staged input row is read once (3 LDS.128)
@@ -478,7 +502,8 @@ struct Conv2dBody {
     __device__ __forceinline__ explicit Conv2dBody(const ConvParams<R>& prm) : p(prm) {}
 
     __device__ __forceinline__ void produce(const Sched& s, int32_t bx, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
-        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h);
+        HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h,
+                           &p.split);
     }
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         if (s.staging == STAGE_DIRECT) {
@@ -505,7 +530,7 @@ struct Conv2dBody {
     __device__ __forceinline__ bool can_merge(const Sched& s) const { return s.staging == STAGE_TMA; }
     __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
                                               uint64_t* full, int lane) {
-        if (n == 2) HaloTile<R>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h);
+        if (n == 2) HaloTile<R>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
         else produce(s, bx, by, stage, full, lane);
     }
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,

@@ -209,7 +209,7 @@ def _stream(stream):
     return s.cuda_stream
 
 
-L2_HINTS = {"none": 0, "stream_first": 1, "reuse_last": 2, "both": 3}
+L2_HINTS = {"none": 0, "stream_first": 1, "reuse_last": 2, "both": 3, "halo_last": 4, "halo_last_stream_first": 5}
 
 
 def make_opts(backend="agent", active_agents=0, max_agents=0, stages=0, batch=0, staging=0, steal=1,

@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--staging", default="default")
     ap.add_argument("--cluster", type=int, default=2)
     ap.add_argument("--clusters", type=int, default=0, help="num_clusters M of the plan (static backend)")
+    ap.add_argument("--l2", default=None, help="l2_hint name (ctaclust.L2_HINTS)")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--warm", type=int, default=1)
     ap.add_argument("--scale", type=int, default=24)
@@ -43,6 +44,8 @@ def main():
         kw["cluster_size"] = a.cluster
     if a.clusters:
         kw["num_clusters"] = a.clusters
+    if a.l2:
+        kw["l2_hint"] = a.l2
     dev = "cuda"
     k = a.kernel
     if k == "matvec":

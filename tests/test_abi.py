@@ -141,7 +141,7 @@ def test_planner_user_order_and_errors():
     with pytest.raises(cc.CtaclustError) as e:                   # host-only plan cannot launch
         cc._check(cc.lib().cc_launch(p.handle, 0, ctypes.byref(cc.CensusArgs(4, 4)), None, None, None))
     assert e.value.status == -7
-    for bad in (dict(l2_hint=4), dict(l2_hint=-1), dict(carveout=101), dict(carveout=-2)):
+    for bad in (dict(l2_hint=8), dict(l2_hint=-1), dict(carveout=101), dict(carveout=-2)):
         with pytest.raises(cc.CtaclustError) as e:               # options are validated first
             cc._check(cc.lib().cc_launch(p.handle, 0, ctypes.byref(cc.CensusArgs(4, 4)),
                                          ctypes.byref(cc.make_opts(**bad)), None, None))

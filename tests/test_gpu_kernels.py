@@ -177,7 +177,9 @@ JVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(
              dict(backend="agent", order="row", staging="direct"),
              dict(backend="agent", order="row", l2_hint="both"),
              dict(backend="agent", order="row", staging="l1", l2_hint="both", carveout=25),
-             dict(backend="static", order="row", num_clusters=592), dict(backend="static", order="tile", tile=(2, 2))]
+             dict(backend="static", order="row", num_clusters=592), dict(backend="static", order="tile", tile=(2, 2)),
+             dict(backend="agent", order="row", l2_hint="halo_last"),
+             dict(backend="static", order="row", num_clusters=296, l2_hint="halo_last_stream_first")]
 
 
 @pytest.mark.parametrize("v", JVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
@@ -224,7 +226,10 @@ CVARIANTS = [dict(backend="default"), dict(backend="agent", order="tile", tile=(
              dict(backend="agent", order="tile", tile=(8, 8), staging="l1"),
              dict(backend="agent", order="col", staging="direct"),
              dict(backend="agent", order="row", l2_hint="both", carveout=100),
-             dict(backend="static", order="row", num_clusters=740), dict(backend="static", order="col", staging="direct")]
+             dict(backend="static", order="row", num_clusters=740), dict(backend="static", order="col", staging="direct"),
+             dict(backend="agent", order="row", l2_hint="halo_last"),
+             dict(backend="agent", order="tile", tile=(4, 4), l2_hint="halo_last_stream_first"),
+             dict(backend="static", order="row", num_clusters=296, l2_hint="halo_last")]
 
 
 @pytest.mark.parametrize("v", CVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
