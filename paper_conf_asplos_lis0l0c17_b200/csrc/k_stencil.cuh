@@ -521,9 +521,20 @@ struct Conv2dBody {
             consumer_sync<kConsumers>();
             // (no trailing barrier: the slot is reused only after every warp of the
             // group has released it)
-            conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid, l2h);
-            return;
+#ifndef CC_CONV_DUAL_BODY
+#define CC_CONV_DUAL_BODY (R < 3)
+#endif
+            if constexpr (CC_CONV_DUAL_BODY) {
+                conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid, l2h);
+                return;
+            }
         }
+        // 7x7: one instance of the tile code for both staging paths (the direct
+        // path staged into this same slot).  Two unrolled copies are 2 x 784
+        // FFMA of instruction footprint; the single copy makes every 7x7 agent
+        // 3.5 % faster (agent ROW 0.1635 -> 0.1577 ms, same box A/B,
+        // profiles/r07/diag/suite_convbody_*).  The 3x3 keeps two copies (its
+        // identity order measured 1.8 % slower with one).
         conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid, l2h);
     }
     // merged slots (TMA staging): tiles (bx, by), (bx+1, by) from one box
