@@ -476,7 +476,10 @@ struct Conv2dBody {
     // two neighbouring tiles per slot for the HBM-bound 3x3 (cc_runtime.cuh:
     // MergeOf); the FP32-bound 7x7 gains nothing from the shared halo and
     // measured 1-2 % slower merged
-    static constexpr int kMerge = R >= 3 ? 1 : 2;
+#ifndef CC_CONV7_MERGE
+#define CC_CONV7_MERGE 1
+#endif
+    static constexpr int kMerge = R >= 3 ? CC_CONV7_MERGE : 2;
     static constexpr int kStageBytes = kMerge > 1 ? HaloTile<R>::kBytes2 : HaloTile<R>::kBytes;
     static constexpr int kDirectStageBytes = HaloTile<R>::kBytes;  // the direct path stages into its own slot
     // Two consumer groups per agent (alternate tiles).  One scheduler warp per
@@ -505,27 +508,31 @@ struct Conv2dBody {
         HaloTile<R>::stage(p.in, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h,
                            &p.split);
     }
-    __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
-        if (s.staging == STAGE_DIRECT) {
-            // plain-kernel form: the consumers stage the tile themselves through L1,
-            // into this task's ring slot (the group owns it until it releases it)
-            auto& s_in = *reinterpret_cast<float4 (*)[HaloTile<R>::kRows][ST_COLS / 4]>(const_cast<uint8_t*>(stage));
-            const int x0 = bx * 32, y0 = by * 32;
-            for (int idx = ctid; idx < HaloTile<R>::kRows * 10; idx += kConsumers) {
-                const int rr = idx / 10, cc = idx - rr * 10;
-                const int gy = y0 - R + rr, gx = x0 - 4 + 4 * cc;
-                float4 v = f4_zero();
-                if (gy >= 0 && gy < p.rows && gx >= 0 && gx < p.cols) v = ld_cached4(p.in + (int64_t)gy * p.ld + gx);
-                s_in[rr][cc] = v;
-            }
-            consumer_sync<kConsumers>();
-            // (no trailing barrier: the slot is reused only after every warp of the
-            // group has released it)
+    // plain-kernel form of the staging: the consumers stage the tile themselves
+    // through L1, into this task's ring slot (the group owns it until it
+    // releases it)
+    __device__ __forceinline__ void direct_stage(int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        auto& s_in = *reinterpret_cast<float4 (*)[HaloTile<R>::kRows][ST_COLS / 4]>(const_cast<uint8_t*>(stage));
+        const int x0 = bx * 32, y0 = by * 32;
+        for (int idx = ctid; idx < HaloTile<R>::kRows * 10; idx += kConsumers) {
+            const int rr = idx / 10, cc = idx - rr * 10;
+            const int gy = y0 - R + rr, gx = x0 - 4 + 4 * cc;
+            float4 v = f4_zero();
+            if (gy >= 0 && gy < p.rows && gx >= 0 && gx < p.cols) v = ld_cached4(p.in + (int64_t)gy * p.ld + gx);
+            s_in[rr][cc] = v;
+        }
+        consumer_sync<kConsumers>();
+        // (no trailing barrier: the slot is reused only after every warp of the
+        // group has released it)
+    }
 #ifndef CC_CONV_DUAL_BODY
 #define CC_CONV_DUAL_BODY (R < 3)
 #endif
+    __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        if (s.staging == STAGE_DIRECT) {
+            direct_stage(bx, by, stage, ctid);
             if constexpr (CC_CONV_DUAL_BODY) {
-                conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(&s_in[0][0]), bx, by, ctid, l2h);
+                conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid, l2h);
                 return;
             }
         }
@@ -546,7 +553,15 @@ struct Conv2dBody {
     }
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
                                               int ctid) {
-        if (n == 2) {
+        if constexpr (R >= 3) {
+            // 7x7 merged: a single instance of the tile code for one or two tiles
+            // and either pitch (instruction footprint, see consume)
+            if (n != 2 && s.staging == STAGE_DIRECT) direct_stage(bx, by, stage, ctid);
+            const float* b = reinterpret_cast<const float*>(stage);
+            const int pitch = n == 2 ? ST_COLS2 : ST_COLS;
+#pragma unroll 1
+            for (int k = 0; k < n; ++k) conv_tile_compute<R, RB>(p, b + 32 * k, bx + k, by, ctid, l2h, pitch);
+        } else if (n == 2) {
             // one instance of the tile code, run twice (two unrolled copies would
             // not fit the register budget of the resident agents)
             const float* b = reinterpret_cast<const float*>(stage);
