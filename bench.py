@@ -193,9 +193,13 @@ def main():
     x, p, y1 = col(10), col(11), col(15)
     r, x1_0, y2 = row(12), row(13), row(16)
     x2_0 = col(14)
-    tmp, y = torch.empty(m, device=dev), torch.empty(n, device=dev)
-    q, s = torch.empty(m, device=dev), torch.empty(n, device=dev)
-    x1, x2 = x1_0.clone(), x2_0.clone() if rank == 0 else torch.zeros(n, device=dev)
+    # the three column-indexed (transposed-product) outputs live in one buffer
+    # so that N > 1 sums them over the ranks with a single all-reduce per step
+    tsum = torch.empty(3 * n, device=dev)
+    y, s, x2 = tsum[:n], tsum[n:2 * n], tsum[2 * n:]
+    tmp, q = torch.empty(m, device=dev), torch.empty(m, device=dev)
+    x1 = x1_0.clone()
+    x2.copy_(x2_0 if rank == 0 else torch.zeros(n, device=dev))
     torch.cuda.synchronize()
 
     def run_step(backend, order, ev=None, count=None, staging=None):
@@ -210,9 +214,8 @@ def main():
         if ev is not None: ev[2].record(stream)
         nl += cc.launch(pl, "mvt", cc.mvt_args(A, y1, y2, x1, x2), cc.make_opts(**kw), stream)
         if ev is not None: ev[3].record(stream)
-        if world > 1:
-            for t_ in (y, s, x2):                    # transposed products: one sum over ranks
-                comm.allreduce_sum(t_, stream)
+        if world > 1:                                # transposed products: one sum over ranks
+            comm.allreduce_sum(tsum, stream)
         if count is not None:
             count[0] += nl
 
