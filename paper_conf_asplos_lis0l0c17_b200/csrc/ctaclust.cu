@@ -131,7 +131,44 @@ struct cc_plan_s {
     int32_t* d_user = nullptr;
     int32_t* d_ws = nullptr;
     DevFacts* facts = nullptr;
+    // workspace ownership: the stream of the last agent launch that used d_ws
+    // and an event recorded after it (outside graph capture)
+    std::mutex ws_mu;
+    cudaStream_t ws_stream = nullptr;
+    cudaEvent_t ws_done = nullptr;
+    bool ws_pending = false;
 };
+
+// The agent backends share the plan's self-resetting workspace (queue heads,
+// agent and claim counters).  Two launches in flight at once on different
+// streams would interleave their queue atomics and break exactly-once
+// coverage, so such a launch is refused (CC_ERR_BUSY) while the previous one
+// on another stream has not finished.  Same-stream launches are ordered by
+// the stream; launches being captured into a CUDA graph are the caller's to
+// order (no query is legal during capture).
+static cc_status ws_acquire(cc_plan_s* p, cudaStream_t st, bool* record) {
+    *record = false;
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    CC_CUDA(cudaStreamIsCapturing(st, &cs));
+    if (cs != cudaStreamCaptureStatusNone) return CC_OK;
+    std::lock_guard<std::mutex> lk(p->ws_mu);
+    if (p->ws_pending && p->ws_stream != st) {
+        cudaError_t q = cudaEventQuery(p->ws_done);
+        if (q == cudaErrorNotReady)
+            return fail(CC_ERR_BUSY, "plan workspace in use by an unfinished launch on another stream");
+        if (q != cudaSuccess) return cuda_fail(q, "workspace event");
+    }
+    *record = true;
+    return CC_OK;
+}
+static cc_status ws_release(cc_plan_s* p, cudaStream_t st) {
+    std::lock_guard<std::mutex> lk(p->ws_mu);
+    if (!p->ws_done) CC_CUDA(cudaEventCreateWithFlags(&p->ws_done, cudaEventDisableTiming));
+    CC_CUDA(cudaEventRecord(p->ws_done, st));
+    p->ws_stream = st;
+    p->ws_pending = true;
+    return CC_OK;
+}
 
 extern "C" cc_status cc_plan_create(const cc_plan_desc* d, cc_plan* out) {
     if (!d || !out) return fail(CC_ERR_INVALID_ARG, "null argument");
@@ -201,6 +238,7 @@ extern "C" cc_status cc_plan_destroy(cc_plan p) {
     if (!p) return CC_OK;
     if (p->d_ws) cudaFree(p->d_ws);
     if (p->d_user) cudaFree(p->d_user);
+    if (p->ws_done) cudaEventDestroy(p->ws_done);
     delete p;
     return CC_OK;
 }
@@ -475,7 +513,10 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
         s.stages = S;
         const int grid = c.p->facts->num_sms * maxa;
+        bool rec = false;
+        CC_TRY(ws_acquire(c.p, c.st, &rec));
         k_agent<Body><<<grid, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
+        if (cudaPeekAtLastError() == cudaSuccess && rec) CC_TRY(ws_release(c.p, c.st));
         break;
     }
     case CC_BACKEND_AGENT_STATIC: {
@@ -870,6 +911,7 @@ extern "C" const char* cc_status_string(cc_status s) {
     case CC_ERR_NCCL: return "NCCL error";
     case CC_ERR_UNSUPPORTED: return "unsupported";
     case CC_ERR_NO_DEVICE: return "plan has no device";
+    case CC_ERR_BUSY: return "plan workspace busy on another stream";
     }
     return "unknown status";
 }

@@ -28,7 +28,8 @@ STAGINGS = {"default": 0, "tma": 1, "l1": 2, "direct": 3}
 KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7,
            "hist64": 8, "jacobi5_halo": 9}
 STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_ERR_NOT_PERMUTATION",
-          -4: "CC_ERR_CUDA", -5: "CC_ERR_NCCL", -6: "CC_ERR_UNSUPPORTED", -7: "CC_ERR_NO_DEVICE"}
+          -4: "CC_ERR_CUDA", -5: "CC_ERR_NCCL", -6: "CC_ERR_UNSUPPORTED", -7: "CC_ERR_NO_DEVICE",
+          -8: "CC_ERR_BUSY"}
 
 # every symbol include/ctaclust.h declares (checked by tests/test_abi.py)
 EXPORTS = ["cc_plan_create", "cc_plan_destroy", "cc_plan_info", "cc_plan_table", "cc_plan_lookup",

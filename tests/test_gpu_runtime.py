@@ -129,3 +129,28 @@ def test_user_order():
     torch.cuda.synchronize()
     assert torch.all(cen == 1)
     assert np.array_equal(mp.cpu().numpy(), u)
+
+
+def test_workspace_busy_across_streams():
+    """Agent launches sharing a plan's self-resetting workspace must be
+    stream-ordered: a launch on another stream while the previous one is
+    still running is refused with CC_ERR_BUSY (-8), and goes through once the
+    first stream has finished.  Graph-captured launches are not checked."""
+    N = 16384
+    a = torch.rand(N, N, device="cuda")
+    b = torch.empty_like(a)
+    a2, b2 = torch.rand(N, N, device="cuda"), torch.empty_like(a)
+    sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+    torch.cuda.synchronize()
+    ops.jacobi5(a, b, 20, backend="agent", order="row", stream=sa)       # ~7 ms of sweeps on sa
+    with pytest.raises(cc.CtaclustError) as e:
+        ops.jacobi5(a2, b2, 1, backend="agent", order="row", stream=sb)
+    assert e.value.status == -8
+    ops.jacobi5(a2, b2, 1, backend="agent", order="row", stream=sa)      # same stream: ordered, fine
+    sa.synchronize()
+    ops.jacobi5(a2, b2, 1, backend="agent", order="row", stream=sb)      # finished: fine
+    ops.jacobi5(a2, b2, 1, backend="static", order="row", stream=sa)     # static: no workspace
+    torch.cuda.synchronize()
+    cen, *_ = ops.census(512, 512, "agent", "row")
+    torch.cuda.synchronize()
+    assert bool(torch.all(cen == 1))
