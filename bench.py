@@ -149,7 +149,8 @@ def run_reference(a):
             "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(1e3 * dt / a.steps, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (counter-hash U[0,1), seed 3)",
-            "config": {"workload": f"ATAX+BICG+MVT fp32 n={a.n} (config 2)", "sample": f"rows 0..{rows - 1}"},
+            "config": {"workload": f"ATAX+BICG+MVT fp32 n={a.n} (BASELINE config 2)",
+                       "sample": f"rows 0..{rows - 1} per step (oracle, fp64, one host thread)"},
             "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
                              "sample": f"ATAX+BICG+MVT on rows 0..{rows - 1} of the {a.n}x{a.n} matrix, per step"},
             "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
