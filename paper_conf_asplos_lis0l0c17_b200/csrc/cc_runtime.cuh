@@ -454,6 +454,7 @@ struct RingShared {
     uint64_t empty[MAX_STAGES];
     int4 slot[MAX_STAGES];       // (v, lin, bx, by) decoded once by the scheduler warp
     int4 slot2[MAX_STAGES];      // merged slots: (v, lin) of the second CTA, and n
+    int4 slot3[MAX_STAGES];      // merged slots of 3-4 CTAs: (v, lin) of the third and fourth
 };
 
 __device__ __forceinline__ uint8_t* ring_base(uint8_t* dyn) {
@@ -528,7 +529,22 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
                         lin_to_bxby_warp(s, s_uwin, v2, lane, &lin2, &bx2, &by2);
                         if (by2 == by && bx2 == bx + 1) {
                             n = 2;
-                            if (lane == 0) R.slot2[st] = make_int4(v2, lin2, 2, 0);
+                            if constexpr (MergeOf<Body>::value > 2) {
+                                // longer runs (left to right): up to 4 tiles per slot
+                                int4 x34 = make_int4(-1, 0, -1, 0);
+#pragma unroll 1
+                                for (int k = 2; k < MergeOf<Body>::value; ++k) {
+                                    const int32_t vk = producer_next<kStatic>(s, P, lane);
+                                    if (vk < 0) break;
+                                    int32_t link, bxk, byk;
+                                    lin_to_bxby_warp(s, s_uwin, vk, lane, &link, &bxk, &byk);
+                                    if (byk != by || bxk != bx + k) { pending = vk; break; }
+                                    if (k == 2) { x34.x = vk; x34.y = link; } else { x34.z = vk; x34.w = link; }
+                                    n = k + 1;
+                                }
+                                if (lane == 0) R.slot3[st] = x34;
+                            }
+                            if (lane == 0) R.slot2[st] = make_int4(v2, lin2, n, 0);
                         } else if (by2 == by && bx2 == bx - 1) {       // popped right to left
                             n = 2;
                             if (lane == 0) {
@@ -585,6 +601,9 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
                 if (ctid == 0) {
                     record(s, sl.x, sl.y);
                     if (s2.z > 1) record(s, s2.x, s2.y);
+                    if constexpr (MergeOf<Body>::value > 2) {
+                        if (s2.z > 2) { const int4 s3 = R.slot3[st]; record(s, s3.x, s3.y); if (s2.z > 3) record(s, s3.z, s3.w); }
+                    }
                 }
             } else {
                 body.consume(s, sl.z, sl.w, ring + (size_t)st * s.stage_bytes, ctid);

@@ -25,7 +25,14 @@ namespace cc {
 
 enum : int32_t { STAGE_TMA = 1, STAGE_L1 = 2, STAGE_DIRECT = 3 };
 constexpr int ST_COLS = 40;                 // staged floats per row (x0-4 .. x0+35)
-constexpr int ST_COLS2 = 72;                // merged slot: two neighbouring tiles (x0-4 .. x0+67)
+// Merged slots: up to ST_MERGE horizontally adjacent tiles of a cluster in one
+// TMA box (x0-4 .. x0+32*ST_MERGE+3).  Build option CC_STENCIL_MERGE (2 or 4).
+#ifndef CC_STENCIL_MERGE
+#define CC_STENCIL_MERGE 2
+#endif
+constexpr int ST_MERGE = CC_STENCIL_MERGE;
+static_assert(ST_MERGE == 2 || ST_MERGE == 4, "merged tiles per slot");
+constexpr int ST_COLS2 = 32 * ST_MERGE + 8;  // merged slot width in floats (72 for two tiles)
 
 // Split staging for CC_L2_HINT_HALO_LAST: the tile's box as two TMA loads --
 // the first 32 rows (evict_first: nothing reads them again after this tile
@@ -40,7 +47,7 @@ template <int H>
 struct HaloTile {
     static constexpr int kRows = 32 + 2 * H;
     static constexpr int kBytes = ((kRows * ST_COLS * 4) + 127) & ~127;
-    static constexpr int kBytes2 = ((kRows * ST_COLS2 * 4) + 127) & ~127;   // two tiles, one box
+    static constexpr int kBytes2 = ((kRows * ST_COLS2 * 4) + 127) & ~127;   // merged tiles, one box
     // warp-collective: stage the merged box of tiles (bx, by), (bx+1, by) by TMA
     __device__ __forceinline__ static void stage2(int32_t x0, int32_t y0, uint8_t* dst, uint64_t* full, int lane,
                                                   const CUtensorMap* tmap2, int32_t l2_hint,
@@ -251,7 +258,7 @@ template <bool HALO>
 struct Jacobi5BodyT {
     static constexpr int RB = 2;                  // output rows per consumer thread
     static constexpr int kConsumers = 256 / RB;
-    static constexpr int kMerge = HALO ? 1 : 2;    // two neighbouring tiles per slot (cc_runtime.cuh: MergeOf)
+    static constexpr int kMerge = HALO ? 1 : ST_MERGE;   // neighbouring tiles per slot (cc_runtime.cuh: MergeOf)
     static constexpr int kTileBytes = HALO ? HaloTile<1>::kBytes : HaloTile<1>::kBytes2;
     static constexpr int kStageBytes = kTileBytes + (HALO ? 2 * 32 * 8 : 0);   // + the two LL halo rows (words)
     static constexpr int kDefaultStages = 4;
@@ -303,14 +310,19 @@ struct Jacobi5BodyT {
     __device__ __forceinline__ bool can_merge(const Sched& s) const { return s.staging == STAGE_TMA; }
     __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
                                               uint64_t* full, int lane) {
-        if (n == 2) HaloTile<1>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
+        if (n >= 2) HaloTile<1>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
         else produce(s, bx, by, stage, full, lane);
     }
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
                                               int ctid) {
-        if (n == 2) {
-            consume_at(s, bx, by, stage, ctid, ST_COLS2, 0);
-            consume_at(s, bx + 1, by, stage, ctid, ST_COLS2, 32);
+        if (n >= 2) {
+            if constexpr (ST_MERGE == 2) {
+                consume_at(s, bx, by, stage, ctid, ST_COLS2, 0);
+                consume_at(s, bx + 1, by, stage, ctid, ST_COLS2, 32);
+            } else {
+#pragma unroll 1
+                for (int k = 0; k < n; ++k) consume_at(s, bx + k, by, stage, ctid, ST_COLS2, 32 * k);
+            }
         } else {
             consume_at(s, bx, by, stage, ctid, ST_COLS, 0);
         }
@@ -479,7 +491,7 @@ struct Conv2dBody {
 #ifndef CC_CONV7_MERGE
 #define CC_CONV7_MERGE 1
 #endif
-    static constexpr int kMerge = R >= 3 ? CC_CONV7_MERGE : 2;
+    static constexpr int kMerge = R >= 3 ? CC_CONV7_MERGE : ST_MERGE;
     static constexpr int kStageBytes = kMerge > 1 ? HaloTile<R>::kBytes2 : HaloTile<R>::kBytes;
     static constexpr int kDirectStageBytes = HaloTile<R>::kBytes;  // the direct path stages into its own slot
     // Two consumer groups per agent (alternate tiles).  One scheduler warp per
@@ -548,7 +560,7 @@ struct Conv2dBody {
     __device__ __forceinline__ bool can_merge(const Sched& s) const { return s.staging == STAGE_TMA; }
     __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
                                               uint64_t* full, int lane) {
-        if (n == 2) HaloTile<R>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
+        if (n >= 2) HaloTile<R>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
         else produce(s, bx, by, stage, full, lane);
     }
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
@@ -556,17 +568,17 @@ struct Conv2dBody {
         if constexpr (R >= 3) {
             // 7x7 merged: a single instance of the tile code for one or two tiles
             // and either pitch (instruction footprint, see consume)
-            if (n != 2 && s.staging == STAGE_DIRECT) direct_stage(bx, by, stage, ctid);
+            if (n < 2 && s.staging == STAGE_DIRECT) direct_stage(bx, by, stage, ctid);
             const float* b = reinterpret_cast<const float*>(stage);
-            const int pitch = n == 2 ? ST_COLS2 : ST_COLS;
+            const int pitch = n >= 2 ? ST_COLS2 : ST_COLS;
 #pragma unroll 1
             for (int k = 0; k < n; ++k) conv_tile_compute<R, RB>(p, b + 32 * k, bx + k, by, ctid, l2h, pitch);
-        } else if (n == 2) {
-            // one instance of the tile code, run twice (two unrolled copies would
+        } else if (n >= 2) {
+            // one instance of the tile code, run n times (two unrolled copies would
             // not fit the register budget of the resident agents)
             const float* b = reinterpret_cast<const float*>(stage);
 #pragma unroll 1
-            for (int k = 0; k < 2; ++k) conv_tile_compute<R, RB>(p, b + 32 * k, bx + k, by, ctid, l2h, ST_COLS2);
+            for (int k = 0; k < n; ++k) conv_tile_compute<R, RB>(p, b + 32 * k, bx + k, by, ctid, l2h, ST_COLS2);
         } else {
             consume(s, bx, by, stage, ctid);
         }
