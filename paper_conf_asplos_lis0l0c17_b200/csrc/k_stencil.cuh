@@ -464,6 +464,24 @@ __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const 
         }
     }
     if (gx >= p.cols) return;
+#ifndef CC_CONV_INTERIOR_FAST
+#define CC_CONV_INTERIOR_FAST 1
+#endif
+    if (CC_CONV_INTERIOR_FAST) {
+        // interior thread block of outputs (every output of its RB x 4 block
+        // has a full window): plain float4 stores, no per-element masks
+        const int gy0 = by * 32 + r0;
+        if (gx >= R && gx + 4 <= p.cols - R && gy0 >= R && gy0 + RB <= p.rows - R) {
+#pragma unroll
+            for (int j = 0; j < RB; ++j) {
+                float* dst = p.out + (int64_t)(gy0 + j) * p.ld + gx;
+                const float4 o = make_float4(acc[j][0], acc[j][1], acc[j][2], acc[j][3]);
+                if (l2_hint & L2H_STREAM_FIRST) st4_h(dst, o, l2_evict_first());
+                else *reinterpret_cast<float4*>(dst) = o;
+            }
+            return;
+        }
+    }
 #pragma unroll
     for (int j = 0; j < RB; ++j) {
         const int gy = by * 32 + r0 + j;
