@@ -236,13 +236,17 @@ __device__ __forceinline__ float4 ll_take4(const uint64_t* staged, const uint64_
     return ll_load4(src, tag, valid, status);
 }
 
-__device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, float lw, float re,
-                                               int gy, int gx, int rows, int cols) {
+__device__ __forceinline__ float4 jacobi_core4(float4 c, float4 up, float4 dn, float lw, float re) {
     float4 o;
     o.x = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.x, lw), c.y), up.x), dn.x));
     o.y = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.y, c.x), c.z), up.y), dn.y));
     o.z = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.z, c.y), c.w), up.z), dn.z));
     o.w = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.w, c.z), re), up.w), dn.w));
+    return o;
+}
+__device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, float lw, float re,
+                                               int gy, int gx, int rows, int cols) {
+    float4 o = jacobi_core4(c, up, dn, lw, re);
     const bool row_bd = (gy == 0) || (gy == rows - 1);
     const int cl = cols - 1;
     if (row_bd || gx == 0 || gx == cl) o.x = c.x;
@@ -402,6 +406,20 @@ struct Jacobi5BodyT {
                 if (top && gy == 1) ll_store4(p.h.up_ll + opar + p.h.ldl + gx, o, sw, valid);
                 if (bot && gy == p.rows - 2) ll_store4(p.h.dn_ll + opar + gx, o, sw, valid);
 #endif
+            }
+            return;
+        }
+#ifndef CC_JACOBI_INTERIOR_FAST
+#define CC_JACOBI_INTERIOR_FAST 1
+#endif
+        if (CC_JACOBI_INTERIOR_FAST && gx >= 1 && gx + 4 <= p.cols - 1 && gy0 >= 1 && gy0 + RB <= p.rows - 1) {
+            // interior block: no boundary cells, plain float4 stores (same arithmetic)
+#pragma unroll
+            for (int j = 0; j < RB; ++j) {
+                float* dst = p.b + (int64_t)(gy0 + j) * p.ld + gx;
+                const float4 o = jacobi_core4(row[j + 1], row[j], row[j + 2], lw[j], re[j]);
+                if (l2h & L2H_STREAM_FIRST) st4_h(dst, o, l2_evict_first());
+                else *reinterpret_cast<float4*>(dst) = o;
             }
             return;
         }
