@@ -20,7 +20,18 @@ DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": (
                  "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1)),
                  "jacobi5_halo": ("row", (1, 1))}
 
+# Plans are cached for the life of the process and never evicted: a plan may
+# only be destroyed once every stream that used it has synchronized
+# (cc_plan_destroy), which a cache cannot know.  Call release_plans() after a
+# device-wide synchronize to drop them.
 _plans: dict = {}
+
+
+def release_plans() -> None:
+    """Synchronize the device and drop every cached plan (frees their device
+    tables and workspaces)."""
+    torch.cuda.synchronize()
+    _plans.clear()
 
 
 def plan_for(kernel: str, args, order=None, tile=None, num_clusters: int = 0, device: int = 0,
