@@ -130,10 +130,12 @@ void oracle_jacobi5(int64_t rows, int64_t cols, const float* u0, int iters,
     for (int64_t k = 0; k < rows * cols; ++k) out[k] = a[k];
 }
 
-/* fp32 variant of one sweep with the exact fp32 expression the paper's
- * PolyBench form uses, 0.2f*(c+w+e+n+s) summed left to right.  Used only for
- * the integer-exact / rounding-order pins of the GPU sweep (tests decide
- * which one they compare against). */
+/* fp32 variant: the PolyBench jacobi-2d statement (reading R14) evaluated in
+ * fp32 exactly as C evaluates it, left to right with no contraction:
+ *     B[i][j] = 0.2f * (A[i][j] + A[i][j-1] + A[i][1+j] + A[1+i][j] + A[i-1][j])
+ * i.e. centre, west, east, south (row i+1), north (row i-1).  This is the
+ * sum order the GPU sweep reproduces bit for bit; pinned by the fp64 oracle
+ * and by an order-sensitive by-hand case (tests/test_oracle_kernels.py). */
 void oracle_jacobi5_f32(int64_t rows, int64_t cols, const float* u0, int iters,
                         float* out, float* work)
 {
@@ -144,8 +146,8 @@ void oracle_jacobi5_f32(int64_t rows, int64_t cols, const float* u0, int iters,
         for (int64_t i = 1; i + 1 < rows; ++i)
             for (int64_t j = 1; j + 1 < cols; ++j) {
                 float c = a[i * cols + j], w = a[i * cols + j - 1], e = a[i * cols + j + 1];
-                float n = a[(i - 1) * cols + j], s = a[(i + 1) * cols + j];
-                b[i * cols + j] = 0.2f * ((((c + w) + e) + n) + s);
+                float s = a[(i + 1) * cols + j], n = a[(i - 1) * cols + j];
+                b[i * cols + j] = 0.2f * ((((c + w) + e) + s) + n);
             }
         float* sw = a; a = b; b = sw;
     }

@@ -125,7 +125,7 @@ __device__ __forceinline__ void store4_out(float* dst, float4 o, int gx, int col
 
 // ---------------------------------------------------------------------------
 // Jacobi 5-point sweep (reading R14, PolyBench jacobi-2d form):
-//   b[i][j] = 0.2f * ((((c + w) + e) + n) + s)     on the interior,
+//   b[i][j] = 0.2f * ((((c + w) + e) + s) + n)     on the interior (s = row i+1, n = row i-1),
 //   b[i][j] = a[i][j]                               on the boundary.
 // fp32, summed in that fixed order with no contraction, so the sweep is
 // bit-reproducible against oracle_jacobi5_f32 in every staging mode.
@@ -236,12 +236,13 @@ __device__ __forceinline__ float4 ll_take4(const uint64_t* staged, const uint64_
     return ll_load4(src, tag, valid, status);
 }
 
+// PolyBench order: centre, west, east, south (row i+1 = dn), north (row i-1 = up)
 __device__ __forceinline__ float4 jacobi_core4(float4 c, float4 up, float4 dn, float lw, float re) {
     float4 o;
-    o.x = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.x, lw), c.y), up.x), dn.x));
-    o.y = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.y, c.x), c.z), up.y), dn.y));
-    o.z = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.z, c.y), c.w), up.z), dn.z));
-    o.w = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.w, c.z), re), up.w), dn.w));
+    o.x = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.x, lw), c.y), dn.x), up.x));
+    o.y = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.y, c.x), c.z), dn.y), up.y));
+    o.z = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.z, c.y), c.w), dn.z), up.z));
+    o.w = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(c.w, c.z), re), dn.w), up.w));
     return o;
 }
 __device__ __forceinline__ float4 jacobi_point4(float4 c, float4 up, float4 dn, float lw, float re,

@@ -74,8 +74,6 @@ def test_integer_exact_mode_is_exact():
 def test_jacobi_constant_is_fixed_point():
     u = np.full((9, 13), 3.25, np.float32)
     assert np.allclose(O.jacobi5(u, 7), 3.25, rtol=0, atol=1e-12)
-    for c in (1.0, 0.5, 2.0, 0.25):                        # fp32 sweep: 0.2f*5c rounds to c
-        assert np.array_equal(O.jacobi5_f32(np.full((6, 7), c, np.float32), 3), np.full((6, 7), c, np.float32))
 
 
 def test_jacobi_linear_field_is_harmonic():
@@ -97,6 +95,64 @@ def test_jacobi_eigenmode_closed_form(p, q, t):
     got = O.jacobi5(u, t)
     # the fp32-rounded start is an eigenvector up to 6e-8 relative
     assert np.allclose(got, lam ** t * u64, rtol=0, atol=2e-7)
+
+
+# ---- fp32 Jacobi (the bit-exact reference of the GPU sweep) ----
+# Pins written as functions of the routine under test so that
+# tests/test_oracle_mutants.py can run them against deliberately broken
+# builds of oracle.c and show that each plausible mistake fails one of them.
+def pin_jacobi_f32_tracks_fp64(f32):
+    """fp32 sweeps stay within a few ulp of the fp64 definition on U[0,1)
+    fields (no cancellation: every term is positive).  A dropped, duplicated
+    or mis-indexed neighbour moves results by ~20 %, far above 1e-6."""
+    for it in (1, 3, 7):
+        u = rnd(31, 37, 53)
+        ref = O.jacobi5(u, it)
+        got = f32(u, it).astype(np.float64)
+        assert np.max(np.abs(got - ref) / np.abs(ref)) <= 1e-6, it
+
+
+def pin_jacobi_f32_eigenmode(f32):
+    """The separable sine mode decays by its closed-form eigenvalue in fp32 too."""
+    R, C = 13, 21
+    i, j = np.meshgrid(np.arange(R), np.arange(C), indexing="ij")
+    for p, q, t in ((1, 1, 1), (2, 3, 5), (3, 1, 20)):
+        u64 = np.sin(np.pi * p * i / (R - 1)) * np.sin(np.pi * q * j / (C - 1))
+        lam = 0.2 * (1 + 2 * np.cos(np.pi * p / (R - 1)) + 2 * np.cos(np.pi * q / (C - 1)))
+        assert np.max(np.abs(f32(u64.astype(np.float32), t) - lam ** t * u64)) <= 5e-7, (p, q, t)
+
+
+def pin_jacobi_f32_by_hand(f32):
+    """3x3 grids: only the centre moves.  (a) arange: 0.2f*(4+3+5+7+1) = 0.2f*20
+    rounds to 4.0.  (b) the PolyBench sum order, by hand: with c = 2^24,
+    w = e = n = 1 and s = -2^24, ((((c+w)+e)+s)+n) in fp32 is
+    2^24 -> 2^24 (ties to even) -> 0 -> 1, so the centre becomes 0.2f; adding
+    n before s would give 0, the exact sum 3 would give 0.6."""
+    u = np.arange(9, dtype=np.float32).reshape(3, 3)
+    want = u.copy()
+    want[1, 1] = 4.0
+    assert np.array_equal(f32(u, 1), want)
+    v = np.zeros((3, 3), np.float32)
+    v[1, 1], v[1, 0], v[1, 2], v[2, 1], v[0, 1] = 2.0 ** 24, 1, 1, -(2.0 ** 24), 1
+    got = f32(v, 1)
+    assert got[1, 1] == np.float32(0.2)
+    want = v.copy()
+    want[1, 1] = np.float32(0.2)
+    assert np.array_equal(got, want)
+
+
+def pin_jacobi_f32_fixed_points(f32):
+    for c in (1.0, 0.5, 2.0, 0.25):                       # 0.2f*5c rounds to c
+        assert np.array_equal(f32(np.full((6, 7), c, np.float32), 3), np.full((6, 7), c, np.float32))
+
+
+JACOBI_F32_PINS = [pin_jacobi_f32_tracks_fp64, pin_jacobi_f32_eigenmode, pin_jacobi_f32_by_hand,
+                   pin_jacobi_f32_fixed_points]
+
+
+@pytest.mark.parametrize("pin", JACOBI_F32_PINS, ids=lambda f: f.__name__)
+def test_jacobi_f32_pins(pin):
+    pin(O.jacobi5_f32)
 
 
 def test_jacobi_single_sweep_tiny_by_hand():
