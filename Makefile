@@ -8,7 +8,7 @@ NVFLAGS := -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -lineinfo \
            -Xcompiler -fPIC -Xcompiler -Wall -Xptxas -v --expt-relaxed-constexpr -I include $(CC_DEFS)
 HDRS := $(wildcard $(SRC)/*.cuh) include/ctaclust.h
 
-all: $(LIB) oracle/liboracle.so
+all: $(LIB) oracle/liboracle.so oracle/liboracle_omp.so
 
 $(LIB): $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu $(HDRS)
 	$(NVCC) $(NVFLAGS) -shared -o $@ $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu -ldl 2> $(PTXLOG) || (cat $(PTXLOG); exit 1)
@@ -16,7 +16,11 @@ $(LIB): $(SRC)/ctaclust.cu $(SRC)/cc_comm.cu $(HDRS)
 oracle/liboracle.so: oracle/oracle.c
 	gcc -O2 -fPIC -shared -std=c11 -o $@ $<
 
+# the same oracle with its OpenMP pragmas live: all-core timing (bench.py cpu_baseline) only
+oracle/liboracle_omp.so: oracle/oracle.c
+	gcc -O2 -fPIC -shared -std=c11 -fopenmp -o $@ $<
+
 clean:
-	rm -f $(LIB) oracle/liboracle.so build_ptxas.log
+	rm -f $(LIB) oracle/liboracle.so oracle/liboracle_omp.so build_ptxas.log
 
 .PHONY: all clean

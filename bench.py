@@ -1,20 +1,28 @@
 #!/usr/bin/env python
-"""bench.py -- BASELINE config 2 on B200: PolyBench ATAX + BICG + MVT, fp32,
+"""bench.py -- locality-aware CTA clustering on B200, one BASELINE config per run.
+
+Default (the headline, BASELINE config 2): PolyBench ATAX + BICG + MVT, fp32,
 n = 16384, column clustering (the paper's X-partition for ATX/MVT/BC, Table 2
-P:2297-2301) with the agent runtime, row-sharded over N GPUs.
+P:2297-2301) with the agent runtime, row-sharded over N GPUs.  `--config`
+selects another BASELINE config through the same drivers (drivers.py):
+jacobi (config 3, slab-sharded, boundary-first overlapped halo exchange),
+conv3 / conv7 (config 4), spmv (config 5).
 
-One step = ATAX (2 passes) + BICG (1 fused pass) + MVT (1 fused pass) over the
-1 GiB matrix: four streaming passes, HBM-bound.  `value` is algorithmic HBM
-bytes per second (whole job); the same step under the default hardware CTA
-order is timed back to back and reported as `speedup_vs_default`.
+A step = one pass of the config's hot path over its whole input (ATAX: 4
+streaming passes over the 1 GiB matrix; Jacobi: 100 sweeps).  `value` is
+whole-job algorithmic HBM bytes per second; the same step in the default
+hardware CTA order and in the persistence-only identity order is timed back
+to back (`speedup_vs_default`, `speedup_vs_identity`).
 
-    python bench.py [--gpus N --steps K --warmup W] [--impl reference] [--suite out.json]
+    python bench.py [--config atax|jacobi|conv3|conv7|spmv] [--gpus N --steps K --warmup W]
+                    [--impl reference] [--suite out.json]
 
 Rules kept: W >= 3 warm-ups; K timed steps bracketed by barrier + synchronize,
-CUDA events on the launching stream, max over ranks; the matrix (1 GiB) is
-larger than L2 (126 MB) so no flush is needed; nvidia-smi clocks sampled during
-the timed region.  The oracle (oracle/, CPU) is only run in the cpu_baseline
-leg and in --impl reference.
+CUDA events on the launching stream, max over ranks; every config's inputs
+exceed L2 (126 MB) except where stated in `config.l2`; SM clocks and
+throttle reasons sampled through NVML during the timed region.  The oracle
+(oracle/, CPU) runs only in the cpu_baseline leg, the sampled parity probe
+after the timed region (rank 0) and --impl reference.
 """
 from __future__ import annotations
 
@@ -23,32 +31,58 @@ import json
 import os
 import subprocess
 import sys
+import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "speedup & L2 sector reduction vs default CTA order; HBM GB/s vs roofline"
-N_DIM = 16384
+NSM = 148
+
+# headline launch options per config (the measured best clustered variant,
+# DESIGN.md §10), overridable from the command line
+HEADLINE = {
+    "atax": dict(backend="agent", order="col"),
+    "jacobi": dict(backend="agent", order="row"),
+    "conv3": dict(backend="agent", order="row"),
+    "conv7": dict(backend="static", order="row", num_clusters=7 * NSM),
+    "spmv": dict(backend="agent", order="row"),
+}
+WORKLOAD = {
+    "atax": "ATAX+BICG+MVT fp32 n=16384 (BASELINE config 2)",
+    "jacobi": "Jacobi 5-point fp32 16384x16384, 100 sweeps per step (BASELINE config 3)",
+    "conv3": "conv2d 3x3 fp32 8192x8192 (BASELINE config 4)",
+    "conv7": "conv2d 7x7 fp32 8192x8192 (BASELINE config 4)",
+    "spmv": "CSR SpMV fp32 R-MAT scale 24, edge factor 16 (BASELINE config 5)",
+}
 
 
 def parse():
     ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="atax", choices=sorted(HEADLINE))
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=300)
+    ap.add_argument("--steps", type=int, default=0, help="timed steps (default per config)")
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=N_DIM)
-    ap.add_argument("--backend", default="agent")
-    ap.add_argument("--order", default="col")
+    ap.add_argument("--n", type=int, default=0, help="problem size override (atax n, jacobi/conv side, spmv scale)")
+    ap.add_argument("--iters", type=int, default=100, help="jacobi sweeps per step")
+    ap.add_argument("--backend", default=None)
+    ap.add_argument("--order", default=None)
     ap.add_argument("--active-agents", type=int, default=0)
     ap.add_argument("--stages", type=int, default=0)
     ap.add_argument("--batch", type=int, default=0)
-    ap.add_argument("--staging", default="default", choices=["default", "tma", "direct"])
+    ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
+    ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
+    ap.add_argument("--no-graph", action="store_true", help="jacobi: eager launches instead of one CUDA graph")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--suite", default=None, help="also run every BASELINE config, write JSON here")
-    return ap.parse_args()
+    ap.add_argument("--no-parity", action="store_true")
+    ap.add_argument("--suite", default=None, help="also run every BASELINE config's variants, write JSON here")
+    a = ap.parse_args()
+    if not a.steps:
+        a.steps = {"atax": 100, "jacobi": 10, "conv3": 200, "conv7": 200, "spmv": 50}[a.config]
+    return a
 
 
 def peaks():
@@ -58,107 +92,249 @@ def peaks():
         return None
 
 
-def step_bytes(m, n):
-    """Algorithmic bytes of one step (each pass reads A once; vectors once;
-    outputs written once; MVT's x1/x2 read and written)."""
-    A = 4 * m * n
-    atax = (A + 4 * n + 4 * m) + (A + 4 * m + 4 * n)
-    bicg = A + 4 * (n + m) + 4 * (m + n)
-    mvt = A + 4 * (n + m) + 8 * (m + n)
-    return {"atax": atax, "bicg": bicg, "mvt": mvt, "total": atax + bicg + mvt}
+def sizes(a):
+    if a.config == "atax":
+        return {"n": a.n or 16384}
+    if a.config == "jacobi":
+        return {"side": a.n or 16384, "iters": a.iters}
+    if a.config in ("conv3", "conv7"):
+        return {"side": a.n or 8192, "R": 1 if a.config == "conv3" else 3}
+    return {"scale": a.n or 24}
 
 
 # ------------------------------------------------------------------ clocks
 class Clocks:
-    def __init__(self, device_index):
-        self.p = None
-        self.path = os.path.join("/tmp", f"cc_clocks_{os.getpid()}.csv")
-        q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
-             "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-             "clocks_event_reasons.sw_power_cap")
+    """SM clock and throttle reasons sampled through NVML every ~2 ms on a
+    background thread while the timed region runs (nvidia-smi fallback)."""
+    REASONS = {"hw_slowdown": 0x8, "hw_thermal_slowdown": 0x40, "sw_thermal_slowdown": 0x20,
+               "sw_power_cap": 0x4, "hw_power_brake_slowdown": 0x80}
+
+    def __init__(self, torch_device):
+        self.samples, self.reasons, self.err = [], 0, None
+        self._stop = threading.Event()
+        self.max_mhz = None
         try:
-            self.f = open(self.path, "w")
-            self.p = subprocess.Popen(["nvidia-smi", "-i", str(device_index), f"--query-gpu={q}",
-                                       "--format=csv,noheader,nounits", "-lms", "20"],
-                                      stdout=self.f, stderr=subprocess.DEVNULL)
-        except Exception:
-            self.p = None
+            import pynvml as N
+            import torch
+            N.nvmlInit()
+            pr = torch.cuda.get_device_properties(torch_device)
+            bus = f"{pr.pci_domain_id:08x}:{pr.pci_bus_id:02x}:{pr.pci_device_id:02x}.0"
+            self.h = N.nvmlDeviceGetHandleByPciBusId(bus)
+            self.N = N
+            self.max_mhz = N.nvmlDeviceGetMaxClockInfo(self.h, N.NVML_CLOCK_SM)
+        except Exception as e:
+            self.h, self.err = None, repr(e)[:120]
+        self.t = threading.Thread(target=self._run, daemon=True)
+        self.t.start()
+
+    def _run(self):
+        while not self._stop.is_set() and self.h is not None:
+            try:
+                self.samples.append(self.N.nvmlDeviceGetClockInfo(self.h, self.N.NVML_CLOCK_SM))
+                self.reasons |= int(self.N.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception as e:
+                self.err = repr(e)[:120]
+                return
+            time.sleep(0.002)
 
     def stop(self):
-        if self.p is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.p.terminate()
-        try:
-            self.p.wait(timeout=5)
-        except Exception:
-            self.p.kill()
-        self.f.close()
-        sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in open(self.path):
-            parts = [x.strip() for x in ln.split(",")]
-            if len(parts) < 7:
-                continue
-            try:
-                sm.append(float(parts[0]))
-                mx.append(float(parts[1]))
-            except ValueError:
-                continue
-            for nm, v in zip(names, parts[3:7]):
-                if v.lower().startswith("active"):
-                    reasons.add(nm)
-        os.unlink(self.path)
-        sm.sort()
-        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "samples": len(sm), "reasons": sorted(reasons)}
+        self._stop.set()
+        self.t.join(timeout=2)
+        if self.h is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "samples": 0, "reasons": [f"nvml unavailable: {self.err}"]}
+        s = sorted(self.samples)
+        return {"sm_mhz": s[len(s) // 2] if s else None, "sm_max_mhz": self.max_mhz, "samples": len(s),
+                "reasons": sorted(k for k, b in self.REASONS.items() if self.reasons & b), "source": "nvml"}
 
 
-# ------------------------------------------------------------------ oracle legs
-def oracle_sample(rows, n, reps, min_secs=0.0):
-    """The oracle (plain C, fp64, one thread) on rows [0, rows) of the same A:
-    ATAX + BICG + MVT, `reps` times and then on until `min_secs` have passed.
-    Returns (GB/s in the metric's algorithmic bytes, secs, reps run)."""
+# ------------------------------------------------------------------ oracle legs (CPU)
+def cpu_info():
+    model = None
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                model = ln.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    return {"cpu_count": os.cpu_count(), "model": model}
+
+
+def oracle_sample(cfg, sz, min_secs, omp=False):
+    """The oracle (plain C, fp64) on a bounded sample of the config's workload,
+    repeated until `min_secs` have passed.  Returns (GB/s in the config's
+    algorithmic bytes, secs, description, threads)."""
     import numpy as np
     import oracle as O
-    from paper_conf_asplos_lis0l0c17_b200 import synth
-    A = synth.matrix(3, rows, n)
-    x, p = synth.uniform(10, n), synth.uniform(11, n)
-    r, x1 = synth.uniform(12, rows), synth.uniform(13, rows)
-    x2, y1, y2 = synth.uniform(14, n), synth.uniform(15, n), synth.uniform(16, rows)
+    from paper_conf_asplos_lis0l0c17_b200 import drivers, synth
+    O.use_openmp(omp)
     t0 = time.perf_counter()
-    done = 0
-    while done < reps or time.perf_counter() - t0 < min_secs:
-        O.atax(A, x)
-        O.bicg(A, p, r)
-        O.mvt(A, x1, x2, y1, y2)
-        done += 1
+    done, nbytes = 0, 0
+    if cfg == "atax":
+        n, rows = sz["n"], 4096
+        A = synth.matrix(3, rows, n)
+        x, p = synth.uniform(10, n), synth.uniform(11, n)
+        r, x1 = synth.uniform(12, rows), synth.uniform(13, rows)
+        x2, y1, y2 = synth.uniform(14, n), synth.uniform(15, n), synth.uniform(16, rows)
+        t0 = time.perf_counter()
+        while done < 1 or time.perf_counter() - t0 < min_secs:
+            O.atax(A, x)
+            O.bicg(A, p, r)
+            O.mvt(A, x1, x2, y1, y2)
+            done += 1
+        nbytes = done * drivers.atax_family_bytes(rows, n)["total"]
+        desc = f"ATAX+BICG+MVT on rows 0..{rows - 1} of the {n}x{n} matrix x{done}"
+    elif cfg == "jacobi":
+        rows, cols = 1024, sz["side"]
+        u0 = synth.matrix(4, rows, cols)
+        t0 = time.perf_counter()
+        while done < 1 or time.perf_counter() - t0 < min_secs:
+            O.jacobi5(u0, 4)
+            done += 4
+        nbytes = done * 8 * rows * cols
+        desc = f"{done} fp64 sweeps of a {rows}x{cols} slab"
+    elif cfg in ("conv3", "conv7"):
+        R = sz["R"]
+        rows, cols = 1024, sz["side"]
+        img = synth.matrix(5, rows, cols)
+        w = synth.uniform(6, (2 * R + 1) ** 2).reshape(2 * R + 1, 2 * R + 1)
+        t0 = time.perf_counter()
+        while done < 1 or time.perf_counter() - t0 < min_secs:
+            O.conv2d(img, w)
+            done += 1
+        nbytes = done * 8 * rows * cols
+        desc = f"{done} x {2 * R + 1}x{2 * R + 1} conv of a {rows}x{cols} block"
+    else:
+        scale = min(sz["scale"], 20)
+        rp, col = synth.rmat_csr(7, scale, 16)
+        val, xv = synth.uniform(8, len(col)), synth.uniform(9, len(rp) - 1)
+        t0 = time.perf_counter()
+        while done < 1 or time.perf_counter() - t0 < min_secs:
+            O.spmv_csr(rp, col, val, xv)
+            done += 1
+        nbytes = done * (8 * len(col) + 4 * len(rp) + 8 * (len(rp) - 1))
+        desc = f"{done} x SpMV of R-MAT scale {scale} ({len(col)} nnz)"
     dt = time.perf_counter() - t0
-    return done * step_bytes(rows, n)["total"] / dt / 1e9, dt, done
+    thr = O.omp_threads()
+    O.use_openmp(False)
+    return nbytes / dt / 1e9, dt, desc, thr
 
 
 def run_reference(a):
-    import torch.distributed as dist
+    """--impl reference: the oracle as it stands, all host cores (OpenMP
+    build), on a bounded sample of the config per step; rank 0 only."""
     rank = int(os.environ.get("RANK", "0"))
     if int(os.environ.get("WORLD_SIZE", "1")) > 1 and rank != 0:
         return 0
-    rows = 2048
-    for _ in range(max(0, a.warmup)):
-        oracle_sample(256, a.n, 1)
-    gbs, dt, _ = oracle_sample(rows, a.n, a.steps)
+    sz = sizes(a)
+    steps = max(1, min(a.steps, 10))
+    oracle_sample(a.config, sz, 0.0, omp=True)                 # warm-up (builds, page-in)
+    tot_b, tot_t, desc, thr = 0.0, 0.0, "", 1
+    for _ in range(steps):
+        gbs, dt, desc, thr = oracle_sample(a.config, sz, 1.0, omp=True)
+        tot_b += gbs * dt
+        tot_t += dt
+    gbs = tot_b / tot_t
+    ci = cpu_info()
     line = {"impl": "reference", "metric": METRIC, "value": round(gbs, 4), "unit": "GB/s", "n_gpus": a.gpus,
-            "steps": a.steps, "warmup": a.warmup, "ms_per_step": round(1e3 * dt / a.steps, 3),
+            "steps": steps, "warmup": a.warmup, "ms_per_step": round(1e3 * tot_t / steps, 3),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic (counter-hash U[0,1), seed 3)",
-            "config": {"workload": f"ATAX+BICG+MVT fp32 n={a.n} (BASELINE config 2)",
-                       "sample": f"rows 0..{rows - 1} per step (oracle, fp64, one host thread)"},
-            "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                             "sample": f"ATAX+BICG+MVT on rows 0..{rows - 1} of the {a.n}x{a.n} matrix, per step"},
+            "data": "synthetic (counter-hash generators, same seeds as the GPU arm)",
+            "config": {"workload": WORKLOAD[a.config], "sample": desc + " per step (oracle, fp64, OpenMP)"},
+            "cpu_baseline": {"value": round(gbs, 4), "unit": "GB/s", "cores": thr, "kind": "oracle",
+                             "sample": desc, "cpu": ci},
             "e2e": {"value": round(gbs, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
 
 
+def parity_probe(cfg, D, world):
+    """Sampled comparison of this rank's results with the oracle (after the
+    timed region, on a fresh step from the initial state)."""
+    import numpy as np
+    import oracle as O
+    from paper_conf_asplos_lis0l0c17_b200 import synth
+
+    def rel(got, ref):
+        got = np.asarray(got, dtype=np.float64)
+        ref = np.asarray(ref, dtype=np.float64)
+        m = ref != 0
+        return float(np.max(np.abs(got[m] - ref[m]) / np.abs(ref[m]))) if m.any() else 0.0
+
+    if cfg == "atax":
+        n, lo, hi = D.n, D.lo, D.hi
+        rows = [lo, lo + 1, (lo + hi) // 2, hi - 1]
+        cols = [0, 1, n // 3, n - 1]
+        errs = {}
+        Ar = np.stack([synth.uniform(3, n, i * n) for i in rows])
+        xv, p, y1 = synth.uniform(10, n), synth.uniform(11, n), synth.uniform(15, n)
+        x1_0 = synth.uniform_at(13, rows)
+        errs["tmp"] = rel(D.tmp.cpu().numpy()[[i - lo for i in rows]], O.matvec(Ar, xv))
+        errs["q"] = rel(D.q.cpu().numpy()[[i - lo for i in rows]], O.matvec(Ar, p))
+        errs["x1"] = rel(D.x1.cpu().numpy()[[i - lo for i in rows]], x1_0 + O.matvec(Ar, y1))
+        m = D.m_total
+        Ac = np.stack([synth.uniform_at(3, np.arange(m) * n + j) for j in cols])   # columns as rows
+        r, y2, x2_0 = synth.uniform(12, m), synth.uniform(16, m), synth.uniform_at(14, cols)
+        errs["s"] = rel(D.s.cpu().numpy()[cols], O.matvec(Ac, r))
+        errs["x2"] = rel(D.x2.cpu().numpy()[cols], x2_0 + O.matvec(Ac, y2))
+        tmp_all = getattr(D, "tmp_all", None)
+        if tmp_all is not None:                    # y = A^T tmp with the GPU's fp32 tmp (pass 2 alone)
+            errs["y"] = rel(D.y.cpu().numpy()[cols], O.matvec(Ac, tmp_all.cpu().numpy()))
+        return {"max_rel_err": max(errs.values()), "per_output": errs, "tol": 1e-4,
+                "ok": max(errs.values()) <= 1e-4, "sample": f"rows {rows}, cols {cols}"}
+    if cfg == "jacobi":
+        T, cols = D.iters, D.cols
+        got = D.result().cpu().numpy()
+        pts = [(D.lo, 5), (D.lo + 1, cols // 2), ((D.lo + D.hi) // 2, cols - 2), (D.hi - 1, 1), (D.hi - 1, cols // 3)]
+        bad = 0
+        for (r, c) in pts:                          # light cone of radius T around (r, c)
+            r0, r1 = max(r - T, 0), min(r + T + 1, D.rows)
+            c0, c1 = max(c - T, 0), min(c + T + 1, cols)
+            win = np.stack([synth.uniform(4, c1 - c0, i * cols + c0) for i in range(r0, r1)])
+            ref = O.jacobi5_f32(win, T)[r - r0, c - c0]
+            bad += int(got[r - D.lo, c] != ref)
+        return {"mismatches": bad, "points": len(pts), "ok": bad == 0, "criterion": "bit-exact vs fp32 oracle",
+                "sample": "light cones of radius iters around 5 owned points"}
+    if cfg in ("conv3", "conv7"):
+        R, cols = D.R, D.cols
+        got = D.result().cpu().numpy()
+        errs = []
+        rlo, rhi = max(D.lo, R), min(D.hi, D.rows - R) - 8       # 8-row blocks inside the owned rows
+        for (r, c) in [(rlo, R), ((rlo + rhi) // 2, cols // 2), (rhi, cols - 1 - R - 16)]:
+            r = min(max(r, rlo), rhi)
+            img = np.stack([synth.uniform(5, 16 + 2 * R, i * cols + c - R) for i in range(r - R, r + 8 + R)])
+            ref = O.conv2d(img, D.w)[R:R + 8, R:R + 16]
+            errs.append(rel(got[r - D.lo: r - D.lo + 8, c: c + 16], ref))
+        return {"max_rel_err": max(errs), "ok": max(errs) <= 1e-4, "tol": 1e-4, "sample": "3 blocks of 8x16 outputs"}
+    if cfg == "spmv":
+        rp = D.A.row_ptr.cpu().numpy()
+        rows = sorted({0, 1, D.A.rows // 2, D.A.rows - 1} | {int(i) for i in np.argsort(np.diff(rp))[-3:]})
+        col, val = D.A.col.cpu().numpy(), D.A.val.cpu().numpy()   # the generator's input (not a GPU result)
+        xv = D.xv.cpu().numpy()
+        y = D.y.cpu().numpy()
+        errs = []
+        for i in rows:
+            a0, a1 = rp[i], rp[i + 1]
+            ref = O.spmv_csr(np.array([0, a1 - a0], np.int32), col[a0:a1], val[a0:a1], xv)[0]
+            errs.append(abs(y[i] - ref) / abs(ref) if ref else abs(y[i]))
+        return {"max_rel_err": float(max(errs)), "ok": max(errs) <= 1e-4, "tol": 1e-4,
+                "sample": f"local rows {rows} (incl. the 3 heaviest)"}
+    return None
+
+
 # ------------------------------------------------------------------ GPU arm
+def build_driver(a, X, dev):
+    from paper_conf_asplos_lis0l0c17_b200 import drivers
+    sz = sizes(a)
+    if a.config == "atax":
+        return drivers.AtaxFamily(sz["n"], X, dev)
+    if a.config == "jacobi":
+        return drivers.JacobiSlab(sz["side"], sz["side"], sz["iters"], X, dev, overlap=not a.no_overlap)
+    if a.config in ("conv3", "conv7"):
+        return drivers.ConvSlab(sz["side"], sz["side"], sz["R"], X, dev)
+    return drivers.SpmvBlock(sz["scale"], X, dev)
+
+
 def main():
     a = parse()
     if a.impl == "reference":
@@ -166,7 +342,7 @@ def main():
     import torch
     import torch.distributed as dist
 
-    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc, ops, shard, synth
+    from paper_conf_asplos_lis0l0c17_b200 import drivers, ops
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -174,194 +350,146 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    comm = None
-    if world > 1:
-        # the library's own NCCL communicator (cc_comm_*); torch.distributed only
-        # carries the unique id
-        box = [cc.Comm.unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(box, src=0)
-        comm = cc.Comm(box[0], world, rank, local)
+    X = drivers.make_exchange("nccl", world, rank, local)
     dev = torch.device("cuda", local)
-    n = a.n
-    lo, hi = shard.row_range(n, world, rank)
-    m = hi - lo
-    stream = torch.cuda.current_stream()
-
-    # inputs: generated in place on the device by the shared counter-hash generator
-    A = synth.matrix(3, m, n, backend="torch", device=dev, row0=lo)
-    col = lambda seed: synth.uniform(seed, n, backend="torch", device=dev)
-    row = lambda seed: synth.uniform(seed, m, lo, backend="torch", device=dev)
-    x, p, y1 = col(10), col(11), col(15)
-    r, x1_0, y2 = row(12), row(13), row(16)
-    x2_0 = col(14)
-    # the three column-indexed (transposed-product) outputs live in one buffer
-    # so that N > 1 sums them over the ranks with a single all-reduce per step
-    tsum = torch.empty(3 * n, device=dev)
-    y, s, x2 = tsum[:n], tsum[n:2 * n], tsum[2 * n:]
-    tmp, q = torch.empty(m, device=dev), torch.empty(m, device=dev)
-    x1 = x1_0.clone()
-    x2.copy_(x2_0 if rank == 0 else torch.zeros(n, device=dev))
+    D = build_driver(a, X, dev)
     torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    head = dict(HEADLINE[a.config])
+    if a.backend:
+        head["backend"] = a.backend
+        if a.backend != "static":
+            head.pop("num_clusters", None)
+    if a.order:
+        head["order"] = a.order
+    for k, v in (("active_agents", a.active_agents), ("stages", a.stages), ("batch", a.batch)):
+        if v:
+            head[k] = v
+    if a.staging != "default":
+        head["staging"] = a.staging
+    use_graph = a.config == "jacobi" and not a.no_graph
 
-    def run_step(backend, order, ev=None, count=None, staging=None):
-        kw = dict(backend=backend, active_agents=a.active_agents, stages=a.stages, batch=a.batch,
-                  staging=a.staging if staging is None else staging)
-        nl = 0
-        if ev is not None: ev[0].record(stream)
-        pl = ops.plan_for("atax", cc.atax_args(A, x, tmp, y), order)
-        nl += cc.launch(pl, "atax", cc.atax_args(A, x, tmp, y), cc.make_opts(**kw), stream)
-        if ev is not None: ev[1].record(stream)
-        nl += cc.launch(pl, "bicg", cc.bicg_args(A, p, r, q, s), cc.make_opts(**kw), stream)
-        if ev is not None: ev[2].record(stream)
-        nl += cc.launch(pl, "mvt", cc.mvt_args(A, y1, y2, x1, x2), cc.make_opts(**kw), stream)
-        if ev is not None: ev[3].record(stream)
-        if world > 1:                                # transposed products: one sum over ranks
-            comm.allreduce_sum(tsum, stream)
-        if count is not None:
-            count[0] += nl
-
-    def timed(backend, order, steps, per_kernel=False, staging=None):
-        for _ in range(max(3, a.warmup)):
-            run_step(backend, order, staging=staging)
-        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(steps)] if per_kernel else None
-        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    def bar():
         if world > 1:
             dist.barrier()
+
+    def maxr(v):
+        if world > 1:
+            t = torch.tensor([v], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            return t.item()
+        return v
+
+    def timed(opts, steps, per_kernel=False):
+        """(ms per step, per-kernel ms or None, launches in the timed region)"""
+        if use_graph:
+            D.graph = None
+            D.capture(opts)
+        for _ in range(max(3, a.warmup)):
+            D.step(opts)
+        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(steps)] \
+            if per_kernel and a.config == "atax" else None
+        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        bar()
         torch.cuda.synchronize()
-        count = [0]
+        n = 0
         t0.record(stream)
         for k in range(steps):
-            run_step(backend, order, evs[k] if evs else None, count, staging)
+            n += D.step(opts, ev=evs[k]) if evs else D.step(opts)
         t1.record(stream)
         torch.cuda.synchronize()
-        ms = t0.elapsed_time(t1)
-        if world > 1:
-            tt = torch.tensor([ms], device=dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            ms = tt.item()
+        ms = maxr(t0.elapsed_time(t1)) / steps
         per = None
         if evs:
             per = {"atax": sum(e[0].elapsed_time(e[1]) for e in evs) / steps,
                    "bicg": sum(e[1].elapsed_time(e[2]) for e in evs) / steps,
                    "mvt": sum(e[2].elapsed_time(e[3]) for e in evs) / steps}
-        return ms / steps, per, count[0]
+        if use_graph:
+            D.graph = None
+        return ms, per, n
 
-    # -------- clustered (headline) and default-order comparator
+    # -------- clustered (headline), then the comparators
     clocks = Clocks(local)
-    ms_clu, per_clu, launches = timed(a.backend, a.order, a.steps, per_kernel=True)
+    ms_clu, per_clu, launches = timed(head, a.steps, per_kernel=True)
     clk = clocks.stop()
-    # default hardware CTA order: the same TMA-staged body, and the plain
-    # direct-load kernel; the faster one is the comparator
-    ms_def_tma, per_def_tma, _ = timed("default", "row", a.steps, per_kernel=True, staging="tma")
-    ms_def_dir, per_def_dir, _ = timed("default", "row", a.steps, per_kernel=True, staging="direct")
-    ms_def, per_def, def_kind = ((ms_def_tma, per_def_tma, "tma-staged") if ms_def_tma <= ms_def_dir
-                                 else (ms_def_dir, per_def_dir, "direct-load"))
-    ms_id, _, _ = timed("identity", "row", max(20, a.steps // 5))
-    bytes_all = step_bytes(n, n)              # whole job: every rank's rows together
-    value = bytes_all["total"] / (ms_clu * 1e-3) / 1e9
+    cmp_steps = max(3, a.steps // 2)
+    dflt = {"backend": "default"}
+    ms_def_tma, per_def_tma, _ = timed(dict(dflt, staging="tma"), cmp_steps, per_kernel=True)
+    ms_def_dir, per_def_dir = None, None
+    if a.config != "spmv":
+        ms_def_dir, per_def_dir, _ = timed(dict(dflt, staging="direct"), cmp_steps, per_kernel=True)
+    if ms_def_dir is None or ms_def_tma <= ms_def_dir:
+        ms_def, per_def, def_kind = ms_def_tma, per_def_tma, "tma-staged"
+    else:
+        ms_def, per_def, def_kind = ms_def_dir, per_def_dir, "direct-load"
+    ms_id, _, _ = timed({"backend": "identity"}, cmp_steps)
+    total_bytes = D.bytes_per_step()
+    value = total_bytes / (ms_clu * 1e-3) / 1e9
 
-    # -------- roofline of the dominant kernel (largest share of the step)
+    # -------- home fraction of the headline schedule (untimed launch with exec_sm)
+    home = home_fraction(a, D, head, local) if world == 1 else None
+
+    # -------- roofline of the dominant kernel
     pk = peaks()
-    peak = pk["hbm_gbs"] if pk else 6650.0
-    # kernels = instantiations in the launch list: the fused row+column gemv
-    # (GemvBody<32,256,1,1>) runs BICG and MVT; ATAX is two single-direction
-    # passes (<1,0>, <0,1>).  The dominant one is the largest share of the step.
-    b_local = step_bytes(m, n)
-    groups = {"gemv_fused": (("bicg", "mvt"), 2, "k_agent<GemvBody<32, 256, 1, 1>> (BICG, MVT)"),
-              "atax": (("atax",), 2, "k_agent<GemvBody<32, 256, 1, 0>> + <0, 1> (ATAX passes)")}
-    gms = {g: sum(per_clu[k] for k in ks) for g, (ks, _, _) in groups.items()}
-    dom = max(gms, key=gms.get)
-    dom_calls, dom_launches, dom_name = groups[dom]
-    dom_bytes = sum(b_local[k] for k in dom_calls)
-    achieved = dom_bytes / (gms[dom] * 1e-3) / 1e9        # = bytes per launch / mean launch time
-    # DRAM bytes per launch of that kernel from the newest committed ncu capture
-    # (profiles/ncu_<round>_summary.json, scripts/ncu_suite.sh); the L2-sector
-    # reduction vs default order comes from the same capture.
-    traffic, l2red, prof_name = None, None, None
-    import glob
-    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "ncu_r*_summary.json")))
-    if profs:
-        try:
-            pj = json.load(open(profs[-1]))
-            prof_name = os.path.relpath(profs[-1], ROOT)
-            suf = f"_{a.backend}-{a.order}" + ("" if a.staging in ("default", "tma") else f"-{a.staging}")
-            per_l = [pj.get("dram_bytes_per_launch", {}).get(k + suf) for k in dom_calls]
-            if all(t_ is not None for t_ in per_l):     # the ATAX entry covers its two launches
-                traffic = sum(per_l) / dom_launches
-            l2red = {f"{r['kernel']}:{r['variant']}": round(r["l2_sm_sector_reduction_vs_default"], 4)
-                     for r in pj.get("rows", []) if r.get("l2_sm_sector_reduction_vs_default") is not None
-                     and r["kernel"] in ("atax", "bicg", "mvt")}
-        except Exception:
-            traffic = None
+    roof = roofline(a, D, head, ms_clu, per_clu, launches, clk, pk)
 
-    # -------- e2e through the public API with host buffers (pinned), H2D/D2H inside
-    e2e = None
-    if not a.no_e2e:
-        hA = A.cpu().pin_memory()
-        hv = {k: v.cpu().pin_memory() for k, v in dict(x=x, p=p, r=r, y1=y1, y2=y2, x1=x1_0, x2=x2_0).items()}
-        outs = {k: torch.empty(v.numel(), pin_memory=True) for k, v in dict(tmp=tmp, y=y, q=q, s=s, x1=x1, x2=x2).items()}
-        e_steps = max(3, min(10, a.steps))
+    # -------- e2e through the public API with host buffers (pinned), H2D / D2H inside
+    e2e = None if a.no_e2e else e2e_run(a, D, head, stream, bar, maxr, total_bytes)
 
-        def e2e_step():
-            A.copy_(hA, non_blocking=True)
-            for k, t_ in dict(x=x, p=p, r=r, y1=y1, y2=y2, x1=x1, x2=x2).items():
-                t_.copy_(hv[k], non_blocking=True)
-            run_step(a.backend, a.order)
-            for k, t_ in dict(tmp=tmp, y=y, q=q, s=s, x1=x1, x2=x2).items():
-                outs[k].copy_(t_, non_blocking=True)
-        e2e_step()
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
-        t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        t0.record(stream)
-        for _ in range(e_steps):
-            e2e_step()
-        t1.record(stream)
-        torch.cuda.synchronize()
-        ems = t0.elapsed_time(t1) / e_steps
-        if world > 1:
-            tt = torch.tensor([ems], device=dev)
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            ems = tt.item()
-        h2d = hA.numel() * 4 + sum(v.numel() * 4 for v in hv.values())
-        d2h = sum(v.numel() * 4 for v in outs.values())
-        e2e = {"value": round(bytes_all["total"] / (ems * 1e-3) / 1e9, 3), "unit": "GB/s",
-               "ms_per_step": round(ems, 3), "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
-
+    # -------- oracle legs (rank 0): sampled parity, CPU baseline
+    parity = None
+    if not a.no_parity:
+        if a.config == "atax":
+            D.reset()
+            D.step(head)
+            torch.cuda.synchronize()
+            if world > 1:                          # gather tmp (padded blocks) for the y = A^T tmp check
+                spans = [shard_rows(D.m_total, world, g) for g in range(world)]
+                cap = max(hi - lo for lo, hi in spans)
+                send = torch.zeros(cap, device=dev)
+                send[: D.m] = D.tmp
+                recv = torch.zeros(cap * world, device=dev)
+                X.allgather(send, recv)
+                torch.cuda.synchronize()
+                D.tmp_all = torch.cat([recv[g * cap: g * cap + (hi - lo)] for g, (lo, hi) in enumerate(spans)])
+            else:
+                D.tmp_all = D.tmp
+        elif a.config == "jacobi":
+            D.reset()
+            D.step(head)
+            torch.cuda.synchronize()
+        if rank == 0:
+            parity = parity_probe(a.config, D, world)
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu_baseline:
-        # bounded sample: rows 0..4095 of the same matrix, repeated for >= 10 s
-        gbs, dt, reps = oracle_sample(4096, n, 2, min_secs=10.0)
-        cpu = {"value": round(gbs, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-               "sample": f"ATAX+BICG+MVT on rows 0..4095 of the {n}x{n} matrix x{reps} reps ({dt:.1f} s)"}
+        g1, dt1, desc1, _ = oracle_sample(a.config, sizes(a), 8.0, omp=False)
+        gN, dtN, descN, thr = oracle_sample(a.config, sizes(a), 8.0, omp=True)
+        cpu = {"value": round(gN, 4), "unit": "GB/s", "cores": thr, "kind": "oracle",
+               "sample": f"{descN} ({dtN:.1f} s, OpenMP build, {thr} threads)",
+               "single_thread": {"value": round(g1, 4), "unit": "GB/s", "cores": 1,
+                                 "sample": f"{desc1} ({dt1:.1f} s)"},
+               "cpu": cpu_info()}
 
     if rank == 0:
+        l2red, prof = l2_reductions(a.config, head)
         line = {"metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": a.steps,
                 "warmup": max(3, a.warmup), "ms_per_step": round(ms_clu, 4), "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "f32",
-                "data": "synthetic (counter-hash U[0,1), generated on device)",
-                "config": {"workload": f"ATAX+BICG+MVT fp32 n={n} (BASELINE config 2)",
-                           "backend": a.backend, "order": a.order, "active_agents": a.active_agents or "max",
-                           "stages": a.stages or "default", "batch": a.batch or "default", "staging": a.staging,
-                           "tile": "32x256", "parallelism": f"row-shard x{world}",
-                           "l2": "inputs (1 GiB) larger than L2 (126 MB); no flush"},
+                "data": "synthetic (counter-hash generators, generated on device)",
+                "config": config_block(a, D, head, world, use_graph),
                 "speedup_vs_default": round(ms_def / ms_clu, 4),
+                "speedup_vs_identity": round(ms_id / ms_clu, 4),
                 "ms_per_step_default": round(ms_def, 4), "default_kind": def_kind,
-                "ms_per_step_default_tma": round(ms_def_tma, 4), "ms_per_step_default_direct": round(ms_def_dir, 4),
+                "ms_per_step_default_tma": round(ms_def_tma, 4),
+                "ms_per_step_default_direct": None if ms_def_dir is None else round(ms_def_dir, 4),
                 "ms_per_step_identity": round(ms_id, 4),
-                "per_kernel_ms": {k: round(v, 4) for k, v in per_clu.items()},
-                "per_kernel_ms_default": {k: round(v, 4) for k, v in per_def.items()},
-                "roofline": {"bound": "hbm", "kernel": dom_name, "achieved": round(achieved, 2),
-                             "peak": peak, "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if pk else "fallback 6.65 TB/s",
-                             "unit": "GB/s", "frac": round(achieved / peak, 4), "traffic": traffic,
-                             "launches_per_step": dom_launches, "share_of_step": round(gms[dom] / sum(gms.values()), 4),
-                             "algorithmic_bytes_per_launch": dom_bytes // dom_launches,
-                             "note": "peak is the copy (read+write) figure while these kernels stream reads of A; "
-                                     "traffic is ncu's cold-cache DRAM bytes per launch"},
-                "clocks": clk, "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": launches,
-                "l2_sector_reduction": {"source": prof_name, "vs_default_order": l2red,
-                                        "metric": "1 - lts__t_sectors_srcunit_tex(variant) / (default order)"}}
+                "roofline": roof, "clocks": clk, "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": launches,
+                "home_fraction": home, "parity": parity,
+                "l2_sector_reduction": {"source": prof, "metric": "1 - lts__t_sectors_srcunit_tex(variant) / (reference order)",
+                                        **l2red}}
+        if per_clu:
+            line["per_kernel_ms"] = {k: round(v, 4) for k, v in per_clu.items()}
+            line["per_kernel_ms_default"] = {k: round(v, 4) for k, v in per_def.items()}
         print(json.dumps(line), flush=True)
     if a.suite and rank == 0 and world == 1:
         import bench_suite
@@ -369,6 +497,220 @@ def main():
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def shard_rows(n, world, g):
+    from paper_conf_asplos_lis0l0c17_b200 import shard
+    return shard.row_range(n, world, g)
+
+
+def config_block(a, D, head, world, use_graph):
+    c = {"workload": WORKLOAD[a.config], **{k: v for k, v in head.items()},
+         "parallelism": {"atax": f"row-shard x{world}", "jacobi": f"slab-shard x{world} (halo 1 row/sweep)",
+                         "conv3": f"slab-shard x{world} (halo 1 row)", "conv7": f"slab-shard x{world} (halo 3 rows)",
+                         "spmv": f"nnz-balanced row blocks x{world}"}[a.config]}
+    if a.config == "atax":
+        c.update(n=D.n, tile="32x256", l2="inputs (1 GiB) larger than L2 (126 MB); no flush")
+    elif a.config == "jacobi":
+        c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32", graph=use_graph,
+                 overlap=getattr(D, "overlap", False),
+                 l2="2 x 1 GiB ping-pong buffers, larger than L2; no flush")
+    elif a.config in ("conv3", "conv7"):
+        c.update(rows=D.rows, cols=D.cols, R=D.R, tile="32x32",
+                 l2="image 256 MiB in + 256 MiB out, larger than L2; no flush")
+    else:
+        c.update(rows=D.rows, nnz=D.nnz, l2="col/val 2 GiB larger than L2; x (64 MiB) fits, as it would in use")
+    return c
+
+
+def l2_reductions(cfg, head):
+    """L2-sector reductions vs default order and vs the identity (persistence
+    only) order from the newest committed ncu summary (scripts/ncu_suite.sh);
+    ncu cannot run inside this process."""
+    import glob
+    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "ncu_r*_summary.json")))
+    if not profs:
+        return {}, None
+    try:
+        pj = json.load(open(profs[-1]))
+    except Exception:
+        return {}, None
+    kern = {"atax": ("atax", "bicg", "mvt"), "jacobi": ("jacobi",), "conv3": ("conv3",), "conv7": ("conv7",),
+            "spmv": ("spmv",)}[cfg]
+    rows = [r for r in pj.get("rows", []) if r.get("kernel") in kern]
+    by = {(r["kernel"], r["variant"]): r for r in rows}
+    vs_def, vs_id = {}, {}
+    for (k, v), r in by.items():
+        if r.get("l2_sm_sector_reduction_vs_default") is not None:
+            vs_def[f"{k}:{v}"] = round(r["l2_sm_sector_reduction_vs_default"], 4)
+        idr = by.get((k, "identity"))
+        if idr and r.get("l2_sectors_sm") and idr.get("l2_sectors_sm") and v != "identity":
+            vs_id[f"{k}:{v}"] = round(1 - r["l2_sectors_sm"] / idr["l2_sectors_sm"], 4)
+    return {"vs_default_order": vs_def, "vs_identity_order": vs_id}, os.path.relpath(profs[-1], ROOT)
+
+
+def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
+    peak_hbm = pk["hbm_gbs"] if pk else 6650.0
+    src = "MEASURED_PEAKS.json hbm_gbs (copy)" if pk else "fallback 6.65 TB/s"
+    traffic = traffic_from_profiles(a.config, head)
+    if a.config == "atax":
+        from paper_conf_asplos_lis0l0c17_b200 import drivers
+        b_local = drivers.atax_family_bytes(D.m, D.n)
+        groups = {"gemv_fused": (("bicg", "mvt"), 2, "k_agent<GemvBody<32, 256, 1, 1>> (BICG, MVT)"),
+                  "atax": (("atax",), 2, "k_agent<GemvBody<32, 256, 1, 0>> + <0, 1> (ATAX passes)")}
+        gms = {g: sum(per_clu[k] for k in ks) for g, (ks, _, _) in groups.items()}
+        dom = max(gms, key=gms.get)
+        calls, nl, name = groups[dom]
+        dbytes = sum(b_local[k] for k in calls)
+        ach = dbytes / (gms[dom] * 1e-3) / 1e9
+        tr = None
+        if traffic and all(traffic.get(k) for k in calls):
+            tr = sum(traffic[k] for k in calls) / nl
+        return {"bound": "hbm", "kernel": name, "achieved": round(ach, 2), "peak": peak_hbm, "peak_source": src,
+                "unit": "GB/s", "frac": round(ach / peak_hbm, 4), "traffic": tr, "launches_per_step": nl,
+                "share_of_step": round(gms[dom] / sum(gms.values()), 4),
+                "algorithmic_bytes_per_launch": dbytes // nl,
+                "timing": "CUDA events around each kernel on the launching stream, mean over the timed steps"}
+    # single-kernel configs: every launch in the step is the headline kernel
+    nl = max(1, launches // a.steps)
+    ms_launch = ms_clu / nl
+    body = {"jacobi": "Jacobi5BodyT<false>", "conv3": "Conv2dBody<1>", "conv7": "Conv2dBody<3>",
+            "spmv": "SpmvBody"}[a.config]
+    kern = {"agent": "k_agent", "static": "k_static", "default": "k_default", "identity": "k_agent"}.get(
+        head.get("backend"), "k_agent") + f"<{body}>"
+    bpl = D.bytes_per_step() // nl if D.x.world == 1 else None
+    tr = traffic.get(a.config) if traffic else None
+    if a.config == "conv7":
+        mhz = clk.get("sm_mhz") or 1965.0
+        peak = NSM * 128 * 2 * mhz * 1e6 / 1e12
+        fl = D.flops_per_step() / nl
+        ach = fl / (ms_launch * 1e-3) / 1e12
+        return {"bound": "alu", "kernel": kern, "achieved": round(ach, 2), "peak": round(peak, 2), "unit": "TFLOP/s",
+                "frac": round(ach / peak, 4), "peak_source": f"148 SM x 128 FP32 FMA/clk x 2 x {mhz:.0f} MHz "
+                                                             "(median SM clock under load)",
+                "traffic": tr, "launches_per_step": nl, "share_of_step": 1.0,
+                "algorithmic_flops_per_launch": fl, "algorithmic_bytes_per_launch": bpl,
+                "timing": "step time / launches (one kernel per step)"}
+    ach = (D.bytes_per_step() / nl) / (ms_launch * 1e-3) / 1e9
+    return {"bound": "hbm", "kernel": kern, "achieved": round(ach, 2), "peak": peak_hbm, "peak_source": src,
+            "unit": "GB/s", "frac": round(ach / peak_hbm, 4), "traffic": tr, "launches_per_step": nl,
+            "share_of_step": 1.0 if D.x.world == 1 else None, "algorithmic_bytes_per_launch": bpl,
+            "timing": "step time / launches: the step is back-to-back launches of this one kernel"
+                      + (" (whole-job bytes, includes the exchange at N > 1)" if D.x.world > 1 else "")}
+
+
+def traffic_from_profiles(cfg, head):
+    """ncu dram bytes per launch of the headline variant from the newest
+    committed summary (cold-cache, one launch)."""
+    import glob
+    profs = sorted(glob.glob(os.path.join(ROOT, "profiles", "ncu_r*_summary.json")))
+    if not profs:
+        return None
+    try:
+        d = json.load(open(profs[-1])).get("dram_bytes_per_launch", {})
+    except Exception:
+        return None
+    b, o = head.get("backend"), head.get("order")
+    suf = b + (f"-{o}" if o and b in ("agent", "static") else "")
+    if b == "static" and head.get("num_clusters"):
+        suf += f"-m{head['num_clusters'] // NSM}"
+    out = {}
+    for k in ("atax", "bicg", "mvt", "jacobi", "conv3", "conv7", "spmv"):
+        if f"{k}_{suf}" in d:
+            out[k] = d[f"{k}_{suf}"]
+    return out
+
+
+def home_fraction(a, D, head, device):
+    """Share of logical CTAs executed on their home SM (the SM of dense rank i
+    for cluster i) in one untimed launch of the headline schedule with exec_sm
+    recording (stealing on)."""
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    if head.get("backend") not in ("agent", "static"):
+        return None
+    try:
+        if a.config == "atax":
+            args = cc.bicg_args(D.A, D.p, D.r, D.q, D.s)
+            kern = "bicg"
+        elif a.config == "jacobi":
+            args = cc.jacobi5_args(D.a, D.b, 1)[0]
+            kern = "jacobi5"
+        elif a.config in ("conv3", "conv7"):
+            args, D._w = cc.conv2d_args(D.inp, D.out, D.w)
+            kern = "conv2d"
+        else:
+            Am = D.A
+            args = cc.SpmvArgs(Am.rows, Am.cols, Am.col.numel(), Am.row_ptr.data_ptr(), Am.col.data_ptr(),
+                               Am.val.data_ptr(), D.xv.data_ptr(), D.y.data_ptr(), Am.part.data_ptr())
+            kern = "spmv"
+        kw = dict(head)
+        order, nc = kw.pop("order", None), kw.pop("num_clusters", 0)
+        from paper_conf_asplos_lis0l0c17_b200 import ops
+        p = ops.plan_for(kern, args, order, kw.pop("tile", None), nc, device)
+        V = p.V
+        sm = torch.full((V,), -1, dtype=torch.int32, device="cuda")
+        cc.launch(p, kern, args, cc.make_opts(exec_sm=sm, **kw))
+        torch.cuda.synchronize()
+        perm, off = p.table()
+        rank_of = cc.sm_rank_table(device)
+        smv = sm.cpu().numpy()
+        rank_exec = np.where(smv >= 0, rank_of[np.clip(smv, 0, len(rank_of) - 1)], -1)
+        cluster = np.empty(V, np.int64)
+        cluster[perm] = np.repeat(np.arange(p.M), np.diff(off))
+        if head.get("backend") == "static":
+            # static binding: cluster i is one CTA; "home" = all of a cluster on one SM
+            same = [len(set(smv[perm[off[i]:off[i + 1]]])) <= 1 for i in range(p.M)]
+            return {"value": round(float(np.mean(same)), 4), "kind": "clusters executed on one SM (static binding)"}
+        home = cluster % NSM if p.M > NSM else cluster
+        return {"value": round(float(np.mean(rank_exec == home)), 4),
+                "kind": "tasks run on their cluster's home SM (stealing on)", "launch": kern}
+    except Exception as e:
+        return {"error": repr(e)[:200]}
+
+
+def e2e_run(a, D, head, stream, bar, maxr, total_bytes):
+    """The same metric through the public API with the step's inputs copied
+    from pinned host memory and its outputs read back, inside the timed region."""
+    import torch
+    if a.config == "atax":
+        ins, outs = D.inputs(), D.outputs()
+    elif a.config == "jacobi":
+        ins, outs = {"u": D.a}, {"u": D.a}
+    elif a.config in ("conv3", "conv7"):
+        ins, outs = {"inp": D.inp}, {"out": D.out}
+    else:
+        Am = D.A
+        ins = {"row_ptr": Am.row_ptr, "col": Am.col, "val": Am.val, "x": D.xv}
+        outs = {"y": D.y}
+    h_in = {k: v.cpu().pin_memory() for k, v in ins.items()}
+    h_out = {k: torch.empty(v.shape, dtype=v.dtype, pin_memory=True) for k, v in outs.items()}
+
+    def step():
+        for k, t_ in ins.items():
+            t_.copy_(h_in[k], non_blocking=True)
+        D.step(head)
+        for k, t_ in outs.items():
+            h_out[k].copy_(t_, non_blocking=True)
+    steps = max(3, min(10, a.steps))
+    if a.config == "jacobi":
+        D.graph = None
+        steps = 3
+    step()
+    torch.cuda.synchronize()
+    bar()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for _ in range(steps):
+        step()
+    t1.record(stream)
+    torch.cuda.synchronize()
+    ms = maxr(t0.elapsed_time(t1) / steps)
+    h2d = sum(v.numel() * v.element_size() for v in h_in.values())
+    d2h = sum(v.numel() * v.element_size() for v in h_out.values())
+    return {"value": round(total_bytes / (ms * 1e-3) / 1e9, 3), "unit": "GB/s", "ms_per_step": round(ms, 3),
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
 
 
 if __name__ == "__main__":

@@ -221,12 +221,19 @@ typedef struct { const float* A; int64_t lda; int32_t m, n; const float* p; cons
 /* MVT: x1 += A y1 ; x2 += A^T y2 (one fused pass, in place). */
 typedef struct { const float* A; int64_t lda; int32_t m, n; const float* y1; const float* y2; float* x1; float* x2; } cc_mvt_args;
 
-/* 5-point Jacobi sweeps (R14): b[i][j] = 0.2f*(c + w + e + n + s) on the interior,
- * boundary rows/cols copied.  `iters` sweeps ping-pong a -> b -> a ...; on
- * return *result_is_b (HOST, optional) says which buffer holds the last sweep.
- * rows x cols fp32 DEVICE with leading dim ld (% 4 == 0).  Logical CTA = 32 x 32
- * output tile; grid ceil(cols/32) x ceil(rows/32). */
-typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t iters; int32_t* result_is_b; } cc_jacobi5_args;
+/* 5-point Jacobi sweeps (R14, PolyBench jacobi-2d): b[i][j] =
+ * 0.2f*((((c + w) + e) + s) + n) in fp32 on the interior (s = row i+1,
+ * n = row i-1), boundary rows/cols copied.  `iters` sweeps ping-pong
+ * a -> b -> a ...; on return *result_is_b (HOST, optional) says which buffer
+ * holds the last sweep.  rows x cols fp32 DEVICE with leading dim ld (% 4 == 0).
+ * Row window (for the slab-sharded driver's boundary / interior split,
+ * S§8(e)): when row_hi > row_lo only output rows [row_lo, row_hi) of b are
+ * written (rows outside it are left untouched; every input row is still
+ * read as in the full sweep); 0 <= row_lo < row_hi <= rows.  row_lo = row_hi
+ * = 0: all rows.  Logical CTA = 32 x 32 output tile of the window; grid
+ * ceil(cols/32) x ceil((row_hi - row_lo)/32) (ceil(rows/32) without a window). */
+typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t iters; int32_t* result_is_b;
+                 int32_t row_lo, row_hi; } cc_jacobi5_args;
 
 /* CC_K_JACOBI5_HALO -- S§8(f)4: one rank's slab of the slab-sharded Jacobi
  * (S§8(e), config 3) with the per-sweep halo exchange fused into the sweep

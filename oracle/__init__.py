@@ -24,19 +24,45 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 
-def build(force: bool = False) -> str:
-    """Compile oracle.c with plain gcc -O2 (no -ffast-math: keep IEEE order)."""
-    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-fPIC", "-shared", "-std=c11",
-                               "-o", _LIB + ".tmp", _SRC])
-        os.replace(_LIB + ".tmp", _LIB)
-    return _LIB
+_LIB_OMP = os.path.join(_HERE, "liboracle_omp.so")
+_omp = False
+
+
+def build(force: bool = False, omp: bool = False) -> str:
+    """Compile oracle.c with plain gcc -O2 (no -ffast-math: keep IEEE order).
+    omp=True: the same source with -fopenmp (all-core timing only)."""
+    lib = _LIB_OMP if omp else _LIB
+    if force or not os.path.exists(lib) or os.path.getmtime(lib) < os.path.getmtime(_SRC):
+        flags = ["-fopenmp"] if omp else []
+        subprocess.check_call(["gcc", "-O2", "-fPIC", "-shared", "-std=c11"] + flags +
+                              ["-o", lib + ".tmp", _SRC])
+        os.replace(lib + ".tmp", lib)
+    return lib
+
+
+def use_openmp(on: bool = True) -> None:
+    """Route the wrappers below to the OpenMP build (bench.py cpu_baseline's
+    all-core leg) or back to the plain serial build."""
+    global _lib, _omp
+    if on != _omp:
+        _omp, _lib = on, None
+
+
+def omp_threads() -> int:
+    """Threads the OpenMP build uses (omp_get_max_threads), 1 for the plain build."""
+    if not _omp:
+        return 1
+    try:
+        return int(ctypes.CDLL(build(omp=True)).omp_get_max_threads())
+    except AttributeError:
+        g = ctypes.CDLL("libgomp.so.1")
+        return int(g.omp_get_max_threads())
 
 
 def _load():
     global _lib
     if _lib is None:
-        _lib = ctypes.CDLL(build())
+        _lib = ctypes.CDLL(build(omp=_omp))
     return _lib
 
 

@@ -16,6 +16,13 @@
  * function is that definition, evaluated directly, with no tiling, blocking
  * or reordering.
  *
+ * OpenMP: built plainly (gcc -O2, liboracle.so) the `#pragma omp` lines are
+ * ignored and every loop runs serially.  The same file built with -fopenmp
+ * (liboracle_omp.so) is only used to time the oracle on all host cores
+ * (bench.py cpu_baseline); the pragmas split independent outputs across
+ * threads (rows, or the columns of a transposed product inside each row
+ * step), so every output keeps its summation order and value.
+ *
  * Parity status (see DESIGN.md §Oracle pins): every function here is pinned
  * by tests/test_oracle_kernels.py against closed forms, special cases and
  * independent library routines (numpy / scipy).
@@ -32,6 +39,7 @@
 void oracle_matvec(int64_t m, int64_t n, const float* A, int64_t lda,
                    const float* x, double* y_out)
 {
+    #pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < m; ++i) {
         double acc = 0.0;
         for (int64_t j = 0; j < n; ++j)
@@ -45,9 +53,12 @@ static void matvec_t(int64_t m, int64_t n, const float* A, int64_t lda,
                      const double* x, double* y_out)
 {
     for (int64_t j = 0; j < n; ++j) y_out[j] = 0.0;
-    for (int64_t i = 0; i < m; ++i)
+    #pragma omp parallel
+    for (int64_t i = 0; i < m; ++i) {
+        #pragma omp for schedule(static)
         for (int64_t j = 0; j < n; ++j)
             y_out[j] += (double)A[i * lda + j] * x[i];
+    }
 }
 
 /* ------------------------------------------------------------------------
@@ -71,9 +82,12 @@ void oracle_atax_pass2(int64_t m, int64_t n, const float* A, int64_t lda,
                        const float* tmp, double* y_out)
 {
     for (int64_t j = 0; j < n; ++j) y_out[j] = 0.0;
-    for (int64_t i = 0; i < m; ++i)
+    #pragma omp parallel
+    for (int64_t i = 0; i < m; ++i) {
+        #pragma omp for schedule(static)
         for (int64_t j = 0; j < n; ++j)
             y_out[j] += (double)A[i * lda + j] * (double)tmp[i];
+    }
 }
 
 /* BICG: q = A p ; s = A^T r.  A is m x n; p has n, r has m; q has m, s has n. */
@@ -82,9 +96,12 @@ void oracle_bicg(int64_t m, int64_t n, const float* A, int64_t lda,
 {
     oracle_matvec(m, n, A, lda, p, q_out);
     for (int64_t j = 0; j < n; ++j) s_out[j] = 0.0;
-    for (int64_t i = 0; i < m; ++i)
+    #pragma omp parallel
+    for (int64_t i = 0; i < m; ++i) {
+        #pragma omp for schedule(static)
         for (int64_t j = 0; j < n; ++j)
             s_out[j] += (double)A[i * lda + j] * (double)r[i];
+    }
 }
 
 /* MVT: x1 += A y1 ; x2 += A^T y2.  A is n x n (PolyBench), here m x n:
@@ -94,6 +111,7 @@ void oracle_mvt(int64_t m, int64_t n, const float* A, int64_t lda,
                 const float* y1, const float* y2,
                 double* x1_out, double* x2_out)
 {
+    #pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < m; ++i) {
         double acc = (double)x1_in[i];
         for (int64_t j = 0; j < n; ++j)
@@ -101,9 +119,12 @@ void oracle_mvt(int64_t m, int64_t n, const float* A, int64_t lda,
         x1_out[i] = acc;
     }
     for (int64_t j = 0; j < n; ++j) x2_out[j] = (double)x2_in[j];
-    for (int64_t i = 0; i < m; ++i)
+    #pragma omp parallel
+    for (int64_t i = 0; i < m; ++i) {
+        #pragma omp for schedule(static)
         for (int64_t j = 0; j < n; ++j)
             x2_out[j] += (double)A[i * lda + j] * (double)y2[i];
+    }
 }
 
 /* ------------------------------------------------------------------------
@@ -121,7 +142,8 @@ void oracle_jacobi5(int64_t rows, int64_t cols, const float* u0, int iters,
     double* b = work + rows * cols;
     for (int64_t k = 0; k < rows * cols; ++k) { a[k] = (double)u0[k]; b[k] = a[k]; }
     for (int t = 0; t < iters; ++t) {
-        for (int64_t i = 1; i + 1 < rows; ++i)
+        #pragma omp parallel for schedule(static)
+        for (int64_t i = 1; i < rows - 1; ++i)
             for (int64_t j = 1; j + 1 < cols; ++j)
                 b[i * cols + j] = 0.2 * (a[i * cols + j] + a[i * cols + j - 1] + a[i * cols + j + 1]
                                          + a[(i - 1) * cols + j] + a[(i + 1) * cols + j]);
@@ -164,7 +186,8 @@ void oracle_conv2d(int64_t rows, int64_t cols, const float* in, int R,
 {
     const int K = 2 * R + 1;
     for (int64_t k = 0; k < rows * cols; ++k) out[k] = 0.0;
-    for (int64_t i = R; i + R < rows; ++i)
+    #pragma omp parallel for schedule(static)
+    for (int64_t i = R; i < rows - R; ++i)
         for (int64_t j = R; j + R < cols; ++j) {
             double acc = 0.0;
             for (int a = -R; a <= R; ++a)
@@ -181,6 +204,7 @@ void oracle_conv2d(int64_t rows, int64_t cols, const float* in, int R,
 void oracle_spmv_csr(int64_t rows, const int32_t* row_ptr, const int32_t* col,
                      const float* val, const float* x, double* y_out)
 {
+    #pragma omp parallel for schedule(dynamic, 1024)
     for (int64_t i = 0; i < rows; ++i) {
         double acc = 0.0;
         for (int64_t k = row_ptr[i]; k < row_ptr[i + 1]; ++k)

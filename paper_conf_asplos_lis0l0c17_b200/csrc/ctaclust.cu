@@ -325,7 +325,15 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
     case CC_K_ATAX: { auto* c = (const cc_atax_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
     case CC_K_BICG: { auto* c = (const cc_bicg_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
     case CC_K_MVT: { auto* c = (const cc_mvt_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
-    case CC_K_JACOBI5: { auto* c = (const cc_jacobi5_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
+    case CC_K_JACOBI5: {
+        auto* c = (const cc_jacobi5_args*)a;
+        if (c->row_lo != 0 || c->row_hi != 0) {
+            if (c->row_lo < 0 || c->row_hi <= c->row_lo || c->row_hi > c->rows)
+                return fail(CC_ERR_INVALID_ARG, "jacobi5 row window [%d, %d) outside [0, %d]", c->row_lo, c->row_hi, c->rows);
+            *gx = cdiv(c->cols, 32); *gy = cdiv(c->row_hi - c->row_lo, 32); return CC_OK;
+        }
+        *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK;
+    }
     case CC_K_JACOBI5_HALO: { auto* c = (const cc_jacobi5_halo_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
     case CC_K_CONV2D: { auto* c = (const cc_conv2d_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
     case CC_K_SPMV: {
@@ -719,6 +727,9 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             JacobiParams jp;
             memset(&jp, 0, sizeof jp);
             jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
+            const bool win = x->row_lo != 0 || x->row_hi != 0;
+            jp.row0 = win ? x->row_lo : 0;
+            jp.row_end = win ? x->row_hi : x->rows;
             if (x->rows > 0 && x->cols > 0) {
                 CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 34));
                 CC_TRY(make_tmap(&jp.tmap2, src, x->rows, x->cols, x->ld, ST_COLS2, 34));
@@ -745,6 +756,7 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             JacobiParams jp;
             memset(&jp, 0, sizeof jp);
             jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
+            jp.row0 = 0; jp.row_end = x->rows;
             if (up || dn) {
                 jp.h.ll = x->ll; jp.h.up_ll = x->up_ll; jp.h.dn_ll = x->dn_ll;
                 jp.h.ldl = (x->cols + 31) & ~31;

@@ -161,7 +161,9 @@ struct JacobiHalo {
     uint32_t sweep;           // absolute sweep number of this launch (1-based)
     int32_t* status;          // optional: 1 = a poll timed out (results invalid)
 };
-struct JacobiParams { CUtensorMap tmap; CUtensorMap tmap2; SplitMaps split; const float* a; float* b; int64_t ld; int32_t rows, cols; JacobiHalo h; };
+// row0 / row_end: the output row window [row0, row_end) (logical tile row by
+// covers rows row0 + 32*by ..); the full sweep has row0 = 0, row_end = rows
+struct JacobiParams { CUtensorMap tmap; CUtensorMap tmap2; SplitMaps split; const float* a; float* b; int64_t ld; int32_t rows, cols; int32_t row0, row_end; JacobiHalo h; };
 
 __device__ __forceinline__ uint64_t globaltimer() {
     uint64_t t;
@@ -300,22 +302,22 @@ struct Jacobi5BodyT {
             const uint32_t ll_bytes = (top ? 256u : 0u) + (bot ? 256u : 0u);
             stage_commit(full, lane, (uint32_t)(HaloTile<1>::kRows * ST_COLS * 4) + ll_bytes);
             if (lane == 0) {
-                tma_load_2d(stage, &p.tmap, bx * 32 - 4, by * 32 - 1, full);
+                tma_load_2d(stage, &p.tmap, bx * 32 - 4, p.row0 + by * 32 - 1, full);
                 uint8_t* extra = stage + kTileBytes;
                 if (top) bulk_g2s(extra, p.h.ll + par + bx * 32, 256u, full);
                 if (bot) bulk_g2s(extra + 256, p.h.ll + par + p.h.ldl + bx * 32, 256u, full);
             }
             return;
         }
-        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, by * 32, stage, full, lane, s.staging, &p.tmap, l2h,
-                           &p.split);
+        HaloTile<1>::stage(p.a, p.ld, p.rows, p.cols, bx * 32, p.row0 + by * 32, stage, full, lane, s.staging, &p.tmap,
+                           l2h, &p.split);
     }
 
     // merged slots (plain sweep, TMA staging): tiles (bx, by), (bx+1, by) in one box
     __device__ __forceinline__ bool can_merge(const Sched& s) const { return s.staging == STAGE_TMA; }
     __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
                                               uint64_t* full, int lane) {
-        if (n >= 2) HaloTile<1>::stage2(bx * 32, by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
+        if (n >= 2) HaloTile<1>::stage2(bx * 32, p.row0 + by * 32, stage, full, lane, &p.tmap2, l2h, &p.split);
         else produce(s, bx, by, stage, full, lane);
     }
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
@@ -344,7 +346,7 @@ struct Jacobi5BodyT {
         by = phys_row(by);
         const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
         const int gx = bx * 32 + 4 * c4;
-        const int gy0 = by * 32 + r0;
+        const int gy0 = p.row0 + by * 32 + r0;
         const bool in_col = gx < p.cols;
         float4 row[RB + 2];                        // input rows gy0-1 .. gy0+RB
         float lw[RB], re[RB];
@@ -400,7 +402,7 @@ struct Jacobi5BodyT {
 #pragma unroll
             for (int j = 0; j < RB; ++j) {
                 const int gy = gy0 + j;
-                if (gy >= p.rows) break;
+                if (gy >= p.row_end) break;
                 const float4 o = jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols);
                 store4_masked(p.b + (int64_t)gy * p.ld + gx, o, gx, p.cols);
 #ifndef CC_LL_NOSTORE
@@ -413,7 +415,8 @@ struct Jacobi5BodyT {
 #ifndef CC_JACOBI_INTERIOR_FAST
 #define CC_JACOBI_INTERIOR_FAST 1
 #endif
-        if (CC_JACOBI_INTERIOR_FAST && gx >= 1 && gx + 4 <= p.cols - 1 && gy0 >= 1 && gy0 + RB <= p.rows - 1) {
+        if (CC_JACOBI_INTERIOR_FAST && gx >= 1 && gx + 4 <= p.cols - 1 && gy0 >= 1 && gy0 + RB <= p.rows - 1 &&
+            gy0 + RB <= p.row_end) {
             // interior block: no boundary cells, plain float4 stores (same arithmetic)
 #pragma unroll
             for (int j = 0; j < RB; ++j) {
@@ -427,7 +430,7 @@ struct Jacobi5BodyT {
 #pragma unroll
         for (int j = 0; j < RB; ++j) {
             const int gy = gy0 + j;
-            if (gy >= p.rows) break;
+            if (gy >= p.row_end) break;
             store4_out(p.b + (int64_t)gy * p.ld + gx,
                        jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols), gx,
                        p.cols, l2h);

@@ -1,0 +1,422 @@
+"""Per-rank drivers of the BASELINE configs, sharded over G GPUs.
+
+One process per GPU.  Each driver owns this rank's shard of one config's
+inputs on the device and runs one "step" of the hot path on it -- the
+library's kernels through ``ops`` plus the config's exchange step through an
+:class:`Exchange` -- asynchronously on the current stream.  The data-path
+exchanges are exactly the ones S§8(e) lists:
+
+* ATAX / BICG / MVT (config 2): rows of A per rank; the three transposed
+  products are summed over the ranks with ONE all-reduce per step.
+* Jacobi (config 3): slabs of rows + one halo row per side; per sweep the
+  boundary tile rows are computed first, then the halo exchange runs on a
+  communication stream while the interior tile rows compute (the classic
+  boundary-first overlap); the whole 100-sweep step can be captured in one
+  CUDA graph.
+* conv2d (config 4): slabs + R halo rows; one exchange per step.
+* SpMV (config 5): nnz-balanced row blocks (merge-path measure), x replicated,
+  y all-gathered (padded blocks).
+
+At world = 1 every driver is the unsharded computation with no exchange.
+Nothing here does arithmetic of the method: kernels run in libctaclust,
+exchanges in NCCL (the library's communicator) or, for the multi-process
+tests on one GPU, torch.distributed.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+from . import ctaclust as cc
+from . import ops, shard, synth
+
+
+# ----------------------------------------------------------------------------
+# exchanges
+# ----------------------------------------------------------------------------
+class Exchange:
+    """The collective steps a driver needs.  world == 1: all no-ops."""
+    world, rank = 1, 0
+
+    def allreduce_sum(self, t, stream=None):
+        pass
+
+    def halo_exchange(self, slab, halo, stream=None):
+        pass
+
+    def allgather(self, send, recv, stream=None):
+        recv[: send.numel()].copy_(send)
+
+    @property
+    def capturable(self) -> bool:
+        return True
+
+
+class LibExchange(Exchange):
+    """NCCL through the library's own communicator (cc_comm_*, cc_halo_exchange,
+    cc_allreduce_sum, cc_allgather); rank 0's unique id travels over the
+    torch.distributed process group.  Capturable into CUDA graphs."""
+
+    def __init__(self, world: int, rank: int, device: int):
+        self.world, self.rank = world, rank
+        box = [cc.Comm.unique_id() if rank == 0 else None]
+        if world > 1:
+            dist.broadcast_object_list(box, src=0)
+        self.comm = cc.Comm(box[0], world, rank, device)
+
+    def allreduce_sum(self, t, stream=None):
+        self.comm.allreduce_sum(t, stream)
+
+    def halo_exchange(self, slab, halo, stream=None):
+        self.comm.halo_exchange(slab, halo, stream)
+
+    def allgather(self, send, recv, stream=None):
+        self.comm.allgather(send, recv, stream)
+
+
+class TorchExchange(Exchange):
+    """torch.distributed collectives; device tensors are staged through host
+    memory when the backend is gloo (several ranks sharing one GPU in the
+    multi-process GPU tests, where NCCL refuses duplicate devices).  Not
+    capturable."""
+
+    def __init__(self):
+        self.world, self.rank = dist.get_world_size(), dist.get_rank()
+        self.staged = dist.get_backend() == "gloo"
+
+    @property
+    def capturable(self) -> bool:
+        return False
+
+    def _h(self, t):
+        return t.cpu() if self.staged and t.is_cuda else t
+
+    def allreduce_sum(self, t, stream=None):
+        if self.world == 1:
+            return
+        h = self._h(t)
+        dist.all_reduce(h, op=dist.ReduceOp.SUM)
+        if h is not t:
+            t.copy_(h)
+
+    def halo_exchange(self, slab, halo, stream=None):
+        if self.world == 1 or halo == 0:
+            return
+        up, dn = self.rank > 0, self.rank < self.world - 1
+        rows = slab.shape[0]
+        own0, own1 = (halo if up else 0), (rows - halo if dn else rows)
+        reqs, bufs = [], {}
+        if up:
+            reqs.append(dist.isend(self._h(slab[own0: own0 + halo].contiguous()), self.rank - 1))
+            bufs["top"] = self._h(torch.empty_like(slab[0:halo]))
+            reqs.append(dist.irecv(bufs["top"], self.rank - 1))
+        if dn:
+            reqs.append(dist.isend(self._h(slab[own1 - halo: own1].contiguous()), self.rank + 1))
+            bufs["bot"] = self._h(torch.empty_like(slab[0:halo]))
+            reqs.append(dist.irecv(bufs["bot"], self.rank + 1))
+        for r in reqs:
+            r.wait()
+        if up:
+            slab[0:halo].copy_(bufs["top"])
+        if dn:
+            slab[rows - halo: rows].copy_(bufs["bot"])
+
+    def allgather(self, send, recv, stream=None):
+        if self.world == 1:
+            recv[: send.numel()].copy_(send)
+            return
+        out = [self._h(torch.empty_like(send)) for _ in range(self.world)]
+        dist.all_gather(out, self._h(send.contiguous()))
+        recv.copy_(torch.cat([o.to(recv.device) for o in out]))
+
+
+def make_exchange(kind: str, world: int, rank: int, device: int) -> Exchange:
+    if world == 1:
+        return Exchange()
+    if kind == "nccl":
+        return LibExchange(world, rank, device)
+    return TorchExchange()
+
+
+# ----------------------------------------------------------------------------
+# config 2: ATAX + BICG + MVT, row-sharded
+# ----------------------------------------------------------------------------
+def atax_family_bytes(m: int, n: int) -> dict:
+    """Algorithmic bytes of one ATAX (2 passes) + BICG + MVT step over an m x n
+    A (each pass reads A once; vectors read once; outputs written once; MVT's
+    x1 / x2 read and written)."""
+    A = 4 * m * n
+    atax = (A + 4 * n + 4 * m) + (A + 4 * m + 4 * n)
+    bicg = A + 4 * (n + m) + 4 * (m + n)
+    mvt = A + 4 * (n + m) + 8 * (m + n)
+    return {"atax": atax, "bicg": bicg, "mvt": mvt, "total": atax + bicg + mvt}
+
+
+class AtaxFamily:
+    """Rank `rank`'s rows [lo, hi) of the n x n problem (seeds as DESIGN §4).
+
+    State: x1 (row-indexed, local) and x2 (column-indexed, replicated) carry
+    over steps (MVT accumulates in place).  The column-indexed outputs y, s, x2
+    share one buffer so one all-reduce per step sums them.  Every step the
+    ranks other than 0 zero their x2 slice before MVT, so after the sum
+    x2 = x2_prev + sum over ranks of A_g^T y2_g (rank 0 carries x2_prev)."""
+
+    def __init__(self, n: int, xchg: Exchange, device, m_total: int | None = None):
+        self.n, self.x = n, xchg
+        self.m_total = n if m_total is None else m_total
+        self.lo, self.hi = shard.row_range(self.m_total, xchg.world, xchg.rank)
+        m = self.m = self.hi - self.lo
+        dev = self.dev = torch.device(device)
+        self.A = synth.matrix(3, m, n, backend="torch", device=dev, row0=self.lo)
+        col = lambda seed: synth.uniform(seed, n, backend="torch", device=dev)
+        row = lambda seed: synth.uniform(seed, m, self.lo, backend="torch", device=dev)
+        self.xv, self.p, self.y1 = col(10), col(11), col(15)
+        self.r, self.x1_0, self.y2 = row(12), row(13), row(16)
+        self.x2_0 = col(14)
+        self.tsum = torch.empty(3 * n, device=dev)
+        self.y, self.s, self.x2 = self.tsum[:n], self.tsum[n:2 * n], self.tsum[2 * n:]
+        self.tmp, self.q = torch.empty(m, device=dev), torch.empty(m, device=dev)
+        self.x1 = torch.empty(m, device=dev)
+        self.reset()
+
+    def reset(self):
+        """Back to the initial state (x1 = x1_0, x2 = x2_0)."""
+        self.x1.copy_(self.x1_0)
+        self.x2.copy_(self.x2_0)
+
+    def inputs(self) -> dict:
+        return dict(A=self.A, x=self.xv, p=self.p, r=self.r, y1=self.y1, y2=self.y2, x1=self.x1, x2=self.x2)
+
+    def outputs(self) -> dict:
+        return dict(tmp=self.tmp, y=self.y, q=self.q, s=self.s, x1=self.x1, x2=self.x2)
+
+    def step(self, opts: dict, stream=None, ev=None) -> int:
+        """One ATAX + BICG + MVT step (+ the all-reduce at world > 1).  `ev`:
+        optional 4 events recorded around the three kernels.  Returns the
+        number of library kernels queued."""
+        nl = 0
+        if ev is not None:
+            ev[0].record(stream)
+        nl += _launch("atax", cc.atax_args(self.A, self.xv, self.tmp, self.y), opts, stream)
+        if ev is not None:
+            ev[1].record(stream)
+        nl += _launch("bicg", cc.bicg_args(self.A, self.p, self.r, self.q, self.s), opts, stream)
+        if ev is not None:
+            ev[2].record(stream)
+        if self.x.world > 1 and self.x.rank != 0:
+            self.x2.zero_()
+        nl += _launch("mvt", cc.mvt_args(self.A, self.y1, self.y2, self.x1, self.x2), opts, stream)
+        if ev is not None:
+            ev[3].record(stream)
+        self.x.allreduce_sum(self.tsum, stream)
+        return nl
+
+    def bytes_per_step(self) -> int:
+        return atax_family_bytes(self.m_total, self.n)["total"]
+
+
+def _launch(kernel, args, opts, stream, **plan_kw):
+    kw = dict(opts)
+    order = kw.pop("order", None)
+    tile = kw.pop("tile", None)
+    num_clusters = kw.pop("num_clusters", 0)
+    dev = torch.cuda.current_device()
+    p = ops.plan_for(kernel, args, order, tile, num_clusters, dev, **plan_kw)
+    return cc.launch(p, kernel, args, cc.make_opts(**kw), stream)
+
+
+# ----------------------------------------------------------------------------
+# config 3: Jacobi, slab-sharded with boundary-first overlap
+# ----------------------------------------------------------------------------
+class JacobiSlab:
+    """This rank's slab of the rows x cols Jacobi (u0 = seed 4), `iters` sweeps
+    per step.
+
+    Per sweep (world > 1, overlap on): the first and last owned tile rows are
+    computed first (row windows of CC_K_JACOBI5); the halo exchange of the
+    freshly written boundary rows runs on `comm_stream` while the interior
+    rows compute; the next sweep waits for both.  Without overlap (or at
+    world = 1) a sweep is one launch, then the exchange."""
+
+    def __init__(self, rows: int, cols: int, iters: int, xchg: Exchange, device, overlap: bool = True):
+        self.rows, self.cols, self.iters, self.x = rows, cols, iters, xchg
+        self.lo, self.hi, self.llo, self.lhi = shard.slab_range(rows, xchg.world, xchg.rank, 1)
+        L = self.lhi - self.llo
+        dev = self.dev = torch.device(device)
+        ld = (cols + 3) & ~3
+        self.u0 = synth.matrix(4, L, cols, backend="torch", device=dev, row0=self.llo)
+        self.a = torch.zeros(L, ld, device=dev)[:, :cols]
+        self.b = torch.zeros(L, ld, device=dev)[:, :cols]
+        own0, own1 = self.lo - self.llo, self.hi - self.llo
+        self.own = (own0, own1)
+        self.overlap = overlap and xchg.world > 1 and own1 - own0 > 64
+        if self.overlap:
+            t1, b0 = own0 + 32, own1 - 32
+            self.windows_b = [(own0, t1), (b0, own1)]
+            self.window_i = (t1, b0) if b0 > t1 else None
+        self.comm_stream = torch.cuda.Stream(device=dev) if xchg.world > 1 else None
+        self.ev_b = [torch.cuda.Event() for _ in range(2)]
+        self.ev_x = [torch.cuda.Event() for _ in range(2)]
+        self.graph = None
+        self.reset()
+
+    def reset(self):
+        self.a.copy_(self.u0)
+        self.b.copy_(self.u0)        # boundary rows / halo rows defined in both buffers
+
+    def _sweep(self, src, dst, opts, stream, k):
+        nl = 0
+        if not self.overlap:
+            nl += _launch("jacobi5", cc.jacobi5_args(src, dst, 1)[0], opts, stream)
+            self.x.halo_exchange(dst, 1, stream)
+            return nl
+        cur = torch.cuda.current_stream() if stream is None else stream
+        for w in self.windows_b:
+            nl += _launch("jacobi5", cc.jacobi5_args(src, dst, 1, row_window=w)[0], opts, stream)
+        eb, ex = self.ev_b[k & 1], self.ev_x[k & 1]
+        eb.record(cur)
+        self.comm_stream.wait_event(eb)
+        with torch.cuda.stream(self.comm_stream):
+            self.x.halo_exchange(dst, 1, self.comm_stream)
+        ex.record(self.comm_stream)
+        if self.window_i is not None:
+            nl += _launch("jacobi5", cc.jacobi5_args(src, dst, 1, row_window=self.window_i)[0], opts, stream)
+        cur.wait_event(ex)
+        return nl
+
+    def step(self, opts: dict, stream=None) -> int:
+        """`iters` sweeps; the result is in self.result() afterwards.  The
+        buffers ping-pong within the step and the step starts from a (an even
+        `iters` returns the result to a; odd steps alternate)."""
+        if self.graph is not None:
+            self.graph.replay()
+            return self.graph_launches
+        nl = 0
+        for k in range(self.iters):
+            src, dst = (self.a, self.b) if k % 2 == 0 else (self.b, self.a)
+            nl += self._sweep(src, dst, opts, stream, k)
+        if self.iters % 2:
+            self.a, self.b = self.b, self.a
+        return nl
+
+    def capture(self, opts: dict) -> bool:
+        """Capture one step (all `iters` sweeps, both streams) into a CUDA graph;
+        later steps replay it.  Plans and tensor maps are created by an eager
+        step first (no allocation is legal during capture).  Returns False when
+        the exchange cannot be captured."""
+        if not self.x.capturable or self.iters % 2:
+            return False
+        self.step(opts)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream(device=self.dev)
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            with torch.cuda.graph(g, stream=s):
+                n = self.step(opts)
+        torch.cuda.current_stream().wait_stream(s)
+        self.graph, self.graph_launches = g, n
+        return True
+
+    def result(self):
+        """Owned rows of the field after the last step."""
+        return self.a[self.own[0]: self.own[1]]
+
+    def bytes_per_step(self) -> int:
+        return 8 * self.rows * self.cols * self.iters
+
+
+# ----------------------------------------------------------------------------
+# config 4: conv2d, slab-sharded
+# ----------------------------------------------------------------------------
+class ConvSlab:
+    """This rank's slab (owned rows + R halo rows per side) of the rows x cols
+    image (seed 5), filter seed 6 normalised to sum 1.  One step =
+    the halo exchange (world > 1) + one conv launch; owned output rows are
+    exact (every owned row is >= R rows from a slab edge that is not the
+    image border)."""
+
+    def __init__(self, rows: int, cols: int, R: int, xchg: Exchange, device, w=None):
+        self.rows, self.cols, self.R, self.x = rows, cols, R, xchg
+        self.lo, self.hi, self.llo, self.lhi = shard.slab_range(rows, xchg.world, xchg.rank, R)
+        dev = self.dev = torch.device(device)
+        K = 2 * R + 1
+        if w is None:
+            import numpy as np
+            w = synth.uniform(6, K * K).reshape(K, K)
+            w = (w / w.astype(np.float64).sum()).astype(np.float32)
+        self.w = w
+        self.inp = synth.matrix(5, self.lhi - self.llo, cols, backend="torch", device=dev, row0=self.llo)
+        self.out = torch.empty_like(self.inp)
+
+    def inputs(self) -> dict:
+        return dict(inp=self.inp)
+
+    def outputs(self) -> dict:
+        return dict(out=self.result())
+
+    def step(self, opts: dict, stream=None) -> int:
+        self.x.halo_exchange(self.inp, self.R, stream)
+        args, self._w = cc.conv2d_args(self.inp, self.out, self.w)
+        return _launch("conv2d", args, opts, stream)
+
+    def result(self):
+        return self.out[self.lo - self.llo: self.hi - self.llo]
+
+    def bytes_per_step(self) -> int:
+        return 8 * self.rows * self.cols
+
+    def flops_per_step(self) -> int:
+        return 2 * (2 * self.R + 1) ** 2 * (self.rows - 2 * self.R) * (self.cols - 2 * self.R)
+
+
+# ----------------------------------------------------------------------------
+# config 5: CSR SpMV, nnz-balanced row blocks
+# ----------------------------------------------------------------------------
+class SpmvBlock:
+    """This rank's nnz-balanced row block of the R-MAT matrix (seed 7, values
+    seed 8, x seed 9).  x is replicated; one step = local SpMV + all-gather of
+    y (blocks padded to the largest)."""
+
+    def __init__(self, scale: int, xchg: Exchange, device, edge_factor: int = 16):
+        self.x = xchg
+        dev = self.dev = torch.device(device)
+        rp, col = synth.rmat_csr(7, scale, edge_factor, backend="torch", device=dev)
+        self.rows, self.nnz = rp.numel() - 1, col.numel()
+        val = synth.uniform(8, self.nnz, backend="torch", device=dev)
+        self.xv = synth.uniform(9, self.rows, backend="torch", device=dev)
+        self.lo, self.hi = shard.spmv_row_range(rp, xchg.world, xchg.rank)
+        if xchg.world > 1:
+            lrp, lcol, lval = shard.spmv_local(rp, col, val, self.lo, self.hi)
+            lrp, lcol, lval = lrp.contiguous(), lcol.contiguous(), lval.contiguous()
+            del rp, col, val
+        else:
+            lrp, lcol, lval = rp, col, val
+        self.A = ops.SpmvMatrix(lrp, lcol, lval, n_cols=self.rows)
+        self.local_nnz = lcol.numel()
+        self.cap = self._cap(xchg)
+        self.y = torch.zeros(self.cap, device=dev)
+        self.yall = torch.zeros(self.cap * xchg.world, device=dev)
+
+    def _cap(self, xchg):
+        n = torch.tensor([self.hi - self.lo], device=self.dev)
+        if xchg.world > 1:
+            h = n.cpu()
+            dist.all_reduce(h, op=dist.ReduceOp.MAX)
+            n = h
+        return int(n.item())
+
+    def step(self, opts: dict, stream=None) -> int:
+        nl = _launch_spmv(self.A, self.xv, self.y, opts, stream)
+        if self.x.world > 1:
+            self.x.allgather(self.y, self.yall, stream)
+        return nl
+
+    def bytes_per_step(self) -> int:
+        return 8 * self.nnz + 4 * (self.rows + 1) + 8 * self.rows
+
+
+def _launch_spmv(Am, x, y, opts, stream):
+    args = cc.SpmvArgs(Am.rows, Am.cols, Am.col.numel(), Am.row_ptr.data_ptr(), Am.col.data_ptr(),
+                       Am.val.data_ptr(), x.data_ptr(), y.data_ptr(), Am.part.data_ptr())
+    return _launch("spmv", args, opts, stream)

@@ -88,6 +88,14 @@ def uniform(seed: int, count: int, start: int = 0, *, backend: str = "numpy",
     return out
 
 
+def uniform_at(seed: int, idx, stream: int = 0) -> np.ndarray:
+    """U[0,1) fp32 values at arbitrary logical indices (numpy): the same
+    values :func:`uniform` gives at those indices (e.g. one column of a
+    row-major matrix: idx = i * cols + j)."""
+    h = hash_u32_np(seed, np.asarray(idx, dtype=np.uint64), stream)
+    return (h >> np.uint32(8)).astype(np.float32) * np.float32(2.0 ** -24)
+
+
 def bytes_u8(seed: int, count: int, start: int = 0, *, kind: str = "uniform", backend: str = "numpy",
              device=None, chunk: int = 1 << 26):
     """``count`` uint8 values: ``uniform`` = top byte of the hash; ``skewed`` =
