@@ -74,7 +74,8 @@ def parse():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
-    ap.add_argument("--no-graph", action="store_true", help="jacobi: eager launches instead of one CUDA graph")
+    ap.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
+    ap.add_argument("--hot", type=int, default=16384, help="spmv: hub slots of the inspector (0: plain CSR)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-parity", action="store_true")
@@ -281,7 +282,7 @@ def parity_probe(cfg, D, world):
         if tmp_all is not None:                    # y = A^T tmp with the GPU's fp32 tmp (pass 2 alone)
             errs["y"] = rel(D.y.cpu().numpy()[cols], O.matvec(Ac, tmp_all.cpu().numpy()))
         return {"max_rel_err": max(errs.values()), "per_output": errs, "tol": 1e-4,
-                "ok": max(errs.values()) <= 1e-4, "sample": f"rows {rows}, cols {cols}"}
+                "ok": bool(max(errs.values()) <= 1e-4), "sample": f"rows {rows}, cols {cols}"}
     if cfg == "jacobi":
         T, cols = D.iters, D.cols
         got = D.result().cpu().numpy()
@@ -305,7 +306,8 @@ def parity_probe(cfg, D, world):
             img = np.stack([synth.uniform(5, 16 + 2 * R, i * cols + c - R) for i in range(r - R, r + 8 + R)])
             ref = O.conv2d(img, D.w)[R:R + 8, R:R + 16]
             errs.append(rel(got[r - D.lo: r - D.lo + 8, c: c + 16], ref))
-        return {"max_rel_err": max(errs), "ok": max(errs) <= 1e-4, "tol": 1e-4, "sample": "3 blocks of 8x16 outputs"}
+        return {"max_rel_err": float(max(errs)), "ok": bool(max(errs) <= 1e-4), "tol": 1e-4,
+                "sample": "3 blocks of 8x16 outputs"}
     if cfg == "spmv":
         rp = D.A.row_ptr.cpu().numpy()
         rows = sorted({0, 1, D.A.rows // 2, D.A.rows - 1} | {int(i) for i in np.argsort(np.diff(rp))[-3:]})
@@ -317,7 +319,7 @@ def parity_probe(cfg, D, world):
             a0, a1 = rp[i], rp[i + 1]
             ref = O.spmv_csr(np.array([0, a1 - a0], np.int32), col[a0:a1], val[a0:a1], xv)[0]
             errs.append(abs(y[i] - ref) / abs(ref) if ref else abs(y[i]))
-        return {"max_rel_err": float(max(errs)), "ok": max(errs) <= 1e-4, "tol": 1e-4,
+        return {"max_rel_err": float(max(errs)), "ok": bool(max(errs) <= 1e-4), "tol": 1e-4,
                 "sample": f"local rows {rows} (incl. the 3 heaviest)"}
     return None
 
@@ -332,7 +334,7 @@ def build_driver(a, X, dev):
         return drivers.JacobiSlab(sz["side"], sz["side"], sz["iters"], X, dev, overlap=not a.no_overlap)
     if a.config in ("conv3", "conv7"):
         return drivers.ConvSlab(sz["side"], sz["side"], sz["R"], X, dev)
-    return drivers.SpmvBlock(sz["scale"], X, dev)
+    return drivers.SpmvBlock(sz["scale"], X, dev, hot=a.hot)
 
 
 def main():
@@ -367,7 +369,7 @@ def main():
             head[k] = v
     if a.staging != "default":
         head["staging"] = a.staging
-    use_graph = a.config == "jacobi" and not a.no_graph
+    use_graph = a.config != "atax" and not a.no_graph     # atax: eager, per-kernel events
 
     def bar():
         if world > 1:
@@ -505,21 +507,22 @@ def shard_rows(n, world, g):
 
 
 def config_block(a, D, head, world, use_graph):
-    c = {"workload": WORKLOAD[a.config], **{k: v for k, v in head.items()},
+    c = {"workload": WORKLOAD[a.config], **{k: v for k, v in head.items()}, "graph": use_graph,
          "parallelism": {"atax": f"row-shard x{world}", "jacobi": f"slab-shard x{world} (halo 1 row/sweep)",
                          "conv3": f"slab-shard x{world} (halo 1 row)", "conv7": f"slab-shard x{world} (halo 3 rows)",
                          "spmv": f"nnz-balanced row blocks x{world}"}[a.config]}
     if a.config == "atax":
         c.update(n=D.n, tile="32x256", l2="inputs (1 GiB) larger than L2 (126 MB); no flush")
     elif a.config == "jacobi":
-        c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32", graph=use_graph,
+        c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32",
                  overlap=getattr(D, "overlap", False),
                  l2="2 x 1 GiB ping-pong buffers, larger than L2; no flush")
     elif a.config in ("conv3", "conv7"):
         c.update(rows=D.rows, cols=D.cols, R=D.R, tile="32x32",
                  l2="image 256 MiB in + 256 MiB out, larger than L2; no flush")
     else:
-        c.update(rows=D.rows, nnz=D.nnz, l2="col/val 2 GiB larger than L2; x (64 MiB) fits, as it would in use")
+        c.update(rows=D.rows, nnz=D.nnz, hub_slots=D.A.n_hot,
+                 l2="col/val 2 GiB larger than L2; x (64 MiB) fits, as it would in use")
     return c
 
 
@@ -641,9 +644,7 @@ def home_fraction(a, D, head, device):
             args, D._w = cc.conv2d_args(D.inp, D.out, D.w)
             kern = "conv2d"
         else:
-            Am = D.A
-            args = cc.SpmvArgs(Am.rows, Am.cols, Am.col.numel(), Am.row_ptr.data_ptr(), Am.col.data_ptr(),
-                               Am.val.data_ptr(), D.xv.data_ptr(), D.y.data_ptr(), Am.part.data_ptr())
+            args = D.A.args(D.xv, D.y)
             kern = "spmv"
         kw = dict(head)
         order, nc = kw.pop("order", None), kw.pop("num_clusters", 0)
@@ -682,7 +683,9 @@ def e2e_run(a, D, head, stream, bar, maxr, total_bytes):
         ins, outs = {"inp": D.inp}, {"out": D.out}
     else:
         Am = D.A
-        ins = {"row_ptr": Am.row_ptr, "col": Am.col, "val": Am.val, "x": D.xv}
+        ins = {"row_ptr": Am.row_ptr, "col": Am.col_kernel, "val": Am.val, "x": D.xv}
+        if Am.hot is not None:
+            ins["hot"] = Am.hot
         outs = {"y": D.y}
     h_in = {k: v.cpu().pin_memory() for k, v in ins.items()}
     h_out = {k: torch.empty(v.shape, dtype=v.dtype, pin_memory=True) for k, v in outs.items()}

@@ -297,9 +297,19 @@ typedef struct { const float* in; float* out; int64_t ld; int32_t rows, cols; in
  * the merge-path diagonals [4096 b, 4096 (b+1)) of the row-ends x nonzeros merge
  * grid (so power-law rows are balanced); grid = ceil((rows+nnz)/4096) x 1.
  * part (DEVICE, grid+1 entries) is the split table cc_spmv_partition fills once
- * per matrix structure. */
+ * per matrix structure.
+ * Hub-column form (n_hot > 0, the output of cc_spmv_inspect): `col` holds the
+ * inspector's encoding -- a reference to hub slot k is stored as -(k+1), any
+ * other column as itself -- `hot` (DEVICE int32[n_hot]) the column of each
+ * slot and `xh` (DEVICE float[n_hot], caller-owned scratch) receives the hub
+ * values: each launch first gathers xh[n_hot-1-k] = x[hot[k]] (one small
+ * kernel, counted in *launches), then the SpMV reads hub references from that
+ * dense 4 * n_hot-byte array, which every SM keeps in L1.  Same y bits as the
+ * plain form (the products and their order do not change).  n_hot = 0: plain
+ * CSR, hot/xh ignored. */
 typedef struct { int32_t rows, cols; int64_t nnz; const int32_t* row_ptr; const int32_t* col;
-                 const float* val; const float* x; float* y; const int32_t* part; } cc_spmv_args;
+                 const float* val; const float* x; float* y; const int32_t* part;
+                 const int32_t* hot; float* xh; int32_t n_hot; } cc_spmv_args;
 /* CC_K_HIST64 -- 64-bin histogram, the paper's HST (Table 2; data-
  * related); reading R24 (CUDA SDK histogram64):
  *     counts[k] = #{ i < n : data[i] >> 2 == k },  k = 0..63.
@@ -314,6 +324,20 @@ typedef struct { const uint8_t* data; int64_t n; uint32_t* counts; } cc_hist64_a
  * cc_kernel_grid) with the merge-path row coordinate of each logical CTA's
  * first diagonal.  Asynchronous on `stream`. */
 cc_status cc_spmv_partition(const cc_spmv_args* args, int32_t* part, void* stream);
+
+/* Inspector for the data-related class ("a lightweight inspector
+ * kernel before runtime to profile local data access ... in order to predict
+ * global data organization"): find the (up to) max_hot most-referenced
+ * columns of the plain CSR in `args` (args->col, args->cols; n_hot ignored)
+ * and write the hub-column form: hot[slot] = column (DEVICE int32[max_hot]),
+ * col_hot[k] = -(slot+1) for a hub reference, else col[k] (DEVICE int32[nnz];
+ * may not alias col).  scratch: DEVICE int32[cols + 65536 + 2].  Columns with
+ * no reference are never hubs; ties at the degree threshold are taken in an
+ * unspecified order.  *n_hot (HOST) = slots used.  Runs on `stream` and
+ * synchronizes it (one 256 KB degree histogram is read back to pick the
+ * threshold).  Errors: INVALID_ARG (null, max_hot < 0), CUDA. */
+cc_status cc_spmv_inspect(const cc_spmv_args* args, int32_t max_hot, int32_t* hot, int32_t* col_hot,
+                          int32_t* scratch, int32_t* n_hot, void* stream);
 
 /* Listing 3 microbenchmark (section 3.1): `ctas` one-warp CTAs
  * in hardware order; thread 0 of CTA b times one L1-allocating load

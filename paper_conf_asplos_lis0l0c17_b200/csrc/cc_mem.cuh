@@ -127,6 +127,12 @@ __device__ __forceinline__ float ld_cached_issue(const float* p) {
     asm volatile("ld.global.f32 %0, [%1];" : "=f"(v) : "l"(p));
     return v;
 }
+// hub values of the SpMV hub-column form: allocate in L1 and keep (evict_last)
+__device__ __forceinline__ float ld_hot_issue(const float* p) {
+    float v;
+    asm volatile("ld.global.nc.L1::evict_last.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}
 __device__ __forceinline__ int32_t ld_stream_i32_issue(const int32_t* p) {
     int32_t v;
     asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));

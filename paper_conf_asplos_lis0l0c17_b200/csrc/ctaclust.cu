@@ -812,8 +812,17 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         if (x->rows < 0 || x->cols < 0 || x->nnz < 0 || x->nnz > INT32_MAX) return fail(CC_ERR_INVALID_ARG, "spmv sizes");
         if (!x->row_ptr || !x->part || !x->y || (x->nnz && (!x->col || !x->val || !x->x)))
             return fail(CC_ERR_INVALID_ARG, "spmv null pointer");
+        if (x->n_hot < 0 || (x->n_hot > 0 && (!x->hot || !x->xh)))
+            return fail(CC_ERR_INVALID_ARG, "spmv hub-column form: n_hot %d, hot/xh required", x->n_hot);
         if (x->rows) CC_CUDA(cudaMemsetAsync(x->y, 0, sizeof(float) * x->rows, st));
-        s = launch_body<SpmvBody>(c, SpmvParams{x->rows, x->nnz, x->row_ptr, x->col, x->val, x->x, x->y, x->part});
+        if (x->n_hot > 0) {
+            k_spmv_hot_gather<<<std::min(148 * 4, (x->n_hot + 255) / 256), 256, 0, st>>>(x->x, x->hot, x->xh, x->n_hot);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return cuda_fail(e, "spmv hub gather");
+            if (launches) ++*launches;
+        }
+        s = launch_body<SpmvBody>(c, SpmvParams{x->rows, x->nnz, x->row_ptr, x->col, x->val, x->x, x->y, x->part,
+                                                x->n_hot > 0 ? x->xh + x->n_hot : nullptr});
         break;
     }
     case CC_K_HIST64: {
@@ -910,6 +919,44 @@ extern "C" cc_status cc_spmv_partition(const cc_spmv_args* x, int32_t* part, voi
     k_spmv_partition<<<(n + 255) / 256, 256, 0, (cudaStream_t)stream>>>(x->row_ptr, x->rows, x->nnz, gx, part);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "spmv partition");
+    return CC_OK;
+}
+
+extern "C" cc_status cc_spmv_inspect(const cc_spmv_args* x, int32_t max_hot, int32_t* hot, int32_t* col_hot,
+                                     int32_t* scratch, int32_t* n_hot, void* stream) {
+    if (!x || !n_hot || !scratch || max_hot < 0 || (x->nnz && (!x->col || !col_hot)) || (max_hot && !hot))
+        return fail(CC_ERR_INVALID_ARG, "spmv inspect: null argument or max_hot < 0");
+    if (x->cols < 0 || x->nnz < 0 || x->nnz > INT32_MAX) return fail(CC_ERR_INVALID_ARG, "spmv inspect: sizes");
+    *n_hot = 0;
+    cudaStream_t st = (cudaStream_t)stream;
+    const int32_t cols = x->cols;
+    int32_t* deg = scratch;
+    int32_t* hist = scratch + cols;
+    int32_t* ctr = hist + 65536;
+    const int grid = 148 * 8;
+    CC_CUDA(cudaMemsetAsync(scratch, 0, sizeof(int32_t) * ((size_t)cols + 65536 + 2), st));
+    if (x->nnz) k_spmv_col_degree<<<grid, 256, 0, st>>>(x->col, x->nnz, deg);
+    if (cols) k_spmv_deg_hist<<<grid, 256, 0, st>>>(deg, cols, hist);
+    std::vector<int32_t> h(65536);
+    CC_CUDA(cudaMemcpyAsync(h.data(), hist, sizeof(int32_t) * 65536, cudaMemcpyDeviceToHost, st));
+    CC_CUDA(cudaStreamSynchronize(st));
+    // threshold t >= 1: every column with degree > t is a hub (`above` of
+    // them, <= max_hot) and columns of degree t fill the remaining slots; t = 0:
+    // every referenced column fits (unreferenced ones are never hubs)
+    int64_t above = 0;
+    int32_t t = 65535;
+    for (; t >= 1; --t) {
+        if (above + h[t] > max_hot) break;
+        above += h[t];
+    }
+    if (t < 0) t = 0;
+    const int32_t used = (int32_t)std::min<int64_t>(above + (t >= 1 ? h[t] : 0), max_hot);
+    k_spmv_hot_assign<<<grid, 256, 0, st>>>(deg, cols, t, (int32_t)above, max_hot, ctr, hot);
+    if (x->nnz) k_spmv_col_encode<<<grid, 256, 0, st>>>(x->col, x->nnz, deg, col_hot);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "spmv inspect");
+    CC_CUDA(cudaStreamSynchronize(st));
+    *n_hot = used;
     return CC_OK;
 }
 

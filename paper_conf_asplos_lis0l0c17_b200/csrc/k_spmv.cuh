@@ -27,7 +27,52 @@ struct SpmvParams {
     int32_t rows; int64_t nnz;
     const int32_t* row_ptr; const int32_t* col; const float* val; const float* x; float* y;
     const int32_t* part;   // part[b] = row coordinate of diagonal b*IPC
+    const float* xh_end;   // hub-column form: one past the gathered hub values (col -(k+1) -> xh_end[-(k+1)])
 };
+
+// Hub gather of the hub-column form (cc_spmv_inspect): xh[n_hot-1-k] = x[hot[k]].
+__global__ void k_spmv_hot_gather(const float* __restrict__ x, const int32_t* __restrict__ hot, float* xh,
+                                  int32_t n_hot) {
+    for (int32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < n_hot; k += gridDim.x * blockDim.x)
+        xh[n_hot - 1 - k] = x[hot[k]];
+}
+
+// ---- inspector (cc_spmv_inspect) ---------------------------------------------
+// references per column
+__global__ void k_spmv_col_degree(const int32_t* __restrict__ col, int64_t nnz, int32_t* deg) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz; k += (int64_t)gridDim.x * blockDim.x)
+        atomicAdd(deg + col[k], 1);
+}
+// histogram of min(degree, 65535)
+__global__ void k_spmv_deg_hist(const int32_t* __restrict__ deg, int32_t cols, int32_t* hist) {
+    for (int32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cols; c += gridDim.x * blockDim.x) {
+        const int32_t d = deg[c];
+        atomicAdd(hist + (d < 65535 ? d : 65535), 1);
+    }
+}
+// slot per hub column (degree > t, or == t while slots remain), -1 otherwise;
+// deg[] is overwritten with the slot id.  ctr[0]: hubs above t, ctr[1]: ties.
+__global__ void k_spmv_hot_assign(int32_t* deg, int32_t cols, int32_t t, int32_t n_gt, int32_t max_hot,
+                                  int32_t* ctr, int32_t* hot) {
+    for (int32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < cols; c += gridDim.x * blockDim.x) {
+        const int32_t d = deg[c] < 65535 ? deg[c] : 65535;
+        int32_t slot = -1;
+        if (d > t && d > 0) slot = atomicAdd(ctr, 1);
+        else if (d == t && d > 0) {
+            const int32_t e = atomicAdd(ctr + 1, 1);
+            if (n_gt + e < max_hot) slot = n_gt + e;
+        }
+        deg[c] = slot;
+        if (slot >= 0) hot[slot] = c;
+    }
+}
+__global__ void k_spmv_col_encode(const int32_t* __restrict__ col, int64_t nnz, const int32_t* __restrict__ slot,
+                                  int32_t* col_hot) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nnz; k += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t c = col[k], sl = slot[c];
+        col_hot[k] = sl >= 0 ? -(sl + 1) : c;
+    }
+}
 
 #ifndef CC_SPMV_IPT
 #define CC_SPMV_IPT 16
@@ -142,7 +187,12 @@ struct SpmvBody {
                     v[k] = ld_stream_f32_issue(p.val + y0 + (ok ? j : 0));
                 }
 #pragma unroll
-                for (int k = 0; k < SPMV_GB; ++k) xv[k] = ld_cached_issue(p.x + c[k]);
+                for (int k = 0; k < SPMV_GB; ++k) {
+                    // hub references (negative, hub-column form) read the dense
+                    // hub array, which stays in L1; others gather x
+                    if (c[k] >= 0) xv[k] = ld_cached_issue(p.x + c[k]);
+                    else xv[k] = ld_hot_issue(p.xh_end + c[k]);
+                }
 #pragma unroll
                 for (int k = 0; k < SPMV_GB; ++k) {
                     const int32_t j = t + (k0 + k) * kConsumers;
@@ -159,7 +209,8 @@ struct SpmvBody {
                 if (j < nz) {
                     const int32_t c = hf ? ld_stream_i32_h(p.col + y0 + j, pf) : ld_stream_i32(p.col + y0 + j);
                     const float v = hf ? ld_stream_f32_h(p.val + y0 + j, pf) : ld_stream_f32(p.val + y0 + j);
-                    s_prod[j + j / SPMV_IPT] = v * (hl ? ld_cached_h(p.x + c, pl) : ld_cached(p.x + c));
+                    const float* xp = c >= 0 ? p.x + c : p.xh_end + c;
+                    s_prod[j + j / SPMV_IPT] = v * (hl ? ld_cached_h(xp, pl) : ld_cached(xp));
                 }
             }
         }

@@ -34,7 +34,7 @@ STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_E
 # every symbol include/ctaclust.h declares (checked by tests/test_abi.py)
 EXPORTS = ["cc_plan_create", "cc_plan_destroy", "cc_plan_info", "cc_plan_table", "cc_plan_lookup",
            "cc_plan_invert", "cc_device_info", "cc_sm_rank_table", "cc_launch_opts_default",
-           "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_l1_reuse_probe", "cc_comm_unique_id",
+           "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_spmv_inspect", "cc_l1_reuse_probe", "cc_comm_unique_id",
            "cc_comm_init", "cc_comm_destroy", "cc_halo_exchange", "cc_allreduce_sum", "cc_allgather",
            "cc_peer_access", "cc_ipc_handle", "cc_ipc_open", "cc_ipc_close", "cc_status_string", "cc_last_error", "cc_last_cuda_error", "cc_version"]
 
@@ -97,7 +97,7 @@ class Conv2dArgs(ctypes.Structure):
 
 class SpmvArgs(ctypes.Structure):
     _fields_ = [("rows", _i32), ("cols", _i32), ("nnz", _i64), ("row_ptr", _vp), ("col", _vp), ("val", _vp),
-                ("x", _vp), ("y", _vp), ("part", _vp)]
+                ("x", _vp), ("y", _vp), ("part", _vp), ("hot", _vp), ("xh", _vp), ("n_hot", _i32)]
 
 
 _lib = None
@@ -349,6 +349,15 @@ def l1_reuse_probe(ctas: int, stagger_cycles: int, inp, smid, ticks, sink, strea
 
 def spmv_partition(args: SpmvArgs, part, stream=None):
     _check(lib().cc_spmv_partition(ctypes.byref(args), _vp(part.data_ptr()), _vp(_stream(stream))))
+
+
+def spmv_inspect(args: SpmvArgs, max_hot: int, hot, col_hot, scratch, stream=None) -> int:
+    """cc_spmv_inspect: hub columns of the plain CSR in `args` into `hot` and the
+    encoded column array `col_hot` (device tensors); returns the slots used."""
+    n = _i32()
+    _check(lib().cc_spmv_inspect(ctypes.byref(args), _i32(max_hot), _vp(_ptr(hot)), _vp(_ptr(col_hot)),
+                                 _vp(scratch.data_ptr()), ctypes.byref(n), _vp(_stream(stream))))
+    return n.value
 
 
 # ---- multi-GPU exchange steps (NCCL, one process per GPU) ---------------------

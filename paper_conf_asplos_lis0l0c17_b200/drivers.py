@@ -244,7 +244,7 @@ class JacobiSlab:
         L = self.lhi - self.llo
         dev = self.dev = torch.device(device)
         ld = (cols + 3) & ~3
-        self.u0 = synth.matrix(4, L, cols, backend="torch", device=dev, row0=self.llo)
+        self.u0 = synth.matrix(4, L, cols, backend="torch", device=dev, row0=self.llo, ld=ld)[:, :cols]
         self.a = torch.zeros(L, ld, device=dev)[:, :cols]
         self.b = torch.zeros(L, ld, device=dev)[:, :cols]
         own0, own1 = self.lo - self.llo, self.hi - self.llo
@@ -326,10 +326,40 @@ class JacobiSlab:
         return 8 * self.rows * self.cols * self.iters
 
 
+class GraphStep:
+    """Mixin: capture one step (all its launches and exchanges) into a CUDA
+    graph and replay it -- removes the host-side marshalling of each call from
+    the timed region.  The first (eager) step creates the plans and tensor
+    maps; nothing is allocated during capture."""
+    graph = None
+
+    def capture(self, opts: dict) -> bool:
+        if not self.x.capturable:
+            return False
+        self.graph = None
+        self.step(opts)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream(device=self.dev)
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            with torch.cuda.graph(g, stream=s):
+                n = self.step(opts)
+        torch.cuda.current_stream().wait_stream(s)
+        self.graph, self.graph_launches = g, n
+        return True
+
+    def step(self, opts: dict, stream=None) -> int:
+        if self.graph is not None:
+            self.graph.replay()
+            return self.graph_launches
+        return self.step_eager(opts, stream)
+
+
 # ----------------------------------------------------------------------------
 # config 4: conv2d, slab-sharded
 # ----------------------------------------------------------------------------
-class ConvSlab:
+class ConvSlab(GraphStep):
     """This rank's slab (owned rows + R halo rows per side) of the rows x cols
     image (seed 5), filter seed 6 normalised to sum 1.  One step =
     the halo exchange (world > 1) + one conv launch; owned output rows are
@@ -346,8 +376,10 @@ class ConvSlab:
             w = synth.uniform(6, K * K).reshape(K, K)
             w = (w / w.astype(np.float64).sum()).astype(np.float32)
         self.w = w
-        self.inp = synth.matrix(5, self.lhi - self.llo, cols, backend="torch", device=dev, row0=self.llo)
-        self.out = torch.empty_like(self.inp)
+        ld = (cols + 3) & ~3                       # 16-byte rows (TMA strides, float4 access)
+        self.inp = synth.matrix(5, self.lhi - self.llo, cols, ld=ld, backend="torch", device=dev,
+                                row0=self.llo)[:, :cols]
+        self.out = torch.empty(self.lhi - self.llo, ld, device=dev)[:, :cols]
 
     def inputs(self) -> dict:
         return dict(inp=self.inp)
@@ -355,7 +387,7 @@ class ConvSlab:
     def outputs(self) -> dict:
         return dict(out=self.result())
 
-    def step(self, opts: dict, stream=None) -> int:
+    def step_eager(self, opts: dict, stream=None) -> int:
         self.x.halo_exchange(self.inp, self.R, stream)
         args, self._w = cc.conv2d_args(self.inp, self.out, self.w)
         return _launch("conv2d", args, opts, stream)
@@ -373,12 +405,12 @@ class ConvSlab:
 # ----------------------------------------------------------------------------
 # config 5: CSR SpMV, nnz-balanced row blocks
 # ----------------------------------------------------------------------------
-class SpmvBlock:
+class SpmvBlock(GraphStep):
     """This rank's nnz-balanced row block of the R-MAT matrix (seed 7, values
     seed 8, x seed 9).  x is replicated; one step = local SpMV + all-gather of
     y (blocks padded to the largest)."""
 
-    def __init__(self, scale: int, xchg: Exchange, device, edge_factor: int = 16):
+    def __init__(self, scale: int, xchg: Exchange, device, edge_factor: int = 16, hot: int = 0):
         self.x = xchg
         dev = self.dev = torch.device(device)
         rp, col = synth.rmat_csr(7, scale, edge_factor, backend="torch", device=dev)
@@ -392,7 +424,7 @@ class SpmvBlock:
             del rp, col, val
         else:
             lrp, lcol, lval = rp, col, val
-        self.A = ops.SpmvMatrix(lrp, lcol, lval, n_cols=self.rows)
+        self.A = ops.SpmvMatrix(lrp, lcol, lval, n_cols=self.rows, hot=hot)
         self.local_nnz = lcol.numel()
         self.cap = self._cap(xchg)
         self.y = torch.zeros(self.cap, device=dev)
@@ -406,7 +438,7 @@ class SpmvBlock:
             n = h
         return int(n.item())
 
-    def step(self, opts: dict, stream=None) -> int:
+    def step_eager(self, opts: dict, stream=None) -> int:
         nl = _launch_spmv(self.A, self.xv, self.y, opts, stream)
         if self.x.world > 1:
             self.x.allgather(self.y, self.yall, stream)
@@ -417,6 +449,4 @@ class SpmvBlock:
 
 
 def _launch_spmv(Am, x, y, opts, stream):
-    args = cc.SpmvArgs(Am.rows, Am.cols, Am.col.numel(), Am.row_ptr.data_ptr(), Am.col.data_ptr(),
-                       Am.val.data_ptr(), x.data_ptr(), y.data_ptr(), Am.part.data_ptr())
-    return _launch("spmv", args, opts, stream)
+    return _launch("spmv", Am.args(x, y), opts, stream)

@@ -122,25 +122,42 @@ def conv2d(inp, w, out=None, backend="agent", order=None, tile=None, num_cluster
 
 
 class SpmvMatrix:
-    """A CSR matrix resident on the device plus its merge-path split table."""
+    """A CSR matrix resident on the device plus its merge-path split table.
 
-    def __init__(self, row_ptr, col, val, n_cols=None, stream=None):
+    hot = H > 0 runs the inspector (cc_spmv_inspect) once: the H most
+    referenced columns become hub slots, `col_kernel` holds the encoded
+    column array and every launch gathers the hub values into a dense array
+    read through L1 (the hub-column form of cc_spmv_args)."""
+
+    def __init__(self, row_ptr, col, val, n_cols=None, stream=None, hot: int = 0):
         self.row_ptr, self.col, self.val = row_ptr, col, val
         self.rows = row_ptr.numel() - 1
         self.cols = self.rows if n_cols is None else n_cols
-        x = torch.empty(0, device=row_ptr.device)
+        dev = row_ptr.device
+        x = torch.empty(0, device=dev)
         probe = cc.SpmvArgs(self.rows, self.cols, col.numel(), row_ptr.data_ptr(), col.data_ptr(),
                             val.data_ptr(), x.data_ptr(), x.data_ptr(), None)
         gx, _ = cc.kernel_grid("spmv", probe)
-        self.part = torch.empty(gx + 1, dtype=torch.int32, device=row_ptr.device)
+        self.part = torch.empty(gx + 1, dtype=torch.int32, device=dev)
         cc.spmv_partition(probe, self.part, stream)
+        self.col_kernel, self.hot, self.xh, self.n_hot = col, None, None, 0
+        if hot > 0:
+            self.hot = torch.empty(hot, dtype=torch.int32, device=dev)
+            self.col_kernel = torch.empty_like(col)
+            scratch = torch.empty(self.cols + 65536 + 2, dtype=torch.int32, device=dev)
+            self.n_hot = cc.spmv_inspect(probe, hot, self.hot, self.col_kernel, scratch, stream)
+            self.xh = torch.empty(max(self.n_hot, 1), dtype=torch.float32, device=dev)
+
+    def args(self, x, y) -> cc.SpmvArgs:
+        return cc.SpmvArgs(self.rows, self.cols, self.col.numel(), self.row_ptr.data_ptr(),
+                           self.col_kernel.data_ptr(), self.val.data_ptr(), x.data_ptr(), y.data_ptr(),
+                           self.part.data_ptr(), None if self.hot is None else self.hot.data_ptr(),
+                           None if self.xh is None else self.xh.data_ptr(), self.n_hot)
 
 
 def spmv(Amat: SpmvMatrix, x, y=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
     y = torch.empty(Amat.rows, dtype=torch.float32, device=x.device) if y is None else y
-    args = cc.SpmvArgs(Amat.rows, Amat.cols, Amat.col.numel(), Amat.row_ptr.data_ptr(), Amat.col.data_ptr(),
-                       Amat.val.data_ptr(), x.data_ptr(), y.data_ptr(), Amat.part.data_ptr())
-    _launch("spmv", args, backend, order, tile, num_clusters, _dev(x), stream, **kw)
+    _launch("spmv", Amat.args(x, y), backend, order, tile, num_clusters, _dev(x), stream, **kw)
     return y
 
 

@@ -1,0 +1,69 @@
+#!/usr/bin/env python
+"""Round-2 A/B experiments (one box, graph-timed like bench_suite):
+  spmv   hub-column form (inspector slots 0 / 4K / 16K / 32K / 64K) x backends
+  stencil TILE(2, h) orders (vertical runs of merged pairs) vs ROW / identity / default
+    python scripts/exp_r10.py spmv|stencil out.json
+"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import bench_suite as B  # noqa: E402
+
+
+def spmv():
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    rp, col = synth.rmat_csr(7, 24, 16, backend="torch", device="cuda")
+    n, nnz = rp.numel() - 1, col.numel()
+    val = synth.uniform(8, nnz, backend="torch", device="cuda")
+    x = synth.uniform(9, n, backend="torch", device="cuda")
+    y = torch.empty(n, device="cuda")
+    nbytes = 8 * nnz + 4 * (n + 1) + 8 * n
+    out = {}
+    for hot in (0, 4096, 16384, 32768, 65536):
+        Am = ops.SpmvMatrix(rp, col, val, hot=hot)
+        variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
+                    ("identity", dict(backend="identity")),
+                    ("static-row-m5", dict(backend="static", order="row", num_clusters=5 * 148))]
+        r = B.measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 20, nbytes, graph=True, inner=B.GRAPH_INNER)
+        out[f"hot{hot}"] = r
+        print(hot, [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+        del Am
+        torch.cuda.empty_cache()
+    return out
+
+
+def stencil():
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    out = {}
+    N = 8192
+    img = synth.matrix(5, N, N, backend="torch", device="cuda")
+    o = torch.empty_like(img)
+    w = synth.uniform(6, 9).reshape(3, 3)
+    w = (w / w.astype(np.float64).sum()).astype(np.float32)
+    tiles = [(2, 2), (2, 4), (2, 8), (2, 16), (4, 4)]
+    variants = [("default", dict(backend="default")), ("default-direct", dict(backend="default", staging="direct")),
+                ("identity", dict(backend="identity")), ("agent-row", dict(backend="agent", order="row"))] + \
+               [(f"agent-tile{tw}x{th}", dict(backend="agent", order="tile", tile=(tw, th))) for tw, th in tiles]
+    r = B.measure(variants, lambda kw: ops.conv2d(img, w, out=o, **kw), 20, 8 * N * N, graph=True, inner=B.GRAPH_INNER)
+    out["conv3"] = r
+    print("conv3", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    del img, o
+    M = 16384
+    a = synth.matrix(4, M, M, backend="torch", device="cuda")
+    b = a.clone()
+    r = B.measure(variants, lambda kw: ops.jacobi5(a, b, 2, **kw), 10, 2 * 8 * M * M, graph=True, inner=5)
+    out["jacobi"] = r
+    print("jacobi", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    return out
+
+
+if __name__ == "__main__":
+    what, path = sys.argv[1], sys.argv[2]
+    res = spmv() if what == "spmv" else stencil()
+    json.dump(res, open(path, "w"), indent=1)

@@ -30,6 +30,7 @@ def main():
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--warm", type=int, default=1)
     ap.add_argument("--scale", type=int, default=24)
+    ap.add_argument("--hot", type=int, default=0, help="spmv: hub-column form with this many hub slots")
     ap.add_argument("--small", action="store_true",
                     help="reduced problem (categorizer probe, P:2275): n/4 matrices, scale-18 SpMV")
     a = ap.parse_args()
@@ -79,7 +80,7 @@ def main():
         rp, col = synth.rmat_csr(7, 18 if a.small else a.scale, 16, backend="torch", device=dev)
         val = synth.uniform(8, col.numel(), backend="torch", device=dev)
         x = synth.uniform(9, rp.numel() - 1, backend="torch", device=dev)
-        Am = ops.SpmvMatrix(rp, col, val)
+        Am = ops.SpmvMatrix(rp, col, val, hot=a.hot)
         y = torch.empty(rp.numel() - 1, device=dev)
         if a.backend == "cusparse":          # vendor library, for context only
             Acsr = torch.sparse_csr_tensor(rp, col, val, (rp.numel() - 1, rp.numel() - 1))

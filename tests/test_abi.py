@@ -47,8 +47,8 @@ int main(void) {
   S(cc_launch_opts) O(cc_launch_opts, d_census) O(cc_launch_opts, d_map) O(cc_launch_opts, l2_hint) O(cc_launch_opts, carveout)
   S(cc_matvec_args) O(cc_matvec_args, y) S(cc_atax_args) O(cc_atax_args, y)
   S(cc_bicg_args) O(cc_bicg_args, s) S(cc_mvt_args) O(cc_mvt_args, x2)
-  S(cc_jacobi5_args) O(cc_jacobi5_args, result_is_b) S(cc_conv2d_args) O(cc_conv2d_args, w)
-  S(cc_spmv_args) O(cc_spmv_args, part) O(cc_spmv_args, nnz)
+  S(cc_jacobi5_args) O(cc_jacobi5_args, result_is_b) O(cc_jacobi5_args, row_hi) S(cc_conv2d_args) O(cc_conv2d_args, w)
+  S(cc_spmv_args) O(cc_spmv_args, part) O(cc_spmv_args, nnz) O(cc_spmv_args, xh) O(cc_spmv_args, n_hot)
   S(cc_hist64_args) O(cc_hist64_args, n) O(cc_hist64_args, counts)
   S(cc_jacobi5_halo_args) O(cc_jacobi5_halo_args, sweep0) O(cc_jacobi5_halo_args, ll)
   O(cc_jacobi5_halo_args, dn_ll) O(cc_jacobi5_halo_args, status)

@@ -388,6 +388,43 @@ def test_spmv(v):
                               O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), vi, xi)), name
 
 
+@pytest.mark.parametrize("hot", [1, 64, 100000])
+def test_spmv_hub_form(hot):
+    """Hub-column form (cc_spmv_inspect, P:1925 inspector): the inspector picks
+    the most-referenced columns (every hub's degree >= every other column's),
+    the encoding decodes back to col, and y has the plain form's bits under
+    every backend (same products, same order) and matches the oracle."""
+    for name, rp, col, n in _edge_matrices():
+        val = synth.uniform(8, len(col))
+        x = synth.uniform(9, n)
+        plain = _csr_dev(rp, col, val)
+        Am = ops.SpmvMatrix(plain.row_ptr, plain.col, plain.val, hot=hot)
+        deg = np.bincount(col, minlength=n) if len(col) else np.zeros(n, np.int64)
+        hubs = Am.hot[: Am.n_hot].cpu().numpy()
+        assert Am.n_hot == min(hot, int(np.count_nonzero(deg))), name
+        assert len(set(hubs.tolist())) == Am.n_hot
+        if Am.n_hot:
+            rest = np.setdiff1d(np.arange(n), hubs)
+            assert deg[hubs].min() >= (deg[rest].max() if rest.size else 0), name
+        enc = Am.col_kernel.cpu().numpy()
+        dec = enc.copy()
+        neg = enc < 0
+        dec[neg] = hubs[-enc[neg] - 1]
+        assert np.array_equal(dec, col), name
+        ref = O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), val, x)
+        for v in (dict(backend="default"), dict(backend="agent", order="row"), dict(backend="identity"),
+                  dict(backend="static", order="row", num_clusters=740), dict(backend="agent", l2_hint="both")):
+            y0 = ops.spmv(plain, dev(x), **v)
+            y1 = ops.spmv(Am, dev(x), **v)
+            torch.cuda.synchronize()
+            got = y1.cpu().numpy()
+            nz = ref != 0
+            assert np.all(got[~nz] == 0), (name, v)
+            assert relerr(got[nz], ref[nz]) <= TOL, (name, v)
+            if v["backend"] in ("default", "static"):     # deterministic schedules: the same bits
+                assert np.array_equal(got, y0.cpu().numpy()), (name, v)
+
+
 def test_spmv_full_size_sampled():
     """Config 5 at full size (R-MAT scale 24, edge factor 16, ~263 M nnz) in the
     bench suite's launch configs: 3000 sampled rows plus the 20 heaviest rows
@@ -408,8 +445,11 @@ def test_spmv_full_size_sampled():
     sub_col = col[idx].cpu().numpy()
     sub_val = val[idx].cpu().numpy()
     ref = O.spmv_csr(sub_rp.astype(np.int32), sub_col.astype(np.int32), sub_val, x.cpu().numpy())
-    for v in (dict(backend="default"), dict(backend="agent", order="row"), dict(backend="identity")):
-        y = ops.spmv(Am, x, **v)
+    Ah = ops.SpmvMatrix(rp, col, val, hot=16384)
+    for M, v in ((Am, dict(backend="default")), (Am, dict(backend="agent", order="row")),
+                 (Am, dict(backend="identity")), (Ah, dict(backend="agent", order="row")),
+                 (Ah, dict(backend="default"))):
+        y = ops.spmv(M, x, **v)
         torch.cuda.synchronize()
         got = y[torch.from_numpy(rows).cuda()].cpu().numpy()
         nz = ref != 0

@@ -31,15 +31,23 @@ def rel(got, ref):
 
 
 # ---------------------------------------------------------------- row windows
+def padded(u0, fill=0.0):
+    """device copy with a 16-byte leading dimension (ragged widths keep ld % 4 == 0)"""
+    rows, cols = u0.shape
+    t = torch.full((rows, (cols + 3) & ~3), fill, device="cuda")[:, :cols]
+    t.copy_(torch.from_numpy(np.ascontiguousarray(u0)))
+    return t
+
+
 @pytest.mark.parametrize("backend,order", [("agent", "row"), ("default", None), ("identity", None),
                                            ("static", "row"), ("agent", "tile")])
 @pytest.mark.parametrize("rows,cols,win", [(130, 100, (1, 33)), (130, 100, (33, 97)), (130, 100, (97, 130)),
                                             (130, 100, (0, 130)), (77, 45, (5, 6)), (77, 45, (0, 40))])
 def test_jacobi_row_window(backend, order, rows, cols, win):
     u0 = synth.matrix(4, rows, cols)
-    a = torch.from_numpy(u0).cuda()
+    a = padded(u0)
     sentinel = np.float32(-7.0)
-    b = torch.full_like(a, float(sentinel))
+    b = padded(np.full_like(u0, sentinel))
     kw = dict(backend=backend)
     if order:
         kw["order"] = order
@@ -59,8 +67,8 @@ def test_jacobi_windows_compose_to_full_sweep():
     """boundary windows + interior window = the full sweep, several sweeps"""
     rows, cols, T = 200, 130, 5
     u0 = synth.matrix(4, rows, cols)
-    a = torch.from_numpy(u0).cuda()
-    b = a.clone()
+    a = padded(u0)
+    b = padded(u0)
     wins = [(0, 32), (168, 200), (32, 168)]
     for k in range(T):
         src, dst = (a, b) if k % 2 == 0 else (b, a)
@@ -159,8 +167,8 @@ WORKER = textwrap.dedent("""
         m = inner != 0
         ok = bool(np.all(got[~m] == 0)) and rel(got[m], inner[m]) <= 1e-4
         info = str(rel(got[m], inner[m]))
-    elif cfg == "spmv":
-        d = drivers.SpmvBlock(10, X, "cuda")
+    elif cfg.startswith("spmv"):
+        d = drivers.SpmvBlock(10, X, "cuda", hot=64 if cfg == "spmv-hot" else 0)
         d.step(dict(backend="agent", order="row", max_agents=1))
         torch.cuda.synchronize()
         rp, col = synth.rmat_csr(7, 10, 16)
@@ -188,7 +196,7 @@ def _port():
 
 @pytest.mark.parametrize("cfg,world", [("atax", 2), ("atax", 4), ("jacobi", 2), ("jacobi", 3), ("jacobi", 4),
                                        ("jacobi-nooverlap", 3), ("conv1", 2), ("conv3", 3), ("spmv", 2),
-                                       ("spmv", 3)])
+                                       ("spmv", 3), ("spmv-hot", 2)])
 def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     script = tmp_path / "w.py"
     script.write_text(WORKER.format(root=ROOT))
