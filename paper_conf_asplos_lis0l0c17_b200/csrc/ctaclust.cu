@@ -592,14 +592,15 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     if (g.V == 0) return CC_OK;
     const int C = c.o->cluster_size;
     if (C != 1 && C != 2 && C != 4 && C != 8) return fail(CC_ERR_INVALID_ARG, "cluster_size %d (1, 2, 4 or 8)", C);
-    CUtensorMap m_rows, m_halo;
-    CC_TRY(make_tmap(&m_rows, prm.in, prm.rows, prm.cols, prm.ld, TBC_COLS, 32));
-    CC_TRY(make_tmap(&m_halo, prm.in, prm.rows, prm.cols, prm.ld, TBC_COLS, TBC_HALO));
+    using G = TbcGeom<R, tbc_tw<R>()>;
+    CUtensorMap m_c, m_b;
+    CC_TRY(make_tmap(&m_c, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, 32 - 2 * R));
+    CC_TRY(make_tmap(&m_b, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, 2 * R));
     Sched s{};
     s.g = g;
     s.census = c.o->d_census;
     s.exec_sm = c.o->d_exec_sm;
-    const size_t smem = tbc_smem_bytes(C);
+    const size_t smem = tbc_smem_bytes<R>();
     CC_CUDA(cudaFuncSetAttribute(k_conv_tbc<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     CC_CUDA(cudaFuncSetAttribute(k_conv_tbc<R>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1));
     cudaLaunchConfig_t cfg = {};
@@ -614,14 +615,15 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     cfg.attrs = at;
     cfg.numAttrs = 1;
     // persistent: as many clusters as can be co-resident (not more than units)
-    const long units = (long)g.gx * ((g.gy + C - 1) / C);
+    const int TW = tbc_tw<R>();
+    const long units = (long)((g.gx + TW - 1) / TW) * ((g.gy + C - 1) / C);
     cfg.gridDim = dim3(C);
     int nc = 0;
     CC_CUDA(cudaOccupancyMaxActiveClusters(&nc, k_conv_tbc<R>, &cfg));
     if (nc < 1) return fail(CC_ERR_UNSUPPORTED, "tbcluster: no cluster of %d fits", C);
     if (nc > units) nc = (int)units;
     cfg.gridDim = dim3(nc * C);
-    CC_CUDA(cudaLaunchKernelEx(&cfg, k_conv_tbc<R>, m_rows, m_halo, s, prm, (int32_t)C));
+    CC_CUDA(cudaLaunchKernelEx(&cfg, k_conv_tbc<R>, m_c, m_b, s, prm, (int32_t)C));
     if (c.nl) ++*c.nl;
     return CC_OK;
 }

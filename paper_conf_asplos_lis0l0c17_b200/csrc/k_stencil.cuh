@@ -455,11 +455,17 @@ struct ConvParams { CUtensorMap tmap; CUtensorMap tmap2; SplitMaps split; const 
 // reads per output by 33 % (3x3) / 43 % (7x7) -- the conv is otherwise
 // shared-memory-bandwidth bound.  The summation order per output is the
 // filter's row-major tap order, as in the oracle.
-template <int R, int RB = 1>
-__device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const float* rows_base,
-                                                  int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0,
-                                                  int pitch = ST_COLS) {
-    // rows_base points at the staged row holding input row y0 - R, column x0 - 4
+// Staged rows as one contiguous box: row rr (input row y0 - R + rr) at base + rr * pitch.
+struct ContigRows {
+    const float* base;
+    int pitch;
+    __device__ __forceinline__ const float* operator()(int rr) const { return base + rr * pitch; }
+};
+
+template <int R, int RB = 1, class RowPtr>
+__device__ __forceinline__ void conv_tile_compute_rows(const ConvParams<R>& p, const RowPtr& rowp,
+                                                       int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0) {
+    // rowp(rr) points at the staged row holding input row y0 - R + rr, column x0 - 4
     constexpr int K = 2 * R + 1;
     const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
     const int gx = bx * 32 + 4 * c4;
@@ -470,7 +476,7 @@ __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const 
         for (int e = 0; e < 4; ++e) acc[j][e] = 0.f;
 #pragma unroll
     for (int ir = 0; ir < K + RB - 1; ++ir) {           // staged rows r0 .. r0+K+RB-2
-        const float4* row = reinterpret_cast<const float4*>(rows_base + (r0 + ir) * pitch + 4 * c4);
+        const float4* row = reinterpret_cast<const float4*>(rowp(r0 + ir) + 4 * c4);
         float4 q0 = row[0], q1 = row[1], q2 = row[2];
         const float win[12] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w, q2.x, q2.y, q2.z, q2.w};
 #pragma unroll
@@ -516,6 +522,13 @@ __device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const 
         o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[j][3] : 0.f;
         store4_out(p.out + (int64_t)gy * p.ld + gx, o, gx, p.cols, l2_hint);
     }
+}
+
+template <int R, int RB = 1>
+__device__ __forceinline__ void conv_tile_compute(const ConvParams<R>& p, const float* rows_base,
+                                                  int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0,
+                                                  int pitch = ST_COLS) {
+    conv_tile_compute_rows<R, RB>(p, ContigRows{rows_base, pitch}, bx, by, ctid, l2_hint);
 }
 
 template <int R>

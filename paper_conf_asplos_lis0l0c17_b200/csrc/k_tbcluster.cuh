@@ -1,25 +1,45 @@
 // k_tbcluster.cuh -- thread-block-cluster backend for conv2d: the hardware
-// form of CTA clustering on Blackwell (BASELINE.json north_star "a second
+// form of CTA clustering on Blackwell (BASELINE.json north_star: "a second
 // backend uses Blackwell thread-block clusters (__cluster_dims__) with DSMEM
-// and TMA").
+// and TMA multicast").
 //
 // A cluster of C CTAs (cluster dims (C,1,1)) is co-scheduled by the hardware
 // on one GPC -- clustering with no software binding at all.  Clusters are
-// persistent: cluster c processes the "units" c, c + NC, c + 2 NC, ... where a
-// unit is C vertically adjacent output tiles (bx, C*ub .. C*ub + C-1) and units
-// are numbered row-major (ub, bx).  Per unit, CTA k of the cluster
-//   1. TMA-loads only its own 32 centre rows (40 columns, x0-4 .. x0+35) into
-//      one of two shared-memory buffers (the next unit's load overlaps the
-//      current unit's compute); the cluster's outermost CTAs also load the
-//      8-row box above / below the cluster;
-//   2. tells its neighbours its rows have landed (remote mbarrier arrive),
-//      waits for theirs, and copies its R-row halos -- the inter-CTA reuse --
-//      straight out of the neighbours' shared memory over DSMEM;
-//   3. tells its neighbours it is done reading (remote arrive), so they may
-//      refill that buffer two units later, and computes its tile.
-// Inside a cluster no halo row is fetched from L2 twice and no cluster-wide
-// barrier is needed per unit.  (cluster.sync emits CCTL.IVALL; this backend
-// carries its reuse in shared memory, so that is irrelevant anyway.)
+// persistent: cluster c processes the units c, c + NC, c + 2 NC, ... where a
+// unit is C vertically adjacent output tile rows of TW horizontally adjacent
+// 32 x 32 tiles (CTA k of the cluster computes tile row C*ub + k).
+//
+// The inter-CTA reuse -- the 2R input rows straddling the boundary between
+// vertically adjacent tiles, which both tiles read -- is fetched from L2
+// ONCE per cluster and delivered to both CTAs by one TMA multicast
+// (cp.async.bulk.tensor ... .multicast::cluster, ctaMask = the two CTAs).
+// Each CTA's stage holds three regions:
+//     X[0], X[1]   2R-row boundary boxes
+//     C            its 32 - 2R interior rows (a plain TMA load, itself only)
+// The boundary between CTA b and b+1 lands in region X[b & 1] of BOTH CTAs
+// (a multicast writes the same shared-memory offset in every destination),
+// which is CTA b's bottom and CTA b+1's top boundary; CTA k therefore reads
+// its top boundary from X[(k-1) & 1] and its bottom one from X[k & 1], and the
+// tile code maps each staged row to its region (ParityRows).  The cluster's
+// outermost boundaries are loaded by CTA 0 / CTA C-1 for themselves.
+//
+// Pipeline (per CTA, S stages, warp-specialised like the agents):
+//   warp 0 lane 0 (producer)  for stage s of unit i: wait empty[s] (this CTA
+//     and CTA k+1 -- the other receiver of its multicast -- released the
+//     stage), arm full[s] with the bytes this CTA receives, issue its
+//     interior load and its bottom-boundary multicast (CTA 0 also its top);
+//   consumer warps            wait full[s], compute, then release the stage:
+//     a local arrive on empty[s] and a remote arrive on CTA k-1's empty[s]
+//     (mbarrier.arrive.release.cluster; the producer waits with
+//     .acquire.cluster) -- the WAR order between this CTA's shared-memory
+//     reads and its neighbour's next multicast into them.
+// No CTA reads another's shared memory: all data arrives by TMA and is
+// observed through the CTA's own full barrier (complete_tx), the standard
+// async-proxy pattern.  A multicast may complete_tx on a peer's full[s]
+// before the peer armed it (the transaction count goes transiently
+// negative); it cannot target an earlier phase, since the issuer waited for
+// the peer's release of that stage, which follows the peer's consumption of
+// the stage's previous phase.
 #pragma once
 #include <cuda.h>
 #include "cc_mem.cuh"
@@ -28,23 +48,25 @@
 
 namespace cc {
 
-constexpr int TBC_COLS = ST_COLS;       // staged columns per row (x0-4 .. x0+35)
-constexpr int TBC_ROW_BYTES = TBC_COLS * 4;
-#ifndef CC_TBC_HALO
-#define CC_TBC_HALO 8
-#endif
-// halo box height: a multiple of 4 rows (4 x 160 B = 5 x 128 B) keeps every
-// TMA destination 128-B aligned; >= R
-constexpr int TBC_HALO = CC_TBC_HALO;
-static_assert(TBC_HALO % 4 == 0 && TBC_HALO >= 3, "halo box");
-constexpr int TBC_ROWS = 2 * TBC_HALO + 32;
-constexpr int TBC_BUF_BYTES = TBC_ROWS * TBC_ROW_BYTES;
-// output rows per thread: 2 for the HBM-bound 3x3 (4 warps per CTA), 4 for the
-// FP32-bound 7x7 (2 warps: each staged row feeds more outputs, as in the agents)
-template <int R> constexpr int tbc_rb() { return R >= 3 ? 4 : 2; }
-template <int R> constexpr int tbc_threads() { return 256 / tbc_rb<R>(); }
-// smem per buffer: [0, 8) top halo box | [8, 40) centre | [40, 48) bottom halo box
-inline size_t tbc_smem_bytes(int) { return 256 + 2 * (size_t)TBC_BUF_BYTES; }
+constexpr int TBC_STAGES = 3;
+
+template <int R, int TW>
+struct TbcGeom {
+    static constexpr int kCols = 32 * TW + 8;                     // staged floats per row (x0-4 ..)
+    static constexpr int kRowB = kCols * 4;
+    static constexpr int kB = 2 * R;                              // boundary box rows
+    static constexpr int kC = 32 - 2 * R;                         // interior rows
+    static constexpr int kRegB = ((kB * kRowB) + 127) & ~127;     // 128-byte aligned regions
+    static constexpr int kCenB = ((kC * kRowB) + 127) & ~127;
+    static constexpr int kStageB = 2 * kRegB + kCenB;             // X[0] | X[1] | C
+    static constexpr uint32_t kRecvBytes = (uint32_t)((32 + 2 * R) * kRowB);   // per CTA per stage
+    static constexpr int kRB = R >= 3 ? 4 : 2;                    // output rows per consumer thread
+    static constexpr int kConsumers = 256 / kRB;
+    static constexpr int kThreads = kConsumers + 32;
+};
+template <int R> constexpr int tbc_tw() { return R >= 3 ? 1 : 2; }   // 3x3: two tiles per CTA per unit
+template <int R> constexpr int tbc_threads() { return TbcGeom<R, tbc_tw<R>()>::kThreads; }
+template <int R> inline size_t tbc_smem_bytes() { return 128 + (size_t)TBC_STAGES * TbcGeom<R, tbc_tw<R>()>::kStageB; }
 
 __device__ __forceinline__ uint32_t cluster_ctarank() {
     uint32_t r;
@@ -70,111 +92,142 @@ __device__ __forceinline__ uint32_t dsmem_addr(const void* p, uint32_t rank) {
     asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(out) : "r"(smem_u32(p)), "r"(rank));
     return out;
 }
-__device__ __forceinline__ float4 ld_dsmem4(uint32_t addr) {
-    float4 v;
-    asm volatile("ld.shared::cluster.v4.f32 {%0,%1,%2,%3}, [%4];"
-                 : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(addr) : "memory");
-    return v;
+// Stage release to the producer of CTA `rank`, and the producer's wait.
+// Default: cluster-scope release / acquire (the PTX memory model's guarantee
+// for ordering this CTA's shared-memory reads before the peer's next async
+// write into them).  CC_TBC_CTA_SCOPE=1 (diagnostic build) uses the plain
+// forms CUTLASS's multicast pipelines use (mbarrier.arrive.shared::cluster,
+// default semantics) to measure what the cluster-scope fences cost.
+#ifndef CC_TBC_CTA_SCOPE
+#define CC_TBC_CTA_SCOPE 0
+#endif
+__device__ __forceinline__ void mbar_arrive_remote_release(uint64_t* bar, uint32_t rank) {
+    if constexpr (CC_TBC_CTA_SCOPE)
+        asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" :: "r"(dsmem_addr(bar, rank)) : "memory");
+    else
+        asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" :: "r"(dsmem_addr(bar, rank))
+                     : "memory");
 }
-// Arrive on the mbarrier at the same offset in CTA `rank`.  Default (CTA-scope)
-// semantics on purpose: the data this orders lives in shared memory -- TMA
-// writes completed on the producer's own barrier, DSMEM reads are not cached --
-// while .release/.acquire.cluster would emit an L1 invalidation (CCTL.IVALL)
-// plus a memory barrier on every unit (38 % of stall samples in ncu r03a).
-__device__ __forceinline__ void mbar_arrive_remote(uint64_t* bar, uint32_t rank) {
-    asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" :: "r"(dsmem_addr(bar, rank)) : "memory");
+__device__ __forceinline__ void mbar_arrive_release_cluster(uint64_t* bar) {
+    if constexpr (CC_TBC_CTA_SCOPE)
+        mbar_arrive(bar);
+    else
+        asm volatile("mbarrier.arrive.release.cluster.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
 }
-__device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) { mbar_wait(bar, parity); }
+// wait with cluster-scope acquire: the remote releases above happen-before what follows
+__device__ __forceinline__ void mbar_wait_acquire_cluster(uint64_t* bar, uint32_t parity) {
+    if constexpr (CC_TBC_CTA_SCOPE) {
+        mbar_wait(bar, parity);
+        return;
+    }
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAITC_%=:\n\t"
+        "mbarrier.try_wait.parity.acquire.cluster.shared::cta.b64 p, [%0], %1, %2;\n\t"
+        "@!p bra WAITC_%=;\n}" :: "r"(smem_u32(bar)), "r"(parity), "r"(1000000u) : "memory");
+}
+// 2D TMA load of box (x, y) multicast to the CTAs in `mask`, each at this
+// CTA's `dst` offset, completion counted on the barrier at `bar`'s offset in each
+__device__ __forceinline__ void tma_load_2d_mc(void* dst, const void* tmap, int32_t x, int32_t y, uint64_t* bar,
+                                               uint16_t mask) {
+    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes.multicast::cluster"
+                 " [%0], [%1, {%2, %3}], [%4], %5;"
+                 :: "r"(smem_u32(dst)), "l"(tmap), "r"(x), "r"(y), "r"(smem_u32(bar)), "h"(mask) : "memory");
+}
+
+// staged row rr (input row y0 - R + rr) of CTA k: top boundary rows [0, 2R)
+// in X[(k-1)&1], interior rows [2R, 32) in C, bottom boundary rows [32, 32+2R) in X[k&1]
+struct ParityRows {
+    const float* top;
+    const float* cen;
+    const float* bot;
+    int pitch, b, c;      // b = 2R, c = 32
+    __device__ __forceinline__ const float* operator()(int rr) const {
+        return rr < b ? top + rr * pitch : rr < c ? cen + (rr - b) * pitch : bot + (rr - c) * pitch;
+    }
+};
 
 // Persistent grid of NC clusters x C CTAs (1D, cluster dims (C,1,1)),
-// tbc_threads<R>() threads, dynamic smem tbc_smem_bytes(C).
+// tbc_threads<R>() threads, dynamic smem tbc_smem_bytes<R>().
+// map_c: box (kCols x (32 - 2R)), map_b: box (kCols x 2R).
 template <int R>
-__global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_constant__ CUtensorMap map_rows,
-                                                          const __grid_constant__ CUtensorMap map_halo,
+__global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_constant__ CUtensorMap map_c,
+                                                          const __grid_constant__ CUtensorMap map_b,
                                                           const __grid_constant__ Sched s,
                                                           const __grid_constant__ ConvParams<R> p, int32_t C) {
-    extern __shared__ __align__(128) uint8_t smem_raw[];
-    __shared__ uint64_t full[2], ready[2], done[2];
-    const uint32_t sbase = smem_u32(smem_raw);
-    float* bufs = reinterpret_cast<float*>(smem_raw + (((sbase + 127) & ~127u) - sbase));
-    const int rank = (int)cluster_ctarank();
-    const int nbrs = (rank > 0 ? 1 : 0) + (rank < C - 1 ? 1 : 0);
+    constexpr int TW = tbc_tw<R>();
+    using G = TbcGeom<R, TW>;
+    extern __shared__ uint8_t smem_raw[];
+    __shared__ uint64_t full[TBC_STAGES], empty[TBC_STAGES];
+    uint8_t* ring = ring_base(smem_raw);
+    const int k = (int)cluster_ctarank();
     const int gx = s.g.gx, gy = s.g.gy;
+    const int ucols = (gx + TW - 1) / TW;                // unit columns
     const int ubs = (gy + C - 1) / C;                    // unit rows
-    const int units = gx * ubs;
+    const int units = ucols * ubs;
     const int c0 = (int)cluster_id_x(), NC = (int)nclusters_x();
+    const bool has_next = k < C - 1;
     if (threadIdx.x == 0) {
-        for (int b = 0; b < 2; ++b) {
+        for (int b = 0; b < TBC_STAGES; ++b) {
             mbar_init(&full[b], 1);
-            if (nbrs) { mbar_init(&ready[b], nbrs); mbar_init(&done[b], nbrs); }
+            mbar_init(&empty[b], has_next ? 2 : 1);      // this CTA's consumers + CTA k+1's
         }
         fence_mbar_init();
     }
     cluster_sync_all();                                  // every barrier of the cluster initialised
 
-    // producer step (thread 0): stage unit `u` of this cluster into buffer b
-    auto stage = [&](int u, int b) {
-        float* buf = bufs + b * (TBC_BUF_BYTES / 4);
-        const int bx = u % gx, ub = u / gx;
-        const int x0 = bx * 32, y0 = (ub * C + rank) * 32;
-        uint32_t bytes = 32 * TBC_ROW_BYTES;
-        if (rank == 0) bytes += TBC_HALO * TBC_ROW_BYTES;
-        if (rank == C - 1) bytes += TBC_HALO * TBC_ROW_BYTES;
-        mbar_arrive_tx(&full[b], bytes);
-        tma_load_2d(buf + TBC_HALO * TBC_COLS, &map_rows, x0 - 4, y0, &full[b]);
-        if (rank == 0) tma_load_2d(buf, &map_halo, x0 - 4, y0 - TBC_HALO, &full[b]);
-        if (rank == C - 1) tma_load_2d(buf + (TBC_HALO + 32) * TBC_COLS, &map_halo, x0 - 4, y0 + 32, &full[b]);
-    };
-
-    int i = 0;
-    if (threadIdx.x == 0 && c0 < units) stage(c0, 0);
-    for (int u = c0; u < units; u += NC, ++i) {
-        const int b = i & 1;
-        const uint32_t par = (uint32_t)(i >> 1) & 1u;
-        // prefetch the next unit into the other buffer once the neighbours are done with it
-        const int un = u + NC;
-        if (threadIdx.x == 0 && un < units) {
-            if (i >= 1 && nbrs) mbar_wait_cluster(&done[b ^ 1], (uint32_t)((i - 1) >> 1) & 1u);
-            stage(un, b ^ 1);
-        }
-        float* buf = bufs + b * (TBC_BUF_BYTES / 4);
-        mbar_wait(&full[b], par);                        // my centre rows (and edge halos) landed
-        if (nbrs) {
-            if (threadIdx.x == 0) {                      // tell the neighbours
-                if (rank > 0) mbar_arrive_remote(&ready[b], rank - 1);
-                if (rank < C - 1) mbar_arrive_remote(&ready[b], rank + 1);
+    if (threadIdx.x < 32) {
+        // ---- producer
+        if (threadIdx.x == 0) {
+            const uint16_t mask = (uint16_t)((1u << k) | (has_next ? 1u << (k + 1) : 0u));
+            int i = 0;
+            for (int u = c0; u < units; u += NC, ++i) {
+                const int st = i % TBC_STAGES;
+                if (i >= TBC_STAGES) mbar_wait_acquire_cluster(&empty[st], (uint32_t)((i / TBC_STAGES) - 1) & 1u);
+                uint8_t* stage = ring + (size_t)st * G::kStageB;
+                const int x0 = (u % ucols) * 32 * TW, y0 = ((u / ucols) * C + k) * 32;
+                mbar_arrive_tx(&full[st], G::kRecvBytes);
+                tma_load_2d(stage + 2 * G::kRegB, &map_c, x0 - 4, y0 + R, &full[st]);     // interior
+                if (k == 0)                                                                  // cluster top
+                    tma_load_2d(stage + G::kRegB, &map_b, x0 - 4, y0 - R, &full[st]);      // X[1]
+                // bottom boundary into X[k & 1]: shared with CTA k+1 (its top) by one multicast
+                tma_load_2d_mc(stage + (k & 1) * G::kRegB, &map_b, x0 - 4, y0 + 32 - R, &full[st], mask);
             }
-            mbar_wait_cluster(&ready[b], par);           // theirs landed too
-            for (int idx = threadIdx.x; idx < 2 * R * 10; idx += tbc_threads<R>()) {
-                const int side = idx / (R * 10), rem = idx - side * R * 10;
-                const int rr = rem / 10, cc = rem - rr * 10;
-                if (side == 0 && rank > 0) {             // rows 8-R.. <- rank-1's centre rows 32-R..
-                    const float* src = buf + (TBC_HALO + 32 - R + rr) * TBC_COLS + 4 * cc;
-                    reinterpret_cast<float4*>(buf + (TBC_HALO - R + rr) * TBC_COLS)[cc] = ld_dsmem4(dsmem_addr(src, rank - 1));
+        }
+    } else {
+        // ---- consumers
+        const int ctid = threadIdx.x - 32;
+        int i = 0;
+        for (int u = c0; u < units; u += NC, ++i) {
+            const int st = i % TBC_STAGES;
+            mbar_wait(&full[st], (uint32_t)(i / TBC_STAGES) & 1u);
+            const uint8_t* stage = ring + (size_t)st * G::kStageB;
+            const float* top = reinterpret_cast<const float*>(stage + ((k - 1) & 1) * G::kRegB);
+            const float* bot = reinterpret_cast<const float*>(stage + (k & 1) * G::kRegB);
+            const float* cen = reinterpret_cast<const float*>(stage + 2 * G::kRegB);
+            const int bx0 = (u % ucols) * TW, by = (u / ucols) * C + k;
+            if (by < gy) {
+#pragma unroll 1
+                for (int t = 0; t < TW; ++t) {
+                    const int bx = bx0 + t;
+                    if (bx >= gx) break;
+                    const ParityRows rows{top + 32 * t, cen + 32 * t, bot + 32 * t, G::kCols, 2 * R, 32};
+                    conv_tile_compute_rows<R, G::kRB>(p, rows, bx, by, ctid);
+                    if (ctid == 0) {
+                        const int32_t lin = by * gx + bx;
+                        if (s.census) atomicAdd(s.census + lin, 1u);
+                        if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();
+                    }
                 }
-                if (side == 1 && rank < C - 1) {         // rows 40.. <- rank+1's centre rows 0..
-                    const float* src = buf + (TBC_HALO + rr) * TBC_COLS + 4 * cc;
-                    reinterpret_cast<float4*>(buf + (TBC_HALO + 32 + rr) * TBC_COLS)[cc] = ld_dsmem4(dsmem_addr(src, rank + 1));
-                }
             }
-            __syncthreads();                             // halos copied (my reads of theirs are done)
-            if (threadIdx.x == 0) {
-                if (rank > 0) mbar_arrive_remote(&done[b], rank - 1);
-                if (rank < C - 1) mbar_arrive_remote(&done[b], rank + 1);
+            consumer_sync<G::kConsumers>();              // every consumer is done reading this stage
+            if (ctid == 0) {
+                mbar_arrive_release_cluster(&empty[st]);
+                if (k > 0) mbar_arrive_remote_release(&empty[st], (uint32_t)(k - 1));
             }
         }
-        const int bx = u % gx, by = (u / gx) * C + rank;
-        if (by < gy) {
-            conv_tile_compute<R, tbc_rb<R>()>(p, buf + (TBC_HALO - R) * TBC_COLS, bx, by, threadIdx.x);
-            if (threadIdx.x == 0) {
-                const int32_t lin = by * gx + bx;
-                if (s.census) atomicAdd(s.census + lin, 1u);
-                if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();
-            }
-        }
-        __syncthreads();                                 // buffer b free for my next use
     }
-    cluster_sync_all();                                  // nobody leaves while a neighbour may read it
+    cluster_sync_all();                                  // no CTA leaves while a peer may still signal it
 }
 
 }  // namespace cc

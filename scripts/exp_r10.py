@@ -63,7 +63,62 @@ def stencil():
     return out
 
 
+def tbc():
+    """thread-block-cluster (TMA multicast) backend vs default / identity / agent, conv 3x3 and 7x7"""
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    out = {}
+    N = 8192
+    img = synth.matrix(5, N, N, backend="torch", device="cuda")
+    o = torch.empty_like(img)
+    for R in (1, 3):
+        K = 2 * R + 1
+        w = synth.uniform(6, K * K).reshape(K, K)
+        w = (w / w.astype(np.float64).sum()).astype(np.float32)
+        variants = [("default", dict(backend="default")), ("identity", dict(backend="identity")),
+                    ("agent-row", dict(backend="agent", order="row"))] + \
+                   [(f"tbc{c}", dict(backend="tbcluster", cluster_size=c)) for c in (1, 2, 4, 8)]
+        if R == 3:
+            variants.append(("static-row-m7", dict(backend="static", order="row", num_clusters=7 * 148)))
+        r = B.measure(variants, lambda kw: ops.conv2d(img, w, out=o, **kw), 20, 8 * N * N, graph=True,
+                      inner=B.GRAPH_INNER)
+        out[f"conv{K}"] = r
+        print(f"conv{K}", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    return out
+
+
+def panel():
+    """ROW clusters over vertical panels: TILE(tw, gy) orders (panel-major, row-major inside a panel)"""
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    out = {}
+    N = 8192
+    img = synth.matrix(5, N, N, backend="torch", device="cuda")
+    o = torch.empty_like(img)
+    w = synth.uniform(6, 9).reshape(3, 3)
+    w = (w / w.astype(np.float64).sum()).astype(np.float32)
+    v3 = [("default", dict(backend="default")), ("identity", dict(backend="identity")),
+          ("agent-row", dict(backend="agent", order="row"))] + \
+         [(f"agent-panel{tw}", dict(backend="agent", order="tile", tile=(tw, 256))) for tw in (32, 64, 128)]
+    r = B.measure(v3, lambda kw: ops.conv2d(img, w, out=o, **kw), 20, 8 * N * N, graph=True, inner=B.GRAPH_INNER)
+    out["conv3"] = r
+    print("conv3", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    del img, o
+    M = 16384
+    a = synth.matrix(4, M, M, backend="torch", device="cuda")
+    b = a.clone()
+    vj = [("default", dict(backend="default")), ("identity", dict(backend="identity")),
+          ("agent-row", dict(backend="agent", order="row"))] + \
+         [(f"agent-panel{tw}", dict(backend="agent", order="tile", tile=(tw, 512))) for tw in (32, 64, 128, 256)]
+    r = B.measure(vj, lambda kw: ops.jacobi5(a, b, 2, **kw), 10, 2 * 8 * M * M, graph=True, inner=5)
+    out["jacobi"] = r
+    print("jacobi", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    return out
+
+
 if __name__ == "__main__":
     what, path = sys.argv[1], sys.argv[2]
-    res = spmv() if what == "spmv" else stencil()
+    res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel}[what]()
     json.dump(res, open(path, "w"), indent=1)

@@ -201,8 +201,8 @@ def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     script = tmp_path / "w.py"
     script.write_text(WORKER.format(root=ROOT))
     port = _port()
-    procs = [subprocess.Popen([sys.executable, str(script), str(r), str(world), port, cfg], stdout=subprocess.PIPE,
-                              stderr=subprocess.STDOUT, text=True) for r in range(world)]
+    procs = [subprocess.Popen([sys.executable, "-X", "faulthandler", str(script), str(r), str(world), port, cfg],
+                              stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True) for r in range(world)]
     outs = []
     for p in procs:
         try:
@@ -211,5 +211,5 @@ def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
             p.kill()
             outs.append(p.communicate()[0])
     res = [ln for o in outs for ln in o.splitlines() if ln.startswith("RESULT")]
-    assert len(res) == world, outs
+    assert len(res) == world, (outs, [p.returncode for p in procs])
     assert all(ln.split()[2] == "True" for ln in res), res
