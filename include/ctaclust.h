@@ -38,8 +38,9 @@ typedef enum {
     CC_ERR_NCCL = -5,            /* reserved for the NCCL-backed entry points */
     CC_ERR_UNSUPPORTED = -6,     /* valid request this build / device cannot serve */
     CC_ERR_NO_DEVICE = -7,       /* plan created host-only (device < 0) was asked to launch */
-    CC_ERR_BUSY = -8             /* agent launch while the plan's workspace is still in use
-                                    by an unfinished launch on another stream */
+    CC_ERR_BUSY = -8             /* reserved (round 1 refused an agent launch on another
+                                    stream while the plan's workspace was in use; cc_launch
+                                    now orders such a launch after the previous one) */
 } cc_status;
 
 /* ---------------------------------------------------------------------------
@@ -360,10 +361,13 @@ cc_status cc_max_agents(int32_t kernel, int32_t device, int32_t* max_agents);
 /* Run `kernel` over the plan's logical grid with the chosen backend, on
  * `stream`.  The plan's grid must equal cc_kernel_grid(kernel, args).  The
  * agent backends use the plan's workspace, which resets itself at the end of
- * each launch, so launches sharing a plan must be stream-ordered: an agent or
- * identity launch on a stream other than the previous one's returns
- * CC_ERR_BUSY while that previous launch is unfinished (synchronize, or use a
- * second plan).  Launches captured into a CUDA graph are not checked.
+ * each launch, so launches sharing a plan never overlap: an agent or identity
+ * launch on a stream other than the previous launch's is made to wait for
+ * that launch's completion (cudaStreamWaitEvent, recorded under the plan's
+ * mutex together with the launch, so concurrent host threads are safe too).
+ * Use a second plan for concurrency.  Launches being captured into a CUDA
+ * graph are neither ordered nor recorded: the capturing code orders them.
+ * The calling thread's current device is unchanged on return (also on errors).
  * `launches` (HOST, optional) receives the number of kernels this call queued. */
 cc_status cc_launch(cc_plan plan, int32_t kernel, const void* args,
                     const cc_launch_opts* opts, void* stream, int32_t* launches);

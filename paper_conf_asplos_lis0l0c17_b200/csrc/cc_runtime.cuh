@@ -108,7 +108,6 @@ __device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
 // The suspend-time hint lets a waiting warp sleep in hardware until the phase
 // completes (or the hint expires) instead of re-issuing try_wait: spinning
 // consumer warps otherwise eat the issue slots the working warps need.
-#ifndef CC_WAIT_BACKOFF
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile(
         "{\n\t.reg .pred p;\n"
@@ -116,50 +115,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
         "@!p bra WAIT_%=;\n}" :: "r"(smem_u32(bar)), "r"(parity), "r"(1000000u) : "memory");
 }
-#else
-// diagnostic build: plain try_wait with an exponential nanosleep backoff (the
-// suspend-hint form wakes on every sync-unit event of the SM and re-issues)
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    uint32_t ok, ns = 32;
-    for (;;) {
-        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-                     "selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-        if (ok) return;
-        __nanosleep(ns);
-        if (ns < CC_WAIT_BACKOFF) ns <<= 1;
-    }
-}
-#endif
-// Non-blocking probe + timed sleep.  The suspend-hint try_wait lowers to
-// SYNCS.PHASECHK.TRYWAIT + NANOSLEEP.SYNCS, which wakes on every sync-unit
-// event of the SM (each TMA completion, each barrier arrival of any agent):
-// ncu counts 148 wake-ups per producer wait on the 7x7 conv, 19 % of all
-// issued instructions spent re-checking barriers.  test_wait never suspends;
-// the warp sleeps a real, exponentially growing interval instead.
-__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
-    uint32_t ok;
-    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-                 "selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-    return ok != 0;
-}
-template <uint32_t kMaxNs>
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
-    if constexpr (kMaxNs == 0) {
-        mbar_wait(bar, parity);
-    } else {
-        uint32_t ns = 32;
-        while (!mbar_test(bar, parity)) {
-            __nanosleep(ns);
-            if (ns < kMaxNs) ns <<= 1;
-        }
-    }
-}
-#ifndef CC_PROD_SLEEP
-#define CC_PROD_SLEEP 0     // producer's wait for a free ring slot (0: suspend-hint try_wait)
-#endif
-#ifndef CC_CONS_SLEEP
-#define CC_CONS_SLEEP 0     // consumers' wait for a staged slot
-#endif
+// (Round 1 measured exponential nanosleep back-off and test_wait + timed
+// sleep in place of the suspend-hint wait, for the producer and the
+// consumers: slower or equal everywhere -- profiles/r05/diag, r07/diag.)
 // 1D bulk async copy global -> shared, completion counted on `bar` (UBLKCP).
 // dst, src 16-byte aligned, bytes a multiple of 16.
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -231,9 +189,6 @@ __device__ __forceinline__ void lin_to_bxby(const Sched& s, int32_t v, int32_t* 
     }
 }
 
-#ifndef CC_INC_DECODE
-#define CC_INC_DECODE 0     // build option: incremental TILE decode (see lin_to_bxby_warp)
-#endif
 // Producer-warp form (v warp-uniform, all 32 lanes present).  A USER order
 // table lookup is a dependent L2 round trip per task on the scheduler's
 // critical path (measured 2.3x slower conv 3x3 than the computed orders);
@@ -254,43 +209,6 @@ __device__ __forceinline__ void lin_to_bxby_warp(const Sched& s, int32_t* win, i
         }
         const int32_t l = ((volatile int32_t*)win)[1 + v - *(volatile int32_t*)win];
         *by = l / s.g.gx; *bx = l - *by * s.g.gx; *lin = l;
-    } else if (CC_INC_DECODE && s.mode != MODE_IDENTITY && s.g.order == ORDER_TILE) {
-        // incremental TILE decode: a cluster's pops are consecutive order
-        // positions, so the successor of the previous position is one step of
-        // the Fig. 7 walk (row-major inside the clipped tw x th tile, tiles
-        // row-major along the band, bands top to bottom) with no integer
-        // division; anything else (first pop, a steal, a batch elsewhere) takes
-        // the full decode (three divisions) and re-seeds the walk state
-        // d = {v, bx, by, ox, oy, wt, ht}.  Measured: TILE orders 6-8 % faster
-        // (conv 3x3, Jacobi; ROW / COL / identity keep the single-division
-        // decode, which is cheaper than the shared-memory state), but the extra
-        // producer code makes every conv 7x7 agent 5 % slower, order-independent
-        // and reproducible (profiles/r07/diag/suite_incdec_*), so it is off by
-        // default.
-        volatile int32_t* d = win + 33;
-        int32_t x, y, ox, oy, wt, ht;
-        if (v == d[0] + 1) {
-            x = d[1]; y = d[2]; ox = d[3]; oy = d[4]; wt = d[5]; ht = d[6];
-            if (++x == ox + wt) {
-                x = ox;
-                if (++y == oy + ht) {                          // next tile of the band, or next band
-                    ox += s.g.tw;
-                    if (ox >= s.g.gx) { ox = 0; oy += s.g.th; }
-                    wt = s.g.gx - ox < s.g.tw ? s.g.gx - ox : s.g.tw;
-                    ht = s.g.gy - oy < s.g.th ? s.g.gy - oy : s.g.th;
-                    x = ox; y = oy;
-                }
-            }
-        } else {
-            decode(s.g, v, &x, &y);
-            ox = (x / s.g.tw) * s.g.tw; oy = (y / s.g.th) * s.g.th;
-            wt = s.g.gx - ox < s.g.tw ? s.g.gx - ox : s.g.tw;
-            ht = s.g.gy - oy < s.g.th ? s.g.gy - oy : s.g.th;
-        }
-        __syncwarp();
-        if (lane == 0) { d[0] = v; d[1] = x; d[2] = y; d[3] = ox; d[4] = oy; d[5] = wt; d[6] = ht; }
-        __syncwarp();
-        *bx = x; *by = y; *lin = y * s.g.gx + x;
     } else {
         lin_to_bxby(s, v, lin, bx, by);
     }
@@ -325,16 +243,9 @@ __device__ __forceinline__ int32_t* q_head(const Sched& s, int32_t q) {
     return s.mode == MODE_IDENTITY ? ws_gq(s) : ws_head(s) + q;
 }
 
-// Position of slot w of queue q.  Build option CC_ALT_DIR: odd clusters are
-// drained back to front, so neighbouring clusters reach their common boundary
-// at the same time (both at the start or both at the end of the launch) and
-// the halo rows they share are re-read from L2 instead of DRAM.  Execution
-// order inside a cluster is not part of the partition (reading R9).
-#ifndef CC_ALT_DIR
-#define CC_ALT_DIR 0
-#endif
+// Position of slot w of queue q.  (Draining odd clusters back to front was
+// measured in round 1 -- +-1 % on the agents, 2-11 % slower static -- and dropped.)
 __device__ __forceinline__ int32_t q_pos(const Sched& s, int32_t q, int32_t w) {
-    if (CC_ALT_DIR && s.mode != MODE_IDENTITY && (q & 1)) return q_start(s, q) + q_size(s, q) - 1 - w;
     return q_start(s, q) + w;
 }
 
@@ -454,7 +365,6 @@ struct RingShared {
     uint64_t empty[MAX_STAGES];
     int4 slot[MAX_STAGES];       // (v, lin, bx, by) decoded once by the scheduler warp
     int4 slot2[MAX_STAGES];      // merged slots: (v, lin) of the second CTA, and n
-    int4 slot3[MAX_STAGES];      // merged slots of 3-4 CTAs: (v, lin) of the third and fourth
 };
 
 __device__ __forceinline__ uint8_t* ring_base(uint8_t* dyn) {
@@ -506,11 +416,11 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         uint32_t ph = 0;                                       // empty-barrier parity
         int32_t t = 0;
         int32_t pending = -1;                                  // popped but not yet staged (merge miss)
-        __shared__ int32_t s_uwin[40];                         // USER-order window / decode walk (lin_to_bxby_warp)
-        if (lane == 0) { s_uwin[0] = -64; s_uwin[33] = -2; }
+        __shared__ int32_t s_uwin[33];                         // USER-order window (lin_to_bxby_warp)
+        if (lane == 0) s_uwin[0] = -64;
         __syncwarp();
         for (;; ++t) {
-            if (t >= S) mbar_wait_sleep<CC_PROD_SLEEP>(&R.empty[st], ph ^ 1u);
+            if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
             const int32_t v = pending >= 0 ? pending : producer_next<kStatic>(s, P, lane);
             pending = -1;
             if (v < 0) {
@@ -529,21 +439,6 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
                         lin_to_bxby_warp(s, s_uwin, v2, lane, &lin2, &bx2, &by2);
                         if (by2 == by && bx2 == bx + 1) {
                             n = 2;
-                            if constexpr (MergeOf<Body>::value > 2) {
-                                // longer runs (left to right): up to 4 tiles per slot
-                                int4 x34 = make_int4(-1, 0, -1, 0);
-#pragma unroll 1
-                                for (int k = 2; k < MergeOf<Body>::value; ++k) {
-                                    const int32_t vk = producer_next<kStatic>(s, P, lane);
-                                    if (vk < 0) break;
-                                    int32_t link, bxk, byk;
-                                    lin_to_bxby_warp(s, s_uwin, vk, lane, &link, &bxk, &byk);
-                                    if (byk != by || bxk != bx + k) { pending = vk; break; }
-                                    if (k == 2) { x34.x = vk; x34.y = link; } else { x34.z = vk; x34.w = link; }
-                                    n = k + 1;
-                                }
-                                if (lane == 0) R.slot3[st] = x34;
-                            }
                             if (lane == 0) R.slot2[st] = make_int4(v2, lin2, n, 0);
                         } else if (by2 == by && bx2 == bx - 1) {       // popped right to left
                             n = 2;
@@ -568,7 +463,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         for (int k = 0; k < Body::kGroups; ++k) {
             if (k > 0) {
                 if (++st == S) { st = 0; ph ^= 1u; }
-                if (t + k >= S) mbar_wait_sleep<CC_PROD_SLEEP>(&R.empty[st], ph ^ 1u);
+                if (t + k >= S) mbar_wait(&R.empty[st], ph ^ 1u);
                 if (lane == 0) R.slot[st] = make_int4(-1, 0, 0, 0);
             }
             __syncwarp();
@@ -592,7 +487,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         int st = grp;                                          // group g takes tasks g, g+G, ...
         uint32_t ph = 0;                                       // full-barrier parity (G <= S)
         for (;;) {
-            mbar_wait_sleep<CC_CONS_SLEEP>(&R.full[st], ph);
+            mbar_wait(&R.full[st], ph);
             const int4 sl = R.slot[st];
             if (sl.x < 0) break;
             if constexpr (MergeOf<Body>::value > 1) {
@@ -601,9 +496,6 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
                 if (ctid == 0) {
                     record(s, sl.x, sl.y);
                     if (s2.z > 1) record(s, s2.x, s2.y);
-                    if constexpr (MergeOf<Body>::value > 2) {
-                        if (s2.z > 2) { const int4 s3 = R.slot3[st]; record(s, s3.x, s3.y); if (s2.z > 3) record(s, s3.z, s3.w); }
-                    }
                 }
             } else {
                 body.consume(s, sl.z, sl.w, ring + (size_t)st * s.stage_bytes, ctid);

@@ -140,29 +140,33 @@ struct cc_plan_s {
 };
 
 // The agent backends share the plan's self-resetting workspace (queue heads,
-// agent and claim counters).  Two launches in flight at once on different
-// streams would interleave their queue atomics and break exactly-once
-// coverage, so such a launch is refused (CC_ERR_BUSY) while the previous one
-// on another stream has not finished.  Same-stream launches are ordered by
-// the stream; launches being captured into a CUDA graph are the caller's to
-// order (no query is legal during capture).
-static cc_status ws_acquire(cc_plan_s* p, cudaStream_t st, bool* record) {
-    *record = false;
+// agent and claim counters).  Two launches in flight at once would interleave
+// their queue atomics and break exactly-once coverage, so launches on one plan
+// are serialised: under the plan's mutex (held across the launch and the event
+// record, so two host threads cannot both pass), a launch on a stream other
+// than the previous one's first makes its stream wait for the previous
+// launch's completion event (cudaStreamWaitEvent: ordering, no host block).
+// Launches captured into a CUDA graph are the caller's to order (no event of
+// another stream may be waited on inside a capture); they record nothing.
+struct WsLease {
+    cc_plan_s* p;
+    cudaStream_t st;
+    bool capturing = false;
+    std::unique_lock<std::mutex> lk;
+    cc_status acquire();
+    cc_status release();
+};
+cc_status WsLease::acquire() {
     cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
     CC_CUDA(cudaStreamIsCapturing(st, &cs));
-    if (cs != cudaStreamCaptureStatusNone) return CC_OK;
-    std::lock_guard<std::mutex> lk(p->ws_mu);
-    if (p->ws_pending && p->ws_stream != st) {
-        cudaError_t q = cudaEventQuery(p->ws_done);
-        if (q == cudaErrorNotReady)
-            return fail(CC_ERR_BUSY, "plan workspace in use by an unfinished launch on another stream");
-        if (q != cudaSuccess) return cuda_fail(q, "workspace event");
-    }
-    *record = true;
+    capturing = cs != cudaStreamCaptureStatusNone;
+    if (capturing) return CC_OK;
+    lk = std::unique_lock<std::mutex>(p->ws_mu);
+    if (p->ws_pending && p->ws_stream != st) CC_CUDA(cudaStreamWaitEvent(st, p->ws_done, 0));
     return CC_OK;
 }
-static cc_status ws_release(cc_plan_s* p, cudaStream_t st) {
-    std::lock_guard<std::mutex> lk(p->ws_mu);
+cc_status WsLease::release() {
+    if (capturing) return CC_OK;
     if (!p->ws_done) CC_CUDA(cudaEventCreateWithFlags(&p->ws_done, cudaEventDisableTiming));
     CC_CUDA(cudaEventRecord(p->ws_done, st));
     p->ws_stream = st;
@@ -193,8 +197,10 @@ extern "C" cc_status cc_plan_create(const cc_plan_desc* d, cc_plan* out) {
     p->facts = facts;
     Grid& g = p->g;
     g.gx = d->gx; g.gy = d->gy; g.order = d->order;
-    g.tw = d->order == CC_ORDER_TILE ? d->tile_w : 1;
-    g.th = d->order == CC_ORDER_TILE ? d->tile_h : 1;
+    // a tile wider / taller than the grid is the whole grid in that direction
+    // (clamped, so the decode's tile products stay inside int32)
+    g.tw = d->order == CC_ORDER_TILE ? std::min(d->tile_w, std::max(d->gx, 1)) : 1;
+    g.th = d->order == CC_ORDER_TILE ? std::min(d->tile_h, std::max(d->gy, 1)) : 1;
     g.V = (int32_t)V; g.M = M; g.q = (int32_t)(V / M); g.r = (int32_t)(V % M);
     if (d->order == CC_ORDER_USER) {
         p->user.assign(d->user_order, d->user_order + V);
@@ -217,16 +223,23 @@ extern "C" cc_status cc_plan_create(const cc_plan_desc* d, cc_plan* out) {
     p->offsets.resize(M + 1);
     for (int i = 0; i <= M; ++i) p->offsets[i] = i < M ? cluster_start(g, i) : g.V;
     if (d->device >= 0) {
+        // the tables are filled on a private non-blocking stream and only that
+        // stream is synchronised: creating a plan does not wait for (or stall)
+        // work queued on the caller's streams
         int prev = 0;
+        cudaStream_t ps = nullptr;
         cudaError_t e = cudaGetDevice(&prev);
         if (e == cudaSuccess) e = cudaSetDevice(d->device);
+        if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&ps, cudaStreamNonBlocking);
         if (e == cudaSuccess) e = cudaMalloc(&p->d_ws, sizeof(int32_t) * ws_ints(M));
-        if (e == cudaSuccess) e = cudaMemset(p->d_ws, 0, sizeof(int32_t) * ws_ints(M));
+        if (e == cudaSuccess) e = cudaMemsetAsync(p->d_ws, 0, sizeof(int32_t) * ws_ints(M), ps);
         if (e == cudaSuccess && d->order == CC_ORDER_USER && V > 0) {
             e = cudaMalloc(&p->d_user, sizeof(int32_t) * V);
-            if (e == cudaSuccess) e = cudaMemcpy(p->d_user, p->user.data(), sizeof(int32_t) * V, cudaMemcpyHostToDevice);
+            if (e == cudaSuccess)
+                e = cudaMemcpyAsync(p->d_user, p->user.data(), sizeof(int32_t) * V, cudaMemcpyHostToDevice, ps);
         }
-        if (e == cudaSuccess) e = cudaDeviceSynchronize();
+        if (e == cudaSuccess) e = cudaStreamSynchronize(ps);
+        if (ps) cudaStreamDestroy(ps);
         cudaSetDevice(prev);
         if (e != cudaSuccess) { cudaFree(p->d_ws); cudaFree(p->d_user); delete p; return cuda_fail(e, "plan device tables"); }
     }
@@ -313,6 +326,23 @@ extern "C" cc_status cc_launch_opts_default(cc_launch_opts* o) {
 }
 
 #define CC_TRY(...) do { cc_status s_ = (__VA_ARGS__); if (s_ != CC_OK) return s_; } while (0)
+
+// switches to a device and back on scope exit (every return path of cc_launch)
+struct DeviceGuard {
+    int prev = -1;
+    bool switched = false;
+    cc_status set(int dev) {
+        CC_CUDA(cudaGetDevice(&prev));
+        if (prev != dev) {
+            CC_CUDA(cudaSetDevice(dev));
+            switched = true;
+        }
+        return CC_OK;
+    }
+    ~DeviceGuard() {
+        if (switched) cudaSetDevice(prev);
+    }
+};
 
 static inline int32_t cdiv(int64_t a, int64_t b) { return (int32_t)((a + b - 1) / b); }
 static inline bool al16(const void* p) { return ((uintptr_t)p & 15) == 0; }
@@ -521,10 +551,10 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
         s.stages = S;
         const int grid = c.p->facts->num_sms * maxa;
-        bool rec = false;
-        CC_TRY(ws_acquire(c.p, c.st, &rec));
+        WsLease lease{c.p, c.st};
+        CC_TRY(lease.acquire());
         k_agent<Body><<<grid, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
-        if (cudaPeekAtLastError() == cudaSuccess && rec) CC_TRY(ws_release(c.p, c.st));
+        if (cudaPeekAtLastError() == cudaSuccess) CC_TRY(lease.release());
         break;
     }
     case CC_BACKEND_AGENT_STATIC: {
@@ -666,9 +696,8 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         return fail(CC_ERR_INVALID_ARG, "plan grid %dx%d != kernel grid %dx%d", p->g.gx, p->g.gy, gx, gy);
     if (o->backend == CC_BACKEND_TBCLUSTER && k != CC_K_CONV2D)
         return fail(CC_ERR_UNSUPPORTED, "TBCLUSTER backend is implemented for conv2d only");
-    int prev = 0;
-    CC_CUDA(cudaGetDevice(&prev));
-    if (prev != p->device) CC_CUDA(cudaSetDevice(p->device));
+    DeviceGuard dg;
+    CC_TRY(dg.set(p->device));                   // restored on every return path
     cudaStream_t st = (cudaStream_t)stream;
     LaunchCtx c{p, o, st, launches};
     cc_status s = CC_OK;
@@ -838,7 +867,6 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
     default:
         s = fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
     }
-    if (prev != p->device) cudaSetDevice(prev);
     return s;
 }
 

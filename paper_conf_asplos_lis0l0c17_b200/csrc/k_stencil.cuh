@@ -25,14 +25,11 @@ namespace cc {
 
 enum : int32_t { STAGE_TMA = 1, STAGE_L1 = 2, STAGE_DIRECT = 3 };
 constexpr int ST_COLS = 40;                 // staged floats per row (x0-4 .. x0+35)
-// Merged slots: up to ST_MERGE horizontally adjacent tiles of a cluster in one
-// TMA box (x0-4 .. x0+32*ST_MERGE+3).  Build option CC_STENCIL_MERGE (2 or 4).
-#ifndef CC_STENCIL_MERGE
-#define CC_STENCIL_MERGE 2
-#endif
-constexpr int ST_MERGE = CC_STENCIL_MERGE;
-static_assert(ST_MERGE == 2 || ST_MERGE == 4, "merged tiles per slot");
-constexpr int ST_COLS2 = 32 * ST_MERGE + 8;  // merged slot width in floats (72 for two tiles)
+// Merged slots: two horizontally adjacent tiles of a cluster in one TMA box
+// (x0-4 .. x0+67).  (Runs of four measured 1-5 % slower in round 1: the
+// larger slots cost an agent per SM.)
+constexpr int ST_MERGE = 2;
+constexpr int ST_COLS2 = 32 * ST_MERGE + 8;  // merged slot width in floats (72)
 
 // Split staging for CC_L2_HINT_HALO_LAST: the tile's box as two TMA loads --
 // the first 32 rows (evict_first: nothing reads them again after this tile
@@ -170,15 +167,10 @@ __device__ __forceinline__ uint64_t globaltimer() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
-// Diagnostic builds only (make CC_DEFS=...; never the shipped library):
-// CC_LL_GPU_SCOPE uses .gpu instead of .sys for the LL words (valid only for
-// virtual slabs on one GPU); CC_LL_NOSTORE drops the deposits (wrong
-// results; to time their share).
-#ifdef CC_LL_GPU_SCOPE
-#define CC_LL_SCOPE "gpu"
-#else
+// LL words are accessed at system scope: across GPUs they are NVLink peer
+// stores / loads.  (A .gpu-scope build and one without the deposits timed the
+// parts of the fused sweep in round 1: identical / -0.5 us.)
 #define CC_LL_SCOPE "sys"
-#endif
 __device__ __forceinline__ uint64_t ll_word(float v, uint32_t tag) {
     return ((uint64_t)tag << 32) | (uint64_t)__float_as_uint(v);
 }
@@ -323,13 +315,8 @@ struct Jacobi5BodyT {
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
                                               int ctid) {
         if (n >= 2) {
-            if constexpr (ST_MERGE == 2) {
-                consume_at(s, bx, by, stage, ctid, ST_COLS2, 0);
-                consume_at(s, bx + 1, by, stage, ctid, ST_COLS2, 32);
-            } else {
-#pragma unroll 1
-                for (int k = 0; k < n; ++k) consume_at(s, bx + k, by, stage, ctid, ST_COLS2, 32 * k);
-            }
+            consume_at(s, bx, by, stage, ctid, ST_COLS2, 0);
+            consume_at(s, bx + 1, by, stage, ctid, ST_COLS2, 32);
         } else {
             consume_at(s, bx, by, stage, ctid, ST_COLS, 0);
         }
@@ -405,17 +392,12 @@ struct Jacobi5BodyT {
                 if (gy >= p.row_end) break;
                 const float4 o = jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows, p.cols);
                 store4_masked(p.b + (int64_t)gy * p.ld + gx, o, gx, p.cols);
-#ifndef CC_LL_NOSTORE
                 if (top && gy == 1) ll_store4(p.h.up_ll + opar + p.h.ldl + gx, o, sw, valid);
                 if (bot && gy == p.rows - 2) ll_store4(p.h.dn_ll + opar + gx, o, sw, valid);
-#endif
             }
             return;
         }
-#ifndef CC_JACOBI_INTERIOR_FAST
-#define CC_JACOBI_INTERIOR_FAST 1
-#endif
-        if (CC_JACOBI_INTERIOR_FAST && gx >= 1 && gx + 4 <= p.cols - 1 && gy0 >= 1 && gy0 + RB <= p.rows - 1 &&
+        if (gx >= 1 && gx + 4 <= p.cols - 1 && gy0 >= 1 && gy0 + RB <= p.rows - 1 &&
             gy0 + RB <= p.row_end) {
             // interior block: no boundary cells, plain float4 stores (same arithmetic)
 #pragma unroll
@@ -492,10 +474,7 @@ __device__ __forceinline__ void conv_tile_compute_rows(const ConvParams<R>& p, c
         }
     }
     if (gx >= p.cols) return;
-#ifndef CC_CONV_INTERIOR_FAST
-#define CC_CONV_INTERIOR_FAST 1
-#endif
-    if (CC_CONV_INTERIOR_FAST) {
+    {
         // interior thread block of outputs (every output of its RB x 4 block
         // has a full window): plain float4 stores, no per-element masks
         const int gy0 = by * 32 + r0;
@@ -540,30 +519,20 @@ struct Conv2dBody {
     static constexpr int kConsumers = 256 / RB;
     // two neighbouring tiles per slot for the HBM-bound 3x3 (cc_runtime.cuh:
     // MergeOf); the FP32-bound 7x7 gains nothing from the shared halo and
-    // measured 1-2 % slower merged
-#ifndef CC_CONV7_MERGE
-#define CC_CONV7_MERGE 1
-#endif
-    static constexpr int kMerge = R >= 3 ? CC_CONV7_MERGE : ST_MERGE;
+    // measured 12 % slower merged
+    static constexpr int kMerge = R >= 3 ? 1 : ST_MERGE;
     static constexpr int kStageBytes = kMerge > 1 ? HaloTile<R>::kBytes2 : HaloTile<R>::kBytes;
     static constexpr int kDirectStageBytes = HaloTile<R>::kBytes;  // the direct path stages into its own slot
     // Two consumer groups per agent (alternate tiles).  One scheduler warp per
     // two groups: with four 2-warp groups per agent (7x7) the single producer,
     // which gets only its fair share of issue slots, could not keep them fed
     // (measured 0.91x -> 0.99x of default order with two groups).
-#ifndef CC_CONV_GROUPS                                  // diagnostic builds: consumer groups per agent
-#define CC_CONV_GROUPS 2
-#endif
-    static constexpr int kGroups = CC_CONV_GROUPS;
+    static constexpr int kGroups = 2;
     static constexpr int kDefaultStages = 2 * kGroups; // two slots per group: the next tile lands while one computes
     static constexpr int kDefaultBatch = 4;
-#ifndef CC_CONV3_MIN_AGENTS                             // 3x3 agents per SM: 4 (56 registers, no
-#define CC_CONV3_MIN_AGENTS 4                           // spill) measured 5 % faster than 5 (40 + spills)
-#endif
-#ifndef CC_CONV7_MIN_AGENTS                             // 7x7 agents per SM (56 registers at 6)
-#define CC_CONV7_MIN_AGENTS (12 / CC_CONV_GROUPS)
-#endif
-    static constexpr int kMinAgents = R >= 3 ? CC_CONV7_MIN_AGENTS : CC_CONV3_MIN_AGENTS;
+    // agents per SM: 3x3 4 (56 registers, no spill; measured 5 % faster than
+    // 5 with spills), 7x7 6 (56 registers)
+    static constexpr int kMinAgents = R >= 3 ? 6 : 4;
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
@@ -590,13 +559,10 @@ struct Conv2dBody {
         // (no trailing barrier: the slot is reused only after every warp of the
         // group has released it)
     }
-#ifndef CC_CONV_DUAL_BODY
-#define CC_CONV_DUAL_BODY (R < 3)
-#endif
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
         if (s.staging == STAGE_DIRECT) {
             direct_stage(bx, by, stage, ctid);
-            if constexpr (CC_CONV_DUAL_BODY) {
+            if constexpr (R < 3) {             // 3x3: a second copy of the tile code for the direct path
                 conv_tile_compute<R, RB>(p, reinterpret_cast<const float*>(stage), bx, by, ctid, l2h);
                 return;
             }
@@ -618,15 +584,7 @@ struct Conv2dBody {
     }
     __device__ __forceinline__ void consume_n(const Sched& s, int32_t bx, int32_t by, int n, const uint8_t* stage,
                                               int ctid) {
-        if constexpr (R >= 3) {
-            // 7x7 merged: a single instance of the tile code for one or two tiles
-            // and either pitch (instruction footprint, see consume)
-            if (n < 2 && s.staging == STAGE_DIRECT) direct_stage(bx, by, stage, ctid);
-            const float* b = reinterpret_cast<const float*>(stage);
-            const int pitch = n >= 2 ? ST_COLS2 : ST_COLS;
-#pragma unroll 1
-            for (int k = 0; k < n; ++k) conv_tile_compute<R, RB>(p, b + 32 * k, bx + k, by, ctid, l2h, pitch);
-        } else if (n >= 2) {
+        if (n >= 2) {
             // one instance of the tile code, run n times (two unrolled copies would
             // not fit the register budget of the resident agents)
             const float* b = reinterpret_cast<const float*>(stage);

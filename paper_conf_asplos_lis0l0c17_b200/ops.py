@@ -20,18 +20,51 @@ DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": (
                  "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1)),
                  "jacobi5_halo": ("row", (1, 1))}
 
-# Plans are cached for the life of the process and never evicted: a plan may
-# only be destroyed once every stream that used it has synchronized
-# (cc_plan_destroy), which a cache cannot know.  Call release_plans() after a
-# device-wide synchronize to drop them.
+# Plans of the computed orders are cached for the life of the process: a plan
+# may only be destroyed once every stream that used it has synchronized
+# (cc_plan_destroy), which a cache cannot know.  Call release_plans() to drop
+# them.  USER-order plans are keyed by the order table's content (a hash) and
+# kept in a small LRU; an evicted one is destroyed only after synchronizing
+# its device.
 _plans: dict = {}
+_user_plans: "OrderedDict" = None
+USER_PLAN_CACHE = 8
 
 
 def release_plans() -> None:
-    """Synchronize the device and drop every cached plan (frees their device
-    tables and workspaces)."""
-    torch.cuda.synchronize()
+    """Synchronize every device holding a cached plan and drop them all (frees
+    their device tables and workspaces)."""
+    devs = {p.device for p in _plans.values()} | {p.device for p in (_user_plans or {}).values()}
+    for d in devs:
+        if d is not None and d >= 0:
+            torch.cuda.synchronize(d)
     _plans.clear()
+    if _user_plans is not None:
+        _user_plans.clear()
+
+
+def _user_plan(gx, gy, user_order, num_clusters, device) -> cc.Plan:
+    import hashlib
+    from collections import OrderedDict
+
+    import numpy as np
+    global _user_plans
+    if _user_plans is None:
+        _user_plans = OrderedDict()
+    arr = np.ascontiguousarray(user_order, dtype=np.int32)
+    key = (gx, gy, hashlib.blake2b(arr.tobytes(), digest_size=16).digest(), num_clusters, device)
+    p = _user_plans.get(key)
+    if p is not None:
+        _user_plans.move_to_end(key)
+        return p
+    p = cc.Plan(gx, gy, "user", num_clusters, user_order=arr, device=device)
+    _user_plans[key] = p
+    while len(_user_plans) > USER_PLAN_CACHE:
+        _, old = _user_plans.popitem(last=False)
+        if old.device is not None and old.device >= 0:
+            torch.cuda.synchronize(old.device)          # no stream may still use it
+        old.close()
+    return p
 
 
 def plan_for(kernel: str, args, order=None, tile=None, num_clusters: int = 0, device: int = 0,
@@ -41,14 +74,9 @@ def plan_for(kernel: str, args, order=None, tile=None, num_clusters: int = 0, de
     order = o if order is None else order
     tile = t if tile is None else tile
     if user_order is not None:
-        # cached per table object (hashing a large table on every launch costs
-        # more host time than the kernel); the plan copies the table when it is
-        # created, so pass a new array to change the order
-        key = (gx, gy, "user", id(user_order), num_clusters, device)
-        hit = _plans.get(key)
-        if hit is None or hit[0] is not user_order:
-            hit = _plans[key] = (user_order, cc.Plan(gx, gy, "user", num_clusters, user_order=user_order, device=device))
-        return hit[1]
+        # keyed by content; a per-call hash of the table costs host time
+        # (~0.1 ms per 256 KB), so hot loops should pass a Plan to cc.launch
+        return _user_plan(gx, gy, user_order, num_clusters, device)
     key = (gx, gy, order, tuple(tile) if order == "tile" else (1, 1), num_clusters, device)
     p = _plans.get(key)
     if p is None:

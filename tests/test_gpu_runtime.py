@@ -131,11 +131,12 @@ def test_user_order():
     assert np.array_equal(mp.cpu().numpy(), u)
 
 
-def test_workspace_busy_across_streams():
-    """Agent launches sharing a plan's self-resetting workspace must be
-    stream-ordered: a launch on another stream while the previous one is
-    still running is refused with CC_ERR_BUSY (-8), and goes through once the
-    first stream has finished.  Graph-captured launches are not checked."""
+def test_workspace_ordered_across_streams():
+    """Agent launches sharing a plan's self-resetting workspace never overlap:
+    a launch on another stream while the previous one is still running is
+    ordered after it (no error), from two host threads too, and every logical
+    CTA still runs exactly once (census) in every launch."""
+    import threading
     N = 16384
     a = torch.rand(N, N, device="cuda")
     b = torch.empty_like(a)
@@ -143,14 +144,26 @@ def test_workspace_busy_across_streams():
     sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
     torch.cuda.synchronize()
     ops.jacobi5(a, b, 20, backend="agent", order="row", stream=sa)       # ~7 ms of sweeps on sa
-    with pytest.raises(cc.CtaclustError) as e:
-        ops.jacobi5(a2, b2, 1, backend="agent", order="row", stream=sb)
-    assert e.value.status == -8
-    ops.jacobi5(a2, b2, 1, backend="agent", order="row", stream=sa)      # same stream: ordered, fine
-    sa.synchronize()
-    ops.jacobi5(a2, b2, 1, backend="agent", order="row", stream=sb)      # finished: fine
-    ops.jacobi5(a2, b2, 1, backend="static", order="row", stream=sa)     # static: no workspace
+    ev = torch.cuda.Event(enable_timing=True)
+    ops.jacobi5(a2, b2, 1, backend="agent", order="row", stream=sb)      # queued behind sa's sweeps
+    ev.record(sb)
+    done_a = torch.cuda.Event(enable_timing=True)
+    done_a.record(sa)
     torch.cuda.synchronize()
-    cen, *_ = ops.census(512, 512, "agent", "row")
+    assert done_a.elapsed_time(ev) >= 0                                   # sb's launch finished after sa's
+    # census launches on one plan from two host threads and two streams
+    args = cc.CensusArgs(512, 512)
+    p = ops.plan_for("census", args, "row")
+    cens = [torch.zeros(512 * 512, dtype=torch.int32, device="cuda") for _ in range(8)]
+    streams = [torch.cuda.Stream() for _ in range(2)]
+
+    def run(t):
+        for k in range(t, 8, 2):
+            cc.launch(p, "census", args, cc.make_opts("agent", census=cens[k]), streams[t])
+    th = [threading.Thread(target=run, args=(t,)) for t in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
     torch.cuda.synchronize()
-    assert bool(torch.all(cen == 1))
+    assert all(bool(torch.all(c == 1)) for c in cens)
