@@ -444,14 +444,13 @@ struct ContigRows {
     __device__ __forceinline__ const float* operator()(int rr) const { return base + rr * pitch; }
 };
 
-template <int R, int RB = 1, class RowPtr>
-__device__ __forceinline__ void conv_tile_compute_rows(const ConvParams<R>& p, const RowPtr& rowp,
-                                                       int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0) {
+// The tile's arithmetic, into registers: thread ctid's RB x 4 outputs.
+template <int R, int RB, class RowPtr>
+__device__ __forceinline__ void conv_tile_acc(const ConvParams<R>& p, const RowPtr& rowp, int ctid,
+                                              float (&acc)[RB][4]) {
     // rowp(rr) points at the staged row holding input row y0 - R + rr, column x0 - 4
     constexpr int K = 2 * R + 1;
     const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
-    const int gx = bx * 32 + 4 * c4;
-    float acc[RB][4];
 #pragma unroll
     for (int j = 0; j < RB; ++j)
 #pragma unroll
@@ -473,6 +472,14 @@ __device__ __forceinline__ void conv_tile_compute_rows(const ConvParams<R>& p, c
             }
         }
     }
+}
+
+// ... and out to global memory (interior outputs only; the border stays 0)
+template <int R, int RB>
+__device__ __forceinline__ void conv_tile_store(const ConvParams<R>& p, int32_t bx, int32_t by, int ctid,
+                                                const float (&acc)[RB][4], int32_t l2_hint = 0) {
+    const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
+    const int gx = bx * 32 + 4 * c4;
     if (gx >= p.cols) return;
     {
         // interior thread block of outputs (every output of its RB x 4 block
@@ -501,6 +508,14 @@ __device__ __forceinline__ void conv_tile_compute_rows(const ConvParams<R>& p, c
         o.w = (row_in && gx + 3 >= R && gx + 3 < p.cols - R) ? acc[j][3] : 0.f;
         store4_out(p.out + (int64_t)gy * p.ld + gx, o, gx, p.cols, l2_hint);
     }
+}
+
+template <int R, int RB = 1, class RowPtr>
+__device__ __forceinline__ void conv_tile_compute_rows(const ConvParams<R>& p, const RowPtr& rowp,
+                                                       int32_t bx, int32_t by, int ctid, int32_t l2_hint = 0) {
+    float acc[RB][4];
+    conv_tile_acc<R, RB>(p, rowp, ctid, acc);
+    conv_tile_store<R, RB>(p, bx, by, ctid, acc, l2_hint);
 }
 
 template <int R, int RB = 1>

@@ -23,16 +23,18 @@
 // tile code maps each staged row to its region (ParityRows).  The cluster's
 // outermost boundaries are loaded by CTA 0 / CTA C-1 for themselves.
 //
-// Pipeline (per CTA, S stages, warp-specialised like the agents):
+// Pipeline (per CTA, 2 consumer groups alternating units, 2 stages each,
+// warp-specialised like the agents):
 //   warp 0 lane 0 (producer)  for stage s of unit i: wait empty[s] (this CTA
 //     and CTA k+1 -- the other receiver of its multicast -- released the
 //     stage), arm full[s] with the bytes this CTA receives, issue its
 //     interior load and its bottom-boundary multicast (CTA 0 also its top);
-//   consumer warps            wait full[s], compute, then release the stage:
-//     a local arrive on empty[s] and a remote arrive on CTA k-1's empty[s]
-//     (mbarrier.arrive.release.cluster; the producer waits with
-//     .acquire.cluster) -- the WAR order between this CTA's shared-memory
-//     reads and its neighbour's next multicast into them.
+//   consumer group            wait full[s], compute its tiles into registers,
+//     release the stage -- a local arrive on empty[s] and a remote arrive on
+//     CTA k-1's empty[s] (mbarrier.arrive.release.cluster; the producer of a
+//     CTA with a lower neighbour waits with .acquire.cluster): the WAR order
+//     between this CTA's shared-memory reads and its neighbour's next
+//     multicast into them -- then store the outputs.
 // No CTA reads another's shared memory: all data arrives by TMA and is
 // observed through the CTA's own full barrier (complete_tx), the standard
 // async-proxy pattern.  A multicast may complete_tx on a peer's full[s]
@@ -48,7 +50,8 @@
 
 namespace cc {
 
-constexpr int TBC_STAGES = 3;
+constexpr int TBC_GROUPS = 2;                 // consumer groups, alternate units
+constexpr int TBC_STAGES = 2 * TBC_GROUPS;    // two stages per group
 
 template <int R, int TW>
 struct TbcGeom {
@@ -61,8 +64,8 @@ struct TbcGeom {
     static constexpr int kStageB = 2 * kRegB + kCenB;             // X[0] | X[1] | C
     static constexpr uint32_t kRecvBytes = (uint32_t)((32 + 2 * R) * kRowB);   // per CTA per stage
     static constexpr int kRB = R >= 3 ? 4 : 2;                    // output rows per consumer thread
-    static constexpr int kConsumers = 256 / kRB;
-    static constexpr int kThreads = kConsumers + 32;
+    static constexpr int kConsumers = 256 / kRB;                  // per group (one tile's threads)
+    static constexpr int kThreads = TBC_GROUPS * kConsumers + 32;
 };
 template <int R> constexpr int tbc_tw() { return R >= 3 ? 1 : 2; }   // 3x3: two tiles per CTA per unit
 template <int R> constexpr int tbc_threads() { return TbcGeom<R, tbc_tw<R>()>::kThreads; }
@@ -170,7 +173,7 @@ __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_cons
     if (threadIdx.x == 0) {
         for (int b = 0; b < TBC_STAGES; ++b) {
             mbar_init(&full[b], 1);
-            mbar_init(&empty[b], has_next ? 2 : 1);      // this CTA's consumers + CTA k+1's
+            mbar_init(&empty[b], has_next ? 2 : 1);      // the owning group + CTA k+1's
         }
         fence_mbar_init();
     }
@@ -183,22 +186,29 @@ __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_cons
             int i = 0;
             for (int u = c0; u < units; u += NC, ++i) {
                 const int st = i % TBC_STAGES;
-                if (i >= TBC_STAGES) mbar_wait_acquire_cluster(&empty[st], (uint32_t)((i / TBC_STAGES) - 1) & 1u);
+                if (i >= TBC_STAGES) {
+                    const uint32_t ph = (uint32_t)((i / TBC_STAGES) - 1) & 1u;
+                    if (has_next) mbar_wait_acquire_cluster(&empty[st], ph);     // a peer releases too
+                    else mbar_wait(&empty[st], ph);
+                }
                 uint8_t* stage = ring + (size_t)st * G::kStageB;
                 const int x0 = (u % ucols) * 32 * TW, y0 = ((u / ucols) * C + k) * 32;
                 mbar_arrive_tx(&full[st], G::kRecvBytes);
                 tma_load_2d(stage + 2 * G::kRegB, &map_c, x0 - 4, y0 + R, &full[st]);     // interior
                 if (k == 0)                                                                  // cluster top
                     tma_load_2d(stage + G::kRegB, &map_b, x0 - 4, y0 - R, &full[st]);      // X[1]
-                // bottom boundary into X[k & 1]: shared with CTA k+1 (its top) by one multicast
-                tma_load_2d_mc(stage + (k & 1) * G::kRegB, &map_b, x0 - 4, y0 + 32 - R, &full[st], mask);
+                // bottom boundary into X[k & 1]: shared with CTA k+1 (its top) by one
+                // multicast; a cluster's last CTA loads its own
+                if (has_next) tma_load_2d_mc(stage + (k & 1) * G::kRegB, &map_b, x0 - 4, y0 + 32 - R, &full[st], mask);
+                else tma_load_2d(stage + (k & 1) * G::kRegB, &map_b, x0 - 4, y0 + 32 - R, &full[st]);
             }
         }
     } else {
-        // ---- consumers
-        const int ctid = threadIdx.x - 32;
-        int i = 0;
-        for (int u = c0; u < units; u += NC, ++i) {
+        // ---- consumers: group grp takes units i = grp, grp + G, ...
+        const int grp = (threadIdx.x - 32) / G::kConsumers;
+        const int ctid = (threadIdx.x - 32) % G::kConsumers;
+        int i = grp;
+        for (int u = c0 + grp * NC; u < units; u += TBC_GROUPS * NC, i += TBC_GROUPS) {
             const int st = i % TBC_STAGES;
             mbar_wait(&full[st], (uint32_t)(i / TBC_STAGES) & 1u);
             const uint8_t* stage = ring + (size_t)st * G::kStageB;
@@ -206,24 +216,31 @@ __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_cons
             const float* bot = reinterpret_cast<const float*>(stage + (k & 1) * G::kRegB);
             const float* cen = reinterpret_cast<const float*>(stage + 2 * G::kRegB);
             const int bx0 = (u % ucols) * TW, by = (u / ucols) * C + k;
+            // all TW tiles into registers, release the stage, then store: the
+            // release's cluster-scope fence then has no fresh stores to drain
+            float acc[TW][G::kRB][4];
+#pragma unroll
+            for (int t = 0; t < TW; ++t) {
+                const ParityRows rows{top + 32 * t, cen + 32 * t, bot + 32 * t, G::kCols, 2 * R, 32};
+                conv_tile_acc<R, G::kRB>(p, rows, ctid, acc[t]);
+            }
+            consumer_sync<G::kConsumers>();              // every thread of the group is done reading
+            if (ctid == 0) {
+                mbar_arrive(&empty[st]);
+                if (k > 0) mbar_arrive_remote_release(&empty[st], (uint32_t)(k - 1));
+            }
             if (by < gy) {
-#pragma unroll 1
+#pragma unroll
                 for (int t = 0; t < TW; ++t) {
                     const int bx = bx0 + t;
                     if (bx >= gx) break;
-                    const ParityRows rows{top + 32 * t, cen + 32 * t, bot + 32 * t, G::kCols, 2 * R, 32};
-                    conv_tile_compute_rows<R, G::kRB>(p, rows, bx, by, ctid);
+                    conv_tile_store<R, G::kRB>(p, bx, by, ctid, acc[t]);
                     if (ctid == 0) {
                         const int32_t lin = by * gx + bx;
                         if (s.census) atomicAdd(s.census + lin, 1u);
                         if (s.exec_sm) s.exec_sm[lin] = (int32_t)smid();
                     }
                 }
-            }
-            consumer_sync<G::kConsumers>();              // every consumer is done reading this stage
-            if (ctid == 0) {
-                mbar_arrive_release_cluster(&empty[st]);
-                if (k > 0) mbar_arrive_remote_release(&empty[st], (uint32_t)(k - 1));
             }
         }
     }
