@@ -50,8 +50,14 @@
 
 namespace cc {
 
+#ifndef CC_TBC_SPG
+#define CC_TBC_SPG 2                          // stages per consumer group (round-2 A/B)
+#endif
+#ifndef CC_TBC_TW3
+#define CC_TBC_TW3 2                          // 3x3 tiles per CTA per unit (round-2 A/B)
+#endif
 constexpr int TBC_GROUPS = 2;                 // consumer groups, alternate units
-constexpr int TBC_STAGES = 2 * TBC_GROUPS;    // two stages per group
+constexpr int TBC_STAGES = CC_TBC_SPG * TBC_GROUPS;
 
 template <int R, int TW>
 struct TbcGeom {
@@ -67,7 +73,7 @@ struct TbcGeom {
     static constexpr int kConsumers = 256 / kRB;                  // per group (one tile's threads)
     static constexpr int kThreads = TBC_GROUPS * kConsumers + 32;
 };
-template <int R> constexpr int tbc_tw() { return R >= 3 ? 1 : 2; }   // 3x3: two tiles per CTA per unit
+template <int R> constexpr int tbc_tw() { return R >= 3 ? 1 : CC_TBC_TW3; }   // 3x3: two tiles per CTA per unit
 template <int R> constexpr int tbc_threads() { return TbcGeom<R, tbc_tw<R>()>::kThreads; }
 template <int R> inline size_t tbc_smem_bytes() { return 128 + (size_t)TBC_STAGES * TbcGeom<R, tbc_tw<R>()>::kStageB; }
 

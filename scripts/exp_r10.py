@@ -72,7 +72,7 @@ def tbc():
     N = 8192
     img = synth.matrix(5, N, N, backend="torch", device="cuda")
     o = torch.empty_like(img)
-    for R in (1, 3):
+    for R in ((1,) if os.environ.get("EXP_CONV3_ONLY") else (1, 3)):
         K = 2 * R + 1
         w = synth.uniform(6, K * K).reshape(K, K)
         w = (w / w.astype(np.float64).sum()).astype(np.float32)
@@ -118,7 +118,28 @@ def panel():
     return out
 
 
+def conv7():
+    """conv 7x7 variants of the agent / static backends (tile-shape A/B builds)"""
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    N = 8192
+    img = synth.matrix(5, N, N, backend="torch", device="cuda")
+    o = torch.empty_like(img)
+    w = synth.uniform(6, 49).reshape(7, 7)
+    w = (w / w.astype(np.float64).sum()).astype(np.float32)
+    variants = [("default", dict(backend="default")), ("identity", dict(backend="identity")),
+                ("agent-row", dict(backend="agent", order="row"))] + \
+               [(f"static-row-m{m}", dict(backend="static", order="row", num_clusters=m * 148)) for m in (3, 4, 6, 7, 8)]
+    r = B.measure(variants, lambda kw: ops.conv2d(img, w, out=o, **kw), 20, 8 * N * N, graph=True, inner=B.GRAPH_INNER)
+    fl = 2 * 49 * (N - 6) ** 2
+    for v in r["rows"]:
+        v["tflops"] = round(fl / (v["ms"] * 1e-3) / 1e12, 2)
+    print("conv7", [(v["variant"], v["ms"], v["tflops"]) for v in r["rows"]], flush=True)
+    return {"conv7": r}
+
+
 if __name__ == "__main__":
     what, path = sys.argv[1], sys.argv[2]
-    res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel}[what]()
+    res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel, "conv7": conv7}[what]()
     json.dump(res, open(path, "w"), indent=1)
