@@ -530,16 +530,9 @@ struct Conv2dBody {
     // output rows per consumer thread: the 7x7 filter is FP32-issue bound, so
     // each thread takes 4 rows (784 FFMA per task against a fixed per-task
     // overhead of ~150 instructions per warp); the 3x3 is HBM bound
-#ifndef CC_CONV7_RB                                     // round-2 A/B (scripts/gpu_r10g.sh)
-#define CC_CONV7_RB 4
-#endif
-#ifndef CC_CONV7_GROUPS
-#define CC_CONV7_GROUPS 2
-#endif
-#ifndef CC_CONV7_AGENTS
-#define CC_CONV7_AGENTS 6
-#endif
-    static constexpr int RB = R >= 3 ? CC_CONV7_RB : 2;
+    // (8 rows per thread -- twice the FFMA per shared-memory load -- with 2 or
+    // 4 one-warp groups measured 20-35 % slower in round 2, gpurun_out r10g)
+    static constexpr int RB = R >= 3 ? 4 : 2;
     static constexpr int kConsumers = 256 / RB;
     // two neighbouring tiles per slot for the HBM-bound 3x3 (cc_runtime.cuh:
     // MergeOf); the FP32-bound 7x7 gains nothing from the shared halo and
@@ -551,12 +544,12 @@ struct Conv2dBody {
     // two groups: with four 2-warp groups per agent (7x7) the single producer,
     // which gets only its fair share of issue slots, could not keep them fed
     // (measured 0.91x -> 0.99x of default order with two groups).
-    static constexpr int kGroups = R >= 3 ? CC_CONV7_GROUPS : 2;
+    static constexpr int kGroups = 2;
     static constexpr int kDefaultStages = 2 * kGroups; // two slots per group: the next tile lands while one computes
     static constexpr int kDefaultBatch = 4;
     // agents per SM: 3x3 4 (56 registers, no spill; measured 5 % faster than
     // 5 with spills), 7x7 6 (56 registers)
-    static constexpr int kMinAgents = R >= 3 ? CC_CONV7_AGENTS : 4;
+    static constexpr int kMinAgents = R >= 3 ? 6 : 4;
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)

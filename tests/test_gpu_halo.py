@@ -93,6 +93,42 @@ def test_virtual_slabs_full_width_sampled():
         assert np.array_equal(got[lo - 2: lo + 2], ref[lo - 2: lo + 2])
 
 
+@pytest.mark.parametrize("v", [dict(backend="agent", order="row", max_agents=1), dict(backend="default"),
+                               dict(backend="static", order="row", num_clusters=148)],
+                         ids=lambda v: v["backend"])
+def test_ll_litmus_concurrent_streams(v):
+    """LL protocol litmus: each virtual slab runs all its sweeps on its OWN
+    stream, so neighbouring slabs' sweeps execute truly concurrently and in no
+    fixed relative order (a slab may run several sweeps ahead until it blocks
+    on its neighbour's tags).  Every sweep's result must still be bit-exact and
+    no poll may time out: RAW (a reader takes exactly tag s-1) and WAR (a
+    deposit of sweep s+2 never overwrites words of sweep s before they were
+    read) under real concurrency, not only under the interleaved order."""
+    rows, cols, G, T = 260, 200, 3, 24
+    u0 = synth.matrix(4, rows, cols)
+    slabs = []
+    for g in range(G):
+        lo, hi, llo, lhi = shard.slab_range(rows, G, g, 1)
+        a = torch.from_numpy(np.ascontiguousarray(u0[llo:lhi])).cuda()
+        slabs.append(dict(a=a, b=torch.zeros_like(a), lo=lo, hi=hi, llo=llo,
+                          ll=torch.zeros(cc.ll_words(cols), dtype=torch.int64, device="cuda"),
+                          status=torch.zeros(1, dtype=torch.int32, device="cuda"), st=torch.cuda.Stream()))
+    torch.cuda.synchronize()
+
+    def nb(g):
+        return slabs[g]["ll"].data_ptr() if 0 <= g < G else None
+
+    for s in range(T):                                   # queued slab by slab; streams run concurrently
+        for g, x in enumerate(slabs):
+            src, dst = (x["a"], x["b"]) if s % 2 == 0 else (x["b"], x["a"])
+            ops.jacobi5_halo(src, dst, 1, s, x["ll"], nb(g - 1), nb(g + 1), x["status"], stream=x["st"], **v)
+    torch.cuda.synchronize()
+    got = np.concatenate([(x["a"] if T % 2 == 0 else x["b"])[x["lo"] - x["llo"]: x["hi"] - x["llo"]].cpu().numpy()
+                          for x in slabs])
+    assert [int(x["status"].item()) for x in slabs] == [0] * G
+    assert np.array_equal(got, O.jacobi5_f32(u0, T))
+
+
 def test_missing_neighbour_deposit_times_out_not_hangs():
     """Sweep 2 of slab 0 launched without slab 1's sweep 1: the bounded poll
     gives up after ~4 s and reports it in `status` instead of hanging."""
