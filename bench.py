@@ -75,7 +75,7 @@ def parse():
     ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
     ap.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
-    ap.add_argument("--hot", type=int, default=16384, help="spmv: hub slots of the inspector (0: plain CSR)")
+    ap.add_argument("--hot", type=int, default=0, help="spmv: hub slots of the inspector (0: plain CSR)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-parity", action="store_true")

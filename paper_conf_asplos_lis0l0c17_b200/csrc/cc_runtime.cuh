@@ -488,10 +488,24 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         uint32_t ph = 0;                                       // full-barrier parity (G <= S)
         for (;;) {
             mbar_wait(&R.full[st], ph);
-            const int4 sl = R.slot[st];
+            // lane 0 reads the slot descriptor and broadcasts it: the lane that
+            // later releases the slot (arrive on empty) is the only one that
+            // read it, so the producer's next write is ordered after every read
+            // by that arrive alone (compute-sanitizer racecheck is clean)
+            int4 sl = make_int4(0, 0, 0, 0), s2 = make_int4(0, 0, 1, 0);
+            if (lane == 0) {
+                sl = R.slot[st];
+                if constexpr (MergeOf<Body>::value > 1) s2 = R.slot2[st];
+            }
+            sl.x = __shfl_sync(0xffffffffu, sl.x, 0);
+            sl.y = __shfl_sync(0xffffffffu, sl.y, 0);
+            sl.z = __shfl_sync(0xffffffffu, sl.z, 0);
+            sl.w = __shfl_sync(0xffffffffu, sl.w, 0);
             if (sl.x < 0) break;
             if constexpr (MergeOf<Body>::value > 1) {
-                const int4 s2 = R.slot2[st];
+                s2.x = __shfl_sync(0xffffffffu, s2.x, 0);
+                s2.y = __shfl_sync(0xffffffffu, s2.y, 0);
+                s2.z = __shfl_sync(0xffffffffu, s2.z, 0);
                 body.consume_n(s, sl.z, sl.w, s2.z, ring + (size_t)st * s.stage_bytes, ctid);
                 if (ctid == 0) {
                     record(s, sl.x, sl.y);

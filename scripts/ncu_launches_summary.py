@@ -30,8 +30,8 @@ def main(tag):
     all_us = sum(tot.values())
     out = [f"# bench.py launch list under ncu (our kernels only; gpu__time_duration.sum, --clock-control none, "
            f"cold-cache serialised: compare shares)", "",
-           f"Command: `ncu --metrics gpu__time_duration.sum --clock-control none -k 'regex:k_(agent|default|redirect)' "
-           f"python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu-baseline` (scripts/ncu_bench.sh {tag}). The timed "
+           f"Command: `ncu --metrics gpu__time_duration.sum --clock-control none -k 'regex:k_(agent|default|redirect|static)' "
+           f"python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-parity` (scripts/ncu_bench.sh {tag}). The timed "
            f"step is the agent (COL) ATAX+BICG+MVT; the default-order (TMA and direct) steps and the identity control "
            f"are timed after it in the same run.", "",
            "| kernel | launches | total us | mean us | share |", "|---|---|---|---|---|"]

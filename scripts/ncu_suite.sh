@@ -42,12 +42,17 @@ for k in jacobi conv3 conv7; do
   run ${k}_static-row-m4 1 --kernel $k --backend static --order row --clusters 592
 done
 for k in conv3 conv7; do
+  run ${k}_tbc1 1 --kernel $k --backend tbcluster --cluster 1
   run ${k}_tbc2 1 --kernel $k --backend tbcluster --cluster 2
+  run ${k}_tbc4 1 --kernel $k --backend tbcluster --cluster 4
   run ${k}_tbc8 1 --kernel $k --backend tbcluster --cluster 8
 done
+run conv7_static-row-m7 1 --kernel conv7 --backend static --order row --clusters 1036
 run spmv_default 1 --kernel spmv --backend default
 run spmv_agent-row 1 --kernel spmv --backend agent --order row
 run spmv_identity 1 --kernel spmv --backend identity
+run spmv_default-hot 1 --kernel spmv --backend default --hot 16384
+run spmv_agent-row-hot 1 --kernel spmv --backend agent --order row --hot 16384
 run hist_default 1 --kernel hist --backend default
 run hist_agent-row 1 --kernel hist --backend agent --order row
 run hist_identity 1 --kernel hist --backend identity
