@@ -13,6 +13,7 @@
 #include <mutex>
 #include <map>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "cc_index.cuh"
@@ -592,8 +593,35 @@ static PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
     return fn;
 }
 
+// Encoded tensor maps are cached per (base, shape, leading dim, box): a
+// 100-sweep Jacobi call encodes each of its two ping-pong buffers once, not
+// once per sweep (the encode is ~1-2 us of host time per map).
+struct TmapKey {
+    const void* base; int32_t rows, cols; int64_t ld; int32_t bc, br;
+    bool operator<(const TmapKey& o) const {
+        return std::tie(base, rows, cols, ld, bc, br) < std::tie(o.base, o.rows, o.cols, o.ld, o.bc, o.br);
+    }
+};
+static cc_status make_tmap_uncached(CUtensorMap* m, const float* base, int32_t rows, int32_t cols, int64_t ld,
+                                    int box_cols, int box_rows);
 static cc_status make_tmap(CUtensorMap* m, const float* base, int32_t rows, int32_t cols, int64_t ld, int box_cols,
                            int box_rows) {
+    static std::mutex mu;
+    static std::map<TmapKey, CUtensorMap> cache;
+    const TmapKey k{base, rows, cols, ld, box_cols, box_rows};
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        auto it = cache.find(k);
+        if (it != cache.end()) { *m = it->second; return CC_OK; }
+    }
+    CC_TRY(make_tmap_uncached(m, base, rows, cols, ld, box_cols, box_rows));
+    std::lock_guard<std::mutex> lk(mu);
+    if (cache.size() >= 1024) cache.clear();
+    cache[k] = *m;
+    return CC_OK;
+}
+static cc_status make_tmap_uncached(CUtensorMap* m, const float* base, int32_t rows, int32_t cols, int64_t ld,
+                                    int box_cols, int box_rows) {
     auto enc = tmap_encoder();
     if (!enc) return fail(CC_ERR_UNSUPPORTED, "cuTensorMapEncodeTiled unavailable");
     cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
@@ -624,8 +652,8 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     if (C != 1 && C != 2 && C != 4 && C != 8) return fail(CC_ERR_INVALID_ARG, "cluster_size %d (1, 2, 4 or 8)", C);
     using G = TbcGeom<R, tbc_tw<R>()>;
     CUtensorMap m_c, m_b;
-    CC_TRY(make_tmap(&m_c, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, 32 - 2 * R));
-    CC_TRY(make_tmap(&m_b, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, 2 * R));
+    CC_TRY(make_tmap(&m_c, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, 32));
+    CC_TRY(make_tmap(&m_b, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, G::kHb));
     Sched s{};
     s.g = g;
     s.census = c.o->d_census;

@@ -11,37 +11,42 @@
 //
 // The inter-CTA reuse -- the 2R input rows straddling the boundary between
 // vertically adjacent tiles, which both tiles read -- is fetched from L2
-// ONCE per cluster and delivered to both CTAs by one TMA multicast
-// (cp.async.bulk.tensor ... .multicast::cluster, ctaMask = the two CTAs).
-// Each CTA's stage holds three regions:
-//     X[0], X[1]   2R-row boundary boxes
-//     C            its 32 - 2R interior rows (a plain TMA load, itself only)
-// The boundary between CTA b and b+1 lands in region X[b & 1] of BOTH CTAs
-// (a multicast writes the same shared-memory offset in every destination),
-// which is CTA b's bottom and CTA b+1's top boundary; CTA k therefore reads
-// its top boundary from X[(k-1) & 1] and its bottom one from X[k & 1], and the
-// tile code maps each staged row to its region (ParityRows).  The cluster's
-// outermost boundaries are loaded by CTA 0 / CTA C-1 for themselves.
+// ONCE and delivered to both CTAs of a pair (CTAs 2j and 2j+1 of the
+// cluster) by one TMA multicast (cp.async.bulk.tensor ... .multicast::cluster,
+// ctaMask = the pair).  A multicast writes the same shared-memory offset in
+// every destination, so the pair uses mirrored layouts around the shared box:
+//
+//   even CTA (upper tile)   [ own box: 32 rows | B: Hb rows ]
+//   odd CTA  (lower tile)                      [ B: Hb rows | own box: 32 rows ]
+//
+// B (Hb = 2R rounded up to 4 rows, keeping every TMA destination 128-byte
+// aligned) sits at the same offset in both; the odd CTA's ring is the even
+// one's shifted by 32 rows, so consecutive stages tile the buffer with one
+// stride (32 + Hb rows) in both.  Each CTA's staged rows are contiguous, so
+// the tile code is the agents' (ContigRows), and each CTA issues one 32-row
+// box per unit (the even one also the Hb-row multicast).  A cluster's
+// outermost boundaries, and those between pairs, are loaded by each CTA for
+// itself.
 //
 // Pipeline (per CTA, 2 consumer groups alternating units, 2 stages each,
 // warp-specialised like the agents):
 //   warp 0 lane 0 (producer)  for stage s of unit i: wait empty[s] (this CTA
-//     and CTA k+1 -- the other receiver of its multicast -- released the
-//     stage), arm full[s] with the bytes this CTA receives, issue its
-//     interior load and its bottom-boundary multicast (CTA 0 also its top);
+//     released it and, for an even CTA, so did its partner -- the other
+//     receiver of its multicast), arm full[s] with the bytes this CTA
+//     receives, issue its own 32-row box (and, even CTAs, the B multicast);
 //   consumer group            wait full[s], compute its tiles into registers,
-//     release the stage -- a local arrive on empty[s] and a remote arrive on
-//     CTA k-1's empty[s] (mbarrier.arrive.release.cluster; the producer of a
-//     CTA with a lower neighbour waits with .acquire.cluster): the WAR order
-//     between this CTA's shared-memory reads and its neighbour's next
-//     multicast into them -- then store the outputs.
+//     release the stage -- a local arrive on empty[s] and, odd CTAs, a
+//     remote arrive on the partner's empty[s] (mbarrier.arrive.release.cluster;
+//     the even producer waits with .acquire.cluster): the WAR order between
+//     the odd CTA's shared-memory reads of B and the partner's next
+//     multicast into it -- then store the outputs.
 // No CTA reads another's shared memory: all data arrives by TMA and is
 // observed through the CTA's own full barrier (complete_tx), the standard
-// async-proxy pattern.  A multicast may complete_tx on a peer's full[s]
-// before the peer armed it (the transaction count goes transiently
+// async-proxy pattern.  A multicast may complete_tx on the partner's full[s]
+// before the partner armed it (the transaction count goes transiently
 // negative); it cannot target an earlier phase, since the issuer waited for
-// the peer's release of that stage, which follows the peer's consumption of
-// the stage's previous phase.
+// the partner's release of that stage, which follows the partner's
+// consumption of the stage's previous phase.
 #pragma once
 #include <cuda.h>
 #include "cc_mem.cuh"
@@ -63,19 +68,22 @@ template <int R, int TW>
 struct TbcGeom {
     static constexpr int kCols = 32 * TW + 8;                     // staged floats per row (x0-4 ..)
     static constexpr int kRowB = kCols * 4;
-    static constexpr int kB = 2 * R;                              // boundary box rows
-    static constexpr int kC = 32 - 2 * R;                         // interior rows
-    static constexpr int kRegB = ((kB * kRowB) + 127) & ~127;     // 128-byte aligned regions
-    static constexpr int kCenB = ((kC * kRowB) + 127) & ~127;
-    static constexpr int kStageB = 2 * kRegB + kCenB;             // X[0] | X[1] | C
-    static constexpr uint32_t kRecvBytes = (uint32_t)((32 + 2 * R) * kRowB);   // per CTA per stage
+    static constexpr int kHb = (2 * R + 3) & ~3;                  // shared box rows (>= 2R, multiple of 4)
+    static constexpr int kLead = kHb / 2 - R;                     // unused rows before a CTA's first staged row
+    static constexpr int kStageRows = 32 + kHb;
+    static constexpr int kStageB = kStageRows * kRowB;            // stride of the ring (both parities)
+    static constexpr uint32_t kRecvBytes = (uint32_t)((32 + kHb) * kRowB);    // per CTA per stage
     static constexpr int kRB = R >= 3 ? 4 : 2;                    // output rows per consumer thread
     static constexpr int kConsumers = 256 / kRB;                  // per group (one tile's threads)
     static constexpr int kThreads = TBC_GROUPS * kConsumers + 32;
+    static_assert(kStageB % 128 == 0 && (32 * kRowB) % 128 == 0 && (kHb * kRowB) % 128 == 0, "TMA alignment");
 };
 template <int R> constexpr int tbc_tw() { return R >= 3 ? 1 : CC_TBC_TW3; }   // 3x3: two tiles per CTA per unit
 template <int R> constexpr int tbc_threads() { return TbcGeom<R, tbc_tw<R>()>::kThreads; }
-template <int R> inline size_t tbc_smem_bytes() { return 128 + (size_t)TBC_STAGES * TbcGeom<R, tbc_tw<R>()>::kStageB; }
+template <int R> inline size_t tbc_smem_bytes() {
+    using G = TbcGeom<R, tbc_tw<R>()>;
+    return 128 + (size_t)TBC_STAGES * G::kStageB + (size_t)32 * G::kRowB;   // + the odd CTAs' 32-row shift
+}
 
 __device__ __forceinline__ uint32_t cluster_ctarank() {
     uint32_t r;
@@ -144,21 +152,9 @@ __device__ __forceinline__ void tma_load_2d_mc(void* dst, const void* tmap, int3
                  :: "r"(smem_u32(dst)), "l"(tmap), "r"(x), "r"(y), "r"(smem_u32(bar)), "h"(mask) : "memory");
 }
 
-// staged row rr (input row y0 - R + rr) of CTA k: top boundary rows [0, 2R)
-// in X[(k-1)&1], interior rows [2R, 32) in C, bottom boundary rows [32, 32+2R) in X[k&1]
-struct ParityRows {
-    const float* top;
-    const float* cen;
-    const float* bot;
-    int pitch, b, c;      // b = 2R, c = 32
-    __device__ __forceinline__ const float* operator()(int rr) const {
-        return rr < b ? top + rr * pitch : rr < c ? cen + (rr - b) * pitch : bot + (rr - c) * pitch;
-    }
-};
-
 // Persistent grid of NC clusters x C CTAs (1D, cluster dims (C,1,1)),
 // tbc_threads<R>() threads, dynamic smem tbc_smem_bytes<R>().
-// map_c: box (kCols x (32 - 2R)), map_b: box (kCols x 2R).
+// map_c: box (kCols x 32), map_b: box (kCols x Hb).
 template <int R>
 __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_constant__ CUtensorMap map_c,
                                                           const __grid_constant__ CUtensorMap map_b,
@@ -175,11 +171,13 @@ __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_cons
     const int ubs = (gy + C - 1) / C;                    // unit rows
     const int units = ucols * ubs;
     const int c0 = (int)cluster_id_x(), NC = (int)nclusters_x();
-    const bool has_next = k < C - 1;
+    const bool odd = k & 1;
+    const bool partner = !odd && k + 1 < C;              // even CTA with a lower partner: it multicasts B
+    uint8_t* base = ring + (odd ? (size_t)32 * G::kRowB : 0);
     if (threadIdx.x == 0) {
         for (int b = 0; b < TBC_STAGES; ++b) {
             mbar_init(&full[b], 1);
-            mbar_init(&empty[b], has_next ? 2 : 1);      // the owning group + CTA k+1's
+            mbar_init(&empty[b], partner ? 2 : 1);       // the owning group (+ the partner's)
         }
         fence_mbar_init();
     }
@@ -188,25 +186,29 @@ __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_cons
     if (threadIdx.x < 32) {
         // ---- producer
         if (threadIdx.x == 0) {
-            const uint16_t mask = (uint16_t)((1u << k) | (has_next ? 1u << (k + 1) : 0u));
+            const uint16_t mask = (uint16_t)((1u << k) | (partner ? 1u << (k + 1) : 0u));
             int i = 0;
             for (int u = c0; u < units; u += NC, ++i) {
                 const int st = i % TBC_STAGES;
                 if (i >= TBC_STAGES) {
                     const uint32_t ph = (uint32_t)((i / TBC_STAGES) - 1) & 1u;
-                    if (has_next) mbar_wait_acquire_cluster(&empty[st], ph);     // a peer releases too
+                    if (partner) mbar_wait_acquire_cluster(&empty[st], ph);      // the partner releases too
                     else mbar_wait(&empty[st], ph);
                 }
-                uint8_t* stage = ring + (size_t)st * G::kStageB;
+                uint8_t* stage = base + (size_t)st * G::kStageB;
                 const int x0 = (u % ucols) * 32 * TW, y0 = ((u / ucols) * C + k) * 32;
                 mbar_arrive_tx(&full[st], G::kRecvBytes);
-                tma_load_2d(stage + 2 * G::kRegB, &map_c, x0 - 4, y0 + R, &full[st]);     // interior
-                if (k == 0)                                                                  // cluster top
-                    tma_load_2d(stage + G::kRegB, &map_b, x0 - 4, y0 - R, &full[st]);      // X[1]
-                // bottom boundary into X[k & 1]: shared with CTA k+1 (its top) by one
-                // multicast; a cluster's last CTA loads its own
-                if (has_next) tma_load_2d_mc(stage + (k & 1) * G::kRegB, &map_b, x0 - 4, y0 + 32 - R, &full[st], mask);
-                else tma_load_2d(stage + (k & 1) * G::kRegB, &map_b, x0 - 4, y0 + 32 - R, &full[st]);
+                if (!odd) {
+                    // own rows [y0 - Hb/2, y0 + 32 - Hb/2), then B = the Hb rows
+                    // centred on the boundary below (multicast to the partner)
+                    const int yb = y0 + 32 - G::kHb / 2;
+                    tma_load_2d(stage, &map_c, x0 - 4, yb - 32, &full[st]);
+                    if (partner) tma_load_2d_mc(stage + 32 * G::kRowB, &map_b, x0 - 4, yb, &full[st], mask);
+                    else tma_load_2d(stage + 32 * G::kRowB, &map_b, x0 - 4, yb, &full[st]);
+                } else {
+                    // B arrives from the partner; own rows [y0 + Hb/2, y0 + Hb/2 + 32)
+                    tma_load_2d(stage + G::kHb * G::kRowB, &map_c, x0 - 4, y0 + G::kHb / 2, &full[st]);
+                }
             }
         }
     } else {
@@ -217,23 +219,18 @@ __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_cons
         for (int u = c0 + grp * NC; u < units; u += TBC_GROUPS * NC, i += TBC_GROUPS) {
             const int st = i % TBC_STAGES;
             mbar_wait(&full[st], (uint32_t)(i / TBC_STAGES) & 1u);
-            const uint8_t* stage = ring + (size_t)st * G::kStageB;
-            const float* top = reinterpret_cast<const float*>(stage + ((k - 1) & 1) * G::kRegB);
-            const float* bot = reinterpret_cast<const float*>(stage + (k & 1) * G::kRegB);
-            const float* cen = reinterpret_cast<const float*>(stage + 2 * G::kRegB);
+            // staged row rr = input row y0 - R + rr, contiguous from here in both parities
+            const float* rows0 = reinterpret_cast<const float*>(base + (size_t)st * G::kStageB) + G::kLead * G::kCols;
             const int bx0 = (u % ucols) * TW, by = (u / ucols) * C + k;
             // all TW tiles into registers, release the stage, then store: the
             // release's cluster-scope fence then has no fresh stores to drain
             float acc[TW][G::kRB][4];
 #pragma unroll
-            for (int t = 0; t < TW; ++t) {
-                const ParityRows rows{top + 32 * t, cen + 32 * t, bot + 32 * t, G::kCols, 2 * R, 32};
-                conv_tile_acc<R, G::kRB>(p, rows, ctid, acc[t]);
-            }
+            for (int t = 0; t < TW; ++t) conv_tile_acc<R, G::kRB>(p, ContigRows{rows0 + 32 * t, G::kCols}, ctid, acc[t]);
             consumer_sync<G::kConsumers>();              // every thread of the group is done reading
             if (ctid == 0) {
                 mbar_arrive(&empty[st]);
-                if (k > 0) mbar_arrive_remote_release(&empty[st], (uint32_t)(k - 1));
+                if (odd) mbar_arrive_remote_release(&empty[st], (uint32_t)(k - 1));
             }
             if (by < gy) {
 #pragma unroll

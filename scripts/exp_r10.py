@@ -36,6 +36,65 @@ def spmv():
     return out
 
 
+def spmv_control():
+    """SpMV data-related class: (1) the no-locality control -- the same R-MAT
+    graph with its vertices randomly relabelled; (2) an
+    inspector-built USER order -- logical CTAs (merge-path blocks) sorted by
+    the mean column they gather, so blocks reading similar x regions share a
+    cluster (P:1771 'customized partition provided by users', P:1925)."""
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    rp, col = synth.rmat_csr(7, 24, 16, backend="torch", device="cuda")
+    n, nnz = rp.numel() - 1, col.numel()
+    val = synth.uniform(8, nnz, backend="torch", device="cuda")
+    x = synth.uniform(9, n, backend="torch", device="cuda")
+    y = torch.empty(n, device="cuda")
+    nbytes = 8 * nnz + 4 * (n + 1) + 8 * n
+    out = {}
+    Am = ops.SpmvMatrix(rp, col, val)
+    # inspector USER order over the logical CTAs
+    part = Am.part.cpu().numpy().astype(np.int64)
+    rph = rp.cpu().numpy().astype(np.int64)
+    colh = col.cpu().numpy().astype(np.int64)
+    IPC = 4096
+    nb = part.size - 1
+    d0 = np.arange(nb, dtype=np.int64) * IPC
+    y0 = d0 - part[:-1]                             # first nonzero of each block
+    y1 = np.minimum(d0 + IPC, n + nnz) - part[1:]
+    csum = np.concatenate([[0], np.cumsum(colh)])
+    cnt = np.maximum(y1 - y0, 1)
+    mean_col = (csum[np.minimum(y1, nnz)] - csum[np.minimum(y0, nnz)]) / cnt
+    user = np.argsort(mean_col, kind="stable").astype(np.int32)
+    variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
+                ("identity", dict(backend="identity")),
+                ("agent-user-meancol", dict(backend="agent", order="user", user_order=user))]
+    r = B.measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 20, nbytes, graph=True, inner=B.GRAPH_INNER)
+    out["rmat"] = r
+    print("rmat", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    del Am
+    # no-locality control: relabel every vertex by a random permutation
+    perm = torch.from_numpy(synth.random_permutation(3, n)).cuda()
+    rows_of = torch.repeat_interleave(torch.arange(n, device="cuda"), (rp[1:] - rp[:-1]).long())
+    keys = perm[rows_of] * n + perm[col.long()]
+    keys, idx = torch.sort(keys)
+    val2 = val[idx]
+    del rows_of, idx
+    r2 = (keys // n)
+    col2 = (keys % n).to(torch.int32)
+    del keys
+    counts = torch.bincount(r2, minlength=n)
+    rp2 = torch.zeros(n + 1, dtype=torch.int64, device="cuda")
+    torch.cumsum(counts, 0, out=rp2[1:])
+    Ap = ops.SpmvMatrix(rp2.to(torch.int32), col2, val2)
+    variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
+                ("identity", dict(backend="identity"))]
+    r = B.measure(variants, lambda kw: ops.spmv(Ap, x, y, **kw), 20, nbytes, graph=True, inner=B.GRAPH_INNER)
+    out["rmat_permuted"] = r
+    print("rmat_permuted", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    return out
+
+
 def stencil():
     import numpy as np
     import torch
@@ -141,5 +200,6 @@ def conv7():
 
 if __name__ == "__main__":
     what, path = sys.argv[1], sys.argv[2]
-    res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel, "conv7": conv7}[what]()
+    res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel, "conv7": conv7,
+           "spmv_control": spmv_control}[what]()
     json.dump(res, open(path, "w"), indent=1)

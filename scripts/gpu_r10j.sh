@@ -1,0 +1,15 @@
+# TB-cluster pair layout (parity + perf), SpMV controls (permuted R-MAT, inspector USER order), agent L2 prefetch A/B
+mkdir -p gpurun_out/r10j
+L=paper_conf_asplos_lis0l0c17_b200
+make all > gpurun_out/r10j/build.log 2>&1 || tail -20 gpurun_out/r10j/build.log
+make LIB=$L/lib_nopf.so CC_DEFS="-DCC_SPMV_PREFETCH=0" PTXLOG=/tmp/p_nopf.log > /dev/null 2>&1 &
+timeout -k 10 600 python -m pytest tests/test_gpu_kernels.py -q -x --timeout 400 -k "tbc or conv" > gpurun_out/r10j/t_conv.log 2>&1; echo tconv=$?
+timeout -k 10 600 python scripts/sanitize_targets.py tbc > gpurun_out/r10j/san_tbc_plain.log 2>&1; echo santbc=$?
+timeout -k 10 600 compute-sanitizer --tool racecheck --error-exitcode 9 python scripts/sanitize_targets.py tbc > gpurun_out/r10j/racecheck_tbc.log 2>&1; echo race_tbc=$?
+timeout -k 10 600 compute-sanitizer --tool synccheck --error-exitcode 9 python scripts/sanitize_targets.py tbc > gpurun_out/r10j/synccheck_tbc.log 2>&1; echo sync_tbc=$?
+timeout -k 10 600 python scripts/exp_r10.py tbc gpurun_out/r10j/tbc.json > gpurun_out/r10j/tbc.log 2>&1; echo tbc=$?
+bash scripts/ncu_full.sh r10j conv3_tbc2:"--kernel conv3 --backend tbcluster --cluster 2" > gpurun_out/r10j/ncu.log 2>&1
+timeout -k 10 900 python scripts/exp_r10.py spmv_control gpurun_out/r10j/spmv_control.json > gpurun_out/r10j/spmv_control.log 2>&1; echo spc=$?
+wait
+echo "== nopf"; CTACLUST_LIB=$PWD/$L/lib_nopf.so timeout -k 10 900 python scripts/exp_r10.py spmv gpurun_out/r10j/spmv_nopf.json 2>&1 | head -3 | cut -c1-400
+tail -2 gpurun_out/r10j/t_conv.log; tail -2 gpurun_out/r10j/racecheck_tbc.log gpurun_out/r10j/synccheck_tbc.log; cat gpurun_out/r10j/tbc.log gpurun_out/r10j/spmv_control.log | cut -c1-900
