@@ -23,7 +23,7 @@ def spmv():
     y = torch.empty(n, device="cuda")
     nbytes = 8 * nnz + 4 * (n + 1) + 8 * n
     out = {}
-    for hot in (0, 4096, 16384, 32768, 65536):
+    for hot in [int(h) for h in os.environ.get("EXP_SPMV_HOTS", "0,4096,16384,32768,65536").split(",")]:
         Am = ops.SpmvMatrix(rp, col, val, hot=hot)
         variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
                     ("identity", dict(backend="identity")),

@@ -11,5 +11,6 @@ timeout -k 10 600 python scripts/exp_r10.py tbc gpurun_out/r10j/tbc.json > gpuru
 bash scripts/ncu_full.sh r10j conv3_tbc2:"--kernel conv3 --backend tbcluster --cluster 2" > gpurun_out/r10j/ncu.log 2>&1
 timeout -k 10 900 python scripts/exp_r10.py spmv_control gpurun_out/r10j/spmv_control.json > gpurun_out/r10j/spmv_control.log 2>&1; echo spc=$?
 wait
-echo "== nopf"; CTACLUST_LIB=$PWD/$L/lib_nopf.so timeout -k 10 900 python scripts/exp_r10.py spmv gpurun_out/r10j/spmv_nopf.json 2>&1 | head -3 | cut -c1-400
+echo "== base"; EXP_SPMV_HOTS=0 timeout -k 10 900 python scripts/exp_r10.py spmv gpurun_out/r10j/spmv_base.json 2>&1 | head -3 | cut -c1-400
+echo "== nopf"; EXP_SPMV_HOTS=0 CTACLUST_LIB=$PWD/$L/lib_nopf.so timeout -k 10 900 python scripts/exp_r10.py spmv gpurun_out/r10j/spmv_nopf.json 2>&1 | head -3 | cut -c1-400
 tail -2 gpurun_out/r10j/t_conv.log; tail -2 gpurun_out/r10j/racecheck_tbc.log gpurun_out/r10j/synccheck_tbc.log; cat gpurun_out/r10j/tbc.log gpurun_out/r10j/spmv_control.log | cut -c1-900
