@@ -228,6 +228,17 @@ def _launch(kernel, args, opts, stream, **plan_kw):
 # ----------------------------------------------------------------------------
 # config 3: Jacobi, slab-sharded with boundary-first overlap
 # ----------------------------------------------------------------------------
+def sweep_windows(own0: int, own1: int, band: int = 32):
+    """Row windows of one overlapped sweep of a slab whose owned local rows are
+    [own0, own1) (own1 - own0 > 2 * band): the two boundary windows -- the
+    first and last `band` owned rows, computed first because the halo
+    exchange sends their edge rows -- and the interior window between them
+    (None when empty).  Together they cover the owned rows exactly once."""
+    t1, b0 = own0 + band, own1 - band
+    assert b0 >= t1, "slab too thin to split"
+    return [(own0, t1), (b0, own1)], ((t1, b0) if b0 > t1 else None)
+
+
 class JacobiSlab:
     """This rank's slab of the rows x cols Jacobi (u0 = seed 4), `iters` sweeps
     per step.
@@ -251,9 +262,7 @@ class JacobiSlab:
         self.own = (own0, own1)
         self.overlap = overlap and xchg.world > 1 and own1 - own0 > 64
         if self.overlap:
-            t1, b0 = own0 + 32, own1 - 32
-            self.windows_b = [(own0, t1), (b0, own1)]
-            self.window_i = (t1, b0) if b0 > t1 else None
+            self.windows_b, self.window_i = sweep_windows(own0, own1)
         self.comm_stream = torch.cuda.Stream(device=dev) if xchg.world > 1 else None
         self.ev_b = [torch.cuda.Event() for _ in range(2)]
         self.ev_x = [torch.cuda.Event() for _ in range(2)]

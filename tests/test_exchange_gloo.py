@@ -76,3 +76,20 @@ def test_world1_exchange_is_noop():
     r = torch.zeros(3)
     X.allgather(t, r)
     assert torch.equal(r, t)
+
+
+def test_sweep_windows_cover_owned_rows_once():
+    from paper_conf_asplos_lis0l0c17_b200 import drivers
+    for rows, world in ((16384, 8), (330, 2), (330, 4), (1000, 3)):
+        for g in range(world):
+            lo, hi, llo, lhi = shard.slab_range(rows, world, g, 1)
+            own0, own1 = lo - llo, hi - llo
+            if own1 - own0 <= 64:
+                continue
+            wb, wi = drivers.sweep_windows(own0, own1)
+            cover = np.zeros(lhi - llo, np.int64)
+            for a, b in wb + ([wi] if wi else []):
+                cover[a:b] += 1
+            assert np.all(cover[own0:own1] == 1)            # every owned row exactly once
+            assert not cover[:own0].any() and not cover[own1:].any()   # halo rows never written
+            assert wb[0][0] == own0 and wb[1][1] == own1        # the exchanged edge rows are in the boundary windows
