@@ -117,26 +117,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 }
 // (Round 1 measured exponential nanosleep back-off and test_wait + timed
 // sleep in place of the suspend-hint wait, for the producer and the
-// consumers of the memory-bound bodies: slower or equal -- profiles/r05/diag,
-// r07/diag.)  A compute-bound body whose ring is always full keeps its
-// producer waiting on `empty` nearly all the time, and the suspend-hint wait
-// re-issues on every sync-unit event of the SM (conv 7x7: 15 % of all issued
-// instructions, ncu r10h); such a body sets kProducerSleepNs and its producer
-// polls with test_wait and a fixed sleep instead.
-__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
-    uint32_t ok;
-    asm volatile("{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-                 "selp.u32 %0, 1, 0, p;\n}" : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
-    return ok != 0;
-}
-template <uint32_t kNs>
-__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
-    if constexpr (kNs == 0) {
-        mbar_wait(bar, parity);
-    } else {
-        while (!mbar_test(bar, parity)) __nanosleep(kNs);
-    }
-}
+// consumers: slower or equal -- profiles/r05/diag, r07/diag.  Round 2
+// re-measured a fixed 250-2000 ns producer sleep on the FP32-bound 7x7 conv,
+// whose producer waits on `empty` 5 M times per launch (15 % of its issued
+// instructions, ncu r10h): equal or up to 10 % slower, gpurun_out r10j.)
 // 1D bulk async copy global -> shared, completion counted on `bar` (UBLKCP).
 // dst, src 16-byte aligned, bytes a multiple of 16.
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -376,11 +360,6 @@ template <class B> constexpr int direct_stage_bytes() { return DirectStageBytes<
 // cluster.  Their tiles share halo columns, so one wider copy stages both:
 // the clustered order is what makes the pair co-located, and the shared
 // halo is then reused from shared memory instead of being copied twice.
-template <class B, class = void> struct ProducerSleepNs { static constexpr uint32_t value = 0; };
-template <class B> struct ProducerSleepNs<B, decltype((void)B::kProducerSleepNs)> {
-    static constexpr uint32_t value = B::kProducerSleepNs;
-};
-
 template <class B, class = void> struct MergeOf { static constexpr int value = 1; };
 template <class B> struct MergeOf<B, decltype((void)B::kMerge)> { static constexpr int value = B::kMerge; };
 
@@ -444,7 +423,7 @@ __device__ __forceinline__ void agent_loop(const Sched& s, Body& body) {
         if (lane == 0) s_uwin[0] = -64;
         __syncwarp();
         for (;; ++t) {
-            if (t >= S) mbar_wait_sleep<ProducerSleepNs<Body>::value>(&R.empty[st], ph ^ 1u);
+            if (t >= S) mbar_wait(&R.empty[st], ph ^ 1u);
             const int32_t v = pending >= 0 ? pending : producer_next<kStatic>(s, P, lane);
             pending = -1;
             if (v < 0) {

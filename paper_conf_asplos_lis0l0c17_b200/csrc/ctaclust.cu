@@ -671,13 +671,18 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     at[0].val.clusterDim.y = 1;
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
-    cfg.numAttrs = 1;
+    cfg.numAttrs = C > 1 ? 1 : 0;                // C = 1: a plain launch (implicit 1-CTA clusters)
     // persistent: as many clusters as can be co-resident (not more than units)
     const int TW = tbc_tw<R>();
     const long units = (long)((g.gx + TW - 1) / TW) * ((g.gy + C - 1) / C);
     cfg.gridDim = dim3(C);
     int nc = 0;
-    CC_CUDA(cudaOccupancyMaxActiveClusters(&nc, k_conv_tbc<R>, &cfg));
+    if (C > 1) {
+        CC_CUDA(cudaOccupancyMaxActiveClusters(&nc, k_conv_tbc<R>, &cfg));
+    } else {
+        CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nc, k_conv_tbc<R>, tbc_threads<R>(), smem));
+        nc *= c.p->facts->num_sms;
+    }
     if (nc < 1) return fail(CC_ERR_UNSUPPORTED, "tbcluster: no cluster of %d fits", C);
     if (nc > units) nc = (int)units;
     cfg.gridDim = dim3(nc * C);

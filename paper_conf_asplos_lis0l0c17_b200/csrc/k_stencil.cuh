@@ -550,10 +550,6 @@ struct Conv2dBody {
     // agents per SM: 3x3 4 (56 registers, no spill; measured 5 % faster than
     // 5 with spills), 7x7 6 (56 registers)
     static constexpr int kMinAgents = R >= 3 ? 6 : 4;
-#ifndef CC_CONV7_PROD_NS
-#define CC_CONV7_PROD_NS 0                              // round-2 A/B (scripts/gpu_r10j.sh)
-#endif
-    static constexpr uint32_t kProducerSleepNs = R >= 3 ? CC_CONV7_PROD_NS : 0;
     using Params = ConvParams<R>;
     const ConvParams<R>& p;  // __grid_constant__ kernel parameter (filter in the param bank)
     int32_t l2h = 0;         // cc_l2_hint bits; set by k_agent only (one-shot kernels keep the literal 0)
