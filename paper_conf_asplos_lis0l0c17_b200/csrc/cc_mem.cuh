@@ -127,6 +127,13 @@ __device__ __forceinline__ float ld_cached_issue(const float* p) {
     asm volatile("ld.global.f32 %0, [%1];" : "=f"(v) : "l"(p));
     return v;
 }
+// x gather that skips L1 (cached in L2 only): one L2 request per lane with no
+// L1 tag lookup or fill
+__device__ __forceinline__ float ld_l2only_issue(const float* p) {
+    float v;
+    asm volatile("ld.global.cg.f32 %0, [%1];" : "=f"(v) : "l"(p));
+    return v;
+}
 // hub values of the SpMV hub-column form: allocate in L1 and keep (evict_last)
 __device__ __forceinline__ float ld_hot_issue(const float* p) {
     float v;

@@ -88,6 +88,9 @@ constexpr int SPMV_GB = CC_SPMV_GB;                 // gathers in flight per thr
 #ifndef CC_SPMV_PREFETCH
 #define CC_SPMV_PREFETCH 1
 #endif
+#ifndef CC_SPMV_XCG
+#define CC_SPMV_XCG 0                               // round-2 A/B: x gathers L2-only (ld.global.cg)
+#endif
 #ifndef CC_SPMV_MIN_AGENTS
 #define CC_SPMV_MIN_AGENTS 5
 #endif
@@ -190,7 +193,7 @@ struct SpmvBody {
                 for (int k = 0; k < SPMV_GB; ++k) {
                     // hub references (negative, hub-column form) read the dense
                     // hub array, which stays in L1; others gather x
-                    if (c[k] >= 0) xv[k] = ld_cached_issue(p.x + c[k]);
+                    if (c[k] >= 0) xv[k] = CC_SPMV_XCG ? ld_l2only_issue(p.x + c[k]) : ld_cached_issue(p.x + c[k]);
                     else xv[k] = ld_hot_issue(p.xh_end + c[k]);
                 }
 #pragma unroll

@@ -55,14 +55,11 @@
 
 namespace cc {
 
-#ifndef CC_TBC_SPG
-#define CC_TBC_SPG 2                          // stages per consumer group (round-2 A/B)
-#endif
-#ifndef CC_TBC_TW3
-#define CC_TBC_TW3 2                          // 3x3 tiles per CTA per unit (round-2 A/B)
-#endif
-constexpr int TBC_GROUPS = 2;                 // consumer groups, alternate units
-constexpr int TBC_STAGES = CC_TBC_SPG * TBC_GROUPS;
+// Two consumer groups alternate units, two stages each, and a 3x3 unit is two
+// tiles wide: the measured best (round 2: 3 or 4 stages per group, fewer CTAs
+// per SM, 12-28 % slower; one-tile units 30 % slower; profiles/r10/exp/tbc_*).
+constexpr int TBC_GROUPS = 2;
+constexpr int TBC_STAGES = 2 * TBC_GROUPS;
 
 template <int R, int TW>
 struct TbcGeom {
@@ -78,7 +75,7 @@ struct TbcGeom {
     static constexpr int kThreads = TBC_GROUPS * kConsumers + 32;
     static_assert(kStageB % 128 == 0 && (32 * kRowB) % 128 == 0 && (kHb * kRowB) % 128 == 0, "TMA alignment");
 };
-template <int R> constexpr int tbc_tw() { return R >= 3 ? 1 : CC_TBC_TW3; }   // 3x3: two tiles per CTA per unit
+template <int R> constexpr int tbc_tw() { return R >= 3 ? 1 : 2; }   // 3x3: two tiles per CTA per unit
 template <int R> constexpr int tbc_threads() { return TbcGeom<R, tbc_tw<R>()>::kThreads; }
 template <int R> inline size_t tbc_smem_bytes() {
     using G = TbcGeom<R, tbc_tw<R>()>;
