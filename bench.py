@@ -75,11 +75,16 @@ def parse():
     ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
     ap.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
-    ap.add_argument("--hot", type=int, default=0, help="spmv: hub slots of the inspector (0: plain CSR)")
+    ap.add_argument("--hot", type=int, default=16384, help="spmv: hub slots of the inspector (0: plain CSR)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-parity", action="store_true")
     ap.add_argument("--suite", default=None, help="also run every BASELINE config's variants, write JSON here")
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "torch"],
+                    help="N > 1 exchanges: the library's NCCL communicator (default) or torch.distributed/gloo "
+                         "(tests only)")
+    ap.add_argument("--same-device", action="store_true",
+                    help="tests only: run every rank on GPU 0 (exercises the N > 1 code on a 1-GPU box)")
     a = ap.parse_args()
     if not a.steps:
         a.steps = {"atax": 100, "jacobi": 10, "conv3": 200, "conv7": 200, "spmv": 50}[a.config]
@@ -349,10 +354,15 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if a.same_device:                 # test harness: every rank on GPU 0 (gloo exchanges), never a measurement
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    X = drivers.make_exchange("nccl", world, rank, local)
+        if a.exchange == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
+    X = drivers.make_exchange(a.exchange, world, rank, local)
     dev = torch.device("cuda", local)
     D = build_driver(a, X, dev)
     torch.cuda.synchronize()
@@ -377,7 +387,7 @@ def main():
 
     def maxr(v):
         if world > 1:
-            t = torch.tensor([v], device=dev)
+            t = torch.tensor([v], device=dev if dist.get_backend() == "nccl" else "cpu")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             return t.item()
         return v

@@ -440,11 +440,11 @@ class SpmvBlock(GraphStep):
         self.yall = torch.zeros(self.cap * xchg.world, device=dev)
 
     def _cap(self, xchg):
-        n = torch.tensor([self.hi - self.lo], device=self.dev)
-        if xchg.world > 1:
-            h = n.cpu()
-            dist.all_reduce(h, op=dist.ReduceOp.MAX)
-            n = h
+        """rows of the largest block (the padded all-gather's block size)"""
+        if xchg.world == 1:
+            return self.hi - self.lo
+        n = torch.tensor([self.hi - self.lo], device=self.dev if dist.get_backend() == "nccl" else "cpu")
+        dist.all_reduce(n, op=dist.ReduceOp.MAX)
         return int(n.item())
 
     def step_eager(self, opts: dict, stream=None) -> int:

@@ -213,3 +213,23 @@ def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     res = [ln for o in outs for ln in o.splitlines() if ln.startswith("RESULT")]
     assert len(res) == world, (outs, [p.returncode for p in procs])
     assert all(ln.split()[2] == "True" for ln in res), res
+
+
+@pytest.mark.parametrize("cfg", ["atax", "jacobi", "conv3", "spmv"])
+def test_bench_two_ranks_one_gpu(cfg):
+    """bench.py's N > 1 path end to end (torchrun, 2 ranks, every rank on GPU 0
+    with gloo exchanges -- a harness mode, not a measurement): one JSON line
+    from rank 0 with n_gpus 2 and a passing sampled parity probe."""
+    import json
+    env = dict(os.environ, PYTHONPATH=ROOT)
+    size = {"atax": ["--n", "2048"], "jacobi": ["--n", "1024", "--iters", "10"], "conv3": ["--n", "1024"],
+            "spmv": ["--n", "14"]}[cfg]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", _port(), os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--steps", "3", "--warmup", "3", "--config", cfg, "--exchange", "torch",
+           "--same-device", "--no-e2e", "--no-cpu-baseline", "--no-graph"] + size
+    out = subprocess.run(cmd, capture_output=True, text=True, timeout=600, env=env, cwd=ROOT)
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert out.returncode == 0 and len(lines) == 1, (out.stdout[-3000:], out.stderr[-3000:])
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["parity"]["ok"], d["parity"]
