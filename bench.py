@@ -74,6 +74,8 @@ def parse():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
+    ap.add_argument("--halo", default="exchange", choices=["exchange", "fused"],
+                    help="jacobi N > 1: NCCL halo exchange per sweep, or the fused peer-memory LL halo")
     ap.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
     ap.add_argument("--hot", type=int, default=16384, help="spmv: hub slots of the inspector (0: plain CSR)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -336,7 +338,8 @@ def build_driver(a, X, dev):
     if a.config == "atax":
         return drivers.AtaxFamily(sz["n"], X, dev)
     if a.config == "jacobi":
-        return drivers.JacobiSlab(sz["side"], sz["side"], sz["iters"], X, dev, overlap=not a.no_overlap)
+        return drivers.JacobiSlab(sz["side"], sz["side"], sz["iters"], X, dev, overlap=not a.no_overlap,
+                                  halo=a.halo)
     if a.config in ("conv3", "conv7"):
         return drivers.ConvSlab(sz["side"], sz["side"], sz["R"], X, dev)
     return drivers.SpmvBlock(sz["scale"], X, dev, hot=a.hot)
@@ -525,7 +528,7 @@ def config_block(a, D, head, world, use_graph):
         c.update(n=D.n, tile="32x256", l2="inputs (1 GiB) larger than L2 (126 MB); no flush")
     elif a.config == "jacobi":
         c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32",
-                 overlap=getattr(D, "overlap", False),
+                 overlap=getattr(D, "overlap", False), halo="fused LL (peer memory)" if D.fused else "exchange",
                  l2="2 x 1 GiB ping-pong buffers, larger than L2; no flush")
     elif a.config in ("conv3", "conv7"):
         c.update(rows=D.rows, cols=D.cols, R=D.R, tile="32x32",

@@ -247,9 +247,17 @@ class JacobiSlab:
     computed first (row windows of CC_K_JACOBI5); the halo exchange of the
     freshly written boundary rows runs on `comm_stream` while the interior
     rows compute; the next sweep waits for both.  Without overlap (or at
-    world = 1) a sweep is one launch, then the exchange."""
+    world = 1) a sweep is one launch, then the exchange.
 
-    def __init__(self, rows: int, cols: int, iters: int, xchg: Exchange, device, overlap: bool = True):
+    halo="fused" (world > 1): no exchange step at all -- each sweep is one
+    CC_K_JACOBI5_HALO launch that stores its boundary rows as {value, sweep}
+    words straight into the neighbours' LL buffers (peer memory mapped with
+    CUDA IPC, shard.PeerHaloSlab) and reads its own (S§8(f)4).  Sweeps are
+    numbered absolutely across steps (the LL tags), so fused steps run
+    eagerly (a replayed graph would repeat the tags)."""
+
+    def __init__(self, rows: int, cols: int, iters: int, xchg: Exchange, device, overlap: bool = True,
+                 halo: str = "exchange"):
         self.rows, self.cols, self.iters, self.x = rows, cols, iters, xchg
         self.lo, self.hi, self.llo, self.lhi = shard.slab_range(rows, xchg.world, xchg.rank, 1)
         L = self.lhi - self.llo
@@ -267,14 +275,36 @@ class JacobiSlab:
         self.ev_b = [torch.cuda.Event() for _ in range(2)]
         self.ev_x = [torch.cuda.Event() for _ in range(2)]
         self.graph = None
+        self.fused = halo == "fused" and xchg.world > 1
+        self.peer = None
+        if self.fused:
+            self.overlap = False
+            self.a.copy_(self.u0)
+            self.peer = shard.PeerHaloSlab(self.a, self.b, xchg.world, xchg.rank)
+        self.sweep = 0
         self.reset()
 
     def reset(self):
         self.a.copy_(self.u0)
         self.b.copy_(self.u0)        # boundary rows / halo rows defined in both buffers
+        if self.fused:               # restart at sweep 1: every rank's LL buffer zero first
+            self.peer.ll.zero_()
+            self.peer.status.zero_()
+            torch.cuda.synchronize(self.dev)
+            if self.x.world > 1:
+                dist.barrier()
+        self.sweep = 0
+
+    def _sweep_fused(self, src, dst, opts, stream):
+        pr = self.peer
+        args, _ = cc.jacobi5_halo_args(src, dst, 1, self.sweep, pr.ll, pr.up_ll, pr.dn_ll, pr.status)
+        self.sweep += 1
+        return _launch("jacobi5_halo", args, opts, stream)
 
     def _sweep(self, src, dst, opts, stream, k):
         nl = 0
+        if self.fused:
+            return self._sweep_fused(src, dst, opts, stream)
         if not self.overlap:
             nl += _launch("jacobi5", cc.jacobi5_args(src, dst, 1)[0], opts, stream)
             self.x.halo_exchange(dst, 1, stream)
@@ -313,7 +343,7 @@ class JacobiSlab:
         later steps replay it.  Plans and tensor maps are created by an eager
         step first (no allocation is legal during capture).  Returns False when
         the exchange cannot be captured."""
-        if not self.x.capturable or self.iters % 2:
+        if not self.x.capturable or self.iters % 2 or self.fused:
             return False
         self.step(opts)
         torch.cuda.synchronize()

@@ -148,12 +148,19 @@ WORKER = textwrap.dedent("""
         ok, info = max(errs) <= 1e-4, str(errs)
     elif cfg.startswith("jacobi"):
         rows, cols, T = 330, 200, 6
-        d = drivers.JacobiSlab(rows, cols, T, X, "cuda", overlap=cfg == "jacobi")
+        d = drivers.JacobiSlab(rows, cols, T, X, "cuda", overlap=cfg == "jacobi",
+                               halo="fused" if cfg == "jacobi-fused" else "exchange")
+        ref = O.jacobi5_f32(synth.matrix(4, rows, cols), T)
+        ref2 = O.jacobi5_f32(synth.matrix(4, rows, cols), 2 * T)
         d.step(dict(backend="agent", order="row", max_agents=1))
         torch.cuda.synchronize()
-        ref = O.jacobi5_f32(synth.matrix(4, rows, cols), T)
-        got = d.result().cpu().numpy()
-        ok, info = bool(np.array_equal(got, ref[d.lo:d.hi])), f"overlap={{d.overlap}}"
+        ok = bool(np.array_equal(d.result().cpu().numpy(), ref[d.lo:d.hi]))
+        d.step(dict(backend="agent", order="row", max_agents=1))      # a second step continues the sweeps
+        torch.cuda.synchronize()
+        ok = ok and bool(np.array_equal(d.result().cpu().numpy(), ref2[d.lo:d.hi]))
+        if d.fused:
+            ok = ok and int(d.peer.status.item()) == 0
+        info = f"overlap={{d.overlap}} fused={{d.fused}}"
     elif cfg.startswith("conv"):
         R = int(cfg[4:])
         rows, cols = 190, 150
@@ -195,7 +202,7 @@ def _port():
 
 
 @pytest.mark.parametrize("cfg,world", [("atax", 2), ("atax", 4), ("jacobi", 2), ("jacobi", 3), ("jacobi", 4),
-                                       ("jacobi-nooverlap", 3), ("conv1", 2), ("conv3", 3), ("spmv", 2),
+                                       ("jacobi-nooverlap", 3), ("jacobi-fused", 2), ("jacobi-fused", 3), ("conv1", 2), ("conv3", 3), ("spmv", 2),
                                        ("spmv", 3), ("spmv-hot", 2)])
 def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     script = tmp_path / "w.py"
