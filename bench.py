@@ -65,7 +65,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=0, help="timed steps (default per config)")
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=0, help="problem size override (atax n, jacobi/conv side, spmv scale)")
+    ap.add_argument("--size", "--n", dest="n", type=int, default=0,
+                    help="problem size override (atax n, jacobi/conv side, spmv scale)")
     ap.add_argument("--iters", type=int, default=100, help="jacobi sweeps per step")
     ap.add_argument("--backend", default=None)
     ap.add_argument("--order", default=None)

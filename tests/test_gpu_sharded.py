@@ -229,8 +229,8 @@ def test_bench_two_ranks_one_gpu(cfg):
     from rank 0 with n_gpus 2 and a passing sampled parity probe."""
     import json
     env = dict(os.environ, PYTHONPATH=ROOT)
-    size = {"atax": ["--n", "2048"], "jacobi": ["--n", "1024", "--iters", "10"], "conv3": ["--n", "1024"],
-            "spmv": ["--n", "14"]}[cfg]
+    size = {"atax": ["--size", "2048"], "jacobi": ["--size", "1024", "--iters", "10"], "conv3": ["--size", "1024"],
+            "spmv": ["--size", "14"]}[cfg]
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr", "127.0.0.1", "--master-port", _port(), os.path.join(ROOT, "bench.py"),
            "--gpus", "2", "--steps", "3", "--warmup", "3", "--config", cfg, "--exchange", "torch",
