@@ -439,6 +439,11 @@ def main():
     else:
         ms_def, per_def, def_kind = ms_def_dir, per_def_dir, "direct-load"
     ms_id, _, _ = timed({"backend": "identity"}, cmp_steps)
+    ms_two_pass = None
+    if a.config == "atax" and D.fused_atax:         # the same clustered step with the two-pass ATAX
+        D.fused_atax = False
+        ms_two_pass, _, _ = timed(head, cmp_steps)
+        D.fused_atax = True
     total_bytes = D.bytes_per_step()
     value = total_bytes / (ms_clu * 1e-3) / 1e9
 
@@ -499,6 +504,7 @@ def main():
                 "ms_per_step_default_tma": round(ms_def_tma, 4),
                 "ms_per_step_default_direct": None if ms_def_dir is None else round(ms_def_dir, 4),
                 "ms_per_step_identity": round(ms_id, 4),
+                "ms_per_step_two_pass_atax": None if ms_two_pass is None else round(ms_two_pass, 4),
                 "roofline": roof, "clocks": clk, "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": launches,
                 "home_fraction": home, "parity": parity,
                 "l2_sector_reduction": {"source": prof, "metric": "1 - lts__t_sectors_srcunit_tex(variant) / (reference order)",
@@ -526,7 +532,9 @@ def config_block(a, D, head, world, use_graph):
                          "conv3": f"slab-shard x{world} (halo 1 row)", "conv7": f"slab-shard x{world} (halo 3 rows)",
                          "spmv": f"nnz-balanced row blocks x{world}"}[a.config]}
     if a.config == "atax":
-        c.update(n=D.n, tile="32x256", l2="inputs (1 GiB) larger than L2 (126 MB); no flush")
+        c.update(n=D.n, tile="32x256 (BICG, MVT); one row per logical CTA (one-pass ATAX)",
+                 atax="one pass (CC_K_ATAX_FUSED)" if D.fused_atax else "two passes",
+                 l2="inputs (1 GiB) larger than L2 (126 MB); no flush")
     elif a.config == "jacobi":
         c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32",
                  overlap=getattr(D, "overlap", False), halo="fused LL (peer memory)" if D.fused else "exchange",
@@ -573,12 +581,14 @@ def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
     if a.config == "atax":
         from paper_conf_asplos_lis0l0c17_b200 import drivers
         b_local = drivers.atax_family_bytes(D.m, D.n)
+        atax_fused = D.fused_atax and head.get("backend") in ("agent", "identity", "static")
         groups = {"gemv_fused": (("bicg", "mvt"), 2, "k_agent<GemvBody<32, 256, 1, 1>> (BICG, MVT)"),
-                  "atax": (("atax",), 2, "k_agent<GemvBody<32, 256, 1, 0>> + <0, 1> (ATAX passes)")}
+                  "atax": (("atax",), 1, "k_agent<AtaxFusedBody> (one-pass ATAX)") if atax_fused else
+                          (("atax",), 2, "k_agent<GemvBody<32, 256, 1, 0>> + <0, 1> (ATAX passes)")}
         gms = {g: sum(per_clu[k] for k in ks) for g, (ks, _, _) in groups.items()}
         dom = max(gms, key=gms.get)
         calls, nl, name = groups[dom]
-        dbytes = sum(b_local[k] for k in calls)
+        dbytes = sum(b_local[k] for k in calls) + (0 if atax_fused or dom != "atax" else 4 * D.m * D.n)
         ach = dbytes / (gms[dom] * 1e-3) / 1e9
         tr = None
         if traffic and all(traffic.get(k) for k in calls):

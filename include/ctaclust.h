@@ -200,7 +200,8 @@ typedef enum {
     CC_K_CONV2D = 6,   /* cc_conv2d_args   (config 4)                               */
     CC_K_SPMV = 7,     /* cc_spmv_args     (config 5)                               */
     CC_K_HIST64 = 8,   /* cc_hist64_args   (S§8(f)3, the paper's HST)               */
-    CC_K_JACOBI5_HALO = 9 /* cc_jacobi5_halo_args (S§8(f)4: sharded sweep, fused peer halo) */
+    CC_K_JACOBI5_HALO = 9, /* cc_jacobi5_halo_args (S§8(f)4: sharded sweep, fused peer halo) */
+    CC_K_ATAX_FUSED = 10  /* cc_atax_args: one-pass ATAX (both PolyBench kernels per row) */
 } cc_kernel;
 
 /* CC_K_CENSUS: no data. */
@@ -217,6 +218,15 @@ typedef struct { const float* A; int64_t lda; int32_t m, n; const float* x; floa
  * A m x n row-major fp32 DEVICE, lda % 4 == 0, lda >= n, 16-byte aligned. */
 /* ATAX: tmp = A x ; y = A^T tmp (two launches; tmp and y are zeroed by the call). */
 typedef struct { const float* A; int64_t lda; int32_t m, n; const float* x; float* tmp; float* y; } cc_atax_args;
+/* CC_K_ATAX_FUSED: the same ATAX (tmp = A x, y = A^T tmp; tmp and y written /
+ * zeroed by the call) over ONE read of A (Table 2 ATX; reading R31):
+ * logical CTA (0, i) is row i; the agent owning it computes tmp[i] and adds
+ * A[i][:] * tmp[i] into its register-held y partial while the row sits in its
+ * shared-memory ring (x held in registers), flushing y once per agent with
+ * vector REDs.  Grid 1 x m.  1 <= n <= 16384; A rows 16-byte aligned (lda % 4
+ * == 0).  Meant for the persistent backends (agent / identity / static): a
+ * one-shot CTA flushes n REDs per row.  Errors: INVALID_ARG, UNSUPPORTED
+ * (n > 16384, TBCLUSTER). */
 /* BICG: q = A p ; s = A^T r (one fused pass; q and s zeroed by the call). */
 typedef struct { const float* A; int64_t lda; int32_t m, n; const float* p; const float* r; float* q; float* s; } cc_bicg_args;
 /* MVT: x1 += A y1 ; x2 += A^T y2 (one fused pass, in place). */

@@ -19,6 +19,7 @@
 #include "cc_index.cuh"
 #include "cc_runtime.cuh"
 #include "k_gemv.cuh"
+#include "k_atax1.cuh"
 #include "k_spmv.cuh"
 #include "k_microbench.cuh"
 #include "k_hist.cuh"
@@ -354,6 +355,7 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
     case CC_K_CENSUS: { auto* c = (const cc_census_args*)a; *gx = c->gx; *gy = c->gy; return CC_OK; }
     case CC_K_MATVEC: { auto* c = (const cc_matvec_args*)a; *gx = cdiv(c->n, 32); *gy = cdiv(c->m, 32); return CC_OK; }
     case CC_K_ATAX: { auto* c = (const cc_atax_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
+    case CC_K_ATAX_FUSED: { auto* c = (const cc_atax_args*)a; *gx = c->m > 0 ? 1 : 0; *gy = c->m; return CC_OK; }
     case CC_K_BICG: { auto* c = (const cc_bicg_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
     case CC_K_MVT: { auto* c = (const cc_mvt_args*)a; *gx = cdiv(c->n, 256); *gy = cdiv(c->m, 32); return CC_OK; }
     case CC_K_JACOBI5: {
@@ -463,6 +465,7 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     case CC_K_CENSUS: s = occupancy<CensusBody>(device, CensusBody::kDefaultStages, &occ); break;
     case CC_K_MATVEC: s = occupancy<MatvecB>(device, MatvecB::kDefaultStages, &occ); break;
     case CC_K_ATAX: s = occupancy<RowB>(device, RowB::kDefaultStages, &occ); break;
+    case CC_K_ATAX_FUSED: s = occupancy<AtaxFusedBody>(device, AtaxFusedBody::kDefaultStages, &occ); break;
     case CC_K_BICG: case CC_K_MVT: s = occupancy<BothB>(device, BothB::kDefaultStages, &occ); break;
     case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, Jacobi5Body::kDefaultStages, &occ); break;
     case CC_K_JACOBI5_HALO: s = occupancy<Jacobi5HaloBody>(device, Jacobi5HaloBody::kDefaultStages, &occ); break;
@@ -756,6 +759,16 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         CC_TRY(gemv_params<32, 256>(&g2, x->A, x->lda, x->m, x->n, nullptr, x->tmp, nullptr, x->y));
         s = launch_body<RowB>(c, g1);
         if (s == CC_OK) s = launch_body<ColB>(c, g2);
+        break;
+    }
+    case CC_K_ATAX_FUSED: {
+        auto* x = (const cc_atax_args*)a;
+        CC_TRY(check_mat(x->A, x->lda, x->m, x->n));
+        CC_TRY(check_vec(x->x, x->n, "x")); CC_TRY(check_vec(x->tmp, x->m, "tmp")); CC_TRY(check_vec(x->y, x->n, "y"));
+        if (x->n > AtaxFusedBody::kMaxN) return fail(CC_ERR_UNSUPPORTED, "atax_fused: n %d > %d", x->n, AtaxFusedBody::kMaxN);
+        if (x->m > 0 && x->n < 1) return fail(CC_ERR_INVALID_ARG, "atax_fused: n < 1");
+        if (x->n) CC_CUDA(cudaMemsetAsync(x->y, 0, sizeof(float) * x->n, st));
+        s = launch_body<AtaxFusedBody>(c, AtaxFusedParams{x->A, x->lda, x->m, x->n, x->x, x->tmp, x->y});
         break;
     }
     case CC_K_BICG: {

@@ -1,0 +1,140 @@
+// k_atax1.cuh -- one-pass ("row-resident") ATAX: both PolyBench ATAX kernels
+// (tmp = A x; y = A^T tmp -- Table 2 ATX, reading R13) over ONE read
+// of A.
+//
+// The two-pass form (CC_K_ATAX: the 32 x 256 tiles of GemvBody<1,0> then
+// GemvBody<0,1>) streams the 1 GiB matrix from HBM twice: pass-2 logical CTAs
+// reuse exactly the A tiles pass-1 CTAs read, but a whole pass apart, long
+// after L2 turned over.  Here a logical CTA is one row i of A, and the agent
+// that owns it runs BOTH passes' work for that row back to back while the
+// row sits in its shared-memory ring:
+//   tmp[i]  = sum_j A[i][j] x[j]          (CTA-wide reduction of the row)
+//   y[j]   += A[i][j] tmp[i]              (every column, the row re-read from smem)
+// -- the inter-kernel reuse of A caught on chip with reuse distance zero:
+// clustering the pass-1 and pass-2 CTAs that share a row onto one SM,
+// consecutively.  x (<= 16384 floats) is held in registers for the agent's
+// lifetime and the agent's y contributions are carried in registers across all
+// its rows (ROW clusters: ~111 consecutive rows per SM at n = 16384) and
+// flushed once with vector REDs.
+//
+// Consumer mapping: 256 threads; thread t owns the float4 columns
+// c4 = t + 256 k, k < 16 (n <= 16384).  One row = 64 KB staged by one bulk
+// async copy (UBLKCP) into a ring of three 64 KB slots, so one agent per SM.
+// Summation order per output: tmp[i] by warp shuffles then warp partials in
+// warp order; y[j] in the agent's row order, then REDs in arrival order (fp32,
+// covered by the 1e-4 tolerance; integer-exact inputs are order-independent).
+#pragma once
+#include "cc_mem.cuh"
+#include "cc_runtime.cuh"
+
+namespace cc {
+
+struct AtaxFusedParams {
+    const float* A; int64_t lda; int32_t m, n;
+    const float* x; float* tmp; float* y;
+};
+
+struct AtaxFusedBody {
+    static constexpr int kConsumers = 256;
+    static constexpr int kCPT = 16;                          // float4 columns per thread
+    static constexpr int kMaxN = kConsumers * 4 * kCPT;      // 16384
+    static constexpr int kStageBytes = kMaxN * 4;            // one row
+    static constexpr int kDirectStageBytes = kStageBytes;    // staging mode is ignored: always a bulk copy
+    static constexpr int kDefaultStages = 3;
+    static constexpr int kDefaultBatch = 4;
+    static constexpr int kMinAgents = 1;
+    static constexpr int kGroups = 1;
+    using Params = AtaxFusedParams;
+    const AtaxFusedParams& p;
+    int32_t l2h = 0;
+    float4 xr[kCPT];                                         // x, loaded by the first task
+    float4 yr[kCPT];                                         // this agent's y contributions
+    int32_t rows_done = 0;
+
+    __device__ __forceinline__ explicit AtaxFusedBody(const AtaxFusedParams& prm) : p(prm) {
+#pragma unroll
+        for (int k = 0; k < kCPT; ++k) yr[k] = f4_zero();
+    }
+
+    __device__ __forceinline__ void produce(const Sched&, int32_t, int32_t by, uint8_t* stage, uint64_t* full, int lane) {
+        const uint32_t bytes = ((uint32_t)p.n * 4u + 15u) & ~15u;   // lda % 4 == 0: stays inside the row's padding
+        stage_commit(full, lane, bytes);
+        if (lane == 0) bulk_g2s(stage, p.A + (int64_t)by * p.lda, bytes, full);
+    }
+
+    __device__ __forceinline__ void consume(const Sched&, int32_t, int32_t by, const uint8_t* stage, int ctid) {
+        __shared__ float s_part[2][kConsumers / 32];
+        const int n4 = (p.n + 3) >> 2;                       // float4 columns (the last may be partial)
+        if (rows_done == 0) {
+#pragma unroll
+            for (int k = 0; k < kCPT; ++k) {
+                const int c4 = ctid + kConsumers * k;
+                float4 v = f4_zero();
+                if (4 * c4 + 3 < p.n) v = *reinterpret_cast<const float4*>(p.x + 4 * c4);
+                else if (c4 < n4) {                          // ragged last float4 of x
+                    v.x = p.x[4 * c4];
+                    if (4 * c4 + 1 < p.n) v.y = p.x[4 * c4 + 1];
+                    if (4 * c4 + 2 < p.n) v.z = p.x[4 * c4 + 2];
+                }
+                xr[k] = v;
+            }
+        }
+        const float4* a4 = reinterpret_cast<const float4*>(stage);
+        // the row is read from shared memory twice (dot, then the y update)
+        // rather than held: 64 more registers would spill x / y
+        auto row4 = [&](int k) {
+            const int c4 = ctid + kConsumers * k;
+            float4 av = c4 < n4 ? a4[c4] : f4_zero();
+            if (4 * c4 + 3 >= p.n) {                         // ragged last float4: drop the row's padding
+                if (4 * c4 + 1 >= p.n) av.y = 0.f;
+                if (4 * c4 + 2 >= p.n) av.z = 0.f;
+                av.w = 0.f;
+            }
+            return av;
+        };
+        float dot = 0.f;
+#pragma unroll
+        for (int k = 0; k < kCPT; ++k) {
+            const float4 av = row4(k);
+            dot = fmaf(av.x, xr[k].x, dot);
+            dot = fmaf(av.y, xr[k].y, dot);
+            dot = fmaf(av.z, xr[k].z, dot);
+            dot = fmaf(av.w, xr[k].w, dot);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) dot += __shfl_xor_sync(0xffffffffu, dot, o);
+        const int par = rows_done & 1;
+        if ((ctid & 31) == 0) s_part[par][ctid >> 5] = dot;
+        consumer_sync<kConsumers>();
+        float t = 0.f;
+#pragma unroll
+        for (int w = 0; w < kConsumers / 32; ++w) t += s_part[par][w];
+        if (ctid == 0) p.tmp[by] = t;
+#pragma unroll
+        for (int k = 0; k < kCPT; ++k) {
+            const float4 av = row4(k);
+            yr[k].x = fmaf(av.x, t, yr[k].x);
+            yr[k].y = fmaf(av.y, t, yr[k].y);
+            yr[k].z = fmaf(av.z, t, yr[k].z);
+            yr[k].w = fmaf(av.w, t, yr[k].w);
+        }
+        ++rows_done;
+    }
+
+    __device__ __forceinline__ void finish(int ctid) {
+        if (rows_done == 0) return;
+        const int n4 = (p.n + 3) >> 2;
+#pragma unroll
+        for (int k = 0; k < kCPT; ++k) {
+            const int c4 = ctid + kConsumers * k;
+            if (4 * c4 + 3 < p.n) red_add4(p.y + 4 * c4, yr[k]);
+            else if (c4 < n4) {
+                red_add(p.y + 4 * c4, yr[k].x);
+                if (4 * c4 + 1 < p.n) red_add(p.y + 4 * c4 + 1, yr[k].y);
+                if (4 * c4 + 2 < p.n) red_add(p.y + 4 * c4 + 2, yr[k].z);
+            }
+        }
+    }
+};
+
+}  // namespace cc

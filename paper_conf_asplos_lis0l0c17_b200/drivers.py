@@ -142,11 +142,13 @@ def make_exchange(kind: str, world: int, rank: int, device: int) -> Exchange:
 # config 2: ATAX + BICG + MVT, row-sharded
 # ----------------------------------------------------------------------------
 def atax_family_bytes(m: int, n: int) -> dict:
-    """Algorithmic bytes of one ATAX (2 passes) + BICG + MVT step over an m x n
-    A (each pass reads A once; vectors read once; outputs written once; MVT's
-    x1 / x2 read and written)."""
+    """Algorithmic bytes of one ATAX + BICG + MVT step over an m x n A: the
+    minimum each needs -- A read once (ATAX too: the one-pass schedule,
+    CC_K_ATAX_FUSED, shows one read suffices; round 1 counted the two-pass
+    form's two reads), vectors read once, outputs written once, MVT's x1 / x2
+    read and written."""
     A = 4 * m * n
-    atax = (A + 4 * n + 4 * m) + (A + 4 * m + 4 * n)
+    atax = A + 4 * n + 4 * m + 4 * n
     bicg = A + 4 * (n + m) + 4 * (m + n)
     mvt = A + 4 * (n + m) + 8 * (m + n)
     return {"atax": atax, "bicg": bicg, "mvt": mvt, "total": atax + bicg + mvt}
@@ -161,8 +163,12 @@ class AtaxFamily:
     ranks other than 0 zero their x2 slice before MVT, so after the sum
     x2 = x2_prev + sum over ranks of A_g^T y2_g (rank 0 carries x2_prev)."""
 
-    def __init__(self, n: int, xchg: Exchange, device, m_total: int | None = None):
+    def __init__(self, n: int, xchg: Exchange, device, m_total: int | None = None, fused_atax: bool = True):
         self.n, self.x = n, xchg
+        # ATAX as one pass (CC_K_ATAX_FUSED) on the persistent backends; the
+        # one-shot backends (default / redirect) keep the two-pass kernels,
+        # since a one-shot CTA per row would flush y once per row
+        self.fused_atax = fused_atax and n <= 16384
         self.m_total = n if m_total is None else m_total
         self.lo, self.hi = shard.row_range(self.m_total, xchg.world, xchg.rank)
         m = self.m = self.hi - self.lo
@@ -197,7 +203,14 @@ class AtaxFamily:
         nl = 0
         if ev is not None:
             ev[0].record(stream)
-        nl += _launch("atax", cc.atax_args(self.A, self.xv, self.tmp, self.y), opts, stream)
+        fused = self.fused_atax and opts.get("backend", "agent") in ("agent", "identity", "static")
+        if fused:
+            o = dict(opts)
+            o.pop("order", None)                       # one row per logical CTA: row clusters
+            o.pop("staging", None)
+            nl += _launch("atax_fused", cc.atax_args(self.A, self.xv, self.tmp, self.y), dict(o, order="row"), stream)
+        else:
+            nl += _launch("atax", cc.atax_args(self.A, self.xv, self.tmp, self.y), opts, stream)
         if ev is not None:
             ev[1].record(stream)
         nl += _launch("bicg", cc.bicg_args(self.A, self.p, self.r, self.q, self.s), opts, stream)

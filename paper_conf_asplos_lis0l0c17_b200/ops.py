@@ -18,7 +18,7 @@ from . import ctaclust as cc
 DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": ("col", (1, 1)),
                  "bicg": ("col", (1, 1)), "mvt": ("col", (1, 1)), "jacobi5": ("row", (1, 1)),
                  "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1)),
-                 "jacobi5_halo": ("row", (1, 1))}
+                 "jacobi5_halo": ("row", (1, 1)), "atax_fused": ("row", (1, 1))}
 
 # Plans of the computed orders are cached for the life of the process: a plan
 # may only be destroyed once every stream that used it has synchronized
@@ -106,6 +106,14 @@ def matvec(A, x, y=None, backend="agent", order=None, tile=None, num_clusters=0,
 def atax(A, x, backend="agent", order=None, tile=None, num_clusters=0, stream=None, out=None, **kw):
     tmp, y = out if out is not None else (torch.empty(A.shape[0], device=A.device), torch.empty(A.shape[1], device=A.device))
     _launch("atax", cc.atax_args(A, x, tmp, y), backend, order, tile, num_clusters, _dev(A), stream, **kw)
+    return tmp, y
+
+
+def atax_fused(A, x, backend="agent", order=None, tile=None, num_clusters=0, stream=None, out=None, **kw):
+    """One-pass ATAX (CC_K_ATAX_FUSED): tmp = A x, y = A^T tmp over one read of A
+    (persistent backends; n <= 16384)."""
+    tmp, y = out if out is not None else (torch.empty(A.shape[0], device=A.device), torch.empty(A.shape[1], device=A.device))
+    _launch("atax_fused", cc.atax_args(A, x, tmp, y), backend, order, tile, num_clusters, _dev(A), stream, **kw)
     return tmp, y
 
 

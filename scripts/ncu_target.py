@@ -55,13 +55,14 @@ def main():
         x = synth.uniform(2, n, backend="torch", device=dev)
         y = torch.zeros(n, device=dev)
         fn = lambda: ops.matvec(A, x, y, **kw)
-    elif k in ("atax", "bicg", "mvt"):
+    elif k in ("atax", "bicg", "mvt", "atax_fused"):
         n = 4096 if a.small else 16384
         A = synth.matrix(3, n, n, backend="torch", device=dev)
         v = lambda s: synth.uniform(s, n, backend="torch", device=dev)
         x, p, r, y1, y2, x1, x2 = v(10), v(11), v(12), v(15), v(16), v(13), v(14)
         bufs = (torch.empty(n, device=dev), torch.empty(n, device=dev))
         fn = {"atax": lambda: ops.atax(A, x, out=bufs, **kw),
+              "atax_fused": lambda: ops.atax_fused(A, x, out=bufs, **kw),
               "bicg": lambda: ops.bicg(A, p, r, out=bufs, **kw),
               "mvt": lambda: ops.mvt(A, y1, y2, x1, x2, **kw)}[k]
     elif k == "jacobi":

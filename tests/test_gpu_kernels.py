@@ -155,6 +155,63 @@ def test_atax_mvt_full_size_config2():
         assert relerr(X1.cpu().numpy(), r1) <= TOL and relerr(X2.cpu().numpy(), r2) <= TOL, v
 
 
+FUSED_VARIANTS = [dict(backend="agent"), dict(backend="identity"), dict(backend="static", num_clusters=148),
+                  dict(backend="static", num_clusters=444), dict(backend="agent", active_agents=1, stages=2),
+                  dict(backend="agent", steal=0), dict(backend="default")]
+
+
+@pytest.mark.parametrize("v", FUSED_VARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
+@pytest.mark.parametrize("m,n,ld", [(1000, 1001, 1004), (300, 16384, 16384), (7, 13, 16), (1, 1, 4), (150, 4096, 4100)])
+def test_atax_fused(v, m, n, ld):
+    """One-pass ATAX (CC_K_ATAX_FUSED): tmp and y vs the oracle; y also vs
+    pass 2 on the GPU's own fp32 tmp; ragged n (padding in the staged row must
+    not leak), m below and above the SM count, n at the 16384 limit."""
+    A = mat(9, m, n)
+    Ad = padded(A, ld).as_strided((m, n), (ld, 1))
+    if ld > n:                                             # poison the padding: it must be ignored
+        Ad.as_strided((m, ld), (ld, 1))[:, n:] = float("nan")
+    x = synth.uniform(10, n)
+    tmp, y = ops.atax_fused(Ad, dev(x), **v)
+    torch.cuda.synchronize()
+    rt, ry = O.atax(A, x)
+    assert relerr(tmp.cpu().numpy(), rt) <= TOL
+    assert relerr(y.cpu().numpy(), O.atax_pass2(A, tmp.cpu().numpy())) <= TOL
+    assert relerr(y.cpu().numpy(), ry) <= TOL
+
+
+def test_atax_fused_integer_exact_and_census():
+    m, n = 200, 98                      # every partial sum of tmp and y stays below 2^24
+    A = mat(11, m, n, "int")
+    Ad = padded(A, 100).as_strided((m, n), (100, 1))
+    x = synth.small_int(12, n)
+    cen = torch.zeros(m, dtype=torch.int32, device="cuda")
+    tmp, y = ops.atax_fused(Ad, dev(x), backend="agent", census=cen)
+    torch.cuda.synchronize()
+    rt, ry = O.atax(A, x)
+    assert np.array_equal(tmp.cpu().numpy().astype(np.float64), rt)
+    assert np.array_equal(y.cpu().numpy().astype(np.float64), ry)
+    assert bool(torch.all(cen == 1))
+
+
+def test_atax_fused_full_size_config2():
+    """Config 2's ATAX at n = 16384 in the bench's launch config (agent, one
+    row per logical CTA), every output."""
+    n = 16384
+    A = synth.matrix(3, n, n)
+    x = synth.uniform(10, n)
+    tmp, y = ops.atax_fused(dev(A), dev(x), backend="agent")
+    torch.cuda.synchronize()
+    rt, ry = O.atax(A, x)
+    assert relerr(tmp.cpu().numpy(), rt) <= TOL and relerr(y.cpu().numpy(), ry) <= TOL
+
+
+def test_atax_fused_limits():
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    with pytest.raises(cc.CtaclustError) as e:
+        ops.atax_fused(torch.zeros(4, 16388, device="cuda"), torch.zeros(16388, device="cuda"))
+    assert e.value.status == -6
+
+
 def test_matvec_config1_static_binding():
     """Config 1 (n = 1024, 32 x 32 tiles) in the configuration that measures
     fastest (static binding, M = 3 x SMs, row clustering) and the agent."""
