@@ -17,8 +17,8 @@
 // its rows (ROW clusters: ~111 consecutive rows per SM at n = 16384) and
 // flushed once with vector REDs.
 //
-// Consumer mapping: 256 threads; thread t owns the float4 columns
-// c4 = t + 256 k, k < 16 (n <= 16384).  One row = 64 KB staged by one bulk
+// Consumer mapping: 512 threads; thread t owns the float4 columns
+// c4 = t + 512 k, k < 8 (n <= 16384).  One row = 64 KB staged by one bulk
 // async copy (UBLKCP) into a ring of three 64 KB slots, so one agent per SM.
 // Summation order per output: tmp[i] by warp shuffles then warp partials in
 // warp order; y[j] in the agent's row order, then REDs in arrival order (fp32,
@@ -35,8 +35,11 @@ struct AtaxFusedParams {
 };
 
 struct AtaxFusedBody {
-    static constexpr int kConsumers = 256;
-    static constexpr int kCPT = 16;                          // float4 columns per thread
+    // 16 consumer warps: a row's dot product and its y update are latency
+    // chains through shared memory, so more warps per row (not more rows in
+    // flight -- the ring already holds three) is what keeps HBM busy
+    static constexpr int kConsumers = 512;
+    static constexpr int kCPT = 8;                           // float4 columns per thread
     static constexpr int kMaxN = kConsumers * 4 * kCPT;      // 16384
     static constexpr int kStageBytes = kMaxN * 4;            // one row
     static constexpr int kDirectStageBytes = kStageBytes;    // staging mode is ignored: always a bulk copy
