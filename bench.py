@@ -577,7 +577,7 @@ def l2_reductions(cfg, head):
 def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
     peak_hbm = pk["hbm_gbs"] if pk else 6650.0
     src = "MEASURED_PEAKS.json hbm_gbs (copy)" if pk else "fallback 6.65 TB/s"
-    traffic = traffic_from_profiles(a.config, head)
+    traffic = traffic_from_profiles(a.config, head, a.hot)
     if a.config == "atax":
         from paper_conf_asplos_lis0l0c17_b200 import drivers
         b_local = drivers.atax_family_bytes(D.m, D.n)
@@ -626,7 +626,7 @@ def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
                       + (" (whole-job bytes, includes the exchange at N > 1)" if D.x.world > 1 else "")}
 
 
-def traffic_from_profiles(cfg, head):
+def traffic_from_profiles(cfg, head, hot=0):
     """ncu dram bytes per launch of the headline variant from the newest
     committed summary (cold-cache, one launch)."""
     import glob
@@ -645,6 +645,8 @@ def traffic_from_profiles(cfg, head):
     for k in ("atax", "bicg", "mvt", "jacobi", "conv3", "conv7", "spmv"):
         if f"{k}_{suf}" in d:
             out[k] = d[f"{k}_{suf}"]
+    if cfg == "spmv" and hot and f"spmv_{suf}-hot" in d:        # the hub-column form's capture
+        out["spmv"] = d[f"spmv_{suf}-hot"]
     return out
 
 

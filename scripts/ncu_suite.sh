@@ -29,6 +29,9 @@ for k in atax bicg mvt; do
   run ${k}_identity $per --kernel $k --backend identity
   run ${k}_static-col-m3 $per --kernel $k --backend static --order col --clusters 444
 done
+run atax_fused_agent-row 1 --kernel atax_fused --backend agent --order row
+run atax_fused_identity 1 --kernel atax_fused --backend identity
+run atax_fused_static-row-m1 1 --kernel atax_fused --backend static --order row --clusters 148
 for k in jacobi conv3 conv7; do
   run ${k}_default 1 --kernel $k --backend default
   run ${k}_default-l1 1 --kernel $k --backend default --staging l1
