@@ -244,7 +244,13 @@ typedef struct { const float* A; int64_t lda; int32_t m, n; const float* y1; con
  * = 0: all rows.  Logical CTA = 32 x 32 output tile of the window; grid
  * ceil(cols/32) x ceil((row_hi - row_lo)/32) (ceil(rows/32) without a window). */
 typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t iters; int32_t* result_is_b;
-                 int32_t row_lo, row_hi; } cc_jacobi5_args;
+                 int32_t row_lo, row_hi;
+                 int32_t fuse;   /* sweeps per launch (reading R32): 0 or 1 = one; 2, 3 or 4 = that many
+                                    consecutive sweeps per launch (each tile staged once with a fuse-row
+                                    halo, the intermediate sweeps recomputed on chip), bit-identical to
+                                    single sweeps; iters % fuse remaining sweeps run one per launch.
+                                    Not with a row window (UNSUPPORTED). */
+               } cc_jacobi5_args;
 
 /* CC_K_JACOBI5_HALO -- S§8(f)4: one rank's slab of the slab-sharded Jacobi
  * (S§8(e), config 3) with the per-sweep halo exchange fused into the sweep

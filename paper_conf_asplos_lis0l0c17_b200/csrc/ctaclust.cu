@@ -798,9 +798,28 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         CC_TRY(check_mat(x->a, x->ld, x->rows, x->cols));
         CC_TRY(check_mat(x->b, x->ld, x->rows, x->cols));
         if (x->iters < 0) return fail(CC_ERR_INVALID_ARG, "iters < 0");
+        const int fuse = x->fuse <= 1 ? 1 : x->fuse;
+        if (fuse > 4) return fail(CC_ERR_INVALID_ARG, "jacobi5: fuse %d outside [0, 4]", x->fuse);
+        if (fuse > 1 && (x->row_lo != 0 || x->row_hi != 0))
+            return fail(CC_ERR_UNSUPPORTED, "jacobi5: fused sweeps with a row window");
         float* src = x->a;
         float* dst = x->b;
-        for (int it = 0; it < x->iters && s == CC_OK; ++it) {
+        int launches_done = 0;
+        // fused launches first (each runs `fuse` sweeps), then single sweeps
+        for (int it = 0; fuse > 1 && it + fuse <= x->iters && s == CC_OK; it += fuse) {
+            JacobiParams jp;
+            memset(&jp, 0, sizeof jp);
+            jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
+            jp.row0 = 0; jp.row_end = x->rows;
+            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 32 + 2 * fuse));
+            s = fuse == 2 ? launch_body<Jacobi5MultiBody<2>>(c, jp)
+              : fuse == 3 ? launch_body<Jacobi5MultiBody<3>>(c, jp)
+                          : launch_body<Jacobi5MultiBody<4>>(c, jp);
+            std::swap(src, dst);
+            ++launches_done;
+        }
+        const int single = fuse > 1 ? x->iters % fuse : x->iters;
+        for (int it = 0; it < single && s == CC_OK; ++it) {
             JacobiParams jp;
             memset(&jp, 0, sizeof jp);
             jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
@@ -814,8 +833,9 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             }
             s = launch_body<Jacobi5Body>(c, jp);
             std::swap(src, dst);
+            ++launches_done;
         }
-        if (x->result_is_b) *x->result_is_b = (x->iters & 1) ? 1 : 0;
+        if (x->result_is_b) *x->result_is_b = (launches_done & 1) ? 1 : 0;
         break;
     }
     case CC_K_JACOBI5_HALO: {

@@ -130,10 +130,11 @@ def mvt(A, y1, y2, x1, x2, backend="agent", order=None, tile=None, num_clusters=
 
 
 def jacobi5(a, b, iters, backend="agent", order=None, tile=None, num_clusters=0, stream=None, row_window=None,
-            **kw):
+            fuse=1, **kw):
     """`iters` sweeps ping-ponging a <-> b; returns the buffer holding the result.
-    `row_window` = (lo, hi) writes only output rows [lo, hi) of each sweep."""
-    args, flag = cc.jacobi5_args(a, b, iters, row_window=row_window)
+    `row_window` = (lo, hi) writes only output rows [lo, hi) of each sweep;
+    `fuse` = sweeps per launch (1-4, bit-identical)."""
+    args, flag = cc.jacobi5_args(a, b, iters, row_window=row_window, fuse=fuse)
     _launch("jacobi5", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
     return b if flag.value else a
 

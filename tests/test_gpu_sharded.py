@@ -240,3 +240,34 @@ def test_bench_two_ranks_one_gpu(cfg):
     assert out.returncode == 0 and len(lines) == 1, (out.stdout[-3000:], out.stderr[-3000:])
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["parity"]["ok"], d["parity"]
+
+
+# ---------------------------------------------------------------- fused sweeps (R32)
+@pytest.mark.parametrize("fuse", [2, 3, 4])
+@pytest.mark.parametrize("v", [dict(backend="agent", order="row"), dict(backend="default"), dict(backend="identity"),
+                               dict(backend="static", order="row", num_clusters=148),
+                               dict(backend="agent", order="tile", tile=(2, 2))], ids=lambda v: v["backend"])
+@pytest.mark.parametrize("rows,cols,T", [(130, 100, 8), (77, 45, 7), (5, 9, 5), (300, 260, 12)])
+def test_jacobi_fused_sweeps_bit_exact(fuse, v, rows, cols, T):
+    """K sweeps per launch (halo recomputed on chip) equal T single sweeps bit
+    for bit, T not a multiple of K included, images smaller than one staged box."""
+    u0 = synth.matrix(4, rows, cols)
+    a = padded(u0)
+    b = padded(np.zeros_like(u0))
+    out = ops.jacobi5(a, b, T, fuse=fuse, **v)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), O.jacobi5_f32(u0, T))
+
+
+def test_jacobi_fused_full_width_sampled():
+    """16384 columns (config 3's width), 4 sweeps per launch, 12 sweeps:
+    sampled rows and the rows at tile seams, bit-exact."""
+    rows, cols, T = 520, 16384, 12
+    u0 = synth.matrix(4, rows, cols)
+    a = padded(u0)
+    out = ops.jacobi5(a, torch.empty_like(a), T, fuse=4, backend="agent", order="row")
+    torch.cuda.synchronize()
+    ref = O.jacobi5_f32(u0, T)
+    got = out.cpu().numpy()
+    assert np.array_equal(got[::7], ref[::7])
+    assert np.array_equal(got[30:35], ref[30:35]) and np.array_equal(got[255:259], ref[255:259])
