@@ -75,6 +75,7 @@ def parse():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
+    ap.add_argument("--fuse", type=int, default=4, help="jacobi (one GPU): sweeps per launch, 1-4 (R32)")
     ap.add_argument("--halo", default="exchange", choices=["exchange", "fused"],
                     help="jacobi N > 1: NCCL halo exchange per sweep, or the fused peer-memory LL halo")
     ap.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
@@ -340,7 +341,7 @@ def build_driver(a, X, dev):
         return drivers.AtaxFamily(sz["n"], X, dev)
     if a.config == "jacobi":
         return drivers.JacobiSlab(sz["side"], sz["side"], sz["iters"], X, dev, overlap=not a.no_overlap,
-                                  halo=a.halo)
+                                  halo=a.halo, fuse=a.fuse)
     if a.config in ("conv3", "conv7"):
         return drivers.ConvSlab(sz["side"], sz["side"], sz["R"], X, dev)
     return drivers.SpmvBlock(sz["scale"], X, dev, hot=a.hot)
@@ -509,6 +510,8 @@ def main():
                 "home_fraction": home, "parity": parity,
                 "l2_sector_reduction": {"source": prof, "metric": "1 - lts__t_sectors_srcunit_tex(variant) / (reference order)",
                                         **l2red}}
+        if a.config == "jacobi":
+            line["sweeps_per_second"] = round(D.iters / (ms_clu * 1e-3), 1)
         if per_clu:
             line["per_kernel_ms"] = {k: round(v, 4) for k, v in per_clu.items()}
             line["per_kernel_ms_default"] = {k: round(v, 4) for k, v in per_def.items()}
@@ -536,7 +539,8 @@ def config_block(a, D, head, world, use_graph):
                  atax="one pass (CC_K_ATAX_FUSED)" if D.fused_atax else "two passes",
                  l2="inputs (1 GiB) larger than L2 (126 MB); no flush")
     elif a.config == "jacobi":
-        c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32",
+        c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32", sweeps_per_launch=D.fuse,
+                 bytes="one read + one write of the field per launch (per sweep when unfused)",
                  overlap=getattr(D, "overlap", False), halo="fused LL (peer memory)" if D.fused else "exchange",
                  l2="2 x 1 GiB ping-pong buffers, larger than L2; no flush")
     elif a.config in ("conv3", "conv7"):
@@ -601,7 +605,8 @@ def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
     # single-kernel configs: every launch in the step is the headline kernel
     nl = max(1, launches // a.steps)
     ms_launch = ms_clu / nl
-    body = {"jacobi": "Jacobi5BodyT<false>", "conv3": "Conv2dBody<1>", "conv7": "Conv2dBody<3>",
+    body = {"jacobi": f"Jacobi5MultiBody<{D.fuse}>" if a.config == "jacobi" and D.fuse > 1 else "Jacobi5BodyT<false>",
+            "conv3": "Conv2dBody<1>", "conv7": "Conv2dBody<3>",
             "spmv": "SpmvBody"}[a.config]
     kern = {"agent": "k_agent", "static": "k_static", "default": "k_default", "identity": "k_agent"}.get(
         head.get("backend"), "k_agent") + f"<{body}>"
@@ -664,7 +669,7 @@ def home_fraction(a, D, head, device):
             args = cc.bicg_args(D.A, D.p, D.r, D.q, D.s)
             kern = "bicg"
         elif a.config == "jacobi":
-            args = cc.jacobi5_args(D.a, D.b, 1)[0]
+            args = cc.jacobi5_args(D.a, D.b, D.fuse, fuse=D.fuse)[0]       # one launch of the headline kernel
             kern = "jacobi5"
         elif a.config in ("conv3", "conv7"):
             args, D._w = cc.conv2d_args(D.inp, D.out, D.w)

@@ -270,8 +270,11 @@ class JacobiSlab:
     eagerly (a replayed graph would repeat the tags)."""
 
     def __init__(self, rows: int, cols: int, iters: int, xchg: Exchange, device, overlap: bool = True,
-                 halo: str = "exchange"):
+                 halo: str = "exchange", fuse: int = 1):
         self.rows, self.cols, self.iters, self.x = rows, cols, iters, xchg
+        # K sweeps per launch (R32) on the unsharded field; a sharded slab would
+        # need a K-row halo per K sweeps (not built: world > 1 runs single sweeps)
+        self.fuse = fuse if xchg.world == 1 else 1
         self.lo, self.hi, self.llo, self.lhi = shard.slab_range(rows, xchg.world, xchg.rank, 1)
         L = self.lhi - self.llo
         dev = self.dev = torch.device(device)
@@ -343,6 +346,12 @@ class JacobiSlab:
         if self.graph is not None:
             self.graph.replay()
             return self.graph_launches
+        if self.fuse > 1:
+            args, flag = cc.jacobi5_args(self.a, self.b, self.iters, fuse=self.fuse)
+            nl = _launch("jacobi5", args, opts, stream)
+            if flag.value:
+                self.a, self.b = self.b, self.a
+            return nl
         nl = 0
         for k in range(self.iters):
             src, dst = (self.a, self.b) if k % 2 == 0 else (self.b, self.a)
@@ -351,12 +360,17 @@ class JacobiSlab:
             self.a, self.b = self.b, self.a
         return nl
 
+    def launches_per_step(self) -> int:
+        if self.fuse > 1:
+            return self.iters // self.fuse + self.iters % self.fuse
+        return self.iters
+
     def capture(self, opts: dict) -> bool:
         """Capture one step (all `iters` sweeps, both streams) into a CUDA graph;
         later steps replay it.  Plans and tensor maps are created by an eager
         step first (no allocation is legal during capture).  Returns False when
         the exchange cannot be captured."""
-        if not self.x.capturable or self.iters % 2 or self.fused:
+        if not self.x.capturable or self.launches_per_step() % 2 or self.fused:
             return False
         self.step(opts)
         torch.cuda.synchronize()
@@ -375,7 +389,9 @@ class JacobiSlab:
         return self.a[self.own[0]: self.own[1]]
 
     def bytes_per_step(self) -> int:
-        return 8 * self.rows * self.cols * self.iters
+        """one read and one write of the field per launch: per sweep unfused,
+        per K sweeps with K fused sweeps per launch (R32)"""
+        return 8 * self.rows * self.cols * self.launches_per_step()
 
 
 class GraphStep:
