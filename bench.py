@@ -397,11 +397,13 @@ def main():
             return t.item()
         return v
 
+    captured = [False]
+
     def timed(opts, steps, per_kernel=False):
         """(ms per step, per-kernel ms or None, launches in the timed region)"""
         if use_graph:
             D.graph = None
-            D.capture(opts)
+            captured[0] = bool(D.capture(opts))
         for _ in range(max(3, a.warmup)):
             D.step(opts)
         evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(steps)] \
@@ -429,6 +431,7 @@ def main():
     clocks = Clocks(local)
     ms_clu, per_clu, launches = timed(head, a.steps, per_kernel=True)
     clk = clocks.stop()
+    head_captured = captured[0]
     cmp_steps = max(3, a.steps // 2)
     dflt = {"backend": "default"}
     ms_def_tma, per_def_tma, _ = timed(dict(dflt, staging="tma"), cmp_steps, per_kernel=True)
@@ -498,7 +501,7 @@ def main():
                 "warmup": max(3, a.warmup), "ms_per_step": round(ms_clu, 4), "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "f32",
                 "data": "synthetic (counter-hash generators, generated on device)",
-                "config": config_block(a, D, head, world, use_graph),
+                "config": config_block(a, D, head, world, use_graph and head_captured),
                 "speedup_vs_default": round(ms_def / ms_clu, 4),
                 "speedup_vs_identity": round(ms_id / ms_clu, 4),
                 "ms_per_step_default": round(ms_def, 4), "default_kind": def_kind,

@@ -272,10 +272,13 @@ class JacobiSlab:
     def __init__(self, rows: int, cols: int, iters: int, xchg: Exchange, device, overlap: bool = True,
                  halo: str = "exchange", fuse: int = 1):
         self.rows, self.cols, self.iters, self.x = rows, cols, iters, xchg
-        # K sweeps per launch (R32) on the unsharded field; a sharded slab would
-        # need a K-row halo per K sweeps (not built: world > 1 runs single sweeps)
-        self.fuse = fuse if xchg.world == 1 else 1
-        self.lo, self.hi, self.llo, self.lhi = shard.slab_range(rows, xchg.world, xchg.rank, 1)
+        # K sweeps per launch (R32).  Sharded, the slab keeps K halo rows per
+        # side and exchanges them once per K sweeps: a slab edge acts as a fixed
+        # boundary inside the launch, so after K sweeps the error it causes has
+        # reached halo row K-1 at most and every owned row is exact.
+        self.fuse = fuse if halo != "fused" else 1
+        self.hw = self.fuse if xchg.world > 1 else 1               # halo rows per side
+        self.lo, self.hi, self.llo, self.lhi = shard.slab_range(rows, xchg.world, xchg.rank, self.hw)
         L = self.lhi - self.llo
         dev = self.dev = torch.device(device)
         ld = (cols + 3) & ~3
@@ -284,7 +287,7 @@ class JacobiSlab:
         self.b = torch.zeros(L, ld, device=dev)[:, :cols]
         own0, own1 = self.lo - self.llo, self.hi - self.llo
         self.own = (own0, own1)
-        self.overlap = overlap and xchg.world > 1 and own1 - own0 > 64
+        self.overlap = overlap and xchg.world > 1 and own1 - own0 > 64 and self.fuse == 1
         if self.overlap:
             self.windows_b, self.window_i = sweep_windows(own0, own1)
         self.comm_stream = torch.cuda.Stream(device=dev) if xchg.world > 1 else None
@@ -346,11 +349,22 @@ class JacobiSlab:
         if self.graph is not None:
             self.graph.replay()
             return self.graph_launches
-        if self.fuse > 1:
+        if self.fuse > 1 and self.x.world == 1:
             args, flag = cc.jacobi5_args(self.a, self.b, self.iters, fuse=self.fuse)
             nl = _launch("jacobi5", args, opts, stream)
             if flag.value:
                 self.a, self.b = self.b, self.a
+            return nl
+        if self.fuse > 1:                                 # sharded: K sweeps, then the K-row halo exchange
+            nl, done = 0, 0
+            while done < self.iters:
+                k = min(self.fuse, self.iters - done)
+                args, flag = cc.jacobi5_args(self.a, self.b, k, fuse=k if k > 1 else 1)
+                nl += _launch("jacobi5", args, opts, stream)
+                if flag.value:
+                    self.a, self.b = self.b, self.a
+                self.x.halo_exchange(self.a, self.hw, stream)
+                done += k
             return nl
         nl = 0
         for k in range(self.iters):
@@ -361,8 +375,10 @@ class JacobiSlab:
         return nl
 
     def launches_per_step(self) -> int:
-        if self.fuse > 1:
+        if self.fuse > 1 and self.x.world == 1:
             return self.iters // self.fuse + self.iters % self.fuse
+        if self.fuse > 1:
+            return -(-self.iters // self.fuse)
         return self.iters
 
     def capture(self, opts: dict) -> bool:

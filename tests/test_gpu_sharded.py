@@ -149,7 +149,8 @@ WORKER = textwrap.dedent("""
     elif cfg.startswith("jacobi"):
         rows, cols, T = 330, 200, 6
         d = drivers.JacobiSlab(rows, cols, T, X, "cuda", overlap=cfg == "jacobi",
-                               halo="fused" if cfg == "jacobi-fused" else "exchange")
+                               halo="fused" if cfg == "jacobi-fused" else "exchange",
+                               fuse=int(cfg[-1]) if cfg.startswith("jacobi-k") else 1)
         ref = O.jacobi5_f32(synth.matrix(4, rows, cols), T)
         ref2 = O.jacobi5_f32(synth.matrix(4, rows, cols), 2 * T)
         d.step(dict(backend="agent", order="row", max_agents=1))
@@ -202,7 +203,8 @@ def _port():
 
 
 @pytest.mark.parametrize("cfg,world", [("atax", 2), ("atax", 4), ("jacobi", 2), ("jacobi", 3), ("jacobi", 4),
-                                       ("jacobi-nooverlap", 3), ("jacobi-fused", 2), ("jacobi-fused", 3), ("conv1", 2), ("conv3", 3), ("spmv", 2),
+                                       ("jacobi-nooverlap", 3), ("jacobi-fused", 2), ("jacobi-fused", 3),
+                                       ("jacobi-k4", 2), ("jacobi-k3", 3), ("conv1", 2), ("conv3", 3), ("spmv", 2),
                                        ("spmv", 3), ("spmv-hot", 2)])
 def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     script = tmp_path / "w.py"
