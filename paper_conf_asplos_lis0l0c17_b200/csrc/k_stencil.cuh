@@ -481,7 +481,7 @@ struct Jacobi5MultiBody {
     }
 
     __device__ __forceinline__ void consume(const Sched&, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
-        __shared__ float s_scr[kGroups][kRows * ST_COLS];
+        __shared__ __align__(16) float s_scr[kGroups][kRows * ST_COLS];   // float4 reads in sweep K
         float* X = reinterpret_cast<float*>(const_cast<uint8_t*>(stage));   // the group owns its slot
         float* Y = s_scr[(threadIdx.x - PRODUCER_THREADS) / kConsumers];
         sweep<1>(X, Y, bx, by, ctid);
