@@ -459,24 +459,36 @@ struct Jacobi5MultiBody {
         if (lane == 0) tma_load_2d(stage, &p.tmap, bx * 32 - 4, by * 32 - K, full);
     }
 
-    // one intermediate sweep s (1 <= s < K): staged rows [s, kRows - s),
-    // columns [4 - K + s, 36 + K - s), src -> dst (pitch ST_COLS)
+    // one intermediate sweep S (1 <= S < K) over staged rows [S, kRows - S) and
+    // the whole staged width (10 float4 chunks), src -> dst (pitch ST_COLS).
+    // Only the region [4-K+S, 36+K-S) is needed; the extra columns are
+    // computed from in-bounds neighbours (the adjacent row's ends) and never
+    // read by a valid point.  Thread = (chunk, a run of kRS rows): the three
+    // rows it needs slide down in registers.
+    static constexpr int kRS = 4;
     template <int S>
     __device__ __forceinline__ void sweep(const float* src, float* dst, int32_t bx, int32_t by, int ctid) const {
-        constexpr int H = kRows - 2 * S, W = 32 + 2 * (K - S), R0 = S, C0 = 4 - K + S;
-        const int gy0 = by * 32 - K, gx0 = bx * 32 - 4;
-        for (int idx = ctid; idx < H * W; idx += kConsumers) {
-            const int r = R0 + idx / W, c = C0 + idx % W;
-            const int gy = gy0 + r, gx = gx0 + c;
-            const float* q = src + r * ST_COLS + c;
-            float v;
-            if (gy <= 0 || gy >= p.rows - 1 || gx <= 0 || gx >= p.cols - 1) {
-                v = q[0];                                      // global boundary (or outside): unchanged
-            } else {
-                v = __fmul_rn(0.2f, __fadd_rn(__fadd_rn(__fadd_rn(__fadd_rn(q[0], q[-1]), q[1]), q[ST_COLS]),
-                                              q[-ST_COLS]));
-            }
-            dst[r * ST_COLS + c] = v;
+        constexpr int H = kRows - 2 * S;
+        constexpr int G = (H + kRS - 1) / kRS;                 // row runs
+        static_assert(G * 10 <= kConsumers, "one unit per thread");
+        if (ctid >= G * 10) return;
+        const int chunk = ctid % 10, rg = ctid / 10;
+        const int r0 = S + rg * kRS;
+        const int r1 = r0 + kRS < kRows - S ? r0 + kRS : kRows - S;
+        const int gx = bx * 32 - 4 + 4 * chunk, gyb = by * 32 - K;
+        const float* q = src + 4 * chunk;
+        float4 up = *reinterpret_cast<const float4*>(q + (r0 - 1) * ST_COLS);
+        float4 cur = *reinterpret_cast<const float4*>(q + r0 * ST_COLS);
+#pragma unroll
+        for (int k = 0; k < kRS; ++k) {
+            const int r = r0 + k;
+            if (r >= r1) break;
+            const float4 down = *reinterpret_cast<const float4*>(q + (r + 1) * ST_COLS);
+            const float lw = q[r * ST_COLS - 1], re = q[r * ST_COLS + 4];
+            *reinterpret_cast<float4*>(dst + r * ST_COLS + 4 * chunk) =
+                jacobi_point4(cur, up, down, lw, re, gyb + r, gx, p.rows, p.cols);
+            up = cur;
+            cur = down;
         }
     }
 
