@@ -811,7 +811,10 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             memset(&jp, 0, sizeof jp);
             jp.a = src; jp.b = dst; jp.ld = x->ld; jp.rows = x->rows; jp.cols = x->cols;
             jp.row0 = 0; jp.row_end = x->rows;
-            if (x->rows > 0 && x->cols > 0) CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 32 + 2 * fuse));
+            if (x->rows > 0 && x->cols > 0) {
+                CC_TRY(make_tmap(&jp.tmap, src, x->rows, x->cols, x->ld, ST_COLS, 32 + 2 * fuse));
+                CC_TRY(make_tmap(&jp.tmap2, src, x->rows, x->cols, x->ld, ST_COLS2, 32 + 2 * fuse));
+            }
             s = fuse == 2 ? launch_body<Jacobi5MultiBody<2>>(c, jp)
               : fuse == 3 ? launch_body<Jacobi5MultiBody<3>>(c, jp)
                           : launch_body<Jacobi5MultiBody<4>>(c, jp);

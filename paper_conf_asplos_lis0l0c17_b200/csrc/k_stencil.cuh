@@ -442,7 +442,8 @@ struct Jacobi5MultiBody {
     static constexpr int RB = 2;
     static constexpr int kConsumers = 256 / RB;
     static constexpr int kRows = 32 + 2 * K;                    // staged rows
-    static constexpr int kStageBytes = ((kRows * ST_COLS * 4) + 127) & ~127;
+    static constexpr int kMerge = 2;                            // two neighbouring tiles per slot (MergeOf)
+    static constexpr int kStageBytes = ((kRows * ST_COLS2 * 4) + 127) & ~127;
     static constexpr int kDirectStageBytes = kStageBytes;     // always TMA-staged
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
@@ -458,77 +459,97 @@ struct Jacobi5MultiBody {
         stage_commit(full, lane, (uint32_t)(kRows * ST_COLS * 4));
         if (lane == 0) tma_load_2d(stage, &p.tmap, bx * 32 - 4, by * 32 - K, full);
     }
+    // merged slots: tiles (bx, by), (bx+1, by) in one 72-column box
+    __device__ __forceinline__ bool can_merge(const Sched&) const { return true; }
+    __device__ __forceinline__ void produce_n(const Sched& s, int32_t bx, int32_t by, int n, uint8_t* stage,
+                                              uint64_t* full, int lane) {
+        if (n < 2) { produce(s, bx, by, stage, full, lane); return; }
+        stage_commit(full, lane, (uint32_t)(kRows * ST_COLS2 * 4));
+        if (lane == 0) tma_load_2d(stage, &p.tmap2, bx * 32 - 4, by * 32 - K, full);
+    }
 
     // one intermediate sweep S (1 <= S < K) over staged rows [S, kRows - S) and
-    // the whole staged width (10 float4 chunks), src -> dst (pitch ST_COLS).
-    // Only the region [4-K+S, 36+K-S) is needed; the extra columns are
-    // computed from in-bounds neighbours (the adjacent row's ends) and never
-    // read by a valid point.  Thread = (chunk, a run of kRS rows): the three
-    // rows it needs slide down in registers.
-    static constexpr int kRS = 4;
+    // the whole staged width (pitch / 4 float4 chunks), src -> dst.  Only the
+    // region K - S columns / rows inside the box edge is needed; the extra
+    // columns are computed from in-bounds neighbours (the adjacent row's ends)
+    // and never read by a valid point.  Thread = (chunk, a run of rows): the
+    // three rows it needs slide down in registers.
     template <int S>
-    __device__ __forceinline__ void sweep(const float* src, float* dst, int32_t bx, int32_t by, int ctid) const {
+    __device__ __forceinline__ void sweep(const float* src, float* dst, int pitch, int32_t bx, int32_t by,
+                                          int ctid) const {
         constexpr int H = kRows - 2 * S;
-        constexpr int G = (H + kRS - 1) / kRS;                 // row runs
-        static_assert(G * 10 <= kConsumers, "one unit per thread");
-        if (ctid >= G * 10) return;
-        const int chunk = ctid % 10, rg = ctid / 10;
-        const int r0 = S + rg * kRS;
-        const int r1 = r0 + kRS < kRows - S ? r0 + kRS : kRows - S;
+        const int nch = pitch >> 2;
+        const int runs = kConsumers / nch;                      // row runs that fit the group
+        const int rs = (H + runs - 1) / runs;                   // rows per run (<= 8)
+        const int G = (H + rs - 1) / rs;
+        if (ctid >= G * nch) return;
+        const int chunk = ctid % nch, rg = ctid / nch;
+        const int r0 = S + rg * rs;
+        const int r1 = r0 + rs < kRows - S ? r0 + rs : kRows - S;
         const int gx = bx * 32 - 4 + 4 * chunk, gyb = by * 32 - K;
         const float* q = src + 4 * chunk;
-        float4 up = *reinterpret_cast<const float4*>(q + (r0 - 1) * ST_COLS);
-        float4 cur = *reinterpret_cast<const float4*>(q + r0 * ST_COLS);
+        float4 up = *reinterpret_cast<const float4*>(q + (r0 - 1) * pitch);
+        float4 cur = *reinterpret_cast<const float4*>(q + r0 * pitch);
 #pragma unroll
-        for (int k = 0; k < kRS; ++k) {
+        for (int k = 0; k < 8; ++k) {
             const int r = r0 + k;
             if (r >= r1) break;
-            const float4 down = *reinterpret_cast<const float4*>(q + (r + 1) * ST_COLS);
-            const float lw = q[r * ST_COLS - 1], re = q[r * ST_COLS + 4];
-            *reinterpret_cast<float4*>(dst + r * ST_COLS + 4 * chunk) =
+            const float4 down = *reinterpret_cast<const float4*>(q + (r + 1) * pitch);
+            const float lw = q[r * pitch - 1], re = q[r * pitch + 4];
+            *reinterpret_cast<float4*>(dst + r * pitch + 4 * chunk) =
                 jacobi_point4(cur, up, down, lw, re, gyb + r, gx, p.rows, p.cols);
             up = cur;
             cur = down;
         }
     }
 
-    __device__ __forceinline__ void consume(const Sched&, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
-        __shared__ __align__(16) float s_scr[kGroups][kRows * ST_COLS];   // float4 reads in sweep K
-        float* X = reinterpret_cast<float*>(const_cast<uint8_t*>(stage));   // the group owns its slot
-        float* Y = s_scr[(threadIdx.x - PRODUCER_THREADS) / kConsumers];
-        sweep<1>(X, Y, bx, by, ctid);
-        consumer_sync<kConsumers>();
-        if constexpr (K >= 3) { sweep<2>(Y, X, bx, by, ctid); consumer_sync<kConsumers>(); }
-        if constexpr (K >= 4) { sweep<3>(X, Y, bx, by, ctid); consumer_sync<kConsumers>(); }
-        const float* F = (K & 1) ? X : Y;                          // holds sweep K-1
-        // final sweep K on the 32 x 32 tile (rows 32*by.., the float4 path)
+    // the last sweep on tile (bx, by) whose columns start coff floats into the box
+    __device__ __forceinline__ void final_sweep(const float* F, int pitch, int coff, int32_t bx, int32_t by,
+                                                int ctid) const {
         const int r0 = (ctid >> 3) * RB, c4 = ctid & 7;
         const int gx = bx * 32 + 4 * c4, gy0 = by * 32 + r0;
-        if (gx < p.cols) {
-            const float* t = F + (K - 1 + r0) * ST_COLS + 4 + 4 * c4;     // staged row of input row gy0 - 1
-            float4 row[RB + 2];
-            float lw[RB], re[RB];
+        if (gx >= p.cols) return;
+        const float* t = F + (K - 1 + r0) * pitch + coff + 4 + 4 * c4;      // staged row of input row gy0 - 1
+        float4 row[RB + 2];
+        float lw[RB], re[RB];
 #pragma unroll
-            for (int k = 0; k < RB + 2; ++k) row[k] = *reinterpret_cast<const float4*>(t + k * ST_COLS);
+        for (int k = 0; k < RB + 2; ++k) row[k] = *reinterpret_cast<const float4*>(t + k * pitch);
 #pragma unroll
-            for (int j = 0; j < RB; ++j) {
-                lw[j] = t[(j + 1) * ST_COLS - 1];
-                re[j] = t[(j + 1) * ST_COLS + 4];
-            }
-            const bool inner = gx >= 1 && gx + 4 <= p.cols - 1 && gy0 >= 1 && gy0 + RB <= p.rows - 1;
-#pragma unroll
-            for (int j = 0; j < RB; ++j) {
-                const int gy = gy0 + j;
-                if (gy >= p.rows) break;
-                float* dst = p.b + (int64_t)gy * p.ld + gx;
-                if (inner) *reinterpret_cast<float4*>(dst) = jacobi_core4(row[j + 1], row[j], row[j + 2], lw[j], re[j]);
-                else store4_masked(dst, jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows,
-                                                      p.cols), gx, p.cols);
-            }
+        for (int j = 0; j < RB; ++j) {
+            lw[j] = t[(j + 1) * pitch - 1];
+            re[j] = t[(j + 1) * pitch + 4];
         }
+        const bool inner = gx >= 1 && gx + 4 <= p.cols - 1 && gy0 >= 1 && gy0 + RB <= p.rows - 1;
+#pragma unroll
+        for (int j = 0; j < RB; ++j) {
+            const int gy = gy0 + j;
+            if (gy >= p.rows) break;
+            float* dst = p.b + (int64_t)gy * p.ld + gx;
+            if (inner) *reinterpret_cast<float4*>(dst) = jacobi_core4(row[j + 1], row[j], row[j + 2], lw[j], re[j]);
+            else store4_masked(dst, jacobi_point4(row[j + 1], row[j], row[j + 2], lw[j], re[j], gy, gx, p.rows,
+                                                  p.cols), gx, p.cols);
+        }
+    }
+
+    __device__ __forceinline__ void consume_n(const Sched&, int32_t bx, int32_t by, int n, const uint8_t* stage,
+                                              int ctid) {
+        __shared__ __align__(16) float s_scr[kGroups][kRows * ST_COLS2];   // float4 reads in sweep K
+        const int pitch = n >= 2 ? ST_COLS2 : ST_COLS;
+        float* X = reinterpret_cast<float*>(const_cast<uint8_t*>(stage));   // the group owns its slot
+        float* Y = s_scr[(threadIdx.x - PRODUCER_THREADS) / kConsumers];
+        sweep<1>(X, Y, pitch, bx, by, ctid);
+        consumer_sync<kConsumers>();
+        if constexpr (K >= 3) { sweep<2>(Y, X, pitch, bx, by, ctid); consumer_sync<kConsumers>(); }
+        if constexpr (K >= 4) { sweep<3>(X, Y, pitch, bx, by, ctid); consumer_sync<kConsumers>(); }
+        const float* F = (K & 1) ? X : Y;                          // holds sweep K-1
+        final_sweep(F, pitch, 0, bx, by, ctid);
+        if (n >= 2) final_sweep(F, pitch, 32, bx + 1, by, ctid);
         // K even: sweep K read the scratch buffer, which the group's next task
         // overwrites in its first sweep -- every thread must be done with it
         if constexpr (!(K & 1)) consumer_sync<kConsumers>();
+    }
+    __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t by, const uint8_t* stage, int ctid) {
+        consume_n(s, bx, by, 1, stage, ctid);
     }
     __device__ __forceinline__ void finish(int) {}
 };
