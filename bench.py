@@ -75,7 +75,7 @@ def parse():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
-    ap.add_argument("--fuse", type=int, default=2, help="jacobi: sweeps per launch, 1-4 (R32; 2 measured best)")
+    ap.add_argument("--fuse", type=int, default=3, help="jacobi: sweeps per launch, 1-4 (R32; 3 measured best)")
     ap.add_argument("--halo", default="exchange", choices=["exchange", "fused"],
                     help="jacobi N > 1: NCCL halo exchange per sweep, or the fused peer-memory LL halo")
     ap.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
