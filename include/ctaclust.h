@@ -155,7 +155,9 @@ typedef struct {
     int32_t stages;         /* agent backends: depth of the per-agent shared-memory ring
                                the scheduler warp stages upcoming tasks into -- the
                                B200 form of "prefetch the next CTA" (§4.3(III),
-                               Listing 5 l.34-37); 0 => the kernel's default, 1..8   */
+                               Listing 5 l.34-37); 0 => the kernel's default, 1..8;
+                               rounded up to a multiple of the body's consumer
+                               groups (each ring slot belongs to one group)          */
     int32_t batch;          /* logical CTAs claimed per queue atomic; 0 => default   */
     int32_t staging;        /* how a task's input tile reaches the body (cc_staging):
                                0 default (= TMA), 1 TMA: one 2D tensor load per tile,

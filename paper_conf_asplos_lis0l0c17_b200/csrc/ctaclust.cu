@@ -500,6 +500,22 @@ struct LaunchCtx {
     int32_t* nl;
 };
 
+// Ring depth of an agent launch: the requested stages rounded UP to a
+// multiple of the body's consumer groups.  Group g consumes tasks g, g+G, ...,
+// i.e. slots (g + kG) mod S; with S % G == 0 every slot belongs to one group,
+// so a group's successive waits on a slot are for consecutive phases.  With
+// S % G != 0 two groups share a slot, and a group can reach its wait for a
+// slot while the other group's fill of it is still in flight -- the
+// one-bit phase parity then reports the phase two back as complete and the
+// group consumes the wrong task (round 2: stages = 3 with two groups hung or
+// faulted on full-size stencils; scripts/probe_stages.py).
+template <class Body>
+static int ring_depth(int requested) {
+    int S = requested > 0 ? requested : Body::kDefaultStages;
+    S = ((S + Body::kGroups - 1) / Body::kGroups) * Body::kGroups;
+    return S < MAX_STAGES ? S : MAX_STAGES - MAX_STAGES % Body::kGroups;
+}
+
 template <class Body>
 static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& prm) {
     const Grid& g = c.p->g;
@@ -538,8 +554,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         break;
     case CC_BACKEND_AGENT:
     case CC_BACKEND_AGENT_IDENTITY: {
-        int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
-        if (S < Body::kGroups) S = Body::kGroups;             // every consumer group needs a slot
+        int S = ring_depth<Body>(o.stages);
         int occ = 0;
         CC_TRY(set_carveout(k_agent<Body>, o.carveout));
         if (o.carveout < 0) CC_TRY(occupancy<Body>(c.p->device, S, &occ, direct));
@@ -562,8 +577,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         break;
     }
     case CC_BACKEND_AGENT_STATIC: {
-        int S = o.stages > 0 ? o.stages : Body::kDefaultStages;
-        if (S < Body::kGroups) S = Body::kGroups;
+        int S = ring_depth<Body>(o.stages);
         CC_TRY(set_carveout(k_static<Body>, o.carveout));
         s.active_agents = 1;
         s.throttle = 0;

@@ -167,3 +167,20 @@ def test_workspace_ordered_across_streams():
         t.join()
     torch.cuda.synchronize()
     assert all(bool(torch.all(c == 1)) for c in cens)
+
+
+@pytest.mark.parametrize("stages", [3, 5, 7])
+def test_ring_depth_not_multiple_of_groups(stages):
+    """Regression (round 2): a ring depth that is not a multiple of the body's
+    consumer groups let two groups share a slot, and on full-size launches a
+    group could take the parity of a fill still in flight for the other group
+    (hang / launch failure).  The launcher now rounds the depth up; a large
+    two-group stencil launch with such a request must be exact."""
+    from paper_conf_asplos_lis0l0c17_b200 import synth
+    import oracle as O
+    u0 = synth.matrix(4, 8192, 8192)
+    a = torch.from_numpy(u0).cuda()
+    out = ops.jacobi5(a, torch.empty_like(a), 2, backend="agent", order="row", stages=stages)
+    torch.cuda.synchronize()
+    ref = O.jacobi5_f32(u0, 2)
+    assert np.array_equal(out.cpu().numpy(), ref)
