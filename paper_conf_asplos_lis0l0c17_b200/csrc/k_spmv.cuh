@@ -153,9 +153,12 @@ struct SpmvBody {
 
     __device__ __forceinline__ void consume(const Sched& s, int32_t bx, int32_t /*by*/, const uint8_t*, int ctid) {
         __shared__ int32_t s_rowend[SPMV_ROWCAP];
-        // products of the CTA's nonzeros, index j stored at j + j/IPT (the pad
-        // keeps each thread's IPT-long private run conflict-free)
-        __shared__ float s_prod[SPMV_IPC + SPMV_IPC / SPMV_IPT];
+        // products of the CTA's nonzeros, index j stored at j + j/32: the
+        // coalesced writes (a warp's 32 consecutive j) are conflict-free, and
+        // the merge walk's reads (lane t at ~15 t: its run starts after the
+        // rows ended before it) spread over the banks (round 2: j + j/16 put
+        // them ~16 words apart -- 41 % excess shared wavefronts, ncu r10l)
+        __shared__ float s_prod[SPMV_IPC + SPMV_IPC / 32];
         __shared__ float s_wv[SPMV_THREADS / 32];
         __shared__ int32_t s_wf[SPMV_THREADS / 32];
         const int t = ctid, lane = t & 31, warp = t >> 5;
@@ -200,7 +203,7 @@ struct SpmvBody {
 #pragma unroll
                 for (int k = 0; k < SPMV_GB; ++k) {
                     const int32_t j = t + (k0 + k) * kConsumers;
-                    if (j < nz) s_prod[j + j / SPMV_IPT] = v[k] * xv[k];
+                    if (j < nz) s_prod[j + j / 32] = v[k] * xv[k];
                 }
             }
         } else if (l2h != 0) {
@@ -214,7 +217,7 @@ struct SpmvBody {
                     const int32_t c = hf ? ld_stream_i32_h(p.col + y0 + j, pf) : ld_stream_i32(p.col + y0 + j);
                     const float v = hf ? ld_stream_f32_h(p.val + y0 + j, pf) : ld_stream_f32(p.val + y0 + j);
                     const float* xp = c >= 0 ? p.x + c : p.xh_end + c;
-                    s_prod[j + j / SPMV_IPT] = v * (hl ? ld_cached_h(xp, pl) : ld_cached(xp));
+                    s_prod[j + j / 32] = v * (hl ? ld_cached_h(xp, pl) : ld_cached(xp));
                 }
             }
         }
@@ -243,7 +246,7 @@ struct SpmvBody {
             for (int it = 0; it < SPMV_IPT; ++it) {
                 if (it < items) {
                     if (cj < re) {
-                        sum += s_prod[cj + cj / SPMV_IPT];
+                        sum += s_prod[cj + cj / 32];
                         ++cj;
                     } else {
                         if (!has_end) { first_row = cx; first_val = sum; has_end = true; }
