@@ -57,7 +57,6 @@ struct Sched {
     uint32_t* census;             // optional outputs (see ctaclust.h)
     int32_t* exec_sm;
     int32_t* map;
-    int32_t oneshot;              // 1: default / redirect launch (one task per CTA)
 };
 
 __device__ __forceinline__ int32_t* ws_agent_ctr(const Sched& s) { return s.ws; }
@@ -361,15 +360,6 @@ template <class B> constexpr int direct_stage_bytes() { return DirectStageBytes<
 // cluster.  Their tiles share halo columns, so one wider copy stages both:
 // the clustered order is what makes the pair co-located, and the shared
 // halo is then reused from shared memory instead of being copied twice.
-// Persistent-only shared memory: a body may ask for kPersistentSmemBytes of
-// dynamic shared memory after the ring, allocated only for the persistent
-// backends (agent / identity / static) -- state an agent keeps across all its
-// tasks (HistBody's per-lane counters).  One-shot CTAs do not pay for it.
-template <class B, class = void> struct PersistentSmem { static constexpr int value = 0; };
-template <class B> struct PersistentSmem<B, decltype((void)B::kPersistentSmemBytes)> {
-    static constexpr int value = B::kPersistentSmemBytes;
-};
-
 template <class B, class = void> struct MergeOf { static constexpr int value = 1; };
 template <class B> struct MergeOf<B, decltype((void)B::kMerge)> { static constexpr int value = B::kMerge; };
 

@@ -406,12 +406,10 @@ using ColB = GemvBody<32, 256, false, true>;
 using BothB = GemvBody<32, 256, true, true>;
 
 template <class Body>
-static size_t dyn_smem(int stages, bool direct = false, bool persistent = false) {
+static size_t dyn_smem(int stages, bool direct = false) {
     // direct loads stage nothing: keep the ring minimal so L1 keeps the space
-    // (bodies whose direct path needs a per-task buffer size it themselves);
-    // persistent launches add the body's persistent-only region after the ring
-    return (size_t)stages * (direct ? direct_stage_bytes<Body>() : Body::kStageBytes) + 128 +
-           (persistent ? (size_t)PersistentSmem<Body>::value : 0);
+    // (bodies whose direct path needs a per-task buffer size it themselves)
+    return (size_t)stages * (direct ? direct_stage_bytes<Body>() : Body::kStageBytes) + 128;
 }
 
 // Opt every instantiation of a body into large dynamic shared memory once.
@@ -426,7 +424,7 @@ static cc_status prepare_body(int device) {
         CC_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, device));
         cudaFuncAttributes fa{};
         CC_CUDA(cudaFuncGetAttributes(&fa, k_agent<Body>));
-        const int mx = (int)std::min(dyn_smem<Body>(MAX_STAGES, false, true), (size_t)(optin - (int)fa.sharedSizeBytes));
+        const int mx = (int)std::min(dyn_smem<Body>(MAX_STAGES), (size_t)(optin - (int)fa.sharedSizeBytes));
         const int one = (int)dyn_smem<Body>(1);
         CC_CUDA(cudaFuncSetAttribute(k_agent<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
         CC_CUDA(cudaFuncSetAttribute(k_static<Body>, cudaFuncAttributeMaxDynamicSharedMemorySize, mx));
@@ -450,7 +448,7 @@ static cc_status occupancy(int device, int stages, int* occ, bool direct = false
         CC_CUDA(cudaGetDevice(&prev));
         CC_CUDA(cudaSetDevice(device));
         CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_agent<Body>, Body::kGroups * Body::kConsumers + PRODUCER_THREADS,
-                                                              dyn_smem<Body>(stages, direct, true)));
+                                                              dyn_smem<Body>(stages, direct)));
         CC_CUDA(cudaSetDevice(prev));
         cache[device][stages][direct] = n > 0 ? n : -1;
     }
@@ -546,14 +544,12 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         CC_TRY(set_carveout(k_default<Body>, o.carveout));
         s.map = nullptr;
         s.stages = 1;
-        s.oneshot = 1;
         k_default<Body><<<dim3(g.gx, g.gy), threads, dyn_smem<Body>(1, direct), c.st>>>(s, prm);
         break;
     }
     case CC_BACKEND_REDIRECT:
         CC_TRY(set_carveout(k_redirect<Body>, o.carveout));
         s.stages = 1;
-        s.oneshot = 1;
         k_redirect<Body><<<g.V, threads, dyn_smem<Body>(1, direct), c.st>>>(s, prm);
         break;
     case CC_BACKEND_AGENT:
@@ -565,7 +561,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         else {
             CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_agent<Body>,
                                                                   Body::kGroups * Body::kConsumers + PRODUCER_THREADS,
-                                                                  dyn_smem<Body>(S, direct, true)));
+                                                                  dyn_smem<Body>(S, direct)));
             if (occ < 1) return fail(CC_ERR_UNSUPPORTED, "carveout %d leaves no room for one agent", o.carveout);
         }
         const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
@@ -576,7 +572,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         const int grid = c.p->facts->num_sms * maxa;
         WsLease lease{c.p, c.st};
         CC_TRY(lease.acquire());
-        k_agent<Body><<<grid, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct, true), c.st>>>(s, prm);
+        k_agent<Body><<<grid, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
         if (cudaPeekAtLastError() == cudaSuccess) CC_TRY(lease.release());
         break;
     }
@@ -588,7 +584,7 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
         s.steal = 0;
         s.mode = MODE_STATIC;
         s.stages = S;
-        k_static<Body><<<g.M, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct, true), c.st>>>(s, prm);
+        k_static<Body><<<g.M, Body::kGroups * Body::kConsumers + PRODUCER_THREADS, dyn_smem<Body>(S, direct), c.st>>>(s, prm);
         break;
     }
     default:
