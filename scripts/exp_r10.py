@@ -198,8 +198,31 @@ def conv7():
     return {"conv7": r}
 
 
+def hist():
+    """HST (S8(f)3): default vs persistent variants, uniform and skewed bytes,
+    1 GiB (round 2 measured per-lane privatised 16-bit counters here: 0.53-0.74
+    ms against 0.29 ms for the shared-atomic default -- rejected and removed,
+    profiles/r11/exp/hist_privatised.json)"""
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    out = {}
+    n = 1 << 30
+    for kind in ("uniform", "skewed"):
+        data = synth.bytes_u8(31, n, kind=kind, backend="torch", device="cuda")
+        counts = torch.empty(64, dtype=torch.int32, device="cuda")
+        variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
+                    ("agent-row-s2", dict(backend="agent", order="row", stages=2)),
+                    ("identity", dict(backend="identity")),
+                    ("static-row-m1", dict(backend="static", order="row", num_clusters=148))]
+        r = B.measure(variants, lambda kw: ops.hist64(data, counts, **kw), 20, n, graph=True, inner=B.GRAPH_INNER)
+        out[kind] = r
+        print(kind, [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+        del data
+    return out
+
+
 if __name__ == "__main__":
     what, path = sys.argv[1], sys.argv[2]
     res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel, "conv7": conv7,
-           "spmv_control": spmv_control}[what]()
+           "spmv_control": spmv_control, "hist": hist}[what]()
     json.dump(res, open(path, "w"), indent=1)
