@@ -668,9 +668,10 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     const int C = c.o->cluster_size;
     if (C != 1 && C != 2 && C != 4 && C != 8) return fail(CC_ERR_INVALID_ARG, "cluster_size %d (1, 2, 4 or 8)", C);
     using G = TbcGeom<R, tbc_tw<R>()>;
-    CUtensorMap m_c, m_b;
+    CUtensorMap m_c, m_b, m_f;
     CC_TRY(make_tmap(&m_c, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, 32));
     CC_TRY(make_tmap(&m_b, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, G::kHb));
+    CC_TRY(make_tmap(&m_f, prm.in, prm.rows, prm.cols, prm.ld, G::kCols, 32 + G::kHb));
     Sched s{};
     s.g = g;
     s.census = c.o->d_census;
@@ -703,7 +704,7 @@ static cc_status launch_tbc(const LaunchCtx& c, const ConvParams<R>& prm) {
     if (nc < 1) return fail(CC_ERR_UNSUPPORTED, "tbcluster: no cluster of %d fits", C);
     if (nc > units) nc = (int)units;
     cfg.gridDim = dim3(nc * C);
-    CC_CUDA(cudaLaunchKernelEx(&cfg, k_conv_tbc<R>, m_c, m_b, s, prm, (int32_t)C));
+    CC_CUDA(cudaLaunchKernelEx(&cfg, k_conv_tbc<R>, m_c, m_b, m_f, s, prm, (int32_t)C));
     if (c.nl) ++*c.nl;
     return CC_OK;
 }

@@ -151,10 +151,11 @@ __device__ __forceinline__ void tma_load_2d_mc(void* dst, const void* tmap, int3
 
 // Persistent grid of NC clusters x C CTAs (1D, cluster dims (C,1,1)),
 // tbc_threads<R>() threads, dynamic smem tbc_smem_bytes<R>().
-// map_c: box (kCols x 32), map_b: box (kCols x Hb).
+// map_c: box (kCols x 32), map_b: box (kCols x Hb), map_f: box (kCols x (32 + Hb)).
 template <int R>
 __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_constant__ CUtensorMap map_c,
                                                           const __grid_constant__ CUtensorMap map_b,
+                                                          const __grid_constant__ CUtensorMap map_f,
                                                           const __grid_constant__ Sched s,
                                                           const __grid_constant__ ConvParams<R> p, int32_t C) {
     constexpr int TW = tbc_tw<R>();
@@ -199,9 +200,12 @@ __global__ void __launch_bounds__(tbc_threads<R>()) k_conv_tbc(const __grid_cons
                     // own rows [y0 - Hb/2, y0 + 32 - Hb/2), then B = the Hb rows
                     // centred on the boundary below (multicast to the partner)
                     const int yb = y0 + 32 - G::kHb / 2;
-                    tma_load_2d(stage, &map_c, x0 - 4, yb - 32, &full[st]);
-                    if (partner) tma_load_2d_mc(stage + 32 * G::kRowB, &map_b, x0 - 4, yb, &full[st], mask);
-                    else tma_load_2d(stage + 32 * G::kRowB, &map_b, x0 - 4, yb, &full[st]);
+                    if (partner) {
+                        tma_load_2d(stage, &map_c, x0 - 4, yb - 32, &full[st]);
+                        tma_load_2d_mc(stage + 32 * G::kRowB, &map_b, x0 - 4, yb, &full[st], mask);
+                    } else {                                 // no partner: own rows and B as one box
+                        tma_load_2d(stage, &map_f, x0 - 4, yb - 32, &full[st]);
+                    }
                 } else {
                     // B arrives from the partner; own rows [y0 + Hb/2, y0 + Hb/2 + 32)
                     tma_load_2d(stage + G::kHb * G::kRowB, &map_c, x0 - 4, y0 + G::kHb / 2, &full[st]);
