@@ -83,6 +83,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-parity", action="store_true")
+    ap.add_argument("--no-ncu", action="store_true", help="skip the live ncu L2-sector / DRAM count of the step")
     ap.add_argument("--suite", default=None, help="also run every BASELINE config's variants, write JSON here")
     ap.add_argument("--exchange", default="nccl", choices=["nccl", "torch"],
                     help="N > 1 exchanges: the library's NCCL communicator (default) or torch.distributed/gloo "
@@ -495,6 +496,17 @@ def main():
                                  "sample": f"{desc1} ({dt1:.1f} s)"},
                "cpu": cpu_info()}
 
+    live = None
+    if rank == 0 and world == 1 and not a.no_ncu:
+        live = live_ncu(a, head, "tma" if def_kind == "tma-staged" else "direct")
+        if live and a.config == "atax" and roof.get("kernel", "").startswith("k_agent<GemvBody<32, 256, 1, 1>>"):
+            pk_ = live["headline_per_kernel"].get("void k_agent<GemvBody<32, 256, 1, 1>>", {})
+            if pk_:
+                roof["traffic"] = (pk_.get("dram__bytes_read.sum", 0) + pk_.get("dram__bytes_write.sum", 0)) / 2
+                roof["traffic_source"] = "ncu in this run (per launch, cold L2)"
+        elif live and a.config != "atax":
+            roof["traffic"] = live["dram_bytes_per_step"]["headline"] / max(1, roof.get("launches_per_step") or 1)
+            roof["traffic_source"] = "ncu in this run (per launch, cold L2)"
     if rank == 0:
         l2red, prof = l2_reductions(a.config, head)
         line = {"metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": a.steps,
@@ -511,8 +523,9 @@ def main():
                 "ms_per_step_two_pass_atax": None if ms_two_pass is None else round(ms_two_pass, 4),
                 "roofline": roof, "clocks": clk, "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": launches,
                 "home_fraction": home, "parity": parity,
-                "l2_sector_reduction": {"source": prof, "metric": "1 - lts__t_sectors_srcunit_tex(variant) / (reference order)",
-                                        **l2red}}
+                "l2_sector_reduction": live if live else
+                {"source": prof, "metric": "1 - lts__t_sectors_srcunit_tex(variant) / (reference order)", **l2red},
+                "l2_sector_reduction_suite": {"source": prof, **l2red} if live else None}
         if a.config == "jacobi":
             line["sweeps_per_second"] = round(D.iters / (ms_clu * 1e-3), 1)
         if per_clu:
@@ -553,6 +566,61 @@ def config_block(a, D, head, world, use_graph):
         c.update(rows=D.rows, nnz=D.nnz, hub_slots=D.A.n_hot,
                  l2="col/val 2 GiB larger than L2; x (64 MiB) fits, as it would in use")
     return c
+
+
+def live_ncu(a, head, dflt_staging):
+    """L2 sectors and DRAM bytes of one step of the headline schedule, default
+    order and the identity control, measured in this run: scripts/ncu_step.py
+    under `ncu --profile-from-start off --cache-control all` (a separate
+    process, after the timed region; counts only, never a timing).  None when
+    ncu is unavailable or fails."""
+    import csv
+    import io
+    import shutil
+    ncu = shutil.which("ncu") or ("/usr/local/cuda/bin/ncu" if os.path.exists("/usr/local/cuda/bin/ncu") else None)
+    if not ncu:
+        return None
+    metrics = "lts__t_sectors_srcunit_tex.sum,dram__bytes_read.sum,dram__bytes_write.sum"
+    variants = {"headline": head, "default": dict(backend="default", staging=dflt_staging),
+                "identity": dict(backend="identity")}
+    out = {}
+    for name, opts in variants.items():
+        cmd = [ncu, "--profile-from-start", "off", "--metrics", metrics, "--cache-control", "all",
+               "--clock-control", "none", "--csv", sys.executable, os.path.join(ROOT, "scripts", "ncu_step.py"),
+               "--config", a.config, "--opts", json.dumps(opts), "--hot", str(a.hot), "--fuse", str(a.fuse)]
+        if a.n:
+            cmd += ["--size", str(a.n)]
+        try:
+            r = subprocess.run(cmd, capture_output=True, text=True, timeout=240)
+        except Exception:
+            return None
+        rows = [row for row in csv.reader(io.StringIO(r.stdout)) if len(row) > 10]
+        if not rows or rows[0][0] != "ID":
+            return None
+        h = rows[0]
+        per_kernel, tot = {}, {}
+        for row in rows[1:]:
+            d = dict(zip(h, row))
+            try:
+                v = float(d["Metric Value"].replace(",", ""))
+            except ValueError:
+                continue
+            m = d["Metric Name"]
+            tot[m] = tot.get(m, 0.0) + v
+            k = d["Kernel Name"].split("(")[0]
+            per_kernel.setdefault(k, {}).setdefault(m, 0.0)
+            per_kernel[k][m] += v
+        out[name] = {"l2_sectors": tot.get("lts__t_sectors_srcunit_tex.sum"),
+                     "dram_bytes": tot.get("dram__bytes_read.sum", 0.0) + tot.get("dram__bytes_write.sum", 0.0),
+                     "per_kernel": per_kernel}
+    h, d, i = out["headline"], out["default"], out["identity"]
+    return {"source": "ncu in this run (scripts/ncu_step.py, --cache-control all, one step per schedule)",
+            "metric": "1 - lts__t_sectors_srcunit_tex(headline step) / (reference step)",
+            "vs_default_order": round(1 - h["l2_sectors"] / d["l2_sectors"], 4) if d["l2_sectors"] else None,
+            "vs_identity_order": round(1 - h["l2_sectors"] / i["l2_sectors"], 4) if i["l2_sectors"] else None,
+            "l2_sectors_per_step": {k: v["l2_sectors"] for k, v in out.items()},
+            "dram_bytes_per_step": {k: v["dram_bytes"] for k, v in out.items()},
+            "headline_per_kernel": h["per_kernel"]}
 
 
 def l2_reductions(cfg, head):

@@ -4,7 +4,7 @@ TAG=${1:-r02}
 OUT=gpurun_out/ncu_$TAG
 mkdir -p $OUT
 timeout -k 5 900 ncu --metrics gpu__time_duration.sum --clock-control none -k 'regex:k_(agent|default|redirect|static)' -c 400 --csv \
-   --log-file $OUT/bench_launches.csv python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-parity > $OUT/bench_under_ncu.log 2>&1
+   --log-file $OUT/bench_launches.csv python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --no-parity --no-ncu > $OUT/bench_under_ncu.log 2>&1
 echo launches rc=$?
 timeout -k 5 900 ncu --set full --import-source on --clock-control none -k 'regex:k_agent' -s 2 -c 2 \
    -o $OUT/full_atax_agent python scripts/ncu_target.py --kernel atax --backend agent --order col --warm 1 --reps 1 > $OUT/full_atax.log 2>&1
