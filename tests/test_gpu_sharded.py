@@ -19,7 +19,7 @@ import pytest
 import torch
 
 import oracle as O
-from paper_conf_asplos_lis0l0c17_b200 import drivers, ops, shard, synth
+from paper_conf_asplos_lis0l0c17_b200 import drivers, ops, synth
 
 pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
