@@ -117,7 +117,10 @@ typedef enum {
     CC_BACKEND_AGENT = 1,          /* agent-based clustering (Listing 5; "CLU",
                                       with throttling "CLU+TOT")                       */
     CC_BACKEND_TBCLUSTER = 2,      /* Blackwell thread-block clusters: the hardware form
-                                      of clustering (conv2d only in this build)        */
+                                      of clustering (conv2d only in this build): a
+                                      persistent grid of clusters of cluster_size CTAs
+                                      on vertically adjacent tiles; the rows a CTA pair
+                                      shares are fetched once and TMA-multicast to both */
     CC_BACKEND_AGENT_IDENTITY = 3, /* persistence-only control: same agents, one global
                                       queue in row-major order, no locality grouping   */
     CC_BACKEND_REDIRECT = 4,       /* redirection-based clustering "RD" (Listing 4,
@@ -173,7 +176,7 @@ typedef struct {
                                once whatever the hardware does with agent placement
                                (reading R10); 0 => paper-faithful: CTAs of a cluster
                                with no active agent are NOT run (census shows it)       */
-    int32_t cluster_size;   /* TBCLUSTER: CTAs per cluster along y (1..8)               */
+    int32_t cluster_size;   /* TBCLUSTER: CTAs per cluster along y (1, 2, 4 or 8)       */
     uint32_t* d_census;     /* DEVICE, |V|, optional: census[lin] += 1 per execution;
                                caller zeroes it                                        */
     int32_t* d_exec_sm;     /* DEVICE, |V|, optional: %smid that executed lin          */
