@@ -304,6 +304,14 @@ typedef struct {
  * base: add the exporter's offset; close with cc_ipc_close).  Errors:
  * INVALID_ARG, UNSUPPORTED (no P2P path), CUDA. */
 cc_status cc_peer_access(int32_t device, int32_t peer);
+
+/* L2 residency for the reused operand (S§8(f)2; SpMV's x): set an
+ * access-policy window on `stream` so later launches on it (also when
+ * captured into a graph) mark [ptr, ptr + bytes) persisting in L2 with
+ * `hit_ratio` in (0, 1], after raising the device's persisting-L2 limit to
+ * cover it (clamped to the device maximum).  bytes = 0 clears the window and
+ * resets the persisting lines.  Errors: INVALID_ARG, CUDA. */
+cc_status cc_l2_persist(void* stream, const void* ptr, size_t bytes, float hit_ratio);
 cc_status cc_ipc_handle(const void* dptr, void* handle64, uint64_t* offset);
 cc_status cc_ipc_open(const void* handle64, int32_t device, void** dptr);
 cc_status cc_ipc_close(void* dptr);

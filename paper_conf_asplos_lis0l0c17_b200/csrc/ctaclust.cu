@@ -981,6 +981,32 @@ extern "C" cc_status cc_peer_access(int32_t device, int32_t peer) {
     if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceEnablePeerAccess");
     return CC_OK;
 }
+extern "C" cc_status cc_l2_persist(void* stream, const void* ptr, size_t bytes, float hit_ratio) {
+    cudaStream_t st = (cudaStream_t)stream;
+    cudaStreamAttrValue v;
+    memset(&v, 0, sizeof v);
+    if (bytes == 0) {
+        v.accessPolicyWindow.num_bytes = 0;
+        CC_CUDA(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v));
+        CC_CUDA(cudaCtxResetPersistingL2Cache());
+        return CC_OK;
+    }
+    if (!ptr || !(hit_ratio > 0.f && hit_ratio <= 1.f)) return fail(CC_ERR_INVALID_ARG, "l2 persist: ptr / hit_ratio");
+    int dev = 0, max_persist = 0, max_window = 0;
+    CC_CUDA(cudaGetDevice(&dev));
+    CC_CUDA(cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, dev));
+    CC_CUDA(cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, dev));
+    const size_t win = std::min(bytes, (size_t)max_window);
+    CC_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min(win, (size_t)max_persist)));
+    v.accessPolicyWindow.base_ptr = const_cast<void*>(ptr);
+    v.accessPolicyWindow.num_bytes = win;
+    v.accessPolicyWindow.hitRatio = hit_ratio;
+    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    CC_CUDA(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v));
+    return CC_OK;
+}
+
 // IPC maps whole allocations: the handle names the allocation holding dptr
 // (a caching allocator hands out sub-blocks), *offset is dptr's byte offset in it.
 extern "C" cc_status cc_ipc_handle(const void* dptr, void* handle64, uint64_t* offset) {

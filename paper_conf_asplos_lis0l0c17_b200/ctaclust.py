@@ -36,7 +36,7 @@ EXPORTS = ["cc_plan_create", "cc_plan_destroy", "cc_plan_info", "cc_plan_table",
            "cc_plan_invert", "cc_device_info", "cc_sm_rank_table", "cc_launch_opts_default",
            "cc_kernel_grid", "cc_max_agents", "cc_launch", "cc_spmv_partition", "cc_spmv_inspect", "cc_l1_reuse_probe", "cc_comm_unique_id",
            "cc_comm_init", "cc_comm_destroy", "cc_halo_exchange", "cc_allreduce_sum", "cc_allgather",
-           "cc_peer_access", "cc_ipc_handle", "cc_ipc_open", "cc_ipc_close", "cc_status_string", "cc_last_error", "cc_last_cuda_error", "cc_version"]
+           "cc_peer_access", "cc_l2_persist", "cc_ipc_handle", "cc_ipc_open", "cc_ipc_close", "cc_status_string", "cc_last_error", "cc_last_cuda_error", "cc_version"]
 
 
 class CtaclustError(RuntimeError):
@@ -299,6 +299,13 @@ def ll_words(cols: int) -> int:
 
 def peer_access(device: int, peer: int):
     _check(lib().cc_peer_access(_i32(device), _i32(peer)))
+
+
+def l2_persist(t, hit_ratio: float = 1.0, stream=None):
+    """cc_l2_persist: keep device tensor t (or None: clear) L2-persisting for
+    launches on `stream`."""
+    ptr, nbytes = (None, 0) if t is None else (t.data_ptr(), t.numel() * t.element_size())
+    _check(lib().cc_l2_persist(_vp(_stream(stream)), _vp(ptr), ctypes.c_size_t(nbytes), ctypes.c_float(hit_ratio)))
 
 
 def ipc_handle(t) -> tuple[bytes, int]:

@@ -36,6 +36,32 @@ def spmv():
     return out
 
 
+def spmv_persist():
+    """SpMV with x (64 MiB) held L2-persisting through an access-policy window
+    (cc_l2_persist) vs without; eager launches on one stream (the window is a
+    stream attribute), 5 per event pair"""
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc, ops, synth
+    rp, col = synth.rmat_csr(7, 24, 16, backend="torch", device="cuda")
+    n, nnz = rp.numel() - 1, col.numel()
+    val = synth.uniform(8, nnz, backend="torch", device="cuda")
+    x = synth.uniform(9, n, backend="torch", device="cuda")
+    y = torch.empty(n, device="cuda")
+    nbytes = 8 * nnz + 4 * (n + 1) + 8 * n
+    out = {}
+    for hot in (0, 16384):
+        Am = ops.SpmvMatrix(rp, col, val, hot=hot)
+        variants = [("default", dict(backend="default")), ("agent-row", dict(backend="agent", order="row")),
+                    ("identity", dict(backend="identity"))]
+        for persist in (False, True):
+            cc.l2_persist(x if persist else None, 1.0)
+            r = B.measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 20, nbytes, inner=5)
+            out[f"hot{hot}-persist{int(persist)}"] = r
+            print(hot, persist, [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+        cc.l2_persist(None)
+    return out
+
+
 def spmv_control():
     """SpMV data-related class: (1) the no-locality control -- the same R-MAT
     graph with its vertices randomly relabelled; (2) an
@@ -224,5 +250,5 @@ def hist():
 if __name__ == "__main__":
     what, path = sys.argv[1], sys.argv[2]
     res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel, "conv7": conv7,
-           "spmv_control": spmv_control, "hist": hist}[what]()
+           "spmv_control": spmv_control, "hist": hist, "spmv_persist": spmv_persist}[what]()
     json.dump(res, open(path, "w"), indent=1)

@@ -31,6 +31,7 @@ def main():
     ap.add_argument("--warm", type=int, default=1)
     ap.add_argument("--scale", type=int, default=24)
     ap.add_argument("--hot", type=int, default=0, help="spmv: hub-column form with this many hub slots")
+    ap.add_argument("--persist-x", action="store_true", help="spmv: x L2-persisting (cc_l2_persist)")
     ap.add_argument("--small", action="store_true",
                     help="reduced problem (categorizer probe, P:2275): n/4 matrices, scale-18 SpMV")
     a = ap.parse_args()
@@ -83,6 +84,9 @@ def main():
         x = synth.uniform(9, rp.numel() - 1, backend="torch", device=dev)
         Am = ops.SpmvMatrix(rp, col, val, hot=a.hot)
         y = torch.empty(rp.numel() - 1, device=dev)
+        if a.persist_x:
+            from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+            cc.l2_persist(x)
         if a.backend == "cusparse":          # vendor library, for context only
             Acsr = torch.sparse_csr_tensor(rp, col, val, (rp.numel() - 1, rp.numel() - 1))
             fn = lambda: torch.mv(Acsr, x)
