@@ -601,3 +601,26 @@ def test_stencils_degenerate(v, rows, cols):
     out = ops.jacobi5(a2, b, 3, **v)
     torch.cuda.synchronize()
     assert np.array_equal(out.cpu().numpy(), O.jacobi5_f32(img, 3)), v
+
+
+def test_spmv_with_l2_persisting_x():
+    """cc_l2_persist: results unchanged with x held L2-persisting on the stream,
+    and the window clears."""
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    rp, col = synth.rmat_csr(7, 12, 16)
+    val, x = synth.uniform(8, len(col)), synth.uniform(9, len(rp) - 1)
+    Am = _csr_dev(rp, col, val)
+    xd = dev(x)
+    ref = O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), val, x)
+    cc.l2_persist(xd, 1.0)
+    try:
+        for v in (dict(backend="default"), dict(backend="agent", order="row")):
+            y = ops.spmv(Am, xd, **v)
+            torch.cuda.synchronize()
+            got = y.cpu().numpy()
+            nz = ref != 0
+            assert relerr(got[nz], ref[nz]) <= TOL
+    finally:
+        cc.l2_persist(None)
+    with pytest.raises(cc.CtaclustError):
+        cc.l2_persist(xd, 0.0)
