@@ -378,6 +378,8 @@ def main():
         head["backend"] = a.backend
         if a.backend != "static":
             head.pop("num_clusters", None)
+        if a.backend not in ("agent", "identity", "static"):
+            head.pop("shub", None)                 # the shared-memory hub tier needs persistent agents
     if a.order:
         head["order"] = a.order
     for k, v in (("active_agents", a.active_agents), ("stages", a.stages), ("batch", a.batch)):
@@ -443,7 +445,7 @@ def main():
         ms_def, per_def, def_kind = ms_def_tma, per_def_tma, "tma-staged"
     else:
         ms_def, per_def, def_kind = ms_def_dir, per_def_dir, "direct-load"
-    ms_id, _, _ = timed({"backend": "identity"}, cmp_steps)
+    ms_id, _, _ = timed(identity_opts(head), cmp_steps)
     ms_two_pass = None
     if a.config == "atax" and D.fused_atax:         # the same clustered step with the two-pass ATAX
         D.fused_atax = False
@@ -582,7 +584,7 @@ def live_ncu(a, head, dflt_staging):
         return None
     metrics = "lts__t_sectors_srcunit_tex.sum,dram__bytes_read.sum,dram__bytes_write.sum"
     variants = {"headline": head, "default": dict(backend="default", staging=dflt_staging),
-                "identity": dict(backend="identity")}
+                "identity": identity_opts(head)}
     out = {}
     for name, opts in variants.items():
         cmd = [ncu, "--profile-from-start", "off", "--metrics", metrics, "--cache-control", "all",
@@ -649,6 +651,12 @@ def l2_reductions(cfg, head):
     return {"vs_default_order": vs_def, "vs_identity_order": vs_id}, os.path.relpath(profs[-1], ROOT)
 
 
+def identity_opts(head):
+    """the persistence-only control of a headline schedule: the same body
+    (SpMV's shared-memory hub tier included) in identity order"""
+    return dict(backend="identity", **({"shub": True} if head.get("shub") else {}))
+
+
 def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
     peak_hbm = pk["hbm_gbs"] if pk else 6650.0
     src = "MEASURED_PEAKS.json hbm_gbs (copy)" if pk else "fallback 6.65 TB/s"
@@ -678,7 +686,7 @@ def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
     ms_launch = ms_clu / nl
     body = {"jacobi": f"Jacobi5MultiBody<{D.fuse}>" if a.config == "jacobi" and D.fuse > 1 else "Jacobi5BodyT<false>",
             "conv3": "Conv2dBody<1>", "conv7": "Conv2dBody<3>",
-            "spmv": "SpmvBody"}[a.config]
+            "spmv": "SpmvShubBody" if head.get("shub") else "SpmvBody"}[a.config]
     kern = {"agent": "k_agent", "static": "k_static", "default": "k_default", "identity": "k_agent"}.get(
         head.get("backend"), "k_agent") + f"<{body}>"
     bpl = D.bytes_per_step() // nl if D.x.world == 1 else None
@@ -747,8 +755,9 @@ def home_fraction(a, D, head, device):
             kern = "conv2d"
         else:
             args = D.A.args(D.xv, D.y)
-            kern = "spmv"
+            kern = "spmv_shub" if head.get("shub") else "spmv"
         kw = dict(head)
+        kw.pop("shub", None)
         order, nc = kw.pop("order", None), kw.pop("num_clusters", 0)
         from paper_conf_asplos_lis0l0c17_b200 import ops
         p = ops.plan_for(kern, args, order, kw.pop("tile", None), nc, device)

@@ -206,7 +206,8 @@ typedef enum {
     CC_K_SPMV = 7,     /* cc_spmv_args     (config 5)                               */
     CC_K_HIST64 = 8,   /* cc_hist64_args   (S§8(f)3, the paper's HST)               */
     CC_K_JACOBI5_HALO = 9, /* cc_jacobi5_halo_args (S§8(f)4: sharded sweep, fused peer halo) */
-    CC_K_ATAX_FUSED = 10  /* cc_atax_args: one-pass ATAX (both PolyBench kernels per row) */
+    CC_K_ATAX_FUSED = 10, /* cc_atax_args: one-pass ATAX (both PolyBench kernels per row) */
+    CC_K_SPMV_SHUB = 11   /* cc_spmv_args: SpMV with the hub array in each agent's shared memory */
 } cc_kernel;
 
 /* CC_K_CENSUS: no data. */
@@ -336,7 +337,18 @@ typedef struct { const float* in; float* out; int64_t ld; int32_t rows, cols; in
  * kernel, counted in *launches), then the SpMV reads hub references from that
  * dense 4 * n_hot-byte array, which every SM keeps in L1.  Same y bits as the
  * plain form (the products and their order do not change).  n_hot = 0: plain
- * CSR, hot/xh ignored. */
+ * CSR, hot/xh ignored.
+ * CC_K_SPMV_SHUB: the same computation and y bits, for the persistent
+ * backends only (agent / identity / static; others UNSUPPORTED): each agent
+ * copies the CC_SPMV_SHUB_SLOTS hottest hub values (slots 0 .. , the
+ * inspector numbers slots in non-increasing degree order) into its shared
+ * memory once, with one bulk copy when its first task is staged, and every
+ * logical CTA it runs reads them from there (LDS) instead of through L1 / L2;
+ * slots past the tier are read from xh as in the plain hub form.  The hub
+ * columns are the x entries all logical CTAs share (inter-CTA reuse
+ * of the data-related class), caught on chip by the persistent agent.
+ * xh 16-byte aligned. */
+#define CC_SPMV_SHUB_SLOTS 8192
 typedef struct { int32_t rows, cols; int64_t nnz; const int32_t* row_ptr; const int32_t* col;
                  const float* val; const float* x; float* y; const int32_t* part;
                  const int32_t* hot; float* xh; int32_t n_hot; } cc_spmv_args;
@@ -363,7 +375,12 @@ cc_status cc_spmv_partition(const cc_spmv_args* args, int32_t* part, void* strea
  * col_hot[k] = -(slot+1) for a hub reference, else col[k] (DEVICE int32[nnz];
  * may not alias col).  scratch: DEVICE int32[cols + 65536 + 2].  Columns with
  * no reference are never hubs; ties at the degree threshold are taken in an
- * unspecified order.  *n_hot (HOST) = slots used.  Runs on `stream` and
+ * unspecified order.  Slots [0, min(n_hot, CC_SPMV_SHUB_SLOTS)) hold the most
+ * referenced hubs (every one referenced at least as often as any later slot;
+ * degrees clamped at 65535), the rest the others; inside each range slots
+ * follow column order only roughly (they are handed out by atomic counters),
+ * which keeps a row's sorted column run on few lines of the hub array.
+ * *n_hot (HOST) = slots used.  Runs on `stream` and
  * synchronizes it (one 256 KB degree histogram is read back to pick the
  * threshold).  Errors: INVALID_ARG (null, max_hot < 0), CUDA. */
 cc_status cc_spmv_inspect(const cc_spmv_args* args, int32_t max_hot, int32_t* hot, int32_t* col_hot,

@@ -369,7 +369,7 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
     }
     case CC_K_JACOBI5_HALO: { auto* c = (const cc_jacobi5_halo_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
     case CC_K_CONV2D: { auto* c = (const cc_conv2d_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
-    case CC_K_SPMV: {
+    case CC_K_SPMV: case CC_K_SPMV_SHUB: {
         auto* c = (const cc_spmv_args*)a;
         int64_t b = ((int64_t)c->rows + c->nnz + SPMV_IPC - 1) / SPMV_IPC;
         if (b > INT32_MAX - 1) return fail(CC_ERR_OVERFLOW, "spmv grid");
@@ -405,11 +405,19 @@ using RowB = GemvBody<32, 256, true, false>;
 using ColB = GemvBody<32, 256, false, true>;
 using BothB = GemvBody<32, 256, true, true>;
 
+// the header's tier size is the shipped build's
+static_assert(SpmvShubBody::kHubSlots == CC_SPMV_SHUB_SLOTS || CC_SHUB_SLOTS != 8192,
+              "include/ctaclust.h CC_SPMV_SHUB_SLOTS out of date");
+
+// bytes a body keeps in dynamic shared memory after its ring (kExtraSmem)
+template <class B, class = void> struct ExtraSmem { static constexpr int value = 0; };
+template <class B> struct ExtraSmem<B, decltype((void)B::kExtraSmem)> { static constexpr int value = B::kExtraSmem; };
+
 template <class Body>
 static size_t dyn_smem(int stages, bool direct = false) {
     // direct loads stage nothing: keep the ring minimal so L1 keeps the space
     // (bodies whose direct path needs a per-task buffer size it themselves)
-    return (size_t)stages * (direct ? direct_stage_bytes<Body>() : Body::kStageBytes) + 128;
+    return (size_t)stages * (direct ? direct_stage_bytes<Body>() : Body::kStageBytes) + 128 + ExtraSmem<Body>::value;
 }
 
 // Opt every instantiation of a body into large dynamic shared memory once.
@@ -471,6 +479,7 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     case CC_K_JACOBI5_HALO: s = occupancy<Jacobi5HaloBody>(device, Jacobi5HaloBody::kDefaultStages, &occ); break;
     case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, Conv2dBody<3>::kDefaultStages, &occ); break;
     case CC_K_SPMV: s = occupancy<SpmvBody>(device, SpmvBody::kDefaultStages, &occ); break;
+    case CC_K_SPMV_SHUB: s = occupancy<SpmvShubBody>(device, SpmvShubBody::kDefaultStages, &occ); break;
     case CC_K_HIST64: s = occupancy<HistBody>(device, HistBody::kDefaultStages, &occ); break;
     default: return fail(CC_ERR_INVALID_ARG, "unknown kernel %d", k);
     }
@@ -922,13 +931,19 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         }
         break;
     }
-    case CC_K_SPMV: {
+    case CC_K_SPMV: case CC_K_SPMV_SHUB: {
         auto* x = (const cc_spmv_args*)a;
         if (x->rows < 0 || x->cols < 0 || x->nnz < 0 || x->nnz > INT32_MAX) return fail(CC_ERR_INVALID_ARG, "spmv sizes");
         if (!x->row_ptr || !x->part || !x->y || (x->nnz && (!x->col || !x->val || !x->x)))
             return fail(CC_ERR_INVALID_ARG, "spmv null pointer");
         if (x->n_hot < 0 || (x->n_hot > 0 && (!x->hot || !x->xh)))
             return fail(CC_ERR_INVALID_ARG, "spmv hub-column form: n_hot %d, hot/xh required", x->n_hot);
+        if (k == CC_K_SPMV_SHUB) {
+            if (o->backend != CC_BACKEND_AGENT && o->backend != CC_BACKEND_AGENT_IDENTITY &&
+                o->backend != CC_BACKEND_AGENT_STATIC)
+                return fail(CC_ERR_UNSUPPORTED, "spmv_shub: persistent backends only (agent / identity / static)");
+            if (x->n_hot > 0 && !al16(x->xh)) return fail(CC_ERR_INVALID_ARG, "spmv_shub: xh must be 16-byte aligned");
+        }
         if (x->rows) CC_CUDA(cudaMemsetAsync(x->y, 0, sizeof(float) * x->rows, st));
         if (x->n_hot > 0) {
             k_spmv_hot_gather<<<std::min(148 * 4, (x->n_hot + 255) / 256), 256, 0, st>>>(x->x, x->hot, x->xh, x->n_hot);
@@ -936,8 +951,9 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             if (e != cudaSuccess) return cuda_fail(e, "spmv hub gather");
             if (launches) ++*launches;
         }
-        s = launch_body<SpmvBody>(c, SpmvParams{x->rows, x->nnz, x->row_ptr, x->col, x->val, x->x, x->y, x->part,
-                                                x->n_hot > 0 ? x->xh + x->n_hot : nullptr});
+        const SpmvParams sp{x->rows, x->nnz, x->row_ptr, x->col, x->val, x->x, x->y, x->part,
+                            x->n_hot > 0 ? x->xh + x->n_hot : nullptr, x->n_hot};
+        s = k == CC_K_SPMV_SHUB ? launch_body<SpmvShubBody>(c, sp) : launch_body<SpmvBody>(c, sp);
         break;
     }
     case CC_K_HIST64: {
@@ -1072,7 +1088,6 @@ extern "C" cc_status cc_spmv_inspect(const cc_spmv_args* x, int32_t max_hot, int
     const int32_t cols = x->cols;
     int32_t* deg = scratch;
     int32_t* hist = scratch + cols;
-    int32_t* ctr = hist + 65536;
     const int grid = 148 * 8;
     CC_CUDA(cudaMemsetAsync(scratch, 0, sizeof(int32_t) * ((size_t)cols + 65536 + 2), st));
     if (x->nnz) k_spmv_col_degree<<<grid, 256, 0, st>>>(x->col, x->nnz, deg);
@@ -1080,18 +1095,29 @@ extern "C" cc_status cc_spmv_inspect(const cc_spmv_args* x, int32_t max_hot, int
     std::vector<int32_t> h(65536);
     CC_CUDA(cudaMemcpyAsync(h.data(), hist, sizeof(int32_t) * 65536, cudaMemcpyDeviceToHost, st));
     CC_CUDA(cudaStreamSynchronize(st));
-    // threshold t >= 1: every column with degree > t is a hub (`above` of
-    // them, <= max_hot) and columns of degree t fill the remaining slots; t = 0:
-    // every referenced column fits (unreferenced ones are never hubs)
-    int64_t above = 0;
-    int32_t t = 65535;
-    for (; t >= 1; --t) {
-        if (above + h[t] > max_hot) break;
-        above += h[t];
-    }
-    if (t < 0) t = 0;
-    const int32_t used = (int32_t)std::min<int64_t>(above + (t >= 1 ? h[t] : 0), max_hot);
-    k_spmv_hot_assign<<<grid, 256, 0, st>>>(deg, cols, t, (int32_t)above, max_hot, ctr, hot);
+    // degree-sorted view of the histogram: G(d) = #columns of degree > d; the
+    // k-th most referenced column (k >= 1) has the degree d with
+    // G(d) < k <= G(d) + h[d].  Unreferenced columns are never hubs.
+    int64_t referenced = 0;
+    for (int32_t d = 1; d < 65536; ++d) referenced += h[d];
+    const int32_t used = (int32_t)std::min<int64_t>(referenced, max_hot);
+    const int32_t T = std::min(used, (int32_t)CC_SPMV_SHUB_SLOTS);
+    auto kth = [&](int64_t k, int64_t* above) {   // degree of the k-th, and G(that degree)
+        int64_t g = 0;
+        for (int32_t d = 65535; d >= 1; --d) {
+            if (g + h[d] >= k) { *above = g; return d; }
+            g += h[d];
+        }
+        *above = g;
+        return 1;
+    };
+    int64_t n_a = 0, g_b = 0;
+    const int32_t dA = T > 0 ? kth(T, &n_a) : 65536;
+    const int32_t dB = used > 0 ? kth(used, &g_b) : 65536;
+    const int32_t n_b = dA > dB ? (int32_t)(g_b - T) : 0;
+    int32_t* ctr = hist;                            // the histogram is on the host now: its first words count
+    CC_CUDA(cudaMemsetAsync(ctr, 0, 4 * sizeof(int32_t), st));
+    k_spmv_hot_assign<<<grid, 256, 0, st>>>(deg, cols, dA, (int32_t)n_a, T, dB, n_b, used, ctr, hot);
     if (x->nnz) k_spmv_col_encode<<<grid, 256, 0, st>>>(x->col, x->nnz, deg, col_hot);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "spmv inspect");

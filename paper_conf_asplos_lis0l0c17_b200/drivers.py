@@ -533,4 +533,6 @@ class SpmvBlock(GraphStep):
 
 
 def _launch_spmv(Am, x, y, opts, stream):
-    return _launch("spmv", Am.args(x, y), opts, stream)
+    kw = dict(opts)
+    shub = kw.pop("shub", False)              # CC_K_SPMV_SHUB: hub tier in the agents' shared memory
+    return _launch("spmv_shub" if shub else "spmv", Am.args(x, y), kw, stream)

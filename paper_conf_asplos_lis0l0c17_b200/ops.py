@@ -18,7 +18,7 @@ from . import ctaclust as cc
 DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": ("col", (1, 1)),
                  "bicg": ("col", (1, 1)), "mvt": ("col", (1, 1)), "jacobi5": ("row", (1, 1)),
                  "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1)),
-                 "jacobi5_halo": ("row", (1, 1)), "atax_fused": ("row", (1, 1))}
+                 "jacobi5_halo": ("row", (1, 1)), "atax_fused": ("row", (1, 1)), "spmv_shub": ("row", (1, 1))}
 
 # Plans of the computed orders are cached for the life of the process: a plan
 # may only be destroyed once every stream that used it has synchronized
@@ -192,9 +192,13 @@ class SpmvMatrix:
                            None if self.xh is None else self.xh.data_ptr(), self.n_hot)
 
 
-def spmv(Amat: SpmvMatrix, x, y=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+def spmv(Amat: SpmvMatrix, x, y=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None,
+         shub=False, **kw):
+    """y = A x.  shub=True: the hottest cc.SPMV_SHUB_SLOTS hub values in each
+    agent's shared memory (CC_K_SPMV_SHUB, persistent backends)."""
     y = torch.empty(Amat.rows, dtype=torch.float32, device=x.device) if y is None else y
-    _launch("spmv", Amat.args(x, y), backend, order, tile, num_clusters, _dev(x), stream, **kw)
+    _launch("spmv_shub" if shub else "spmv", Amat.args(x, y), backend, order, tile, num_clusters, _dev(x), stream,
+            **kw)
     return y
 
 

@@ -247,8 +247,89 @@ def hist():
     return out
 
 
+def _stripe_order(gx, gy, sw):
+    """USER order of column stripes sw tiles wide: v runs stripe by stripe,
+    row-major inside a stripe -- with one cluster per stripe every SM walks
+    down its own columns while all of them stay on the same band of rows"""
+    import numpy as np
+    s, by, k = np.meshgrid(np.arange(gx // sw), np.arange(gy), np.arange(sw), indexing="ij")
+    return (by * gx + s * sw + k).reshape(-1).astype(np.int32)
+
+
+def stripe():
+    """column-striped clusters (one stripe per SM, lock-step row band) vs
+    identity / ROW / default: conv 3x3 8192^2 (128 stripes of 2 tiles) and
+    Jacobi 16384^2 (128 stripes of 4 tiles)"""
+    import numpy as np
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    out = {}
+    N = 8192
+    img = synth.matrix(5, N, N, backend="torch", device="cuda")
+    o = torch.empty_like(img)
+    w = synth.uniform(6, 9).reshape(3, 3)
+    w = (w / w.astype(np.float64).sum()).astype(np.float32)
+    u3 = _stripe_order(256, 256, 2)
+    base = [("default", dict(backend="default")), ("identity", dict(backend="identity")),
+            ("agent-row", dict(backend="agent", order="row"))]
+    v3 = base + [("agent-stripe", dict(backend="agent", order="user", user_order=u3, num_clusters=128))] + \
+        [(f"static-stripe-s{st}", dict(backend="static", order="user", user_order=u3, num_clusters=128, stages=st))
+         for st in (4, 8, 12)]
+    r = B.measure(v3, lambda kw: ops.conv2d(img, w, out=o, **kw), 20, 8 * N * N, graph=True, inner=B.GRAPH_INNER)
+    out["conv3"] = r
+    print("conv3", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    del img, o
+    M = 16384
+    a = synth.matrix(4, M, M, backend="torch", device="cuda")
+    b = a.clone()
+    uj = _stripe_order(512, 512, 4)
+    vj = base + [("agent-stripe", dict(backend="agent", order="user", user_order=uj, num_clusters=128))] + \
+        [(f"static-stripe-s{st}", dict(backend="static", order="user", user_order=uj, num_clusters=128, stages=st))
+         for st in (4, 8, 12)]
+    r = B.measure(vj, lambda kw: ops.jacobi5(a, b, 2, **kw), 10, 2 * 8 * M * M, graph=True, inner=5)
+    out["jacobi"] = r
+    print("jacobi", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    return out
+
+
+def spmv_shub():
+    """hub array in each agent's shared memory (CC_K_SPMV_SHUB) vs the L1 hub
+    form and plain CSR; EXP_SHUB_HOTS lists the hub sizes (<= the build's
+    capacity)"""
+    import torch
+    from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+    rp, col = synth.rmat_csr(7, 24, 16, backend="torch", device="cuda")
+    n, nnz = rp.numel() - 1, col.numel()
+    val = synth.uniform(8, nnz, backend="torch", device="cuda")
+    x = synth.uniform(9, n, backend="torch", device="cuda")
+    y = torch.empty(n, device="cuda")
+    nbytes = 8 * nnz + 4 * (n + 1) + 8 * n
+    out = {}
+    A0 = ops.SpmvMatrix(rp, col, val, hot=16384)
+    base = [("default-l1hub16k", dict(backend="default")), ("agent-row-l1hub16k", dict(backend="agent", order="row")),
+            ("identity-l1hub16k", dict(backend="identity"))]
+    r = B.measure(base, lambda kw: ops.spmv(A0, x, y, **kw), 20, nbytes, graph=True, inner=B.GRAPH_INNER)
+    out["l1hub16k"] = r
+    print("l1hub16k", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+    del A0
+    for hot in [int(h) for h in os.environ.get("EXP_SHUB_HOTS", "16384,32768,43008").split(",")]:
+        Am = ops.SpmvMatrix(rp, col, val, hot=hot)
+        variants = [("default-l1hub", dict(backend="default")),
+                    ("shub-agent-row", dict(backend="agent", order="row", shub=True)),
+                    ("shub-identity", dict(backend="identity", shub=True)),
+                    ("shub-static-row-m1", dict(backend="static", order="row", num_clusters=148, shub=True)),
+                    ("shub-agent-row-s12", dict(backend="agent", order="row", shub=True, stages=6, batch=4))]
+        r = B.measure(variants, lambda kw: ops.spmv(Am, x, y, **kw), 20, nbytes, graph=True, inner=B.GRAPH_INNER)
+        out[f"shub{hot}"] = r
+        print(f"shub{hot}", [(v["variant"], v["ms"], v["frac_hbm"]) for v in r["rows"]], flush=True)
+        del Am
+        torch.cuda.empty_cache()
+    return out
+
+
 if __name__ == "__main__":
     what, path = sys.argv[1], sys.argv[2]
     res = {"spmv": spmv, "stencil": stencil, "tbc": tbc, "panel": panel, "conv7": conv7,
-           "spmv_control": spmv_control, "hist": hist, "spmv_persist": spmv_persist}[what]()
+           "spmv_control": spmv_control, "hist": hist, "spmv_persist": spmv_persist,
+           "stripe": stripe, "spmv_shub": spmv_shub}[what]()
     json.dump(res, open(path, "w"), indent=1)

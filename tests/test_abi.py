@@ -170,3 +170,12 @@ def test_kernel_grid():
     assert cc.kernel_grid("hist64", cc.Hist64Args(None, 0, None)) == (0, 1)
     with pytest.raises(cc.CtaclustError):
         cc.kernel_grid("hist64", cc.Hist64Args(None, 1 << 32, None))
+
+
+def test_kernel_ids_match_header():
+    """cc_kernel enum values and CC_SPMV_SHUB_SLOTS as the binding mirrors them"""
+    import re
+    h = open(HEADER).read()
+    ids = {m.group(1).lower(): int(m.group(2)) for m in re.finditer(r"\bCC_K_(\w+) = (\d+)", h)}
+    assert ids == cc.KERNELS
+    assert int(re.search(r"#define CC_SPMV_SHUB_SLOTS (\d+)", h).group(1)) == cc.SPMV_SHUB_SLOTS

@@ -11,7 +11,7 @@ import pytest
 import torch
 
 import oracle as O
-from paper_conf_asplos_lis0l0c17_b200 import ops, synth
+from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc, ops, synth
 
 pytestmark = pytest.mark.gpu
 TOL = 1e-4
@@ -463,6 +463,9 @@ def test_spmv_hub_form(hot):
         if Am.n_hot:
             rest = np.setdiff1d(np.arange(n), hubs)
             assert deg[hubs].min() >= (deg[rest].max() if rest.size else 0), name
+            dh = np.minimum(deg[hubs], 65535)
+            T = min(Am.n_hot, cc.SPMV_SHUB_SLOTS)               # the shared-memory tier: the hottest slots
+            assert T == Am.n_hot or dh[:T].min() >= dh[T:].max(), name
         enc = Am.col_kernel.cpu().numpy()
         dec = enc.copy()
         neg = enc < 0
@@ -480,6 +483,71 @@ def test_spmv_hub_form(hot):
             assert relerr(got[nz], ref[nz]) <= TOL, (name, v)
             if v["backend"] in ("default", "static"):     # deterministic schedules: the same bits
                 assert np.array_equal(got, y0.cpu().numpy()), (name, v)
+
+
+SHUB_VARIANTS = [dict(backend="agent", order="row"), dict(backend="identity"),
+                 dict(backend="static", order="row", num_clusters=740), dict(backend="static", order="row", num_clusters=3),
+                 dict(backend="agent", order="row", stages=6, batch=5), dict(backend="agent", order="row", steal=0),
+                 dict(backend="agent", order="row", l2_hint="both"), dict(backend="agent", order="col")]
+
+
+@pytest.mark.parametrize("hot", [0, 1, 7, 64, 43008])
+def test_spmv_shub(hot):
+    """CC_K_SPMV_SHUB (hub array in each agent's shared memory, one bulk copy
+    per agent): the oracle's y under every persistent schedule, including the
+    hub tail that is not a multiple of 16 bytes (n_hot = 1, 7), an all-hub
+    matrix (rmat12: every column a hub slot) and plain CSR (hot = 0); bit-exact
+    in the integer-exact mode."""
+    for name, rp, col, n in _edge_matrices():
+        val = synth.uniform(8, len(col))
+        x = synth.uniform(9, n)
+        plain = _csr_dev(rp, col, val)
+        Am = ops.SpmvMatrix(plain.row_ptr, plain.col, plain.val, hot=hot) if hot else plain
+        ref = O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), val, x)
+        vi, xi = synth.small_int(10, len(col)), synth.small_int(11, n)
+        Ai = ops.SpmvMatrix(plain.row_ptr, plain.col, dev(vi.astype(np.float32)), hot=hot) if hot else \
+            _csr_dev(rp, col, vi)
+        refi = O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), vi, xi)
+        for v in SHUB_VARIANTS:
+            y = ops.spmv(Am, dev(x), shub=True, **v)
+            torch.cuda.synchronize()
+            got = y.cpu().numpy()
+            nz = ref != 0
+            assert np.all(got[~nz] == 0), (name, v)
+            assert relerr(got[nz], ref[nz]) <= TOL, (name, v)
+            yi = ops.spmv(Ai, dev(xi), shub=True, **v)
+            torch.cuda.synchronize()
+            assert np.array_equal(yi.cpu().numpy().astype(np.float64), refi), (name, v)
+
+
+def test_spmv_shub_tiers():
+    """SHUB is for persistent agents only; with more hub slots than its
+    shared-memory tier (include/ctaclust.h CC_SPMV_SHUB_SLOTS) the colder
+    slots are read from the L1 array -- both tiers against the oracle, and
+    bit-exact in the integer-exact mode."""
+    from paper_conf_asplos_lis0l0c17_b200 import ctaclust as cc
+    rp, col = synth.rmat_csr(7, 17, 16)
+    n = len(rp) - 1
+    val, x = synth.uniform(8, len(col)), synth.uniform(9, n)
+    plain = _csr_dev(rp, col, val)
+    for b in ("default", "redirect"):
+        with pytest.raises(cc.CtaclustError):
+            ops.spmv(plain, dev(x), backend=b, shub=True)
+    ref = O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), val, x)
+    vi, xi = synth.small_int(10, len(col)), synth.small_int(11, n)
+    refi = O.spmv_csr(rp.astype(np.int32), col.astype(np.int32), vi, xi)
+    for hot in (cc.SPMV_SHUB_SLOTS - 1, cc.SPMV_SHUB_SLOTS + 3, cc.SPMV_SHUB_SLOTS + 6, 3 * cc.SPMV_SHUB_SLOTS):
+        Am = ops.SpmvMatrix(plain.row_ptr, plain.col, plain.val, hot=hot)
+        Ai = ops.SpmvMatrix(plain.row_ptr, plain.col, dev(vi.astype(np.float32)), hot=hot)
+        assert Am.n_hot == hot
+        for v in (dict(backend="agent", order="row"), dict(backend="identity"),
+                  dict(backend="static", order="row", num_clusters=296)):
+            y = ops.spmv(Am, dev(x), shub=True, **v)
+            yi = ops.spmv(Ai, dev(xi), shub=True, **v)
+            torch.cuda.synchronize()
+            nz = ref != 0
+            assert relerr(y.cpu().numpy()[nz], ref[nz]) <= TOL, (hot, v)
+            assert np.array_equal(yi.cpu().numpy().astype(np.float64), refi), (hot, v)
 
 
 def test_spmv_full_size_sampled():
@@ -503,9 +571,11 @@ def test_spmv_full_size_sampled():
     sub_val = val[idx].cpu().numpy()
     ref = O.spmv_csr(sub_rp.astype(np.int32), sub_col.astype(np.int32), sub_val, x.cpu().numpy())
     Ah = ops.SpmvMatrix(rp, col, val, hot=16384)
+    As = ops.SpmvMatrix(rp, col, val, hot=43008)
     for M, v in ((Am, dict(backend="default")), (Am, dict(backend="agent", order="row")),
                  (Am, dict(backend="identity")), (Ah, dict(backend="agent", order="row")),
-                 (Ah, dict(backend="default"))):
+                 (Ah, dict(backend="default")), (As, dict(backend="agent", order="row", shub=True)),
+                 (As, dict(backend="identity", shub=True))):
         y = ops.spmv(M, x, **v)
         torch.cuda.synchronize()
         got = y[torch.from_numpy(rows).cuda()].cpu().numpy()

@@ -176,8 +176,8 @@ WORKER = textwrap.dedent("""
         ok = bool(np.all(got[~m] == 0)) and rel(got[m], inner[m]) <= 1e-4
         info = str(rel(got[m], inner[m]))
     elif cfg.startswith("spmv"):
-        d = drivers.SpmvBlock(10, X, "cuda", hot=64 if cfg == "spmv-hot" else 0)
-        d.step(dict(backend="agent", order="row", max_agents=1))
+        d = drivers.SpmvBlock(10, X, "cuda", hot=64 if cfg in ("spmv-hot", "spmv-shub") else 0)
+        d.step(dict(backend="agent", order="row", max_agents=1, **({{"shub": True}} if cfg == "spmv-shub" else {{}})))
         torch.cuda.synchronize()
         rp, col = synth.rmat_csr(7, 10, 16)
         val, x = synth.uniform(8, len(col)), synth.uniform(9, len(rp) - 1)
@@ -205,7 +205,7 @@ def _port():
 @pytest.mark.parametrize("cfg,world", [("atax", 2), ("atax", 4), ("jacobi", 2), ("jacobi", 3), ("jacobi", 4),
                                        ("jacobi-nooverlap", 3), ("jacobi-fused", 2), ("jacobi-fused", 3),
                                        ("jacobi-k4", 2), ("jacobi-k3", 3), ("conv1", 2), ("conv3", 3), ("spmv", 2),
-                                       ("spmv", 3), ("spmv-hot", 2)])
+                                       ("spmv", 3), ("spmv-hot", 2), ("spmv-shub", 2)])
 def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     script = tmp_path / "w.py"
     script.write_text(WORKER.format(root=ROOT))
