@@ -471,37 +471,56 @@ struct Jacobi5MultiBody {
     }
 
     // one intermediate sweep S (1 <= S < K) over staged rows [S, kRows - S) and
-    // the whole staged width (pitch / 4 float4 chunks), src -> dst.  Only the
+    // the whole staged width (P / 4 float4 chunks), src -> dst.  Only the
     // region K - S columns / rows inside the box edge is needed; the extra
     // columns are computed from in-bounds neighbours (the adjacent row's ends)
     // and never read by a valid point.  Thread = (chunk, a run of rows): the
-    // three rows it needs slide down in registers.
-    template <int S>
-    __device__ __forceinline__ void sweep(const float* src, float* dst, int pitch, int32_t bx, int32_t by,
-                                          int ctid) const {
+    // three rows it needs slide down in registers.  P (the box pitch: one
+    // tile or a merged pair) is a template parameter so that the chunk / run
+    // split is compile-time; a box with no global-boundary point among those
+    // it computes (every box but the image's outer ring) takes the plain
+    // 5-point form, without jacobi_point4's per-element boundary selects.
+    template <int S, int P>
+    __device__ __forceinline__ void sweep(const float* src, float* dst, int32_t bx, int32_t by, int ctid) const {
         constexpr int H = kRows - 2 * S;
-        const int nch = pitch >> 2;
-        const int runs = kConsumers / nch;                      // row runs that fit the group
-        const int rs = (H + runs - 1) / runs;                   // rows per run (<= 8)
-        const int G = (H + rs - 1) / rs;
+        constexpr int nch = P / 4;
+        constexpr int runs = kConsumers / nch;                  // row runs that fit the group
+        constexpr int rs = (H + runs - 1) / runs;               // rows per run
+        constexpr int G = (H + rs - 1) / rs;
+        static_assert(rs <= 8, "row run length");
         if (ctid >= G * nch) return;
         const int chunk = ctid % nch, rg = ctid / nch;
         const int r0 = S + rg * rs;
-        const int r1 = r0 + rs < kRows - S ? r0 + rs : kRows - S;
-        const int gx = bx * 32 - 4 + 4 * chunk, gyb = by * 32 - K;
+        const int n = r0 + rs <= kRows - S ? rs : kRows - S - r0;
+        const int gx0 = bx * 32 - 4, gyb = by * 32 - K;
+        const int gx = gx0 + 4 * chunk;
         const float* q = src + 4 * chunk;
-        float4 up = *reinterpret_cast<const float4*>(q + (r0 - 1) * pitch);
-        float4 cur = *reinterpret_cast<const float4*>(q + r0 * pitch);
+        float4 up = *reinterpret_cast<const float4*>(q + (r0 - 1) * P);
+        float4 cur = *reinterpret_cast<const float4*>(q + r0 * P);
+        const bool interior = gyb + S >= 1 && gyb + kRows - S <= p.rows - 1 && gx0 >= 1 && gx0 + P <= p.cols - 1;
+        if (interior) {
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {
-            const int r = r0 + k;
-            if (r >= r1) break;
-            const float4 down = *reinterpret_cast<const float4*>(q + (r + 1) * pitch);
-            const float lw = q[r * pitch - 1], re = q[r * pitch + 4];
-            *reinterpret_cast<float4*>(dst + r * pitch + 4 * chunk) =
-                jacobi_point4(cur, up, down, lw, re, gyb + r, gx, p.rows, p.cols);
-            up = cur;
-            cur = down;
+            for (int k = 0; k < rs; ++k) {
+                if (k >= n) break;
+                const int r = r0 + k;
+                const float4 down = *reinterpret_cast<const float4*>(q + (r + 1) * P);
+                const float lw = q[r * P - 1], re = q[r * P + 4];
+                *reinterpret_cast<float4*>(dst + r * P + 4 * chunk) = jacobi_core4(cur, up, down, lw, re);
+                up = cur;
+                cur = down;
+            }
+        } else {
+#pragma unroll
+            for (int k = 0; k < rs; ++k) {
+                if (k >= n) break;
+                const int r = r0 + k;
+                const float4 down = *reinterpret_cast<const float4*>(q + (r + 1) * P);
+                const float lw = q[r * P - 1], re = q[r * P + 4];
+                *reinterpret_cast<float4*>(dst + r * P + 4 * chunk) =
+                    jacobi_point4(cur, up, down, lw, re, gyb + r, gx, p.rows, p.cols);
+                up = cur;
+                cur = down;
+            }
         }
     }
 
@@ -533,19 +552,29 @@ struct Jacobi5MultiBody {
         }
     }
 
+    // sweeps 1 .. K-1 on the box, ping-ponging X -> Y -> X ...
+    template <int P>
+    __device__ __forceinline__ void sweeps(float* X, float* Y, int32_t bx, int32_t by, int ctid) const {
+        sweep<1, P>(X, Y, bx, by, ctid);
+        consumer_sync<kConsumers>();
+        if constexpr (K >= 3) { sweep<2, P>(Y, X, bx, by, ctid); consumer_sync<kConsumers>(); }
+        if constexpr (K >= 4) { sweep<3, P>(X, Y, bx, by, ctid); consumer_sync<kConsumers>(); }
+    }
+
     __device__ __forceinline__ void consume_n(const Sched&, int32_t bx, int32_t by, int n, const uint8_t* stage,
                                               int ctid) {
         __shared__ __align__(16) float s_scr[kGroups][kRows * ST_COLS2];   // float4 reads in sweep K
-        const int pitch = n >= 2 ? ST_COLS2 : ST_COLS;
         float* X = reinterpret_cast<float*>(const_cast<uint8_t*>(stage));   // the group owns its slot
         float* Y = s_scr[(threadIdx.x - PRODUCER_THREADS) / kConsumers];
-        sweep<1>(X, Y, pitch, bx, by, ctid);
-        consumer_sync<kConsumers>();
-        if constexpr (K >= 3) { sweep<2>(Y, X, pitch, bx, by, ctid); consumer_sync<kConsumers>(); }
-        if constexpr (K >= 4) { sweep<3>(X, Y, pitch, bx, by, ctid); consumer_sync<kConsumers>(); }
         const float* F = (K & 1) ? X : Y;                          // holds sweep K-1
-        final_sweep(F, pitch, 0, bx, by, ctid);
-        if (n >= 2) final_sweep(F, pitch, 32, bx + 1, by, ctid);
+        if (n >= 2) {
+            sweeps<ST_COLS2>(X, Y, bx, by, ctid);
+            final_sweep(F, ST_COLS2, 0, bx, by, ctid);
+            final_sweep(F, ST_COLS2, 32, bx + 1, by, ctid);
+        } else {
+            sweeps<ST_COLS>(X, Y, bx, by, ctid);
+            final_sweep(F, ST_COLS, 0, bx, by, ctid);
+        }
         // K even: sweep K read the scratch buffer, which the group's next task
         // overwrites in its first sweep -- every thread must be done with it
         if constexpr (!(K & 1)) consumer_sync<kConsumers>();

@@ -31,6 +31,7 @@ def main():
     ap.add_argument("--warm", type=int, default=1)
     ap.add_argument("--scale", type=int, default=24)
     ap.add_argument("--hot", type=int, default=0, help="spmv: hub-column form with this many hub slots")
+    ap.add_argument("--fuse", type=int, default=1, help="jacobi: sweeps per launch (cc_jacobi5_args.fuse)")
     ap.add_argument("--persist-x", action="store_true", help="spmv: x L2-persisting (cc_l2_persist)")
     ap.add_argument("--small", action="store_true",
                     help="reduced problem (categorizer probe, P:2275): n/4 matrices, scale-18 SpMV")
@@ -70,7 +71,7 @@ def main():
         N = 4096 if a.small else 16384
         a_ = synth.matrix(4, N, N, backend="torch", device=dev)
         b_ = torch.empty_like(a_)
-        fn = lambda: ops.jacobi5(a_, b_, 1, **kw)
+        fn = lambda: ops.jacobi5(a_, b_, a.fuse, fuse=a.fuse, **kw)   # one launch of `fuse` sweeps
     elif k in ("conv3", "conv7"):
         N, R = (2048 if a.small else 8192), (1 if k == "conv3" else 3)
         img = synth.matrix(5, N, N, backend="torch", device=dev)
