@@ -509,6 +509,11 @@ def main():
         elif live and a.config != "atax":
             roof["traffic"] = live["dram_bytes_per_step"]["headline"] / max(1, roof.get("launches_per_step") or 1)
             roof["traffic_source"] = "ncu in this run (per launch, cold L2)"
+            if a.config == "spmv":
+                roof["request_roofs"] = request_roofs(live)
+                for k, m in live["headline_per_kernel"].items():
+                    if "Spmv" in k:
+                        roof["traffic"] = m.get("dram__bytes_read.sum", 0.0) + m.get("dram__bytes_write.sum", 0.0)
     if rank == 0:
         l2red, prof = l2_reductions(a.config, head)
         line = {"metric": METRIC, "value": round(value, 3), "unit": "GB/s", "n_gpus": world, "steps": a.steps,
@@ -570,6 +575,26 @@ def config_block(a, D, head, world, use_graph):
     return c
 
 
+SPMV_REQ_METRICS = ("l1tex__m_l1tex2xbar_req_cycles_active.avg.pct_of_peak_sustained_elapsed",
+                    "lts__t_tag_requests.avg.pct_of_peak_sustained_elapsed",
+                    "lts__t_tag_requests.max.pct_of_peak_sustained_elapsed")
+
+
+def request_roofs(live):
+    """SpMV: utilisation of the L1 -> L2 request port and of the L2 tag
+    lookups (average and busiest slice) by the headline SpMV kernel, from the
+    live ncu pass -- the roofs the gathers actually hit (one 32-byte sector per
+    x gather), next to the HBM roofline the line reports."""
+    for k, m in (live or {}).get("headline_per_kernel", {}).items():
+        if "Spmv" in k and all(x in m for x in SPMV_REQ_METRICS):
+            return {"kernel": k.replace("void ", ""), "unit": "% of peak sustained",
+                    "l1_to_l2_request_port": round(m[SPMV_REQ_METRICS[0]], 2),
+                    "l2_tag_lookups_avg": round(m[SPMV_REQ_METRICS[1]], 2),
+                    "l2_tag_lookups_busiest_slice": round(m[SPMV_REQ_METRICS[2]], 2),
+                    "source": "ncu in this run (scripts/ncu_step.py, one headline step)"}
+    return None
+
+
 def live_ncu(a, head, dflt_staging):
     """L2 sectors and DRAM bytes of one step of the headline schedule, default
     order and the identity control, measured in this run: scripts/ncu_step.py
@@ -583,6 +608,8 @@ def live_ncu(a, head, dflt_staging):
     if not ncu:
         return None
     metrics = "lts__t_sectors_srcunit_tex.sum,dram__bytes_read.sum,dram__bytes_write.sum"
+    if a.config == "spmv":                   # the request-side roofs of the gather-bound SpMV
+        metrics += "," + ",".join(SPMV_REQ_METRICS)
     variants = {"headline": head, "default": dict(backend="default", staging=dflt_staging),
                 "identity": identity_opts(head)}
     out = {}
@@ -608,7 +635,8 @@ def live_ncu(a, head, dflt_staging):
             except ValueError:
                 continue
             m = d["Metric Name"]
-            tot[m] = tot.get(m, 0.0) + v
+            if "pct" not in m:                   # utilisations are per kernel, not additive
+                tot[m] = tot.get(m, 0.0) + v
             k = d["Kernel Name"].split("(")[0]
             per_kernel.setdefault(k, {}).setdefault(m, 0.0)
             per_kernel[k][m] += v
@@ -682,7 +710,11 @@ def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
                 "algorithmic_bytes_per_launch": dbytes // nl,
                 "timing": "CUDA events around each kernel on the launching stream, mean over the timed steps"}
     # single-kernel configs: every launch in the step is the headline kernel
+    # (SpMV's hub form adds one tiny hub-gather launch per step, 64 KB: it is
+    # counted in the step time, not as a launch of the headline kernel)
     nl = max(1, launches // a.steps)
+    if a.config == "spmv" and D.A.n_hot > 0:
+        nl = max(1, nl - 1)
     ms_launch = ms_clu / nl
     body = {"jacobi": f"Jacobi5MultiBody<{D.fuse}>" if a.config == "jacobi" and D.fuse > 1 else "Jacobi5BodyT<false>",
             "conv3": "Conv2dBody<1>", "conv7": "Conv2dBody<3>",
