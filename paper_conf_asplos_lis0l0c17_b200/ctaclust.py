@@ -278,6 +278,7 @@ def jacobi5_args(a, b, iters, rows=None, cols=None, row_window=None, fuse=1) -> 
     lo, hi = (0, 0) if row_window is None else (int(row_window[0]), int(row_window[1]))
     args = Jacobi5Args(a.data_ptr(), b.data_ptr(), _lda(a), rows, cols, iters, ctypes.addressof(flag), lo, hi,
                        int(fuse))
+    args._keep = flag            # result_is_b points into it: it must live as long as the struct
     return args, flag
 
 
@@ -290,6 +291,7 @@ def jacobi5_halo_args(a, b, iters, sweep0=0, ll=None, up_ll=None, dn_ll=None, st
     flag = _i32(0)
     args = Jacobi5HaloArgs(a.data_ptr(), b.data_ptr(), _lda(a), a.shape[0], a.shape[1], iters, sweep0,
                            ctypes.addressof(flag), _ptr(ll), up_ll, dn_ll, _ptr(status))
+    args._keep = flag
     return args, flag
 
 
@@ -334,7 +336,9 @@ def conv2d_args(inp, out, w, rows=None, cols=None) -> tuple[Conv2dArgs, np.ndarr
     K = w.shape[0]
     rows = inp.shape[0] if rows is None else rows
     cols = inp.shape[1] if cols is None else cols
-    return Conv2dArgs(inp.data_ptr(), out.data_ptr(), _lda(inp), rows, cols, K // 2, w.ctypes.data), w
+    args = Conv2dArgs(inp.data_ptr(), out.data_ptr(), _lda(inp), rows, cols, K // 2, w.ctypes.data)
+    args._keep = w               # the filter is read from this host array at launch
+    return args, w
 
 
 class Hist64Args(ctypes.Structure):

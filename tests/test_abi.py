@@ -179,3 +179,21 @@ def test_kernel_ids_match_header():
     ids = {m.group(1).lower(): int(m.group(2)) for m in re.finditer(r"\bCC_K_(\w+) = (\d+)", h)}
     assert ids == cc.KERNELS
     assert int(re.search(r"#define CC_SPMV_SHUB_SLOTS (\d+)", h).group(1)) == cc.SPMV_SHUB_SLOTS
+
+
+def test_arg_structs_own_their_host_buffers():
+    """jacobi5_args' result_is_b flag and conv2d_args' filter are host memory
+    the library reads or writes at launch: the struct must keep them alive
+    even when the caller keeps only the struct (`jacobi5_args(...)[0]`; a
+    dropped flag was a use-after-free that crashed sharded runs)."""
+    import gc
+    import torch
+    a = torch.zeros(8, 8)
+    args = cc.jacobi5_args(a, a, 1)[0]
+    gc.collect()
+    assert ctypes.addressof(args._keep) == args.result_is_b
+    c = cc.conv2d_args(a, a, np.ones((3, 3)))[0]
+    gc.collect()
+    assert c._keep.ctypes.data == c.w
+    h = cc.jacobi5_halo_args(a, a, 1)[0]
+    assert ctypes.addressof(h._keep) == h.result_is_b

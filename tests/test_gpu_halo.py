@@ -170,7 +170,7 @@ WORKER = textwrap.dedent("""
     import oracle as O
     from paper_conf_asplos_lis0l0c17_b200 import shard, synth
     rank, world = int(sys.argv[1]), int(sys.argv[2])
-    dist.init_process_group("gloo", init_method="tcp://127.0.0.1:" + sys.argv[3], rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method="file://" + sys.argv[3], rank=rank, world_size=world)
     torch.cuda.set_device(0)
     rows, cols, T = 120, 96, 6
     u0 = synth.matrix(4, rows, cols)
@@ -195,12 +195,8 @@ def test_two_processes_ipc_one_gpu(tmp_path):
     slice; the kernel's bounded wait keeps a failure from hanging."""
     script = tmp_path / "w.py"
     script.write_text(WORKER.format(root=ROOT))
-    import socket
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = str(s.getsockname()[1])
-    s.close()
-    procs = [subprocess.Popen([sys.executable, str(script), str(r), "2", port], stdout=subprocess.PIPE,
+    store = str(tmp_path / "store")            # file rendezvous: no port to race for
+    procs = [subprocess.Popen([sys.executable, str(script), str(r), "2", store], stdout=subprocess.PIPE,
                               stderr=subprocess.STDOUT, text=True) for r in range(2)]
     outs = []
     for p in procs:

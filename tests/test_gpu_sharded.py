@@ -121,7 +121,7 @@ WORKER = textwrap.dedent("""
     import oracle as O
     from paper_conf_asplos_lis0l0c17_b200 import drivers, shard, synth
     rank, world, cfg = int(sys.argv[1]), int(sys.argv[2]), sys.argv[4]
-    dist.init_process_group("gloo", init_method="tcp://127.0.0.1:" + sys.argv[3], rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method="file://" + sys.argv[3], rank=rank, world_size=world)
     torch.cuda.set_device(0)
     X = drivers.make_exchange("torch", world, rank, 0)
     def rel(got, ref):
@@ -209,8 +209,8 @@ def _port():
 def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     script = tmp_path / "w.py"
     script.write_text(WORKER.format(root=ROOT))
-    port = _port()
-    procs = [subprocess.Popen([sys.executable, "-X", "faulthandler", str(script), str(r), str(world), port, cfg],
+    store = str(tmp_path / "store")            # file rendezvous: no port to race for
+    procs = [subprocess.Popen([sys.executable, "-X", "faulthandler", str(script), str(r), str(world), store, cfg],
                               stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True) for r in range(world)]
     outs = []
     for p in procs:
@@ -220,7 +220,10 @@ def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
             p.kill()
             outs.append(p.communicate()[0])
     res = [ln for o in outs for ln in o.splitlines() if ln.startswith("RESULT")]
-    assert len(res) == world, (outs, [p.returncode for p in procs])
+    if len(res) != world:                       # the whole of every rank's output (faulthandler stacks)
+        for r, o in enumerate(outs):
+            print(f"---- rank {r} (exit {procs[r].returncode}) ----\n{o}")
+    assert len(res) == world, [p.returncode for p in procs]
     assert all(ln.split()[2] == "True" for ln in res), res
 
 
