@@ -52,6 +52,13 @@ def main(groups):
                             backend=b, order="col", num_clusters=148 if b == "static" else 0)
             torch.cuda.synchronize()
             check(f"bicg {b}", np.concatenate([q.cpu(), s.cpu()]), np.concatenate([q_ref, s_ref]))
+        x = synth.uniform(10, n)
+        tmp_ref, y_ref = O.atax(A, x)
+        for b in ("agent", "identity", "static"):
+            tmp, y = ops.atax_fused(torch.from_numpy(A).to(dev), torch.from_numpy(x).to(dev), backend=b,
+                                    order="row", num_clusters=148 if b == "static" else 0)
+            torch.cuda.synchronize()
+            check(f"atax one-pass {b}", np.concatenate([tmp.cpu(), y.cpu()]), np.concatenate([tmp_ref, y_ref]))
     if "stencil" in groups:
         u0 = synth.matrix(4, 70, 100)
         for b in ("agent", "identity", "static", "default"):
@@ -59,6 +66,13 @@ def main(groups):
             out = ops.jacobi5(a, torch.zeros_like(a), 3, backend=b, order="row", num_clusters=148 if b == "static" else 0)
             torch.cuda.synchronize()
             check(f"jacobi {b}", out.cpu().numpy(), O.jacobi5_f32(u0, 3), exact=True)
+        for K in (2, 3, 4):                      # fused sweeps (Jacobi5MultiBody<K>)
+            for b in ("agent", "static"):
+                a = torch.from_numpy(u0).to(dev)
+                out = ops.jacobi5(a, torch.zeros_like(a), 2 * K, fuse=K, backend=b, order="row",
+                                  num_clusters=148 if b == "static" else 0)
+                torch.cuda.synchronize()
+                check(f"jacobi fuse={K} {b}", out.cpu().numpy(), O.jacobi5_f32(u0, 2 * K), exact=True)
         for R in (1, 3):
             K = 2 * R + 1
             w = synth.uniform(6, K * K).reshape(K, K)
@@ -108,6 +122,16 @@ def main(groups):
                 y = ops.spmv(Am, t(x), backend=b, order="row")
                 torch.cuda.synchronize()
                 check(f"spmv {b} hot={hot}", y.cpu().numpy(), ref)
+            for b in ("agent", "static"):           # shared-memory hub tier (CC_K_SPMV_SHUB)
+                y = ops.spmv(Am, t(x), backend=b, order="row", shub=True, num_clusters=148 if b == "static" else 0)
+                torch.cuda.synchronize()
+                check(f"spmv shub {b} hot={hot}", y.cpu().numpy(), ref)
+        rp, col = synth.rmat_csr(7, 14, 4)         # both tiers: more hubs than the shared tier holds
+        val, x = synth.uniform(8, len(col)), synth.uniform(9, len(rp) - 1)
+        Am = ops.SpmvMatrix(t(rp.astype(np.int32)), t(col.astype(np.int32)), t(val), hot=cc.SPMV_SHUB_SLOTS + 7)
+        y = ops.spmv(Am, t(x), backend="agent", order="row", shub=True)
+        torch.cuda.synchronize()
+        check("spmv shub two tiers", y.cpu().numpy(), O.spmv_csr(rp, col, val, x))
     print("ALL OK" if ok else "SOME FAILED", flush=True)
     return 0 if ok else 1
 
