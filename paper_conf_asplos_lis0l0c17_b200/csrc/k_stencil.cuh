@@ -449,7 +449,10 @@ struct Jacobi5MultiBody {
     static constexpr int kDirectStageBytes = kStageBytes;     // always TMA-staged
     static constexpr int kDefaultStages = 4;
     static constexpr int kDefaultBatch = 4;
-    static constexpr int kMinAgents = 4;
+    // three agents per SM: the ring (4 x ~11 KB) and the intermediate-sweep
+    // scratch (2 x ~11 KB) fit three per SM anyway, and 3 (not 4) in
+    // __launch_bounds__ lets a thread keep 72 registers instead of 56
+    static constexpr int kMinAgents = 3;
     static constexpr int kGroups = 2;
     using Params = JacobiParams;
     const JacobiParams& p;
