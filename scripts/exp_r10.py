@@ -215,7 +215,8 @@ def conv7():
     w = (w / w.astype(np.float64).sum()).astype(np.float32)
     variants = [("default", dict(backend="default")), ("identity", dict(backend="identity")),
                 ("agent-row", dict(backend="agent", order="row"))] + \
-               [(f"static-row-m{m}", dict(backend="static", order="row", num_clusters=m * 148)) for m in (3, 4, 6, 7, 8)]
+               [(f"static-row-m{m}", dict(backend="static", order="row", num_clusters=m * 148))
+                for m in [int(v) for v in os.environ.get("EXP_C7_M", "3,4,6,7,8").split(",")]]
     r = B.measure(variants, lambda kw: ops.conv2d(img, w, out=o, **kw), 20, 8 * N * N, graph=True, inner=B.GRAPH_INNER)
     fl = 2 * 49 * (N - 6) ** 2
     for v in r["rows"]:
