@@ -207,7 +207,8 @@ typedef enum {
     CC_K_HIST64 = 8,   /* cc_hist64_args   (S§8(f)3, the paper's HST)               */
     CC_K_JACOBI5_HALO = 9, /* cc_jacobi5_halo_args (S§8(f)4: sharded sweep, fused peer halo) */
     CC_K_ATAX_FUSED = 10, /* cc_atax_args: one-pass ATAX (both PolyBench kernels per row) */
-    CC_K_SPMV_SHUB = 11   /* cc_spmv_args: SpMV with the hub array in each agent's shared memory */
+    CC_K_SPMV_SHUB = 11,  /* cc_spmv_args: SpMV with the hub array in each agent's shared memory */
+    CC_K_JACOBI5_WAVE = 12 /* cc_jacobi5_args: fused sweeps as strip wavefronts carried across tiles (R34) */
 } cc_kernel;
 
 /* CC_K_CENSUS: no data. */
@@ -257,6 +258,26 @@ typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t ite
                                     single sweeps; iters % fuse remaining sweeps run one per launch.
                                     Not with a row window (UNSUPPORTED). */
                } cc_jacobi5_args;
+
+/* CC_K_JACOBI5_WAVE -- the same sweeps (CC_K_JACOBI5's arithmetic, bit-identical,
+ * `iters` sweeps ping-ponging a -> b -> a, *result_is_b as there) run K = fuse
+ * (1..8; 0 = 1) at a time by warp agents streaming column strips
+ * (reading R34, §4.2 P:1793 / Listing 5).  Logical CTA
+ * (bx, by) = output rows [64 by, 64 by + 64) x columns [WS bx, WS bx + WS),
+ * WS = 120 for K <= 4 and 112 for K = 5..8; grid ceil(cols/WS) x ceil(rows/64).
+ * One launch runs K sweeps: a warp ingests its tile's input rows from 64 by - K
+ * to 64 by + 64 + K and keeps every intermediate sweep's last two rows in
+ * registers; when its next logical CTA is the tile directly below (the next
+ * position of a COL-ordered cluster) it carries them over instead of re-reading
+ * and re-sweeping the 2K-row overlap.  The tail launch runs iters % K sweeps
+ * on the same grid.  Backends: DEFAULT (one warp per logical CTA, hardware
+ * order), AGENT, AGENT_IDENTITY (agents = worker warps, 24 (fuse <= 3), 20 (4) or 15
+ * in one CTA per SM beside a scheduler warp that pops their logical CTAs; max_agents / active_agents
+ * count workers per SM; batch > 0 = tiles per queue claim, 0 = chunked
+ * claims: 3/4 of a queue in one contiguous chunk per agent, the rest tile by
+ * tile), AGENT_STATIC (worker i runs cluster i: ceil(M / workers) CTAs).  No row
+ * window (UNSUPPORTED); TBCLUSTER / REDIRECT UNSUPPORTED; fuse outside [0, 8]
+ * INVALID_ARG. */
 
 /* CC_K_JACOBI5_HALO -- S§8(f)4: one rank's slab of the slab-sharded Jacobi
  * (S§8(e), config 3) with the per-sweep halo exchange fused into the sweep

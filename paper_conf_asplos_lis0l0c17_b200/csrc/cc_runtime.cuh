@@ -44,7 +44,7 @@ struct Sched {
     const int32_t* user;          // USER order table: v -> lin (device)
     const int32_t* rank_of_smid;  // %smid -> dense SM rank or -1 (device)
     int32_t smid_span;
-    int32_t* ws;                  // workspace: agent_ctr[M+1] | head[M] | gq | done | claimed
+    int32_t* ws;                  // workspace: agent_ctr[M+1] | head[M] | gq | done | claimed | chunk[M]
     int32_t mode;                 // MODE_AGENT / MODE_IDENTITY / MODE_STATIC
     int32_t active_agents;
     int32_t throttle;             // active_agents < agents launched per SM
@@ -64,7 +64,9 @@ __device__ __forceinline__ int32_t* ws_head(const Sched& s) { return s.ws + s.g.
 __device__ __forceinline__ int32_t* ws_gq(const Sched& s) { return s.ws + 2 * s.g.M + 1; }
 __device__ __forceinline__ int32_t* ws_done(const Sched& s) { return s.ws + 2 * s.g.M + 2; }
 __device__ __forceinline__ int32_t* ws_claimed(const Sched& s) { return s.ws + 2 * s.g.M + 3; }
-inline size_t ws_ints(int32_t M) { return (size_t)(2 * M + 4); }
+// chunk counters per cluster (warp-agent kernels, k_jwave.cuh), after the rest
+__device__ __forceinline__ int32_t* ws_chunk(const Sched& s) { return s.ws + 2 * s.g.M + 4; }
+inline size_t ws_ints(int32_t M) { return (size_t)(3 * M + 4); }
 
 // ---------------------------------------------------------------------------
 // PTX helpers

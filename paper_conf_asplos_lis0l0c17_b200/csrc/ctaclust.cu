@@ -23,6 +23,7 @@
 #include "k_spmv.cuh"
 #include "k_microbench.cuh"
 #include "k_hist.cuh"
+#include "k_jwave.cuh"
 #include "k_stencil.cuh"
 #include "k_tbcluster.cuh"
 
@@ -368,6 +369,12 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
         *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK;
     }
     case CC_K_JACOBI5_HALO: { auto* c = (const cc_jacobi5_halo_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
+    case CC_K_JACOBI5_WAVE: {
+        auto* c = (const cc_jacobi5_args*)a;
+        if (c->fuse < 0 || c->fuse > 8) return fail(CC_ERR_INVALID_ARG, "jacobi5_wave: fuse %d outside [0, 8]", c->fuse);
+        const int K = c->fuse < 1 ? 1 : c->fuse;
+        *gx = cdiv(c->cols, jw_strip_cols(jw_halo_chunks(K))); *gy = cdiv(c->rows, JW_ROWS); return CC_OK;
+    }
     case CC_K_CONV2D: { auto* c = (const cc_conv2d_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
     case CC_K_SPMV: case CC_K_SPMV_SHUB: {
         auto* c = (const cc_spmv_args*)a;
@@ -465,6 +472,8 @@ static cc_status occupancy(int device, int stages, int* occ, bool direct = false
     return CC_OK;
 }
 
+template <int K, int HL> static cc_status jw_occupancy(int device, int* warps);
+
 extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     if (!out) return fail(CC_ERR_INVALID_ARG, "null out");
     int occ = 0;
@@ -477,6 +486,7 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     case CC_K_BICG: case CC_K_MVT: s = occupancy<BothB>(device, BothB::kDefaultStages, &occ); break;
     case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, Jacobi5Body::kDefaultStages, &occ); break;
     case CC_K_JACOBI5_HALO: s = occupancy<Jacobi5HaloBody>(device, Jacobi5HaloBody::kDefaultStages, &occ); break;
+    case CC_K_JACOBI5_WAVE: s = jw_occupancy<4, 1>(device, &occ); break;
     case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, Conv2dBody<3>::kDefaultStages, &occ); break;
     case CC_K_SPMV: s = occupancy<SpmvBody>(device, SpmvBody::kDefaultStages, &occ); break;
     case CC_K_SPMV_SHUB: s = occupancy<SpmvShubBody>(device, SpmvShubBody::kDefaultStages, &occ); break;
@@ -603,6 +613,128 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
     if (c.nl) ++*c.nl;
     return CC_OK;
+}
+
+// ---- CC_K_JACOBI5_WAVE: warp agents (k_jwave.cuh) -------------------------
+// opt the kernel into its dynamic shared memory (once per device)
+template <int K, int HL, int KIND>
+static cc_status jw_prepare(int device) {
+    static std::mutex mu;
+    static bool done[64] = {false};
+    if (device < 0 || device >= 64) return fail(CC_ERR_INVALID_ARG, "device");
+    std::lock_guard<std::mutex> lk(mu);
+    if (!done[device]) {
+        CC_CUDA(cudaFuncSetAttribute(k_jwave<K, HL, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, jw_smem(K, KIND)));
+        done[device] = true;
+    }
+    return CC_OK;
+}
+
+// worker warps per SM the hardware keeps resident
+template <int K, int HL>
+static cc_status jw_occupancy(int device, int* warps) {
+    static std::mutex mu;
+    static int cache[64] = {};
+    if (device < 0 || device >= 64) return fail(CC_ERR_INVALID_ARG, "device");
+    std::lock_guard<std::mutex> lk(mu);
+    if (!cache[device]) {
+        int prev = 0, n = 0;
+        CC_CUDA(cudaGetDevice(&prev));
+        CC_CUDA(cudaSetDevice(device));
+        cc_status st = jw_prepare<K, HL, JW_DYNAMIC>(device);
+        if (st == CC_OK)
+            CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_jwave<K, HL, JW_DYNAMIC>,
+                                                                  jw_threads(K, JW_DYNAMIC), jw_smem(K, JW_DYNAMIC)));
+        CC_CUDA(cudaSetDevice(prev));
+        if (st != CC_OK) return st;
+        cache[device] = n > 0 ? n * jw_workers(K, JW_DYNAMIC) : -1;
+    }
+    *warps = cache[device];
+    if (*warps < 0) return fail(CC_ERR_UNSUPPORTED, "jacobi5_wave: no resident CTA");
+    return CC_OK;
+}
+
+template <int K, int HL>
+static cc_status jw_launch_k(const LaunchCtx& c, const JWaveParams& prm) {
+    const Grid& g = c.p->g;
+    if (g.V == 0) return CC_OK;
+    const cc_launch_opts& o = *c.o;
+    Sched s{};
+    s.g = g;
+    s.user = c.p->d_user;
+    s.rank_of_smid = c.p->facts->d_rank;
+    s.smid_span = c.p->facts->smid_span;
+    s.ws = c.p->d_ws;
+    s.steal = o.steal;
+    s.batch = o.batch > 0 ? o.batch : JW_BATCH;
+    s.stages = 1;
+    s.census = o.d_census;
+    s.exec_sm = o.d_exec_sm;
+    s.map = o.d_map;
+    switch (o.backend) {
+    case CC_BACKEND_DEFAULT:                       // hardware order: warp w of the grid = logical CTA w
+        CC_TRY(jw_prepare<K, HL, JW_ONESHOT>(c.p->device));
+        CC_TRY(set_carveout(k_jwave<K, HL, JW_ONESHOT>, o.carveout));
+        s.map = nullptr;
+        k_jwave<K, HL, JW_ONESHOT><<<cdiv(g.V, jw_workers(K, JW_ONESHOT)), jw_threads(K, JW_ONESHOT),
+                                     jw_smem(K, JW_ONESHOT), c.st>>>(s, prm);
+        break;
+    case CC_BACKEND_AGENT:
+    case CC_BACKEND_AGENT_IDENTITY: {
+        int occ = 0;
+        CC_TRY(set_carveout(k_jwave<K, HL, JW_DYNAMIC>, o.carveout));
+        CC_TRY(jw_occupancy<K, HL>(c.p->device, &occ));
+        const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
+        constexpr int nw = jw_workers(K, JW_DYNAMIC);
+        const int ctas = (maxa + nw - 1) / nw;                         // per SM (workers + a scheduler each)
+        const int launched = ctas * nw;
+        s.active_agents = o.active_agents > 0 ? std::min(o.active_agents, launched) : launched;
+        s.throttle = s.active_agents < launched;
+        s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
+        WsLease lease{c.p, c.st};
+        CC_TRY(lease.acquire());
+        k_jwave<K, HL, JW_DYNAMIC><<<c.p->facts->num_sms * ctas, jw_threads(K, JW_DYNAMIC), jw_smem(K, JW_DYNAMIC),
+                                     c.st>>>(s, prm);
+        if (cudaPeekAtLastError() == cudaSuccess) CC_TRY(lease.release());
+        break;
+    }
+    case CC_BACKEND_AGENT_STATIC:                  // worker warp i runs cluster i (Eq. 7 order)
+        CC_TRY(jw_prepare<K, HL, JW_STATIC>(c.p->device));
+        CC_TRY(set_carveout(k_jwave<K, HL, JW_STATIC>, o.carveout));
+        s.active_agents = 1;
+        s.steal = 0;
+        s.mode = MODE_STATIC;
+        k_jwave<K, HL, JW_STATIC><<<cdiv(g.M, jw_workers(K, JW_STATIC)), jw_threads(K, JW_STATIC), jw_smem(K, JW_STATIC),
+                                    c.st>>>(s, prm);
+        break;
+    default:
+        return fail(CC_ERR_UNSUPPORTED, "backend %d not available for jacobi5_wave", o.backend);
+    }
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
+    if (c.nl) ++*c.nl;
+    return CC_OK;
+}
+
+template <int HL>
+static cc_status jw_launch(const LaunchCtx& c, const JWaveParams& prm, int K) {
+    switch (K) {
+    case 1: return jw_launch_k<1, HL>(c, prm);
+    case 2: return jw_launch_k<2, HL>(c, prm);
+    case 3: return jw_launch_k<3, HL>(c, prm);
+    case 4: return jw_launch_k<4, HL>(c, prm);
+    default: break;
+    }
+    if constexpr (HL == 2) {
+        switch (K) {
+        case 5: return jw_launch_k<5, 2>(c, prm);
+        case 6: return jw_launch_k<6, 2>(c, prm);
+        case 7: return jw_launch_k<7, 2>(c, prm);
+        case 8: return jw_launch_k<8, 2>(c, prm);
+        default: break;
+        }
+    }
+    return fail(CC_ERR_INVALID_ARG, "jacobi5_wave: %d sweeps per launch with %d halo chunks", K, HL);
 }
 
 // ---- thread-block-cluster backend (conv2d) --------------------------------
@@ -861,6 +993,28 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
             s = launch_body<Jacobi5Body>(c, jp);
             std::swap(src, dst);
             ++launches_done;
+        }
+        if (x->result_is_b) *x->result_is_b = (launches_done & 1) ? 1 : 0;
+        break;
+    }
+    case CC_K_JACOBI5_WAVE: {
+        auto* x = (const cc_jacobi5_args*)a;
+        CC_TRY(check_mat(x->a, x->ld, x->rows, x->cols));
+        CC_TRY(check_mat(x->b, x->ld, x->rows, x->cols));
+        if (x->iters < 0) return fail(CC_ERR_INVALID_ARG, "iters < 0");
+        if (x->row_lo != 0 || x->row_hi != 0) return fail(CC_ERR_UNSUPPORTED, "jacobi5_wave: row window");
+        const int K = x->fuse < 1 ? 1 : x->fuse;                  // grid check above bounds it by 8
+        const int hl = jw_halo_chunks(K);
+        float* src = x->a;
+        float* dst = x->b;
+        int launches_done = 0;
+        for (int it = 0; it < x->iters && s == CC_OK;) {
+            const int k = x->iters - it >= K ? K : x->iters - it;  // the tail runs fewer sweeps, same strips
+            const JWaveParams jp{src, dst, x->ld, x->rows, x->cols};
+            s = hl == 1 ? jw_launch<1>(c, jp, k) : jw_launch<2>(c, jp, k);
+            std::swap(src, dst);
+            ++launches_done;
+            it += k;
         }
         if (x->result_is_b) *x->result_is_b = (launches_done & 1) ? 1 : 0;
         break;

@@ -26,7 +26,8 @@ BACKENDS = {"default": 0, "agent": 1, "tbcluster": 2, "identity": 3, "redirect":
 K_CENSUS, K_MATVEC, K_ATAX, K_BICG, K_MVT, K_JACOBI5, K_CONV2D, K_SPMV = range(8)
 STAGINGS = {"default": 0, "tma": 1, "l1": 2, "direct": 3}
 KERNELS = {"census": 0, "matvec": 1, "atax": 2, "bicg": 3, "mvt": 4, "jacobi5": 5, "conv2d": 6, "spmv": 7,
-           "hist64": 8, "jacobi5_halo": 9, "atax_fused": 10, "spmv_shub": 11}
+           "hist64": 8, "jacobi5_halo": 9, "atax_fused": 10, "spmv_shub": 11,
+           "jacobi5_wave": 12}
 SPMV_SHUB_SLOTS = 8192     # include/ctaclust.h CC_SPMV_SHUB_SLOTS (shared-memory hub tier)
 STATUS = {0: "CC_OK", -1: "CC_ERR_INVALID_ARG", -2: "CC_ERR_OVERFLOW", -3: "CC_ERR_NOT_PERMUTATION",
           -4: "CC_ERR_CUDA", -5: "CC_ERR_NCCL", -6: "CC_ERR_UNSUPPORTED", -7: "CC_ERR_NO_DEVICE",
@@ -271,7 +272,7 @@ def mvt_args(A, y1, y2, x1, x2, m=None, n=None) -> MvtArgs:
 
 def jacobi5_args(a, b, iters, rows=None, cols=None, row_window=None, fuse=1) -> tuple[Jacobi5Args, ctypes.c_int32]:
     """`row_window` = (row_lo, row_hi): write only output rows [row_lo, row_hi).
-    `fuse`: sweeps per launch (1-4)."""
+    `fuse`: sweeps per launch (1-4; 1-8 for jacobi5_wave)."""
     flag = _i32(0)
     rows = a.shape[0] if rows is None else rows
     cols = a.shape[1] if cols is None else cols

@@ -18,7 +18,8 @@ from . import ctaclust as cc
 DEFAULT_ORDER = {"census": ("row", (1, 1)), "matvec": ("row", (1, 1)), "atax": ("col", (1, 1)),
                  "bicg": ("col", (1, 1)), "mvt": ("col", (1, 1)), "jacobi5": ("row", (1, 1)),
                  "conv2d": ("row", (1, 1)), "spmv": ("row", (1, 1)), "hist64": ("row", (1, 1)),
-                 "jacobi5_halo": ("row", (1, 1)), "atax_fused": ("row", (1, 1)), "spmv_shub": ("row", (1, 1))}
+                 "jacobi5_halo": ("row", (1, 1)), "atax_fused": ("row", (1, 1)), "spmv_shub": ("row", (1, 1)),
+                 "jacobi5_wave": ("col", (1, 1))}
 
 # Plans of the computed orders are cached for the life of the process: a plan
 # may only be destroyed once every stream that used it has synchronized
@@ -136,6 +137,16 @@ def jacobi5(a, b, iters, backend="agent", order=None, tile=None, num_clusters=0,
     `fuse` = sweeps per launch (1-4, bit-identical)."""
     args, flag = cc.jacobi5_args(a, b, iters, row_window=row_window, fuse=fuse)
     _launch("jacobi5", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
+    return b if flag.value else a
+
+
+def jacobi5_wave(a, b, iters, fuse=4, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+    """`iters` sweeps, `fuse` (1-8) per launch, by warp agents streaming column
+    strips (CC_K_JACOBI5_WAVE, reading R34); COL clusters let an agent carry
+    its sweep levels from one tile to the one below.  Bit-identical to
+    jacobi5; returns the buffer holding the result."""
+    args, flag = cc.jacobi5_args(a, b, iters, fuse=fuse)
+    _launch("jacobi5_wave", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
     return b if flag.value else a
 
 

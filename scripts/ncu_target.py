@@ -3,7 +3,7 @@
 NVTX-free marker: the variant runs `--reps` launches after `--warm` warm-ups).
 
     python scripts/ncu_target.py --kernel bicg --backend agent --order col [--reps 2]
-Kernels: matvec atax bicg mvt jacobi conv3 conv7 spmv.  Sizes are the BASELINE
+Kernels: matvec atax bicg mvt jacobi jwave conv3 conv7 spmv.  Sizes are the BASELINE
 configs (jacobi: one sweep of 16384^2).
 """
 import argparse
@@ -72,6 +72,12 @@ def main():
         a_ = synth.matrix(4, N, N, backend="torch", device=dev)
         b_ = torch.empty_like(a_)
         fn = lambda: ops.jacobi5(a_, b_, a.fuse, fuse=a.fuse, **kw)   # one launch of `fuse` sweeps
+    elif k == "jwave":
+        N = 4096 if a.small else 16384
+        a_ = synth.matrix(4, N, N, backend="torch", device=dev)
+        b_ = torch.empty_like(a_)
+        kw.pop("stages"); kw.pop("staging")
+        fn = lambda: ops.jacobi5_wave(a_, b_, a.fuse, fuse=a.fuse, **kw)   # one launch of `fuse` sweeps
     elif k in ("conv3", "conv7"):
         N, R = (2048 if a.small else 8192), (1 if k == "conv3" else 3)
         img = synth.matrix(5, N, N, backend="torch", device=dev)

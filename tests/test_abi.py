@@ -163,6 +163,13 @@ def test_kernel_grid():
     assert cc.kernel_grid("atax", cc.AtaxArgs(None, 1004, 1001, 1001)) == (4, 32)
     assert cc.kernel_grid("jacobi5", cc.Jacobi5Args(None, None, 16384, 16384, 16384, 1)) == (512, 512)
     assert cc.kernel_grid("conv2d", cc.Conv2dArgs(None, None, 8192, 8192, 8192, 3)) == (256, 256)
+    # jacobi5_wave (R34): 64-row tiles, 120-column strips for fuse <= 4, 112 for 5..8
+    J = cc.Jacobi5Args
+    assert cc.kernel_grid("jacobi5_wave", J(None, None, 16384, 16384, 16384, 100, None, 0, 0, 4)) == (137, 256)
+    assert cc.kernel_grid("jacobi5_wave", J(None, None, 16384, 16384, 16384, 100, None, 0, 0, 8)) == (147, 256)
+    assert cc.kernel_grid("jacobi5_wave", J(None, None, 128, 65, 120, 1, None, 0, 0, 0)) == (1, 2)
+    with pytest.raises(cc.CtaclustError):
+        cc.kernel_grid("jacobi5_wave", J(None, None, 128, 64, 64, 1, None, 0, 0, 9))
     a = cc.SpmvArgs(1 << 24, 1 << 24, 1 << 28)
     assert cc.kernel_grid("spmv", a) == (((1 << 24) + (1 << 28) + 4095) // 4096, 1)
     assert cc.kernel_grid("hist64", cc.Hist64Args(None, 1 << 30, None)) == (32768, 1)
