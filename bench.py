@@ -44,7 +44,7 @@ NSM = 148
 # DESIGN.md §10), overridable from the command line
 HEADLINE = {
     "atax": dict(backend="agent", order="col"),
-    "jacobi": dict(backend="agent", order="row"),
+    "jacobi": dict(backend="agent", order="col"),      # wave kernel (R34); the tile-fused one: ROW
     "conv3": dict(backend="agent", order="row"),
     "conv7": dict(backend="static", order="row", num_clusters=7 * NSM),
     "spmv": dict(backend="agent", order="row"),
@@ -75,7 +75,11 @@ def parse():
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--staging", default="default", choices=["default", "tma", "direct", "l1"])
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
-    ap.add_argument("--fuse", type=int, default=3, help="jacobi: sweeps per launch, 1-4 (R32; 3 measured best)")
+    ap.add_argument("--fuse", type=int, default=0,
+                    help="jacobi: sweeps per launch (0: 8 for the wave kernel, 3 for the tile-fused one)")
+    ap.add_argument("--jkernel", choices=("wave", "tile"), default="wave",
+                    help="jacobi: strip wavefronts carried across tiles (CC_K_JACOBI5_WAVE, R34) or tile-fused "
+                         "sweeps (CC_K_JACOBI5, R32)")
     ap.add_argument("--halo", default="exchange", choices=["exchange", "fused"],
                     help="jacobi N > 1: NCCL halo exchange per sweep, or the fused peer-memory LL halo")
     ap.add_argument("--no-graph", action="store_true", help="eager launches instead of one CUDA graph per step")
@@ -101,6 +105,11 @@ def peaks():
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
     except Exception:
         return None
+
+
+def jacobi_fuse(a):
+    f = getattr(a, "fuse", 0) or 0
+    return f if f > 0 else (8 if getattr(a, "jkernel", "tile") == "wave" else 3)
 
 
 def sizes(a):
@@ -342,7 +351,7 @@ def build_driver(a, X, dev):
         return drivers.AtaxFamily(sz["n"], X, dev)
     if a.config == "jacobi":
         return drivers.JacobiSlab(sz["side"], sz["side"], sz["iters"], X, dev, overlap=not a.no_overlap,
-                                  halo=a.halo, fuse=a.fuse)
+                                  halo=a.halo, fuse=jacobi_fuse(a), kernel=getattr(a, "jkernel", "tile"))
     if a.config in ("conv3", "conv7"):
         return drivers.ConvSlab(sz["side"], sz["side"], sz["R"], X, dev)
     return drivers.SpmvBlock(sz["scale"], X, dev, hot=a.hot)
@@ -380,6 +389,8 @@ def main():
             head.pop("num_clusters", None)
         if a.backend not in ("agent", "identity", "static"):
             head.pop("shub", None)                 # the shared-memory hub tier needs persistent agents
+    if a.config == "jacobi" and a.jkernel == "tile" and not a.order:
+        head["order"] = "row"
     if a.order:
         head["order"] = a.order
     for k, v in (("active_agents", a.active_agents), ("stages", a.stages), ("batch", a.batch)):
@@ -562,7 +573,11 @@ def config_block(a, D, head, world, use_graph):
                  atax="one pass (CC_K_ATAX_FUSED)" if D.fused_atax else "two passes",
                  l2="inputs (1 GiB) larger than L2 (126 MB); no flush")
     elif a.config == "jacobi":
-        c.update(rows=D.rows, cols=D.cols, iters=D.iters, tile="32x32", sweeps_per_launch=D.fuse,
+        wave = D.kname == "jacobi5_wave"
+        c.update(rows=D.rows, cols=D.cols, iters=D.iters, sweeps_per_launch=D.fuse,
+                 kernel="CC_K_JACOBI5_WAVE (strip wavefronts, R34)" if wave else "CC_K_JACOBI5 (tile-fused, R32)",
+                 tile="64 rows x 120/112-column strips" if wave else "32x32",
+                 launches=[list(c_) for c_ in D.calls()] if wave and D.x.world == 1 else None,
                  bytes="one read + one write of the field per launch (per sweep when unfused)",
                  overlap=getattr(D, "overlap", False), halo="fused LL (peer memory)" if D.fused else "exchange",
                  l2="2 x 1 GiB ping-pong buffers, larger than L2; no flush")
@@ -616,7 +631,8 @@ def live_ncu(a, head, dflt_staging):
     for name, opts in variants.items():
         cmd = [ncu, "--profile-from-start", "off", "--metrics", metrics, "--cache-control", "all",
                "--clock-control", "none", "--csv", sys.executable, os.path.join(ROOT, "scripts", "ncu_step.py"),
-               "--config", a.config, "--opts", json.dumps(opts), "--hot", str(a.hot), "--fuse", str(a.fuse)]
+               "--config", a.config, "--opts", json.dumps(opts), "--hot", str(a.hot), "--fuse", str(jacobi_fuse(a)),
+               "--jkernel", a.jkernel]
         if a.n:
             cmd += ["--size", str(a.n)]
         try:
@@ -716,11 +732,16 @@ def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
     if a.config == "spmv" and D.A.n_hot > 0:
         nl = max(1, nl - 1)
     ms_launch = ms_clu / nl
+    if a.config == "jacobi" and D.kname == "jacobi5_wave":
+        kind = {"agent": 0, "identity": 0, "static": 1, "default": 2}.get(head.get("backend"), 0)
+        jk = f"k_jwave<{D.fuse}, {1 if D.fuse <= 4 else 2}, {kind}>"
     body = {"jacobi": f"Jacobi5MultiBody<{D.fuse}>" if a.config == "jacobi" and D.fuse > 1 else "Jacobi5BodyT<false>",
             "conv3": "Conv2dBody<1>", "conv7": "Conv2dBody<3>",
             "spmv": "SpmvShubBody" if head.get("shub") else "SpmvBody"}[a.config]
     kern = {"agent": "k_agent", "static": "k_static", "default": "k_default", "identity": "k_agent"}.get(
         head.get("backend"), "k_agent") + f"<{body}>"
+    if a.config == "jacobi" and D.kname == "jacobi5_wave":
+        kern = jk
     bpl = D.bytes_per_step() // nl if D.x.world == 1 else None
     tr = traffic.get(a.config) if traffic else None
     if a.config == "conv7":
@@ -781,7 +802,7 @@ def home_fraction(a, D, head, device):
             kern = "bicg"
         elif a.config == "jacobi":
             args = cc.jacobi5_args(D.a, D.b, D.fuse, fuse=D.fuse)[0]       # one launch of the headline kernel
-            kern = "jacobi5"
+            kern = D.kname
         elif a.config in ("conv3", "conv7"):
             args, D._w = cc.conv2d_args(D.inp, D.out, D.w)
             kern = "conv2d"

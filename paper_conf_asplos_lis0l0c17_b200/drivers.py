@@ -270,8 +270,11 @@ class JacobiSlab:
     eagerly (a replayed graph would repeat the tags)."""
 
     def __init__(self, rows: int, cols: int, iters: int, xchg: Exchange, device, overlap: bool = True,
-                 halo: str = "exchange", fuse: int = 1):
+                 halo: str = "exchange", fuse: int = 1, kernel: str = "tile"):
         self.rows, self.cols, self.iters, self.x = rows, cols, iters, xchg
+        # kernel="wave": the K fused sweeps run as strip wavefronts
+        # (CC_K_JACOBI5_WAVE, R34, K <= 8); "tile": tile-fused (CC_K_JACOBI5, K <= 4)
+        self.kname = "jacobi5_wave" if kernel == "wave" and halo != "fused" else "jacobi5"
         # K sweeps per launch (R32).  Sharded, the slab keeps K halo rows per
         # side and exchanges them once per K sweeps: a slab edge acts as a fixed
         # boundary inside the launch, so after K sweeps the error it causes has
@@ -349,18 +352,20 @@ class JacobiSlab:
         if self.graph is not None:
             self.graph.replay()
             return self.graph_launches
-        if self.fuse > 1 and self.x.world == 1:
-            args, flag = cc.jacobi5_args(self.a, self.b, self.iters, fuse=self.fuse)
-            nl = _launch("jacobi5", args, opts, stream)
-            if flag.value:
-                self.a, self.b = self.b, self.a
+        if (self.fuse > 1 or self.kname == "jacobi5_wave") and self.x.world == 1:
+            nl = 0
+            for it, k in self.calls():
+                args, flag = cc.jacobi5_args(self.a, self.b, it, fuse=k)
+                nl += _launch(self.kname, args, opts, stream)
+                if flag.value:
+                    self.a, self.b = self.b, self.a
             return nl
         if self.fuse > 1:                                 # sharded: K sweeps, then the K-row halo exchange
             nl, done = 0, 0
             while done < self.iters:
                 k = min(self.fuse, self.iters - done)
                 args, flag = cc.jacobi5_args(self.a, self.b, k, fuse=k if k > 1 else 1)
-                nl += _launch("jacobi5", args, opts, stream)
+                nl += _launch(self.kname, args, opts, stream)
                 if flag.value:
                     self.a, self.b = self.b, self.a
                 self.x.halo_exchange(self.a, self.hw, stream)
@@ -374,7 +379,27 @@ class JacobiSlab:
             self.a, self.b = self.b, self.a
         return nl
 
+    def calls(self):
+        """(iters, fuse) per library call of an unsharded step: the iters // K
+        full launches, then the remainder -- as two launches when one would
+        leave the step with an odd launch count (a replayed graph must end in
+        the buffer it started from)."""
+        K = max(1, self.fuse)
+        full, r = divmod(self.iters, K)
+        if self.kname == "jacobi5" and K > 1:       # CC_K_JACOBI5 runs the remainder one sweep per launch
+            return [(self.iters, K)]
+        out = [(full * K, K)] if full else []
+        if r:
+            if (full + 1) % 2 and r >= 2:          # one more launch would make the count odd: two
+                h = r // 2
+                out += [(2 * h, h)] if r % 2 == 0 else [(h, h), (r - h, r - h)]
+            else:
+                out += [(r, r)]
+        return out
+
     def launches_per_step(self) -> int:
+        if self.kname == "jacobi5_wave" and self.x.world == 1:
+            return sum(-(-it // k) for it, k in self.calls())
         if self.fuse > 1 and self.x.world == 1:
             return self.iters // self.fuse + self.iters % self.fuse
         if self.fuse > 1:

@@ -21,12 +21,13 @@ def main():
     ap.add_argument("--size", type=int, default=0)
     ap.add_argument("--hot", type=int, default=16384)
     ap.add_argument("--fuse", type=int, default=3)
+    ap.add_argument("--jkernel", default="tile")
     a = ap.parse_args()
     import torch
     import bench
     from paper_conf_asplos_lis0l0c17_b200 import drivers
     ns = argparse.Namespace(config=a.config, n=a.size, iters=100, no_overlap=True, halo="exchange", fuse=a.fuse,
-                            hot=a.hot)
+                            hot=a.hot, jkernel=a.jkernel)
     D = bench.build_driver(ns, drivers.Exchange(), torch.device("cuda", 0))
     opts = json.loads(a.opts)
     if a.config == "jacobi":                   # one launch's worth of sweeps is enough for per-launch counts
