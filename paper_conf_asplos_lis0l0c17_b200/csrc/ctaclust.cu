@@ -668,6 +668,7 @@ static cc_status jw_launch_k(const LaunchCtx& c, const JWaveParams& prm) {
     s.steal = o.steal;
     s.batch = o.batch > 0 ? o.batch : JW_BATCH;
     s.stages = 1;
+    s.l2_hint = o.l2_hint;                         // bit 1: stores evict_first; bit 2: row loads evict_last
     s.census = o.d_census;
     s.exec_sm = o.d_exec_sm;
     s.map = o.d_map;

@@ -49,6 +49,10 @@ struct JWaveParams { const float* a; float* b; int64_t ld; int32_t rows, cols; }
 // rows [e0 - K, e1 + K) streamed
 struct JwRun { int32_t bx, e0, e1; };
 
+__device__ __forceinline__ void cp_async_cg16_h(void* dst, const void* src, uint32_t src_bytes, uint64_t pol) {
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(src_bytes), "l"(pol) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 // wait until at most n of this thread's cp.async groups are pending
 __device__ __forceinline__ void cp_async_wait_dyn(int n) {
@@ -434,7 +438,10 @@ k_jwave(const __grid_constant__ Sched s, const __grid_constant__ JWaveParams p) 
         auto issue_one = [&]() -> bool {
             if (pf_row >= pf_end && !refill()) return false;
             const bool in = pf_ptr != nullptr && (uint32_t)pf_row < (uint32_t)rows;
-            cp_async_cg16(my + (n_iss % JW_DEPTH) * 32, in ? pf_ptr : p.a, in ? 16u : 0u);
+            if (s.l2_hint & L2H_REUSE_LAST)                        // rows stay for the neighbour strip's halo
+                cp_async_cg16_h(my + (n_iss % JW_DEPTH) * 32, in ? pf_ptr : p.a, in ? 16u : 0u, l2_evict_last());
+            else
+                cp_async_cg16(my + (n_iss % JW_DEPTH) * 32, in ? pf_ptr : p.a, in ? 16u : 0u);
             cp_async_commit();
             if (pf_ptr) pf_ptr += ld;
             ++pf_row;
@@ -469,8 +476,9 @@ k_jwave(const __grid_constant__ Sched s, const __grid_constant__ JWaveParams p) 
             const float4 o = slow ? jw_ingest<K, PH, true>(S, x, i, rows, keep)
                                   : jw_ingest<K, PH, false>(S, x, i, rows, keep);
             if (st_kind && i >= st_from) {
-                if (st_kind == 1) *reinterpret_cast<float4*>(st_ptr) = o;
-                else store4_masked(st_ptr, o, W.cur_bx * WS - 4 * HL + 4 * lane, cols);
+                if (st_kind == 2) store4_out(st_ptr, o, W.cur_bx * WS - 4 * HL + 4 * lane, cols, s.l2_hint);
+                else if (s.l2_hint & L2H_STREAM_FIRST) st4_h(st_ptr, o, l2_evict_first());
+                else *reinterpret_cast<float4*>(st_ptr) = o;
             }
             st_ptr += ld;
             ++i;

@@ -45,7 +45,11 @@ def main():
         wpsm = cc.max_agents("jacobi5_wave", 0) if f <= 4 else None
         launches = -(-T // f)
         base = {"fuse": f, "launches": launches, "hbm_floor_ms": round(launches * 8 * N * N / B._peak() / 1e6, 3)}
-        for name, kw in (("agent-col", dict(backend="agent", order="col")),
+        extra = []
+        if os.environ.get("JW_HINTS"):
+            extra = [(f"{b}-{h}", dict(backend=b, l2_hint=h, **({"order": "col"} if b == "agent" else {})))
+                     for b in ("agent", "default") for h in ("stream_first", "reuse_last", "both")]
+        for name, kw in extra + [("agent-col", dict(backend="agent", order="col")),
                          ("agent-col-b8", dict(backend="agent", order="col", batch=8)),
                          ("agent-col-b4", dict(backend="agent", order="col", batch=4)),
                          ("agent-col-b2", dict(backend="agent", order="col", batch=2)),
@@ -59,7 +63,7 @@ def main():
                          ("agent-tile1x16-b16", dict(backend="agent", order="tile", tile=(1, 16), batch=16)),
                          ("agent-tile1x8-b8", dict(backend="agent", order="tile", tile=(1, 8), batch=8)),
                          ("identity", dict(backend="identity")),
-                         ("default", dict(backend="default"))):
+                         ("default", dict(backend="default"))]:
             timed(f"wave{f}-{name}", lambda kw=kw, f=f: ops.jacobi5_wave(a, b, T, fuse=f, **kw),
                   dict(base, warps_per_sm=wpsm))
     json.dump({"N": N, "sweeps": T, "rows": rows}, open(sys.argv[1], "w"), indent=1)

@@ -1,4 +1,4 @@
-# round-2 final pass: GPU suite, smoke, bench every config (default flags), reference arm, bench launch list
+# final pass: GPU suite, smoke, bench every config (default flags), reference arm, bench launch list + ncu captures
 mkdir -p gpurun_out/final
 make all > gpurun_out/final/build.log 2>&1 || tail -20 gpurun_out/final/build.log
 timeout -k 10 2400 python -m pytest tests/ -m gpu -q --timeout 900 > gpurun_out/final/t_gpu.log 2>&1; echo gpu=$?

@@ -5,7 +5,7 @@ initcheck).  Sizes are small so the instrumented runs finish in seconds;
 each launch is checked against the oracle so a tool-induced schedule change
 that broke the result would show as FAIL too.
 
-    python scripts/sanitize_targets.py [group ...]   groups: runtime gemv stencil tbc halo spmv
+    python scripts/sanitize_targets.py [group ...]   groups: runtime gemv stencil tbc halo spmv wave
 """
 import os
 import sys
@@ -34,6 +34,16 @@ def main(groups):
         ok &= good
         print(("ok   " if good else "FAIL ") + name, flush=True)
 
+    if "wave" in groups:                     # CC_K_JACOBI5_WAVE: mailboxes, chunk claims, steals, cp.async rings
+        u0 = synth.matrix(4, 300, 250)
+        for b, kw in (("agent", dict(order="col")), ("agent", dict(order="row", active_agents=3)),
+                      ("identity", {}), ("static", dict(order="col", num_clusters=7)), ("default", {})):
+            for fuse in (3, 8):
+                a_ = torch.from_numpy(u0).to(dev)
+                got = ops.jacobi5_wave(a_, torch.zeros_like(a_), 2 * fuse + 1, fuse=fuse, backend=b, **kw)
+                torch.cuda.synchronize()
+                check(f"jacobi5_wave {b} {kw} fuse={fuse}", got.cpu().numpy(), O.jacobi5_f32(u0, 2 * fuse + 1),
+                      exact=True)
     if "runtime" in groups:
         for b in ("agent", "identity", "static", "default", "redirect"):
             cen, _, _, _ = ops.census(13, 11, b, "row", num_clusters=148 if b == "static" else 0)

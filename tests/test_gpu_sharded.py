@@ -103,6 +103,23 @@ def test_atax_family_driver_world1():
         assert rel(got.cpu().numpy(), ref) <= 1e-4
 
 
+@pytest.mark.parametrize("fuse,T", [(8, 100), (8, 13), (3, 7), (6, 20)])
+def test_jacobi_wave_driver_world1_graph(fuse, T):
+    """The bench's config-3 driver with the wavefront kernel: the even launch
+    split (graph replay must end in the buffer it started from), captured and
+    replayed, bit-exact."""
+    rows, cols = 200, 300
+    d = drivers.JacobiSlab(rows, cols, T, drivers.Exchange(), "cuda", fuse=fuse, kernel="wave")
+    assert sum(it for it, _ in d.calls()) == T
+    opts = dict(backend="agent", order="col")
+    if d.launches_per_step() % 2 == 0:
+        assert d.capture(opts)
+    d.reset()
+    d.step(opts)
+    torch.cuda.synchronize()
+    assert np.array_equal(d.result().cpu().numpy(), O.jacobi5_f32(synth.matrix(4, rows, cols), T))
+
+
 def test_jacobi_driver_world1_graph():
     rows, cols, T = 160, 96, 6
     d = drivers.JacobiSlab(rows, cols, T, drivers.Exchange(), "cuda")
@@ -150,7 +167,8 @@ WORKER = textwrap.dedent("""
         rows, cols, T = 330, 200, 6
         d = drivers.JacobiSlab(rows, cols, T, X, "cuda", overlap=cfg == "jacobi",
                                halo="fused" if cfg == "jacobi-fused" else "exchange",
-                               fuse=int(cfg[-1]) if cfg.startswith("jacobi-k") else 1)
+                               fuse=int(cfg[-1]) if cfg[:8] in ("jacobi-k", "jacobi-w") else 1,
+                               kernel="wave" if cfg.startswith("jacobi-w") else "tile")
         ref = O.jacobi5_f32(synth.matrix(4, rows, cols), T)
         ref2 = O.jacobi5_f32(synth.matrix(4, rows, cols), 2 * T)
         d.step(dict(backend="agent", order="row", max_agents=1))
@@ -204,7 +222,8 @@ def _port():
 
 @pytest.mark.parametrize("cfg,world", [("atax", 2), ("atax", 4), ("jacobi", 2), ("jacobi", 3), ("jacobi", 4),
                                        ("jacobi-nooverlap", 3), ("jacobi-fused", 2), ("jacobi-fused", 3),
-                                       ("jacobi-k4", 2), ("jacobi-k3", 3), ("conv1", 2), ("conv3", 3), ("spmv", 2),
+                                       ("jacobi-k4", 2), ("jacobi-k3", 3), ("jacobi-w4", 2), ("jacobi-w5", 3),
+                                       ("conv1", 2), ("conv3", 3), ("spmv", 2),
                                        ("spmv", 3), ("spmv-hot", 2), ("spmv-shub", 2)])
 def test_sharded_driver_ranks_one_gpu(tmp_path, cfg, world):
     script = tmp_path / "w.py"
