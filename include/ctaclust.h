@@ -343,7 +343,6 @@ cc_status cc_ipc_close(void* dptr);
  * in/out rows x cols fp32 DEVICE, leading dim ld (% 4 == 0).  Logical CTA = 32x32
  * output tile; grid ceil(cols/32) x ceil(rows/32). */
 typedef struct { const float* in; float* out; int64_t ld; int32_t rows, cols; int32_t R; const float* w; } cc_conv2d_args;
-
 /* CSR SpMV y = A x (R16).  DEVICE row_ptr[rows+1], col[nnz], val[nnz], x[cols],
  * y[rows] (zeroed by the call), int32 indices, nnz < 2^31.  Logical CTA b owns
  * the merge-path diagonals [4096 b, 4096 (b+1)) of the row-ends x nonzeros merge

@@ -472,7 +472,7 @@ static cc_status occupancy(int device, int stages, int* occ, bool direct = false
     return CC_OK;
 }
 
-template <int K, int HL> static cc_status jw_occupancy(int device, int* warps);
+template <class B> static cc_status jw_occupancy(int device, int* warps);
 
 extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     if (!out) return fail(CC_ERR_INVALID_ARG, "null out");
@@ -486,7 +486,7 @@ extern "C" cc_status cc_max_agents(int32_t k, int32_t device, int32_t* out) {
     case CC_K_BICG: case CC_K_MVT: s = occupancy<BothB>(device, BothB::kDefaultStages, &occ); break;
     case CC_K_JACOBI5: s = occupancy<Jacobi5Body>(device, Jacobi5Body::kDefaultStages, &occ); break;
     case CC_K_JACOBI5_HALO: s = occupancy<Jacobi5HaloBody>(device, Jacobi5HaloBody::kDefaultStages, &occ); break;
-    case CC_K_JACOBI5_WAVE: s = jw_occupancy<4, 1>(device, &occ); break;
+    case CC_K_JACOBI5_WAVE: s = jw_occupancy<JwJacobi<4, 1>>(device, &occ); break;
     case CC_K_CONV2D: s = occupancy<Conv2dBody<3>>(device, Conv2dBody<3>::kDefaultStages, &occ); break;
     case CC_K_SPMV: s = occupancy<SpmvBody>(device, SpmvBody::kDefaultStages, &occ); break;
     case CC_K_SPMV_SHUB: s = occupancy<SpmvShubBody>(device, SpmvShubBody::kDefaultStages, &occ); break;
@@ -617,21 +617,21 @@ static cc_status launch_body(const LaunchCtx& c, const typename Body::Params& pr
 
 // ---- CC_K_JACOBI5_WAVE: warp agents (k_jwave.cuh) -------------------------
 // opt the kernel into its dynamic shared memory (once per device)
-template <int K, int HL, int KIND>
+template <class B, int KIND>
 static cc_status jw_prepare(int device) {
     static std::mutex mu;
     static bool done[64] = {false};
     if (device < 0 || device >= 64) return fail(CC_ERR_INVALID_ARG, "device");
     std::lock_guard<std::mutex> lk(mu);
     if (!done[device]) {
-        CC_CUDA(cudaFuncSetAttribute(k_jwave<K, HL, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, jw_smem(K, KIND)));
+        CC_CUDA(cudaFuncSetAttribute(k_strip<B, KIND>, cudaFuncAttributeMaxDynamicSharedMemorySize, jw_smem<B>(KIND)));
         done[device] = true;
     }
     return CC_OK;
 }
 
 // worker warps per SM the hardware keeps resident
-template <int K, int HL>
+template <class B>
 static cc_status jw_occupancy(int device, int* warps) {
     static std::mutex mu;
     static int cache[64] = {};
@@ -641,21 +641,22 @@ static cc_status jw_occupancy(int device, int* warps) {
         int prev = 0, n = 0;
         CC_CUDA(cudaGetDevice(&prev));
         CC_CUDA(cudaSetDevice(device));
-        cc_status st = jw_prepare<K, HL, JW_DYNAMIC>(device);
+        cc_status st = jw_prepare<B, JW_DYNAMIC>(device);
         if (st == CC_OK)
-            CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_jwave<K, HL, JW_DYNAMIC>,
-                                                                  jw_threads(K, JW_DYNAMIC), jw_smem(K, JW_DYNAMIC)));
+            CC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, k_strip<B, JW_DYNAMIC>, jw_threads<B>(JW_DYNAMIC),
+                                                                  jw_smem<B>(JW_DYNAMIC)));
         CC_CUDA(cudaSetDevice(prev));
         if (st != CC_OK) return st;
-        cache[device] = n > 0 ? n * jw_workers(K, JW_DYNAMIC) : -1;
+        cache[device] = n > 0 ? n * jw_workers<B>(JW_DYNAMIC) : -1;
     }
     *warps = cache[device];
-    if (*warps < 0) return fail(CC_ERR_UNSUPPORTED, "jacobi5_wave: no resident CTA");
+    if (*warps < 0) return fail(CC_ERR_UNSUPPORTED, "strip kernel: no resident CTA");
     return CC_OK;
 }
 
-template <int K, int HL>
-static cc_status jw_launch_k(const LaunchCtx& c, const JWaveParams& prm) {
+// one launch of a strip kernel (CC_K_JACOBI5_WAVE): warp agents
+template <class B>
+static cc_status strip_launch(const LaunchCtx& c, const typename B::Params& prm) {
     const Grid& g = c.p->g;
     if (g.V == 0) return CC_OK;
     const cc_launch_opts& o = *c.o;
@@ -668,25 +669,26 @@ static cc_status jw_launch_k(const LaunchCtx& c, const JWaveParams& prm) {
     s.steal = o.steal;
     s.batch = o.batch > 0 ? o.batch : JW_BATCH;
     s.stages = 1;
-    s.l2_hint = o.l2_hint;                         // bit 1: stores evict_first; bit 2: row loads evict_last
+    // (L2 eviction hints on the row loads / stores measured no gain and cost
+    // the row loop registers: not supported here, r15)
     s.census = o.d_census;
     s.exec_sm = o.d_exec_sm;
     s.map = o.d_map;
     switch (o.backend) {
     case CC_BACKEND_DEFAULT:                       // hardware order: warp w of the grid = logical CTA w
-        CC_TRY(jw_prepare<K, HL, JW_ONESHOT>(c.p->device));
-        CC_TRY(set_carveout(k_jwave<K, HL, JW_ONESHOT>, o.carveout));
+        CC_TRY(jw_prepare<B, JW_ONESHOT>(c.p->device));
+        CC_TRY(set_carveout(k_strip<B, JW_ONESHOT>, o.carveout));
         s.map = nullptr;
-        k_jwave<K, HL, JW_ONESHOT><<<cdiv(g.V, jw_workers(K, JW_ONESHOT)), jw_threads(K, JW_ONESHOT),
-                                     jw_smem(K, JW_ONESHOT), c.st>>>(s, prm);
+        k_strip<B, JW_ONESHOT><<<cdiv(g.V, jw_workers<B>(JW_ONESHOT)), jw_threads<B>(JW_ONESHOT),
+                                  jw_smem<B>(JW_ONESHOT), c.st>>>(s, prm);
         break;
     case CC_BACKEND_AGENT:
     case CC_BACKEND_AGENT_IDENTITY: {
         int occ = 0;
-        CC_TRY(set_carveout(k_jwave<K, HL, JW_DYNAMIC>, o.carveout));
-        CC_TRY(jw_occupancy<K, HL>(c.p->device, &occ));
+        CC_TRY(set_carveout(k_strip<B, JW_DYNAMIC>, o.carveout));
+        CC_TRY(jw_occupancy<B>(c.p->device, &occ));
         const int maxa = o.max_agents > 0 ? std::min(o.max_agents, occ) : occ;
-        constexpr int nw = jw_workers(K, JW_DYNAMIC);
+        constexpr int nw = jw_workers<B>(JW_DYNAMIC);
         const int ctas = (maxa + nw - 1) / nw;                         // per SM (workers + a scheduler each)
         const int launched = ctas * nw;
         s.active_agents = o.active_agents > 0 ? std::min(o.active_agents, launched) : launched;
@@ -694,22 +696,22 @@ static cc_status jw_launch_k(const LaunchCtx& c, const JWaveParams& prm) {
         s.mode = o.backend == CC_BACKEND_AGENT ? MODE_AGENT : MODE_IDENTITY;
         WsLease lease{c.p, c.st};
         CC_TRY(lease.acquire());
-        k_jwave<K, HL, JW_DYNAMIC><<<c.p->facts->num_sms * ctas, jw_threads(K, JW_DYNAMIC), jw_smem(K, JW_DYNAMIC),
-                                     c.st>>>(s, prm);
+        k_strip<B, JW_DYNAMIC><<<c.p->facts->num_sms * ctas, jw_threads<B>(JW_DYNAMIC), jw_smem<B>(JW_DYNAMIC),
+                                  c.st>>>(s, prm);
         if (cudaPeekAtLastError() == cudaSuccess) CC_TRY(lease.release());
         break;
     }
     case CC_BACKEND_AGENT_STATIC:                  // worker warp i runs cluster i (Eq. 7 order)
-        CC_TRY(jw_prepare<K, HL, JW_STATIC>(c.p->device));
-        CC_TRY(set_carveout(k_jwave<K, HL, JW_STATIC>, o.carveout));
+        CC_TRY(jw_prepare<B, JW_STATIC>(c.p->device));
+        CC_TRY(set_carveout(k_strip<B, JW_STATIC>, o.carveout));
         s.active_agents = 1;
         s.steal = 0;
         s.mode = MODE_STATIC;
-        k_jwave<K, HL, JW_STATIC><<<cdiv(g.M, jw_workers(K, JW_STATIC)), jw_threads(K, JW_STATIC), jw_smem(K, JW_STATIC),
-                                    c.st>>>(s, prm);
+        k_strip<B, JW_STATIC><<<cdiv(g.M, jw_workers<B>(JW_STATIC)), jw_threads<B>(JW_STATIC), jw_smem<B>(JW_STATIC),
+                                 c.st>>>(s, prm);
         break;
     default:
-        return fail(CC_ERR_UNSUPPORTED, "backend %d not available for jacobi5_wave", o.backend);
+        return fail(CC_ERR_UNSUPPORTED, "backend %d not available for the strip kernels", o.backend);
     }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "kernel launch");
@@ -720,18 +722,18 @@ static cc_status jw_launch_k(const LaunchCtx& c, const JWaveParams& prm) {
 template <int HL>
 static cc_status jw_launch(const LaunchCtx& c, const JWaveParams& prm, int K) {
     switch (K) {
-    case 1: return jw_launch_k<1, HL>(c, prm);
-    case 2: return jw_launch_k<2, HL>(c, prm);
-    case 3: return jw_launch_k<3, HL>(c, prm);
-    case 4: return jw_launch_k<4, HL>(c, prm);
+    case 1: return strip_launch<JwJacobi<1, HL>>(c, prm);
+    case 2: return strip_launch<JwJacobi<2, HL>>(c, prm);
+    case 3: return strip_launch<JwJacobi<3, HL>>(c, prm);
+    case 4: return strip_launch<JwJacobi<4, HL>>(c, prm);
     default: break;
     }
     if constexpr (HL == 2) {
         switch (K) {
-        case 5: return jw_launch_k<5, 2>(c, prm);
-        case 6: return jw_launch_k<6, 2>(c, prm);
-        case 7: return jw_launch_k<7, 2>(c, prm);
-        case 8: return jw_launch_k<8, 2>(c, prm);
+        case 5: return strip_launch<JwJacobi<5, 2>>(c, prm);
+        case 6: return strip_launch<JwJacobi<6, 2>>(c, prm);
+        case 7: return strip_launch<JwJacobi<7, 2>>(c, prm);
+        case 8: return strip_launch<JwJacobi<8, 2>>(c, prm);
         default: break;
         }
     }

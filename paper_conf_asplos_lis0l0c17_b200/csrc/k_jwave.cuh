@@ -49,10 +49,6 @@ struct JWaveParams { const float* a; float* b; int64_t ld; int32_t rows, cols; }
 // rows [e0 - K, e1 + K) streamed
 struct JwRun { int32_t bx, e0, e1; };
 
-__device__ __forceinline__ void cp_async_cg16_h(void* dst, const void* src, uint32_t src_bytes, uint64_t pol) {
-    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;"
-                 :: "r"(smem_u32(dst)), "l"(src), "r"(src_bytes), "l"(pol) : "memory");
-}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 // wait until at most n of this thread's cp.async groups are pending
 __device__ __forceinline__ void cp_async_wait_dyn(int n) {
@@ -222,30 +218,78 @@ __device__ __forceinline__ void st_release_cta(int32_t* p, int32_t v) {
     asm volatile("st.release.cta.shared::cta.b32 [%0], %1;" :: "r"(smem_u32(p)), "r"(v) : "memory");
 }
 
-// Worker warps per CTA.  One-shot: JW_WARPS per CTA, 3 (K <= 4) or 2 CTAs
-// per SM.  Persistent kinds: ONE CTA per SM, its workers plus one scheduler
-// warp, sized so that a thread keeps the registers the sweep levels need
-// (65536 / threads: 24 + 1 warps -> 80 for K <= 3, 20 + 1 -> 96 for K = 4,
-// 15 + 1 -> 128 for K >= 5); any more workers and ptxas moves sweep levels
-// to local memory (measured: 15-25 % slower).
-__host__ __device__ constexpr int jw_workers(int K, int kind) {
-    return kind == JW_ONESHOT ? JW_WARPS : (K <= 3 ? 24 : K == 4 ? 20 : 15);
+// ---------------------------------------------------------------------------
+// Strip bodies.  A body says what one ingested input row does to a warp's
+// registers: kVec float4 per lane (a strip is 128 kVec loaded columns),
+// kHaloLanes lanes at each strip edge that load but do not store (the output
+// strip is WS = (32 - 2 kHaloLanes) 4 kVec columns), kLag (ingesting row i
+// yields output row i - kLag, so a fresh run starts kLag rows above its first
+// output row), kPhases (the ingest count modulo which the body rotates its
+// registers, a template parameter of ingest()).
+// ---------------------------------------------------------------------------
+
+// Jacobi, K fused sweeps (R34)
+template <int K, int HL>
+struct JwJacobi {
+    static constexpr int kVec = 1, kHaloLanes = HL, kLag = K, kPhases = 3;
+    static constexpr int kWorkers = K <= 3 ? 24 : K == 4 ? 20 : 15;   // persistent kinds, one CTA per SM
+    static constexpr int kOneshotBlocks = K <= 4 ? 3 : 2;
+    static_assert(K >= 1 && 4 * HL >= K, "the strip's halo columns must cover K sweeps");
+    using Params = JWaveParams;
+    float4 S[K][3];
+    uint32_t keep;          // this lane's global boundary columns (bit e = column gcol + e)
+    bool edge;              // the strip holds a boundary column
+    __device__ __forceinline__ void init(const Params&) {
+#pragma unroll
+        for (int l = 0; l < K; ++l)
+#pragma unroll
+            for (int m = 0; m < 3; ++m) S[l][m] = make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+    // per strip: returns this lane's store kind (0 none, 1 full float4s, 2 masked ragged edge)
+    __device__ __forceinline__ int32_t set_strip(int32_t gcol, int lane, const Params& p) {
+        const int32_t cols = p.cols;
+        keep = 0;
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+            if (gcol + e == 0 || gcol + e == cols - 1) keep |= 1u << e;
+        edge = __any_sync(0xffffffffu, keep != 0);
+        return (lane < HL || lane >= 32 - HL || gcol >= cols) ? 0 : (gcol + 3 < cols ? 1 : 2);
+    }
+    template <int PH>
+    __device__ __forceinline__ void ingest(const float4 (&x)[1], int32_t i, float4 (&o)[1], const Params& p) {
+        const int32_t rows = p.rows;
+        const bool slow = edge || (uint32_t)(i - 1) < (uint32_t)K || (uint32_t)(i - rows) < (uint32_t)K;
+        o[0] = slow ? jw_ingest<K, PH, true>(S, x[0], i, rows, keep) : jw_ingest<K, PH, false>(S, x[0], i, rows, keep);
+    }
+};
+
+// Worker warps per CTA.  One-shot: JW_WARPS per CTA, B::kOneshotBlocks CTAs
+// per SM.  Persistent kinds: ONE CTA per SM, B::kWorkers workers plus one
+// scheduler warp, sized so that a thread keeps the registers the body needs
+// (65536 / threads: 24 + 1 warps -> 80, 20 + 1 -> 96, 15 + 1 -> 128); more
+// workers and ptxas moves the body's registers to local memory (measured:
+// 15-25 % slower).
+template <class B> __host__ __device__ constexpr int jw_workers(int kind) {
+    return kind == JW_ONESHOT ? JW_WARPS : B::kWorkers;
 }
-__host__ __device__ constexpr int jw_threads(int K, int kind) {
-    return (jw_workers(K, kind) + (kind == JW_ONESHOT ? 0 : 1)) * 32;
+template <class B> __host__ __device__ constexpr int jw_threads(int kind) {
+    return (jw_workers<B>(kind) + (kind == JW_ONESHOT ? 0 : 1)) * 32;
 }
 // dynamic shared memory: the workers' cp.async rings
-__host__ __device__ constexpr int jw_smem(int K, int kind) { return jw_workers(K, kind) * JW_DEPTH * 32 * 16; }
+template <class B> __host__ __device__ constexpr int jw_smem(int kind) {
+    return jw_workers<B>(kind) * JW_DEPTH * 32 * 16 * B::kVec;
+}
+template <class B> __host__ __device__ constexpr int jw_ws() { return (32 - 2 * B::kHaloLanes) * 4 * B::kVec; }
 
-template <int K, int HL, int KIND>
-__global__ void __launch_bounds__(jw_threads(K, KIND), (KIND == JW_ONESHOT ? (K <= 4 ? 3 : 2) : 1))
-k_jwave(const __grid_constant__ Sched s, const __grid_constant__ JWaveParams p) {
-    static_assert(K >= 1 && 4 * HL >= K, "the strip's halo columns must cover K sweeps");
-    constexpr int WS = jw_strip_cols(HL);
-    constexpr int NW = jw_workers(K, KIND);                             // worker warps
+template <class B, int KIND>
+__global__ void __launch_bounds__(jw_threads<B>(KIND), (KIND == JW_ONESHOT ? B::kOneshotBlocks : 1))
+k_strip(const __grid_constant__ Sched s, const __grid_constant__ typename B::Params p) {
+    constexpr int NW = jw_workers<B>(KIND);                              // worker warps
+    constexpr int V = B::kVec, LAG = B::kLag;
+    constexpr int WS = jw_ws<B>();
+    constexpr int HC = 4 * V * B::kHaloLanes;                            // halo columns per side
     static_assert(NW < 32, "live-worker mask");
     extern __shared__ __align__(16) float4 jw_dyn[];
-    float4 (*ring)[JW_DEPTH][32] = reinterpret_cast<float4 (*)[JW_DEPTH][32]>(jw_dyn);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int32_t rows = p.rows, cols = p.cols;
     const int64_t ld = p.ld;
@@ -367,7 +411,7 @@ k_jwave(const __grid_constant__ Sched s, const __grid_constant__ JWaveParams p) 
     };
 
     // Run bookkeeping touched only when a run ends or the prefetch cursor
-    // leaves one lives in shared memory; the registers hold the sweep levels
+    // leaves one lives in shared memory; the registers hold the body's state
     // and the per-row cursors.
     struct JwWarp { JwRun nxt; int32_t cur_bx, cur_e1, has_nxt, more, pf_in_nxt, pf_done; };
     __shared__ JwWarp sW[NW];
@@ -377,36 +421,39 @@ k_jwave(const __grid_constant__ Sched s, const __grid_constant__ JWaveParams p) 
     if (pop(first)) {
         if (lane == 0) { W.cur_bx = first.bx; W.cur_e1 = first.e1; W.has_nxt = 0; W.more = 1; W.pf_in_nxt = 0; W.pf_done = 0; }
         __syncwarp();
-        float4* my = &ring[warp][0][lane];
-        // ---- prefetch cursor: rows [pf_row, pf_end) from pf_ptr on (null: this lane's columns are outside)
+        float4* my = jw_dyn + (size_t)warp * JW_DEPTH * 32 * V + lane * V;   // [slot][lane][v], slot stride 32 V
+        // ---- prefetch cursor: rows [pf_row, pf_end) from pf_ptr on; pf_ok: this
+        // lane's float4 chunks inside the image (bit v)
         int32_t pf_row = 0, pf_end = 0;
-        const float* pf_ptr = nullptr;
+        uint32_t pf_ok = 0;
+        const float* pf_ptr = p.a;
         auto pf_start = [&](const JwRun& r) {
-            const int32_t gcol = r.bx * WS - 4 * HL + 4 * lane;
-            pf_row = r.e0 - K;
-            pf_end = r.e1 + K;
-            pf_ptr = (gcol >= 0 && gcol < cols) ? p.a + (int64_t)pf_row * ld + gcol : nullptr;
+            const int32_t gcol = r.bx * WS - HC + 4 * V * lane;
+            pf_row = r.e0 - LAG;
+            pf_end = r.e1 + LAG;
+            uint32_t ok = 0;
+#pragma unroll
+            for (int v = 0; v < V; ++v)
+                if (gcol + 4 * v >= 0 && gcol + 4 * v < cols) ok |= 1u << v;
+            if constexpr (V > 1) pf_ok = ok;
+            // one float4 per lane: a null cursor says "outside" (no mask register)
+            pf_ptr = ok ? p.a + (int64_t)pf_row * ld + gcol : (V > 1 ? p.a : nullptr);
         };
         pf_start(first);
         int32_t n_iss = 0, n_use = 0;            // rows issued / consumed (one cp.async group each)
+        B body;
+        body.init(p);
         // ---- consumer cursor: ingest row i < i_end of the current run, store
-        // row i - K (through st_ptr) once i >= st_from
-        int32_t i = 0, i_end = 0, st_from = 0, st_kind = 0;   // st_kind: 0 none, 1 float4, 2 masked (ragged edge)
-        uint32_t keep = 0;
-        bool edge = false;
+        // row i - LAG (through st_ptr) once i >= st_from
+        int32_t i = 0, i_end = 0, st_from = 0, st_kind = 0;
         float* st_ptr = p.b;
         auto set_strip = [&](const JwRun& r) {
-            i = r.e0 - K;
-            i_end = r.e1 + K;
-            st_from = r.e0 + K;
-            const int32_t gcol = r.bx * WS - 4 * HL + 4 * lane;
-            keep = 0;
-#pragma unroll
-            for (int e = 0; e < 4; ++e)
-                if (gcol + e == 0 || gcol + e == cols - 1) keep |= 1u << e;
-            edge = __any_sync(0xffffffffu, keep != 0);
-            st_kind = (lane < HL || lane >= 32 - HL || gcol >= cols) ? 0 : (gcol + 3 < cols ? 1 : 2);
-            st_ptr = p.b + (int64_t)(i - K) * ld + (st_kind ? gcol : 0);
+            i = r.e0 - LAG;
+            i_end = r.e1 + LAG;
+            st_from = r.e0 + LAG;
+            const int32_t gcol = r.bx * WS - HC + 4 * V * lane;
+            st_kind = body.set_strip(gcol, lane, p);
+            st_ptr = p.b + (int64_t)(i - LAG) * ld + (st_kind ? gcol : 0);
         };
         set_strip(first);
         // the prefetch cursor ran off its run: extend the current run when the
@@ -437,30 +484,27 @@ k_jwave(const __grid_constant__ Sched s, const __grid_constant__ JWaveParams p) 
         };
         auto issue_one = [&]() -> bool {
             if (pf_row >= pf_end && !refill()) return false;
-            const bool in = pf_ptr != nullptr && (uint32_t)pf_row < (uint32_t)rows;
-            if (s.l2_hint & L2H_REUSE_LAST)                        // rows stay for the neighbour strip's halo
-                cp_async_cg16_h(my + (n_iss % JW_DEPTH) * 32, in ? pf_ptr : p.a, in ? 16u : 0u, l2_evict_last());
-            else
-                cp_async_cg16(my + (n_iss % JW_DEPTH) * 32, in ? pf_ptr : p.a, in ? 16u : 0u);
+            const bool row_in = (uint32_t)pf_row < (uint32_t)rows;
+            float4* dst = my + (n_iss % JW_DEPTH) * 32 * V;
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+                const bool in = row_in && (V > 1 ? ((pf_ok >> v) & 1u) != 0 : pf_ptr != nullptr);
+                cp_async_cg16(dst + v, in ? pf_ptr + 4 * v : p.a, in ? 16u : 0u);
+            }
             cp_async_commit();
-            if (pf_ptr) pf_ptr += ld;
+            if (V > 1 ? pf_ok != 0 : pf_ptr != nullptr) pf_ptr += ld;
             ++pf_row;
             ++n_iss;
             return true;
         };
         while (n_iss < JW_DEPTH - 1 && issue_one()) {}
 
-        float4 S[K][3];
-#pragma unroll
-        for (int l = 0; l < K; ++l)
-#pragma unroll
-            for (int m = 0; m < 3; ++m) S[l][m] = make_float4(0.f, 0.f, 0.f, 0.f);
-        // one ingested row; the phase (ingest count mod 3) picks the slot rotation
+        // one ingested row; the phase (ingest count mod kPhases) picks the body's register rotation
         auto step = [&](auto phase) -> bool {
             constexpr int PH = decltype(phase)::value;
             if (i >= i_end) {
                 if (!W.has_nxt) return false;
-                const JwRun r = W.nxt;                             // a fresh run: the levels restart
+                const JwRun r = W.nxt;                             // a fresh run: the body restarts
                 __syncwarp();
                 if (lane == 0) { W.has_nxt = 0; W.pf_in_nxt = 0; W.cur_bx = r.bx; W.cur_e1 = r.e1; }
                 __syncwarp();
@@ -469,29 +513,41 @@ k_jwave(const __grid_constant__ Sched s, const __grid_constant__ JWaveParams p) 
             const int ahead = n_iss - n_use - 1;                   // groups issued after row i's
             if (ahead >= JW_DEPTH - 2) asm volatile("cp.async.wait_group %0;" :: "n"(JW_DEPTH - 2) : "memory");
             else cp_async_wait_dyn(ahead);
-            const float4 x = my[(n_use % JW_DEPTH) * 32];
+            float4 x[V], o[V];
+            const float4* src = my + (n_use % JW_DEPTH) * 32 * V;
+#pragma unroll
+            for (int v = 0; v < V; ++v) x[v] = src[v];
             ++n_use;
             if (n_iss - n_use < JW_DEPTH - 1) issue_one();
-            const bool slow = edge || (uint32_t)(i - 1) < (uint32_t)K || (uint32_t)(i - rows) < (uint32_t)K;
-            const float4 o = slow ? jw_ingest<K, PH, true>(S, x, i, rows, keep)
-                                  : jw_ingest<K, PH, false>(S, x, i, rows, keep);
+            body.template ingest<PH>(x, i, o, p);
             if (st_kind && i >= st_from) {
-                if (st_kind == 2) store4_out(st_ptr, o, W.cur_bx * WS - 4 * HL + 4 * lane, cols, s.l2_hint);
-                else if (s.l2_hint & L2H_STREAM_FIRST) st4_h(st_ptr, o, l2_evict_first());
-                else *reinterpret_cast<float4*>(st_ptr) = o;
+                if (st_kind == 2) {                                // ragged right edge (rare): column from smem
+                    const int32_t gcol = W.cur_bx * WS - HC + 4 * V * lane;
+#pragma unroll
+                    for (int v = 0; v < V; ++v)
+                        if (gcol + 4 * v < cols) store4_masked(st_ptr + 4 * v, o[v], gcol + 4 * v, cols);
+                } else {
+#pragma unroll
+                    for (int v = 0; v < V; ++v) *reinterpret_cast<float4*>(st_ptr + 4 * v) = o[v];
+                }
             }
             st_ptr += ld;
             ++i;
             return true;
         };
+        constexpr int NP = B::kPhases;
+        static_assert(NP >= 1 && NP <= 7, "phases");
         for (;;) {
             if (!step(std::integral_constant<int, 0>{})) break;
-            if (!step(std::integral_constant<int, 1>{})) break;
-            if (!step(std::integral_constant<int, 2>{})) break;
+            if constexpr (NP > 1) if (!step(std::integral_constant<int, 1 % NP>{})) break;
+            if constexpr (NP > 2) if (!step(std::integral_constant<int, 2 % NP>{})) break;
+            if constexpr (NP > 3) if (!step(std::integral_constant<int, 3 % NP>{})) break;
+            if constexpr (NP > 4) if (!step(std::integral_constant<int, 4 % NP>{})) break;
+            if constexpr (NP > 5) if (!step(std::integral_constant<int, 5 % NP>{})) break;
+            if constexpr (NP > 6) if (!step(std::integral_constant<int, 6 % NP>{})) break;
         }
         asm volatile("cp.async.wait_all;" ::: "memory");
     }
-
 }
 
 }  // namespace cc

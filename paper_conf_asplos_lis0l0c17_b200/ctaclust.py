@@ -277,6 +277,8 @@ def jacobi5_args(a, b, iters, rows=None, cols=None, row_window=None, fuse=1) -> 
     rows = a.shape[0] if rows is None else rows
     cols = a.shape[1] if cols is None else cols
     lo, hi = (0, 0) if row_window is None else (int(row_window[0]), int(row_window[1]))
+    if _lda(b) != _lda(a):
+        raise CtaclustError(-1, f"jacobi5: a and b share one leading dimension (got {_lda(a)} and {_lda(b)})")
     args = Jacobi5Args(a.data_ptr(), b.data_ptr(), _lda(a), rows, cols, iters, ctypes.addressof(flag), lo, hi,
                        int(fuse))
     args._keep = flag            # result_is_b points into it: it must live as long as the struct
@@ -337,6 +339,8 @@ def conv2d_args(inp, out, w, rows=None, cols=None) -> tuple[Conv2dArgs, np.ndarr
     K = w.shape[0]
     rows = inp.shape[0] if rows is None else rows
     cols = inp.shape[1] if cols is None else cols
+    if _lda(out) != _lda(inp):
+        raise CtaclustError(-1, f"conv2d: in and out share one leading dimension (got {_lda(inp)} and {_lda(out)})")
     args = Conv2dArgs(inp.data_ptr(), out.data_ptr(), _lda(inp), rows, cols, K // 2, w.ctypes.data)
     args._keep = w               # the filter is read from this host array at launch
     return args, w

@@ -162,8 +162,13 @@ def jacobi5_halo(a, b, iters, sweep0=0, ll=None, up_ll=None, dn_ll=None, status=
     return b if flag.value else a
 
 
+def _like(t):
+    """an output with t's shape and strides (the C ABI has one leading dimension for in and out)"""
+    return torch.empty_strided(t.shape, t.stride(), dtype=t.dtype, device=t.device)
+
+
 def conv2d(inp, w, out=None, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
-    out = torch.empty_like(inp) if out is None else out
+    out = _like(inp) if out is None else out
     args, _w = cc.conv2d_args(inp, out, w)
     _launch("conv2d", args, backend, order, tile, num_clusters, _dev(inp), stream, **kw)
     return out

@@ -4,7 +4,7 @@ OUT=${1:-gpurun_out/san}
 mkdir -p $OUT
 CS=/usr/local/cuda/bin/compute-sanitizer
 for tool in memcheck racecheck synccheck initcheck; do
-  for grp in ${GROUPS:-runtime gemv stencil tbc halo spmv wave}; do
+  for grp in ${SAN_GROUPS:-runtime gemv stencil tbc halo spmv wave}; do
     timeout -k 10 900 $CS --tool $tool --print-limit 20 --error-exitcode 9 \
       python scripts/sanitize_targets.py $grp > $OUT/${tool}_${grp}.log 2>&1
     rc=$?

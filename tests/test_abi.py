@@ -204,3 +204,17 @@ def test_arg_structs_own_their_host_buffers():
     assert c._keep.ctypes.data == c.w
     h = cc.jacobi5_halo_args(a, a, 1)[0]
     assert ctypes.addressof(h._keep) == h.result_is_b
+
+
+def test_in_out_share_leading_dimension():
+    """The C ABI carries one leading dimension for a kernel's input and output
+    (cc_conv2d_args.ld, cc_jacobi5_args.ld): the binding refuses a pair whose
+    strides differ instead of writing the output with the input's pitch."""
+    import torch
+    a = torch.zeros(8, 72)[:, :70]
+    b = torch.zeros(8, 70)
+    with pytest.raises(cc.CtaclustError):
+        cc.conv2d_args(a, b, [[1.0]])
+    with pytest.raises(cc.CtaclustError):
+        cc.jacobi5_args(a, b, 1)
+    cc.conv2d_args(a, torch.zeros(8, 72)[:, :70], [[1.0]])
