@@ -734,7 +734,7 @@ def roofline(a, D, head, ms_clu, per_clu, launches, clk, pk):
     ms_launch = ms_clu / nl
     if a.config == "jacobi" and D.kname == "jacobi5_wave":
         kind = {"agent": 0, "identity": 0, "static": 1, "default": 2}.get(head.get("backend"), 0)
-        jk = f"k_jwave<{D.fuse}, {1 if D.fuse <= 4 else 2}, {kind}>"
+        jk = f"k_strip<JwJacobi<{D.fuse}, {1 if D.fuse <= 4 else 2}>, {kind}>"
     body = {"jacobi": f"Jacobi5MultiBody<{D.fuse}>" if a.config == "jacobi" and D.fuse > 1 else "Jacobi5BodyT<false>",
             "conv3": "Conv2dBody<1>", "conv7": "Conv2dBody<3>",
             "spmv": "SpmvShubBody" if head.get("shub") else "SpmvBody"}[a.config]

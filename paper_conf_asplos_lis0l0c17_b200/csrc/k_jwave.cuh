@@ -421,7 +421,9 @@ k_strip(const __grid_constant__ Sched s, const __grid_constant__ typename B::Par
     if (pop(first)) {
         if (lane == 0) { W.cur_bx = first.bx; W.cur_e1 = first.e1; W.has_nxt = 0; W.more = 1; W.pf_in_nxt = 0; W.pf_done = 0; }
         __syncwarp();
-        float4* my = jw_dyn + (size_t)warp * JW_DEPTH * 32 * V + lane * V;   // [slot][lane][v], slot stride 32 V
+        // this lane's ring entries as a 32-bit shared address ([slot][lane][v], slot stride 32 V float4):
+        // one register, no generic-to-shared conversion per row
+        const uint32_t my = smem_u32(jw_dyn) + (uint32_t)(((warp * JW_DEPTH * 32) + lane) * V * 16);
         // ---- prefetch cursor: rows [pf_row, pf_end) from pf_ptr on; pf_ok: this
         // lane's float4 chunks inside the image (bit v)
         int32_t pf_row = 0, pf_end = 0;
@@ -485,11 +487,12 @@ k_strip(const __grid_constant__ Sched s, const __grid_constant__ typename B::Par
         auto issue_one = [&]() -> bool {
             if (pf_row >= pf_end && !refill()) return false;
             const bool row_in = (uint32_t)pf_row < (uint32_t)rows;
-            float4* dst = my + (n_iss % JW_DEPTH) * 32 * V;
+            const uint32_t dst = my + (uint32_t)(n_iss % JW_DEPTH) * (32 * V * 16);
 #pragma unroll
             for (int v = 0; v < V; ++v) {
                 const bool in = row_in && (V > 1 ? ((pf_ok >> v) & 1u) != 0 : pf_ptr != nullptr);
-                cp_async_cg16(dst + v, in ? pf_ptr + 4 * v : p.a, in ? 16u : 0u);
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;"
+                             :: "r"(dst + 16 * v), "l"(in ? pf_ptr + 4 * v : p.a), "r"(in ? 16u : 0u) : "memory");
             }
             cp_async_commit();
             if (V > 1 ? pf_ok != 0 : pf_ptr != nullptr) pf_ptr += ld;
@@ -514,9 +517,11 @@ k_strip(const __grid_constant__ Sched s, const __grid_constant__ typename B::Par
             if (ahead >= JW_DEPTH - 2) asm volatile("cp.async.wait_group %0;" :: "n"(JW_DEPTH - 2) : "memory");
             else cp_async_wait_dyn(ahead);
             float4 x[V], o[V];
-            const float4* src = my + (n_use % JW_DEPTH) * 32 * V;
+            const uint32_t src = my + (uint32_t)(n_use % JW_DEPTH) * (32 * V * 16);
 #pragma unroll
-            for (int v = 0; v < V; ++v) x[v] = src[v];
+            for (int v = 0; v < V; ++v)
+                asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                             : "=f"(x[v].x), "=f"(x[v].y), "=f"(x[v].z), "=f"(x[v].w) : "r"(src + 16 * v) : "memory");
             ++n_use;
             if (n_iss - n_use < JW_DEPTH - 1) issue_one();
             body.template ingest<PH>(x, i, o, p);
