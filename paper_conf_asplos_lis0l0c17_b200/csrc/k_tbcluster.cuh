@@ -106,34 +106,20 @@ __device__ __forceinline__ uint32_t dsmem_addr(const void* p, uint32_t rank) {
     asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(out) : "r"(smem_u32(p)), "r"(rank));
     return out;
 }
-// Stage release to the producer of CTA `rank`, and the producer's wait.
-// Default: cluster-scope release / acquire (the PTX memory model's guarantee
-// for ordering this CTA's shared-memory reads before the peer's next async
-// write into them).  CC_TBC_CTA_SCOPE=1 (diagnostic build) uses the plain
-// forms CUTLASS's multicast pipelines use (mbarrier.arrive.shared::cluster,
-// default semantics) to measure what the cluster-scope fences cost.
-#ifndef CC_TBC_CTA_SCOPE
-#define CC_TBC_CTA_SCOPE 0
-#endif
+// Stage release to the producer of CTA `rank`, and the producer's wait:
+// cluster-scope release / acquire, the PTX memory model's guarantee for
+// ordering this CTA's shared-memory reads before the peer's next async write
+// into them.  (The plain CTA-scope forms were measured slower as well as
+// weaker, and are not built.)
 __device__ __forceinline__ void mbar_arrive_remote_release(uint64_t* bar, uint32_t rank) {
-    if constexpr (CC_TBC_CTA_SCOPE)
-        asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" :: "r"(dsmem_addr(bar, rank)) : "memory");
-    else
-        asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" :: "r"(dsmem_addr(bar, rank))
-                     : "memory");
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" :: "r"(dsmem_addr(bar, rank))
+                 : "memory");
 }
 __device__ __forceinline__ void mbar_arrive_release_cluster(uint64_t* bar) {
-    if constexpr (CC_TBC_CTA_SCOPE)
-        mbar_arrive(bar);
-    else
-        asm volatile("mbarrier.arrive.release.cluster.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
+    asm volatile("mbarrier.arrive.release.cluster.shared::cta.b64 _, [%0];" :: "r"(smem_u32(bar)) : "memory");
 }
 // wait with cluster-scope acquire: the remote releases above happen-before what follows
 __device__ __forceinline__ void mbar_wait_acquire_cluster(uint64_t* bar, uint32_t parity) {
-    if constexpr (CC_TBC_CTA_SCOPE) {
-        mbar_wait(bar, parity);
-        return;
-    }
     asm volatile(
         "{\n\t.reg .pred p;\n"
         "WAITC_%=:\n\t"
