@@ -271,13 +271,14 @@ typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t ite
  * position of a COL-ordered cluster) it carries them over instead of re-reading
  * and re-sweeping the 2K-row overlap.  The tail launch runs iters % K sweeps
  * on the same grid.  Backends: DEFAULT (one warp per logical CTA, hardware
- * order), AGENT, AGENT_IDENTITY (agents = worker warps, 24 (fuse <= 3), 20 (4) or 15
- * in one CTA per SM beside a scheduler warp that pops their logical CTAs; max_agents / active_agents
- * count workers per SM; batch > 0 = tiles per queue claim, 0 = chunked
- * claims: 3/4 of a queue in one contiguous chunk per agent, the rest tile by
- * tile), AGENT_STATIC (worker i runs cluster i: ceil(M / workers) CTAs).  No row
- * window (UNSUPPORTED); TBCLUSTER / REDIRECT UNSUPPORTED; fuse outside [0, 8]
- * INVALID_ARG. */
+ * order); AGENT and AGENT_IDENTITY (agents = worker warps: 24 (fuse <= 3),
+ * 20 (fuse 4) or 15 in one CTA per SM beside a scheduler warp that pops their
+ * logical CTAs; max_agents / active_agents count workers per SM; batch > 0 =
+ * tiles per queue claim, 0 = chunked claims: 3/4 of a queue in one contiguous
+ * chunk per agent, the rest tile by tile); AGENT_STATIC (worker i runs
+ * cluster i: ceil(M / workers) CTAs).  The L2 hint and staging options are
+ * ignored.  No row window (UNSUPPORTED); TBCLUSTER / REDIRECT UNSUPPORTED;
+ * fuse outside [0, 8] INVALID_ARG. */
 
 /* CC_K_JACOBI5_HALO -- S§8(f)4: one rank's slab of the slab-sharded Jacobi
  * (S§8(e), config 3) with the per-sweep halo exchange fused into the sweep
