@@ -37,7 +37,10 @@ namespace cc {
 constexpr int JW_ROWS = 64;     // output rows per logical CTA
 constexpr int JW_WARPS = 8;     // worker warps per CTA of the one-shot kernel
 constexpr int JW_DEPTH = 8;     // rows in flight per warp (cp.async ring)
-constexpr int JW_BATCH = 0;     // default claim size: 0 = guided (jw_next)
+constexpr int JW_BATCH = 0;     // default claim size: 0 = chunked claims (jw_claim)
+#ifndef JW_TAIL
+#define JW_TAIL 4               // chunked claims: the last 1/JW_TAIL of a queue goes tile by tile
+#endif
 enum : int { JW_DYNAMIC = 0, JW_STATIC = 1, JW_ONESHOT = 2 };
 
 __host__ __device__ constexpr int jw_halo_chunks(int K) { return K <= 4 ? 1 : 2; }
@@ -116,7 +119,7 @@ struct JwSched {
 __device__ __forceinline__ int32_t jw_agents(const Sched& s) {
     return s.mode == MODE_IDENTITY ? s.active_agents * s.g.M : s.active_agents;
 }
-__device__ __forceinline__ int32_t jw_split(int32_t n) { return n - n / 4; }
+__device__ __forceinline__ int32_t jw_split(int32_t n) { return n - n / JW_TAIL; }
 __device__ __forceinline__ int32_t* jw_chunk_ctr(const Sched& s, int32_t q) {
     return ws_chunk(s) + (s.mode == MODE_IDENTITY ? 0 : q);
 }
