@@ -296,7 +296,7 @@ class JacobiSlab:
         self.comm_stream = torch.cuda.Stream(device=dev) if xchg.world > 1 else None
         self.ev_b = [torch.cuda.Event() for _ in range(2)]
         self.ev_x = [torch.cuda.Event() for _ in range(2)]
-        self.graph = None
+        self.graph, self.gi = None, 0
         self.fused = halo == "fused" and xchg.world > 1
         self.peer = None
         if self.fused:
@@ -350,8 +350,12 @@ class JacobiSlab:
         buffers ping-pong within the step and the step starts from a (an even
         `iters` returns the result to a; odd steps alternate)."""
         if self.graph is not None:
-            self.graph.replay()
-            return self.graph_launches
+            g, n = self.graph[self.gi]
+            g.replay()
+            if len(self.graph) == 2:                   # odd launch count: the step ended in the other buffer
+                self.a, self.b = self.b, self.a
+                self.gi ^= 1
+            return n
         if (self.fuse > 1 or self.kname == "jacobi5_wave") and self.x.world == 1:
             nl = 0
             for it, k in self.calls():
@@ -381,21 +385,12 @@ class JacobiSlab:
 
     def calls(self):
         """(iters, fuse) per library call of an unsharded step: the iters // K
-        full launches, then the remainder -- as two launches when one would
-        leave the step with an odd launch count (a replayed graph must end in
-        the buffer it started from)."""
+        full launches, then one launch of the remaining iters % K sweeps."""
         K = max(1, self.fuse)
         full, r = divmod(self.iters, K)
         if self.kname == "jacobi5" and K > 1:       # CC_K_JACOBI5 runs the remainder one sweep per launch
             return [(self.iters, K)]
-        out = [(full * K, K)] if full else []
-        if r:
-            if (full + 1) % 2 and r >= 2:          # one more launch would make the count odd: two
-                h = r // 2
-                out += [(2 * h, h)] if r % 2 == 0 else [(h, h), (r - h, r - h)]
-            else:
-                out += [(r, r)]
-        return out
+        return ([(full * K, K)] if full else []) + ([(r, r)] if r else [])
 
     def launches_per_step(self) -> int:
         if self.kname == "jacobi5_wave" and self.x.world == 1:
@@ -408,21 +403,27 @@ class JacobiSlab:
 
     def capture(self, opts: dict) -> bool:
         """Capture one step (all `iters` sweeps, both streams) into a CUDA graph;
-        later steps replay it.  Plans and tensor maps are created by an eager
-        step first (no allocation is legal during capture).  Returns False when
-        the exchange cannot be captured."""
-        if not self.x.capturable or self.launches_per_step() % 2 or self.fused:
+        later steps replay it.  A step with an odd number of ping-pong launches
+        ends in the other buffer, so it is captured twice, once from each
+        buffer, and the replays alternate.  Plans and tensor maps are created
+        by an eager step first (no allocation is legal during capture).
+        Returns False when the exchange cannot be captured."""
+        if not self.x.capturable or self.fused:
             return False
+        self.graph = None
         self.step(opts)
         torch.cuda.synchronize()
-        g = torch.cuda.CUDAGraph()
+        graphs = []
         s = torch.cuda.Stream(device=self.dev)
         s.wait_stream(torch.cuda.current_stream())
-        with torch.cuda.stream(s):
-            with torch.cuda.graph(g, stream=s):
-                n = self.step(opts)
+        for _ in range(2 if self.launches_per_step() % 2 else 1):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.stream(s):
+                with torch.cuda.graph(g, stream=s):
+                    n = self.step(opts)            # records; the host-side buffer swap follows the recorded step
+            graphs.append((g, n))
         torch.cuda.current_stream().wait_stream(s)
-        self.graph, self.graph_launches = g, n
+        self.graph, self.gi = graphs, 0           # graphs[gi] starts from the current self.a
         return True
 
     def result(self):

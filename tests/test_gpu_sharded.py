@@ -103,21 +103,23 @@ def test_atax_family_driver_world1():
         assert rel(got.cpu().numpy(), ref) <= 1e-4
 
 
-@pytest.mark.parametrize("fuse,T", [(8, 100), (8, 13), (3, 7), (6, 20)])
+@pytest.mark.parametrize("fuse,T", [(8, 100), (8, 13), (3, 7), (6, 20), (8, 16)])
 def test_jacobi_wave_driver_world1_graph(fuse, T):
-    """The bench's config-3 driver with the wavefront kernel: the even launch
-    split (graph replay must end in the buffer it started from), captured and
-    replayed, bit-exact."""
+    """The bench's config-3 driver with the wavefront kernel, captured and
+    replayed (an odd launch count ends in the other buffer: two graphs, one
+    from each buffer, alternate), bit-exact over three consecutive steps."""
     rows, cols = 200, 300
     d = drivers.JacobiSlab(rows, cols, T, drivers.Exchange(), "cuda", fuse=fuse, kernel="wave")
     assert sum(it for it, _ in d.calls()) == T
     opts = dict(backend="agent", order="col")
-    if d.launches_per_step() % 2 == 0:
-        assert d.capture(opts)
+    assert d.capture(opts)
+    assert len(d.graph) == (2 if d.launches_per_step() % 2 else 1)
     d.reset()
-    d.step(opts)
-    torch.cuda.synchronize()
-    assert np.array_equal(d.result().cpu().numpy(), O.jacobi5_f32(synth.matrix(4, rows, cols), T))
+    u0 = synth.matrix(4, rows, cols)
+    for k in range(1, 4):
+        d.step(opts)
+        torch.cuda.synchronize()
+        assert np.array_equal(d.result().cpu().numpy(), O.jacobi5_f32(u0, k * T)), k
 
 
 def test_jacobi_driver_world1_graph():
