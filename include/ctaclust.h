@@ -422,7 +422,9 @@ cc_status cc_l1_reuse_probe(int32_t ctas, int32_t stagger_cycles, const float* i
 
 /* Logical grid a kernel needs for `args` (so the caller can build the plan). */
 cc_status cc_kernel_grid(int32_t kernel, const void* args, int32_t* gx, int32_t* gy);
-/* Occupancy limit (agents per SM) of `kernel`'s agent body on `device`. */
+/* Occupancy limit (agents per SM) of `kernel`'s agent body on `device`
+ * (CC_K_JACOBI5_WAVE: worker warps per SM at fuse = 4; 24 / 20 / 15 for
+ * fuse <= 3 / 4 / 5-8). */
 cc_status cc_max_agents(int32_t kernel, int32_t device, int32_t* max_agents);
 
 /* Run `kernel` over the plan's logical grid with the chosen backend, on
