@@ -45,7 +45,9 @@ def run(u0, ld, iters, fuse, **v):
 @pytest.mark.parametrize("v", WVARIANTS, ids=lambda v: "-".join(str(x) for x in v.values()))
 @pytest.mark.parametrize("rows,cols,ld,iters,fuse", [(100, 70, 72, 10, 4), (64, 64, 64, 1, 1), (129, 33, 36, 7, 3),
                                                      (5, 3, 4, 3, 2), (300, 250, 252, 9, 4), (261, 241, 244, 13, 8),
-                                                     (200, 121, 124, 11, 5), (1, 9, 12, 2, 2), (70, 1, 4, 5, 4)])
+                                                     (200, 121, 124, 11, 5), (1, 9, 12, 2, 2), (70, 1, 4, 5, 4),
+                                                     (3, 200, 200, 9, 8), (200, 3, 4, 17, 8), (2, 2, 4, 8, 8),
+                                                     (65, 113, 116, 16, 8), (64, 112, 112, 0, 8)])
 def test_wave_bit_exact(v, rows, cols, ld, iters, fuse):
     u0 = synth.matrix(4, rows, cols)
     got = run(u0, ld, iters, fuse, **v)
