@@ -26,6 +26,13 @@
 // with jacobi_core4's single-sweep expression (PolyBench order, R14) and the
 // boundary rows / columns are copied, so K fused sweeps are bit-identical to
 // K single sweeps.
+//
+// The runtime around the body is generic (k_strip<Body, KIND>): one-shot
+// warps in hardware order, or persistent workers -- one CTA per SM, its last
+// warp a scheduler that binds to the SM's cluster, claims chunks of the
+// cluster queue (then single tiles, then steals) and posts each worker's next
+// logical CTAs into a shared-memory mailbox, so the workers' row loop carries
+// no scheduler code next to the sweep registers.
 #pragma once
 #include <stdint.h>
 #include <type_traits>
