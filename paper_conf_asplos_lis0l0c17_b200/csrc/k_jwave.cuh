@@ -41,7 +41,10 @@
 
 namespace cc {
 
-constexpr int JW_ROWS = 64;     // output rows per logical CTA
+#ifndef JW_TILE_ROWS
+#define JW_TILE_ROWS 64
+#endif
+constexpr int JW_ROWS = JW_TILE_ROWS;     // output rows per logical CTA
 constexpr int JW_WARPS = 8;     // worker warps per CTA of the one-shot kernel
 constexpr int JW_DEPTH = 8;     // rows in flight per warp (cp.async ring)
 constexpr int JW_BATCH = 0;     // default claim size: 0 = chunked claims (jw_claim)
