@@ -77,6 +77,8 @@ def parse():
     ap.add_argument("--no-overlap", action="store_true", help="jacobi: exchange after the whole sweep")
     ap.add_argument("--fuse", type=int, default=0,
                     help="jacobi: sweeps per launch (0: 8 for the wave kernel, 3 for the tile-fused one)")
+    ap.add_argument("--tile-rows", type=int, default=0,
+                    help="jacobi wave: logical CTA height in rows (0 = 64; DESIGN §10.0)")
     ap.add_argument("--jkernel", choices=("wave", "tile"), default="wave",
                     help="jacobi: strip wavefronts carried across tiles (CC_K_JACOBI5_WAVE, R34) or tile-fused "
                          "sweeps (CC_K_JACOBI5, R32)")
@@ -351,7 +353,8 @@ def build_driver(a, X, dev):
         return drivers.AtaxFamily(sz["n"], X, dev)
     if a.config == "jacobi":
         return drivers.JacobiSlab(sz["side"], sz["side"], sz["iters"], X, dev, overlap=not a.no_overlap,
-                                  halo=a.halo, fuse=jacobi_fuse(a), kernel=getattr(a, "jkernel", "tile"))
+                                  halo=a.halo, fuse=jacobi_fuse(a), kernel=getattr(a, "jkernel", "tile"),
+                                  tile_rows=getattr(a, "tile_rows", 0))
     if a.config in ("conv3", "conv7"):
         return drivers.ConvSlab(sz["side"], sz["side"], sz["R"], X, dev)
     return drivers.SpmvBlock(sz["scale"], X, dev, hot=a.hot)
@@ -457,6 +460,13 @@ def main():
     else:
         ms_def, per_def, def_kind = ms_def_dir, per_def_dir, "direct-load"
     ms_id, _, _ = timed(identity_opts(head), cmp_steps)
+    ms_tall = None
+    if a.config == "jacobi" and getattr(D, "kname", "") == "jacobi5_wave" and world == 1:
+        # context, not a comparator: the same wavefront kernel in hardware order on
+        # 256-row logical CTAs (few restarts), the fastest Jacobi measured
+        t0_, D.trows = D.trows, 256
+        ms_tall, _, _ = timed(dict(dflt), cmp_steps)
+        D.trows = t0_
     ms_two_pass = None
     if a.config == "atax" and D.fused_atax:         # the same clustered step with the two-pass ATAX
         D.fused_atax = False
@@ -540,6 +550,7 @@ def main():
                 "ms_per_step_default_tma": round(ms_def_tma, 4),
                 "ms_per_step_default_direct": None if ms_def_dir is None else round(ms_def_dir, 4),
                 "ms_per_step_identity": round(ms_id, 4),
+                "ms_per_step_default_256row_tiles": None if ms_tall is None else round(ms_tall, 4),
                 "ms_per_step_two_pass_atax": None if ms_two_pass is None else round(ms_two_pass, 4),
                 "roofline": roof, "clocks": clk, "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": launches,
                 "home_fraction": home, "parity": parity,

@@ -257,16 +257,19 @@ typedef struct { float* a; float* b; int64_t ld; int32_t rows, cols; int32_t ite
                                     halo, the intermediate sweeps recomputed on chip), bit-identical to
                                     single sweeps; iters % fuse remaining sweeps run one per launch.
                                     Not with a row window (UNSUPPORTED). */
+                 int32_t tile_rows; /* CC_K_JACOBI5_WAVE only: logical CTA height in rows, 0 = 64; 8..1024
+                                    (INVALID_ARG otherwise).  Small tiles favour the carried COL clusters,
+                                    tall ones hardware order; ignored by CC_K_JACOBI5. */
                } cc_jacobi5_args;
 
 /* CC_K_JACOBI5_WAVE -- the same sweeps (CC_K_JACOBI5's arithmetic, bit-identical,
  * `iters` sweeps ping-ponging a -> b -> a, *result_is_b as there) run K = fuse
  * (1..8; 0 = 1) at a time by warp agents streaming column strips
  * (reading R34, §4.2 P:1793 / Listing 5).  Logical CTA
- * (bx, by) = output rows [64 by, 64 by + 64) x columns [WS bx, WS bx + WS),
- * WS = 120 for K <= 4 and 112 for K = 5..8; grid ceil(cols/WS) x ceil(rows/64).
- * One launch runs K sweeps: a warp ingests its tile's input rows from 64 by - K
- * to 64 by + 64 + K and keeps every intermediate sweep's last two rows in
+ * (bx, by) = output rows [T by, T by + T) x columns [WS bx, WS bx + WS),
+ * T = tile_rows (default 64), WS = 120 for K <= 4 and 112 for K = 5..8; grid
+ * ceil(cols/WS) x ceil(rows/T).  One launch runs K sweeps: a warp ingests its
+ * tile's input rows from T by - K to T by + T + K and keeps every intermediate sweep's last two rows in
  * registers; when its next logical CTA is the tile directly below (the next
  * position of a COL-ordered cluster) it carries them over instead of re-reading
  * and re-sweeping the 2K-row overlap.  The tail launch runs iters % K sweeps

@@ -373,7 +373,9 @@ extern "C" cc_status cc_kernel_grid(int32_t k, const void* a, int32_t* gx, int32
         auto* c = (const cc_jacobi5_args*)a;
         if (c->fuse < 0 || c->fuse > 8) return fail(CC_ERR_INVALID_ARG, "jacobi5_wave: fuse %d outside [0, 8]", c->fuse);
         const int K = c->fuse < 1 ? 1 : c->fuse;
-        *gx = cdiv(c->cols, jw_strip_cols(jw_halo_chunks(K))); *gy = cdiv(c->rows, JW_ROWS); return CC_OK;
+        const int T = c->tile_rows == 0 ? JW_ROWS : c->tile_rows;
+        if (T < 8 || T > 1024) return fail(CC_ERR_INVALID_ARG, "jacobi5_wave: tile_rows %d outside [8, 1024]", c->tile_rows);
+        *gx = cdiv(c->cols, jw_strip_cols(jw_halo_chunks(K))); *gy = cdiv(c->rows, T); return CC_OK;
     }
     case CC_K_CONV2D: { auto* c = (const cc_conv2d_args*)a; *gx = cdiv(c->cols, 32); *gy = cdiv(c->rows, 32); return CC_OK; }
     case CC_K_SPMV: case CC_K_SPMV_SHUB: {
@@ -1013,7 +1015,7 @@ extern "C" cc_status cc_launch(cc_plan p, int32_t k, const void* a, const cc_lau
         int launches_done = 0;
         for (int it = 0; it < x->iters && s == CC_OK;) {
             const int k = x->iters - it >= K ? K : x->iters - it;  // the tail runs fewer sweeps, same strips
-            const JWaveParams jp{src, dst, x->ld, x->rows, x->cols};
+            const JWaveParams jp{src, dst, x->ld, x->rows, x->cols, x->tile_rows == 0 ? JW_ROWS : x->tile_rows};
             s = hl == 1 ? jw_launch<1>(c, jp, k) : jw_launch<2>(c, jp, k);
             std::swap(src, dst);
             ++launches_done;

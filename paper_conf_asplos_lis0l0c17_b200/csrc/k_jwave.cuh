@@ -41,10 +41,7 @@
 
 namespace cc {
 
-#ifndef JW_TILE_ROWS
-#define JW_TILE_ROWS 64
-#endif
-constexpr int JW_ROWS = JW_TILE_ROWS;     // output rows per logical CTA
+constexpr int JW_ROWS = 64;     // default output rows per logical CTA (cc_jacobi5_args.tile_rows = 0)
 constexpr int JW_WARPS = 8;     // worker warps per CTA of the one-shot kernel
 constexpr int JW_DEPTH = 8;     // rows in flight per warp (cp.async ring)
 constexpr int JW_BATCH = 0;     // default claim size: 0 = chunked claims (jw_claim)
@@ -56,7 +53,7 @@ enum : int { JW_DYNAMIC = 0, JW_STATIC = 1, JW_ONESHOT = 2 };
 __host__ __device__ constexpr int jw_halo_chunks(int K) { return K <= 4 ? 1 : 2; }
 __host__ __device__ constexpr int jw_strip_cols(int hl) { return 128 - 8 * hl; }
 
-struct JWaveParams { const float* a; float* b; int64_t ld; int32_t rows, cols; };
+struct JWaveParams { const float* a; float* b; int64_t ld; int32_t rows, cols; int32_t trows; };
 
 // one vertical run of logical CTAs of strip bx: output rows [e0, e1), input
 // rows [e0 - K, e1 + K) streamed
@@ -418,8 +415,8 @@ k_strip(const __grid_constant__ Sched s, const __grid_constant__ typename B::Par
             if (bx < 0) return false;
         }
         r.bx = bx;
-        r.e0 = by * JW_ROWS;
-        r.e1 = r.e0 + JW_ROWS < rows ? r.e0 + JW_ROWS : rows;
+        r.e0 = by * p.trows;                                  // logical CTA height (parameter bank)
+        r.e1 = r.e0 + p.trows < rows ? r.e0 + p.trows : rows;
         return true;
     };
 

@@ -85,7 +85,7 @@ class MvtArgs(ctypes.Structure):
 
 class Jacobi5Args(ctypes.Structure):
     _fields_ = [("a", _vp), ("b", _vp), ("ld", _i64), ("rows", _i32), ("cols", _i32), ("iters", _i32),
-                ("result_is_b", _vp), ("row_lo", _i32), ("row_hi", _i32), ("fuse", _i32)]
+                ("result_is_b", _vp), ("row_lo", _i32), ("row_hi", _i32), ("fuse", _i32), ("tile_rows", _i32)]
 
 
 class Jacobi5HaloArgs(ctypes.Structure):
@@ -270,9 +270,11 @@ def mvt_args(A, y1, y2, x1, x2, m=None, n=None) -> MvtArgs:
     return MvtArgs(A.data_ptr(), _lda(A), m, n, y1.data_ptr(), y2.data_ptr(), x1.data_ptr(), x2.data_ptr())
 
 
-def jacobi5_args(a, b, iters, rows=None, cols=None, row_window=None, fuse=1) -> tuple[Jacobi5Args, ctypes.c_int32]:
+def jacobi5_args(a, b, iters, rows=None, cols=None, row_window=None, fuse=1,
+                 tile_rows=0) -> tuple[Jacobi5Args, ctypes.c_int32]:
     """`row_window` = (row_lo, row_hi): write only output rows [row_lo, row_hi).
-    `fuse`: sweeps per launch (1-4; 1-8 for jacobi5_wave)."""
+    `fuse`: sweeps per launch (1-4; 1-8 for jacobi5_wave); `tile_rows`:
+    jacobi5_wave's logical CTA height (0 = 64)."""
     flag = _i32(0)
     rows = a.shape[0] if rows is None else rows
     cols = a.shape[1] if cols is None else cols
@@ -280,7 +282,7 @@ def jacobi5_args(a, b, iters, rows=None, cols=None, row_window=None, fuse=1) -> 
     if _lda(b) != _lda(a):
         raise CtaclustError(-1, f"jacobi5: a and b share one leading dimension (got {_lda(a)} and {_lda(b)})")
     args = Jacobi5Args(a.data_ptr(), b.data_ptr(), _lda(a), rows, cols, iters, ctypes.addressof(flag), lo, hi,
-                       int(fuse))
+                       int(fuse), int(tile_rows))
     args._keep = flag            # result_is_b points into it: it must live as long as the struct
     return args, flag
 

@@ -270,11 +270,12 @@ class JacobiSlab:
     eagerly (a replayed graph would repeat the tags)."""
 
     def __init__(self, rows: int, cols: int, iters: int, xchg: Exchange, device, overlap: bool = True,
-                 halo: str = "exchange", fuse: int = 1, kernel: str = "tile"):
+                 halo: str = "exchange", fuse: int = 1, kernel: str = "tile", tile_rows: int = 0):
         self.rows, self.cols, self.iters, self.x = rows, cols, iters, xchg
         # kernel="wave": the K fused sweeps run as strip wavefronts
         # (CC_K_JACOBI5_WAVE, R34, K <= 8); "tile": tile-fused (CC_K_JACOBI5, K <= 4)
         self.kname = "jacobi5_wave" if kernel == "wave" and halo != "fused" else "jacobi5"
+        self.trows = tile_rows                                     # wave: logical CTA height (0 = 64)
         # K sweeps per launch (R32).  Sharded, the slab keeps K halo rows per
         # side and exchanges them once per K sweeps: a slab edge acts as a fixed
         # boundary inside the launch, so after K sweeps the error it causes has
@@ -359,7 +360,7 @@ class JacobiSlab:
         if (self.fuse > 1 or self.kname == "jacobi5_wave") and self.x.world == 1:
             nl = 0
             for it, k in self.calls():
-                args, flag = cc.jacobi5_args(self.a, self.b, it, fuse=k)
+                args, flag = cc.jacobi5_args(self.a, self.b, it, fuse=k, tile_rows=self.trows)
                 nl += _launch(self.kname, args, opts, stream)
                 if flag.value:
                     self.a, self.b = self.b, self.a
@@ -368,7 +369,7 @@ class JacobiSlab:
             nl, done = 0, 0
             while done < self.iters:
                 k = min(self.fuse, self.iters - done)
-                args, flag = cc.jacobi5_args(self.a, self.b, k, fuse=k if k > 1 else 1)
+                args, flag = cc.jacobi5_args(self.a, self.b, k, fuse=k if k > 1 else 1, tile_rows=self.trows)
                 nl += _launch(self.kname, args, opts, stream)
                 if flag.value:
                     self.a, self.b = self.b, self.a

@@ -140,12 +140,13 @@ def jacobi5(a, b, iters, backend="agent", order=None, tile=None, num_clusters=0,
     return b if flag.value else a
 
 
-def jacobi5_wave(a, b, iters, fuse=4, backend="agent", order=None, tile=None, num_clusters=0, stream=None, **kw):
+def jacobi5_wave(a, b, iters, fuse=4, backend="agent", order=None, tile=None, num_clusters=0, stream=None,
+                 tile_rows=0, **kw):
     """`iters` sweeps, `fuse` (1-8) per launch, by warp agents streaming column
     strips (CC_K_JACOBI5_WAVE, reading R34); COL clusters let an agent carry
     its sweep levels from one tile to the one below.  Bit-identical to
     jacobi5; returns the buffer holding the result."""
-    args, flag = cc.jacobi5_args(a, b, iters, fuse=fuse)
+    args, flag = cc.jacobi5_args(a, b, iters, fuse=fuse, tile_rows=tile_rows)
     _launch("jacobi5_wave", args, backend, order, tile, num_clusters, _dev(a), stream, **kw)
     return b if flag.value else a
 

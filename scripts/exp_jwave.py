@@ -64,6 +64,7 @@ def main():
                          ("agent-tile1x8-b8", dict(backend="agent", order="tile", tile=(1, 8), batch=8)),
                          ("identity", dict(backend="identity")),
                          ("default", dict(backend="default"))]:
+            kw = dict(kw, tile_rows=int(os.environ.get("JW_TROWS", "0")))
             timed(f"wave{f}-{name}", lambda kw=kw, f=f: ops.jacobi5_wave(a, b, T, fuse=f, **kw),
                   dict(base, warps_per_sm=wpsm))
     json.dump({"N": N, "sweeps": T, "rows": rows}, open(sys.argv[1], "w"), indent=1)

@@ -170,6 +170,10 @@ def test_kernel_grid():
     assert cc.kernel_grid("jacobi5_wave", J(None, None, 128, 65, 120, 1, None, 0, 0, 0)) == (1, 2)
     with pytest.raises(cc.CtaclustError):
         cc.kernel_grid("jacobi5_wave", J(None, None, 128, 64, 64, 1, None, 0, 0, 9))
+    assert cc.kernel_grid("jacobi5_wave", J(None, None, 16384, 16384, 16384, 100, None, 0, 0, 8, 256)) == (147, 64)
+    assert cc.kernel_grid("jacobi5_wave", J(None, None, 16384, 1000, 16384, 100, None, 0, 0, 8, 16)) == (147, 63)
+    with pytest.raises(cc.CtaclustError):
+        cc.kernel_grid("jacobi5_wave", J(None, None, 128, 64, 64, 1, None, 0, 0, 8, 4))
     a = cc.SpmvArgs(1 << 24, 1 << 24, 1 << 28)
     assert cc.kernel_grid("spmv", a) == (((1 << 24) + (1 << 28) + 4095) // 4096, 1)
     assert cc.kernel_grid("hist64", cc.Hist64Args(None, 1 << 30, None)) == (32768, 1)

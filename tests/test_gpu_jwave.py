@@ -65,6 +65,19 @@ def test_wave_every_fuse_multi_strip(fuse):
         assert np.array_equal(run(u0, 392, 2 * fuse + 1, fuse, **v), want), (fuse, v)
 
 
+@pytest.mark.parametrize("tile_rows", [8, 16, 100, 256])
+@pytest.mark.parametrize("v", [dict(backend="agent", order="col"), dict(backend="default"), dict(backend="identity"),
+                               dict(backend="static", order="col", num_clusters=11)],
+                         ids=lambda v: "-".join(str(x) for x in v.values()))
+def test_wave_tile_rows(v, tile_rows):
+    """cc_jacobi5_args.tile_rows: logical CTAs of any height, carried or restarted, bit-exact."""
+    u0 = synth.matrix(9, 333, 252)
+    a = torch.from_numpy(u0).cuda()
+    out = ops.jacobi5_wave(a, torch.zeros_like(a), 19, fuse=8, tile_rows=tile_rows, **v)
+    torch.cuda.synchronize()
+    assert np.array_equal(out.cpu().numpy(), O.jacobi5_f32(u0, 19)), (v, tile_rows)
+
+
 @pytest.mark.parametrize("v", [dict(backend="agent", order="col"), dict(backend="static", order="col"),
                                dict(backend="identity"), dict(backend="default")],
                          ids=lambda v: "-".join(str(x) for x in v.values()))
